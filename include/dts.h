@@ -1,0 +1,161 @@
+/*
+ * dts.h -- C ABI of libdts.so, a B200-native (sm_100a) distance threshold
+ * search over 4-D (t, x, y, z) trajectory line segments.
+ *
+ * Operation (Gowanlock & Casanova, §III "Problem statement"):
+ * given an entry database D of line segments, a query set Q of line segments
+ * and a distance d, return every triple (q, l, [t_start, t_end]) such that query
+ * segment q and entry segment l are within Euclidean distance d of each other
+ * in (x, y, z) during the closed time interval [t_start, t_end].  The index
+ * (temporal bins, §IV-B.1, and a flattened spatial grid, §IV-A.1)
+ * only prunes candidates; every result is decided by the refinement
+ * compare() of Alg. 1 l.14, whose reading is fixed in DESIGN.md
+ * §"Readings" (strict temporal overlap, closed distance inequality, linear
+ * interpolation along each segment, fp64 arithmetic).
+ *
+ * Conventions shared by every entry point:
+ *  - Segments are 64-byte records in the order of dts_segment below, stored
+ *    contiguously (array of structs, row i = segment id i).  The id reported
+ *    for a segment is its position in the array passed (reading c6).
+ *  - Results are sorted by (query_id, entry_id), contain no duplicates, and
+ *    are byte-identical across reruns and independent of dts_index_params
+ *    (reading c7).
+ *  - Functions returning dts_status never throw and never abort; on error
+ *    every output pointer is set to NULL / 0, nothing is leaked, and
+ *    dts_last_error() returns a message (thread-local, valid until the next
+ *    call on the same thread).
+ *  - "device" arguments are CUDA device pointers on the index's device;
+ *    "host" arguments are ordinary (pageable or pinned) host pointers.
+ *  - cuda_stream is a cudaStream_t (NULL = the legacy default stream).  All
+ *    entry points are synchronous with respect to the host on return.
+ */
+#ifndef DTS_H
+#define DTS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    DTS_OK = 0,
+    DTS_EINVAL = -1,      /* invalid argument or invalid segment data            */
+    DTS_ENOMEM = -2,      /* device or pinned host allocation failed             */
+    DTS_ECUDA = -3,       /* CUDA runtime error (message in dts_last_error)      */
+    DTS_ENOTSUP = -4,     /* no sm_100 device / unsupported configuration        */
+    DTS_EINTERNAL = -5    /* internal invariant violated (a bug)                 */
+} dts_status;
+
+/* One trajectory line segment: spatiotemporal start and end point. */
+typedef struct {
+    double t_start, x_start, y_start, z_start;
+    double t_end, x_end, y_end, z_end;
+} dts_segment;
+
+/* One result triple (q, l, [t_start, t_end]) of P:L32; 24 bytes.
+ * t_start <= t_end, both absolute times inside the two segments' common
+ * temporal extent.  A tangency at exactly d gives t_start == t_end. */
+typedef struct {
+    uint32_t query_id;    /* position in Q as passed, plus query_id_base */
+    uint32_t entry_id;    /* position in D as passed                     */
+    double t_start;
+    double t_end;
+} dts_result;
+
+/* Index construction parameters; zero means "choose automatically". */
+typedef struct {
+    int      device;            /* CUDA ordinal                                        */
+    uint32_t temporal_bins;     /* m of P:L76; 0 = bin width = max segment duration    */
+    uint32_t cells_per_dim;     /* grid resolution cap per axis; 0 = from extents     */
+    double   d_hint;            /* typical search distance, sizes grid cells; 0 = none */
+    uint64_t mem_budget_bytes;  /* reserved (0 = free HBM)                             */
+} dts_index_params;
+
+/* Per-search statistics (optional output of the *_ex entry points). */
+typedef struct {
+    uint64_t candidates;        /* candidate (query, entry) pairs refined per pass      */
+    uint64_t cell_lookups;      /* (bin, cell) probes issued per pass                   */
+    uint64_t results;           /* results returned                                     */
+    uint32_t max_results_per_query;
+    uint32_t time_kernels;      /* in: nonzero = record CUDA-event times below        */
+    float    ms_prep;           /* query keys + sort                                    */
+    float    ms_count;          /* pass 1 (fused candidate streaming + refine, count)   */
+    float    ms_scan;           /* exclusive scan of per-query counts                   */
+    float    ms_scatter;        /* pass 2 (fused streaming + refine, scatter)           */
+    float    ms_canon;          /* per-query sort by entry id                           */
+} dts_search_stats;
+
+typedef struct dts_index dts_index;   /* opaque; owns the device copy of D + index */
+
+/* Build the index over n host segments D (copied; caller keeps ownership).
+ * n == 0 builds an empty index.  Errors: DTS_EINVAL for NULL D with n > 0,
+ * n >= 2^32, non-finite coordinates or times, t_end < t_start, or a segment
+ * whose speed overflows fp64; DTS_ENOMEM; DTS_ECUDA; DTS_ENOTSUP. */
+dts_status dts_build_index(const dts_segment* D, size_t n,
+                           const dts_index_params* params,      /* NULL = defaults */
+                           dts_index** out_index);
+
+/* Same, from device memory: D_dev points to n dts_segment records in device
+ * memory of params->device, 16-byte aligned. Not retained after return. */
+dts_status dts_build_index_device(const dts_segment* D_dev, size_t n,
+                                  const dts_index_params* params,
+                                  void* cuda_stream, dts_index** out_index);
+
+/* Search nq host query segments Q (copied) at distance d >= 0 (finite).
+ * On success *out_results is library-allocated pinned host memory holding
+ * *out_count results (NULL / 0 when there are none); release it with
+ * dts_free_results.  query_id_base is added to every reported query id
+ * (callers that shard Q).  Errors: DTS_EINVAL (NULL with nq > 0, nq >= 2^32,
+ * bad d, invalid query segments, query_id_base + nq > 2^32), DTS_ENOMEM,
+ * DTS_ECUDA. */
+dts_status dts_search(const dts_index* index,
+                      const dts_segment* Q, size_t nq, double d,
+                      uint32_t query_id_base, void* cuda_stream,
+                      dts_result** out_results, size_t* out_count);
+
+dts_status dts_search_ex(const dts_index* index,
+                         const dts_segment* Q, size_t nq, double d,
+                         uint32_t query_id_base, void* cuda_stream,
+                         dts_result** out_results, size_t* out_count,
+                         dts_search_stats* stats);                /* may be NULL */
+
+/* Device-resident search: Q_dev holds nq segments in device memory
+ * (16-byte aligned); results are returned in library-owned device memory
+ * (*out_results_dev, NULL when empty), freed with dts_free_results_device. */
+dts_status dts_search_device(const dts_index* index,
+                             const dts_segment* Q_dev, size_t nq, double d,
+                             uint32_t query_id_base, void* cuda_stream,
+                             dts_result** out_results_dev, size_t* out_count,
+                             dts_search_stats* stats);            /* may be NULL */
+
+void dts_free_results(dts_result* results);          /* NULL is a no-op */
+void dts_free_results_device(dts_result* results);   /* NULL is a no-op */
+void dts_free_index(dts_index* index);               /* NULL is a no-op */
+
+/* Introspection of a built index (for tests and benchmarks). */
+typedef struct {
+    uint64_t n;                 /* entries                                   */
+    uint64_t cells;             /* non-empty (bin, cell) keys                */
+    uint32_t bins;              /* m                                         */
+    uint32_t grid[3];           /* cells per axis                            */
+    double   bin_width;         /* b of P:L76                                */
+    double   cell_width[3];
+    double   max_extent[3];     /* max |x_end - x_start| etc.        */
+    double   max_duration;
+    float    ms_build;          /* device time of the last build (CUDA events) */
+} dts_index_info;
+
+dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);
+
+/* Number of kernels this library has launched in the process so far. */
+uint64_t dts_kernel_launches(void);
+
+const char* dts_last_error(void);
+const char* dts_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* DTS_H */

@@ -1,0 +1,297 @@
+"""Thin Python binding of libdts.so (include/dts.h): argument marshalling only.
+
+Every step of the distance threshold search (§III) runs in the
+library's sm_100a kernels; this module converts numpy arrays / torch tensors
+to pointers and back.  There is no CPU fallback: if libdts.so is missing or
+the device is not an sm_100 part, the calls raise.
+
+Names follow the C ABI: build_index, build_index_device, search, search_ex,
+search_device, free_results (implicit, by garbage collection), index info.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+__all__ = ["RESULT_DTYPE", "IndexParams", "Index", "DeviceResults", "DTSError",
+           "build_index", "build_index_device", "search", "search_ex", "search_device",
+           "lib_path", "load", "EXPORTED_SYMBOLS"]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIB_PATH = os.path.join(_HERE, "libdts.so")
+
+RESULT_DTYPE = np.dtype([("query_id", "<u4"), ("entry_id", "<u4"),
+                         ("t_start", "<f8"), ("t_end", "<f8")], align=True)
+assert RESULT_DTYPE.itemsize == 24
+
+EXPORTED_SYMBOLS = (
+    "dts_build_index", "dts_build_index_device", "dts_search", "dts_search_ex",
+    "dts_search_device", "dts_free_results", "dts_free_results_device", "dts_free_index",
+    "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
+)
+
+_STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
+           -4: "DTS_ENOTSUP", -5: "DTS_EINTERNAL"}
+
+
+class DTSError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{_STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class IndexParams(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("temporal_bins", ctypes.c_uint32),
+                ("cells_per_dim", ctypes.c_uint32), ("d_hint", ctypes.c_double),
+                ("mem_budget_bytes", ctypes.c_uint64)]
+
+
+class SearchStats(ctypes.Structure):
+    _fields_ = [("candidates", ctypes.c_uint64), ("cell_lookups", ctypes.c_uint64),
+                ("results", ctypes.c_uint64), ("max_results_per_query", ctypes.c_uint32),
+                ("time_kernels", ctypes.c_uint32), ("ms_prep", ctypes.c_float),
+                ("ms_count", ctypes.c_float), ("ms_scan", ctypes.c_float),
+                ("ms_scatter", ctypes.c_float), ("ms_canon", ctypes.c_float)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+class IndexInfo(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_uint64), ("cells", ctypes.c_uint64), ("bins", ctypes.c_uint32),
+                ("grid", ctypes.c_uint32 * 3), ("bin_width", ctypes.c_double),
+                ("cell_width", ctypes.c_double * 3), ("max_extent", ctypes.c_double * 3),
+                ("max_duration", ctypes.c_double), ("ms_build", ctypes.c_float)]
+
+    def as_dict(self):
+        out = {}
+        for k, _ in self._fields_:
+            v = getattr(self, k)
+            out[k] = list(v) if isinstance(v, ctypes.Array) else v
+        return out
+
+
+_lib = None
+
+
+def lib_path() -> str:
+    return _LIB_PATH
+
+
+def load():
+    """Load libdts.so (raises if it has not been built)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"{_LIB_PATH} not built; run __graft_entry__.build() "
+                          "or python paper_conf_ipps_gowanlockc15_b200/build.py")
+    lib = ctypes.CDLL(_LIB_PATH)
+    P = ctypes.c_void_p
+    S = ctypes.c_size_t
+    pp = ctypes.POINTER(ctypes.c_void_p)
+    ps = ctypes.POINTER(ctypes.c_size_t)
+    lib.dts_build_index.argtypes = [P, S, ctypes.POINTER(IndexParams), pp]
+    lib.dts_build_index_device.argtypes = [P, S, ctypes.POINTER(IndexParams), P, pp]
+    lib.dts_search.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps]
+    lib.dts_search_ex.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
+                                  ctypes.POINTER(SearchStats)]
+    lib.dts_search_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
+                                      ctypes.POINTER(SearchStats)]
+    for f in ("dts_build_index", "dts_build_index_device", "dts_search", "dts_search_ex",
+              "dts_search_device", "dts_index_get_info"):
+        getattr(lib, f).restype = ctypes.c_int
+    lib.dts_index_get_info.argtypes = [P, ctypes.POINTER(IndexInfo)]
+    lib.dts_free_results.argtypes = [P]
+    lib.dts_free_results.restype = None
+    lib.dts_free_results_device.argtypes = [P]
+    lib.dts_free_results_device.restype = None
+    lib.dts_free_index.argtypes = [P]
+    lib.dts_free_index.restype = None
+    lib.dts_last_error.restype = ctypes.c_char_p
+    lib.dts_version.restype = ctypes.c_char_p
+    lib.dts_kernel_launches.restype = ctypes.c_uint64
+    lib.dts_kernel_launches.argtypes = []
+    _lib = lib
+    return lib
+
+
+def _check(rc: int):
+    if rc != 0:
+        raise DTSError(rc, _lib.dts_last_error().decode())
+
+
+def _segments(a) -> np.ndarray:
+    a = np.ascontiguousarray(np.asarray(a, dtype=np.float64))
+    if a.size == 0:
+        return a.reshape(0, 8)
+    if a.ndim != 2 or a.shape[1] != 8:
+        raise ValueError("segments must have shape (n, 8)")
+    return a
+
+
+def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0) -> IndexParams:
+    return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0)
+
+
+def _stream_ptr(stream) -> int:
+    if stream is None:
+        return 0
+    if hasattr(stream, "cuda_stream"):
+        return int(stream.cuda_stream)
+    return int(stream)
+
+
+class Index:
+    """Owns a dts_index*; freed with dts_free_index."""
+
+    def __init__(self, handle: int, device: int):
+        self._h = ctypes.c_void_p(handle)
+        self.device = device
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self) -> dict:
+        inf = IndexInfo()
+        _check(load().dts_index_get_info(self._h, ctypes.byref(inf)))
+        return inf.as_dict()
+
+    def free(self):
+        if self._h and self._h.value:
+            load().dts_free_index(self._h)
+            self._h = ctypes.c_void_p(0)
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+class DeviceResults:
+    """Results in library-owned device memory (dts_free_results_device on
+    release).  Exposes __cuda_array_interface__ as a flat uint8 buffer."""
+
+    def __init__(self, ptr: int, count: int, device: int):
+        self.ptr = ptr
+        self.count = count
+        self.device = device
+
+    @property
+    def __cuda_array_interface__(self):
+        return {"shape": (self.count * RESULT_DTYPE.itemsize,), "typestr": "|u1",
+                "data": (self.ptr or 0, False), "version": 3}
+
+    def tensor(self):
+        import torch
+        if self.count == 0:
+            return torch.empty(0, dtype=torch.uint8, device=f"cuda:{self.device}")
+        return torch.as_tensor(self, device=f"cuda:{self.device}")
+
+    def numpy(self) -> np.ndarray:
+        if self.count == 0:
+            return np.empty(0, dtype=RESULT_DTYPE)
+        return self.tensor().cpu().numpy().view(RESULT_DTYPE)
+
+    def free(self):
+        if self.ptr:
+            load().dts_free_results_device(ctypes.c_void_p(self.ptr))
+            self.ptr = 0
+            self.count = 0
+
+    def __del__(self):
+        try:
+            self.free()
+        except Exception:
+            pass
+
+
+def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int = 0,
+                d_hint: float = 0.0) -> Index:
+    """dts_build_index: D is host (n, 8) float64 (copied)."""
+    lib = load()
+    D = _segments(D)
+    p = _params(device, temporal_bins, cells_per_dim, d_hint)
+    h = ctypes.c_void_p()
+    _check(lib.dts_build_index(D.ctypes.data if D.size else None, D.shape[0], ctypes.byref(p),
+                               ctypes.byref(h)))
+    return Index(h.value, device)
+
+
+def build_index_device(D_dev, n: int = None, device: int = 0, temporal_bins: int = 0,
+                       cells_per_dim: int = 0, d_hint: float = 0.0, stream=None) -> Index:
+    """dts_build_index_device: D_dev is a CUDA tensor (n, 8) float64."""
+    lib = load()
+    ptr = D_dev.data_ptr() if hasattr(D_dev, "data_ptr") else int(D_dev)
+    if n is None:
+        n = D_dev.shape[0]
+    p = _params(device, temporal_bins, cells_per_dim, d_hint)
+    h = ctypes.c_void_p()
+    _check(lib.dts_build_index_device(ctypes.c_void_p(ptr), n, ctypes.byref(p),
+                                      ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(h)))
+    return Index(h.value, device)
+
+
+def _host_results(ptr, count) -> np.ndarray:
+    if count == 0:
+        return np.empty(0, dtype=RESULT_DTYPE)
+    out = np.empty(count, dtype=RESULT_DTYPE)
+    ctypes.memmove(out.ctypes.data, ptr, count * RESULT_DTYPE.itemsize)
+    load().dts_free_results(ctypes.c_void_p(ptr))
+    return out
+
+
+def search_ex(index: Index, Q, d: float, query_id_base: int = 0, stream=None,
+              time_kernels: bool = False):
+    """dts_search_ex: host Q -> (results structured array, stats dict)."""
+    lib = load()
+    Q = _segments(Q)
+    out = ctypes.c_void_p()
+    cnt = ctypes.c_size_t()
+    st = SearchStats()
+    st.time_kernels = 1 if time_kernels else 0
+    _check(lib.dts_search_ex(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
+                             float(d), int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
+                             ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
+    return _host_results(out.value, cnt.value), st.as_dict()
+
+
+def search(index: Index, Q, d: float, query_id_base: int = 0, stream=None) -> np.ndarray:
+    """dts_search: host Q -> results sorted by (query_id, entry_id)."""
+    lib = load()
+    Q = _segments(Q)
+    out = ctypes.c_void_p()
+    cnt = ctypes.c_size_t()
+    _check(lib.dts_search(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0], float(d),
+                          int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
+                          ctypes.byref(out), ctypes.byref(cnt)))
+    return _host_results(out.value, cnt.value)
+
+
+def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=None,
+                  n: int = None, time_kernels: bool = False):
+    """dts_search_device: Q_dev CUDA tensor (nq, 8) float64 -> (DeviceResults, stats)."""
+    lib = load()
+    ptr = Q_dev.data_ptr() if hasattr(Q_dev, "data_ptr") else int(Q_dev)
+    if n is None:
+        n = Q_dev.shape[0]
+    out = ctypes.c_void_p()
+    cnt = ctypes.c_size_t()
+    st = SearchStats()
+    st.time_kernels = 1 if time_kernels else 0
+    _check(lib.dts_search_device(index.handle, ctypes.c_void_p(ptr), n, float(d),
+                                 int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
+                                 ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
+    return DeviceResults(out.value or 0, cnt.value, index.device), st.as_dict()
+
+
+def kernel_launches() -> int:
+    return int(load().dts_kernel_launches())
+
+
+def version() -> str:
+    return load().dts_version().decode()

@@ -1,0 +1,306 @@
+// api.cu -- the C ABI of include/dts.h: argument validation, device checks,
+// host <-> device copies, ownership and error reporting.  Every step of the
+// search itself runs in the kernels of build.cu / search.cu / prims.cu.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdlib>
+#include <map>
+#include <mutex>
+#include <new>
+#include <string>
+
+#include "internal.cuh"
+
+namespace dts {
+
+std::atomic<unsigned long long> g_launches{0};
+static thread_local std::string g_err;
+void set_last_error(const std::string& msg) { g_err = msg; }
+
+namespace {
+
+std::mutex g_mu;
+bool g_pool_ready[64] = {false};
+
+// Verify the device is an sm_100 part (the cubins are sm_100a-only) and make
+// the stream-ordered pool keep its memory between calls.
+void prepare_device(int dev) {
+    int count = 0;
+    if (cudaGetDeviceCount(&count) != cudaSuccess || count == 0) {
+        cudaGetLastError();
+        throw Error(DTS_ENOTSUP, "no CUDA device available");
+    }
+    if (dev < 0 || dev >= count) throw Error(DTS_EINVAL, "device ordinal out of range");
+    DTS_CUDA(cudaSetDevice(dev));
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (dev < 64 && !g_pool_ready[dev]) {
+        cudaDeviceProp prop;
+        DTS_CUDA(cudaGetDeviceProperties(&prop, dev));
+        if (prop.major != 10 || prop.minor != 0)
+            throw Error(DTS_ENOTSUP, std::string("libdts is built for sm_100a; device is ") +
+                                         prop.name + " sm_" + std::to_string(prop.major) +
+                                         std::to_string(prop.minor));
+        cudaMemPool_t pool;
+        DTS_CUDA(cudaDeviceGetDefaultMemPool(&pool, dev));
+        unsigned long long thr = ~0ull;
+        DTS_CUDA(cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr));
+        g_pool_ready[dev] = true;
+    }
+}
+
+// Pinned host result blocks, recycled (the result D2H is part of the
+// search response time; cudaMallocHost per call would dominate it).
+constexpr size_t HDR = 64;
+std::multimap<size_t, void*> g_pinned_free;
+size_t g_pinned_cached = 0;
+
+void* pinned_alloc(size_t bytes) {
+    {
+        std::lock_guard<std::mutex> lk(g_mu);
+        auto it = g_pinned_free.lower_bound(bytes);
+        if (it != g_pinned_free.end() && it->first <= 2 * bytes + (1u << 20)) {
+            void* b = it->second;
+            g_pinned_cached -= it->first;
+            g_pinned_free.erase(it);
+            return static_cast<char*>(b) + HDR;
+        }
+    }
+    void* b = nullptr;
+    cudaError_t e = cudaMallocHost(&b, bytes + HDR);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        throw Error(DTS_ENOMEM, "cudaMallocHost failed for the result buffer");
+    }
+    *static_cast<size_t*>(b) = bytes;
+    return static_cast<char*>(b) + HDR;
+}
+
+void pinned_free(void* p) {
+    if (!p) return;
+    void* b = static_cast<char*>(p) - HDR;
+    size_t bytes = *static_cast<size_t*>(b);
+    std::lock_guard<std::mutex> lk(g_mu);
+    if (g_pinned_cached + bytes <= (size_t(4) << 30)) {
+        g_pinned_free.emplace(bytes, b);
+        g_pinned_cached += bytes;
+    } else {
+        cudaFreeHost(b);
+    }
+}
+
+void free_index_memory(dts_index* idx) {
+    if (!idx) return;
+    cudaSetDevice(idx->device);
+    cudaDeviceSynchronize();
+    if (idx->block) cudaFree(idx->block);
+    if (idx->ht.slots) cudaFree(idx->ht.slots);
+    idx->block = nullptr;
+    idx->ht.slots = nullptr;
+}
+
+dts_index_params defaults() {
+    dts_index_params p{};
+    return p;
+}
+
+void check_params(const dts_index_params& p) {
+    if (!(p.d_hint >= 0.0) || !std::isfinite(p.d_hint))
+        throw Error(DTS_EINVAL, "d_hint must be finite and >= 0");
+}
+
+void check_aligned(const void* p, const char* what) {
+    if (reinterpret_cast<uintptr_t>(p) & 15u)
+        throw Error(DTS_EINVAL, std::string(what) + " must be 16-byte aligned");
+}
+
+template <typename F>
+dts_status guarded(F&& f) {
+    try {
+        g_err.clear();
+        f();
+        return DTS_OK;
+    } catch (const Error& e) {
+        g_err = e.what();
+        return e.status;
+    } catch (const std::bad_alloc&) {
+        g_err = "host allocation failed";
+        return DTS_ENOMEM;
+    } catch (const std::exception& e) {
+        g_err = e.what();
+        return DTS_EINTERNAL;
+    } catch (...) {
+        g_err = "unknown internal error";
+        return DTS_EINTERNAL;
+    }
+}
+
+dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* params,
+                        bool host, cudaStream_t s, dts_index** out_index) {
+    if (out_index) *out_index = nullptr;
+    dts_index* idx = nullptr;
+    dts_status st = guarded([&] {
+        if (!out_index) throw Error(DTS_EINVAL, "out_index is NULL");
+        if (n > 0 && !D) throw Error(DTS_EINVAL, "D is NULL with n > 0");
+        if (n >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "n must be < 2^32");
+        dts_index_params p = params ? *params : defaults();
+        check_params(p);
+        prepare_device(p.device);
+        idx = new dts_index();
+        idx->device = p.device;
+        if (n == 0) return;
+        if (host) {
+            DevBuf<dts_segment> dD(n, s);
+            DTS_CUDA(cudaMemcpyAsync(dD.p, D, n * sizeof(dts_segment), cudaMemcpyHostToDevice, s));
+            build_index_device(idx, dD.p, n, p, s);
+        } else {
+            check_aligned(D, "D_dev");
+            build_index_device(idx, D, n, p, s);
+        }
+        DTS_CUDA(cudaStreamSynchronize(s));
+    });
+    if (st != DTS_OK) {
+        if (idx) {
+            free_index_memory(idx);
+            delete idx;
+        }
+        return st;
+    }
+    *out_index = idx;
+    return DTS_OK;
+}
+
+dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                         uint32_t qid_base, cudaStream_t s, bool host, dts_result** out_results,
+                         size_t* out_count, dts_search_stats* stats) {
+    if (out_results) *out_results = nullptr;
+    if (out_count) *out_count = 0;
+    dts_result* ret = nullptr;
+    size_t cnt = 0;
+    dts_status st = guarded([&] {
+        if (!index) throw Error(DTS_EINVAL, "index is NULL");
+        if (!out_results || !out_count) throw Error(DTS_EINVAL, "output pointer is NULL");
+        if (nq > 0 && !Q) throw Error(DTS_EINVAL, "Q is NULL with nq > 0");
+        if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
+        if ((uint64_t)qid_base + nq > (uint64_t(1) << 32))
+            throw Error(DTS_EINVAL, "query_id_base + nq exceeds 2^32");
+        if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
+        prepare_device(index->device);
+        SearchOut so;
+        if (host) {
+            DevBuf<dts_segment> dQ(nq, s);
+            if (nq)
+                DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment),
+                                         cudaMemcpyHostToDevice, s));
+            search_device(index, dQ.p, nq, d, qid_base, s, &so, stats);
+            if (so.count) {
+                dts_result* h = nullptr;
+                try {
+                    h = static_cast<dts_result*>(pinned_alloc(so.count * sizeof(dts_result)));
+                    DTS_CUDA(cudaMemcpyAsync(h, so.results, so.count * sizeof(dts_result),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                } catch (...) {
+                    pinned_free(h);
+                    cudaFreeAsync(so.results, s);
+                    throw;
+                }
+                cudaFreeAsync(so.results, s);
+                ret = h;
+                cnt = so.count;
+            }
+            DTS_CUDA(cudaStreamSynchronize(s));
+        } else {
+            check_aligned(Q, "Q_dev");
+            search_device(index, Q, nq, d, qid_base, s, &so, stats);
+            ret = so.results;
+            cnt = so.count;
+        }
+    });
+    if (st == DTS_OK) {
+        *out_results = ret;
+        *out_count = cnt;
+    }
+    return st;
+}
+
+}  // namespace
+}  // namespace dts
+
+using namespace dts;
+
+extern "C" {
+
+dts_status dts_build_index(const dts_segment* D, size_t n, const dts_index_params* params,
+                           dts_index** out_index) {
+    return build_common(D, n, params, true, cudaStreamPerThread, out_index);
+}
+
+dts_status dts_build_index_device(const dts_segment* D_dev, size_t n,
+                                  const dts_index_params* params, void* cuda_stream,
+                                  dts_index** out_index) {
+    return build_common(D_dev, n, params, false, static_cast<cudaStream_t>(cuda_stream),
+                        out_index);
+}
+
+dts_status dts_search(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                      uint32_t query_id_base, void* cuda_stream, dts_result** out_results,
+                      size_t* out_count) {
+    return search_common(index, Q, nq, d, query_id_base, static_cast<cudaStream_t>(cuda_stream),
+                         true, out_results, out_count, nullptr);
+}
+
+dts_status dts_search_ex(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                         uint32_t query_id_base, void* cuda_stream, dts_result** out_results,
+                         size_t* out_count, dts_search_stats* stats) {
+    return search_common(index, Q, nq, d, query_id_base, static_cast<cudaStream_t>(cuda_stream),
+                         true, out_results, out_count, stats);
+}
+
+dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                             double d, uint32_t query_id_base, void* cuda_stream,
+                             dts_result** out_results_dev, size_t* out_count,
+                             dts_search_stats* stats) {
+    return search_common(index, Q_dev, nq, d, query_id_base,
+                         static_cast<cudaStream_t>(cuda_stream), false, out_results_dev,
+                         out_count, stats);
+}
+
+void dts_free_results(dts_result* results) { pinned_free(results); }
+
+void dts_free_results_device(dts_result* results) {
+    if (results) cudaFree(results);
+}
+
+void dts_free_index(dts_index* index) {
+    if (!index) return;
+    free_index_memory(index);
+    delete index;
+}
+
+dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
+    return guarded([&] {
+        if (!idx || !info) throw Error(DTS_EINVAL, "NULL argument");
+        dts_index_info r{};
+        r.n = idx->n;
+        r.cells = idx->n_cells;
+        r.bins = (uint32_t)idx->gp.m;
+        for (int a = 0; a < 3; ++a) {
+            r.grid[a] = (uint32_t)idx->gp.nc[a];
+            r.cell_width[a] = idx->gp.w[a];
+            r.max_extent[a] = idx->max_ext[a];
+        }
+        r.bin_width = idx->gp.b;
+        r.max_duration = idx->gp.maxdur;
+        r.ms_build = idx->ms_build;
+        *info = r;
+    });
+}
+
+const char* dts_last_error(void) { return g_err.c_str(); }
+
+const char* dts_version(void) { return "dts 0.1 (sm_100a)"; }
+
+uint64_t dts_kernel_launches(void) { return g_launches.load(); }
+
+}  // extern "C"

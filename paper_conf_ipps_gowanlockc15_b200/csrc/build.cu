@@ -1,0 +1,372 @@
+// build.cu -- GPU index builder.
+//
+// The paper builds its indexes on the host (P:L76 temporal bins over D sorted
+// by t_start; P:L44 flatly structured grid of non-empty cells G with a lookup
+// array A; P:L86-P:L87 spatial subbins sized by the max per-dimension extent).
+// Here the index is built on the device and each entry is stored once:
+//
+//   1. k_bounds       fp64 min/max reduction: t_min, t_max, spatial
+//                     bounds and max per-axis extent (P:L86-P:L87), max
+//                     duration; validation of every segment.
+//   2. host           bin width b, cell widths w_a >= extent_a + d_hint.
+//   3. k_keys         key = (bin of t_start, cell of the MBB midpoint), row-major
+//                     (bin, z, y, x) so that x-adjacent cells are adjacent runs.
+//   4. radix sort     stable (key, id): within a cell entries stay in id order.
+//   5. k_gather       sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz)
+//                     + per-bin [min t_start, max t_end] extents (B_start/B_end
+//                     of P:L76) with warp-aggregated atomics.
+//   6. k_count_cells / k_insert / k_ends
+//                     non-empty cells -> open-addressing hash table
+//                     key -> [start, end) (the role of G and A of P:L44, with no
+//                     duplicated ids since every entry is in exactly one cell).
+#include <algorithm>
+#include <cmath>
+
+#include "internal.cuh"
+
+namespace dts {
+namespace {
+
+struct Bounds {
+    double tmin, tmax;
+    double lo[3], hi[3];
+    double ext[3];
+    double maxdur;
+    double absmax;
+    int bad;
+};
+
+constexpr int BT = 256;
+
+__device__ __forceinline__ void bounds_init(Bounds& b) {
+    b.tmin = INFINITY; b.tmax = -INFINITY;
+    for (int a = 0; a < 3; ++a) { b.lo[a] = INFINITY; b.hi[a] = -INFINITY; b.ext[a] = 0.0; }
+    b.maxdur = 0.0; b.absmax = 0.0; b.bad = 0;
+}
+
+__device__ __forceinline__ void bounds_merge(Bounds& b, const Bounds& o) {
+    b.tmin = fmin(b.tmin, o.tmin); b.tmax = fmax(b.tmax, o.tmax);
+    for (int a = 0; a < 3; ++a) {
+        b.lo[a] = fmin(b.lo[a], o.lo[a]); b.hi[a] = fmax(b.hi[a], o.hi[a]);
+        b.ext[a] = fmax(b.ext[a], o.ext[a]);
+    }
+    b.maxdur = fmax(b.maxdur, o.maxdur); b.absmax = fmax(b.absmax, o.absmax);
+    b.bad |= o.bad;
+}
+
+__device__ __forceinline__ void bounds_shfl(Bounds& b, int off) {
+    Bounds o;
+    o.tmin = __shfl_xor_sync(0xffffffffu, b.tmin, off);
+    o.tmax = __shfl_xor_sync(0xffffffffu, b.tmax, off);
+    for (int a = 0; a < 3; ++a) {
+        o.lo[a] = __shfl_xor_sync(0xffffffffu, b.lo[a], off);
+        o.hi[a] = __shfl_xor_sync(0xffffffffu, b.hi[a], off);
+        o.ext[a] = __shfl_xor_sync(0xffffffffu, b.ext[a], off);
+    }
+    o.maxdur = __shfl_xor_sync(0xffffffffu, b.maxdur, off);
+    o.absmax = __shfl_xor_sync(0xffffffffu, b.absmax, off);
+    o.bad = __shfl_xor_sync(0xffffffffu, b.bad, off);
+    bounds_merge(b, o);
+}
+
+__device__ void block_reduce_write(Bounds& b, Bounds* out) {
+    __shared__ Bounds sm[BT / 32];
+    for (int off = 16; off; off >>= 1) bounds_shfl(b, off);
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (lane == 0) sm[warp] = b;
+    __syncthreads();
+    if (warp == 0) {
+        Bounds c;
+        if (lane < BT / 32) c = sm[lane]; else bounds_init(c);
+        for (int off = 16; off; off >>= 1) bounds_shfl(c, off);
+        if (lane == 0) *out = c;
+    }
+}
+
+// Segment validity (readings c4, c8): finite coordinates and times,
+// t_end >= t_start, finite velocity.
+__global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, size_t n,
+                                              Bounds* __restrict__ partial) {
+    Bounds b;
+    bounds_init(b);
+    for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT) {
+        double4 s0 = D[2 * i], s1 = D[2 * i + 1];   // (t0,x0,y0,z0), (t1,x1,y1,z1)
+        double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
+        bool fin = isfinite(s0.x) && isfinite(s1.x);
+        for (int a = 0; a < 3; ++a) fin = fin && isfinite(p0[a]) && isfinite(p1[a]);
+        if (!fin) { b.bad |= 1; continue; }
+        if (s1.x < s0.x) { b.bad |= 2; continue; }
+        double dur = s1.x - s0.x;
+        b.tmin = fmin(b.tmin, s0.x);
+        b.tmax = fmax(b.tmax, s1.x);
+        b.maxdur = fmax(b.maxdur, dur);
+        b.absmax = fmax(b.absmax, fmax(fabs(s0.x), fabs(s1.x)));
+        for (int a = 0; a < 3; ++a) {
+            double lo = fmin(p0[a], p1[a]), hi = fmax(p0[a], p1[a]);
+            b.lo[a] = fmin(b.lo[a], lo);
+            b.hi[a] = fmax(b.hi[a], hi);
+            double e = hi - lo;
+            b.ext[a] = fmax(b.ext[a], e);
+            b.absmax = fmax(b.absmax, fmax(fabs(lo), fabs(hi)));
+            if (dur > 0.0 && !isfinite(e / dur)) b.bad |= 4;
+            if (!isfinite(e)) b.bad |= 4;
+        }
+    }
+    block_reduce_write(b, &partial[blockIdx.x]);
+}
+
+__global__ void __launch_bounds__(BT) k_bounds_final(const Bounds* __restrict__ partial, int np,
+                                                    Bounds* __restrict__ out) {
+    Bounds b;
+    bounds_init(b);
+    for (int i = threadIdx.x; i < np; i += BT) bounds_merge(b, partial[i]);
+    block_reduce_write(b, out);
+}
+
+__global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size_t n, GridParams g,
+                                            unsigned long long* __restrict__ keys,
+                                            uint32_t* __restrict__ ids) {
+    size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (i >= n) return;
+    double4 s0 = D[2 * i], s1 = D[2 * i + 1];
+    int32_t bin = bin_of(g, s0.x);
+    int32_t cx = cell_of(g, 0, 0.5 * (s0.y + s1.y));
+    int32_t cy = cell_of(g, 1, 0.5 * (s0.z + s1.z));
+    int32_t cz = cell_of(g, 2, 0.5 * (s0.w + s1.w));
+    keys[i] = make_key(g, bin, cx, cy, cz);
+    ids[i] = (uint32_t)i;
+}
+
+__device__ __forceinline__ double velocity(double p0, double p1, double dur) {
+    return dur > 0.0 ? (p1 - p0) / dur : 0.0;
+}
+
+__global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
+                                              const uint32_t* __restrict__ ids, GridParams g,
+                                              SegSoA soa,
+                                              unsigned long long* __restrict__ bin_t0min,
+                                              unsigned long long* __restrict__ bin_t1max) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    bool ok = p < n;
+    int32_t bin = -1;
+    unsigned long long o0 = ~0ull, o1 = 0ull;
+    if (ok) {
+        uint32_t i = ids[p];
+        double4 s0 = D[2 * (size_t)i], s1 = D[2 * (size_t)i + 1];
+        double dur = s1.x - s0.x;
+        soa.st[p] = make_double2(s0.x, s1.x);
+        soa.sx[p] = make_double2(s0.y, velocity(s0.y, s1.y, dur));
+        soa.sy[p] = make_double2(s0.z, velocity(s0.z, s1.z, dur));
+        soa.sz[p] = make_double2(s0.w, velocity(s0.w, s1.w, dur));
+        soa.eid[p] = i;
+        bin = bin_of(g, s0.x);
+        o0 = ordered_bits(s0.x);
+        o1 = ordered_bits(s1.x);
+    }
+    // per-bin extents, warp-aggregated when the warp is inside one bin
+    const int lane = threadIdx.x & 31;
+    int32_t b0 = __shfl_sync(0xffffffffu, bin, 0);
+    if (__all_sync(0xffffffffu, bin == b0 || bin < 0)) {
+        for (int off = 16; off; off >>= 1) {
+            unsigned long long a = __shfl_xor_sync(0xffffffffu, o0, off);
+            unsigned long long c = __shfl_xor_sync(0xffffffffu, o1, off);
+            o0 = a < o0 ? a : o0;
+            o1 = c > o1 ? c : o1;
+        }
+        if (lane == 0 && b0 >= 0) {
+            atomicMin(&bin_t0min[b0], o0);
+            atomicMax(&bin_t1max[b0], o1);
+        }
+    } else if (ok) {
+        atomicMin(&bin_t0min[bin], o0);
+        atomicMax(&bin_t1max[bin], o1);
+    }
+}
+
+__global__ void k_fill_u64(unsigned long long* __restrict__ a, size_t n, unsigned long long v) {
+    size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (i < n) a[i] = v;
+}
+
+__global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n) {
+    size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (i < n) {
+        double v = from_ordered_bits(a[i]);
+        a[i] = (unsigned long long)__double_as_longlong(v);
+    }
+}
+
+__global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __restrict__ keys,
+                                                   size_t n,
+                                                   unsigned long long* __restrict__ count) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    int f = (p < n) && (p == 0 || keys[p] != keys[p - 1]);
+    int c = __syncthreads_count(f);
+    if (threadIdx.x == 0 && c) atomicAdd(count, (unsigned long long)c);
+}
+
+__global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restrict__ keys,
+                                              size_t n, HashTable ht) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p >= n) return;
+    unsigned long long k = keys[p];
+    if (p != 0 && keys[p - 1] == k) return;
+    unsigned long long h = hash_key(k, ht.log2cap);
+    while (true) {
+        unsigned long long prev = atomicCAS(&ht.slots[h].key, EMPTY_KEY, k);
+        if (prev == EMPTY_KEY || prev == k) {
+            ht.slots[h].start = (uint32_t)p;
+            return;
+        }
+        h = (h + 1) & ht.mask;
+    }
+}
+
+__global__ void __launch_bounds__(BT) k_ends(const unsigned long long* __restrict__ keys, size_t n,
+                                            HashTable ht) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p >= n) return;
+    unsigned long long k = keys[p];
+    if (p + 1 != n && keys[p + 1] == k) return;
+    unsigned long long h = hash_key(k, ht.log2cap);
+    while (ht.slots[h].key != k) h = (h + 1) & ht.mask;
+    ht.slots[h].end = (uint32_t)(p + 1);
+}
+
+inline unsigned grid_for(size_t n) { return (unsigned)((n + BT - 1) / BT); }
+
+}  // namespace
+
+// Host-side choice of the temporal bins and spatial cells.
+static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g) {
+    const double span_t = b.tmax - b.tmin;
+    g.tmin = b.tmin;
+    g.maxdur = b.maxdur;
+    const uint64_t MAXBINS = 1u << 22;
+    double bw;
+    if (p.temporal_bins > 0 && span_t > 0.0) bw = span_t / (double)p.temporal_bins;
+    else bw = b.maxdur;                               // one bin per max duration
+    if (!(bw > 0.0) || !std::isfinite(bw)) bw = span_t > 0.0 ? span_t : 1.0;
+    double mb = std::floor(span_t / bw) + 1.0;
+    if (mb > (double)MAXBINS) { bw = span_t / (double)(MAXBINS - 1); mb = (double)MAXBINS; }
+    g.b = bw;
+    g.inv_b = 1.0 / bw;
+    g.m = (int32_t)mb;
+
+    const double MAXC = (double)(1u << 20);
+    for (int a = 0; a < 3; ++a) {
+        const double span = b.hi[a] - b.lo[a];
+        double w = b.ext[a] + (p.d_hint > 0.0 ? p.d_hint : 0.0);
+        if (p.cells_per_dim > 0) w = std::max(w, span / (double)p.cells_per_dim);
+        w = std::max(w, span / (MAXC - 1.0));
+        w = std::max(w, 1e-12 * b.absmax);
+        if (!(w > 0.0) || !std::isfinite(w)) w = 1.0;
+        g.o[a] = b.lo[a];
+        g.w[a] = w;
+        g.half_ext[a] = 0.5 * b.ext[a];
+        g.nc[a] = (int32_t)std::min(std::floor(span / w) + 1.0, MAXC);
+    }
+    // keep the key space below 2^62: coarsen the finest axis until it fits
+    while ((double)g.m * g.nc[0] * g.nc[1] * g.nc[2] >= 4.6e18) {
+        int a = 0;
+        for (int j = 1; j < 3; ++j) if (g.nc[j] > g.nc[a]) a = j;
+        g.w[a] *= 2.0;
+        g.nc[a] = (int32_t)std::floor((b.hi[a] - b.lo[a]) / g.w[a]) + 1;
+    }
+    for (int a = 0; a < 3; ++a) g.inv_w[a] = 1.0 / g.w[a];
+    g.cells_per_bin = (unsigned long long)g.nc[0] * g.nc[1] * g.nc[2];
+}
+
+void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
+                        const dts_index_params& p, cudaStream_t s) {
+    idx->n = n;
+    if (n == 0) return;
+    const double4* D = reinterpret_cast<const double4*>(D_dev);
+    cudaEvent_t e0, e1;
+    DTS_CUDA(cudaEventCreate(&e0));
+    DTS_CUDA(cudaEventCreate(&e1));
+    DTS_CUDA(cudaEventRecord(e0, s));
+
+    // 1. bounds + validation
+    const int np = (int)std::min<size_t>(grid_for(n), 148 * 8);
+    DevBuf<Bounds> partial(np, s), total(1, s);
+    k_bounds<<<np, BT, 0, s>>>(D, n, partial.p);
+    DTS_LAUNCH_CHECK();
+    k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
+    DTS_LAUNCH_CHECK();
+    Bounds hb;
+    DTS_CUDA(cudaMemcpyAsync(&hb, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
+    DTS_CUDA(cudaStreamSynchronize(s));
+    if (hb.bad & 1) throw Error(DTS_EINVAL, "entry segment with a non-finite coordinate or time");
+    if (hb.bad & 2) throw Error(DTS_EINVAL, "entry segment with t_end < t_start");
+    if (hb.bad & 4) throw Error(DTS_EINVAL, "entry segment whose speed overflows fp64");
+
+    // 2. grid
+    GridParams g{};
+    choose_grid(hb, p, g);
+    idx->gp = g;
+    for (int a = 0; a < 3; ++a) idx->max_ext[a] = hb.ext[a];
+
+    // 3-4. keys + sort
+    DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
+    DevBuf<uint32_t> ids(n, s), ids_tmp(n, s);
+    k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p);
+    DTS_LAUNCH_CHECK();
+    const unsigned long long max_key = (unsigned long long)g.m * g.cells_per_bin - 1ull;
+    idx->key_bits = bits_for(max_key);
+    radix_sort_pairs(keys.p, ids.p, keys_tmp.p, ids_tmp.p, n, idx->key_bits, s);
+    keys_tmp.release();
+    ids_tmp.release();
+
+    // 5. gather into the SoA layout + bin extents
+    const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
+    const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double);
+    char* blk = nullptr;
+    DTS_CUDA(cudaMallocAsync((void**)&blk, bytes_soa + bytes_bins + 256, s));
+    idx->block = blk;
+    idx->soa.st = reinterpret_cast<double2*>(blk);
+    idx->soa.sx = idx->soa.st + n;
+    idx->soa.sy = idx->soa.sx + n;
+    idx->soa.sz = idx->soa.sy + n;
+    idx->bin_t0min = reinterpret_cast<double*>(idx->soa.sz + n);
+    idx->bin_t1max = idx->bin_t0min + g.m;
+    idx->soa.eid = reinterpret_cast<uint32_t*>(idx->bin_t1max + g.m);
+    unsigned long long* b0 = reinterpret_cast<unsigned long long*>(idx->bin_t0min);
+    unsigned long long* b1 = reinterpret_cast<unsigned long long*>(idx->bin_t1max);
+    k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b0, g.m, ~0ull);
+    DTS_LAUNCH_CHECK();
+    k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
+    DTS_LAUNCH_CHECK();
+    k_gather<<<grid_for(n), BT, 0, s>>>(D, n, ids.p, g, idx->soa, b0, b1);
+    DTS_LAUNCH_CHECK();
+    k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
+    DTS_LAUNCH_CHECK();
+
+    // 6. non-empty cells -> hash table
+    DevBuf<unsigned long long> ncell(1, s);
+    DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
+    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, ncell.p);
+    DTS_LAUNCH_CHECK();
+    unsigned long long hc = 0;
+    DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
+    DTS_CUDA(cudaStreamSynchronize(s));
+    idx->n_cells = hc;
+    int log2cap = 6;
+    while ((1ull << log2cap) < 2 * hc) ++log2cap;
+    idx->ht.log2cap = log2cap;
+    idx->ht.mask = (1ull << log2cap) - 1;
+    DTS_CUDA(cudaMallocAsync((void**)&idx->ht.slots, sizeof(CellSlot) << log2cap, s));
+    DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
+    k_insert<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
+    DTS_LAUNCH_CHECK();
+    k_ends<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
+    DTS_LAUNCH_CHECK();
+
+    DTS_CUDA(cudaEventRecord(e1, s));
+    DTS_CUDA(cudaEventSynchronize(e1));
+    DTS_CUDA(cudaEventElapsedTime(&idx->ms_build, e0, e1));
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+}
+
+}  // namespace dts

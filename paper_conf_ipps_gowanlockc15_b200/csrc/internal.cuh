@@ -1,0 +1,201 @@
+// internal.cuh -- shared internals of libdts (CUDA side only; never included
+// by the oracle).  Layouts, grid parameters, error plumbing and the device
+// helpers used by both the index builder and the search kernels.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <atomic>
+#include <cstring>
+#include <stdexcept>
+#include <string>
+
+#include "../../include/dts.h"
+
+namespace dts {
+
+// ---------------------------------------------------------------- errors
+struct Error : std::runtime_error {
+    dts_status status;
+    Error(dts_status s, const std::string& m) : std::runtime_error(m), status(s) {}
+};
+
+void set_last_error(const std::string& msg);
+
+#define DTS_CUDA(call)                                                              \
+    do {                                                                            \
+        cudaError_t _e = (call);                                                    \
+        if (_e != cudaSuccess) {                                                    \
+            if (_e == cudaErrorMemoryAllocation)                                    \
+                throw ::dts::Error(DTS_ENOMEM, std::string(#call) + ": " +          \
+                                   cudaGetErrorString(_e));                         \
+            throw ::dts::Error(DTS_ECUDA, std::string(#call) + ": " +               \
+                               cudaGetErrorString(_e));                             \
+        }                                                                           \
+    } while (0)
+
+// Every kernel launch is followed by DTS_LAUNCH_CHECK(), which also counts it
+// (dts_kernel_launches(), used by the benchmark's gpu_launches claim).
+extern std::atomic<unsigned long long> g_launches;
+#define DTS_LAUNCH_CHECK()                                                          \
+    do {                                                                            \
+        ::dts::g_launches.fetch_add(1, std::memory_order_relaxed);                  \
+        DTS_CUDA(cudaGetLastError());                                               \
+    } while (0)
+
+// Stream-ordered device buffer (pool allocator; freed on scope exit).
+template <typename T>
+struct DevBuf {
+    T* p = nullptr;
+    size_t n = 0;
+    cudaStream_t s = nullptr;
+    DevBuf() = default;
+    DevBuf(size_t count, cudaStream_t st) { alloc(count, st); }
+    void alloc(size_t count, cudaStream_t st) {
+        release();
+        s = st;
+        n = count;
+        if (count) DTS_CUDA(cudaMallocAsync((void**)&p, count * sizeof(T), st));
+    }
+    void release() {
+        if (p) cudaFreeAsync(p, s);
+        p = nullptr;
+        n = 0;
+    }
+    T* detach() { T* r = p; p = nullptr; n = 0; return r; }
+    ~DevBuf() { release(); }
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+};
+
+// ---------------------------------------------------------------- layout
+// Entry segments in the index live in key order as four 16-byte streams
+// (SoA, one 128-bit load each):
+//   st = (t_start, t_end)   sx = (x_start, vx)   sy = (y_start, vy)   sz = (z_start, vz)
+// with v = (end - start) / (t_end - t_start) precomputed at build (0 for a
+// zero-duration segment, which can never overlap strictly in time).  The
+// position at time t is start + (t - t_start) * v.
+struct SegSoA {
+    double2* st;
+    double2* sx;
+    double2* sy;
+    double2* sz;
+    uint32_t* eid;   // caller's entry id of each sorted position
+};
+
+// Hash slot of one non-empty (bin, cell) key: entries [start, end) of the
+// sorted arrays.  16 bytes, one 128-bit load.
+struct __align__(16) CellSlot {
+    unsigned long long key;
+    uint32_t start;
+    uint32_t end;
+};
+static constexpr unsigned long long EMPTY_KEY = ~0ull;
+
+// Grid parameters (passed by value to kernels).
+struct GridParams {
+    double tmin;        // temporal origin  (t_min of P:L76)
+    double inv_b;       // 1 / bin width
+    double b;           // bin width        (b of P:L76)
+    double maxdur;      // max(t_end - t_start) over D
+    double o[3];        // spatial origin (per-axis min over D)
+    double w[3];        // cell width per axis
+    double inv_w[3];
+    double half_ext[3]; // half of the max per-axis extent
+    int32_t m;          // bins
+    int32_t nc[3];      // cells per axis
+    unsigned long long cells_per_bin;  // nc0*nc1*nc2
+};
+
+struct HashTable {
+    CellSlot* slots;
+    unsigned long long mask;   // capacity - 1 (power of two)
+    int log2cap;
+};
+
+// ---------------------------------------------------------------- device helpers
+__device__ __forceinline__ unsigned long long hash_key(unsigned long long k, int log2cap) {
+    return (k * 0x9E3779B97F4A7C15ull) >> (64 - log2cap);
+}
+
+__device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {
+    double f = floor((t - g.tmin) * g.inv_b);
+    if (!(f > 0.0)) return 0;                       // also maps NaN to 0
+    if (f >= (double)(g.m - 1)) return g.m - 1;
+    return (int32_t)f;
+}
+
+__device__ __forceinline__ int32_t cell_of(const GridParams& g, int a, double v) {
+    double f = floor((v - g.o[a]) * g.inv_w[a]);
+    if (!(f > 0.0)) return 0;
+    if (f >= (double)(g.nc[a] - 1)) return g.nc[a] - 1;
+    return (int32_t)f;
+}
+
+__device__ __forceinline__ unsigned long long make_key(const GridParams& g, int32_t bin,
+                                                       int32_t cx, int32_t cy, int32_t cz) {
+    return (unsigned long long)bin * g.cells_per_bin +
+           ((unsigned long long)cz * (unsigned long long)g.nc[1] + (unsigned long long)cy) *
+               (unsigned long long)g.nc[0] +
+           (unsigned long long)cx;
+}
+
+// Monotone map of doubles to unsigned 64-bit integers (for atomic min/max).
+__device__ __forceinline__ unsigned long long ordered_bits(double x) {
+    unsigned long long u = (unsigned long long)__double_as_longlong(x);
+    return (u & 0x8000000000000000ull) ? ~u : (u | 0x8000000000000000ull);
+}
+__host__ __device__ inline double from_ordered_bits(unsigned long long u) {
+    unsigned long long v = (u & 0x8000000000000000ull) ? (u & ~0x8000000000000000ull) : ~u;
+#ifdef __CUDA_ARCH__
+    return __longlong_as_double((long long)v);
+#else
+    double d;
+    memcpy(&d, &v, 8);
+    return d;
+#endif
+}
+
+// ---------------------------------------------------------------- primitives (prims.cu)
+// Exclusive scan of n values; out has n + 1 entries, out[n] = total.
+void scan_exclusive_u32_to_u32(const uint32_t* in, uint32_t* out, size_t n, cudaStream_t s);
+void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size_t n,
+                               cudaStream_t s);
+
+// Stable LSD radix sort of (key, value) pairs on key bits [0, nbits).
+// Sorts in place from the caller's view: on return keys/vals hold the result.
+// keys_tmp / vals_tmp are caller-provided scratch of n entries each.
+void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
+                      uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s);
+
+int bits_for(unsigned long long max_value);
+
+}  // namespace dts
+
+// The opaque index (definition shared by build.cu, search.cu and api.cu).
+struct dts_index {
+    int device = 0;
+    uint64_t n = 0;
+    dts::GridParams gp{};
+    dts::SegSoA soa{};
+    dts::HashTable ht{};
+    unsigned long long n_cells = 0;
+    double* bin_t0min = nullptr;   // per bin: min t_start (bin extent)
+    double* bin_t1max = nullptr;   // per bin: max t_end   (B_end of P:L76)
+    void* block = nullptr;         // single device allocation backing the arrays above
+    double max_ext[3] = {0, 0, 0};
+    float ms_build = 0.f;
+    int key_bits = 0;
+};
+
+namespace dts {
+void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
+                        const dts_index_params& p, cudaStream_t s);
+struct SearchOut {
+    dts_result* results = nullptr;   // device, cudaMalloc'd (caller owns)
+    size_t count = 0;
+};
+void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
+                   uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats);
+}  // namespace dts

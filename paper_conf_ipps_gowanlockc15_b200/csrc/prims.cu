@@ -1,0 +1,243 @@
+// prims.cu -- device-wide primitives written for this library: exclusive
+// scan (reduce / scan-of-partials / downsweep) and a stable LSD radix sort of
+// (u64 key, u32 value) pairs with warp-level match-based ranking.
+//
+// These implement the "radix sort and prefix scan" of the index builder
+// (BASELINE.json north_star) and the exclusive scan of
+// per-query result counts of the two-pass compaction (§8(a6)).
+#include "internal.cuh"
+
+namespace dts {
+
+int bits_for(unsigned long long v) {
+    int b = 0;
+    while (v) { ++b; v >>= 1; }
+    return b;
+}
+
+// ============================================================== scan
+namespace {
+constexpr int SCAN_THREADS = 256;
+constexpr int SCAN_ITEMS = 4;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;   // 1024
+
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_scan(T v) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T u = __shfl_up_sync(0xffffffffu, v, o);
+        if (lane >= o) v += u;
+    }
+    return v;
+}
+
+// Block-wide exclusive scan of one value per thread; returns the exclusive
+// prefix and writes the block total to *total.
+template <typename T>
+__device__ __forceinline__ T block_exclusive_scan(T v, T* total) {
+    __shared__ T warp_sums[SCAN_THREADS / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    T inc = warp_inclusive_scan(v);
+    if (lane == 31) warp_sums[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+        T s = (lane < SCAN_THREADS / 32) ? warp_sums[lane] : T(0);
+        s = warp_inclusive_scan(s);
+        if (lane < SCAN_THREADS / 32) warp_sums[lane] = s;
+    }
+    __syncthreads();
+    T warp_prefix = warp ? warp_sums[warp - 1] : T(0);
+    *total = warp_sums[SCAN_THREADS / 32 - 1];
+    __syncthreads();
+    return warp_prefix + inc - v;
+}
+
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_reduce(const Tin* __restrict__ in, size_t n,
+                                                              Tout* __restrict__ sums) {
+    size_t base = (size_t)blockIdx.x * SCAN_TILE;
+    Tout s = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_ITEMS; ++i) {
+        size_t idx = base + (size_t)i * SCAN_THREADS + threadIdx.x;
+        if (idx < n) s += (Tout)in[idx];
+    }
+    Tout total;
+    block_exclusive_scan<Tout>(s, &total);
+    if (threadIdx.x == 0) sums[blockIdx.x] = total;
+}
+
+// Downsweep: out[i] = prefix(block) + exclusive scan inside the block.
+// prefix == nullptr means a single-block scan; then out[n] = total.
+template <typename Tin, typename Tout>
+__global__ void __launch_bounds__(SCAN_THREADS) k_scan_down(const Tin* __restrict__ in, size_t n,
+                                                            const Tout* __restrict__ prefix,
+                                                            Tout* __restrict__ out) {
+    size_t base = (size_t)blockIdx.x * SCAN_TILE + (size_t)threadIdx.x * SCAN_ITEMS;
+    Tout v[SCAN_ITEMS];
+    Tout s = 0;
+#pragma unroll
+    for (int i = 0; i < SCAN_ITEMS; ++i) {
+        size_t idx = base + i;
+        v[i] = idx < n ? (Tout)in[idx] : Tout(0);
+        s += v[i];
+    }
+    Tout total;
+    Tout run = block_exclusive_scan<Tout>(s, &total);
+    Tout bp = prefix ? prefix[blockIdx.x] : Tout(0);
+    run += bp;
+#pragma unroll
+    for (int i = 0; i < SCAN_ITEMS; ++i) {
+        size_t idx = base + i;
+        if (idx < n) out[idx] = run;
+        run += v[i];
+    }
+    if (prefix == nullptr && threadIdx.x == 0) out[n] = total;
+    if (prefix != nullptr && blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+        out[n] = prefix[gridDim.x];
+}
+
+template <typename Tin, typename Tout>
+void scan_exclusive(const Tin* in, Tout* out, size_t n, cudaStream_t s) {
+    if (n <= (size_t)SCAN_TILE) {
+        k_scan_down<Tin, Tout><<<1, SCAN_THREADS, 0, s>>>(in, n, nullptr, out);
+        DTS_LAUNCH_CHECK();
+        return;
+    }
+    size_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;
+    DevBuf<Tout> sums(nb, s), pre(nb + 1, s);
+    k_scan_reduce<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, sums.p);
+    DTS_LAUNCH_CHECK();
+    scan_exclusive<Tout, Tout>(sums.p, pre.p, nb, s);
+    k_scan_down<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, pre.p, out);
+    DTS_LAUNCH_CHECK();
+}
+}  // namespace
+
+void scan_exclusive_u32_to_u32(const uint32_t* in, uint32_t* out, size_t n, cudaStream_t s) {
+    scan_exclusive<uint32_t, uint32_t>(in, out, n, s);
+}
+void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size_t n,
+                               cudaStream_t s) {
+    scan_exclusive<uint32_t, unsigned long long>(in, out, n, s);
+}
+
+// ============================================================== radix sort
+namespace {
+constexpr int RS_THREADS = 256;
+constexpr int RS_WARPS = RS_THREADS / 32;
+constexpr int RS_ITEMS = 8;                       // per thread
+constexpr int RS_TILE = RS_THREADS * RS_ITEMS;    // 2048 keys per CTA
+constexpr int RS_RADIX = 256;                     // 8-bit digits
+
+// Per-tile digit histogram; counts laid out digit-major so that one
+// exclusive scan yields every (digit, tile) output offset.
+__global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const unsigned long long* __restrict__ keys,
+                                                        size_t n, int shift,
+                                                        uint32_t* __restrict__ counts,
+                                                        uint32_t ntiles) {
+    __shared__ uint32_t h[RS_RADIX];
+    h[threadIdx.x] = 0;
+    __syncthreads();
+    size_t base = (size_t)blockIdx.x * RS_TILE;
+#pragma unroll
+    for (int i = 0; i < RS_ITEMS; ++i) {
+        size_t idx = base + (size_t)i * RS_THREADS + threadIdx.x;
+        if (idx < n) atomicAdd(&h[(uint32_t)(keys[idx] >> shift) & (RS_RADIX - 1)], 1u);
+    }
+    __syncthreads();
+    counts[(size_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+}
+
+// Stable scatter.  Warp w of a tile owns the contiguous chunk
+// [tile + w*256, tile + (w+1)*256); within a warp items are visited in
+// (item, lane) order = input order, ranked with __match_any_sync, and
+// warp-private digit counters; a cross-warp prefix per digit then orders the
+// chunks.  Output position = offset(digit, tile) + warp prefix + rank.
+__global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
+    const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
+    int shift, const uint32_t* __restrict__ offsets, uint32_t ntiles,
+    unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
+    __shared__ uint32_t wcnt[RS_WARPS][RS_RADIX + 1];
+    __shared__ uint32_t tile_base[RS_RADIX];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int j = lane; j < RS_RADIX + 1; j += 32) wcnt[warp][j] = 0;
+    tile_base[threadIdx.x] = offsets[(size_t)threadIdx.x * ntiles + blockIdx.x];
+    __syncwarp();
+
+    const size_t wbase = (size_t)blockIdx.x * RS_TILE + (size_t)warp * (32 * RS_ITEMS);
+    unsigned long long k[RS_ITEMS];
+    uint32_t v[RS_ITEMS], dig[RS_ITEMS], rank[RS_ITEMS];
+#pragma unroll
+    for (int i = 0; i < RS_ITEMS; ++i) {
+        size_t idx = wbase + (size_t)i * 32 + lane;
+        bool ok = idx < n;
+        k[i] = ok ? keys[idx] : 0ull;
+        v[i] = ok ? vals[idx] : 0u;
+        dig[i] = ok ? ((uint32_t)(k[i] >> shift) & (RS_RADIX - 1)) : (uint32_t)RS_RADIX;
+    }
+    const uint32_t lt_mask = (1u << lane) - 1u;
+#pragma unroll
+    for (int i = 0; i < RS_ITEMS; ++i) {
+        uint32_t peers = __match_any_sync(0xffffffffu, dig[i]);
+        int leader = __ffs(peers) - 1;
+        uint32_t old = 0;
+        if (lane == leader) {
+            old = wcnt[warp][dig[i]];
+            wcnt[warp][dig[i]] = old + __popc(peers);
+        }
+        old = __shfl_sync(0xffffffffu, old, leader);
+        rank[i] = old + __popc(peers & lt_mask);
+        __syncwarp();
+    }
+    __syncthreads();
+    {
+        const int dgt = threadIdx.x;   // RS_THREADS == RS_RADIX
+        uint32_t run = 0;
+#pragma unroll
+        for (int w = 0; w < RS_WARPS; ++w) {
+            uint32_t c = wcnt[w][dgt];
+            wcnt[w][dgt] = run;
+            run += c;
+        }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int i = 0; i < RS_ITEMS; ++i) {
+        if (dig[i] < (uint32_t)RS_RADIX) {
+            uint32_t dst = tile_base[dig[i]] + wcnt[warp][dig[i]] + rank[i];
+            keys_out[dst] = k[i];
+            vals_out[dst] = v[i];
+        }
+    }
+}
+static_assert(RS_THREADS == RS_RADIX, "one thread per digit in the cross-warp prefix");
+}  // namespace
+
+void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
+                      uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
+    if (n <= 1 || nbits <= 0) return;
+    const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
+    const size_t ncount = (size_t)RS_RADIX * ntiles;
+    DevBuf<uint32_t> counts(ncount, s), offs(ncount + 1, s);
+    unsigned long long *kin = keys, *kout = keys_tmp;
+    uint32_t *vin = vals, *vout = vals_tmp;
+    int passes = 0;
+    for (int shift = 0; shift < nbits; shift += 8, ++passes) {
+        k_rs_hist<<<ntiles, RS_THREADS, 0, s>>>(kin, n, shift, counts.p, ntiles);
+        DTS_LAUNCH_CHECK();
+        scan_exclusive_u32_to_u32(counts.p, offs.p, ncount, s);
+        k_rs_scatter<<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs.p, ntiles, kout, vout);
+        DTS_LAUNCH_CHECK();
+        unsigned long long* tk = kin; kin = kout; kout = tk;
+        uint32_t* tv = vin; vin = vout; vout = tv;
+    }
+    if (passes & 1) {
+        DTS_CUDA(cudaMemcpyAsync(keys, kin, n * sizeof(unsigned long long),
+                                 cudaMemcpyDeviceToDevice, s));
+        DTS_CUDA(cudaMemcpyAsync(vals, vin, n * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+    }
+}
+
+}  // namespace dts

@@ -1,0 +1,218 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle on the
+same seeded inputs.  Rule: tests/parity.py (pair set outside the 1e-9*d tie
+band identical, endpoints within 1e-9 normalised time, canonical order)."""
+import os
+
+import numpy as np
+import pytest
+
+import synth
+import dts_parity as parity
+
+pytestmark = pytest.mark.gpu
+
+THREADS = max(1, min(32, os.cpu_count() or 1))
+
+
+@pytest.fixture(scope="module")
+def dts():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_gowanlockc15_b200 as m
+    m.load()
+    return m
+
+
+def run_and_compare(dts, oracle_mod, D, Q, d, **params):
+    idx = dts.build_index(D, **params)
+    got = dts.search(idx, Q, d)
+    ora = oracle_mod.search(D, Q, d, threads=THREADS)
+    info = parity.compare(got, ora, D, Q, d, oracle_mod)
+    idx.free()
+    return got, info
+
+
+# ------------------------------------------------------------------ C0
+@pytest.mark.parametrize("d", [0.0, 0.01, 0.05, 0.2])
+def test_c0_exhaustive(dts, oracle_mod, d):
+    c = synth.make_config("C0")
+    got, info = run_and_compare(dts, oracle_mod, c.D, c.Q, d)
+    if d >= 0.05:
+        assert info["common"] > 0
+
+
+def test_c0_headline_has_hits_and_crossings(dts, oracle_mod):
+    c = synth.make_config("C0")
+    got, info = run_and_compare(dts, oracle_mod, c.D, c.Q, c.d)
+    assert info["common"] >= 20
+
+
+# ------------------------------------------------ random / adversarial sets
+def test_random_adversarial_sets(dts, oracle_mod):
+    total = 0
+    for seed in range(300):
+        D, Q = synth.adversarial(1000 + seed, 50, 50)
+        d = [0.0, 0.03, 0.1, 0.3][seed % 4]
+        _, info = run_and_compare(dts, oracle_mod, D, Q, d)
+        total += info["common"]
+    assert total > 1000
+
+
+def test_paper_example_on_gpu(dts):
+    import json
+    ex = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "paper_example.json")))
+    idx = dts.build_index(np.array(ex["D"]))
+    got = dts.search(idx, np.array(ex["Q"]), ex["d"])
+    assert got.shape[0] == 2
+    for r, e in zip(got, ex["expected"]):
+        assert (int(r["query_id"]), int(r["entry_id"])) == tuple(e[:2])
+        assert abs(r["t_start"] - e[2]) < 1e-12 and abs(r["t_end"] - e[3]) < 1e-12
+
+
+def test_golden_pairs_on_gpu(dts):
+    import json
+    spec = json.load(open(os.path.join(os.path.dirname(__file__), "golden", "pairs.json")))
+    for p in spec["pairs"]:
+        idx = dts.build_index(np.array([p["l"]]))
+        got = dts.search(idx, np.array([p["q"]]), p["d"])
+        if p["expected"] is None:
+            assert got.shape[0] == 0, p["id"]
+        elif not p["tie_band"]:
+            assert got.shape[0] == 1, p["id"]
+            assert abs(got[0]["t_start"] - p["expected"][0]) < 1e-12, p["id"]
+            assert abs(got[0]["t_end"] - p["expected"][1]) < 1e-12, p["id"]
+
+
+# ------------------------------------------------ index invariance, determinism
+def test_index_parameter_invariance_and_determinism(dts, oracle_mod):
+    c = synth.make_config("C2", scale=0.02)
+    d = 0.5
+    ref = None
+    for params in ({}, {"temporal_bins": 7}, {"temporal_bins": 5000}, {"cells_per_dim": 3},
+                   {"d_hint": 2.0}, {"d_hint": 0.01, "temporal_bins": 1}):
+        idx = dts.build_index(c.D, **params)
+        for _ in range(2):
+            got = dts.search(idx, c.Q, d)
+            if ref is None:
+                ref = got
+                parity.compare(got, oracle_mod.search(c.D, c.Q, d, threads=THREADS), c.D, c.Q, d,
+                               oracle_mod)
+            assert got.tobytes() == ref.tobytes(), params
+        idx.free()
+
+
+def test_device_api_matches_host_api(dts):
+    import torch
+    c = synth.make_config("C0")
+    idx_h = dts.build_index(c.D)
+    host = dts.search(idx_h, c.Q, c.d, query_id_base=7)
+    Dd = torch.from_numpy(c.D).cuda()
+    Qd = torch.from_numpy(c.Q).cuda()
+    idx_d = dts.build_index_device(Dd)
+    res, stats = dts.search_device(idx_d, Qd, c.d, query_id_base=7, time_kernels=True)
+    dev = res.numpy()
+    assert dev.tobytes() == host.tobytes()
+    assert stats["results"] == host.shape[0]
+    assert stats["candidates"] >= host.shape[0]
+    assert np.all(host["query_id"] >= 7)
+
+
+# ------------------------------------------------ configs at reduced / full size
+@pytest.mark.parametrize("name,scale,dlist", [
+    ("C1", 1.0, (0.001, 0.005, 0.02)),
+    ("C2", 0.05, (0.03, 0.09, 0.5, 2.0)),
+    ("C3", 0.05, (1.0, 5.0, 20.0, 50.0)),
+])
+def test_configs_sampled(dts, oracle_mod, name, scale, dlist):
+    c = synth.make_config(name, scale=scale)
+    idx = dts.build_index(c.D)
+    g = synth.rng(99)
+    qs = np.sort(g.choice(c.Q.shape[0], size=min(96, c.Q.shape[0]), replace=False))
+    for d in dlist:
+        got = dts.search(idx, c.Q, d)
+        ora = oracle_mod.search_queries(c.D, c.Q, qs, d, threads=THREADS)
+        parity.compare(parity.restrict(got, qs), ora, c.D, c.Q, d, oracle_mod)
+    idx.free()
+
+
+def test_c2_small_exhaustive_large_d(dts, oracle_mod):
+    """Many candidates per query, > 32 stencil cells (chunked lookups) and
+    > 32 results per query (CTA sort path)."""
+    c = synth.make_config("C2", scale=0.004)
+    for d in (2.0, 8.0):
+        got, info = run_and_compare(dts, oracle_mod, c.D, c.Q, d)
+        assert info["common"] > 0
+
+
+def test_c4_full_size_sampled(dts, oracle_mod):
+    """BASELINE.json configs[4] at full size, in the bench's launch
+    configuration (device-resident build + search): sampled queries against
+    the oracle, plus size-independent properties."""
+    import torch
+    c = synth.make_config("C4")
+    Dd = torch.from_numpy(c.D).cuda()
+    Qd = torch.from_numpy(c.Q).cuda()
+    idx = dts.build_index_device(Dd)
+    res, stats = dts.search_device(idx, Qd, c.d)
+    got = res.numpy()
+    parity.assert_canonical(got)
+    # every query is a copy of an entry (Q sampled from D): its self pair is a
+    # result over the whole segment
+    nq = c.Q.shape[0]
+    assert np.unique(got["query_id"]).size == nq
+    g = synth.rng(123)
+    qs = np.sort(g.choice(nq, size=48, replace=False))
+    ora = oracle_mod.search_queries(c.D, c.Q, qs, c.d, threads=THREADS)
+    parity.compare(parity.restrict(got, qs), ora, c.D, c.Q, c.d, oracle_mod)
+
+
+# ------------------------------------------------ edge cases and errors
+def test_empty_inputs(dts):
+    D, Q = synth.random_small(5, 10, 10)
+    idx = dts.build_index(D)
+    assert dts.search(idx, np.empty((0, 8)), 0.1).shape[0] == 0
+    empty = dts.build_index(np.empty((0, 8)))
+    assert dts.search(empty, Q, 0.1).shape[0] == 0
+    far = Q.copy()
+    far[:, [0, 4]] += 1e6
+    assert dts.search(idx, far, 0.1).shape[0] == 0
+
+
+def test_huge_result_segment(dts, oracle_mod):
+    """One query with > 4096 results exercises the radix-sorted segment path."""
+    g = synth.rng(77)
+    n = 6000
+    D = np.zeros((n, 8))
+    D[:, 0] = 0.0
+    D[:, 4] = 1.0
+    D[:, 1:4] = g.uniform(0, 0.01, size=(n, 3))
+    D[:, 5:8] = D[:, 1:4]
+    D = D[g.permutation(n)]
+    Q = np.array([[0.0, 0, 0, 0, 1.0, 0.005, 0.005, 0.005], [0.0, 0.5, 0.5, 0.5, 1.0, 1, 1, 1]])
+    got, info = run_and_compare(dts, oracle_mod, D, Q, 0.05)
+    assert info["common"] > 4096
+
+
+def test_invalid_inputs_raise(dts):
+    D, Q = synth.random_small(6, 10, 10)
+    bad = D.copy()
+    bad[3, 2] = np.nan
+    with pytest.raises(dts.DTSError) as e:
+        dts.build_index(bad)
+    assert e.value.status == -1
+    bad = D.copy()
+    bad[4, 4] = bad[4, 0] - 1.0
+    with pytest.raises(dts.DTSError):
+        dts.build_index(bad)
+    idx = dts.build_index(D)
+    with pytest.raises(dts.DTSError):
+        dts.search(idx, Q, -1.0)
+    with pytest.raises(dts.DTSError):
+        dts.search(idx, Q, float("inf"))
+    badq = Q.copy()
+    badq[0, 0] = np.inf
+    with pytest.raises(dts.DTSError):
+        dts.search(idx, badq, 0.1)
+    # the index stays usable after an error
+    assert dts.search(idx, Q, 0.1).dtype == dts.RESULT_DTYPE
