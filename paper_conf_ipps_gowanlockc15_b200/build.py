@@ -14,7 +14,7 @@ LIB = os.path.join(HERE, "libdts.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = [
     "-gencode", "arch=compute_100a,code=sm_100a",
-    "-O3", "-lineinfo", "-std=c++17",
+    "-O3", "-lineinfo", "-std=c++17", "--fmad=false",
     "-Xcompiler", "-fPIC,-O2",
     "-Xptxas", "-v",
     "--expt-relaxed-constexpr",

@@ -92,9 +92,12 @@ void pinned_free(void* p) {
 void free_index_memory(dts_index* idx) {
     if (!idx) return;
     cudaSetDevice(idx->device);
+    // stream-ordered frees keep the pool's pages mapped for the next build
+    // (cudaFree of pool memory would unmap and re-map them every time)
     cudaDeviceSynchronize();
-    if (idx->block) cudaFree(idx->block);
-    if (idx->ht.slots) cudaFree(idx->ht.slots);
+    if (idx->block) cudaFreeAsync(idx->block, cudaStreamPerThread);
+    if (idx->ht.slots) cudaFreeAsync(idx->ht.slots, cudaStreamPerThread);
+    cudaStreamSynchronize(cudaStreamPerThread);
     idx->block = nullptr;
     idx->ht.slots = nullptr;
 }
@@ -269,7 +272,11 @@ dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, s
 void dts_free_results(dts_result* results) { pinned_free(results); }
 
 void dts_free_results_device(dts_result* results) {
-    if (results) cudaFree(results);
+    if (results) {
+        cudaDeviceSynchronize();
+        cudaFreeAsync(results, cudaStreamPerThread);
+        cudaStreamSynchronize(cudaStreamPerThread);
+    }
 }
 
 void dts_free_index(dts_index* index) {

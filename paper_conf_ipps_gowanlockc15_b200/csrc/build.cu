@@ -196,11 +196,24 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
     }
 }
 
+// Counts non-empty cells and writes bin_start[0..m]: the entries of bin j are
+// the sorted positions [bin_start[j], bin_start[j+1]) (the index range
+// [B_first, B_last] of P:L76; keys are bin-major).
 __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __restrict__ keys,
-                                                   size_t n,
+                                                   size_t n, GridParams g,
+                                                   uint32_t* __restrict__ bin_start,
                                                    unsigned long long* __restrict__ count) {
     size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    int f = (p < n) && (p == 0 || keys[p] != keys[p - 1]);
+    int f = 0;
+    if (p < n) {
+        const unsigned long long k = keys[p];
+        f = (p == 0 || k != keys[p - 1]);
+        const long long b = (long long)(k / g.cells_per_bin);
+        const long long bp = p == 0 ? -1 : (long long)(keys[p - 1] / g.cells_per_bin);
+        for (long long bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
+        if (p == n - 1)
+            for (long long bb = b + 1; bb <= g.m; ++bb) bin_start[bb] = (uint32_t)n;
+    }
     int c = __syncthreads_count(f);
     if (threadIdx.x == 0 && c) atomicAdd(count, (unsigned long long)c);
 }
@@ -211,7 +224,7 @@ __global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restr
     if (p >= n) return;
     unsigned long long k = keys[p];
     if (p != 0 && keys[p - 1] == k) return;
-    unsigned long long h = hash_key(k, ht.log2cap);
+    unsigned long long h = slot_of(k, ht.log2cap);
     while (true) {
         unsigned long long prev = atomicCAS(&ht.slots[h].key, EMPTY_KEY, k);
         if (prev == EMPTY_KEY || prev == k) {
@@ -228,7 +241,7 @@ __global__ void __launch_bounds__(BT) k_ends(const unsigned long long* __restric
     if (p >= n) return;
     unsigned long long k = keys[p];
     if (p + 1 != n && keys[p + 1] == k) return;
-    unsigned long long h = hash_key(k, ht.log2cap);
+    unsigned long long h = slot_of(k, ht.log2cap);
     while (ht.slots[h].key != k) h = (h + 1) & ht.mask;
     ht.slots[h].end = (uint32_t)(p + 1);
 }
@@ -320,7 +333,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
 
     // 5. gather into the SoA layout + bin extents
     const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
-    const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double);
+    const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
     char* blk = nullptr;
     DTS_CUDA(cudaMallocAsync((void**)&blk, bytes_soa + bytes_bins + 256, s));
     idx->block = blk;
@@ -331,6 +344,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     idx->bin_t0min = reinterpret_cast<double*>(idx->soa.sz + n);
     idx->bin_t1max = idx->bin_t0min + g.m;
     idx->soa.eid = reinterpret_cast<uint32_t*>(idx->bin_t1max + g.m);
+    idx->bin_start = idx->soa.eid + n;
     unsigned long long* b0 = reinterpret_cast<unsigned long long*>(idx->bin_t0min);
     unsigned long long* b1 = reinterpret_cast<unsigned long long*>(idx->bin_t1max);
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b0, g.m, ~0ull);
@@ -345,7 +359,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // 6. non-empty cells -> hash table
     DevBuf<unsigned long long> ncell(1, s);
     DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
-    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, ncell.p);
+    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, g, idx->bin_start, ncell.p);
     DTS_LAUNCH_CHECK();
     unsigned long long hc = 0;
     DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));

@@ -115,8 +115,12 @@ struct HashTable {
 };
 
 // ---------------------------------------------------------------- device helpers
-__device__ __forceinline__ unsigned long long hash_key(unsigned long long k, int log2cap) {
-    return (k * 0x9E3779B97F4A7C15ull) >> (64 - log2cap);
+// Home slot of a (bin, cell) key.  Keys are row-major with x fastest, so the
+// four keys sharing k >> 2 (x-adjacent cells of one row) hash to the same
+// aligned group of four 16-byte slots: a stencil row of three cells is one or
+// two 64-byte groups instead of three random lines.  Linear probing.
+__device__ __forceinline__ unsigned long long slot_of(unsigned long long k, int log2cap) {
+    return (((k >> 2) * 0x9E3779B97F4A7C15ull) >> (64 - (log2cap - 2))) << 2 | (k & 3ull);
 }
 
 __device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {
@@ -183,6 +187,7 @@ struct dts_index {
     unsigned long long n_cells = 0;
     double* bin_t0min = nullptr;   // per bin: min t_start (bin extent)
     double* bin_t1max = nullptr;   // per bin: max t_end   (B_end of P:L76)
+    uint32_t* bin_start = nullptr; // m + 1 sorted-position offsets of the bins
     void* block = nullptr;         // single device allocation backing the arrays above
     double max_ext[3] = {0, 0, 0};
     float ms_build = 0.f;

@@ -1,5 +1,6 @@
 // search.cu -- the search hot path: query prep, fused candidate streaming +
-// fp64 refinement in two passes (count, scatter), and canonical ordering.
+// fp64 refinement (count pass with staged hits), exact-offset emission, and
+// canonical ordering.
 //
 // Paper (§IV): one GPU thread per query segment loops over a
 // candidate set obtained from the index (GPUSpatial: U_k copied from A, Alg. 1
@@ -10,20 +11,25 @@
 //
 // Here:
 //   * queries are keyed and radix-sorted by the same (bin, cell) key as the
-//     entries, so adjacent warps read the same cells (L1/L2 reuse) -- the
-//     generalisation of "Q sorted by t_start";
-//   * one warp per query: lanes probe the query's stencil of (bin, cell)
-//     keys in parallel (bins filtered by their [min t_start, max t_end]
-//     extent, the B_start/B_end test of P:L76), a warp scan flattens the runs
-//     into one candidate sequence, and the 32 lanes stream 32 consecutive
-//     candidates at a time with four 128-bit loads each (warp-cooperative
-//     candidate tiles instead of one thread per query);
+//     entries, so a CTA's queries and adjacent CTAs read neighbouring cells
+//     (L1/L2 reuse) -- the generalisation of "Q sorted by t_start";
+//   * a CTA takes a tile of TQ consecutive sorted queries.  Phase A: all
+//     (query, bin, cell) probes of the tile are spread over the CTA's threads
+//     (bins filtered by their [min t_start, max t_end] extent, the
+//     B_start/B_end test of P:L76; a query whose stencil would need more
+//     probes than its bins hold entries falls back to the bins' contiguous
+//     range, i.e. GPUTemporal's E_k, as GPUSpatioTemporal falls back in
+//     P:L96).  Phase B: a block scan flattens all runs into one candidate
+//     sequence that the threads stream with four 128-bit loads per candidate;
 //   * refinement in fp64 (readings c1-c4, c8), rejecting on cheap tests before
 //     any sqrt or divide;
-//   * pass 1 counts per query, an exclusive scan gives exact offsets, pass 2
-//     writes each result at offset + ballot rank (no result-buffer overflow,
-//     no re-invocation, deterministic); a per-query sort by entry id makes
-//     the order canonical (reading c7).
+//   * pass 1 counts per query AND stages the tile's hits, sorted by (query,
+//     entry id) in shared memory, in a scratch buffer; an exclusive scan of
+//     the counts gives exact offsets; pass 2 copies each tile's staged hits to
+//     their final positions.  Output is exact-size, canonical (reading c7) and
+//     deterministic.  A tile whose hits overflow its staging space is
+//     recomputed in pass 2 (warp per query, ballot-ranked writes at the exact
+//     offsets) and then sorted per query -- the count-then-scatter fallback.
 #include <algorithm>
 #include <vector>
 
@@ -32,24 +38,39 @@
 namespace dts {
 namespace {
 
-constexpr int PT = 256;                 // threads per CTA in the pass kernels
-constexpr int PW = PT / 32;             // warps per CTA (one query each)
+constexpr int TT = 256;                 // threads per tile CTA
+constexpr int TQ = 64;                  // queries per tile
+constexpr int LMAX = 1024;              // probes (runs) per chunk
+constexpr int HMAX = 1024;              // staged hits per tile
+constexpr int PT = 256;                 // threads per CTA in warp-per-query kernels
+constexpr int PW = PT / 32;
 constexpr int SMALL_SORT = 32;          // warp-register sort limit
 constexpr int LARGE_SORT = 4096;        // CTA shared-memory sort limit
+constexpr unsigned long long NONE = ~0ull;
+
+enum : uint32_t { MODE_DEAD = 0, MODE_GRID = 1, MODE_TEMPORAL = 2 };
 
 struct Counters {                       // device-side statistics / flags
     unsigned long long candidates;
     unsigned long long lookups;
+    unsigned long long staged;          // staging slots reserved
     unsigned int max_count;
     unsigned int n_large;
+    unsigned int n_over;                // tiles recomputed in pass 2
     unsigned int bad;
-    unsigned int pad;
 };
 
 // Query in the velocity form used by the refinement.
 struct QState {
     double t0, t1;
     double x0, vx, y0, vy, z0, vz;
+};
+
+struct Stencil {
+    int32_t lb, hb;          // bin range
+    int32_t clo[3], cn[3];   // cell range per axis (start, count)
+    uint32_t mode;
+    uint32_t nlook;          // probes: ncomb (grid), 1 (temporal), 0 (dead)
 };
 
 // ------------------------------------------------------------- refinement
@@ -125,10 +146,88 @@ __device__ __forceinline__ bool load_query(const double4* __restrict__ Q, uint32
     return fin && dur > 0.0;
 }
 
+// Candidate stencil of a query ("superset" argument):
+// entries filed by t_start bin and MBB-midpoint cell can match only if
+//   t_start in (q.t0 - maxdur, q.t1)                           (strict overlap)
+//   midpoint_a in [qlo_a - d - ext_a/2, qhi_a + d + ext_a/2]    (per axis)
+// both widened by a relative 1e-12 slack that covers fp64 rounding of the
+// midpoints and of these bounds (monotone floor() keeps the superset).
+__device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QState& q,
+                                                const double qlo[3], const double qhi[3],
+                                                double d, bool live,
+                                                const uint32_t* __restrict__ bin_start) {
+    Stencil s;
+    s.mode = MODE_DEAD;
+    s.nlook = 0;
+    s.lb = s.hb = 0;
+    for (int a = 0; a < 3; ++a) { s.clo[a] = 0; s.cn[a] = 1; }
+    if (!live) return s;
+    const double mt = 1e-12 * (fabs(q.t0) + g.maxdur);
+    s.lb = bin_of(g, q.t0 - g.maxdur - mt);
+    s.hb = bin_of(g, q.t1);
+    double ncomb = (double)(s.hb - s.lb + 1);
+#pragma unroll
+    for (int a = 0; a < 3; ++a) {
+        const double ms = 1e-12 * (fabs(qlo[a]) + fabs(qhi[a]) + fabs(g.o[a]) + d + g.half_ext[a]);
+        const double r = d + g.half_ext[a] + ms;
+        s.clo[a] = cell_of(g, a, qlo[a] - r);
+        s.cn[a] = cell_of(g, a, qhi[a] + r) - s.clo[a] + 1;
+        ncomb *= (double)s.cn[a];
+    }
+    const uint32_t T = __ldg(&bin_start[s.hb + 1]) - __ldg(&bin_start[s.lb]);
+    if (T == 0) return s;                                  // no entry in these bins
+    if (ncomb >= (double)T) {                              // probing costs more than scanning
+        s.mode = MODE_TEMPORAL;
+        s.nlook = 1;
+    } else {
+        s.mode = MODE_GRID;
+        s.nlook = (uint32_t)ncomb;
+    }
+    return s;
+}
+
+// Resolve probe `loc` of a query's stencil into an entry run [start, start+cnt).
+__device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht,
+                                        const double* __restrict__ bin_t0min,
+                                        const double* __restrict__ bin_t1max,
+                                        const uint32_t* __restrict__ bin_start, uint32_t mode,
+                                        int32_t lb, int32_t hb, const int32_t clo[3],
+                                        const int32_t cn[3], double qt0, double qt1, uint32_t loc,
+                                        uint32_t& start, uint32_t& cnt, uint32_t& probes) {
+    start = 0;
+    cnt = 0;
+    if (mode == MODE_TEMPORAL) {
+        start = __ldg(&bin_start[lb]);
+        cnt = __ldg(&bin_start[hb + 1]) - start;
+        return;
+    }
+    const uint32_t nyx = (uint32_t)cn[0] * (uint32_t)cn[1];
+    const uint32_t nzyx = nyx * (uint32_t)cn[2];
+    const int32_t bin = lb + (int32_t)(loc / nzyx);
+    uint32_t r = loc % nzyx;
+    const int32_t cz = clo[2] + (int32_t)(r / nyx);
+    r %= nyx;
+    const int32_t cy = clo[1] + (int32_t)(r / (uint32_t)cn[0]);
+    const int32_t cx = clo[0] + (int32_t)(r % (uint32_t)cn[0]);
+    if (!(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0)) return;
+    const unsigned long long key = make_key(g, bin, cx, cy, cz);
+    unsigned long long h = slot_of(key, ht.log2cap);
+    ++probes;
+    while (true) {
+        const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(ht.slots) + h);
+        if (sl.x == key) {
+            start = (uint32_t)sl.y;
+            cnt = (uint32_t)(sl.y >> 32) - start;
+            return;
+        }
+        if (sl.x == EMPTY_KEY) return;
+        h = (h + 1) & ht.mask;
+    }
+}
+
 // --------------------------------------------------------------- query prep
 __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uint32_t nq,
-                                             GridParams g, int have_grid,
-                                             unsigned long long* __restrict__ keys,
+                                             GridParams g, unsigned long long* __restrict__ keys,
                                              uint32_t* __restrict__ ids,
                                              Counters* __restrict__ ctr) {
     uint32_t i = blockIdx.x * PT + threadIdx.x;
@@ -149,15 +248,80 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
     }
     if (bad) atomicOr(&ctr->bad, bad);
     unsigned long long key = 0;
-    if (have_grid && !bad)
+    if (!bad)
         key = make_key(g, bin_of(g, s0.x), cell_of(g, 0, 0.5 * (s0.y + s1.y)),
                        cell_of(g, 1, 0.5 * (s0.z + s1.z)), cell_of(g, 2, 0.5 * (s0.w + s1.w)));
     keys[i] = key;
     ids[i] = i;
 }
 
-// ------------------------------------------------------- fused pass kernel
-struct PassArgs {
+// ------------------------------------------------------------- block helpers
+// Exclusive scan of n <= 4*TT u64 values in shared memory (in place); writes
+// the total to a[n].  All TT threads must call it.
+__device__ void block_scan_u64(unsigned long long* a, int n) {
+    __shared__ unsigned long long warp_tot[TT / 32];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    unsigned long long v[4], s = 0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const int j = tid * 4 + k;
+        v[k] = j < n ? a[j] : 0ull;
+        s += v[k];
+    }
+    unsigned long long inc = s;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        unsigned long long u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= o) inc += u;
+    }
+    if (lane == 31) warp_tot[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+        unsigned long long w = lane < TT / 32 ? warp_tot[lane] : 0ull;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned long long u = __shfl_up_sync(0xffffffffu, w, o);
+            if (lane >= o) w += u;
+        }
+        if (lane < TT / 32) warp_tot[lane] = w;
+    }
+    __syncthreads();
+    unsigned long long run = (warp ? warp_tot[warp - 1] : 0ull) + inc - s;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) {
+        const int j = tid * 4 + k;
+        if (j < n) a[j] = run;
+        run += v[k];
+    }
+    if (tid == TT - 1) a[n] = run;
+    __syncthreads();
+}
+
+// Exclusive scan of TQ (= 64) u64 values, threads 0..63 hold v; result in
+// out[0..TQ] (out[TQ] = total).  All threads must call it.
+__device__ __forceinline__ void tile_scan64(unsigned long long v, unsigned long long* out) {
+    __shared__ unsigned long long w0;
+    const int tid = threadIdx.x, lane = tid & 31;
+    unsigned long long inc = v;
+    if (tid < TQ) {
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned long long u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += u;
+        }
+        if (tid == 31) w0 = inc;
+    }
+    __syncthreads();
+    if (tid < TQ) {
+        if (tid >= 32) inc += w0;
+        out[tid + 1] = inc;
+        if (tid == 0) out[0] = 0ull;
+    }
+    __syncthreads();
+}
+
+// ------------------------------------------------------- pass 1: tile count
+struct TileArgs {
     const double4* Q;
     const uint32_t* order;         // sorted position -> query id
     uint32_t nq;
@@ -167,158 +331,346 @@ struct PassArgs {
     HashTable ht;
     const double* bin_t0min;
     const double* bin_t1max;
+    const uint32_t* bin_start;
     uint32_t* counts;              // per query id
-    const unsigned long long* offsets;
-    dts_result* out;
+    dts_result* stage;             // staged hits (tile-contiguous, canonical inside)
+    unsigned long long stage_cap;
+    unsigned long long* tile_base; // per tile: first staged slot or NONE
+    uint32_t* over_tiles;          // tiles to recompute in pass 2
+    uint32_t* large;               // query ids (recomputed tiles) with count > SMALL_SORT
     uint32_t qid_base;
-    uint32_t* large;               // query ids with count > SMALL_SORT
     Counters* ctr;
 };
 
-template <bool SCATTER>
-__global__ void __launch_bounds__(PT) k_pass(const PassArgs a) {
+struct TileSmem {
+    double qt0[TQ], qt1[TQ], qx0[TQ], qvx[TQ], qy0[TQ], qvy[TQ], qz0[TQ], qvz[TQ];
+    int32_t lb[TQ], hb[TQ], clo[3][TQ], cn[3][TQ];
+    uint32_t qid[TQ], mode[TQ], qcount[TQ];
+    unsigned long long lkoff[TQ + 1];
+    uint32_t rstart[LMAX];
+    unsigned long long roff[LMAX + 1];
+    uint8_t rq[LMAX];
+    unsigned long long hkey[HMAX];
+    double h0[HMAX], h1[HMAX];
+    unsigned long long base;
+    uint32_t nhit, over;
+};
+
+__device__ __forceinline__ QState smem_query(const TileSmem& S, int qi) {
+    QState q;
+    q.t0 = S.qt0[qi]; q.t1 = S.qt1[qi];
+    q.x0 = S.qx0[qi]; q.vx = S.qvx[qi];
+    q.y0 = S.qy0[qi]; q.vy = S.qvy[qi];
+    q.z0 = S.qz0[qi]; q.vz = S.qvz[qi];
+    return q;
+}
+
+__device__ __forceinline__ void stage_hit(TileSmem& S, int qi, uint32_t p, double r0, double r1,
+                                          const uint32_t* __restrict__ eid) {
+    atomicAdd(&S.qcount[qi], 1u);
+    const uint32_t pos = atomicAdd(&S.nhit, 1u);
+    if (pos < (uint32_t)HMAX) {
+        const uint32_t e = __ldg(eid + p);
+        S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)e << 10) | pos;
+        S.h0[pos] = r0;
+        S.h1[pos] = r1;
+    } else {
+        S.over = 1u;
+    }
+}
+
+__global__ void __launch_bounds__(TT, 4) k_tile_count(const TileArgs a) {
+    __shared__ TileSmem S;
+    const int tid = threadIdx.x;
+    const uint32_t tile = blockIdx.x;
+    const GridParams& g = a.g;
+    const double d = a.d, d2 = d * d;
+
+    // ---- phase 0: the tile's queries, stencils and probe counts
+    unsigned long long nlook = 0;
+    if (tid < TQ) {
+        const uint32_t sp = tile * TQ + tid;
+        QState q{};
+        double qlo[3] = {0, 0, 0}, qhi[3] = {0, 0, 0};
+        bool live = false;
+        uint32_t qid = 0;
+        if (sp < a.nq) {
+            qid = a.order[sp];
+            live = load_query(a.Q, qid, q, qlo, qhi);
+        }
+        const Stencil st = make_stencil(g, q, qlo, qhi, d, live, a.bin_start);
+        S.qt0[tid] = q.t0; S.qt1[tid] = q.t1;
+        S.qx0[tid] = q.x0; S.qvx[tid] = q.vx;
+        S.qy0[tid] = q.y0; S.qvy[tid] = q.vy;
+        S.qz0[tid] = q.z0; S.qvz[tid] = q.vz;
+        S.lb[tid] = st.lb; S.hb[tid] = st.hb;
+#pragma unroll
+        for (int ax = 0; ax < 3; ++ax) { S.clo[ax][tid] = st.clo[ax]; S.cn[ax][tid] = st.cn[ax]; }
+        S.qid[tid] = qid;
+        S.mode[tid] = st.mode;
+        S.qcount[tid] = 0;
+        nlook = st.nlook;
+    }
+    if (tid == 0) { S.nhit = 0; S.over = 0; }
+    tile_scan64(nlook, S.lkoff);
+    const unsigned long long Ltot = S.lkoff[TQ];
+
+    unsigned long long n_cand = 0;
+    uint32_t n_probe = 0;
+    for (unsigned long long l0 = 0; l0 < Ltot; l0 += LMAX) {
+        const int nl = (int)min((unsigned long long)LMAX, Ltot - l0);
+        // ---- phase A: probes -> runs
+        for (int j = tid; j < nl; j += TT) {
+            const unsigned long long l = l0 + j;
+            int qi = 0;
+#pragma unroll
+            for (int step = 32; step; step >>= 1)
+                if (S.lkoff[qi + step] <= l) qi += step;
+            const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
+            const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
+            const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
+            uint32_t start, cnt;
+            resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
+                    S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, start, cnt, n_probe);
+            S.rstart[j] = start;
+            S.roff[j] = cnt;
+            S.rq[j] = (uint8_t)qi;
+        }
+        __syncthreads();
+        block_scan_u64(S.roff, nl);
+        const unsigned long long C = S.roff[nl];
+        n_cand += C;
+        // ---- phase B: stream the flattened candidates, two per thread in flight
+        for (unsigned long long c = tid; c < C; c += 2 * TT) {
+            const unsigned long long c2 = c + TT;
+            int j1 = 0, j2 = 0;
+#pragma unroll
+            for (int step = LMAX / 2; step; step >>= 1) {
+                if (j1 + step < nl && S.roff[j1 + step] <= c) j1 += step;
+                if (j2 + step < nl && S.roff[j2 + step] <= c2) j2 += step;
+            }
+            const bool v2 = c2 < C;
+            const uint32_t p1 = S.rstart[j1] + (uint32_t)(c - S.roff[j1]);
+            const uint32_t p2 = v2 ? S.rstart[j2] + (uint32_t)(c2 - S.roff[j2]) : p1;
+            const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
+            const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
+            const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
+            const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
+            const int qi1 = S.rq[j1], qi2 = S.rq[j2];
+            double r0, r1;
+            if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, r0, r1))
+                stage_hit(S, qi1, p1, r0, r1, a.soa.eid);
+            if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, r0, r1))
+                stage_hit(S, qi2, p2, r0, r1, a.soa.eid);
+        }
+        __syncthreads();
+    }
+
+    // ---- statistics
+    {
+        unsigned long long pr = n_probe;
+#pragma unroll
+        for (int o = 16; o; o >>= 1) pr += __shfl_xor_sync(0xffffffffu, pr, o);
+        if ((tid & 31) == 0 && pr) atomicAdd(&a.ctr->lookups, pr);
+        if (tid == 0 && n_cand) atomicAdd(&a.ctr->candidates, n_cand);
+    }
+    // ---- per-query counts
+    if (tid < TQ && tile * TQ + tid < a.nq) {
+        const uint32_t cnt = S.qcount[tid];
+        a.counts[S.qid[tid]] = cnt;
+        if (cnt) atomicMax(&a.ctr->max_count, cnt);
+    }
+    // ---- stage the tile's hits in canonical order
+    const uint32_t nh = S.nhit;
+    if (!S.over && nh > 0) {
+        uint32_t P = 2;
+        while (P < nh) P <<= 1;
+        for (uint32_t j = nh + tid; j < P; j += TT) S.hkey[j] = ~0ull;
+        __syncthreads();
+        for (uint32_t k = 2; k <= P; k <<= 1) {
+            for (uint32_t jj = k >> 1; jj > 0; jj >>= 1) {
+                for (uint32_t t = tid; t < P; t += TT) {
+                    const uint32_t u = t ^ jj;
+                    if (u > t) {
+                        const unsigned long long x = S.hkey[t], y = S.hkey[u];
+                        if ((x > y) == ((t & k) == 0)) {
+                            S.hkey[t] = y;
+                            S.hkey[u] = x;
+                        }
+                    }
+                }
+                __syncthreads();
+            }
+        }
+        if (tid == 0) {
+            const unsigned long long b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
+            if (b + nh > a.stage_cap) S.over = 1u;
+            else S.base = b;
+        }
+        __syncthreads();
+        if (!S.over) {
+            const unsigned long long base = S.base;
+            for (uint32_t i = tid; i < nh; i += TT) {
+                const unsigned long long k = S.hkey[i];
+                const uint32_t slot = (uint32_t)(k & 1023ull);
+                dts_result r;
+                r.query_id = S.qid[(uint32_t)(k >> 42)] + a.qid_base;
+                r.entry_id = (uint32_t)(k >> 10);
+                r.t_start = S.h0[slot];
+                r.t_end = S.h1[slot];
+                a.stage[base + i] = r;
+            }
+            if (tid == 0) a.tile_base[tile] = base;
+        }
+    } else if (!S.over && tid == 0) {
+        a.tile_base[tile] = NONE - 1;        // no hits: nothing to emit
+    }
+    __syncthreads();
+    if (S.over) {
+        if (tid == 0) {
+            a.tile_base[tile] = NONE;
+            const uint32_t slot = atomicAdd(&a.ctr->n_over, 1u);
+            a.over_tiles[slot] = tile;
+        }
+        if (tid < TQ && tile * TQ + tid < a.nq && S.qcount[tid] > (uint32_t)SMALL_SORT) {
+            const uint32_t slot = atomicAdd(&a.ctr->n_large, 1u);
+            a.large[slot] = S.qid[tid];
+        }
+    }
+}
+
+// ------------------------------------------------------ pass 2: emission
+__global__ void __launch_bounds__(TT) k_tile_emit(const uint32_t* __restrict__ order, uint32_t nq,
+                                                 const uint32_t* __restrict__ counts,
+                                                 const unsigned long long* __restrict__ offsets,
+                                                 const unsigned long long* __restrict__ tile_base,
+                                                 const dts_result* __restrict__ stage,
+                                                 dts_result* __restrict__ out) {
+    __shared__ unsigned long long qpre[TQ + 1];
+    __shared__ uint32_t qid_s[TQ];
+    const uint32_t tile = blockIdx.x;
+    const unsigned long long tb = tile_base[tile];
+    if (tb >= NONE - 1) return;                      // recomputed or empty tile
+    const int tid = threadIdx.x;
+    unsigned long long cnt = 0;
+    if (tid < TQ) {
+        const uint32_t sp = tile * TQ + tid;
+        uint32_t qid = 0;
+        if (sp < nq) {
+            qid = order[sp];
+            cnt = counts[qid];
+        }
+        qid_s[tid] = qid;
+    }
+    tile_scan64(cnt, qpre);
+    const unsigned long long nh = qpre[TQ];
+    for (unsigned long long i = tid; i < nh; i += TT) {
+        int qi = 0;
+#pragma unroll
+        for (int step = 32; step; step >>= 1)
+            if (qpre[qi + step] <= i) qi += step;
+        out[offsets[qid_s[qi]] + (i - qpre[qi])] = stage[tb + i];
+    }
+}
+
+// -------------------------------- fallback: warp-per-query scatter (pass 2)
+struct PassArgs {
+    const double4* Q;
+    const uint32_t* order;
+    uint32_t nq;
+    double d;
+    GridParams g;
+    SegSoA soa;
+    HashTable ht;
+    const double* bin_t0min;
+    const double* bin_t1max;
+    const uint32_t* bin_start;
+    const unsigned long long* offsets;
+    const uint32_t* tiles;         // tiles to process (TQ sorted positions each)
+    dts_result* out;
+    uint32_t qid_base;
+};
+
+// Warp w of CTA b processes sorted position tiles[b / (TQ/PW)]*TQ + ...; the
+// warp's lanes probe 32 stencil cells at a time, a warp scan flattens the
+// runs, lanes stream 32 candidates at a time and write hits at the query's
+// exact offset + ballot rank (deterministic order, sorted afterwards).
+__global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
     __shared__ uint32_t s_start[PW][32];
     __shared__ uint32_t s_excl[PW][32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t sq = blockIdx.x * PW + warp;
+    constexpr int CTAS_PER_TILE = TQ / PW;
+    const uint32_t tile = a.tiles[blockIdx.x / CTAS_PER_TILE];
+    const uint32_t sq = tile * TQ + (blockIdx.x % CTAS_PER_TILE) * PW + warp;
     if (sq >= a.nq) return;
     const uint32_t qid = a.order[sq];
     QState q;
     double qlo[3], qhi[3];
     const bool live = load_query(a.Q, qid, q, qlo, qhi);
-    const GridParams& g = a.g;
-    const double d = a.d, d2 = d * d;
-
-    uint32_t my_hits = 0;
-    unsigned long long out_pos = SCATTER ? a.offsets[qid] : 0ull;
-    unsigned long long n_cand = 0, n_look = 0;
-
-    if (live) {
-        // temporal stencil: entries with t_start in (q.t0 - maxdur, q.t1)
-        const double mt = 1e-12 * (fabs(q.t0) + g.maxdur);
-        const int32_t lb = bin_of(g, q.t0 - g.maxdur - mt);
-        const int32_t hb = bin_of(g, q.t1);
-        // spatial stencil: MBB midpoint within d + half extent of the query MBB
-        int32_t clo[3], cn[3];
+    const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start);
+    const double d2 = a.d * a.d;
+    unsigned long long out_pos = a.offsets[qid];
+    uint32_t dummy = 0;
+    for (uint32_t c0 = 0; c0 < st.nlook; c0 += 32) {
+        const uint32_t c = c0 + lane;
+        uint32_t start = 0, cnt = 0;
+        if (c < st.nlook)
+            resolve(a.g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, st.mode, st.lb, st.hb,
+                    st.clo, st.cn, q.t0, q.t1, c, start, cnt, dummy);
+        unsigned long long incl = cnt;
 #pragma unroll
-        for (int ax = 0; ax < 3; ++ax) {
-            const double ms = 1e-12 * (fabs(qlo[ax]) + fabs(qhi[ax]) + fabs(g.o[ax]) + d +
-                                       g.half_ext[ax]);
-            const double r = d + g.half_ext[ax] + ms;
-            clo[ax] = cell_of(g, ax, qlo[ax] - r);
-            cn[ax] = cell_of(g, ax, qhi[ax] + r) - clo[ax] + 1;
+        for (int o = 1; o < 32; o <<= 1) {
+            unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += u;
         }
-        const unsigned long long ncomb = (unsigned long long)(hb - lb + 1) * (unsigned)cn[0] *
-                                         (unsigned)cn[1] * (unsigned)cn[2];
-        const unsigned long long nyx = (unsigned long long)cn[0] * (unsigned)cn[1];
-        const unsigned long long nzyx = nyx * (unsigned)cn[2];
-        for (unsigned long long c0 = 0; c0 < ncomb; c0 += 32) {
-            // ---- lookups: one (bin, cell) per lane
-            const unsigned long long c = c0 + lane;
-            uint32_t start = 0, cnt = 0;
-            if (c < ncomb) {
-                const int32_t bin = lb + (int32_t)(c / nzyx);
-                unsigned long long r = c % nzyx;
-                const int32_t cz = clo[2] + (int32_t)(r / nyx);
-                r %= nyx;
-                const int32_t cy = clo[1] + (int32_t)(r / (unsigned)cn[0]);
-                const int32_t cx = clo[0] + (int32_t)(r % (unsigned)cn[0]);
-                if (__ldg(&a.bin_t0min[bin]) < q.t1 && __ldg(&a.bin_t1max[bin]) > q.t0) {
-                    const unsigned long long key = make_key(g, bin, cx, cy, cz);
-                    unsigned long long h = hash_key(key, a.ht.log2cap);
-                    ++n_look;
-                    while (true) {
-                        const ulonglong2 sl =
-                            __ldg(reinterpret_cast<const ulonglong2*>(a.ht.slots) + h);
-                        if (sl.x == key) {
-                            start = (uint32_t)sl.y;
-                            cnt = (uint32_t)(sl.y >> 32) - start;
-                            break;
-                        }
-                        if (sl.x == EMPTY_KEY) break;
-                        h = (h + 1) & a.ht.mask;
-                    }
-                }
-            }
-            // ---- flatten the up-to-32 runs into one candidate sequence
-            uint32_t incl = cnt;
+        const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
+        __syncwarp();
+        s_start[warp][lane] = start;
+        s_excl[warp][lane] = (uint32_t)(incl - cnt);   // < 2^32: runs of one query
+        __syncwarp();
+        for (unsigned long long base = 0; base < total; base += 32) {
+            const unsigned long long t = base + lane;
+            bool hit = false;
+            double r0 = 0.0, r1 = 0.0;
+            uint32_t p = 0;
+            if (t < total) {
+                int j = 0;
 #pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += u;
+                for (int step = 16; step; step >>= 1)
+                    if (s_excl[warp][j + step] <= t) j += step;
+                p = s_start[warp][j] + (uint32_t)(t - s_excl[warp][j]);
+                hit = refine(q, __ldg(a.soa.st + p), __ldg(a.soa.sx + p), __ldg(a.soa.sy + p),
+                             __ldg(a.soa.sz + p), d2, r0, r1);
             }
-            const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-            __syncwarp();
-            s_start[warp][lane] = start;
-            s_excl[warp][lane] = incl - cnt;
-            __syncwarp();
-            n_cand += total;
-            // ---- stream candidates 32 at a time
-            for (uint32_t base = 0; base < total; base += 32) {
-                const uint32_t t = base + lane;
-                bool hit = false;
-                double r0 = 0.0, r1 = 0.0;
-                uint32_t p = 0;
-                if (t < total) {
-                    int j = 0;
-#pragma unroll
-                    for (int step = 16; step; step >>= 1)
-                        if (s_excl[warp][j + step] <= t) j += step;
-                    p = s_start[warp][j] + (t - s_excl[warp][j]);
-                    const double2 st = __ldg(a.soa.st + p);
-                    const double2 sx = __ldg(a.soa.sx + p);
-                    const double2 sy = __ldg(a.soa.sy + p);
-                    const double2 sz = __ldg(a.soa.sz + p);
-                    hit = refine(q, st, sx, sy, sz, d2, r0, r1);
-                }
-                if (SCATTER) {
-                    const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-                    if (hit) {
-                        const unsigned long long pos =
-                            out_pos + __popc(bal & ((1u << lane) - 1u));
-                        dts_result rr;
-                        rr.query_id = qid + a.qid_base;
-                        rr.entry_id = __ldg(a.soa.eid + p);
-                        rr.t_start = r0;
-                        rr.t_end = r1;
-                        a.out[pos] = rr;
-                    }
-                    out_pos += __popc(bal);
-                } else {
-                    my_hits += hit ? 1u : 0u;
-                }
+            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
+            if (hit) {
+                dts_result rr;
+                rr.query_id = qid + a.qid_base;
+                rr.entry_id = __ldg(a.soa.eid + p);
+                rr.t_start = r0;
+                rr.t_end = r1;
+                a.out[out_pos + __popc(bal & ((1u << lane) - 1u))] = rr;
             }
-        }
-    }
-    if (!SCATTER) {
-#pragma unroll
-        for (int o = 16; o; o >>= 1) {
-            my_hits += __shfl_xor_sync(0xffffffffu, my_hits, o);
-            n_look += __shfl_xor_sync(0xffffffffu, n_look, o);
-        }
-        if (lane == 0) {
-            a.counts[qid] = my_hits;
-            atomicAdd(&a.ctr->candidates, n_cand);
-            atomicAdd(&a.ctr->lookups, n_look);
-            if (my_hits) atomicMax(&a.ctr->max_count, my_hits);
-            if (my_hits > (uint32_t)SMALL_SORT) {
-                uint32_t slot = atomicAdd(&a.ctr->n_large, 1u);
-                a.large[slot] = qid;
-            }
+            out_pos += __popc(bal);
         }
     }
 }
 
 // ------------------------------------------------------ canonical order
-// One warp per query with 2..32 results: bitonic sort by entry id across
-// lanes (entry ids of one query are distinct), payload moved by shuffles.
-__global__ void __launch_bounds__(PT) k_canon_small(const uint32_t* __restrict__ counts,
+// Fallback tiles: one warp per query with 2..32 results, bitonic sort by
+// entry id across lanes (entry ids of one query are distinct).
+__global__ void __launch_bounds__(PT) k_canon_small(const uint32_t* __restrict__ tiles,
+                                                   const uint32_t* __restrict__ order, uint32_t nq,
+                                                   const uint32_t* __restrict__ counts,
                                                    const unsigned long long* __restrict__ offsets,
-                                                   uint32_t nq, const dts_result* __restrict__ raw,
+                                                   const dts_result* __restrict__ raw,
                                                    dts_result* __restrict__ out) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t q = blockIdx.x * PW + warp;
-    if (q >= nq) return;
+    constexpr int CTAS_PER_TILE = TQ / PW;
+    const uint32_t tile = tiles[blockIdx.x / CTAS_PER_TILE];
+    const uint32_t sq = tile * TQ + (blockIdx.x % CTAS_PER_TILE) * PW + warp;
+    if (sq >= nq) return;
+    const uint32_t q = order[sq];
     const uint32_t cnt = counts[q];
     if (cnt == 0 || cnt > (uint32_t)SMALL_SORT) return;
     const unsigned long long base = offsets[q];
@@ -441,7 +793,7 @@ struct EventTimer {
     EventTimer(bool enable, cudaStream_t st) : on(enable), s(st) {
         if (on) for (auto& e : ev) DTS_CUDA(cudaEventCreate(&e));
     }
-    void mark() { if (on) DTS_CUDA(cudaEventRecord(ev[k++], s)); }
+    void mark() { if (on && k < 6) DTS_CUDA(cudaEventRecord(ev[k++], s)); }
     float ms(int i) {
         float t = 0.f;
         if (on && i + 1 < k) cudaEventElapsedTime(&t, ev[i], ev[i + 1]);
@@ -480,36 +832,42 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     EventTimer tm(local.time_kernels != 0, s);
     tm.mark();
     // ---- query prep: key + sort
-    DevBuf<unsigned long long> qk(nq, s), qk_tmp(nq, s);
-    DevBuf<uint32_t> order(nq, s), order_tmp(nq, s);
-    k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, 1, qk.p, order.p, ctr.p);
-    DTS_LAUNCH_CHECK();
-    radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
-    qk_tmp.release();
-    order_tmp.release();
-    qk.release();
+    DevBuf<uint32_t> order(nq, s);
+    {
+        DevBuf<unsigned long long> qk(nq, s), qk_tmp(nq, s);
+        DevBuf<uint32_t> order_tmp(nq, s);
+        k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p, order.p, ctr.p);
+        DTS_LAUNCH_CHECK();
+        radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
+    }
     tm.mark();
 
-    // ---- pass 1: count
-    DevBuf<uint32_t> counts(nq, s), large(nq, s);
-    DevBuf<unsigned long long> offsets(nq + 1, s);
-    PassArgs pa;
-    pa.Q = Q;
-    pa.order = order.p;
-    pa.nq = (uint32_t)nq;
-    pa.d = d;
-    pa.g = idx->gp;
-    pa.soa = idx->soa;
-    pa.ht = idx->ht;
-    pa.bin_t0min = idx->bin_t0min;
-    pa.bin_t1max = idx->bin_t1max;
-    pa.counts = counts.p;
-    pa.offsets = offsets.p;
-    pa.out = nullptr;
-    pa.qid_base = qid_base;
-    pa.large = large.p;
-    pa.ctr = ctr.p;
-    k_pass<false><<<blocks(nq, PW), PT, 0, s>>>(pa);
+    // ---- pass 1: tile count + staging
+    const uint32_t ntiles = (uint32_t)((nq + TQ - 1) / TQ);
+    const unsigned long long stage_cap = 4ull * nq + (1ull << 20);
+    DevBuf<uint32_t> counts(nq, s), large(nq, s), over_tiles(ntiles, s);
+    DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s);
+    DevBuf<dts_result> stage(stage_cap, s);
+    TileArgs ta;
+    ta.Q = Q;
+    ta.order = order.p;
+    ta.nq = (uint32_t)nq;
+    ta.d = d;
+    ta.g = idx->gp;
+    ta.soa = idx->soa;
+    ta.ht = idx->ht;
+    ta.bin_t0min = idx->bin_t0min;
+    ta.bin_t1max = idx->bin_t1max;
+    ta.bin_start = idx->bin_start;
+    ta.counts = counts.p;
+    ta.stage = stage.p;
+    ta.stage_cap = stage_cap;
+    ta.tile_base = tile_base.p;
+    ta.over_tiles = over_tiles.p;
+    ta.large = large.p;
+    ta.qid_base = qid_base;
+    ta.ctr = ctr.p;
+    k_tile_count<<<ntiles, TT, 0, s>>>(ta);
     DTS_LAUNCH_CHECK();
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
@@ -532,45 +890,70 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     local.max_results_per_query = h.c.max_count;
 
     if (h.total > 0) {
-        // ---- pass 2: scatter at exact offsets, then canonical order
-        DevBuf<dts_result> raw(h.total, s);
         dts_result* fin = nullptr;
         DTS_CUDA(cudaMallocAsync((void**)&fin, h.total * sizeof(dts_result), s));
         try {
-            pa.out = raw.p;
-            k_pass<true><<<blocks(nq, PW), PT, 0, s>>>(pa);
+            // ---- pass 2: staged tiles are copied to their exact offsets
+            k_tile_emit<<<ntiles, TT, 0, s>>>(order.p, (uint32_t)nq, counts.p, offsets.p,
+                                              tile_base.p, stage.p, fin);
             DTS_LAUNCH_CHECK();
-            tm.mark();
-            k_canon_small<<<blocks(nq, PW), PT, 0, s>>>(counts.p, offsets.p, (uint32_t)nq, raw.p,
-                                                        fin);
-            DTS_LAUNCH_CHECK();
-            if (h.c.n_large) {
-                const unsigned g = (unsigned)std::min<uint32_t>(h.c.n_large, 148 * 4);
-                k_canon_large<<<g, PT, 0, s>>>(large.p, ctr.p, counts.p, offsets.p, raw.p, fin);
+            // ---- overflowed tiles: recompute with exact offsets, then sort
+            if (h.c.n_over) {
+                DevBuf<dts_result> raw(h.total, s);
+                PassArgs pa;
+                pa.Q = Q;
+                pa.order = order.p;
+                pa.nq = (uint32_t)nq;
+                pa.d = d;
+                pa.g = idx->gp;
+                pa.soa = idx->soa;
+                pa.ht = idx->ht;
+                pa.bin_t0min = idx->bin_t0min;
+                pa.bin_t1max = idx->bin_t1max;
+                pa.bin_start = idx->bin_start;
+                pa.offsets = offsets.p;
+                pa.tiles = over_tiles.p;
+                pa.out = raw.p;
+                pa.qid_base = qid_base;
+                const unsigned nb = h.c.n_over * (TQ / PW);
+                k_pass_scatter<<<nb, PT, 0, s>>>(pa);
                 DTS_LAUNCH_CHECK();
-            }
-            if (h.c.max_count > (uint32_t)LARGE_SORT) {
-                std::vector<uint32_t> hl(h.c.n_large);
-                DTS_CUDA(cudaMemcpyAsync(hl.data(), large.p, hl.size() * sizeof(uint32_t),
-                                         cudaMemcpyDeviceToHost, s));
-                DTS_CUDA(cudaStreamSynchronize(s));
-                for (uint32_t qh : hl) {
-                    uint32_t cnt;
-                    unsigned long long base;
-                    DTS_CUDA(cudaMemcpyAsync(&cnt, counts.p + qh, 4, cudaMemcpyDeviceToHost, s));
-                    DTS_CUDA(cudaMemcpyAsync(&base, offsets.p + qh, 8, cudaMemcpyDeviceToHost, s));
-                    DTS_CUDA(cudaStreamSynchronize(s));
-                    if (cnt <= (uint32_t)LARGE_SORT) continue;
-                    DevBuf<unsigned long long> k1(cnt, s), k2(cnt, s);
-                    DevBuf<uint32_t> v1(cnt, s), v2(cnt, s);
-                    k_seg_keys<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, k1.p, v1.p);
-                    DTS_LAUNCH_CHECK();
-                    radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, cnt,
-                                     bits_for(idx->n ? idx->n - 1 : 0), s);
-                    k_seg_gather<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, v1.p,
-                                                                fin + base);
+                tm.mark();
+                k_canon_small<<<nb, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq, counts.p,
+                                                offsets.p, raw.p, fin);
+                DTS_LAUNCH_CHECK();
+                if (h.c.n_large) {
+                    const unsigned gl = (unsigned)std::min<uint32_t>(h.c.n_large, 148 * 4);
+                    k_canon_large<<<gl, PT, 0, s>>>(large.p, ctr.p, counts.p, offsets.p, raw.p,
+                                                    fin);
                     DTS_LAUNCH_CHECK();
                 }
+                if (h.c.max_count > (uint32_t)LARGE_SORT && h.c.n_large) {
+                    std::vector<uint32_t> hl(h.c.n_large);
+                    DTS_CUDA(cudaMemcpyAsync(hl.data(), large.p, hl.size() * sizeof(uint32_t),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                    for (uint32_t qh : hl) {
+                        uint32_t cnt;
+                        unsigned long long base;
+                        DTS_CUDA(cudaMemcpyAsync(&cnt, counts.p + qh, 4, cudaMemcpyDeviceToHost, s));
+                        DTS_CUDA(cudaMemcpyAsync(&base, offsets.p + qh, 8, cudaMemcpyDeviceToHost,
+                                                 s));
+                        DTS_CUDA(cudaStreamSynchronize(s));
+                        if (cnt <= (uint32_t)LARGE_SORT) continue;
+                        DevBuf<unsigned long long> k1(cnt, s), k2(cnt, s);
+                        DevBuf<uint32_t> v1(cnt, s), v2(cnt, s);
+                        k_seg_keys<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, k1.p, v1.p);
+                        DTS_LAUNCH_CHECK();
+                        radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, cnt,
+                                         bits_for(idx->n ? idx->n - 1 : 0), s);
+                        k_seg_gather<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, v1.p,
+                                                                    fin + base);
+                        DTS_LAUNCH_CHECK();
+                    }
+                }
+            } else {
+                tm.mark();
             }
             tm.mark();
             DTS_CUDA(cudaStreamSynchronize(s));

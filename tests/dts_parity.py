@@ -1,7 +1,11 @@
 """Parity rule (BASELINE.json north_star; readings c11, c10):
 
 * the result pair set must equal the oracle's, except pairs whose minimum
-  distance (computed by the oracle's routine) lies within 1e-9*d of d;
+  distance (computed by the oracle's routine) lies within 1e-9*d of d, plus
+  the fp64 rounding floor 1e-12*L of a distance computed from coordinates of
+  magnitude L = max |coordinate| (reading c11: without the floor the band is
+  empty at d = 0, where a pair that touches at one instant is a rounding
+  decision of either implementation);
 * interval endpoints of common pairs agree within 1e-9 in normalised time
   t^ = (t - t_min(D)) / (t_max(D) - t_min(D));
 * results are in canonical (query_id, entry_id) order with no duplicates.
@@ -9,7 +13,16 @@
 import numpy as np
 
 BAND = 1e-9
+FLOOR = 1e-12
 TOL_T = 1e-9
+
+
+def band(D, Q, d):
+    Dv = np.asarray(D).reshape(-1, 8)[:, [1, 2, 3, 5, 6, 7]]
+    Qv = np.asarray(Q).reshape(-1, 8)[:, [1, 2, 3, 5, 6, 7]]
+    L = max(float(np.abs(Dv).max()) if Dv.size else 0.0,
+            float(np.abs(Qv).max()) if Qv.size else 0.0)
+    return BAND * d + FLOOR * L
 
 
 def keys(res) -> np.ndarray:
@@ -35,7 +48,7 @@ def compare(gpu, ora, D, Q, d, oracle_mod, qid_base=0, tol_t=TOL_T):
         qids = (diff >> np.uint64(32)).astype(np.int64) - qid_base
         eids = (diff & np.uint64(0xffffffff)).astype(np.int64)
         dm = oracle_mod.dmin_pairs(D, Q, qids, eids)
-        bad = ~(np.abs(dm - d) <= BAND * d)
+        bad = ~(np.abs(dm - d) <= band(D, Q, d))
         if np.any(bad):
             i = int(np.flatnonzero(bad)[0])
             raise AssertionError(
