@@ -92,12 +92,10 @@ void pinned_free(void* p) {
 void free_index_memory(dts_index* idx) {
     if (!idx) return;
     cudaSetDevice(idx->device);
-    // stream-ordered frees keep the pool's pages mapped for the next build
-    // (cudaFree of pool memory would unmap and re-map them every time)
+    // blocks go back to the device cache (alloc.cu) for the next build
     cudaDeviceSynchronize();
-    if (idx->block) cudaFreeAsync(idx->block, cudaStreamPerThread);
-    if (idx->ht.slots) cudaFreeAsync(idx->ht.slots, cudaStreamPerThread);
-    cudaStreamSynchronize(cudaStreamPerThread);
+    cache_free(idx->block);
+    cache_free(idx->ht.slots);
     idx->block = nullptr;
     idx->ht.slots = nullptr;
 }
@@ -205,10 +203,11 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
                     DTS_CUDA(cudaStreamSynchronize(s));
                 } catch (...) {
                     pinned_free(h);
-                    cudaFreeAsync(so.results, s);
+                    cudaStreamSynchronize(s);
+                    cache_free(so.results);
                     throw;
                 }
-                cudaFreeAsync(so.results, s);
+                cache_free(so.results);
                 ret = h;
                 cnt = so.count;
             }
@@ -274,8 +273,7 @@ void dts_free_results(dts_result* results) { pinned_free(results); }
 void dts_free_results_device(dts_result* results) {
     if (results) {
         cudaDeviceSynchronize();
-        cudaFreeAsync(results, cudaStreamPerThread);
-        cudaStreamSynchronize(cudaStreamPerThread);
+        cache_free(results);
     }
 }
 

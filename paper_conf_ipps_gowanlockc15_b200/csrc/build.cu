@@ -15,10 +15,11 @@
 //   5. k_gather       sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz)
 //                     + per-bin [min t_start, max t_end] extents (B_start/B_end
 //                     of P:L76) with warp-aggregated atomics.
-//   6. k_count_cells / k_insert / k_ends
-//                     non-empty cells -> open-addressing hash table
-//                     key -> [start, end) (the role of G and A of P:L44, with no
-//                     duplicated ids since every entry is in exactly one cell).
+//   6. k_count_cells / k_insert
+//                     bin offsets (B_first of P:L76) and non-empty cells ->
+//                     open-addressing hash table key -> [start, end) (the role
+//                     of G and A of P:L44, with no duplicated ids since every
+//                     entry is in exactly one cell).
 #include <algorithm>
 #include <cmath>
 
@@ -141,18 +142,50 @@ __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
 }
 
+constexpr int GATHER_ITEMS = 4;   // rows in flight per thread
+
+__device__ __forceinline__ void gather_one(const double4& s0, const double4& s1, size_t p,
+                                           uint32_t i, GridParams g, SegSoA& soa,
+                                           unsigned long long* __restrict__ bin_t0min,
+                                           unsigned long long* __restrict__ bin_t1max, bool ok);
+
+// Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
+// (strided by the CTA so stores stay coalesced), all row loads issued first.
 __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
                                               const uint32_t* __restrict__ ids, GridParams g,
                                               SegSoA soa,
                                               unsigned long long* __restrict__ bin_t0min,
                                               unsigned long long* __restrict__ bin_t1max) {
-    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    bool ok = p < n;
+    const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
+    uint32_t id[GATHER_ITEMS];
+    double4 r0[GATHER_ITEMS], r1[GATHER_ITEMS];
+#pragma unroll
+    for (int k = 0; k < GATHER_ITEMS; ++k) {
+        const size_t p = base + (size_t)k * BT;
+        id[k] = p < n ? __ldg(ids + p) : 0u;
+    }
+#pragma unroll
+    for (int k = 0; k < GATHER_ITEMS; ++k) {
+        const size_t p = base + (size_t)k * BT;
+        if (p < n) {
+            r0[k] = D[2 * (size_t)id[k]];
+            r1[k] = D[2 * (size_t)id[k] + 1];
+        }
+    }
+#pragma unroll
+    for (int k = 0; k < GATHER_ITEMS; ++k) {
+        const size_t p = base + (size_t)k * BT;
+        gather_one(r0[k], r1[k], p, id[k], g, soa, bin_t0min, bin_t1max, p < n);
+    }
+}
+
+__device__ __forceinline__ void gather_one(const double4& s0, const double4& s1, size_t p,
+                                           uint32_t i, GridParams g, SegSoA& soa,
+                                           unsigned long long* __restrict__ bin_t0min,
+                                           unsigned long long* __restrict__ bin_t1max, bool ok) {
     int32_t bin = -1;
     unsigned long long o0 = ~0ull, o1 = 0ull;
     if (ok) {
-        uint32_t i = ids[p];
-        double4 s0 = D[2 * (size_t)i], s1 = D[2 * (size_t)i + 1];
         double dur = s1.x - s0.x;
         soa.st[p] = make_double2(s0.x, s1.x);
         soa.sx[p] = make_double2(s0.y, velocity(s0.y, s1.y, dur));
@@ -224,26 +257,19 @@ __global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restr
     if (p >= n) return;
     unsigned long long k = keys[p];
     if (p != 0 && keys[p - 1] == k) return;
+    // the cell's run ends at the next key change (most cells hold 1-3 entries)
+    size_t e = p + 1;
+    while (e < n && keys[e] == k) ++e;
     unsigned long long h = slot_of(k, ht.log2cap);
     while (true) {
         unsigned long long prev = atomicCAS(&ht.slots[h].key, EMPTY_KEY, k);
         if (prev == EMPTY_KEY || prev == k) {
             ht.slots[h].start = (uint32_t)p;
+            ht.slots[h].end = (uint32_t)e;
             return;
         }
         h = (h + 1) & ht.mask;
     }
-}
-
-__global__ void __launch_bounds__(BT) k_ends(const unsigned long long* __restrict__ keys, size_t n,
-                                            HashTable ht) {
-    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    if (p >= n) return;
-    unsigned long long k = keys[p];
-    if (p + 1 != n && keys[p + 1] == k) return;
-    unsigned long long h = slot_of(k, ht.log2cap);
-    while (ht.slots[h].key != k) h = (h + 1) & ht.mask;
-    ht.slots[h].end = (uint32_t)(p + 1);
 }
 
 inline unsigned grid_for(size_t n) { return (unsigned)((n + BT - 1) / BT); }
@@ -335,7 +361,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
     const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
     char* blk = nullptr;
-    DTS_CUDA(cudaMallocAsync((void**)&blk, bytes_soa + bytes_bins + 256, s));
+    blk = static_cast<char*>(cache_alloc(bytes_soa + bytes_bins + 256));
     idx->block = blk;
     idx->soa.st = reinterpret_cast<double2*>(blk);
     idx->soa.sx = idx->soa.st + n;
@@ -351,7 +377,8 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
-    k_gather<<<grid_for(n), BT, 0, s>>>(D, n, ids.p, g, idx->soa, b0, b1);
+    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, ids.p, g,
+                                                                         idx->soa, b0, b1);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
@@ -369,11 +396,9 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     while ((1ull << log2cap) < 2 * hc) ++log2cap;
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
-    DTS_CUDA(cudaMallocAsync((void**)&idx->ht.slots, sizeof(CellSlot) << log2cap, s));
+    idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
     k_insert<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
-    DTS_LAUNCH_CHECK();
-    k_ends<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
     DTS_LAUNCH_CHECK();
 
     DTS_CUDA(cudaEventRecord(e1, s));

@@ -175,6 +175,10 @@ void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long lo
 
 int bits_for(unsigned long long max_value);
 
+// Device block cache (alloc.cu) for memory that outlives one API call.
+void* cache_alloc(size_t bytes);
+void cache_free(void* p);
+
 }  // namespace dts
 
 // The opaque index (definition shared by build.cu, search.cu and api.cu).

@@ -161,6 +161,10 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
     __shared__ uint32_t wcnt[RS_WARPS][RS_RADIX + 1];
     __shared__ uint32_t tile_base[RS_RADIX];
+    __shared__ uint32_t local_off[RS_RADIX];
+    __shared__ uint32_t warp_tot[RS_WARPS];
+    __shared__ unsigned long long sk[RS_TILE];
+    __shared__ uint32_t sv[RS_TILE];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int j = lane; j < RS_RADIX + 1; j += 32) wcnt[warp][j] = 0;
     tile_base[threadIdx.x] = offsets[(size_t)threadIdx.x * ntiles + blockIdx.x];
@@ -192,6 +196,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         __syncwarp();
     }
     __syncthreads();
+    uint32_t tile_count;
     {
         const int dgt = threadIdx.x;   // RS_THREADS == RS_RADIX
         uint32_t run = 0;
@@ -201,15 +206,44 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
             wcnt[w][dgt] = run;
             run += c;
         }
+        tile_count = run;
+    }
+    // tile-local digit offsets (exclusive scan of the tile histogram)
+    {
+        const int lane2 = threadIdx.x & 31, w2 = threadIdx.x >> 5;
+        uint32_t inc = tile_count;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane2 >= o) inc += u;
+        }
+        if (lane2 == 31) warp_tot[w2] = inc;
+        __syncthreads();
+        uint32_t pre = 0;
+        for (int w = 0; w < w2; ++w) pre += warp_tot[w];
+        local_off[threadIdx.x] = pre + inc - tile_count;
     }
     __syncthreads();
+    // stage the tile in digit order in shared memory ...
 #pragma unroll
     for (int i = 0; i < RS_ITEMS; ++i) {
         if (dig[i] < (uint32_t)RS_RADIX) {
-            uint32_t dst = tile_base[dig[i]] + wcnt[warp][dig[i]] + rank[i];
-            keys_out[dst] = k[i];
-            vals_out[dst] = v[i];
+            const uint32_t lpos = local_off[dig[i]] + wcnt[warp][dig[i]] + rank[i];
+            sk[lpos] = k[i];
+            sv[lpos] = v[i];
         }
+    }
+    __syncthreads();
+    // ... then write it out with consecutive threads on consecutive positions
+    // of each digit's output run (coalesced instead of 32 scattered lines)
+    const size_t tbase = (size_t)blockIdx.x * RS_TILE;
+    const uint32_t tn = (uint32_t)min((size_t)RS_TILE, n - tbase);
+    for (uint32_t i = threadIdx.x; i < tn; i += RS_THREADS) {
+        const unsigned long long key = sk[i];
+        const uint32_t dg = (uint32_t)(key >> shift) & (RS_RADIX - 1);
+        const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
+        keys_out[dst] = key;
+        vals_out[dst] = sv[i];
     }
 }
 static_assert(RS_THREADS == RS_RADIX, "one thread per digit in the cross-warp prefix");

@@ -891,7 +891,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 
     if (h.total > 0) {
         dts_result* fin = nullptr;
-        DTS_CUDA(cudaMallocAsync((void**)&fin, h.total * sizeof(dts_result), s));
+        fin = static_cast<dts_result*>(cache_alloc(h.total * sizeof(dts_result)));
         try {
             // ---- pass 2: staged tiles are copied to their exact offsets
             k_tile_emit<<<ntiles, TT, 0, s>>>(order.p, (uint32_t)nq, counts.p, offsets.p,
@@ -958,7 +958,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             tm.mark();
             DTS_CUDA(cudaStreamSynchronize(s));
         } catch (...) {
-            cudaFreeAsync(fin, s);
+            cudaStreamSynchronize(s);
+            cache_free(fin);
             throw;
         }
         out->results = fin;
