@@ -142,20 +142,12 @@ __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
 }
 
-constexpr int GATHER_ITEMS = 4;   // rows in flight per thread
-
-__device__ __forceinline__ void gather_one(const double4& s0, const double4& s1, size_t p,
-                                           uint32_t i, GridParams g, SegSoA& soa,
-                                           unsigned long long* __restrict__ bin_t0min,
-                                           unsigned long long* __restrict__ bin_t1max, bool ok);
+constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
 
 // Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
 __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
-                                              const uint32_t* __restrict__ ids, GridParams g,
-                                              SegSoA soa,
-                                              unsigned long long* __restrict__ bin_t0min,
-                                              unsigned long long* __restrict__ bin_t1max) {
+                                              const uint32_t* __restrict__ ids, SegSoA soa) {
     const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
     uint32_t id[GATHER_ITEMS];
     double4 r0[GATHER_ITEMS], r1[GATHER_ITEMS];
@@ -175,44 +167,15 @@ __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, si
 #pragma unroll
     for (int k = 0; k < GATHER_ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
-        gather_one(r0[k], r1[k], p, id[k], g, soa, bin_t0min, bin_t1max, p < n);
-    }
-}
-
-__device__ __forceinline__ void gather_one(const double4& s0, const double4& s1, size_t p,
-                                           uint32_t i, GridParams g, SegSoA& soa,
-                                           unsigned long long* __restrict__ bin_t0min,
-                                           unsigned long long* __restrict__ bin_t1max, bool ok) {
-    int32_t bin = -1;
-    unsigned long long o0 = ~0ull, o1 = 0ull;
-    if (ok) {
-        double dur = s1.x - s0.x;
-        soa.st[p] = make_double2(s0.x, s1.x);
-        soa.sx[p] = make_double2(s0.y, velocity(s0.y, s1.y, dur));
-        soa.sy[p] = make_double2(s0.z, velocity(s0.z, s1.z, dur));
-        soa.sz[p] = make_double2(s0.w, velocity(s0.w, s1.w, dur));
-        soa.eid[p] = i;
-        bin = bin_of(g, s0.x);
-        o0 = ordered_bits(s0.x);
-        o1 = ordered_bits(s1.x);
-    }
-    // per-bin extents, warp-aggregated when the warp is inside one bin
-    const int lane = threadIdx.x & 31;
-    int32_t b0 = __shfl_sync(0xffffffffu, bin, 0);
-    if (__all_sync(0xffffffffu, bin == b0 || bin < 0)) {
-        for (int off = 16; off; off >>= 1) {
-            unsigned long long a = __shfl_xor_sync(0xffffffffu, o0, off);
-            unsigned long long c = __shfl_xor_sync(0xffffffffu, o1, off);
-            o0 = a < o0 ? a : o0;
-            o1 = c > o1 ? c : o1;
+        if (p < n) {
+            const double4 s0 = r0[k], s1 = r1[k];
+            const double dur = s1.x - s0.x;
+            soa.st[p] = make_double2(s0.x, s1.x);
+            soa.sx[p] = make_double2(s0.y, velocity(s0.y, s1.y, dur));
+            soa.sy[p] = make_double2(s0.z, velocity(s0.z, s1.z, dur));
+            soa.sz[p] = make_double2(s0.w, velocity(s0.w, s1.w, dur));
+            soa.eid[p] = id[k];
         }
-        if (lane == 0 && b0 >= 0) {
-            atomicMin(&bin_t0min[b0], o0);
-            atomicMax(&bin_t1max[b0], o1);
-        }
-    } else if (ok) {
-        atomicMin(&bin_t0min[bin], o0);
-        atomicMax(&bin_t1max[bin], o1);
     }
 }
 
@@ -229,23 +192,50 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
     }
 }
 
-// Counts non-empty cells and writes bin_start[0..m]: the entries of bin j are
-// the sorted positions [bin_start[j], bin_start[j+1]) (the index range
-// [B_first, B_last] of P:L76; keys are bin-major).
+// Counts non-empty cells, writes bin_start[0..m] (the entries of bin j are the
+// sorted positions [bin_start[j], bin_start[j+1]): the index range
+// [B_first, B_last] of P:L76, keys being bin-major) and the per-bin extent
+// [min t_start, max t_end] (B_start / B_end of P:L76) with warp-aggregated
+// atomics on order-preserving integer images of the times.
 __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __restrict__ keys,
                                                    size_t n, GridParams g,
+                                                   const double2* __restrict__ st,
                                                    uint32_t* __restrict__ bin_start,
+                                                   unsigned long long* __restrict__ bin_t0min,
+                                                   unsigned long long* __restrict__ bin_t1max,
                                                    unsigned long long* __restrict__ count) {
     size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
     int f = 0;
+    long long b = -1;
+    unsigned long long o0 = ~0ull, o1 = 0ull;
     if (p < n) {
         const unsigned long long k = keys[p];
         f = (p == 0 || k != keys[p - 1]);
-        const long long b = (long long)(k / g.cells_per_bin);
+        b = (long long)(k / g.cells_per_bin);
         const long long bp = p == 0 ? -1 : (long long)(keys[p - 1] / g.cells_per_bin);
         for (long long bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
         if (p == n - 1)
             for (long long bb = b + 1; bb <= g.m; ++bb) bin_start[bb] = (uint32_t)n;
+        const double2 t = st[p];
+        o0 = ordered_bits(t.x);
+        o1 = ordered_bits(t.y);
+    }
+    const int lane = threadIdx.x & 31;
+    const long long b0 = __shfl_sync(0xffffffffu, b, 0);
+    if (__all_sync(0xffffffffu, b == b0 || b < 0)) {
+        for (int off = 16; off; off >>= 1) {
+            const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
+            const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);
+            o0 = x < o0 ? x : o0;
+            o1 = y > o1 ? y : o1;
+        }
+        if (lane == 0 && b0 >= 0) {
+            atomicMin(&bin_t0min[b0], o0);
+            atomicMax(&bin_t1max[b0], o1);
+        }
+    } else if (b >= 0) {
+        atomicMin(&bin_t0min[b], o0);
+        atomicMax(&bin_t1max[b], o1);
     }
     int c = __syncthreads_count(f);
     if (threadIdx.x == 0 && c) atomicAdd(count, (unsigned long long)c);
@@ -357,7 +347,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     keys_tmp.release();
     ids_tmp.release();
 
-    // 5. gather into the SoA layout + bin extents
+    // 5. gather into the SoA layout
     const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
     const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
     char* blk = nullptr;
@@ -377,16 +367,17 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
-    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, ids.p, g,
-                                                                         idx->soa, b0, b1);
-    DTS_LAUNCH_CHECK();
-    k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
+    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, ids.p,
+                                                                         idx->soa);
     DTS_LAUNCH_CHECK();
 
     // 6. non-empty cells -> hash table
     DevBuf<unsigned long long> ncell(1, s);
     DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
-    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, g, idx->bin_start, ncell.p);
+    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, g, idx->soa.st, idx->bin_start, b0, b1,
+                                             ncell.p);
+    DTS_LAUNCH_CHECK();
+    k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
     unsigned long long hc = 0;
     DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));

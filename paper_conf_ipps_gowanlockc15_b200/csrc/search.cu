@@ -40,7 +40,6 @@ namespace {
 
 constexpr int TT = 256;                 // threads per tile CTA
 constexpr int TQ = 64;                  // queries per tile
-constexpr int LMAX = 1024;              // probes (runs) per chunk
 constexpr int HMAX = 1024;              // staged hits per tile
 constexpr int PT = 256;                 // threads per CTA in warp-per-query kernels
 constexpr int PW = PT / 32;
@@ -181,12 +180,17 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
         s.nlook = 1;
     } else {
         s.mode = MODE_GRID;
-        s.nlook = (uint32_t)ncomb;
+        s.nlook = (uint32_t)(s.hb - s.lb + 1) * (uint32_t)s.cn[1] * (uint32_t)s.cn[2];  // rows
     }
     return s;
 }
 
-// Resolve probe `loc` of a query's stencil into an entry run [start, start+cnt).
+// Resolve probe `loc` of a query's stencil into one entry run [start,
+// start+cnt).  A grid probe is a stencil ROW (bin, cz, cy) over the cells
+// cx in [clo0, clo0 + cn0): keys are row-major with x fastest, so the
+// non-empty cells of that x range are consecutive in the sorted order and
+// form one contiguous run from the first one's start to the last one's end.
+// Their hash slots share one or two 64-byte slot groups (slot_of).
 __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht,
                                         const double* __restrict__ bin_t0min,
                                         const double* __restrict__ bin_t1max,
@@ -201,27 +205,32 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
         cnt = __ldg(&bin_start[hb + 1]) - start;
         return;
     }
-    const uint32_t nyx = (uint32_t)cn[0] * (uint32_t)cn[1];
-    const uint32_t nzyx = nyx * (uint32_t)cn[2];
-    const int32_t bin = lb + (int32_t)(loc / nzyx);
-    uint32_t r = loc % nzyx;
-    const int32_t cz = clo[2] + (int32_t)(r / nyx);
-    r %= nyx;
-    const int32_t cy = clo[1] + (int32_t)(r / (uint32_t)cn[0]);
-    const int32_t cx = clo[0] + (int32_t)(r % (uint32_t)cn[0]);
+    const uint32_t nzy = (uint32_t)cn[1] * (uint32_t)cn[2];
+    const int32_t bin = lb + (int32_t)(loc / nzy);
+    const uint32_t r = loc % nzy;
+    const int32_t cz = clo[2] + (int32_t)(r / (uint32_t)cn[1]);
+    const int32_t cy = clo[1] + (int32_t)(r % (uint32_t)cn[1]);
     if (!(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0)) return;
-    const unsigned long long key = make_key(g, bin, cx, cy, cz);
-    unsigned long long h = slot_of(key, ht.log2cap);
-    ++probes;
-    while (true) {
-        const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(ht.slots) + h);
-        if (sl.x == key) {
-            start = (uint32_t)sl.y;
-            cnt = (uint32_t)(sl.y >> 32) - start;
-            return;
+    const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
+    uint32_t first = 0xffffffffu, last = 0;
+    for (int32_t i = 0; i < cn[0]; ++i) {
+        const unsigned long long key = key0 + (unsigned long long)i;
+        unsigned long long h = slot_of(key, ht.log2cap);
+        ++probes;
+        while (true) {
+            const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(ht.slots) + h);
+            if (sl.x == key) {
+                if (first == 0xffffffffu) first = (uint32_t)sl.y;
+                last = (uint32_t)(sl.y >> 32);
+                break;
+            }
+            if (sl.x == EMPTY_KEY) break;
+            h = (h + 1) & ht.mask;
         }
-        if (sl.x == EMPTY_KEY) return;
-        h = (h + 1) & ht.mask;
+    }
+    if (first != 0xffffffffu) {
+        start = first;
+        cnt = last - first;
     }
 }
 
@@ -256,47 +265,6 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
 }
 
 // ------------------------------------------------------------- block helpers
-// Exclusive scan of n <= 4*TT u64 values in shared memory (in place); writes
-// the total to a[n].  All TT threads must call it.
-__device__ void block_scan_u64(unsigned long long* a, int n) {
-    __shared__ unsigned long long warp_tot[TT / 32];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    unsigned long long v[4], s = 0;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        const int j = tid * 4 + k;
-        v[k] = j < n ? a[j] : 0ull;
-        s += v[k];
-    }
-    unsigned long long inc = s;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        unsigned long long u = __shfl_up_sync(0xffffffffu, inc, o);
-        if (lane >= o) inc += u;
-    }
-    if (lane == 31) warp_tot[warp] = inc;
-    __syncthreads();
-    if (warp == 0) {
-        unsigned long long w = lane < TT / 32 ? warp_tot[lane] : 0ull;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned long long u = __shfl_up_sync(0xffffffffu, w, o);
-            if (lane >= o) w += u;
-        }
-        if (lane < TT / 32) warp_tot[lane] = w;
-    }
-    __syncthreads();
-    unsigned long long run = (warp ? warp_tot[warp - 1] : 0ull) + inc - s;
-#pragma unroll
-    for (int k = 0; k < 4; ++k) {
-        const int j = tid * 4 + k;
-        if (j < n) a[j] = run;
-        run += v[k];
-    }
-    if (tid == TT - 1) a[n] = run;
-    __syncthreads();
-}
-
 // Exclusive scan of TQ (= 64) u64 values, threads 0..63 hold v; result in
 // out[0..TQ] (out[TQ] = total).  All threads must call it.
 __device__ __forceinline__ void tile_scan64(unsigned long long v, unsigned long long* out) {
@@ -347,9 +315,6 @@ struct TileSmem {
     int32_t lb[TQ], hb[TQ], clo[3][TQ], cn[3][TQ];
     uint32_t qid[TQ], mode[TQ], qcount[TQ];
     unsigned long long lkoff[TQ + 1];
-    uint32_t rstart[LMAX];
-    unsigned long long roff[LMAX + 1];
-    uint8_t rq[LMAX];
     unsigned long long hkey[HMAX];
     double h0[HMAX], h1[HMAX];
     unsigned long long base;
@@ -415,64 +380,77 @@ __global__ void __launch_bounds__(TT, 4) k_tile_count(const TileArgs a) {
     tile_scan64(nlook, S.lkoff);
     const unsigned long long Ltot = S.lkoff[TQ];
 
+    // ---- phases A+B, per warp, no block barriers: each warp takes 32 row
+    //      probes of the tile at a time (one per lane), a warp scan flattens
+    //      their runs, and lanes stream the candidates two at a time
+    //      (8 x 128-bit loads in flight per lane), locating their run with a
+    //      shuffle binary search over the lanes' inclusive prefix.
+    const int lane = tid & 31, warp = tid >> 5;
     unsigned long long n_cand = 0;
     uint32_t n_probe = 0;
-    for (unsigned long long l0 = 0; l0 < Ltot; l0 += LMAX) {
-        const int nl = (int)min((unsigned long long)LMAX, Ltot - l0);
-        // ---- phase A: probes -> runs
-        for (int j = tid; j < nl; j += TT) {
-            const unsigned long long l = l0 + j;
-            int qi = 0;
+    for (unsigned long long r0 = (unsigned long long)warp * 32; r0 < Ltot; r0 += TT) {
+        const unsigned long long l = r0 + lane;
+        uint32_t start = 0, cnt = 0;
+        int qi = 0;
+        if (l < Ltot) {
 #pragma unroll
             for (int step = 32; step; step >>= 1)
                 if (S.lkoff[qi + step] <= l) qi += step;
             const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
             const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
             const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
-            uint32_t start, cnt;
             resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
                     S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, start, cnt, n_probe);
-            S.rstart[j] = start;
-            S.roff[j] = cnt;
-            S.rq[j] = (uint8_t)qi;
         }
-        __syncthreads();
-        block_scan_u64(S.roff, nl);
-        const unsigned long long C = S.roff[nl];
-        n_cand += C;
-        // ---- phase B: stream the flattened candidates, two per thread in flight
-        for (unsigned long long c = tid; c < C; c += 2 * TT) {
-            const unsigned long long c2 = c + TT;
+        unsigned long long incl = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
+            if (lane >= o) incl += u;
+        }
+        const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
+        const unsigned long long excl = incl - cnt;
+        n_cand += total;
+        for (unsigned long long base = 0; base < total; base += 64) {
+            const unsigned long long t1 = base + lane, t2 = t1 + 32;
             int j1 = 0, j2 = 0;
 #pragma unroll
-            for (int step = LMAX / 2; step; step >>= 1) {
-                if (j1 + step < nl && S.roff[j1 + step] <= c) j1 += step;
-                if (j2 + step < nl && S.roff[j2 + step] <= c2) j2 += step;
+            for (int step = 16; step; step >>= 1) {
+                if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
+                if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
             }
-            const bool v2 = c2 < C;
-            const uint32_t p1 = S.rstart[j1] + (uint32_t)(c - S.roff[j1]);
-            const uint32_t p2 = v2 ? S.rstart[j2] + (uint32_t)(c2 - S.roff[j2]) : p1;
-            const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
-            const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
-            const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
-            const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
-            const int qi1 = S.rq[j1], qi2 = S.rq[j2];
-            double r0, r1;
-            if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, r0, r1))
-                stage_hit(S, qi1, p1, r0, r1, a.soa.eid);
-            if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, r0, r1))
-                stage_hit(S, qi2, p2, r0, r1, a.soa.eid);
+            const uint32_t s1 = __shfl_sync(0xffffffffu, start, j1);
+            const uint32_t s2 = __shfl_sync(0xffffffffu, start, j2);
+            const unsigned long long e1 = __shfl_sync(0xffffffffu, excl, j1);
+            const unsigned long long e2 = __shfl_sync(0xffffffffu, excl, j2);
+            const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
+            const int qi2 = __shfl_sync(0xffffffffu, qi, j2);
+            const bool v1 = t1 < total, v2 = t2 < total;
+            const uint32_t p1 = v1 ? s1 + (uint32_t)(t1 - e1) : 0u;
+            const uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
+            if (v1) {
+                const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
+                const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
+                const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
+                const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
+                double h0, h1;
+                if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
+                    stage_hit(S, qi1, p1, h0, h1, a.soa.eid);
+                if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
+                    stage_hit(S, qi2, p2, h0, h1, a.soa.eid);
+            }
         }
-        __syncthreads();
     }
+    if (lane != 0) n_cand = 0;
+    __syncthreads();
 
     // ---- statistics
     {
         unsigned long long pr = n_probe;
 #pragma unroll
         for (int o = 16; o; o >>= 1) pr += __shfl_xor_sync(0xffffffffu, pr, o);
-        if ((tid & 31) == 0 && pr) atomicAdd(&a.ctr->lookups, pr);
-        if (tid == 0 && n_cand) atomicAdd(&a.ctr->candidates, n_cand);
+        if (lane == 0 && pr) atomicAdd(&a.ctr->lookups, pr);
+        if (lane == 0 && n_cand) atomicAdd(&a.ctr->candidates, n_cand);
     }
     // ---- per-query counts
     if (tid < TQ && tile * TQ + tid < a.nq) {
