@@ -221,8 +221,29 @@ __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __
         o1 = ordered_bits(t.y);
     }
     const int lane = threadIdx.x & 31;
-    const long long b0 = __shfl_sync(0xffffffffu, b, 0);
-    if (__all_sync(0xffffffffu, b == b0 || b < 0)) {
+    // one atomic pair per CTA when the CTA's 256 sorted positions share a bin
+    // (the common case: bins hold ~10^5 entries), else per warp / per thread
+    const long long bfirst = (long long)(keys[(size_t)blockIdx.x * BT] / g.cells_per_bin);
+    if (__syncthreads_and(b == bfirst || b < 0)) {
+        __shared__ unsigned long long r0[BT / 32], r1[BT / 32];
+        for (int off = 16; off; off >>= 1) {
+            const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
+            const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);
+            o0 = x < o0 ? x : o0;
+            o1 = y > o1 ? y : o1;
+        }
+        if (lane == 0) { r0[threadIdx.x >> 5] = o0; r1[threadIdx.x >> 5] = o1; }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int w = 1; w < BT / 32; ++w) {
+                o0 = r0[w] < o0 ? r0[w] : o0;
+                o1 = r1[w] > o1 ? r1[w] : o1;
+            }
+            atomicMin(&bin_t0min[bfirst], o0);
+            atomicMax(&bin_t1max[bfirst], o1);
+        }
+    } else if (const long long b0 = __shfl_sync(0xffffffffu, b, 0);
+               __all_sync(0xffffffffu, b == b0 || b < 0)) {
         for (int off = 16; off; off >>= 1) {
             const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
             const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);

@@ -31,6 +31,7 @@
 //     recomputed in pass 2 (warp per query, ballot-ranked writes at the exact
 //     offsets) and then sorted per query -- the count-then-scatter fallback.
 #include <algorithm>
+#include <cstdlib>
 #include <vector>
 
 #include "internal.cuh"
@@ -154,7 +155,9 @@ __device__ __forceinline__ bool load_query(const double4* __restrict__ Q, uint32
 __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QState& q,
                                                 const double qlo[3], const double qhi[3],
                                                 double d, bool live,
-                                                const uint32_t* __restrict__ bin_start) {
+                                                const uint32_t* __restrict__ bin_start,
+                                                const double* __restrict__ bin_t0min,
+                                                const double* __restrict__ bin_t1max) {
     Stencil s;
     s.mode = MODE_DEAD;
     s.nlook = 0;
@@ -164,6 +167,18 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
     const double mt = 1e-12 * (fabs(q.t0) + g.maxdur);
     s.lb = bin_of(g, q.t0 - g.maxdur - mt);
     s.hb = bin_of(g, q.t1);
+    // drop end bins whose extent [min t_start, max t_end] (B_start, B_end of
+    // P:L76) does not overlap the query strictly: exact comparisons, so no
+    // candidate is lost (on synchronised timesteps this removes the previous
+    // step's bin, whose segments only touch the query at q.t0)
+    while (s.lb <= s.hb &&
+           !(__ldg(&bin_t0min[s.lb]) < q.t1 && __ldg(&bin_t1max[s.lb]) > q.t0)) ++s.lb;
+    while (s.hb >= s.lb &&
+           !(__ldg(&bin_t0min[s.hb]) < q.t1 && __ldg(&bin_t1max[s.hb]) > q.t0)) --s.hb;
+    if (s.lb > s.hb) {
+        s.lb = s.hb = 0;
+        return s;
+    }
     double ncomb = (double)(s.hb - s.lb + 1);
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
@@ -212,20 +227,32 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     const int32_t cy = clo[1] + (int32_t)(r % (uint32_t)cn[1]);
     if (!(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0)) return;
     const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
+    const ulonglong2* slots = reinterpret_cast<const ulonglong2*>(ht.slots);
     uint32_t first = 0xffffffffu, last = 0;
-    for (int32_t i = 0; i < cn[0]; ++i) {
-        const unsigned long long key = key0 + (unsigned long long)i;
-        unsigned long long h = slot_of(key, ht.log2cap);
-        ++probes;
-        while (true) {
-            const ulonglong2 sl = __ldg(reinterpret_cast<const ulonglong2*>(ht.slots) + h);
-            if (sl.x == key) {
-                if (first == 0xffffffffu) first = (uint32_t)sl.y;
-                last = (uint32_t)(sl.y >> 32);
-                break;
+    constexpr int W = 4;   // home slots of up to W cells issued together
+    for (int32_t i0 = 0; i0 < cn[0]; i0 += W) {
+        ulonglong2 sl[W];
+        unsigned long long hh[W];
+#pragma unroll
+        for (int i = 0; i < W; ++i) {
+            hh[i] = slot_of(key0 + (unsigned long long)(i0 + i), ht.log2cap);
+            if (i0 + i < cn[0]) sl[i] = __ldg(slots + hh[i]);
+        }
+#pragma unroll
+        for (int i = 0; i < W; ++i) {
+            if (i0 + i >= cn[0]) break;
+            const unsigned long long key = key0 + (unsigned long long)(i0 + i);
+            ++probes;
+            ulonglong2 s = sl[i];
+            unsigned long long h = hh[i];
+            while (s.x != key && s.x != EMPTY_KEY) {     // collision: linear probing
+                h = (h + 1) & ht.mask;
+                s = __ldg(slots + h);
             }
-            if (sl.x == EMPTY_KEY) break;
-            h = (h + 1) & ht.mask;
+            if (s.x == key) {
+                if (first == 0xffffffffu) first = (uint32_t)s.y;
+                last = (uint32_t)(s.y >> 32);
+            }
         }
     }
     if (first != 0xffffffffu) {
@@ -344,7 +371,8 @@ __device__ __forceinline__ void stage_hit(TileSmem& S, int qi, uint32_t p, doubl
     }
 }
 
-__global__ void __launch_bounds__(TT, 4) k_tile_count(const TileArgs a) {
+template <int MINB>
+__global__ void __launch_bounds__(TT, MINB) k_tile_count(const TileArgs a) {
     __shared__ TileSmem S;
     const int tid = threadIdx.x;
     const uint32_t tile = blockIdx.x;
@@ -363,7 +391,8 @@ __global__ void __launch_bounds__(TT, 4) k_tile_count(const TileArgs a) {
             qid = a.order[sp];
             live = load_query(a.Q, qid, q, qlo, qhi);
         }
-        const Stencil st = make_stencil(g, q, qlo, qhi, d, live, a.bin_start);
+        const Stencil st =
+            make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
         S.qt0[tid] = q.t0; S.qt1[tid] = q.t1;
         S.qx0[tid] = q.x0; S.qvx[tid] = q.vx;
         S.qy0[tid] = q.y0; S.qvy[tid] = q.vy;
@@ -585,7 +614,8 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
     QState q;
     double qlo[3], qhi[3];
     const bool live = load_query(a.Q, qid, q, qlo, qhi);
-    const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start);
+    const Stencil st =
+        make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
     const double d2 = a.d * a.d;
     unsigned long long out_pos = a.offsets[qid];
     uint32_t dummy = 0;
@@ -845,7 +875,14 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.large = large.p;
     ta.qid_base = qid_base;
     ta.ctr = ctr.p;
-    k_tile_count<<<ntiles, TT, 0, s>>>(ta);
+    // CTAs per SM the tile kernel is register-bounded for (tuning knob,
+    // DTS_TILE_OCC=3|4; 4 = 64 registers, 3 = 85 registers)
+    static const int occ = [] {
+        const char* e = getenv("DTS_TILE_OCC");
+        return (e && atoi(e) == 3) ? 3 : 4;
+    }();
+    if (occ == 3) k_tile_count<3><<<ntiles, TT, 0, s>>>(ta);
+    else k_tile_count<4><<<ntiles, TT, 0, s>>>(ta);
     DTS_LAUNCH_CHECK();
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
