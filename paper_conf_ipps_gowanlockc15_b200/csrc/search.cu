@@ -39,9 +39,7 @@
 namespace dts {
 namespace {
 
-constexpr int TT = 256;                 // threads per tile CTA
-constexpr int TQ = 64;                  // queries per tile
-constexpr int HMAX = 1024;              // staged hits per tile
+constexpr int TQ = 16;                  // queries per warp tile (WQ of wtile.cuh)
 constexpr int PT = 256;                 // threads per CTA in warp-per-query kernels
 constexpr int PW = PT / 32;
 constexpr int SMALL_SORT = 32;          // warp-register sort limit
@@ -58,6 +56,8 @@ struct Counters {                       // device-side statistics / flags
     unsigned int n_large;
     unsigned int n_over;                // tiles recomputed in pass 2
     unsigned int bad;
+    unsigned int work;                  // dynamic warp-tile counter
+    unsigned int pad;
 };
 
 // Query in the velocity form used by the refinement.
@@ -232,22 +232,22 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     constexpr int W = 4;   // home slots of up to W cells issued together
     for (int32_t i0 = 0; i0 < cn[0]; i0 += W) {
         ulonglong2 sl[W];
-        unsigned long long hh[W];
 #pragma unroll
-        for (int i = 0; i < W; ++i) {
-            hh[i] = slot_of(key0 + (unsigned long long)(i0 + i), ht.log2cap);
-            if (i0 + i < cn[0]) sl[i] = __ldg(slots + hh[i]);
-        }
+        for (int i = 0; i < W; ++i)
+            if (i0 + i < cn[0]) sl[i] = __ldg(slots + slot_of(key0 + (unsigned long long)(i0 + i),
+                                                              ht.log2cap));
 #pragma unroll
         for (int i = 0; i < W; ++i) {
             if (i0 + i >= cn[0]) break;
             const unsigned long long key = key0 + (unsigned long long)(i0 + i);
             ++probes;
             ulonglong2 s = sl[i];
-            unsigned long long h = hh[i];
-            while (s.x != key && s.x != EMPTY_KEY) {     // collision: linear probing
-                h = (h + 1) & ht.mask;
-                s = __ldg(slots + h);
+            if (s.x != key && s.x != EMPTY_KEY) {       // collision: linear probing
+                unsigned long long h = slot_of(key, ht.log2cap);
+                do {
+                    h = (h + 1) & ht.mask;
+                    s = __ldg(slots + h);
+                } while (s.x != key && s.x != EMPTY_KEY);
             }
             if (s.x == key) {
                 if (first == 0xffffffffu) first = (uint32_t)s.y;
@@ -292,293 +292,7 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
 }
 
 // ------------------------------------------------------------- block helpers
-// Exclusive scan of TQ (= 64) u64 values, threads 0..63 hold v; result in
-// out[0..TQ] (out[TQ] = total).  All threads must call it.
-__device__ __forceinline__ void tile_scan64(unsigned long long v, unsigned long long* out) {
-    __shared__ unsigned long long w0;
-    const int tid = threadIdx.x, lane = tid & 31;
-    unsigned long long inc = v;
-    if (tid < TQ) {
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned long long u = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane >= o) inc += u;
-        }
-        if (tid == 31) w0 = inc;
-    }
-    __syncthreads();
-    if (tid < TQ) {
-        if (tid >= 32) inc += w0;
-        out[tid + 1] = inc;
-        if (tid == 0) out[0] = 0ull;
-    }
-    __syncthreads();
-}
-
-// ------------------------------------------------------- pass 1: tile count
-struct TileArgs {
-    const double4* Q;
-    const uint32_t* order;         // sorted position -> query id
-    uint32_t nq;
-    double d;
-    GridParams g;
-    SegSoA soa;
-    HashTable ht;
-    const double* bin_t0min;
-    const double* bin_t1max;
-    const uint32_t* bin_start;
-    uint32_t* counts;              // per query id
-    dts_result* stage;             // staged hits (tile-contiguous, canonical inside)
-    unsigned long long stage_cap;
-    unsigned long long* tile_base; // per tile: first staged slot or NONE
-    uint32_t* over_tiles;          // tiles to recompute in pass 2
-    uint32_t* large;               // query ids (recomputed tiles) with count > SMALL_SORT
-    uint32_t qid_base;
-    Counters* ctr;
-};
-
-struct TileSmem {
-    double qt0[TQ], qt1[TQ], qx0[TQ], qvx[TQ], qy0[TQ], qvy[TQ], qz0[TQ], qvz[TQ];
-    int32_t lb[TQ], hb[TQ], clo[3][TQ], cn[3][TQ];
-    uint32_t qid[TQ], mode[TQ], qcount[TQ];
-    unsigned long long lkoff[TQ + 1];
-    unsigned long long hkey[HMAX];
-    double h0[HMAX], h1[HMAX];
-    unsigned long long base;
-    uint32_t nhit, over;
-};
-
-__device__ __forceinline__ QState smem_query(const TileSmem& S, int qi) {
-    QState q;
-    q.t0 = S.qt0[qi]; q.t1 = S.qt1[qi];
-    q.x0 = S.qx0[qi]; q.vx = S.qvx[qi];
-    q.y0 = S.qy0[qi]; q.vy = S.qvy[qi];
-    q.z0 = S.qz0[qi]; q.vz = S.qvz[qi];
-    return q;
-}
-
-__device__ __forceinline__ void stage_hit(TileSmem& S, int qi, uint32_t p, double r0, double r1,
-                                          const uint32_t* __restrict__ eid) {
-    atomicAdd(&S.qcount[qi], 1u);
-    const uint32_t pos = atomicAdd(&S.nhit, 1u);
-    if (pos < (uint32_t)HMAX) {
-        const uint32_t e = __ldg(eid + p);
-        S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)e << 10) | pos;
-        S.h0[pos] = r0;
-        S.h1[pos] = r1;
-    } else {
-        S.over = 1u;
-    }
-}
-
-template <int MINB>
-__global__ void __launch_bounds__(TT, MINB) k_tile_count(const TileArgs a) {
-    __shared__ TileSmem S;
-    const int tid = threadIdx.x;
-    const uint32_t tile = blockIdx.x;
-    const GridParams& g = a.g;
-    const double d = a.d, d2 = d * d;
-
-    // ---- phase 0: the tile's queries, stencils and probe counts
-    unsigned long long nlook = 0;
-    if (tid < TQ) {
-        const uint32_t sp = tile * TQ + tid;
-        QState q{};
-        double qlo[3] = {0, 0, 0}, qhi[3] = {0, 0, 0};
-        bool live = false;
-        uint32_t qid = 0;
-        if (sp < a.nq) {
-            qid = a.order[sp];
-            live = load_query(a.Q, qid, q, qlo, qhi);
-        }
-        const Stencil st =
-            make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
-        S.qt0[tid] = q.t0; S.qt1[tid] = q.t1;
-        S.qx0[tid] = q.x0; S.qvx[tid] = q.vx;
-        S.qy0[tid] = q.y0; S.qvy[tid] = q.vy;
-        S.qz0[tid] = q.z0; S.qvz[tid] = q.vz;
-        S.lb[tid] = st.lb; S.hb[tid] = st.hb;
-#pragma unroll
-        for (int ax = 0; ax < 3; ++ax) { S.clo[ax][tid] = st.clo[ax]; S.cn[ax][tid] = st.cn[ax]; }
-        S.qid[tid] = qid;
-        S.mode[tid] = st.mode;
-        S.qcount[tid] = 0;
-        nlook = st.nlook;
-    }
-    if (tid == 0) { S.nhit = 0; S.over = 0; }
-    tile_scan64(nlook, S.lkoff);
-    const unsigned long long Ltot = S.lkoff[TQ];
-
-    // ---- phases A+B, per warp, no block barriers: each warp takes 32 row
-    //      probes of the tile at a time (one per lane), a warp scan flattens
-    //      their runs, and lanes stream the candidates two at a time
-    //      (8 x 128-bit loads in flight per lane), locating their run with a
-    //      shuffle binary search over the lanes' inclusive prefix.
-    const int lane = tid & 31, warp = tid >> 5;
-    unsigned long long n_cand = 0;
-    uint32_t n_probe = 0;
-    for (unsigned long long r0 = (unsigned long long)warp * 32; r0 < Ltot; r0 += TT) {
-        const unsigned long long l = r0 + lane;
-        uint32_t start = 0, cnt = 0;
-        int qi = 0;
-        if (l < Ltot) {
-#pragma unroll
-            for (int step = 32; step; step >>= 1)
-                if (S.lkoff[qi + step] <= l) qi += step;
-            const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
-            const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
-            const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
-            resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
-                    S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, start, cnt, n_probe);
-        }
-        unsigned long long incl = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += u;
-        }
-        const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
-        const unsigned long long excl = incl - cnt;
-        n_cand += total;
-        for (unsigned long long base = 0; base < total; base += 64) {
-            const unsigned long long t1 = base + lane, t2 = t1 + 32;
-            int j1 = 0, j2 = 0;
-#pragma unroll
-            for (int step = 16; step; step >>= 1) {
-                if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
-                if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
-            }
-            const uint32_t s1 = __shfl_sync(0xffffffffu, start, j1);
-            const uint32_t s2 = __shfl_sync(0xffffffffu, start, j2);
-            const unsigned long long e1 = __shfl_sync(0xffffffffu, excl, j1);
-            const unsigned long long e2 = __shfl_sync(0xffffffffu, excl, j2);
-            const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
-            const int qi2 = __shfl_sync(0xffffffffu, qi, j2);
-            const bool v1 = t1 < total, v2 = t2 < total;
-            const uint32_t p1 = v1 ? s1 + (uint32_t)(t1 - e1) : 0u;
-            const uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
-            if (v1) {
-                const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
-                const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
-                const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
-                const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
-                double h0, h1;
-                if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
-                    stage_hit(S, qi1, p1, h0, h1, a.soa.eid);
-                if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
-                    stage_hit(S, qi2, p2, h0, h1, a.soa.eid);
-            }
-        }
-    }
-    if (lane != 0) n_cand = 0;
-    __syncthreads();
-
-    // ---- statistics
-    {
-        unsigned long long pr = n_probe;
-#pragma unroll
-        for (int o = 16; o; o >>= 1) pr += __shfl_xor_sync(0xffffffffu, pr, o);
-        if (lane == 0 && pr) atomicAdd(&a.ctr->lookups, pr);
-        if (lane == 0 && n_cand) atomicAdd(&a.ctr->candidates, n_cand);
-    }
-    // ---- per-query counts
-    if (tid < TQ && tile * TQ + tid < a.nq) {
-        const uint32_t cnt = S.qcount[tid];
-        a.counts[S.qid[tid]] = cnt;
-        if (cnt) atomicMax(&a.ctr->max_count, cnt);
-    }
-    // ---- stage the tile's hits in canonical order
-    const uint32_t nh = S.nhit;
-    if (!S.over && nh > 0) {
-        uint32_t P = 2;
-        while (P < nh) P <<= 1;
-        for (uint32_t j = nh + tid; j < P; j += TT) S.hkey[j] = ~0ull;
-        __syncthreads();
-        for (uint32_t k = 2; k <= P; k <<= 1) {
-            for (uint32_t jj = k >> 1; jj > 0; jj >>= 1) {
-                for (uint32_t t = tid; t < P; t += TT) {
-                    const uint32_t u = t ^ jj;
-                    if (u > t) {
-                        const unsigned long long x = S.hkey[t], y = S.hkey[u];
-                        if ((x > y) == ((t & k) == 0)) {
-                            S.hkey[t] = y;
-                            S.hkey[u] = x;
-                        }
-                    }
-                }
-                __syncthreads();
-            }
-        }
-        if (tid == 0) {
-            const unsigned long long b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
-            if (b + nh > a.stage_cap) S.over = 1u;
-            else S.base = b;
-        }
-        __syncthreads();
-        if (!S.over) {
-            const unsigned long long base = S.base;
-            for (uint32_t i = tid; i < nh; i += TT) {
-                const unsigned long long k = S.hkey[i];
-                const uint32_t slot = (uint32_t)(k & 1023ull);
-                dts_result r;
-                r.query_id = S.qid[(uint32_t)(k >> 42)] + a.qid_base;
-                r.entry_id = (uint32_t)(k >> 10);
-                r.t_start = S.h0[slot];
-                r.t_end = S.h1[slot];
-                a.stage[base + i] = r;
-            }
-            if (tid == 0) a.tile_base[tile] = base;
-        }
-    } else if (!S.over && tid == 0) {
-        a.tile_base[tile] = NONE - 1;        // no hits: nothing to emit
-    }
-    __syncthreads();
-    if (S.over) {
-        if (tid == 0) {
-            a.tile_base[tile] = NONE;
-            const uint32_t slot = atomicAdd(&a.ctr->n_over, 1u);
-            a.over_tiles[slot] = tile;
-        }
-        if (tid < TQ && tile * TQ + tid < a.nq && S.qcount[tid] > (uint32_t)SMALL_SORT) {
-            const uint32_t slot = atomicAdd(&a.ctr->n_large, 1u);
-            a.large[slot] = S.qid[tid];
-        }
-    }
-}
-
-// ------------------------------------------------------ pass 2: emission
-__global__ void __launch_bounds__(TT) k_tile_emit(const uint32_t* __restrict__ order, uint32_t nq,
-                                                 const uint32_t* __restrict__ counts,
-                                                 const unsigned long long* __restrict__ offsets,
-                                                 const unsigned long long* __restrict__ tile_base,
-                                                 const dts_result* __restrict__ stage,
-                                                 dts_result* __restrict__ out) {
-    __shared__ unsigned long long qpre[TQ + 1];
-    __shared__ uint32_t qid_s[TQ];
-    const uint32_t tile = blockIdx.x;
-    const unsigned long long tb = tile_base[tile];
-    if (tb >= NONE - 1) return;                      // recomputed or empty tile
-    const int tid = threadIdx.x;
-    unsigned long long cnt = 0;
-    if (tid < TQ) {
-        const uint32_t sp = tile * TQ + tid;
-        uint32_t qid = 0;
-        if (sp < nq) {
-            qid = order[sp];
-            cnt = counts[qid];
-        }
-        qid_s[tid] = qid;
-    }
-    tile_scan64(cnt, qpre);
-    const unsigned long long nh = qpre[TQ];
-    for (unsigned long long i = tid; i < nh; i += TT) {
-        int qi = 0;
-#pragma unroll
-        for (int step = 32; step; step >>= 1)
-            if (qpre[qi + step] <= i) qi += step;
-        out[offsets[qid_s[qi]] + (i - qpre[qi])] = stage[tb + i];
-    }
-}
+#include "wtile.cuh"
 
 // -------------------------------- fallback: warp-per-query scatter (pass 2)
 struct PassArgs {
@@ -850,8 +564,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     }
     tm.mark();
 
-    // ---- pass 1: tile count + staging
-    const uint32_t ntiles = (uint32_t)((nq + TQ - 1) / TQ);
+    // ---- pass 1: warp tiles, count + staging
+    const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
     const unsigned long long stage_cap = 4ull * nq + (1ull << 20);
     DevBuf<uint32_t> counts(nq, s), large(nq, s), over_tiles(ntiles, s);
     DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s);
@@ -875,15 +589,22 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.large = large.p;
     ta.qid_base = qid_base;
     ta.ctr = ctr.p;
-    // CTAs per SM the tile kernel is register-bounded for (tuning knob,
-    // DTS_TILE_OCC=3|4; 4 = 64 registers, 3 = 85 registers)
-    static const int occ = [] {
-        const char* e = getenv("DTS_TILE_OCC");
-        return (e && atoi(e) == 3) ? 3 : 4;
-    }();
-    if (occ == 3) k_tile_count<3><<<ntiles, TT, 0, s>>>(ta);
-    else k_tile_count<4><<<ntiles, TT, 0, s>>>(ta);
-    DTS_LAUNCH_CHECK();
+    {
+        int dev = 0, nsm = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+        const unsigned want = (ntiles + WW - 1) / WW;
+        // CTAs per SM the kernel is register-bounded for (tuning knob
+        // DTS_TILE_OCC = 6 | 8: 85 or 64 registers per thread)
+        static const int occ = [] {
+            const char* e = getenv("DTS_TILE_OCC");
+            return (e && atoi(e) == 8) ? 8 : 6;
+        }();
+        const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
+        if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
+        else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);
+        DTS_LAUNCH_CHECK();
+    }
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
     tm.mark();
@@ -909,8 +630,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         fin = static_cast<dts_result*>(cache_alloc(h.total * sizeof(dts_result)));
         try {
             // ---- pass 2: staged tiles are copied to their exact offsets
-            k_tile_emit<<<ntiles, TT, 0, s>>>(order.p, (uint32_t)nq, counts.p, offsets.p,
-                                              tile_base.p, stage.p, fin);
+            k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
+                                                             offsets.p, tile_base.p, stage.p,
+                                                             fin);
             DTS_LAUNCH_CHECK();
             // ---- overflowed tiles: recompute with exact offsets, then sort
             if (h.c.n_over) {

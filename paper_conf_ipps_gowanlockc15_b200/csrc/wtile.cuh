@@ -1,0 +1,296 @@
+// wtile.cuh -- pass 1 (fused candidate streaming + fp64 refinement, count +
+// staging) and pass 2 (emission) of the search, on warp-private query tiles.
+// Included by search.cu inside its anonymous namespace (uses its helpers).
+//
+// A warp owns a tile of WQ consecutive sorted queries and works on it alone
+// (no CTA barrier): warps fetch tiles dynamically, so a warp whose queries
+// sit in a dense region does not hold up others.  Per tile:
+//   0. lanes 0..WQ-1 load one query each: velocity form, stencil, row-probe
+//      count; a shuffle scan gives the tile's probe offsets;
+//   1. rounds of 32 row probes (one per lane) -> runs; a shuffle scan flattens
+//      them; lanes stream the candidates two at a time and refine them;
+//      hits go to the warp's shared-memory stage (query, entry id, interval);
+//   2. per-query counts are written; each staged hit's rank inside its query
+//      is counted against the other staged hits (ordering by entry id), and
+//      the tile's hits are written to the global stage in canonical order.
+// A tile whose hits exceed WH (or the global stage) is marked for the
+// count-then-scatter fallback of pass 2.
+
+constexpr int WQ = 16;                  // queries per warp tile
+constexpr int WH = 128;                 // staged hits per warp tile
+constexpr int WT = 128;                 // threads per CTA (4 independent warps)
+constexpr int WW = WT / 32;
+
+struct WarpSmem {
+    double qt0[WQ], qt1[WQ], qx0[WQ], qvx[WQ], qy0[WQ], qvy[WQ], qz0[WQ], qvz[WQ];
+    int32_t lb[WQ], hb[WQ], clo[3][WQ], cn[3][WQ];
+    uint32_t qid[WQ], mode[WQ], qcount[WQ], qoff[WQ];
+    unsigned long long lkoff[WQ + 1];
+    unsigned long long hkey[WH];        // (query << 42) | (entry id << 10) | slot
+    double h0[WH], h1[WH];
+    uint32_t nhit, over;
+};
+
+struct TileArgs {
+    const double4* Q;
+    const uint32_t* order;             // sorted position -> query id
+    uint32_t nq;
+    double d;
+    GridParams g;
+    SegSoA soa;
+    HashTable ht;
+    const double* bin_t0min;
+    const double* bin_t1max;
+    const uint32_t* bin_start;
+    uint32_t* counts;                  // per query id
+    dts_result* stage;                 // staged hits (tile-contiguous, canonical inside)
+    unsigned long long stage_cap;
+    unsigned long long* tile_base;     // per warp tile: first staged slot, NONE-1 empty, NONE redo
+    uint32_t* over_tiles;              // tiles to recompute in pass 2
+    uint32_t* large;                   // query ids (recomputed tiles) with count > SMALL_SORT
+    uint32_t qid_base;
+    Counters* ctr;
+};
+
+__device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
+    QState q;
+    q.t0 = S.qt0[qi]; q.t1 = S.qt1[qi];
+    q.x0 = S.qx0[qi]; q.vx = S.qvx[qi];
+    q.y0 = S.qy0[qi]; q.vy = S.qvy[qi];
+    q.z0 = S.qz0[qi]; q.vz = S.qvz[qi];
+    return q;
+}
+
+__device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, double r0, double r1,
+                                          const uint32_t* __restrict__ eid) {
+    atomicAdd(&S.qcount[qi], 1u);
+    const uint32_t pos = atomicAdd(&S.nhit, 1u);
+    if (pos < (uint32_t)WH) {
+        const uint32_t e = __ldg(eid + p);
+        S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)e << 10) | pos;
+        S.h0[pos] = r0;
+        S.h1[pos] = r1;
+    } else {
+        S.over = 1u;
+    }
+}
+
+template <int MINB>
+__global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
+    __shared__ WarpSmem SW[WW];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    WarpSmem& S = SW[warp];
+    const GridParams& g = a.g;
+    const double d = a.d, d2 = d * d;
+    const uint32_t ntiles = (a.nq + WQ - 1) / WQ;
+    unsigned long long n_cand = 0;
+    uint32_t n_probe = 0;
+
+    while (true) {
+        uint32_t wt = 0;
+        if (lane == 0) wt = atomicAdd(&a.ctr->work, 1u);
+        wt = __shfl_sync(0xffffffffu, wt, 0);
+        if (wt >= ntiles) break;
+
+        // ---- 0: queries, stencils, probe offsets
+        unsigned long long nlook = 0;
+        const uint32_t sp = wt * WQ + lane;
+        if (lane < WQ) {
+            QState q{};
+            double qlo[3] = {0, 0, 0}, qhi[3] = {0, 0, 0};
+            bool live = false;
+            uint32_t qid = 0;
+            if (sp < a.nq) {
+                qid = a.order[sp];
+                live = load_query(a.Q, qid, q, qlo, qhi);
+            }
+            const Stencil st =
+                make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
+            S.qt0[lane] = q.t0; S.qt1[lane] = q.t1;
+            S.qx0[lane] = q.x0; S.qvx[lane] = q.vx;
+            S.qy0[lane] = q.y0; S.qvy[lane] = q.vy;
+            S.qz0[lane] = q.z0; S.qvz[lane] = q.vz;
+            S.lb[lane] = st.lb; S.hb[lane] = st.hb;
+#pragma unroll
+            for (int ax = 0; ax < 3; ++ax) { S.clo[ax][lane] = st.clo[ax]; S.cn[ax][lane] = st.cn[ax]; }
+            S.qid[lane] = qid;
+            S.mode[lane] = st.mode;
+            S.qcount[lane] = 0;
+            nlook = st.nlook;
+        }
+        if (lane == 0) { S.nhit = 0; S.over = 0; S.lkoff[0] = 0; }
+        {
+            unsigned long long inc = nlook;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long u = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane >= o) inc += u;
+            }
+            if (lane < WQ) S.lkoff[lane + 1] = inc;
+        }
+        __syncwarp();
+        const unsigned long long Ltot = S.lkoff[WQ];
+
+        // ---- 1: rounds of 32 row probes, flattened, candidates two per lane
+        for (unsigned long long r0 = 0; r0 < Ltot; r0 += 32) {
+            const unsigned long long l = r0 + lane;
+            uint32_t start = 0, cnt = 0;
+            int qi = 0;
+            if (l < Ltot) {
+#pragma unroll
+                for (int step = WQ / 2; step; step >>= 1)
+                    if (S.lkoff[qi + step] <= l) qi += step;
+                const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
+                const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
+                const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
+                resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
+                        S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, start, cnt, n_probe);
+            }
+            unsigned long long incl = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
+                if (lane >= o) incl += u;
+            }
+            const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
+            const unsigned long long excl = incl - cnt;
+            n_cand += total;
+            for (unsigned long long base = 0; base < total; base += 64) {
+                const unsigned long long t1 = base + lane, t2 = t1 + 32;
+                int j1 = 0, j2 = 0;
+#pragma unroll
+                for (int step = 16; step; step >>= 1) {
+                    if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
+                    if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
+                }
+                const uint32_t s1 = __shfl_sync(0xffffffffu, start, j1);
+                const uint32_t s2 = __shfl_sync(0xffffffffu, start, j2);
+                const unsigned long long e1 = __shfl_sync(0xffffffffu, excl, j1);
+                const unsigned long long e2 = __shfl_sync(0xffffffffu, excl, j2);
+                const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
+                const int qi2 = __shfl_sync(0xffffffffu, qi, j2);
+                const bool v1 = t1 < total, v2 = t2 < total;
+                if (v1) {
+                    const uint32_t p1 = s1 + (uint32_t)(t1 - e1);
+                    const uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
+                    const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
+                    const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
+                    const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
+                    const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
+                    double h0, h1;
+                    if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
+                        stage_hit(S, qi1, p1, h0, h1, a.soa.eid);
+                    if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
+                        stage_hit(S, qi2, p2, h0, h1, a.soa.eid);
+                }
+            }
+        }
+        __syncwarp();
+
+        // ---- 2: counts, canonical staging
+        const uint32_t nh = S.nhit;
+        const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
+        if (lane < WQ && sp < a.nq) {
+            a.counts[S.qid[lane]] = cnt;
+            if (cnt) atomicMax(&a.ctr->max_count, cnt);
+        }
+        bool over = S.over != 0u;
+        if (!over && nh > 0) {
+            uint32_t inc = cnt;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane >= o) inc += u;
+            }
+            if (lane < WQ) S.qoff[lane] = inc - cnt;
+            unsigned long long b = 0;
+            if (lane == 0) b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
+            b = __shfl_sync(0xffffffffu, b, 0);
+            over = b + nh > a.stage_cap;
+            __syncwarp();
+            if (!over) {
+                for (uint32_t i = lane; i < nh; i += 32) {
+                    const unsigned long long k = S.hkey[i];
+                    const uint32_t q = (uint32_t)(k >> 42), e = (uint32_t)(k >> 10);
+                    uint32_t rank = 0;
+                    for (uint32_t j = 0; j < nh; ++j) {
+                        const unsigned long long kj = S.hkey[j];
+                        rank += ((uint32_t)(kj >> 42) == q && (uint32_t)(kj >> 10) < e) ? 1u : 0u;
+                    }
+                    const uint32_t slot = (uint32_t)(k & 1023ull);
+                    dts_result r;
+                    r.query_id = S.qid[q] + a.qid_base;
+                    r.entry_id = e;
+                    r.t_start = S.h0[slot];
+                    r.t_end = S.h1[slot];
+                    a.stage[b + S.qoff[q] + rank] = r;
+                }
+                if (lane == 0) a.tile_base[wt] = b;
+            }
+        } else if (!over && lane == 0) {
+            a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
+        }
+        if (over) {
+            if (lane == 0) {
+                a.tile_base[wt] = NONE;
+                const uint32_t slot = atomicAdd(&a.ctr->n_over, 1u);
+                a.over_tiles[slot] = wt;
+            }
+            if (lane < WQ && sp < a.nq && cnt > (uint32_t)SMALL_SORT) {
+                const uint32_t slot = atomicAdd(&a.ctr->n_large, 1u);
+                a.large[slot] = S.qid[lane];
+            }
+        }
+        __syncwarp();
+    }
+
+    // ---- statistics
+    unsigned long long pr = n_probe;
+#pragma unroll
+    for (int o = 16; o; o >>= 1) pr += __shfl_xor_sync(0xffffffffu, pr, o);
+    if (lane == 0 && pr) atomicAdd(&a.ctr->lookups, pr);
+    if (lane == 0 && n_cand) atomicAdd(&a.ctr->candidates, n_cand);
+}
+
+// ------------------------------------------------------ pass 2: emission
+// One warp per warp tile: the tile's staged hits are contiguous and grouped
+// by query in canonical order; copy each query's group to its exact offset.
+__global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ order, uint32_t nq,
+                                                  const uint32_t* __restrict__ counts,
+                                                  const unsigned long long* __restrict__ offsets,
+                                                  const unsigned long long* __restrict__ tile_base,
+                                                  const dts_result* __restrict__ stage,
+                                                  dts_result* __restrict__ out) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const uint32_t ntiles = (nq + WQ - 1) / WQ;
+    const uint32_t wt = blockIdx.x * WW + warp;
+    if (wt >= ntiles) return;
+    const unsigned long long tb = tile_base[wt];
+    if (tb >= NONE - 1) return;                      // recomputed or empty tile
+    const uint32_t sp = wt * WQ + lane;
+    uint32_t cnt = 0;
+    unsigned long long off = 0;
+    if (lane < WQ && sp < nq) {
+        const uint32_t qid = order[sp];
+        cnt = counts[qid];
+        off = offsets[qid];
+    }
+    uint32_t incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += u;
+    }
+    const uint32_t excl = incl - cnt;
+    const uint32_t nh = __shfl_sync(0xffffffffu, incl, 31);
+    for (uint32_t base = 0; base < nh; base += 32) {
+        const uint32_t i = base + lane;
+        int q = 0;
+#pragma unroll
+        for (int step = 16; step; step >>= 1)
+            if (__shfl_sync(0xffffffffu, incl, q + step - 1) <= i) q += step;
+        const unsigned long long o = __shfl_sync(0xffffffffu, off, q);
+        const uint32_t e = __shfl_sync(0xffffffffu, excl, q);
+        if (i < nh) out[o + (i - e)] = stage[tb + i];
+    }
+}
