@@ -271,15 +271,20 @@ __global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restr
     // the cell's run ends at the next key change (most cells hold 1-3 entries)
     size_t e = p + 1;
     while (e < n && keys[e] == k) ++e;
-    unsigned long long h = slot_of(k, ht.log2cap);
+    const unsigned long long bmask = ht.mask >> 2;
+    unsigned long long b = bucket_of(k >> 2, ht.log2cap);
     while (true) {
-        unsigned long long prev = atomicCAS(&ht.slots[h].key, EMPTY_KEY, k);
-        if (prev == EMPTY_KEY || prev == k) {
-            ht.slots[h].start = (uint32_t)p;
-            ht.slots[h].end = (uint32_t)e;
-            return;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+            CellSlot& sl = ht.slots[4 * b + i];
+            const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
+            if (prev == EMPTY_KEY) {
+                sl.start = (uint32_t)p;
+                sl.end = (uint32_t)e;
+                return;
+            }
         }
-        h = (h + 1) & ht.mask;
+        b = (b + 1) & bmask;
     }
 }
 

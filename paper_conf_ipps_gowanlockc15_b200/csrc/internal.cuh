@@ -115,12 +115,15 @@ struct HashTable {
 };
 
 // ---------------------------------------------------------------- device helpers
-// Home slot of a (bin, cell) key.  Keys are row-major with x fastest, so the
-// four keys sharing k >> 2 (x-adjacent cells of one row) hash to the same
-// aligned group of four 16-byte slots: a stencil row of three cells is one or
-// two 64-byte groups instead of three random lines.  Linear probing.
-__device__ __forceinline__ unsigned long long slot_of(unsigned long long k, int log2cap) {
-    return (((k >> 2) * 0x9E3779B97F4A7C15ull) >> (64 - (log2cap - 2))) << 2 | (k & 3ull);
+// Bucketed open addressing: a bucket is 4 slots (64 bytes, one line pair).
+// Keys are row-major with x fastest, so the four keys sharing k >> 2
+// (x-adjacent cells of one row) have the same home bucket: a stencil row of
+// three cells reads one or two buckets instead of three random slots.  A key
+// sits in the first bucket, from its home on, that had a free slot when it
+// was inserted (no deletions), so a lookup stops at the first bucket holding
+// the key or a free slot -- almost always the home bucket.
+__device__ __forceinline__ unsigned long long bucket_of(unsigned long long group, int log2cap) {
+    return (group * 0x9E3779B97F4A7C15ull) >> (64 - (log2cap - 2));
 }
 
 __device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {

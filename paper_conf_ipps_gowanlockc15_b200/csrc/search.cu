@@ -205,7 +205,7 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
 // cx in [clo0, clo0 + cn0): keys are row-major with x fastest, so the
 // non-empty cells of that x range are consecutive in the sorted order and
 // form one contiguous run from the first one's start to the last one's end.
-// Their hash slots share one or two 64-byte slot groups (slot_of).
+// Their hash slots sit in one or two home buckets (bucket_of), read whole.
 __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht,
                                         const double* __restrict__ bin_t0min,
                                         const double* __restrict__ bin_t1max,
@@ -227,32 +227,42 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     const int32_t cy = clo[1] + (int32_t)(r % (uint32_t)cn[1]);
     if (!(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0)) return;
     const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
+    const unsigned long long kend = key0 + (unsigned long long)cn[0];   // row keys [key0, kend)
     const ulonglong2* slots = reinterpret_cast<const ulonglong2*>(ht.slots);
+    const unsigned long long bmask = ht.mask >> 2;
     uint32_t first = 0xffffffffu, last = 0;
-    constexpr int W = 4;   // home slots of up to W cells issued together
-    for (int32_t i0 = 0; i0 < cn[0]; i0 += W) {
-        ulonglong2 sl[W];
+    // any slot whose key lies in the row range contributes (a key met on
+    // another group's chain is found twice; min/max make that harmless);
+    // returns whether the bucket has a free slot (end of the chain)
+    auto scan_bucket = [&](const ulonglong2* B) -> bool {
+        bool empty = false;
 #pragma unroll
-        for (int i = 0; i < W; ++i)
-            if (i0 + i < cn[0]) sl[i] = __ldg(slots + slot_of(key0 + (unsigned long long)(i0 + i),
-                                                              ht.log2cap));
-#pragma unroll
-        for (int i = 0; i < W; ++i) {
-            if (i0 + i >= cn[0]) break;
-            const unsigned long long key = key0 + (unsigned long long)(i0 + i);
-            ++probes;
-            ulonglong2 s = sl[i];
-            if (s.x != key && s.x != EMPTY_KEY) {       // collision: linear probing
-                unsigned long long h = slot_of(key, ht.log2cap);
-                do {
-                    h = (h + 1) & ht.mask;
-                    s = __ldg(slots + h);
-                } while (s.x != key && s.x != EMPTY_KEY);
+        for (int i = 0; i < 4; ++i) {
+            const ulonglong2 s = __ldg(B + i);
+            if (s.x >= key0 && s.x < kend) {
+                first = min(first, (uint32_t)s.y);
+                last = max(last, (uint32_t)(s.y >> 32));
             }
-            if (s.x == key) {
-                if (first == 0xffffffffu) first = (uint32_t)s.y;
-                last = (uint32_t)(s.y >> 32);
-            }
+            empty |= (s.x == EMPTY_KEY);
+        }
+        return empty;
+    };
+    const unsigned long long g0 = key0 >> 2, g1 = (kend - 1) >> 2;
+    for (unsigned long long gg = g0; gg <= g1; gg += 2) {
+        // home buckets of two groups issued together (8 x 128-bit loads)
+        const bool two = gg + 1 <= g1;
+        unsigned long long b0 = bucket_of(gg, ht.log2cap);
+        unsigned long long b1 = two ? bucket_of(gg + 1, ht.log2cap) : b0;
+        probes += two ? 2u : 1u;
+        bool e0 = scan_bucket(slots + 4 * b0);
+        bool e1 = two ? scan_bucket(slots + 4 * b1) : true;
+        while (!e0) {                                    // overflow chains (rare)
+            b0 = (b0 + 1) & bmask;
+            e0 = scan_bucket(slots + 4 * b0);
+        }
+        while (!e1) {
+            b1 = (b1 + 1) & bmask;
+            e1 = scan_bucket(slots + 4 * b1);
         }
     }
     if (first != 0xffffffffu) {
