@@ -275,7 +275,7 @@ def run_own(args):
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(args.config, {}).get("k_pass_count")
+            traffic = json.load(open(tf)).get(args.config, {}).get("k_wtile_count")
         except (ValueError, AttributeError):
             traffic = None
 
@@ -331,7 +331,7 @@ def run_own(args):
                                     "the build, P:L135)"},
             "work": {"candidates_per_pass": st0["candidates"], "cell_lookups": st0["cell_lookups"],
                      "results_per_rank": results},
-            "roofline": {"bound": "hbm", "kernel": "k_pass<count> (fused candidate streaming + "
+            "roofline": {"bound": "hbm", "kernel": "k_wtile_count (pass 1: fused candidate streaming + "
                          "fp64 refine)", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,

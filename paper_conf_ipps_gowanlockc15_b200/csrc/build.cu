@@ -146,7 +146,7 @@ constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
 
 // Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
-__global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
+__global__ void __launch_bounds__(BT, 6) k_gather(const double4* __restrict__ D, size_t n,
                                               const uint32_t* __restrict__ ids, SegSoA soa) {
     const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
     uint32_t id[GATHER_ITEMS];
@@ -208,22 +208,24 @@ __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __
     int f = 0;
     long long b = -1;
     unsigned long long o0 = ~0ull, o1 = 0ull;
+    // the bin is recomputed with bin_of() from t_start exactly as k_keys did
+    // (same inputs, same arithmetic), avoiding a 64-bit division of the key
     if (p < n) {
         const unsigned long long k = keys[p];
         f = (p == 0 || k != keys[p - 1]);
-        b = (long long)(k / g.cells_per_bin);
-        const long long bp = p == 0 ? -1 : (long long)(keys[p - 1] / g.cells_per_bin);
+        const double2 t = st[p];
+        b = bin_of(g, t.x);
+        const long long bp = p == 0 ? -1 : (long long)bin_of(g, st[p - 1].x);
         for (long long bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
         if (p == n - 1)
             for (long long bb = b + 1; bb <= g.m; ++bb) bin_start[bb] = (uint32_t)n;
-        const double2 t = st[p];
         o0 = ordered_bits(t.x);
         o1 = ordered_bits(t.y);
     }
     const int lane = threadIdx.x & 31;
     // one atomic pair per CTA when the CTA's 256 sorted positions share a bin
     // (the common case: bins hold ~10^5 entries), else per warp / per thread
-    const long long bfirst = (long long)(keys[(size_t)blockIdx.x * BT] / g.cells_per_bin);
+    const long long bfirst = bin_of(g, st[(size_t)blockIdx.x * BT].x);
     if (__syncthreads_and(b == bfirst || b < 0)) {
         __shared__ unsigned long long r0[BT / 32], r1[BT / 32];
         for (int off = 16; off; off >>= 1) {

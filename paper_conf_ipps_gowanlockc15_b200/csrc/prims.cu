@@ -129,45 +129,53 @@ constexpr int RS_THREADS = 256;
 constexpr int RS_WARPS = RS_THREADS / 32;
 constexpr int RS_ITEMS = 8;                       // per thread
 constexpr int RS_TILE = RS_THREADS * RS_ITEMS;    // 2048 keys per CTA
-constexpr int RS_RADIX = 256;                     // 8-bit digits
 
 // Per-tile digit histogram; counts laid out digit-major so that one
 // exclusive scan yields every (digit, tile) output offset.
+template <int BITS>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const unsigned long long* __restrict__ keys,
                                                         size_t n, int shift,
                                                         uint32_t* __restrict__ counts,
                                                         uint32_t ntiles) {
-    __shared__ uint32_t h[RS_RADIX];
-    h[threadIdx.x] = 0;
+    constexpr int RADIX = 1 << BITS;
+    __shared__ uint32_t h[RADIX];
+    for (int j = threadIdx.x; j < RADIX; j += RS_THREADS) h[j] = 0;
     __syncthreads();
     size_t base = (size_t)blockIdx.x * RS_TILE;
 #pragma unroll
     for (int i = 0; i < RS_ITEMS; ++i) {
         size_t idx = base + (size_t)i * RS_THREADS + threadIdx.x;
-        if (idx < n) atomicAdd(&h[(uint32_t)(keys[idx] >> shift) & (RS_RADIX - 1)], 1u);
+        if (idx < n) atomicAdd(&h[(uint32_t)(keys[idx] >> shift) & (RADIX - 1)], 1u);
     }
     __syncthreads();
-    counts[(size_t)threadIdx.x * ntiles + blockIdx.x] = h[threadIdx.x];
+    for (int j = threadIdx.x; j < RADIX; j += RS_THREADS)
+        counts[(size_t)j * ntiles + blockIdx.x] = h[j];
 }
 
 // Stable scatter.  Warp w of a tile owns the contiguous chunk
 // [tile + w*256, tile + (w+1)*256); within a warp items are visited in
-// (item, lane) order = input order, ranked with __match_any_sync, and
+// (item, lane) order = input order, ranked with __match_any_sync and
 // warp-private digit counters; a cross-warp prefix per digit then orders the
-// chunks.  Output position = offset(digit, tile) + warp prefix + rank.
+// chunks.  The tile is staged in digit order in shared memory and written
+// out with consecutive threads on consecutive output positions.
+template <int BITS>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ offsets, uint32_t ntiles,
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
-    __shared__ uint32_t wcnt[RS_WARPS][RS_RADIX + 1];
-    __shared__ uint32_t tile_base[RS_RADIX];
-    __shared__ uint32_t local_off[RS_RADIX];
+    constexpr int RADIX = 1 << BITS;
+    constexpr int DPT = RADIX / RS_THREADS;       // digits per thread (1 or 2)
+    static_assert(DPT >= 1 && RADIX % RS_THREADS == 0, "RADIX must be a multiple of the CTA");
+    __shared__ uint32_t wcnt[RS_WARPS][RADIX + 1];
+    __shared__ uint32_t tile_base[RADIX];
+    __shared__ uint32_t local_off[RADIX];
     __shared__ uint32_t warp_tot[RS_WARPS];
     __shared__ unsigned long long sk[RS_TILE];
     __shared__ uint32_t sv[RS_TILE];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    for (int j = lane; j < RS_RADIX + 1; j += 32) wcnt[warp][j] = 0;
-    tile_base[threadIdx.x] = offsets[(size_t)threadIdx.x * ntiles + blockIdx.x];
+    for (int j = lane; j < RADIX + 1; j += 32) wcnt[warp][j] = 0;
+    for (int j = threadIdx.x; j < RADIX; j += RS_THREADS)
+        tile_base[j] = offsets[(size_t)j * ntiles + blockIdx.x];
     __syncwarp();
 
     const size_t wbase = (size_t)blockIdx.x * RS_TILE + (size_t)warp * (32 * RS_ITEMS);
@@ -179,7 +187,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         bool ok = idx < n;
         k[i] = ok ? keys[idx] : 0ull;
         v[i] = ok ? vals[idx] : 0u;
-        dig[i] = ok ? ((uint32_t)(k[i] >> shift) & (RS_RADIX - 1)) : (uint32_t)RS_RADIX;
+        dig[i] = ok ? ((uint32_t)(k[i] >> shift) & (RADIX - 1)) : (uint32_t)RADIX;
     }
     const uint32_t lt_mask = (1u << lane) - 1u;
 #pragma unroll
@@ -196,9 +204,12 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         __syncwarp();
     }
     __syncthreads();
-    uint32_t tile_count;
-    {
-        const int dgt = threadIdx.x;   // RS_THREADS == RS_RADIX
+    // cross-warp prefix per digit; this thread owns digits [t*DPT, t*DPT+DPT)
+    uint32_t tile_count[DPT];
+    uint32_t my_total = 0;
+#pragma unroll
+    for (int j = 0; j < DPT; ++j) {
+        const int dgt = threadIdx.x * DPT + j;
         uint32_t run = 0;
 #pragma unroll
         for (int w = 0; w < RS_WARPS; ++w) {
@@ -206,28 +217,33 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
             wcnt[w][dgt] = run;
             run += c;
         }
-        tile_count = run;
+        tile_count[j] = run;
+        my_total += run;
     }
     // tile-local digit offsets (exclusive scan of the tile histogram)
     {
-        const int lane2 = threadIdx.x & 31, w2 = threadIdx.x >> 5;
-        uint32_t inc = tile_count;
+        uint32_t inc = my_total;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
-            if (lane2 >= o) inc += u;
+            if (lane >= o) inc += u;
         }
-        if (lane2 == 31) warp_tot[w2] = inc;
+        if (lane == 31) warp_tot[warp] = inc;
         __syncthreads();
         uint32_t pre = 0;
-        for (int w = 0; w < w2; ++w) pre += warp_tot[w];
-        local_off[threadIdx.x] = pre + inc - tile_count;
+        for (int w = 0; w < warp; ++w) pre += warp_tot[w];
+        uint32_t run = pre + inc - my_total;
+#pragma unroll
+        for (int j = 0; j < DPT; ++j) {
+            local_off[threadIdx.x * DPT + j] = run;
+            run += tile_count[j];
+        }
     }
     __syncthreads();
     // stage the tile in digit order in shared memory ...
 #pragma unroll
     for (int i = 0; i < RS_ITEMS; ++i) {
-        if (dig[i] < (uint32_t)RS_RADIX) {
+        if (dig[i] < (uint32_t)RADIX) {
             const uint32_t lpos = local_off[dig[i]] + wcnt[warp][dig[i]] + rank[i];
             sk[lpos] = k[i];
             sv[lpos] = v[i];
@@ -240,30 +256,40 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     const uint32_t tn = (uint32_t)min((size_t)RS_TILE, n - tbase);
     for (uint32_t i = threadIdx.x; i < tn; i += RS_THREADS) {
         const unsigned long long key = sk[i];
-        const uint32_t dg = (uint32_t)(key >> shift) & (RS_RADIX - 1);
+        const uint32_t dg = (uint32_t)(key >> shift) & (RADIX - 1);
         const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
         keys_out[dst] = key;
         vals_out[dst] = sv[i];
     }
 }
-static_assert(RS_THREADS == RS_RADIX, "one thread per digit in the cross-warp prefix");
+
+template <int BITS>
+void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned long long* kout,
+                uint32_t* vout, size_t n, int shift, uint32_t ntiles, uint32_t* counts,
+                uint32_t* offs, cudaStream_t s) {
+    const size_t ncount = ((size_t)1 << BITS) * ntiles;
+    k_rs_hist<BITS><<<ntiles, RS_THREADS, 0, s>>>(kin, n, shift, counts, ntiles);
+    DTS_LAUNCH_CHECK();
+    scan_exclusive_u32_to_u32(counts, offs, ncount, s);
+    k_rs_scatter<BITS><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs, ntiles, kout, vout);
+    DTS_LAUNCH_CHECK();
+}
 }  // namespace
 
 void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
     if (n <= 1 || nbits <= 0) return;
+    // 9-bit digits when they save a pass (e.g. 33..36-bit keys: 4 passes, not 5)
+    const int bits = ((nbits + 8) / 9 < (nbits + 7) / 8) ? 9 : 8;
     const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
-    const size_t ncount = (size_t)RS_RADIX * ntiles;
+    const size_t ncount = ((size_t)1 << bits) * ntiles;
     DevBuf<uint32_t> counts(ncount, s), offs(ncount + 1, s);
     unsigned long long *kin = keys, *kout = keys_tmp;
     uint32_t *vin = vals, *vout = vals_tmp;
     int passes = 0;
-    for (int shift = 0; shift < nbits; shift += 8, ++passes) {
-        k_rs_hist<<<ntiles, RS_THREADS, 0, s>>>(kin, n, shift, counts.p, ntiles);
-        DTS_LAUNCH_CHECK();
-        scan_exclusive_u32_to_u32(counts.p, offs.p, ncount, s);
-        k_rs_scatter<<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs.p, ntiles, kout, vout);
-        DTS_LAUNCH_CHECK();
+    for (int shift = 0; shift < nbits; shift += bits, ++passes) {
+        if (bits == 9) radix_pass<9>(kin, vin, kout, vout, n, shift, ntiles, counts.p, offs.p, s);
+        else radix_pass<8>(kin, vin, kout, vout, n, shift, ntiles, counts.p, offs.p, s);
         unsigned long long* tk = kin; kin = kout; kout = tk;
         uint32_t* tv = vin; vin = vout; vout = tv;
     }

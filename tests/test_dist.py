@@ -1,0 +1,77 @@
+"""Multi-process (gloo, world_size 2, CPU) checks of the query-sharding
+plumbing of paper_conf_ipps_gowanlockc15_b200.dist: every
+rank searches a contiguous query-id range, the per-rank result counts are
+all-gathered, and rank-order concatenation at the gathered offsets equals
+the unsharded canonical result.  The per-rank search here is the oracle
+(there is no GPU in the CPU suite); on GPUs it is libdts."""
+import os
+import socket
+
+import numpy as np
+import pytest
+
+import synth
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, out_dir, weighted):
+    import torch.distributed as dist
+
+    import oracle
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    c = synth.make_config("C0")
+    weights = (np.arange(c.Q.shape[0]) % 7 + 1.0) if weighted else None
+
+    def local_search(Qs, d, base):
+        r = oracle.search(c.D, Qs, d)
+        r["query_id"] += np.uint32(base)
+        return r
+
+    res, off, total = dts_dist.search_sharded(local_search, c.Q, c.d, rank, world,
+                                              weights=weights)
+    np.save(os.path.join(out_dir, f"r{rank}.npy"), res)
+    with open(os.path.join(out_dir, f"r{rank}.txt"), "w") as f:
+        f.write(f"{off} {total}")
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("weighted", [False, True])
+def test_sharded_search_matches_unsharded(tmp_path, weighted):
+    import torch.multiprocessing as mp
+
+    import oracle
+    world = 2
+    port = _free_port()
+    mp.spawn(_worker, args=(world, port, str(tmp_path), weighted), nprocs=world, join=True)
+    c = synth.make_config("C0")
+    full = oracle.search(c.D, c.Q, c.d)
+    out = np.empty(full.shape[0], dtype=full.dtype)
+    seen = 0
+    for r in range(world):
+        part = np.load(tmp_path / f"r{r}.npy")
+        off, total = map(int, open(tmp_path / f"r{r}.txt").read().split())
+        assert total == full.shape[0]
+        out[off:off + part.shape[0]] = part
+        seen += part.shape[0]
+    assert seen == full.shape[0]
+    assert out.tobytes() == full.tobytes()
+
+
+def test_shard_bounds():
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    assert dts_dist.shard_bounds(10, 3) == [0, 3, 6, 10]
+    b = dts_dist.shard_bounds(8, 2, weights=[1, 1, 1, 1, 1, 1, 10, 10])
+    assert b[0] == 0 and b[-1] == 8 and 0 < b[1] < 8
+    assert b[1] == 7          # first prefix (16 of 26) reaching half the weight
+    assert dts_dist.shard_bounds(0, 4) == [0, 0, 0, 0, 0]
