@@ -12,11 +12,11 @@
 //   3. k_keys         key = (bin of t_start, cell of the MBB midpoint), row-major
 //                     (bin, z, y, x) so that x-adjacent cells are adjacent runs.
 //   4. radix sort     stable (key, id): within a cell entries stay in id order.
-//   5. k_gather       sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz)
-//                     + per-bin [min t_start, max t_end] extents (B_start/B_end
-//                     of P:L76) with warp-aggregated atomics.
+//   5. k_gather       sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz).
 //   6. k_count_cells / k_insert
-//                     bin offsets (B_first of P:L76) and non-empty cells ->
+//                     bin offsets (B_first of P:L76), per-bin [min t_start,
+//                     max t_end] extents (B_start/B_end of P:L76) with
+//                     CTA-aggregated atomics, and non-empty cells ->
 //                     open-addressing hash table key -> [start, end) (the role
 //                     of G and A of P:L44, with no duplicated ids since every
 //                     entry is in exactly one cell).
@@ -146,7 +146,7 @@ constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
 
 // Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
-__global__ void __launch_bounds__(BT, 6) k_gather(const double4* __restrict__ D, size_t n,
+__global__ void __launch_bounds__(BT, 5) k_gather(const double4* __restrict__ D, size_t n,
                                               const uint32_t* __restrict__ ids, SegSoA soa) {
     const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
     uint32_t id[GATHER_ITEMS];
