@@ -146,7 +146,7 @@ constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
 
 // Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
-__global__ void __launch_bounds__(BT, 5) k_gather(const double4* __restrict__ D, size_t n,
+__global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
                                               const uint32_t* __restrict__ ids, SegSoA soa) {
     const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
     uint32_t id[GATHER_ITEMS];

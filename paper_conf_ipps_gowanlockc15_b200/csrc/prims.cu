@@ -5,6 +5,8 @@
 // These implement the "radix sort and prefix scan" of the index builder
 // (BASELINE.json north_star) and the exclusive scan of
 // per-query result counts of the two-pass compaction (§8(a6)).
+#include <cstdlib>
+
 #include "internal.cuh"
 
 namespace dts {
@@ -279,8 +281,14 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
 void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
     if (n <= 1 || nbits <= 0) return;
-    // 9-bit digits when they save a pass (e.g. 33..36-bit keys: 4 passes, not 5)
-    const int bits = ((nbits + 8) / 9 < (nbits + 7) / 8) ? 9 : 8;
+    // 8-bit digits: measured on C4 (35-bit keys) the 9-bit variant's 4 passes
+    // cost more than 5 8-bit passes (45 KB of shared memory per CTA lowers
+    // occupancy; 113 vs 80 us per pass at 20 M keys).  DTS_RADIX_BITS=9 opts in.
+    static const int pref = [] {
+        const char* e = getenv("DTS_RADIX_BITS");
+        return (e && atoi(e) == 9) ? 9 : 8;
+    }();
+    const int bits = (pref == 9 && (nbits + 8) / 9 < (nbits + 7) / 8) ? 9 : 8;
     const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
     const size_t ncount = ((size_t)1 << bits) * ntiles;
     DevBuf<uint32_t> counts(ncount, s), offs(ncount + 1, s);
