@@ -64,6 +64,21 @@ typedef struct {
     double t_end;
 } dts_result;
 
+/* Candidate generator of an index.  All three return the same results; they
+ * differ only in which candidates are refined. */
+typedef enum {
+    DTS_METHOD_GRID = 0,        /* temporal bins x flattened spatial grid, each entry
+                                   filed once by its MBB midpoint (default)           */
+    DTS_METHOD_TEMPORAL = 1,    /* GPUTemporal (P:L72-P:L80): every entry of the bins
+                                   overlapping the query, the range E_k              */
+    DTS_METHOD_SUBBIN = 2       /* GPUSpatioTemporal (P:L82-P:L120): per-dimension
+                                   spatial subbins of each temporal bin, id arrays
+                                   X, Y, Z in (subbin, bin) order, the dimension with
+                                   the fewest entries chosen per query, temporal
+                                   fallback when the query spans several subbins in
+                                   every dimension                                    */
+} dts_method;
+
 /* Index construction parameters; zero means "choose automatically". */
 typedef struct {
     int      device;            /* CUDA ordinal                                        */
@@ -71,6 +86,10 @@ typedef struct {
     uint32_t cells_per_dim;     /* grid resolution cap per axis; 0 = from extents     */
     double   d_hint;            /* typical search distance, sizes grid cells; 0 = none */
     uint64_t mem_budget_bytes;  /* reserved (0 = free HBM)                             */
+    uint32_t method;            /* dts_method                                          */
+    uint32_t subbins;           /* v of P:L87 per dimension (SUBBIN); 0 = 16, always
+                                   capped so a subbin is wider than the largest
+                                   entry extent in that dimension             */
 } dts_index_params;
 
 /* Per-search statistics (optional output of the *_ex entry points). */
@@ -145,6 +164,9 @@ typedef struct {
     double   max_extent[3];     /* max |x_end - x_start| etc.        */
     double   max_duration;
     float    ms_build;          /* device time of the last build (CUDA events) */
+    uint32_t method;            /* dts_method of the index                   */
+    uint32_t subbins[3];        /* v per dimension (SUBBIN), else 0          */
+    uint64_t subbin_ids[3];     /* length of the X, Y, Z id arrays (SUBBIN)  */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

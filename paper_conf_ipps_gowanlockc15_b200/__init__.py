@@ -45,7 +45,11 @@ class DTSError(RuntimeError):
 class IndexParams(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("temporal_bins", ctypes.c_uint32),
                 ("cells_per_dim", ctypes.c_uint32), ("d_hint", ctypes.c_double),
-                ("mem_budget_bytes", ctypes.c_uint64)]
+                ("mem_budget_bytes", ctypes.c_uint64), ("method", ctypes.c_uint32),
+                ("subbins", ctypes.c_uint32)]
+
+
+METHODS = {"grid": 0, "temporal": 1, "subbin": 2}
 
 
 class SearchStats(ctypes.Structure):
@@ -63,7 +67,9 @@ class IndexInfo(ctypes.Structure):
     _fields_ = [("n", ctypes.c_uint64), ("cells", ctypes.c_uint64), ("bins", ctypes.c_uint32),
                 ("grid", ctypes.c_uint32 * 3), ("bin_width", ctypes.c_double),
                 ("cell_width", ctypes.c_double * 3), ("max_extent", ctypes.c_double * 3),
-                ("max_duration", ctypes.c_double), ("ms_build", ctypes.c_float)]
+                ("max_duration", ctypes.c_double), ("ms_build", ctypes.c_float),
+                ("method", ctypes.c_uint32), ("subbins", ctypes.c_uint32 * 3),
+                ("subbin_ids", ctypes.c_uint64 * 3)]
 
     def as_dict(self):
         out = {}
@@ -132,8 +138,11 @@ def _segments(a) -> np.ndarray:
     return a
 
 
-def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0) -> IndexParams:
-    return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0)
+def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0, method="grid",
+            subbins=0) -> IndexParams:
+    m = METHODS[method] if isinstance(method, str) else int(method)
+    return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0,
+                       m, int(subbins))
 
 
 def _stream_ptr(stream) -> int:
@@ -211,11 +220,11 @@ class DeviceResults:
 
 
 def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int = 0,
-                d_hint: float = 0.0) -> Index:
+                d_hint: float = 0.0, method="grid", subbins: int = 0) -> Index:
     """dts_build_index: D is host (n, 8) float64 (copied)."""
     lib = load()
     D = _segments(D)
-    p = _params(device, temporal_bins, cells_per_dim, d_hint)
+    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index(D.ctypes.data if D.size else None, D.shape[0], ctypes.byref(p),
                                ctypes.byref(h)))
@@ -223,13 +232,14 @@ def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int =
 
 
 def build_index_device(D_dev, n: int = None, device: int = 0, temporal_bins: int = 0,
-                       cells_per_dim: int = 0, d_hint: float = 0.0, stream=None) -> Index:
+                       cells_per_dim: int = 0, d_hint: float = 0.0, stream=None,
+                       method="grid", subbins: int = 0) -> Index:
     """dts_build_index_device: D_dev is a CUDA tensor (n, 8) float64."""
     lib = load()
     ptr = D_dev.data_ptr() if hasattr(D_dev, "data_ptr") else int(D_dev)
     if n is None:
         n = D_dev.shape[0]
-    p = _params(device, temporal_bins, cells_per_dim, d_hint)
+    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index_device(ctypes.c_void_p(ptr), n, ctypes.byref(p),
                                       ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(h)))

@@ -96,6 +96,10 @@ void free_index_memory(dts_index* idx) {
     cudaDeviceSynchronize();
     cache_free(idx->block);
     cache_free(idx->ht.slots);
+    for (int a = 0; a < 3; ++a) {
+        cache_free(idx->sb_block[a]);
+        idx->sb_block[a] = nullptr;
+    }
     idx->block = nullptr;
     idx->ht.slots = nullptr;
 }
@@ -108,6 +112,7 @@ dts_index_params defaults() {
 void check_params(const dts_index_params& p) {
     if (!(p.d_hint >= 0.0) || !std::isfinite(p.d_hint))
         throw Error(DTS_EINVAL, "d_hint must be finite and >= 0");
+    if (p.method > DTS_METHOD_SUBBIN) throw Error(DTS_EINVAL, "unknown method");
 }
 
 void check_aligned(const void* p, const char* what) {
@@ -298,6 +303,11 @@ dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
         r.bin_width = idx->gp.b;
         r.max_duration = idx->gp.maxdur;
         r.ms_build = idx->ms_build;
+        r.method = idx->method;
+        for (int a = 0; a < 3; ++a) {
+            r.subbins[a] = idx->method == DTS_METHOD_SUBBIN ? (uint32_t)idx->sb.v[a] : 0u;
+            r.subbin_ids[a] = idx->sb_len[a];
+        }
         *info = r;
     });
 }

@@ -292,7 +292,119 @@ __global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restr
 
 inline unsigned grid_for(size_t n) { return (unsigned)((n + BT - 1) / BT); }
 
+// ---------------------------------------------------------- subbins (ST)
+// Coordinate A of a segment's start (row 0) / end (row 1).
+template <int A>
+__device__ __forceinline__ double coord(const double4& r) {
+    return A == 0 ? r.y : (A == 1 ? r.z : r.w);
+}
+
+// Number of subbins of dimension a that the entry at sorted position p
+// overlaps (its extent [min, max] in a: at most 2 when subbins are
+// wider than the largest extent).
+template <int A>
+__global__ void __launch_bounds__(BT) k_sb_count(const double4* __restrict__ D,
+                                                const uint32_t* __restrict__ eid, size_t n,
+                                                SubbinIndex sb, uint32_t* __restrict__ cnt) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p >= n) return;
+    const uint32_t i = eid[p];
+    const double c0 = coord<A>(D[2 * (size_t)i]), c1 = coord<A>(D[2 * (size_t)i + 1]);
+    cnt[p] = (uint32_t)(subbin_of(sb, A, fmax(c0, c1)) - subbin_of(sb, A, fmin(c0, c1)) + 1);
+}
+
+// One (key = subbin * m + bin, value = p) pair per overlapped subbin.
+template <int A>
+__global__ void __launch_bounds__(BT) k_sb_emit(const double4* __restrict__ D,
+                                               const uint32_t* __restrict__ eid,
+                                               const double2* __restrict__ st, size_t n,
+                                               SubbinIndex sb, GridParams g,
+                                               const unsigned long long* __restrict__ off,
+                                               unsigned long long* __restrict__ keys,
+                                               uint32_t* __restrict__ vals) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p >= n) return;
+    const uint32_t i = eid[p];
+    const double c0 = coord<A>(D[2 * (size_t)i]), c1 = coord<A>(D[2 * (size_t)i + 1]);
+    const int32_t jlo = subbin_of(sb, A, fmin(c0, c1)), jhi = subbin_of(sb, A, fmax(c0, c1));
+    const unsigned long long bin = (unsigned long long)bin_of(g, st[p].x);
+    unsigned long long o = off[p];
+    for (int32_t j = jlo; j <= jhi; ++j, ++o) {
+        keys[o] = (unsigned long long)j * (unsigned long long)g.m + bin;
+        vals[o] = (uint32_t)p;
+    }
+}
+
+// dir[k] = first position of key >= k in the sorted keys, k in [0, nkeys].
+__global__ void __launch_bounds__(BT) k_sb_dir(const unsigned long long* __restrict__ keys,
+                                              size_t len, unsigned long long nkeys,
+                                              uint32_t* __restrict__ dir) {
+    size_t q = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (q >= len) return;
+    const long long k = (long long)keys[q];
+    const long long kp = q == 0 ? -1 : (long long)keys[q - 1];
+    for (long long kk = kp + 1; kk <= k; ++kk) dir[kk] = (uint32_t)q;
+    if (q == len - 1)
+        for (long long kk = k + 1; kk <= (long long)nkeys; ++kk) dir[kk] = (uint32_t)len;
+}
+
 }  // namespace
+
+// GPUSpatioTemporal index (P:L86-P:L92), built on the device over the sorted
+// entries: per dimension, (subbin, bin) keys for every overlap, a stable
+// radix sort (positions stay ascending inside a chunk) and a directory of
+// chunk offsets.
+static void build_subbins(dts_index* idx, const double4* D, size_t n, const Bounds& hb,
+                          const dts_index_params& p, cudaStream_t s) {
+    const GridParams& g = idx->gp;
+    SubbinIndex& sb = idx->sb;
+    const int32_t vreq = p.subbins > 0 ? (int32_t)std::min<uint32_t>(p.subbins, 1u << 16) : 16;
+    sb.m = g.m;
+    for (int a = 0; a < 3; ++a) {
+        const double span = hb.hi[a] - hb.lo[a];
+        int32_t v = vreq;
+        if (hb.ext[a] > 0.0) v = (int32_t)std::min<double>(v, std::max(1.0, std::floor(span / hb.ext[a])));
+        if (!(span > 0.0)) v = 1;
+        sb.v[a] = v;
+        sb.o[a] = hb.lo[a];
+        sb.inv_w[a] = span > 0.0 ? (double)v / span : 0.0;
+    }
+    for (int a = 0; a < 3; ++a) {
+        DevBuf<uint32_t> cnt(n, s);
+        DevBuf<unsigned long long> off(n + 1, s);
+        if (a == 0) k_sb_count<0><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, n, sb, cnt.p);
+        else if (a == 1) k_sb_count<1><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, n, sb, cnt.p);
+        else k_sb_count<2><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, n, sb, cnt.p);
+        DTS_LAUNCH_CHECK();
+        scan_exclusive_u32_to_u64(cnt.p, off.p, n, s);
+        unsigned long long len = 0;
+        DTS_CUDA(cudaMemcpyAsync(&len, off.p + n, sizeof(len), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        if (len >= (1ull << 32)) throw Error(DTS_ENOTSUP, "subbin id array exceeds 2^32 entries");
+        const unsigned long long nkeys = (unsigned long long)sb.v[a] * (unsigned long long)g.m;
+        DevBuf<unsigned long long> keys(len, s), keys_tmp(len, s);
+        DevBuf<uint32_t> vals_tmp(len, s);
+        uint32_t* blk = static_cast<uint32_t*>(cache_alloc((len + nkeys + 1) * sizeof(uint32_t)));
+        idx->sb_block[a] = blk;
+        idx->sb_len[a] = len;
+        if (a == 0)
+            k_sb_emit<0><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+                                                    off.p, keys.p, blk);
+        else if (a == 1)
+            k_sb_emit<1><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+                                                    off.p, keys.p, blk);
+        else
+            k_sb_emit<2><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+                                                    off.p, keys.p, blk);
+        DTS_LAUNCH_CHECK();
+        radix_sort_pairs(keys.p, blk, keys_tmp.p, vals_tmp.p, len, bits_for(nkeys - 1), s);
+        k_sb_dir<<<grid_for(len), BT, 0, s>>>(keys.p, len, nkeys, blk + len);
+        DTS_LAUNCH_CHECK();
+        sb.ids[a] = blk;
+        sb.dir[a] = blk + len;
+        DTS_CUDA(cudaStreamSynchronize(s));
+    }
+}
 
 // Host-side choice of the temporal bins and spatial cells.
 static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g) {
@@ -315,6 +427,9 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
         const double span = b.hi[a] - b.lo[a];
         double w = b.ext[a] + (p.d_hint > 0.0 ? p.d_hint : 0.0);
         if (p.cells_per_dim > 0) w = std::max(w, span / (double)p.cells_per_dim);
+        // temporal and subbin methods use one cell per bin: the sort key is the
+        // bin, so entries are grouped by t_start bin as in P:L76
+        if (p.method != DTS_METHOD_GRID) w = std::max(span, 1.0) * 2.0;
         w = std::max(w, span / (MAXC - 1.0));
         w = std::max(w, 1e-12 * b.absmax);
         if (!(w > 0.0) || !std::isfinite(w)) w = 1.0;
@@ -419,6 +534,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
     k_insert<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
     DTS_LAUNCH_CHECK();
+
+    // 7. GPUSpatioTemporal subbin arrays (DTS_METHOD_SUBBIN)
+    idx->method = p.method;
+    if (p.method == DTS_METHOD_SUBBIN) {
+        keys.release();
+        ids.release();
+        build_subbins(idx, D, n, hb, p, s);
+    }
 
     DTS_CUDA(cudaEventRecord(e1, s));
     DTS_CUDA(cudaEventSynchronize(e1));

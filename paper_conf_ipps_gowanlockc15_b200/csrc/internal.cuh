@@ -114,6 +114,26 @@ struct HashTable {
     int log2cap;
 };
 
+// GPUSpatioTemporal subbins (P:L86-P:L92): per dimension a, v[a] subbins of
+// width >= the largest entry extent in a; ids[a] holds the sorted positions of
+// the entries overlapping subbin j of bin i, chunks in (j, i) lexicographic
+// order; chunk (j, i) is ids[a][dir[a][j*m + i] .. dir[a][j*m + i + 1]).
+struct SubbinIndex {
+    double o[3];
+    double inv_w[3];
+    int32_t v[3];
+    int32_t m;
+    const uint32_t* ids[3];
+    const uint32_t* dir[3];
+};
+
+__device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double x) {
+    double f = floor((x - s.o[a]) * s.inv_w[a]);
+    if (!(f > 0.0)) return 0;
+    if (f >= (double)(s.v[a] - 1)) return s.v[a] - 1;
+    return (int32_t)f;
+}
+
 // ---------------------------------------------------------------- device helpers
 // Bucketed open addressing: a bucket is 4 slots (64 bytes, one line pair).
 // Keys are row-major with x fastest, so the four keys sharing k >> 2
@@ -199,6 +219,10 @@ struct dts_index {
     double max_ext[3] = {0, 0, 0};
     float ms_build = 0.f;
     int key_bits = 0;
+    uint32_t method = 0;           // dts_method
+    dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only
+    uint32_t* sb_block[3] = {nullptr, nullptr, nullptr};   // ids + dir per dimension
+    uint64_t sb_len[3] = {0, 0, 0};
 };
 
 namespace dts {

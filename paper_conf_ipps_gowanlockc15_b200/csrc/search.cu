@@ -70,7 +70,9 @@ struct Stencil {
     int32_t lb, hb;          // bin range
     int32_t clo[3], cn[3];   // cell range per axis (start, count)
     uint32_t mode;
-    uint32_t nlook;          // probes: ncomb (grid), 1 (temporal), 0 (dead)
+    uint32_t nlook;          // probes: rows (grid), 1 (single run), 0 (dead)
+    uint32_t rstart, rcnt;   // MODE_TEMPORAL: the one run (positions or id-array slots)
+    uint32_t rind;           // 0: direct sorted positions; 1 + a: slots of subbin array a
 };
 
 // ------------------------------------------------------------- refinement
@@ -157,10 +159,12 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
                                                 double d, bool live,
                                                 const uint32_t* __restrict__ bin_start,
                                                 const double* __restrict__ bin_t0min,
-                                                const double* __restrict__ bin_t1max) {
+                                                const double* __restrict__ bin_t1max,
+                                                uint32_t method, const SubbinIndex& sb) {
     Stencil s;
     s.mode = MODE_DEAD;
     s.nlook = 0;
+    s.rstart = s.rcnt = s.rind = 0;
     s.lb = s.hb = 0;
     for (int a = 0; a < 3; ++a) { s.clo[a] = 0; s.cn[a] = 1; }
     if (!live) return s;
@@ -179,25 +183,60 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
         s.lb = s.hb = 0;
         return s;
     }
+    // the bins' contiguous entry range: GPUTemporal's E_k
+    const uint32_t b0 = __ldg(&bin_start[s.lb]);
+    const uint32_t T = __ldg(&bin_start[s.hb + 1]) - b0;
+    if (T == 0) return s;                                  // no entry in these bins
+    s.mode = MODE_TEMPORAL;
+    s.nlook = 1;
+    s.rstart = b0;
+    s.rcnt = T;
+    s.rind = 0;
+    if (method == DTS_METHOD_TEMPORAL) return s;
+    if (method == DTS_METHOD_SUBBIN) {
+        // GPUSpatioTemporal: among the dimensions where [qlo-d, qhi+d]
+        // falls in ONE subbin, take the one whose chunk (subbin j, bins
+        // lb..hb) -- contiguous in that dimension's id array -- is smallest;
+        // entries overlapping subbin j are listed once, so no duplicates.
+        // Otherwise fall back to the temporal range.
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            const double ms = 1e-12 * (fabs(qlo[a]) + fabs(qhi[a]) + fabs(sb.o[a]) + d);
+            const int32_t jlo = subbin_of(sb, a, qlo[a] - d - ms);
+            const int32_t jhi = subbin_of(sb, a, qhi[a] + d + ms);
+            if (jlo != jhi) continue;
+            const uint32_t* dir = sb.dir[a] + (size_t)jlo * (size_t)sb.m;
+            const uint32_t c0 = __ldg(dir + s.lb), c1 = __ldg(dir + s.hb + 1);
+            if (c1 - c0 < s.rcnt || (s.rind == 0 && c1 - c0 <= s.rcnt)) {
+                s.rstart = c0;
+                s.rcnt = c1 - c0;
+                s.rind = 1 + a;
+            }
+        }
+        return s;
+    }
     double ncomb = (double)(s.hb - s.lb + 1);
+    int32_t clo[3], cn[3];
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
         const double ms = 1e-12 * (fabs(qlo[a]) + fabs(qhi[a]) + fabs(g.o[a]) + d + g.half_ext[a]);
         const double r = d + g.half_ext[a] + ms;
-        s.clo[a] = cell_of(g, a, qlo[a] - r);
-        s.cn[a] = cell_of(g, a, qhi[a] + r) - s.clo[a] + 1;
-        ncomb *= (double)s.cn[a];
+        clo[a] = cell_of(g, a, qlo[a] - r);
+        cn[a] = cell_of(g, a, qhi[a] + r) - clo[a] + 1;
+        ncomb *= (double)cn[a];
     }
-    const uint32_t T = __ldg(&bin_start[s.hb + 1]) - __ldg(&bin_start[s.lb]);
-    if (T == 0) return s;                                  // no entry in these bins
-    if (ncomb >= (double)T) {                              // probing costs more than scanning
-        s.mode = MODE_TEMPORAL;
-        s.nlook = 1;
-    } else {
+    if (ncomb < (double)T) {                               // else probing costs more than scanning
         s.mode = MODE_GRID;
+#pragma unroll
+        for (int a = 0; a < 3; ++a) { s.clo[a] = clo[a]; s.cn[a] = cn[a]; }
         s.nlook = (uint32_t)(s.hb - s.lb + 1) * (uint32_t)s.cn[1] * (uint32_t)s.cn[2];  // rows
     }
     return s;
+}
+
+// Id array of a single-run query: 1 + a -> subbin array of dimension a.
+__device__ __forceinline__ const uint32_t* sb_ids(const SubbinIndex& sb, uint32_t ind) {
+    return ind == 1 ? sb.ids[0] : (ind == 2 ? sb.ids[1] : sb.ids[2]);
 }
 
 // Resolve probe `loc` of a query's stencil into one entry run [start,
@@ -212,12 +251,13 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
                                         const uint32_t* __restrict__ bin_start, uint32_t mode,
                                         int32_t lb, int32_t hb, const int32_t clo[3],
                                         const int32_t cn[3], double qt0, double qt1, uint32_t loc,
+                                        uint32_t rstart, uint32_t rcnt,
                                         uint32_t& start, uint32_t& cnt, uint32_t& probes) {
     start = 0;
     cnt = 0;
-    if (mode == MODE_TEMPORAL) {
-        start = __ldg(&bin_start[lb]);
-        cnt = __ldg(&bin_start[hb + 1]) - start;
+    if (mode == MODE_TEMPORAL) {                 // the query's single precomputed run
+        start = rstart;
+        cnt = rcnt;
         return;
     }
     const uint32_t nzy = (uint32_t)cn[1] * (uint32_t)cn[2];
@@ -320,6 +360,8 @@ struct PassArgs {
     const uint32_t* tiles;         // tiles to process (TQ sorted positions each)
     dts_result* out;
     uint32_t qid_base;
+    uint32_t method;
+    SubbinIndex sb;
 };
 
 // Warp w of CTA b processes sorted position tiles[b / (TQ/PW)]*TQ + ...; the
@@ -338,8 +380,9 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
     QState q;
     double qlo[3], qhi[3];
     const bool live = load_query(a.Q, qid, q, qlo, qhi);
-    const Stencil st =
-        make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
+    const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start, a.bin_t0min,
+                                    a.bin_t1max, a.method, a.sb);
+    const uint32_t* ind = st.rind ? sb_ids(a.sb, st.rind) : nullptr;   // subbin id array
     const double d2 = a.d * a.d;
     unsigned long long out_pos = a.offsets[qid];
     uint32_t dummy = 0;
@@ -348,7 +391,7 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
         uint32_t start = 0, cnt = 0;
         if (c < st.nlook)
             resolve(a.g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, st.mode, st.lb, st.hb,
-                    st.clo, st.cn, q.t0, q.t1, c, start, cnt, dummy);
+                    st.clo, st.cn, q.t0, q.t1, c, st.rstart, st.rcnt, start, cnt, dummy);
         unsigned long long incl = cnt;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
@@ -371,6 +414,7 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
                 for (int step = 16; step; step >>= 1)
                     if (s_excl[warp][j + step] <= t) j += step;
                 p = s_start[warp][j] + (uint32_t)(t - s_excl[warp][j]);
+                if (ind) p = __ldg(ind + p);
                 hit = refine(q, __ldg(a.soa.st + p), __ldg(a.soa.sx + p), __ldg(a.soa.sy + p),
                              __ldg(a.soa.sz + p), d2, r0, r1);
             }
@@ -599,6 +643,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.large = large.p;
     ta.qid_base = qid_base;
     ta.ctr = ctr.p;
+    ta.method = idx->method;
+    ta.sb = idx->sb;
     {
         int dev = 0, nsm = 148;
         cudaGetDevice(&dev);
@@ -662,6 +708,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 pa.tiles = over_tiles.p;
                 pa.out = raw.p;
                 pa.qid_base = qid_base;
+                pa.method = idx->method;
+                pa.sb = idx->sb;
                 const unsigned nb = h.c.n_over * (TQ / PW);
                 k_pass_scatter<<<nb, PT, 0, s>>>(pa);
                 DTS_LAUNCH_CHECK();

@@ -25,6 +25,7 @@ struct WarpSmem {
     double qt0[WQ], qt1[WQ], qx0[WQ], qvx[WQ], qy0[WQ], qvy[WQ], qz0[WQ], qvz[WQ];
     int32_t lb[WQ], hb[WQ], clo[3][WQ], cn[3][WQ];
     uint32_t qid[WQ], mode[WQ], qcount[WQ], qoff[WQ];
+    uint32_t rstart[WQ], rcnt[WQ], rind[WQ];   // single-run queries (temporal / subbin)
     unsigned long long lkoff[WQ + 1];
     unsigned long long hkey[WH];        // (query << 42) | (entry id << 10) | slot
     double h0[WH], h1[WH];
@@ -50,6 +51,8 @@ struct TileArgs {
     uint32_t* large;                   // query ids (recomputed tiles) with count > SMALL_SORT
     uint32_t qid_base;
     Counters* ctr;
+    uint32_t method;
+    SubbinIndex sb;
 };
 
 __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
@@ -104,8 +107,8 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 qid = a.order[sp];
                 live = load_query(a.Q, qid, q, qlo, qhi);
             }
-            const Stencil st =
-                make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min, a.bin_t1max);
+            const Stencil st = make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min,
+                                            a.bin_t1max, a.method, a.sb);
             S.qt0[lane] = q.t0; S.qt1[lane] = q.t1;
             S.qx0[lane] = q.x0; S.qvx[lane] = q.vx;
             S.qy0[lane] = q.y0; S.qvy[lane] = q.vy;
@@ -115,6 +118,9 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             for (int ax = 0; ax < 3; ++ax) { S.clo[ax][lane] = st.clo[ax]; S.cn[ax][lane] = st.cn[ax]; }
             S.qid[lane] = qid;
             S.mode[lane] = st.mode;
+            S.rstart[lane] = st.rstart;
+            S.rcnt[lane] = st.rcnt;
+            S.rind[lane] = st.rind;
             S.qcount[lane] = 0;
             nlook = st.nlook;
         }
@@ -134,7 +140,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         // ---- 1: rounds of 32 row probes, flattened, candidates two per lane
         for (unsigned long long r0 = 0; r0 < Ltot; r0 += 32) {
             const unsigned long long l = r0 + lane;
-            uint32_t start = 0, cnt = 0;
+            uint32_t start = 0, cnt = 0, ind = 0;
             int qi = 0;
             if (l < Ltot) {
 #pragma unroll
@@ -144,7 +150,9 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
                 const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
                 resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
-                        S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, start, cnt, n_probe);
+                        S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, S.rstart[qi], S.rcnt[qi],
+                        start, cnt, n_probe);
+                ind = S.rind[qi];
             }
             unsigned long long incl = cnt;
 #pragma unroll
@@ -169,10 +177,15 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 const unsigned long long e2 = __shfl_sync(0xffffffffu, excl, j2);
                 const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
                 const int qi2 = __shfl_sync(0xffffffffu, qi, j2);
+                const uint32_t i1 = __shfl_sync(0xffffffffu, ind, j1);
+                const uint32_t i2 = __shfl_sync(0xffffffffu, ind, j2);
                 const bool v1 = t1 < total, v2 = t2 < total;
                 if (v1) {
-                    const uint32_t p1 = s1 + (uint32_t)(t1 - e1);
-                    const uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
+                    uint32_t p1 = s1 + (uint32_t)(t1 - e1);
+                    uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
+                    if (i1) p1 = __ldg(sb_ids(a.sb, i1) + p1);   // subbin id array slot
+                    if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + p2);
+                    else if (!v2) p2 = p1;
                     const double2 st1 = __ldg(a.soa.st + p1), sx1 = __ldg(a.soa.sx + p1);
                     const double2 sy1 = __ldg(a.soa.sy + p1), sz1 = __ldg(a.soa.sz + p1);
                     const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);

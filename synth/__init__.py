@@ -191,6 +191,43 @@ def make_config(name: str, rank: int = 0, scale: float = 1.0) -> Config:
         Q = segments_from_trajectories(tq, pq)
         return Config(name, D, Q, 5.0, (1.0, 5.0, 20.0, 50.0),
                       "sparse long-span random walks (P:L127 shape stretched)")
+    # ---- paper-replica scenarios; sizes exactly as P:L127-P:L141
+    if name == "S1":
+        # Random: 2,500 random-walk trajectories x 400 timesteps = 997,500
+        # segments, start times U[0,100]; query: 100 trajectories x
+        # 400 timesteps = 39,900 segments.  The paper gives no spatial
+        # scale; the walk is C3's ([0,1000]^3, N(0,1) steps).
+        ntraj, nq_traj = max(2, int(2500 * scale)), max(1, int(100 * scale))
+        t, pos = random_walks(rng(11), ntraj, 400, 1000.0, 1.0, 100.0)
+        D = segments_from_trajectories(t, pos)
+        tq, pq = random_walks(rng(11 + 1000 + rank), nq_traj, 400, 1000.0, 1.0, 100.0)
+        Q = segments_from_trajectories(tq, pq)
+        return Config(name, D, Q, 50.0, (1.0, 5.0, 20.0, 50.0, 100.0),
+                      "paper S1: Random (P:L127, P:L139)")
+    if name == "S2":
+        # Merger shape: 131,072 particles x 193 timesteps = 25,165,824
+        # segments; query: 265 trajectories x 193 timesteps = 50,880
+        # segments, drawn from D.
+        n1 = max(1, int(65536 * scale))
+        nq_traj = max(1, int(265 * scale))
+        t, pos = galaxy(rng(12), n1, n1, 193)
+        D = segments_from_trajectories(t, pos)
+        del t, pos
+        Q = _sample_query_trajectories(D, 2 * n1, 192, nq_traj, 12 + 1000 + rank)
+        return Config(name, D, Q, 0.001, (0.001, 0.01, 0.1, 1.0, 5.0),
+                      "paper S2: Merger-shaped (P:L129, P:L140)")
+    if name == "S3":
+        # Random-dense: 65,536 particles x 193 timesteps = 12,582,912 segments
+        # at 0.112 stars/pc^3, i.e. a 585,142 pc^3 cube; query: 265
+        # trajectories x 193 timesteps = 50,880 segments, from D.
+        ntraj, nq_traj = max(2, int(65536 * scale)), max(1, int(265 * scale))
+        side = (ntraj / 0.112) ** (1.0 / 3.0)
+        t, pos = random_walks(rng(13), ntraj, 193, side, 0.05, 100.0)
+        D = segments_from_trajectories(t, pos)
+        del t, pos
+        Q = _sample_query_trajectories(D, ntraj, 192, nq_traj, 13 + 1000 + rank)
+        return Config(name, D, Q, 0.05, (0.01, 0.02, 0.03, 0.05, 0.09),
+                      "paper S3: Random-dense (P:L131, P:L141)")
     raise ValueError(f"unknown config {name!r}")
 
 

@@ -216,3 +216,48 @@ def test_invalid_inputs_raise(dts):
         dts.search(idx, badq, 0.1)
     # the index stays usable after an error
     assert dts.search(idx, Q, 0.1).dtype == dts.RESULT_DTYPE
+
+
+# ------------------------------------------------ candidate generators (§8 f1)
+@pytest.mark.parametrize("method,subbins", [("temporal", 0), ("subbin", 2), ("subbin", 4),
+                                            ("subbin", 16)])
+def test_methods_match_oracle_and_grid(dts, oracle_mod, method, subbins):
+    """GPUTemporal / GPUSpatioTemporal candidate generators return the same
+    bytes as the grid and match the oracle."""
+    cases = [(synth.make_config("C0"), (0.0, 0.05, 0.2)),
+             (synth.make_config("C2", scale=0.004), (0.09, 2.0)),
+             (synth.make_config("C3", scale=0.01), (5.0, 50.0))]
+    for c, dl in cases:
+        grid = dts.build_index(c.D)
+        alt = dts.build_index(c.D, method=method, subbins=subbins)
+        info = alt.info()
+        assert info["method"] == {"temporal": 1, "subbin": 2}[method]
+        if method == "subbin":
+            assert all(v >= 1 for v in info["subbins"])
+            assert all(info["subbin_ids"][a] >= c.D.shape[0] for a in range(3))
+        for d in dl:
+            ref = dts.search(grid, c.Q, d)
+            got = dts.search(alt, c.Q, d)
+            assert got.tobytes() == ref.tobytes(), (method, subbins, d)
+            parity.compare(got, oracle_mod.search(c.D, c.Q, d, threads=THREADS), c.D, c.Q, d,
+                           oracle_mod)
+
+
+def test_subbin_adversarial(dts, oracle_mod):
+    for seed in range(60):
+        D, Q = synth.adversarial(5000 + seed, 50, 50)
+        d = [0.0, 0.03, 0.1, 0.3][seed % 4]
+        idx = dts.build_index(D, method="subbin", subbins=[2, 4, 8][seed % 3])
+        got = dts.search(idx, Q, d)
+        parity.compare(got, oracle_mod.search(D, Q, d), D, Q, d, oracle_mod)
+
+
+def test_subbin_c1_sampled(dts, oracle_mod):
+    c = synth.make_config("C1")
+    idx = dts.build_index(c.D, method="subbin")
+    g = synth.rng(7)
+    qs = np.sort(g.choice(c.Q.shape[0], size=64, replace=False))
+    for d in (0.005, 0.02):
+        got = dts.search(idx, c.Q, d)
+        ora = oracle_mod.search_queries(c.D, c.Q, qs, d, threads=THREADS)
+        parity.compare(parity.restrict(got, qs), ora, c.D, c.Q, d, oracle_mod)

@@ -338,3 +338,18 @@ def test_config_shapes_small():
     ntraj = c2.D.shape[0] // 192
     side = c2.D[:, [1, 2, 3]].max() - c2.D[:, [1, 2, 3]].min()
     assert ntraj / side ** 3 == pytest.approx(0.112, rel=0.1)   # P:L131 density
+
+
+def test_paper_replica_shapes():
+    """S1-S3 reproduce the paper's dataset and query sizes (P:L127-P:L141)."""
+    s1 = synth.make_config("S1", scale=0.02)
+    assert s1.D.shape[0] == synth.segment_count(50, 400)
+    assert s1.Q.shape[0] == synth.segment_count(2, 400)
+    s3 = synth.make_config("S3", scale=0.002)
+    ntraj = s3.D.shape[0] // 192
+    side = s3.D[:, [1, 2, 3, 5, 6, 7]].max() - s3.D[:, [1, 2, 3, 5, 6, 7]].min()
+    assert ntraj / side ** 3 == pytest.approx(0.112, rel=0.15)      # P:L131 density
+    # full sizes follow from the same formulas
+    assert synth.segment_count(2500, 400) == 997_500
+    assert synth.segment_count(2 * 65536, 193) == 25_165_824
+    assert synth.segment_count(65536, 193) == 12_582_912
