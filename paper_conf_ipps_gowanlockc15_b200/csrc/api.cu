@@ -3,6 +3,7 @@
 // search itself runs in the kernels of build.cu / search.cu / prims.cu.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdlib>
 #include <map>
@@ -67,19 +68,29 @@ void* pinned_alloc(size_t bytes) {
         }
     }
     void* b = nullptr;
-    cudaError_t e = cudaMallocHost(&b, bytes + HDR);
+    // very large outputs (streamed searches) fall back to pageable memory
+    cudaError_t e = bytes <= (size_t(16) << 30) ? cudaMallocHost(&b, bytes + HDR)
+                                                : cudaErrorMemoryAllocation;
+    size_t kind = 0;
     if (e != cudaSuccess) {
         cudaGetLastError();
-        throw Error(DTS_ENOMEM, "cudaMallocHost failed for the result buffer");
+        b = std::malloc(bytes + HDR);
+        if (!b) throw Error(DTS_ENOMEM, "host allocation failed for the result buffer");
+        kind = 1;
     }
-    *static_cast<size_t*>(b) = bytes;
+    static_cast<size_t*>(b)[0] = bytes;
+    static_cast<size_t*>(b)[1] = kind;
     return static_cast<char*>(b) + HDR;
 }
 
 void pinned_free(void* p) {
     if (!p) return;
     void* b = static_cast<char*>(p) - HDR;
-    size_t bytes = *static_cast<size_t*>(b);
+    size_t bytes = static_cast<size_t*>(b)[0];
+    if (static_cast<size_t*>(b)[1] == 1) {
+        std::free(b);
+        return;
+    }
     std::lock_guard<std::mutex> lk(g_mu);
     if (g_pinned_cached + bytes <= (size_t(4) << 30)) {
         g_pinned_free.emplace(bytes, b);
@@ -176,6 +187,57 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
     return DTS_OK;
 }
 
+// Host-output search whose results exceed device memory: plan query-id
+// chunks from the per-query counts so each chunk's results fit, search each
+// chunk (ids offset by the chunk start) and copy its results to the host at
+// the chunk's offset.  Concatenation in chunk order is the canonical order.
+dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_t nq, double d,
+                            uint32_t qid_base, cudaStream_t s, const ResultsTooLarge& big,
+                            dts_search_stats* stats, unsigned long long cap) {
+    size_t free_b = 0, total_b = 0;
+    DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
+    const unsigned long long budget = std::max<unsigned long long>(
+        1, std::min<unsigned long long>(cap ? cap : ~0ull,
+                                        (unsigned long long)(0.35 * (double)free_b / 72.0)));
+    dts_result* h = static_cast<dts_result*>(pinned_alloc(big.total * sizeof(dts_result)));
+    dts_search_stats agg{};
+    if (stats) agg.time_kernels = stats->time_kernels;
+    try {
+        unsigned long long off = 0;
+        size_t a = 0;
+        while (a < nq) {
+            size_t b = a;
+            unsigned long long acc = 0;
+            while (b < nq && (b == a || acc + big.counts[b] <= budget)) acc += big.counts[b++];
+            SearchOut so;
+            dts_search_stats cs{};
+            search_device(index, dQ + a, b - a, d, qid_base + (uint32_t)a, s, &so, &cs);
+            if (so.count != acc) {
+                cache_free(so.results);
+                throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
+            }
+            if (so.count) {
+                DTS_CUDA(cudaMemcpyAsync(h + off, so.results, so.count * sizeof(dts_result),
+                                         cudaMemcpyDeviceToHost, s));
+                DTS_CUDA(cudaStreamSynchronize(s));
+                cache_free(so.results);
+            }
+            off += so.count;
+            agg.candidates += cs.candidates;
+            agg.cell_lookups += cs.cell_lookups;
+            agg.max_results_per_query = std::max(agg.max_results_per_query,
+                                                 cs.max_results_per_query);
+            a = b;
+        }
+        agg.results = off;
+    } catch (...) {
+        pinned_free(h);
+        throw;
+    }
+    if (stats) *stats = agg;
+    return h;
+}
+
 dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
                          uint32_t qid_base, cudaStream_t s, bool host, dts_result** out_results,
                          size_t* out_count, dts_search_stats* stats) {
@@ -198,7 +260,20 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
             if (nq)
                 DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment),
                                          cudaMemcpyHostToDevice, s));
-            search_device(index, dQ.p, nq, d, qid_base, s, &so, stats);
+            // DTS_MAX_DEVICE_RESULTS caps the results held on the device at
+            // once (testing knob for the streamed path; default: memory)
+            const char* cap_env = getenv("DTS_MAX_DEVICE_RESULTS");
+            const unsigned long long cap = cap_env ? std::strtoull(cap_env, nullptr, 10) : ~0ull;
+            try {
+                search_device(index, dQ.p, nq, d, qid_base, s, &so, stats, cap ? cap : ~0ull);
+            } catch (ResultsTooLarge& big) {
+                // stream: query-id chunks whose results fit, each searched
+                // and copied out at its offset (the paper processed Q
+                // incrementally when its result buffer filled)
+                ret = search_streamed(index, dQ.p, nq, d, qid_base, s, big, stats, cap);
+                cnt = (size_t)big.total;
+                return;
+            }
             if (so.count) {
                 dts_result* h = nullptr;
                 try {

@@ -10,6 +10,7 @@
 #include <cstring>
 #include <stdexcept>
 #include <string>
+#include <vector>
 
 #include "../../include/dts.h"
 
@@ -232,6 +233,19 @@ struct SearchOut {
     dts_result* results = nullptr;   // device, cudaMalloc'd (caller owns)
     size_t count = 0;
 };
+// Thrown by search_device when the results would not fit in device memory
+// (or exceed max_results): carries the per-query counts (query-id order) so a
+// host caller can stream the search in query chunks.
+struct ResultsTooLarge : Error {
+    unsigned long long total;
+    std::vector<uint32_t> counts;
+    explicit ResultsTooLarge(unsigned long long t)
+        : Error(DTS_ENOMEM, "results (" + std::to_string(t) +
+                                ") do not fit in device memory; dts_search (host) streams them "
+                                "in query chunks"),
+          total(t) {}
+};
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
-                   uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats);
+                   uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
+                   unsigned long long max_results = ~0ull);
 }  // namespace dts

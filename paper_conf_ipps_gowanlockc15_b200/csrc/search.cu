@@ -42,8 +42,6 @@ namespace {
 constexpr int TQ = 16;                  // queries per warp tile (WQ of wtile.cuh)
 constexpr int PT = 256;                 // threads per CTA in warp-per-query kernels
 constexpr int PW = PT / 32;
-constexpr int SMALL_SORT = 32;          // warp-register sort limit
-constexpr int LARGE_SORT = 4096;        // CTA shared-memory sort limit
 constexpr unsigned long long NONE = ~0ull;
 
 enum : uint32_t { MODE_DEAD = 0, MODE_GRID = 1, MODE_TEMPORAL = 2 };
@@ -53,7 +51,6 @@ struct Counters {                       // device-side statistics / flags
     unsigned long long lookups;
     unsigned long long staged;          // staging slots reserved
     unsigned int max_count;
-    unsigned int n_large;
     unsigned int n_over;                // tiles recomputed in pass 2
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
@@ -433,119 +430,46 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
 }
 
 // ------------------------------------------------------ canonical order
-// Fallback tiles: one warp per query with 2..32 results, bitonic sort by
-// entry id across lanes (entry ids of one query are distinct).
-__global__ void __launch_bounds__(PT) k_canon_small(const uint32_t* __restrict__ tiles,
-                                                   const uint32_t* __restrict__ order, uint32_t nq,
-                                                   const uint32_t* __restrict__ counts,
-                                                   const unsigned long long* __restrict__ offsets,
-                                                   const dts_result* __restrict__ raw,
-                                                   dts_result* __restrict__ out) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    constexpr int CTAS_PER_TILE = TQ / PW;
-    const uint32_t tile = tiles[blockIdx.x / CTAS_PER_TILE];
-    const uint32_t sq = tile * TQ + (blockIdx.x % CTAS_PER_TILE) * PW + warp;
-    if (sq >= nq) return;
-    const uint32_t q = order[sq];
-    const uint32_t cnt = counts[q];
-    if (cnt == 0 || cnt > (uint32_t)SMALL_SORT) return;
-    const unsigned long long base = offsets[q];
-    if (cnt == 1) {
-        if (lane == 0) out[base] = raw[base];
-        return;
-    }
-    uint32_t key = 0xffffffffu, qq = 0;
-    double t0 = 0.0, t1 = 0.0;
-    if ((uint32_t)lane < cnt) {
-        const dts_result r = raw[base + lane];
-        key = r.entry_id;
-        qq = r.query_id;
-        t0 = r.t_start;
-        t1 = r.t_end;
-    }
-#pragma unroll
-    for (int k = 2; k <= 32; k <<= 1) {
-#pragma unroll
-        for (int j = k >> 1; j > 0; j >>= 1) {
-            const uint32_t ok = __shfl_xor_sync(0xffffffffu, key, j);
-            const double o0 = __shfl_xor_sync(0xffffffffu, t0, j);
-            const double o1 = __shfl_xor_sync(0xffffffffu, t1, j);
-            const bool up = ((lane & k) == 0);
-            const bool lower = ((lane & j) == 0);
-            const bool take = lower == up ? (ok < key) : (ok > key);
-            if (take) {
-                key = ok;
-                t0 = o0;
-                t1 = o1;
-            }
-        }
-    }
-    qq = __shfl_sync(0xffffffffu, qq, 0);
-    if ((uint32_t)lane < cnt) {
-        dts_result r;
-        r.query_id = qq;
-        r.entry_id = key;
-        r.t_start = t0;
-        r.t_end = t1;
-        out[base + lane] = r;
+// Fallback tiles (staging overflowed): their queries' results were written
+// by k_pass_scatter into a compact buffer, query q at cover_off[q] .. + count
+// (cover_off = exclusive scan, in query-id order, of the counts of those
+// queries only).  One device-wide stable radix sort by (query, entry id)
+// puts them in canonical order; k_place_over copies each to its exact final
+// offset.  Cost is linear in the number of such results.
+__global__ void __launch_bounds__(PT) k_mark_over(const uint32_t* __restrict__ tiles,
+                                                 const uint32_t* __restrict__ order, uint32_t nq,
+                                                 const uint32_t* __restrict__ counts,
+                                                 uint32_t* __restrict__ cover) {
+    const uint32_t tile = tiles[blockIdx.x];
+    const uint32_t sp = tile * TQ + threadIdx.x;
+    if (threadIdx.x < (unsigned)TQ && sp < nq) {
+        const uint32_t q = order[sp];
+        cover[q] = counts[q];
     }
 }
 
-// One CTA per query with 33..LARGE_SORT results: bitonic sort of
-// (entry id << 32 | local index) in shared memory, then gather.
-__global__ void __launch_bounds__(PT) k_canon_large(const uint32_t* __restrict__ large,
-                                                   const Counters* __restrict__ ctr,
-                                                   const uint32_t* __restrict__ counts,
-                                                   const unsigned long long* __restrict__ offsets,
-                                                   const dts_result* __restrict__ raw,
-                                                   dts_result* __restrict__ out) {
-    __shared__ unsigned long long sk[LARGE_SORT];
-    const uint32_t nl = ctr->n_large;
-    for (uint32_t i = blockIdx.x; i < nl; i += gridDim.x) {
-        const uint32_t q = large[i];
-        const uint32_t cnt = counts[q];
-        if (cnt > (uint32_t)LARGE_SORT) continue;     // host path
-        const unsigned long long base = offsets[q];
-        uint32_t P = 64;
-        while (P < cnt) P <<= 1;
-        for (uint32_t j = threadIdx.x; j < P; j += PT)
-            sk[j] = j < cnt ? ((unsigned long long)raw[base + j].entry_id << 32) | j : ~0ull;
-        __syncthreads();
-        for (uint32_t k = 2; k <= P; k <<= 1) {
-            for (uint32_t jj = k >> 1; jj > 0; jj >>= 1) {
-                for (uint32_t t = threadIdx.x; t < P; t += PT) {
-                    const uint32_t u = t ^ jj;
-                    if (u > t) {
-                        const unsigned long long x = sk[t], y = sk[u];
-                        const bool up = (t & k) == 0;
-                        if ((x > y) == up) {
-                            sk[t] = y;
-                            sk[u] = x;
-                        }
-                    }
-                }
-                __syncthreads();
-            }
-        }
-        for (uint32_t j = threadIdx.x; j < cnt; j += PT)
-            out[base + j] = raw[base + (uint32_t)(sk[j] & 0xffffffffull)];
-        __syncthreads();
-    }
+__global__ void __launch_bounds__(PT) k_keys_over(const dts_result* __restrict__ raw,
+                                                 unsigned long long n, uint32_t qid_base,
+                                                 unsigned long long* __restrict__ keys,
+                                                 uint32_t* __restrict__ vals) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
+    if (k >= n) return;
+    const dts_result r = raw[k];
+    keys[k] = ((unsigned long long)(r.query_id - qid_base) << 32) | r.entry_id;
+    vals[k] = (uint32_t)k;
 }
 
-// Huge segments (> LARGE_SORT results of one query): radix sort by entry id.
-__global__ void k_seg_keys(const dts_result* __restrict__ raw, uint32_t cnt,
-                           unsigned long long* __restrict__ keys, uint32_t* __restrict__ idx) {
-    uint32_t j = blockIdx.x * PT + threadIdx.x;
-    if (j < cnt) {
-        keys[j] = raw[j].entry_id;
-        idx[j] = j;
-    }
-}
-__global__ void k_seg_gather(const dts_result* __restrict__ raw, uint32_t cnt,
-                             const uint32_t* __restrict__ idx, dts_result* __restrict__ out) {
-    uint32_t j = blockIdx.x * PT + threadIdx.x;
-    if (j < cnt) out[j] = raw[idx[j]];
+__global__ void __launch_bounds__(PT) k_place_over(const unsigned long long* __restrict__ keys,
+                                                  const uint32_t* __restrict__ vals,
+                                                  unsigned long long n,
+                                                  const unsigned long long* __restrict__ cover_off,
+                                                  const unsigned long long* __restrict__ offsets,
+                                                  const dts_result* __restrict__ raw,
+                                                  dts_result* __restrict__ out) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
+    if (k >= n) return;
+    const uint32_t q = (uint32_t)(keys[k] >> 32);
+    out[offsets[q] + (k - cover_off[q])] = raw[vals[k]];
 }
 
 __global__ void k_validate_only(const double4* __restrict__ Q, uint32_t nq, Counters* ctr) {
@@ -581,7 +505,8 @@ struct EventTimer {
 }  // namespace
 
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
-                   uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats) {
+                   uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
+                   unsigned long long max_results) {
     out->results = nullptr;
     out->count = 0;
     dts_search_stats local{};
@@ -621,7 +546,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // ---- pass 1: warp tiles, count + staging
     const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
     const unsigned long long stage_cap = 4ull * nq + (1ull << 20);
-    DevBuf<uint32_t> counts(nq, s), large(nq, s), over_tiles(ntiles, s);
+    DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s);
     DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s);
     DevBuf<dts_result> stage(stage_cap, s);
     TileArgs ta;
@@ -640,7 +565,6 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.stage_cap = stage_cap;
     ta.tile_base = tile_base.p;
     ta.over_tiles = over_tiles.p;
-    ta.large = large.p;
     ta.qid_base = qid_base;
     ta.ctr = ctr.p;
     ta.method = idx->method;
@@ -681,6 +605,24 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     local.results = h.total;
     local.max_results_per_query = h.c.max_count;
 
+    // ---- results that do not fit the device: report the per-query counts
+    //      so a host caller can stream the search in query chunks
+    if (h.total > 0) {
+        size_t free_b = 0, total_b = 0;
+        DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
+        stage.release();
+        const double per = h.c.n_over ? 24.0 + 48.0 : 24.0;   // fin (+ raw, keys, vals, tmp)
+        if ((double)h.total * per > 0.8 * (double)free_b + 0.5 * (double)stage_cap * 24.0 ||
+            h.total > max_results) {
+            ResultsTooLarge e(h.total);
+            e.counts.resize(nq);
+            DTS_CUDA(cudaMemcpyAsync(e.counts.data(), counts.p, nq * sizeof(uint32_t),
+                                     cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaStreamSynchronize(s));
+            throw e;
+        }
+    }
+
     if (h.total > 0) {
         dts_result* fin = nullptr;
         fin = static_cast<dts_result*>(cache_alloc(h.total * sizeof(dts_result)));
@@ -690,9 +632,21 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                                                              offsets.p, tile_base.p, stage.p,
                                                              fin);
             DTS_LAUNCH_CHECK();
-            // ---- overflowed tiles: recompute with exact offsets, then sort
+            // ---- overflowed tiles: recompute (count-then-scatter) into a
+            //      compact buffer, then one radix sort by (query, entry id)
             if (h.c.n_over) {
-                DevBuf<dts_result> raw(h.total, s);
+                DevBuf<uint32_t> cover(nq, s);
+                DevBuf<unsigned long long> cover_off(nq + 1, s);
+                DTS_CUDA(cudaMemsetAsync(cover.p, 0, nq * sizeof(uint32_t), s));
+                k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq,
+                                                      counts.p, cover.p);
+                DTS_LAUNCH_CHECK();
+                scan_exclusive_u32_to_u64(cover.p, cover_off.p, nq, s);
+                unsigned long long n_raw = 0;
+                DTS_CUDA(cudaMemcpyAsync(&n_raw, cover_off.p + nq, sizeof(n_raw),
+                                         cudaMemcpyDeviceToHost, s));
+                DTS_CUDA(cudaStreamSynchronize(s));
+                DevBuf<dts_result> raw(n_raw, s);
                 PassArgs pa;
                 pa.Q = Q;
                 pa.order = order.p;
@@ -704,7 +658,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 pa.bin_t0min = idx->bin_t0min;
                 pa.bin_t1max = idx->bin_t1max;
                 pa.bin_start = idx->bin_start;
-                pa.offsets = offsets.p;
+                pa.offsets = cover_off.p;          // compact positions
                 pa.tiles = over_tiles.p;
                 pa.out = raw.p;
                 pa.qid_base = qid_base;
@@ -714,39 +668,16 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 k_pass_scatter<<<nb, PT, 0, s>>>(pa);
                 DTS_LAUNCH_CHECK();
                 tm.mark();
-                k_canon_small<<<nb, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq, counts.p,
-                                                offsets.p, raw.p, fin);
+                if (n_raw >= (1ull << 32))
+                    throw Error(DTS_ENOTSUP, "more than 2^32 results in recomputed tiles");
+                DevBuf<unsigned long long> k1(n_raw, s), k2(n_raw, s);
+                DevBuf<uint32_t> v1(n_raw, s), v2(n_raw, s);
+                k_keys_over<<<blocks(n_raw, PT), PT, 0, s>>>(raw.p, n_raw, qid_base, k1.p, v1.p);
                 DTS_LAUNCH_CHECK();
-                if (h.c.n_large) {
-                    const unsigned gl = (unsigned)std::min<uint32_t>(h.c.n_large, 148 * 4);
-                    k_canon_large<<<gl, PT, 0, s>>>(large.p, ctr.p, counts.p, offsets.p, raw.p,
-                                                    fin);
-                    DTS_LAUNCH_CHECK();
-                }
-                if (h.c.max_count > (uint32_t)LARGE_SORT && h.c.n_large) {
-                    std::vector<uint32_t> hl(h.c.n_large);
-                    DTS_CUDA(cudaMemcpyAsync(hl.data(), large.p, hl.size() * sizeof(uint32_t),
-                                             cudaMemcpyDeviceToHost, s));
-                    DTS_CUDA(cudaStreamSynchronize(s));
-                    for (uint32_t qh : hl) {
-                        uint32_t cnt;
-                        unsigned long long base;
-                        DTS_CUDA(cudaMemcpyAsync(&cnt, counts.p + qh, 4, cudaMemcpyDeviceToHost, s));
-                        DTS_CUDA(cudaMemcpyAsync(&base, offsets.p + qh, 8, cudaMemcpyDeviceToHost,
-                                                 s));
-                        DTS_CUDA(cudaStreamSynchronize(s));
-                        if (cnt <= (uint32_t)LARGE_SORT) continue;
-                        DevBuf<unsigned long long> k1(cnt, s), k2(cnt, s);
-                        DevBuf<uint32_t> v1(cnt, s), v2(cnt, s);
-                        k_seg_keys<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, k1.p, v1.p);
-                        DTS_LAUNCH_CHECK();
-                        radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, cnt,
-                                         bits_for(idx->n ? idx->n - 1 : 0), s);
-                        k_seg_gather<<<blocks(cnt, PT), PT, 0, s>>>(raw.p + base, cnt, v1.p,
-                                                                    fin + base);
-                        DTS_LAUNCH_CHECK();
-                    }
-                }
+                radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, n_raw, 32 + bits_for(nq - 1), s);
+                k_place_over<<<blocks(n_raw, PT), PT, 0, s>>>(k1.p, v1.p, n_raw, cover_off.p,
+                                                             offsets.p, raw.p, fin);
+                DTS_LAUNCH_CHECK();
             } else {
                 tm.mark();
             }

@@ -48,7 +48,6 @@ struct TileArgs {
     unsigned long long stage_cap;
     unsigned long long* tile_base;     // per warp tile: first staged slot, NONE-1 empty, NONE redo
     uint32_t* over_tiles;              // tiles to recompute in pass 2
-    uint32_t* large;                   // query ids (recomputed tiles) with count > SMALL_SORT
     uint32_t qid_base;
     Counters* ctr;
     uint32_t method;
@@ -248,10 +247,6 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 a.tile_base[wt] = NONE;
                 const uint32_t slot = atomicAdd(&a.ctr->n_over, 1u);
                 a.over_tiles[slot] = wt;
-            }
-            if (lane < WQ && sp < a.nq && cnt > (uint32_t)SMALL_SORT) {
-                const uint32_t slot = atomicAdd(&a.ctr->n_large, 1u);
-                a.large[slot] = S.qid[lane];
             }
         }
         __syncwarp();

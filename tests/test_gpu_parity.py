@@ -261,3 +261,36 @@ def test_subbin_c1_sampled(dts, oracle_mod):
         got = dts.search(idx, c.Q, d)
         ora = oracle_mod.search_queries(c.D, c.Q, qs, d, threads=THREADS)
         parity.compare(parity.restrict(got, qs), ora, c.D, c.Q, d, oracle_mod)
+
+
+def test_streamed_host_search_matches(dts, oracle_mod, monkeypatch):
+    """Results larger than the device budget are streamed in query chunks by
+    dts_search (host); forced here with DTS_MAX_DEVICE_RESULTS."""
+    c = synth.make_config("C2", scale=0.004)
+    idx = dts.build_index(c.D)
+    ref = dts.search(idx, c.Q, 2.0)
+    assert ref.shape[0] > 500
+    monkeypatch.setenv("DTS_MAX_DEVICE_RESULTS", str(ref.shape[0] // 7))
+    got, st = dts.search_ex(idx, c.Q, 2.0)
+    assert got.tobytes() == ref.tobytes()
+    assert st["results"] == ref.shape[0]
+    # the device API refuses instead of streaming
+    import torch
+    monkeypatch.setenv("DTS_MAX_DEVICE_RESULTS", "0")
+    res, _ = dts.search_device(idx, torch.from_numpy(c.Q).cuda(), 2.0)
+    assert res.count == ref.shape[0]
+
+
+def test_heavy_output_recompute_path(dts, oracle_mod):
+    """Tiles whose hits overflow the staging (many results per query) take the
+    count-then-scatter recompute + radix canonicalisation path."""
+    g = synth.rng(91)
+    n = 3000
+    D = np.zeros((n, 8))
+    D[:, 0], D[:, 4] = 0.0, 1.0
+    D[:, 1:4] = g.uniform(0, 0.02, size=(n, 3))
+    D[:, 5:8] = D[:, 1:4] + g.uniform(-0.01, 0.01, size=(n, 3))
+    Q = D[g.choice(n, size=40, replace=False)].copy()
+    for d in (0.01, 0.05):
+        got, info = run_and_compare(dts, oracle_mod, D, Q, d)
+        assert info["common"] > 1000
