@@ -81,11 +81,18 @@ def main():
                     built[key] = idx
                     build_s = time.perf_counter() - t0
                 idx = built[key]
-                ms, st, nres = timed_search(idx, Qd, d, a.reps)
+                try:
+                    ms, st, nres = timed_search(idx, Qd, d, a.reps)
+                except dts.DTSError as e:        # results exceed device memory
+                    ms, st, nres = None, {"candidates": None, "cell_lookups": None,
+                                          "ms_count": None, "ms_prep": None}, None
+                    print(f"# device search skipped: {e}", flush=True)
                 rt = response_time(idx, c.Q, d)
+                if nres is None:
+                    nres = int(dts.search(idx, c.Q, d).shape[0])
                 rec = {"config": name, "method": method, "d": d, "n": int(c.D.shape[0]),
                        "nq": int(c.Q.shape[0]), "search_ms_device": ms,
-                       "qseg_per_s_device": c.Q.shape[0] / (ms * 1e-3),
+                       "qseg_per_s_device": c.Q.shape[0] / (ms * 1e-3) if ms else None,
                        "response_time_s": rt, "qseg_per_s_response": c.Q.shape[0] / rt,
                        "results": nres, "candidates": st["candidates"],
                        "cell_probes": st["cell_lookups"], "ms_count_pass": st["ms_count"],

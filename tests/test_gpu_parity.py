@@ -274,7 +274,7 @@ def test_streamed_host_search_matches(dts, oracle_mod, monkeypatch):
     got, st = dts.search_ex(idx, c.Q, 2.0)
     assert got.tobytes() == ref.tobytes()
     assert st["results"] == ref.shape[0]
-    # the device API refuses instead of streaming
+    # the cap applies to the host API only; the device API returns everything
     import torch
     monkeypatch.setenv("DTS_MAX_DEVICE_RESULTS", "0")
     res, _ = dts.search_device(idx, torch.from_numpy(c.Q).cuda(), 2.0)
