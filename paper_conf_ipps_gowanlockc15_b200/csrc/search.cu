@@ -610,10 +610,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     if (h.total > 0) {
         size_t free_b = 0, total_b = 0;
         DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
-        stage.release();
         const double per = h.c.n_over ? 24.0 + 48.0 : 24.0;   // fin (+ raw, keys, vals, tmp)
-        if ((double)h.total * per > 0.8 * (double)free_b + 0.5 * (double)stage_cap * 24.0 ||
-            h.total > max_results) {
+        if ((double)h.total * per > 0.8 * (double)free_b || h.total > max_results) {
             ResultsTooLarge e(h.total);
             e.counts.resize(nq);
             DTS_CUDA(cudaMemcpyAsync(e.counts.data(), counts.p, nq * sizeof(uint32_t),
