@@ -607,10 +607,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 
     // ---- results that do not fit the device: report the per-query counts
     //      so a host caller can stream the search in query chunks
-    if (h.total > 0) {
+    const double per = h.c.n_over ? 24.0 + 48.0 : 24.0;   // fin (+ raw, keys, vals, tmp)
+    // (cudaMemGetInfo is slow and jittery -- ms -- so it is asked only when
+    //  the results are large enough to matter)
+    if (h.total > 0 && ((double)h.total * per > 1e9 || h.total > max_results)) {
         size_t free_b = 0, total_b = 0;
         DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
-        const double per = h.c.n_over ? 24.0 + 48.0 : 24.0;   // fin (+ raw, keys, vals, tmp)
         if ((double)h.total * per > 0.8 * (double)free_b || h.total > max_results) {
             ResultsTooLarge e(h.total);
             e.counts.resize(nq);
