@@ -90,6 +90,10 @@ typedef struct {
     uint32_t subbins;           /* v of P:L87 per dimension (SUBBIN); 0 = 16, always
                                    capped so a subbin is wider than the largest
                                    entry extent in that dimension             */
+    const uint32_t* entry_ids;  /* optional: id reported for row i of D (a shard of a
+                                   larger database reports global ids); host memory
+                                   for dts_build_index, device memory for
+                                   dts_build_index_device; NULL = i                   */
 } dts_index_params;
 
 /* Per-search statistics (optional output of the *_ex entry points). */
@@ -148,6 +152,20 @@ dts_status dts_search_device(const dts_index* index,
                              uint32_t query_id_base, void* cuda_stream,
                              dts_result** out_results_dev, size_t* out_count,
                              dts_search_stats* stats);            /* may be NULL */
+
+/* As dts_search_device, but the query id reported for row i of Q_dev is
+ * query_ids[i] (device memory, nq entries; NULL = i).  query_ids must be
+ * increasing for the output to stay in canonical (query_id, entry_id) order
+ * (e.g. the rows of a larger query set routed to one shard). */
+dts_status dts_search_device_ex(const dts_index* index,
+                                const dts_segment* Q_dev, size_t nq, double d,
+                                const uint32_t* query_ids, void* cuda_stream,
+                                dts_result** out_results_dev, size_t* out_count,
+                                dts_search_stats* stats);         /* may be NULL */
+
+/* Sort n results in device memory into canonical (query_id, entry_id) order,
+ * in place (e.g. after concatenating the outputs of shards of D). */
+dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream);
 
 void dts_free_results(dts_result* results);          /* NULL is a no-op */
 void dts_free_results_device(dts_result* results);   /* NULL is a no-op */

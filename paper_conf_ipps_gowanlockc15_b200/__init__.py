@@ -30,6 +30,7 @@ EXPORTED_SYMBOLS = (
     "dts_build_index", "dts_build_index_device", "dts_search", "dts_search_ex",
     "dts_search_device", "dts_free_results", "dts_free_results_device", "dts_free_index",
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
+    "dts_search_device_ex", "dts_canonicalize_device",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -46,7 +47,7 @@ class IndexParams(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("temporal_bins", ctypes.c_uint32),
                 ("cells_per_dim", ctypes.c_uint32), ("d_hint", ctypes.c_double),
                 ("mem_budget_bytes", ctypes.c_uint64), ("method", ctypes.c_uint32),
-                ("subbins", ctypes.c_uint32)]
+                ("subbins", ctypes.c_uint32), ("entry_ids", ctypes.c_void_p)]
 
 
 METHODS = {"grid": 0, "temporal": 1, "subbin": 2}
@@ -104,6 +105,11 @@ def load():
     lib.dts_search.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps]
     lib.dts_search_ex.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
                                   ctypes.POINTER(SearchStats)]
+    lib.dts_search_device_ex.argtypes = [P, P, S, ctypes.c_double, P, P, pp, ps,
+                                         ctypes.POINTER(SearchStats)]
+    lib.dts_search_device_ex.restype = ctypes.c_int
+    lib.dts_canonicalize_device.argtypes = [P, S, P]
+    lib.dts_canonicalize_device.restype = ctypes.c_int
     lib.dts_search_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
                                       ctypes.POINTER(SearchStats)]
     for f in ("dts_build_index", "dts_build_index_device", "dts_search", "dts_search_ex",
@@ -139,10 +145,10 @@ def _segments(a) -> np.ndarray:
 
 
 def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0, method="grid",
-            subbins=0) -> IndexParams:
+            subbins=0, entry_ids_ptr=None) -> IndexParams:
     m = METHODS[method] if isinstance(method, str) else int(method)
     return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0,
-                       m, int(subbins))
+                       m, int(subbins), entry_ids_ptr)
 
 
 def _stream_ptr(stream) -> int:
@@ -220,11 +226,19 @@ class DeviceResults:
 
 
 def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int = 0,
-                d_hint: float = 0.0, method="grid", subbins: int = 0) -> Index:
-    """dts_build_index: D is host (n, 8) float64 (copied)."""
+                d_hint: float = 0.0, method="grid", subbins: int = 0,
+                entry_ids=None) -> Index:
+    """dts_build_index: D is host (n, 8) float64 (copied); entry_ids: optional
+    host uint32 ids reported for the rows of D."""
     lib = load()
     D = _segments(D)
-    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins)
+    ids = None
+    if entry_ids is not None:
+        ids = np.ascontiguousarray(entry_ids, dtype=np.uint32)
+        if ids.shape[0] != D.shape[0]:
+            raise ValueError("entry_ids must have one id per row of D")
+    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins,
+                ids.ctypes.data if ids is not None else None)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index(D.ctypes.data if D.size else None, D.shape[0], ctypes.byref(p),
                                ctypes.byref(h)))
@@ -233,13 +247,17 @@ def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int =
 
 def build_index_device(D_dev, n: int = None, device: int = 0, temporal_bins: int = 0,
                        cells_per_dim: int = 0, d_hint: float = 0.0, stream=None,
-                       method="grid", subbins: int = 0) -> Index:
-    """dts_build_index_device: D_dev is a CUDA tensor (n, 8) float64."""
+                       method="grid", subbins: int = 0, entry_ids=None) -> Index:
+    """dts_build_index_device: D_dev is a CUDA tensor (n, 8) float64;
+    entry_ids: optional CUDA int32/uint32 tensor of reported ids."""
     lib = load()
     ptr = D_dev.data_ptr() if hasattr(D_dev, "data_ptr") else int(D_dev)
     if n is None:
         n = D_dev.shape[0]
-    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins)
+    eptr = None
+    if entry_ids is not None:
+        eptr = entry_ids.data_ptr() if hasattr(entry_ids, "data_ptr") else int(entry_ids)
+    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins, eptr)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index_device(ctypes.c_void_p(ptr), n, ctypes.byref(p),
                                       ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(h)))
@@ -283,8 +301,10 @@ def search(index: Index, Q, d: float, query_id_base: int = 0, stream=None) -> np
 
 
 def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=None,
-                  n: int = None, time_kernels: bool = False):
-    """dts_search_device: Q_dev CUDA tensor (nq, 8) float64 -> (DeviceResults, stats)."""
+                  n: int = None, time_kernels: bool = False, query_ids=None):
+    """dts_search_device (dts_search_device_ex when query_ids, a CUDA int32 /
+    uint32 tensor of increasing reported ids, is given): Q_dev CUDA tensor
+    (nq, 8) float64 -> (DeviceResults, stats)."""
     lib = load()
     ptr = Q_dev.data_ptr() if hasattr(Q_dev, "data_ptr") else int(Q_dev)
     if n is None:
@@ -293,10 +313,31 @@ def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=
     cnt = ctypes.c_size_t()
     st = SearchStats()
     st.time_kernels = 1 if time_kernels else 0
-    _check(lib.dts_search_device(index.handle, ctypes.c_void_p(ptr), n, float(d),
-                                 int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
-                                 ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
+    if query_ids is None:
+        _check(lib.dts_search_device(index.handle, ctypes.c_void_p(ptr), n, float(d),
+                                     int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
+                                     ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
+    else:
+        qptr = query_ids.data_ptr() if hasattr(query_ids, "data_ptr") else int(query_ids)
+        _check(lib.dts_search_device_ex(index.handle, ctypes.c_void_p(ptr), n, float(d),
+                                        ctypes.c_void_p(qptr),
+                                        ctypes.c_void_p(_stream_ptr(stream)),
+                                        ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     return DeviceResults(out.value or 0, cnt.value, index.device), st.as_dict()
+
+
+def canonicalize_device(results_dev, n: int = None, stream=None) -> None:
+    """dts_canonicalize_device: sort results in device memory (a CUDA uint8
+    tensor of n * 24 bytes, or a DeviceResults) by (query_id, entry_id)."""
+    lib = load()
+    if isinstance(results_dev, DeviceResults):
+        ptr, n = results_dev.ptr, results_dev.count
+    else:
+        ptr = results_dev.data_ptr()
+        if n is None:
+            n = results_dev.numel() // RESULT_DTYPE.itemsize
+    _check(lib.dts_canonicalize_device(ctypes.c_void_p(ptr or 0), int(n),
+                                       ctypes.c_void_p(_stream_ptr(stream))))
 
 
 def kernel_launches() -> int:

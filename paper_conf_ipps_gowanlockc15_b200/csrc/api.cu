@@ -169,7 +169,13 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
         if (n == 0) return;
         if (host) {
             DevBuf<dts_segment> dD(n, s);
+            DevBuf<uint32_t> dmap(p.entry_ids ? n : 0, s);
             DTS_CUDA(cudaMemcpyAsync(dD.p, D, n * sizeof(dts_segment), cudaMemcpyHostToDevice, s));
+            if (p.entry_ids) {
+                DTS_CUDA(cudaMemcpyAsync(dmap.p, p.entry_ids, n * sizeof(uint32_t),
+                                         cudaMemcpyHostToDevice, s));
+                p.entry_ids = dmap.p;
+            }
             build_index_device(idx, dD.p, n, p, s);
         } else {
             check_aligned(D, "D_dev");
@@ -241,7 +247,8 @@ dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_
 
 dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
                          uint32_t qid_base, cudaStream_t s, bool host, dts_result** out_results,
-                         size_t* out_count, dts_search_stats* stats) {
+                         size_t* out_count, dts_search_stats* stats,
+                         const uint32_t* qmap = nullptr) {
     if (out_results) *out_results = nullptr;
     if (out_count) *out_count = 0;
     dts_result* ret = nullptr;
@@ -295,7 +302,7 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
             DTS_CUDA(cudaStreamSynchronize(s));
         } else {
             check_aligned(Q, "Q_dev");
-            search_device(index, Q, nq, d, qid_base, s, &so, stats);
+            search_device(index, Q, nq, d, qid_base, s, &so, stats, ~0ull, qmap);
             ret = so.results;
             cnt = so.count;
         }
@@ -338,6 +345,21 @@ dts_status dts_search_ex(const dts_index* index, const dts_segment* Q, size_t nq
                          size_t* out_count, dts_search_stats* stats) {
     return search_common(index, Q, nq, d, query_id_base, static_cast<cudaStream_t>(cuda_stream),
                          true, out_results, out_count, stats);
+}
+
+dts_status dts_search_device_ex(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                double d, const uint32_t* query_ids, void* cuda_stream,
+                                dts_result** out_results_dev, size_t* out_count,
+                                dts_search_stats* stats) {
+    return search_common(index, Q_dev, nq, d, 0, static_cast<cudaStream_t>(cuda_stream), false,
+                         out_results_dev, out_count, stats, query_ids);
+}
+
+dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream) {
+    return guarded([&] {
+        if (n > 0 && !results_dev) throw Error(DTS_EINVAL, "results_dev is NULL with n > 0");
+        canonicalize_device(results_dev, n, static_cast<cudaStream_t>(cuda_stream));
+    });
 }
 
 dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,

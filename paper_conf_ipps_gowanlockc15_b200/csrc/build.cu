@@ -335,6 +335,12 @@ __global__ void __launch_bounds__(BT) k_sb_emit(const double4* __restrict__ D,
     }
 }
 
+__global__ void __launch_bounds__(BT) k_map_ids(uint32_t* __restrict__ eid, size_t n,
+                                               const uint32_t* __restrict__ emap) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p < n) eid[p] = emap[eid[p]];
+}
+
 // dir[k] = first position of key >= k in the sorted keys, k in [0, nkeys].
 __global__ void __launch_bounds__(BT) k_sb_dir(const unsigned long long* __restrict__ keys,
                                               size_t len, unsigned long long nkeys,
@@ -541,6 +547,12 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         keys.release();
         ids.release();
         build_subbins(idx, D, n, hb, p, s);
+    }
+
+    // 8. reported entry ids of a shard (params.entry_ids, device memory here)
+    if (p.entry_ids) {
+        k_map_ids<<<grid_for(n), BT, 0, s>>>(idx->soa.eid, n, p.entry_ids);
+        DTS_LAUNCH_CHECK();
     }
 
     DTS_CUDA(cudaEventRecord(e1, s));

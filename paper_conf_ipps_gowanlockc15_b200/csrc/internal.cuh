@@ -247,5 +247,7 @@ struct ResultsTooLarge : Error {
 };
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
-                   unsigned long long max_results = ~0ull);
+                   unsigned long long max_results = ~0ull, const uint32_t* qmap = nullptr);
+// Sort results in device memory by (query_id, entry_id), in place.
+void canonicalize_device(dts_result* r, size_t n, cudaStream_t s);
 }  // namespace dts

@@ -418,7 +418,7 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
             const uint32_t bal = __ballot_sync(0xffffffffu, hit);
             if (hit) {
                 dts_result rr;
-                rr.query_id = qid + a.qid_base;
+                rr.query_id = qid;                  // local id; mapped by k_place_over
                 rr.entry_id = __ldg(a.soa.eid + p);
                 rr.t_start = r0;
                 rr.t_end = r1;
@@ -449,13 +449,13 @@ __global__ void __launch_bounds__(PT) k_mark_over(const uint32_t* __restrict__ t
 }
 
 __global__ void __launch_bounds__(PT) k_keys_over(const dts_result* __restrict__ raw,
-                                                 unsigned long long n, uint32_t qid_base,
+                                                 unsigned long long n,
                                                  unsigned long long* __restrict__ keys,
                                                  uint32_t* __restrict__ vals) {
     const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
     if (k >= n) return;
     const dts_result r = raw[k];
-    keys[k] = ((unsigned long long)(r.query_id - qid_base) << 32) | r.entry_id;
+    keys[k] = ((unsigned long long)r.query_id << 32) | r.entry_id;
     vals[k] = (uint32_t)k;
 }
 
@@ -465,11 +465,15 @@ __global__ void __launch_bounds__(PT) k_place_over(const unsigned long long* __r
                                                   const unsigned long long* __restrict__ cover_off,
                                                   const unsigned long long* __restrict__ offsets,
                                                   const dts_result* __restrict__ raw,
+                                                  const uint32_t* __restrict__ qmap,
+                                                  uint32_t qid_base,
                                                   dts_result* __restrict__ out) {
     const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
     if (k >= n) return;
     const uint32_t q = (uint32_t)(keys[k] >> 32);
-    out[offsets[q] + (k - cover_off[q])] = raw[vals[k]];
+    dts_result r = raw[vals[k]];
+    r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
+    out[offsets[q] + (k - cover_off[q])] = r;
 }
 
 __global__ void k_validate_only(const double4* __restrict__ Q, uint32_t nq, Counters* ctr) {
@@ -506,7 +510,7 @@ struct EventTimer {
 
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
-                   unsigned long long max_results) {
+                   unsigned long long max_results, const uint32_t* qmap) {
     out->results = nullptr;
     out->count = 0;
     dts_search_stats local{};
@@ -566,6 +570,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.tile_base = tile_base.p;
     ta.over_tiles = over_tiles.p;
     ta.qid_base = qid_base;
+    ta.qmap = qmap;
     ta.ctr = ctr.p;
     ta.method = idx->method;
     ta.sb = idx->sb;
@@ -672,11 +677,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     throw Error(DTS_ENOTSUP, "more than 2^32 results in recomputed tiles");
                 DevBuf<unsigned long long> k1(n_raw, s), k2(n_raw, s);
                 DevBuf<uint32_t> v1(n_raw, s), v2(n_raw, s);
-                k_keys_over<<<blocks(n_raw, PT), PT, 0, s>>>(raw.p, n_raw, qid_base, k1.p, v1.p);
+                k_keys_over<<<blocks(n_raw, PT), PT, 0, s>>>(raw.p, n_raw, k1.p, v1.p);
                 DTS_LAUNCH_CHECK();
                 radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, n_raw, 32 + bits_for(nq - 1), s);
                 k_place_over<<<blocks(n_raw, PT), PT, 0, s>>>(k1.p, v1.p, n_raw, cover_off.p,
-                                                             offsets.p, raw.p, fin);
+                                                             offsets.p, raw.p, qmap, qid_base,
+                                                             fin);
                 DTS_LAUNCH_CHECK();
             } else {
                 tm.mark();
@@ -703,6 +709,43 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         local.ms_canon = tm.ms(4);
     }
     if (stats) *stats = local;
+}
+
+namespace {
+__global__ void __launch_bounds__(PT) k_result_keys(const dts_result* __restrict__ r,
+                                                   unsigned long long n,
+                                                   unsigned long long* __restrict__ keys,
+                                                   uint32_t* __restrict__ vals) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
+    if (k >= n) return;
+    keys[k] = ((unsigned long long)r[k].query_id << 32) | r[k].entry_id;
+    vals[k] = (uint32_t)k;
+}
+__global__ void __launch_bounds__(PT) k_result_gather(const dts_result* __restrict__ r,
+                                                     const uint32_t* __restrict__ vals,
+                                                     unsigned long long n,
+                                                     dts_result* __restrict__ out) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
+    if (k < n) out[k] = r[vals[k]];
+}
+}  // namespace
+
+// Canonical (query_id, entry_id) order of an arbitrary result array, e.g.
+// the concatenated outputs of temporal shards of D: one
+// stable radix sort of the 64-bit (query, entry) keys, then a gather.
+void canonicalize_device(dts_result* r, size_t n, cudaStream_t s) {
+    if (n <= 1) return;
+    if (n >= (size_t(1) << 32)) throw Error(DTS_ENOTSUP, "more than 2^32 results to sort");
+    DevBuf<unsigned long long> k1(n, s), k2(n, s);
+    DevBuf<uint32_t> v1(n, s), v2(n, s);
+    DevBuf<dts_result> tmp(n, s);
+    k_result_keys<<<blocks(n, PT), PT, 0, s>>>(r, n, k1.p, v1.p);
+    DTS_LAUNCH_CHECK();
+    radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, n, 64, s);
+    k_result_gather<<<blocks(n, PT), PT, 0, s>>>(r, v1.p, n, tmp.p);
+    DTS_LAUNCH_CHECK();
+    DTS_CUDA(cudaMemcpyAsync(r, tmp.p, n * sizeof(dts_result), cudaMemcpyDeviceToDevice, s));
+    DTS_CUDA(cudaStreamSynchronize(s));
 }
 
 }  // namespace dts

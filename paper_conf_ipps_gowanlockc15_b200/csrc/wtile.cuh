@@ -49,6 +49,7 @@ struct TileArgs {
     unsigned long long* tile_base;     // per warp tile: first staged slot, NONE-1 empty, NONE redo
     uint32_t* over_tiles;              // tiles to recompute in pass 2
     uint32_t qid_base;
+    const uint32_t* qmap;              // optional reported query ids (else qid + qid_base)
     Counters* ctr;
     uint32_t method;
     SubbinIndex sb;
@@ -231,7 +232,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     }
                     const uint32_t slot = (uint32_t)(k & 1023ull);
                     dts_result r;
-                    r.query_id = S.qid[q] + a.qid_base;
+                    r.query_id = a.qmap ? __ldg(a.qmap + S.qid[q]) : S.qid[q] + a.qid_base;
                     r.entry_id = e;
                     r.t_start = S.h0[slot];
                     r.t_end = S.h1[slot];

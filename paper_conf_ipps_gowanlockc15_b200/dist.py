@@ -66,3 +66,87 @@ def search_sharded(search_fn, Q, d: float, rank: int, world: int, group=None, we
     res = search_fn(Q[lo:hi], d, lo)
     off, total, _ = global_offset(len(res), rank, world, group=group)
     return res, off, total
+
+
+# --------------------------------------------------------------------------
+# Fallback when D exceeds one GPU's HBM: shard D by
+# t_start range.  Rank r holds the entries with t_start in [T_r, T_{r+1});
+# each entry lives on exactly one rank, so per-rank results are disjoint and
+# their union is exact.  A query is routed to every rank whose entries it can
+# overlap strictly in time: q.t_end > T_r and q.t_start < T_{r+1} + maxdur_r.
+# Ranks report global entry ids (index built with entry_ids) and global query
+# ids (search with query_ids); rank 0 concatenates and restores canonical
+# order with one device sort (dts_canonicalize_device).
+
+def temporal_partition(D, world: int):
+    """Split D's rows by t_start quantiles.  Returns (T, rows, maxdur):
+    boundaries T[0..world] (T[0] = -inf, T[world] = +inf), the row indices of
+    each rank (ascending), and each rank's max segment duration."""
+    D = np.asarray(D).reshape(-1, 8)
+    t0 = D[:, 0]
+    srt = np.sort(t0)
+    T = [-np.inf]
+    for r in range(1, world):
+        T.append(float(srt[min(len(srt) - 1, (len(srt) * r) // world)]) if len(srt) else 0.0)
+    T.append(np.inf)
+    T = np.array(T)
+    owner = np.searchsorted(T, t0, side="right") - 1
+    rows = [np.flatnonzero(owner == r).astype(np.int64) for r in range(world)]
+    maxdur = [float((D[rr, 4] - D[rr, 0]).max()) if rr.size else 0.0 for rr in rows]
+    return T, rows, maxdur
+
+
+def route_queries(Q, T, maxdur, rank: int):
+    """Rows of Q that can strictly overlap an entry of `rank` in time (with a
+    relative 1e-9 slack against rounding of t_start + duration)."""
+    Q = np.asarray(Q).reshape(-1, 8)
+    lo, hi = T[rank], T[rank + 1]
+    slack = 1e-9 * (np.abs(hi) + maxdur[rank] + 1.0) if np.isfinite(hi) else 0.0
+    ok = (Q[:, 4] > lo) & (Q[:, 0] < hi + maxdur[rank] + slack)
+    return np.flatnonzero(ok).astype(np.int64)
+
+
+def gather_to_root(local, rank: int, world: int, group=None):
+    """All-gather variable-length uint8 tensors (padded to the largest);
+    returns the concatenation in rank order on rank 0, None elsewhere."""
+    import torch
+    import torch.distributed as dist
+    n = torch.tensor([local.numel()], dtype=torch.int64, device=local.device)
+    sizes = [torch.zeros_like(n) for _ in range(world)]
+    dist.all_gather(sizes, n, group=group)
+    sizes = [int(s.item()) for s in sizes]
+    mx = max(sizes) if sizes else 0
+    pad = torch.zeros(mx, dtype=torch.uint8, device=local.device)
+    pad[:local.numel()] = local
+    parts = [torch.zeros_like(pad) for _ in range(world)]
+    dist.all_gather(parts, pad, group=group)
+    if rank != 0:
+        return None
+    return torch.cat([p[:s] for p, s in zip(parts, sizes)])
+
+
+def search_temporal_sharded(D, Q, d: float, rank: int, world: int, group=None,
+                            method: str = "grid", device: int = 0):
+    """Temporal-range sharding of D over `world` GPUs (one rank each).
+    Returns the canonical global results (numpy) on rank 0, None elsewhere."""
+    import torch
+
+    import paper_conf_ipps_gowanlockc15_b200 as dts
+    T, rows, maxdur = temporal_partition(D, world)
+    dev = torch.device("cuda", device)
+    mine = rows[rank]
+    Dd = torch.from_numpy(np.ascontiguousarray(np.asarray(D)[mine])).to(dev)
+    ids = torch.from_numpy(mine.astype(np.int32)).to(dev)
+    qrows = route_queries(Q, T, maxdur, rank)
+    Qd = torch.from_numpy(np.ascontiguousarray(np.asarray(Q)[qrows])).to(dev)
+    qids = torch.from_numpy(qrows.astype(np.int32)).to(dev)
+    idx = dts.build_index_device(Dd, device=device, method=method, entry_ids=ids)
+    res, _ = dts.search_device(idx, Qd, d, query_ids=qids)
+    local = res.tensor().clone()
+    res.free()
+    idx.free()
+    allres = gather_to_root(local, rank, world, group)
+    if allres is None:
+        return None
+    dts.canonicalize_device(allres)
+    return allres.cpu().numpy().view(dts.RESULT_DTYPE)

@@ -75,3 +75,58 @@ def test_shard_bounds():
     assert b[0] == 0 and b[-1] == 8 and 0 < b[1] < 8
     assert b[1] == 7          # first prefix (16 of 26) reaching half the weight
     assert dts_dist.shard_bounds(0, 4) == [0, 0, 0, 0, 0]
+
+
+def _temporal_worker(rank, world, port, out_dir):
+    import torch.distributed as dist
+
+    import oracle
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    import torch
+    c = synth.make_config("C0")
+    T, rows, maxdur = dts_dist.temporal_partition(c.D, world)
+    mine = rows[rank]
+    qrows = dts_dist.route_queries(c.Q, T, maxdur, rank)
+    # the per-rank search (libdts on GPUs) is the oracle here, ids mapped back
+    r = oracle.search(c.D[mine], c.Q[qrows], c.d)
+    r["entry_id"] = mine[r["entry_id"]].astype(np.uint32)
+    r["query_id"] = qrows[r["query_id"]].astype(np.uint32)
+    local = torch.from_numpy(r.view(np.uint8).copy())
+    allres = dts_dist.gather_to_root(local, rank, world)
+    if rank == 0:
+        np.save(os.path.join(out_dir, "all.npy"), allres.numpy())
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_temporal_sharding_of_D_is_exact(tmp_path):
+    """Each entry on exactly one rank, queries routed by time: the union of
+    the per-rank results is exactly the unsharded result (no duplicates)."""
+    import torch.multiprocessing as mp
+
+    import oracle
+    world = 2
+    mp.spawn(_temporal_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world,
+             join=True)
+    c = synth.make_config("C0")
+    full = oracle.search(c.D, c.Q, c.d)
+    got = np.load(tmp_path / "all.npy").view(full.dtype)
+    keys = got["query_id"].astype(np.int64) * 2**32 + got["entry_id"]
+    order = np.argsort(keys, kind="stable")
+    assert np.unique(keys).size == keys.size                  # disjoint per rank
+    assert got[order].tobytes() == full.tobytes()
+
+
+def test_temporal_partition_properties():
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    c = synth.make_config("C0")
+    for world in (1, 2, 3, 5):
+        T, rows, maxdur = dts_dist.temporal_partition(c.D, world)
+        allrows = np.sort(np.concatenate(rows))
+        assert np.array_equal(allrows, np.arange(c.D.shape[0]))      # a partition
+        for r in range(world):
+            t0 = c.D[rows[r], 0]
+            assert np.all(t0 >= T[r]) and np.all(t0 < T[r + 1])

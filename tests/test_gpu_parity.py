@@ -294,3 +294,43 @@ def test_heavy_output_recompute_path(dts, oracle_mod):
     for d in (0.01, 0.05):
         got, info = run_and_compare(dts, oracle_mod, D, Q, d)
         assert info["common"] > 1000
+
+
+@pytest.mark.parametrize("world", [2, 3])
+def test_temporal_shards_on_one_gpu_match_unsharded(dts, world):
+    """SURVEY §4 'multi-GPU without a cluster': the temporal-range shards of D
+    searched one after another on one GPU (global ids via entry_ids /
+    query_ids), concatenated and canonicalised on the device, give the
+    unsharded result byte for byte."""
+    import torch
+
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    c = synth.make_config("C2", scale=0.004)
+    d = 0.5
+    ref = dts.search(dts.build_index(c.D), c.Q, d)
+    T, rows, maxdur = dts_dist.temporal_partition(c.D, world)
+    parts = []
+    for r in range(world):
+        Dd = torch.from_numpy(np.ascontiguousarray(c.D[rows[r]])).cuda()
+        ids = torch.from_numpy(rows[r].astype(np.int32)).cuda()
+        qrows = dts_dist.route_queries(c.Q, T, maxdur, r)
+        Qd = torch.from_numpy(np.ascontiguousarray(c.Q[qrows])).cuda()
+        qids = torch.from_numpy(qrows.astype(np.int32)).cuda()
+        idx = dts.build_index_device(Dd, entry_ids=ids)
+        res, _ = dts.search_device(idx, Qd, d, query_ids=qids)
+        parts.append(res.tensor().clone())
+        res.free()
+        idx.free()
+    allres = torch.cat(parts)
+    dts.canonicalize_device(allres)
+    got = allres.cpu().numpy().view(dts.RESULT_DTYPE)
+    assert got.tobytes() == ref.tobytes()
+
+
+def test_entry_ids_host_build(dts):
+    c = synth.make_config("C0")
+    ref = dts.search(dts.build_index(c.D), c.Q, c.d)
+    perm = np.random.default_rng(3).permutation(c.D.shape[0])
+    idx = dts.build_index(c.D[perm], entry_ids=perm.astype(np.uint32))
+    got = dts.search(idx, c.Q, c.d)
+    assert got.tobytes() == ref.tobytes()
