@@ -269,7 +269,7 @@ def run_own(args):
     ms_count = statistics.mean(s["ms_count"] for s in stats)
     ms_scatter = statistics.mean(s["ms_scatter"] for s in stats)
     ms_build = statistics.mean(s["ms_build"] for s in stats)
-    alg_bytes = st0["candidates"] * 64 + nq * (64 + 4) + st0["cell_lookups"] * 16
+    alg_bytes = st0["candidates"] * 64 + nq * (64 + 4) + st0["cell_lookups"] * 64
     achieved = alg_bytes / (ms_count * 1e-3) / 1e9
     traffic = None
     tf = os.path.join(ROOT, "profiles", "traffic.json")
@@ -336,7 +336,7 @@ def run_own(args):
                          "frac": achieved / peak, "traffic": traffic,
                          "peak_source": peak_src,
                          "algorithmic_bytes": alg_bytes,
-                         "bytes_model": "64 B per candidate + 68 B per query + 16 B per cell probe"},
+                         "bytes_model": "64 B per candidate + 68 B per query + 64 B per hash-bucket probe"},
             "clocks": clk,
             "gpu_launches": int(launches),
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
@@ -358,7 +358,7 @@ def run_own(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--steps", type=int, default=100)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--config", default="C4")
     ap.add_argument("--d", type=float, default=None)

@@ -160,8 +160,12 @@ __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, si
     for (int k = 0; k < GATHER_ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
         if (p < n) {
-            r0[k] = D[2 * (size_t)id[k]];
-            r1[k] = D[2 * (size_t)id[k] + 1];
+            // read-once rows: streaming (evict-first) loads
+            const double2* row = reinterpret_cast<const double2*>(D + 2 * (size_t)id[k]);
+            const double2 a0 = __ldcs(row), a1 = __ldcs(row + 1);
+            const double2 a2 = __ldcs(row + 2), a3 = __ldcs(row + 3);
+            r0[k] = make_double4(a0.x, a0.y, a1.x, a1.y);
+            r1[k] = make_double4(a2.x, a2.y, a3.x, a3.y);
         }
     }
 #pragma unroll
@@ -275,9 +279,14 @@ __global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restr
     while (e < n && keys[e] == k) ++e;
     const unsigned long long bmask = ht.mask >> 2;
     unsigned long long b = bucket_of(k >> 2, ht.log2cap);
+    // try the slot matching the key's position in its group first: the (up
+    // to) four x-adjacent cells sharing a home bucket then claim distinct
+    // slots without colliding on the same CAS
+    const int first = (int)(k & 3ull);
     while (true) {
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
+        for (int j = 0; j < 4; ++j) {
+            const int i = (first + j) & 3;
             CellSlot& sl = ht.slots[4 * b + i];
             const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
             if (prev == EMPTY_KEY) {
