@@ -94,7 +94,33 @@ typedef struct {
                                    larger database reports global ids); host memory
                                    for dts_build_index, device memory for
                                    dts_build_index_device; NULL = i                   */
+    const uint32_t* entry_traj; /* optional: trajectory id of row i of D ("a
+                                   segment id and a trajectory id"), needed by
+                                   exclude_same_trajectory; same memory kind as D     */
 } dts_index_params;
+
+/* Options of the *_ex searches (pointer fields: host memory for dts_search_ex,
+ * device memory for dts_search_device_ex; all may be NULL / 0). */
+typedef struct {
+    uint32_t query_id_base;     /* added to row indices when query_ids is NULL        */
+    const uint32_t* query_ids;  /* reported id of row i of Q (increasing)             */
+    const uint32_t* query_traj; /* trajectory id of row i of Q                        */
+    uint32_t exclude_same_trajectory;  /* nonzero: drop pairs whose query and entry
+                                   trajectory ids are equal -- "any OTHER stellar
+                                   trajectory" of the application; needs
+                                   query_traj and an index built with entry_traj     */
+} dts_search_options;
+
+/* One trajectory-level result (the stars within d of another star and
+ * the time intervals in which this happens): the union of the segment-level
+ * intervals of one (query trajectory, entry trajectory) pair, split into its
+ * maximal connected pieces. */
+typedef struct {
+    uint32_t query_traj;
+    uint32_t entry_traj;
+    double t_start;
+    double t_end;
+} dts_traj_result;
 
 /* Per-search statistics (optional output of the *_ex entry points). */
 typedef struct {
@@ -138,9 +164,10 @@ dts_status dts_search(const dts_index* index,
                       uint32_t query_id_base, void* cuda_stream,
                       dts_result** out_results, size_t* out_count);
 
+/* dts_search with options (host pointers in opts, may be NULL) and stats. */
 dts_status dts_search_ex(const dts_index* index,
                          const dts_segment* Q, size_t nq, double d,
-                         uint32_t query_id_base, void* cuda_stream,
+                         const dts_search_options* opts, void* cuda_stream,
                          dts_result** out_results, size_t* out_count,
                          dts_search_stats* stats);                /* may be NULL */
 
@@ -153,22 +180,35 @@ dts_status dts_search_device(const dts_index* index,
                              dts_result** out_results_dev, size_t* out_count,
                              dts_search_stats* stats);            /* may be NULL */
 
-/* As dts_search_device, but the query id reported for row i of Q_dev is
- * query_ids[i] (device memory, nq entries; NULL = i).  query_ids must be
- * increasing for the output to stay in canonical (query_id, entry_id) order
- * (e.g. the rows of a larger query set routed to one shard). */
+/* dts_search_device with options (device pointers in opts, may be NULL).
+ * With opts->query_ids the id reported for row i of Q_dev is query_ids[i];
+ * they must be increasing for the output to stay in canonical order (e.g. the
+ * rows of a larger query set routed to one shard of D). */
 dts_status dts_search_device_ex(const dts_index* index,
                                 const dts_segment* Q_dev, size_t nq, double d,
-                                const uint32_t* query_ids, void* cuda_stream,
+                                const dts_search_options* opts, void* cuda_stream,
                                 dts_result** out_results_dev, size_t* out_count,
                                 dts_search_stats* stats);         /* may be NULL */
+
+/* Trajectory-level results from segment-level ones, all in device memory:
+ * every result (q, l, [t_s, t_e]) is mapped to (query_traj[q], entry_traj[l])
+ * (query_traj indexed by reported query id, n_query_ids entries; entry_traj by
+ * entry id, n_entry_ids entries); the intervals of each trajectory pair are
+ * merged into their union's maximal connected pieces (closed intervals that
+ * touch merge).  Output sorted by (query_traj, entry_traj, t_start) in
+ * library-owned device memory (dts_free_results_device). */
+dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n,
+                                         const uint32_t* query_traj, size_t n_query_ids,
+                                         const uint32_t* entry_traj, size_t n_entry_ids,
+                                         void* cuda_stream,
+                                         dts_traj_result** out_dev, size_t* out_count);
 
 /* Sort n results in device memory into canonical (query_id, entry_id) order,
  * in place (e.g. after concatenating the outputs of shards of D). */
 dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream);
 
 void dts_free_results(dts_result* results);          /* NULL is a no-op */
-void dts_free_results_device(dts_result* results);   /* NULL is a no-op */
+void dts_free_results_device(void* results);         /* NULL is a no-op; also for dts_traj_result */
 void dts_free_index(dts_index* index);               /* NULL is a no-op */
 
 /* Introspection of a built index (for tests and benchmarks). */

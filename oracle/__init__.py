@@ -157,3 +157,31 @@ def compare(q, l, d: float):
                                 np.asarray(q, dtype=np.float64).reshape(1, 8),
                                 [0], [0], d)
     return (float(ts[0]), float(te[0])) if hit[0] else None
+
+
+def merge_trajectory_pairs(res, query_traj, entry_traj) -> np.ndarray:
+    """Trajectory-level results (the application of P:L15): map each
+    segment-level result (q, l, [ts, te]) to (query_traj[q], entry_traj[l])
+    and replace the intervals of each pair by the maximal connected pieces of
+    their union (closed intervals: touching ones merge).  Plain loops; sorted
+    by (query_traj, entry_traj, t_start)."""
+    qt = np.asarray(query_traj, dtype=np.int64)[res["query_id"].astype(np.int64)]
+    et = np.asarray(entry_traj, dtype=np.int64)[res["entry_id"].astype(np.int64)]
+    groups = {}
+    for a, b, s, e in zip(qt.tolist(), et.tolist(), res["t_start"].tolist(),
+                          res["t_end"].tolist()):
+        groups.setdefault((a, b), []).append((s, e))
+    out = []
+    for (a, b) in sorted(groups):
+        iv = sorted(groups[(a, b)])
+        lo, hi = iv[0]
+        for s, e in iv[1:]:
+            if s <= hi:
+                hi = max(hi, e)
+            else:
+                out.append((a, b, lo, hi))
+                lo, hi = s, e
+        out.append((a, b, lo, hi))
+    dt = np.dtype([("query_traj", "<u4"), ("entry_traj", "<u4"), ("t_start", "<f8"),
+                   ("t_end", "<f8")], align=True)
+    return np.array(out, dtype=dt)

@@ -30,7 +30,7 @@ EXPORTED_SYMBOLS = (
     "dts_build_index", "dts_build_index_device", "dts_search", "dts_search_ex",
     "dts_search_device", "dts_free_results", "dts_free_results_device", "dts_free_index",
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
-    "dts_search_device_ex", "dts_canonicalize_device",
+    "dts_search_device_ex", "dts_canonicalize_device", "dts_merge_trajectories_device",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -47,10 +47,19 @@ class IndexParams(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("temporal_bins", ctypes.c_uint32),
                 ("cells_per_dim", ctypes.c_uint32), ("d_hint", ctypes.c_double),
                 ("mem_budget_bytes", ctypes.c_uint64), ("method", ctypes.c_uint32),
-                ("subbins", ctypes.c_uint32), ("entry_ids", ctypes.c_void_p)]
+                ("subbins", ctypes.c_uint32), ("entry_ids", ctypes.c_void_p),
+                ("entry_traj", ctypes.c_void_p)]
+
+
+class SearchOptions(ctypes.Structure):
+    _fields_ = [("query_id_base", ctypes.c_uint32), ("query_ids", ctypes.c_void_p),
+                ("query_traj", ctypes.c_void_p), ("exclude_same_trajectory", ctypes.c_uint32)]
 
 
 METHODS = {"grid": 0, "temporal": 1, "subbin": 2}
+
+TRAJ_DTYPE = np.dtype([("query_traj", "<u4"), ("entry_traj", "<u4"),
+                       ("t_start", "<f8"), ("t_end", "<f8")], align=True)
 
 
 class SearchStats(ctypes.Structure):
@@ -103,10 +112,13 @@ def load():
     lib.dts_build_index.argtypes = [P, S, ctypes.POINTER(IndexParams), pp]
     lib.dts_build_index_device.argtypes = [P, S, ctypes.POINTER(IndexParams), P, pp]
     lib.dts_search.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps]
-    lib.dts_search_ex.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
-                                  ctypes.POINTER(SearchStats)]
-    lib.dts_search_device_ex.argtypes = [P, P, S, ctypes.c_double, P, P, pp, ps,
+    lib.dts_search_ex.argtypes = [P, P, S, ctypes.c_double, ctypes.POINTER(SearchOptions), P,
+                                  pp, ps, ctypes.POINTER(SearchStats)]
+    lib.dts_search_device_ex.argtypes = [P, P, S, ctypes.c_double,
+                                         ctypes.POINTER(SearchOptions), P, pp, ps,
                                          ctypes.POINTER(SearchStats)]
+    lib.dts_merge_trajectories_device.argtypes = [P, S, P, S, P, S, P, pp, ps]
+    lib.dts_merge_trajectories_device.restype = ctypes.c_int
     lib.dts_search_device_ex.restype = ctypes.c_int
     lib.dts_canonicalize_device.argtypes = [P, S, P]
     lib.dts_canonicalize_device.restype = ctypes.c_int
@@ -145,10 +157,25 @@ def _segments(a) -> np.ndarray:
 
 
 def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0, method="grid",
-            subbins=0, entry_ids_ptr=None) -> IndexParams:
+            subbins=0, entry_ids_ptr=None, entry_traj_ptr=None) -> IndexParams:
     m = METHODS[method] if isinstance(method, str) else int(method)
     return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0,
-                       m, int(subbins), entry_ids_ptr)
+                       m, int(subbins), entry_ids_ptr, entry_traj_ptr)
+
+
+def _u32_host(a, n, what):
+    if a is None:
+        return None
+    a = np.ascontiguousarray(a, dtype=np.uint32)
+    if a.shape[0] != n:
+        raise ValueError(f"{what} must have {n} entries")
+    return a
+
+
+def _dev_ptr(t):
+    if t is None:
+        return None
+    return t.data_ptr() if hasattr(t, "data_ptr") else int(t)
 
 
 def _stream_ptr(stream) -> int:
@@ -191,14 +218,15 @@ class DeviceResults:
     """Results in library-owned device memory (dts_free_results_device on
     release).  Exposes __cuda_array_interface__ as a flat uint8 buffer."""
 
-    def __init__(self, ptr: int, count: int, device: int):
+    def __init__(self, ptr: int, count: int, device: int, dtype=RESULT_DTYPE):
         self.ptr = ptr
         self.count = count
         self.device = device
+        self.dtype = dtype
 
     @property
     def __cuda_array_interface__(self):
-        return {"shape": (self.count * RESULT_DTYPE.itemsize,), "typestr": "|u1",
+        return {"shape": (self.count * self.dtype.itemsize,), "typestr": "|u1",
                 "data": (self.ptr or 0, False), "version": 3}
 
     def tensor(self):
@@ -209,8 +237,8 @@ class DeviceResults:
 
     def numpy(self) -> np.ndarray:
         if self.count == 0:
-            return np.empty(0, dtype=RESULT_DTYPE)
-        return self.tensor().cpu().numpy().view(RESULT_DTYPE)
+            return np.empty(0, dtype=self.dtype)
+        return self.tensor().cpu().numpy().view(self.dtype)
 
     def free(self):
         if self.ptr:
@@ -227,18 +255,16 @@ class DeviceResults:
 
 def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int = 0,
                 d_hint: float = 0.0, method="grid", subbins: int = 0,
-                entry_ids=None) -> Index:
-    """dts_build_index: D is host (n, 8) float64 (copied); entry_ids: optional
-    host uint32 ids reported for the rows of D."""
+                entry_ids=None, entry_traj=None) -> Index:
+    """dts_build_index: D is host (n, 8) float64 (copied); entry_ids /
+    entry_traj: optional host uint32 reported ids / trajectory ids per row."""
     lib = load()
     D = _segments(D)
-    ids = None
-    if entry_ids is not None:
-        ids = np.ascontiguousarray(entry_ids, dtype=np.uint32)
-        if ids.shape[0] != D.shape[0]:
-            raise ValueError("entry_ids must have one id per row of D")
+    ids = _u32_host(entry_ids, D.shape[0], "entry_ids")
+    traj = _u32_host(entry_traj, D.shape[0], "entry_traj")
     p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins,
-                ids.ctypes.data if ids is not None else None)
+                ids.ctypes.data if ids is not None else None,
+                traj.ctypes.data if traj is not None else None)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index(D.ctypes.data if D.size else None, D.shape[0], ctypes.byref(p),
                                ctypes.byref(h)))
@@ -247,17 +273,16 @@ def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int =
 
 def build_index_device(D_dev, n: int = None, device: int = 0, temporal_bins: int = 0,
                        cells_per_dim: int = 0, d_hint: float = 0.0, stream=None,
-                       method="grid", subbins: int = 0, entry_ids=None) -> Index:
+                       method="grid", subbins: int = 0, entry_ids=None,
+                       entry_traj=None) -> Index:
     """dts_build_index_device: D_dev is a CUDA tensor (n, 8) float64;
-    entry_ids: optional CUDA int32/uint32 tensor of reported ids."""
+    entry_ids / entry_traj: optional CUDA int32/uint32 tensors."""
     lib = load()
     ptr = D_dev.data_ptr() if hasattr(D_dev, "data_ptr") else int(D_dev)
     if n is None:
         n = D_dev.shape[0]
-    eptr = None
-    if entry_ids is not None:
-        eptr = entry_ids.data_ptr() if hasattr(entry_ids, "data_ptr") else int(entry_ids)
-    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins, eptr)
+    p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins,
+                _dev_ptr(entry_ids), _dev_ptr(entry_traj))
     h = ctypes.c_void_p()
     _check(lib.dts_build_index_device(ctypes.c_void_p(ptr), n, ctypes.byref(p),
                                       ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(h)))
@@ -274,16 +299,23 @@ def _host_results(ptr, count) -> np.ndarray:
 
 
 def search_ex(index: Index, Q, d: float, query_id_base: int = 0, stream=None,
-              time_kernels: bool = False):
-    """dts_search_ex: host Q -> (results structured array, stats dict)."""
+              time_kernels: bool = False, query_ids=None, query_traj=None,
+              exclude_same_trajectory: bool = False):
+    """dts_search_ex: host Q (+ optional host uint32 query_ids / query_traj)
+    -> (results structured array, stats dict)."""
     lib = load()
     Q = _segments(Q)
+    qids = _u32_host(query_ids, Q.shape[0], "query_ids")
+    qtraj = _u32_host(query_traj, Q.shape[0], "query_traj")
+    opts = SearchOptions(int(query_id_base), qids.ctypes.data if qids is not None else None,
+                         qtraj.ctypes.data if qtraj is not None else None,
+                         1 if exclude_same_trajectory else 0)
     out = ctypes.c_void_p()
     cnt = ctypes.c_size_t()
     st = SearchStats()
     st.time_kernels = 1 if time_kernels else 0
     _check(lib.dts_search_ex(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
-                             float(d), int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
+                             float(d), ctypes.byref(opts), ctypes.c_void_p(_stream_ptr(stream)),
                              ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     return _host_results(out.value, cnt.value), st.as_dict()
 
@@ -301,7 +333,8 @@ def search(index: Index, Q, d: float, query_id_base: int = 0, stream=None) -> np
 
 
 def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=None,
-                  n: int = None, time_kernels: bool = False, query_ids=None):
+                  n: int = None, time_kernels: bool = False, query_ids=None, query_traj=None,
+                  exclude_same_trajectory: bool = False):
     """dts_search_device (dts_search_device_ex when query_ids, a CUDA int32 /
     uint32 tensor of increasing reported ids, is given): Q_dev CUDA tensor
     (nq, 8) float64 -> (DeviceResults, stats)."""
@@ -313,17 +346,41 @@ def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=
     cnt = ctypes.c_size_t()
     st = SearchStats()
     st.time_kernels = 1 if time_kernels else 0
-    if query_ids is None:
+    if query_ids is None and query_traj is None and not exclude_same_trajectory:
         _check(lib.dts_search_device(index.handle, ctypes.c_void_p(ptr), n, float(d),
                                      int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
                                      ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     else:
-        qptr = query_ids.data_ptr() if hasattr(query_ids, "data_ptr") else int(query_ids)
+        opts = SearchOptions(int(query_id_base), _dev_ptr(query_ids), _dev_ptr(query_traj),
+                             1 if exclude_same_trajectory else 0)
         _check(lib.dts_search_device_ex(index.handle, ctypes.c_void_p(ptr), n, float(d),
-                                        ctypes.c_void_p(qptr),
+                                        ctypes.byref(opts),
                                         ctypes.c_void_p(_stream_ptr(stream)),
                                         ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     return DeviceResults(out.value or 0, cnt.value, index.device), st.as_dict()
+
+
+def merge_trajectories_device(results, query_traj, entry_traj, stream=None):
+    """dts_merge_trajectories_device: DeviceResults (or a CUDA uint8 tensor of
+    24-byte records) + CUDA uint32/int32 tensors of trajectory ids indexed by
+    reported query id / entry id -> DeviceResults-like buffer of 24-byte
+    dts_traj_result records (numpy(TRAJ_DTYPE))."""
+    lib = load()
+    if isinstance(results, DeviceResults):
+        rptr, n, dev = results.ptr, results.count, results.device
+    else:
+        rptr, n, dev = results.data_ptr(), results.numel() // RESULT_DTYPE.itemsize, \
+            results.device.index or 0
+    out = ctypes.c_void_p()
+    cnt = ctypes.c_size_t()
+    _check(lib.dts_merge_trajectories_device(ctypes.c_void_p(rptr or 0), int(n),
+                                             ctypes.c_void_p(_dev_ptr(query_traj)),
+                                             int(query_traj.numel()),
+                                             ctypes.c_void_p(_dev_ptr(entry_traj)),
+                                             int(entry_traj.numel()),
+                                             ctypes.c_void_p(_stream_ptr(stream)),
+                                             ctypes.byref(out), ctypes.byref(cnt)))
+    return DeviceResults(out.value or 0, cnt.value, dev, dtype=TRAJ_DTYPE)
 
 
 def canonicalize_device(results_dev, n: int = None, stream=None) -> None:

@@ -108,6 +108,8 @@ void free_index_memory(dts_index* idx) {
     cudaDeviceSynchronize();
     cache_free(idx->block);
     cache_free(idx->ht.slots);
+    cache_free(idx->etraj);
+    idx->etraj = nullptr;
     for (int a = 0; a < 3; ++a) {
         cache_free(idx->sb_block[a]);
         idx->sb_block[a] = nullptr;
@@ -176,6 +178,12 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
                                          cudaMemcpyHostToDevice, s));
                 p.entry_ids = dmap.p;
             }
+            DevBuf<uint32_t> dtraj(p.entry_traj ? n : 0, s);
+            if (p.entry_traj) {
+                DTS_CUDA(cudaMemcpyAsync(dtraj.p, p.entry_traj, n * sizeof(uint32_t),
+                                         cudaMemcpyHostToDevice, s));
+                p.entry_traj = dtraj.p;
+            }
             build_index_device(idx, dD.p, n, p, s);
         } else {
             check_aligned(D, "D_dev");
@@ -200,7 +208,8 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
 // the chunk's offset.  Concatenation in chunk order is the canonical order.
 dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_t nq, double d,
                             uint32_t qid_base, cudaStream_t s, const ResultsTooLarge& big,
-                            dts_search_stats* stats, unsigned long long cap) {
+                            dts_search_stats* stats, unsigned long long cap,
+                            const uint32_t* qmap, const uint32_t* qtraj, bool excl) {
     size_t free_b = 0, total_b = 0;
     DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
     const unsigned long long budget = std::max<unsigned long long>(
@@ -218,7 +227,8 @@ dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_
             while (b < nq && (b == a || acc + big.counts[b] <= budget)) acc += big.counts[b++];
             SearchOut so;
             dts_search_stats cs{};
-            search_device(index, dQ + a, b - a, d, qid_base + (uint32_t)a, s, &so, &cs);
+            search_device(index, dQ + a, b - a, d, qid_base + (uint32_t)a, s, &so, &cs, ~0ull,
+                          qmap ? qmap + a : nullptr, qtraj ? qtraj + a : nullptr, excl);
             if (so.count != acc) {
                 cache_free(so.results);
                 throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
@@ -248,11 +258,15 @@ dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_
 dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
                          uint32_t qid_base, cudaStream_t s, bool host, dts_result** out_results,
                          size_t* out_count, dts_search_stats* stats,
-                         const uint32_t* qmap = nullptr) {
+                         const dts_search_options* opts = nullptr) {
     if (out_results) *out_results = nullptr;
     if (out_count) *out_count = 0;
     dts_result* ret = nullptr;
     size_t cnt = 0;
+    const uint32_t* qmap = opts ? opts->query_ids : nullptr;
+    const uint32_t* qtraj = opts ? opts->query_traj : nullptr;
+    const bool excl = opts && opts->exclude_same_trajectory;
+    if (opts) qid_base = opts->query_id_base;
     dts_status st = guarded([&] {
         if (!index) throw Error(DTS_EINVAL, "index is NULL");
         if (!out_results || !out_count) throw Error(DTS_EINVAL, "output pointer is NULL");
@@ -268,17 +282,28 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
             if (nq)
                 DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment),
                                          cudaMemcpyHostToDevice, s));
+            DevBuf<uint32_t> dmap(qmap && nq ? nq : 0, s), dtraj(qtraj && nq ? nq : 0, s);
+            if (dmap.p) {
+                DTS_CUDA(cudaMemcpyAsync(dmap.p, qmap, nq * sizeof(uint32_t),
+                                         cudaMemcpyHostToDevice, s));
+            }
+            if (dtraj.p) {
+                DTS_CUDA(cudaMemcpyAsync(dtraj.p, qtraj, nq * sizeof(uint32_t),
+                                         cudaMemcpyHostToDevice, s));
+            }
             // DTS_MAX_DEVICE_RESULTS caps the results held on the device at
             // once (testing knob for the streamed path; default: memory)
             const char* cap_env = getenv("DTS_MAX_DEVICE_RESULTS");
             const unsigned long long cap = cap_env ? std::strtoull(cap_env, nullptr, 10) : ~0ull;
             try {
-                search_device(index, dQ.p, nq, d, qid_base, s, &so, stats, cap ? cap : ~0ull);
+                search_device(index, dQ.p, nq, d, qid_base, s, &so, stats, cap ? cap : ~0ull,
+                              dmap.p, dtraj.p, excl);
             } catch (ResultsTooLarge& big) {
                 // stream: query-id chunks whose results fit, each searched
                 // and copied out at its offset (the paper processed Q
                 // incrementally when its result buffer filled)
-                ret = search_streamed(index, dQ.p, nq, d, qid_base, s, big, stats, cap);
+                ret = search_streamed(index, dQ.p, nq, d, qid_base, s, big, stats, cap, dmap.p,
+                                      dtraj.p, excl);
                 cnt = (size_t)big.total;
                 return;
             }
@@ -302,7 +327,7 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
             DTS_CUDA(cudaStreamSynchronize(s));
         } else {
             check_aligned(Q, "Q_dev");
-            search_device(index, Q, nq, d, qid_base, s, &so, stats, ~0ull, qmap);
+            search_device(index, Q, nq, d, qid_base, s, &so, stats, ~0ull, qmap, qtraj, excl);
             ret = so.results;
             cnt = so.count;
         }
@@ -341,18 +366,41 @@ dts_status dts_search(const dts_index* index, const dts_segment* Q, size_t nq, d
 }
 
 dts_status dts_search_ex(const dts_index* index, const dts_segment* Q, size_t nq, double d,
-                         uint32_t query_id_base, void* cuda_stream, dts_result** out_results,
-                         size_t* out_count, dts_search_stats* stats) {
-    return search_common(index, Q, nq, d, query_id_base, static_cast<cudaStream_t>(cuda_stream),
-                         true, out_results, out_count, stats);
+                         const dts_search_options* opts, void* cuda_stream,
+                         dts_result** out_results, size_t* out_count, dts_search_stats* stats) {
+    return search_common(index, Q, nq, d, 0, static_cast<cudaStream_t>(cuda_stream), true,
+                         out_results, out_count, stats, opts);
 }
 
 dts_status dts_search_device_ex(const dts_index* index, const dts_segment* Q_dev, size_t nq,
-                                double d, const uint32_t* query_ids, void* cuda_stream,
+                                double d, const dts_search_options* opts, void* cuda_stream,
                                 dts_result** out_results_dev, size_t* out_count,
                                 dts_search_stats* stats) {
     return search_common(index, Q_dev, nq, d, 0, static_cast<cudaStream_t>(cuda_stream), false,
-                         out_results_dev, out_count, stats, query_ids);
+                         out_results_dev, out_count, stats, opts);
+}
+
+dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n,
+                                         const uint32_t* query_traj, size_t n_query_ids,
+                                         const uint32_t* entry_traj, size_t n_entry_ids,
+                                         void* cuda_stream, dts_traj_result** out_dev,
+                                         size_t* out_count) {
+    if (out_dev) *out_dev = nullptr;
+    if (out_count) *out_count = 0;
+    dts_traj_result* o = nullptr;
+    size_t c = 0;
+    dts_status st = guarded([&] {
+        if (!out_dev || !out_count) throw Error(DTS_EINVAL, "output pointer is NULL");
+        if (n > 0 && (!results_dev || !query_traj || !entry_traj))
+            throw Error(DTS_EINVAL, "NULL input with n > 0");
+        merge_trajectories_device(results_dev, n, query_traj, n_query_ids, entry_traj,
+                                  n_entry_ids, static_cast<cudaStream_t>(cuda_stream), &o, &c);
+    });
+    if (st == DTS_OK) {
+        *out_dev = o;
+        *out_count = c;
+    }
+    return st;
 }
 
 dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream) {
@@ -373,7 +421,7 @@ dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, s
 
 void dts_free_results(dts_result* results) { pinned_free(results); }
 
-void dts_free_results_device(dts_result* results) {
+void dts_free_results_device(void* results) {
     if (results) {
         cudaDeviceSynchronize();
         cache_free(results);

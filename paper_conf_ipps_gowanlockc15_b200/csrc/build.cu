@@ -350,6 +350,13 @@ __global__ void __launch_bounds__(BT) k_map_ids(uint32_t* __restrict__ eid, size
     if (p < n) eid[p] = emap[eid[p]];
 }
 
+__global__ void __launch_bounds__(BT) k_gather_u32(uint32_t* __restrict__ out,
+                                                  const uint32_t* __restrict__ in,
+                                                  const uint32_t* __restrict__ rows, size_t n) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p < n) out[p] = in[rows[p]];
+}
+
 // dir[k] = first position of key >= k in the sorted keys, k in [0, nkeys].
 __global__ void __launch_bounds__(BT) k_sb_dir(const unsigned long long* __restrict__ keys,
                                               size_t len, unsigned long long nkeys,
@@ -558,7 +565,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         build_subbins(idx, D, n, hb, p, s);
     }
 
-    // 8. reported entry ids of a shard (params.entry_ids, device memory here)
+    // 8. trajectory ids in sorted order (params.entry_traj, device memory here)
+    if (p.entry_traj) {
+        idx->etraj = static_cast<uint32_t*>(cache_alloc(n * sizeof(uint32_t)));
+        k_gather_u32<<<grid_for(n), BT, 0, s>>>(idx->etraj, p.entry_traj, idx->soa.eid, n);
+        DTS_LAUNCH_CHECK();
+    }
+
+    // 9. reported entry ids of a shard (params.entry_ids, device memory here)
     if (p.entry_ids) {
         k_map_ids<<<grid_for(n), BT, 0, s>>>(idx->soa.eid, n, p.entry_ids);
         DTS_LAUNCH_CHECK();

@@ -224,6 +224,7 @@ struct dts_index {
     dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only
     uint32_t* sb_block[3] = {nullptr, nullptr, nullptr};   // ids + dir per dimension
     uint64_t sb_len[3] = {0, 0, 0};
+    uint32_t* etraj = nullptr;     // trajectory id per sorted position (optional)
 };
 
 namespace dts {
@@ -247,7 +248,12 @@ struct ResultsTooLarge : Error {
 };
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
-                   unsigned long long max_results = ~0ull, const uint32_t* qmap = nullptr);
+                   unsigned long long max_results = ~0ull, const uint32_t* qmap = nullptr,
+                   const uint32_t* qtraj = nullptr, bool exclude_same_traj = false);
+// Trajectory-level merge (traj.cu); output in cache_alloc'd device memory.
+void merge_trajectories_device(const dts_result* r, size_t n, const uint32_t* qtraj,
+                               size_t nqid, const uint32_t* etraj, size_t neid,
+                               cudaStream_t s, dts_traj_result** out, size_t* count);
 // Sort results in device memory by (query_id, entry_id), in place.
 void canonicalize_device(dts_result* r, size_t n, cudaStream_t s);
 }  // namespace dts

@@ -359,6 +359,9 @@ struct PassArgs {
     uint32_t qid_base;
     uint32_t method;
     SubbinIndex sb;
+    const uint32_t* etraj;
+    const uint32_t* qtraj;
+    uint32_t excl;
 };
 
 // Warp w of CTA b processes sorted position tiles[b / (TQ/PW)]*TQ + ...; the
@@ -380,6 +383,7 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
     const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start, a.bin_t0min,
                                     a.bin_t1max, a.method, a.sb);
     const uint32_t* ind = st.rind ? sb_ids(a.sb, st.rind) : nullptr;   // subbin id array
+    const uint32_t qtraj = a.excl ? __ldg(a.qtraj + qid) : 0u;
     const double d2 = a.d * a.d;
     unsigned long long out_pos = a.offsets[qid];
     uint32_t dummy = 0;
@@ -412,8 +416,9 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
                     if (s_excl[warp][j + step] <= t) j += step;
                 p = s_start[warp][j] + (uint32_t)(t - s_excl[warp][j]);
                 if (ind) p = __ldg(ind + p);
-                hit = refine(q, __ldg(a.soa.st + p), __ldg(a.soa.sx + p), __ldg(a.soa.sy + p),
-                             __ldg(a.soa.sz + p), d2, r0, r1);
+                if (!(a.excl && __ldg(a.etraj + p) == qtraj))
+                    hit = refine(q, __ldg(a.soa.st + p), __ldg(a.soa.sx + p),
+                                 __ldg(a.soa.sy + p), __ldg(a.soa.sz + p), d2, r0, r1);
             }
             const uint32_t bal = __ballot_sync(0xffffffffu, hit);
             if (hit) {
@@ -510,7 +515,8 @@ struct EventTimer {
 
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
-                   unsigned long long max_results, const uint32_t* qmap) {
+                   unsigned long long max_results, const uint32_t* qmap,
+                   const uint32_t* qtraj, bool exclude_same_traj) {
     out->results = nullptr;
     out->count = 0;
     dts_search_stats local{};
@@ -571,6 +577,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.over_tiles = over_tiles.p;
     ta.qid_base = qid_base;
     ta.qmap = qmap;
+    ta.etraj = idx->etraj;
+    ta.qtraj = qtraj;
+    ta.excl = (qtraj && idx->etraj && exclude_same_traj) ? 1u : 0u;
+    if (exclude_same_traj && !(qtraj && idx->etraj))
+        throw Error(DTS_EINVAL, "exclude_same_trajectory needs query_traj and an index built "
+                                "with entry_traj");
     ta.ctr = ctr.p;
     ta.method = idx->method;
     ta.sb = idx->sb;
@@ -669,6 +681,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 pa.qid_base = qid_base;
                 pa.method = idx->method;
                 pa.sb = idx->sb;
+                pa.etraj = ta.etraj;
+                pa.qtraj = ta.qtraj;
+                pa.excl = ta.excl;
                 const unsigned nb = h.c.n_over * (TQ / PW);
                 k_pass_scatter<<<nb, PT, 0, s>>>(pa);
                 DTS_LAUNCH_CHECK();

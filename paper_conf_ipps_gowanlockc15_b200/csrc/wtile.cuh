@@ -26,6 +26,7 @@ struct WarpSmem {
     int32_t lb[WQ], hb[WQ], clo[3][WQ], cn[3][WQ];
     uint32_t qid[WQ], mode[WQ], qcount[WQ], qoff[WQ];
     uint32_t rstart[WQ], rcnt[WQ], rind[WQ];   // single-run queries (temporal / subbin)
+    uint32_t qtraj[WQ];                        // trajectory ids (exclude_same_trajectory)
     unsigned long long lkoff[WQ + 1];
     unsigned long long hkey[WH];        // (query << 42) | (entry id << 10) | slot
     double h0[WH], h1[WH];
@@ -50,6 +51,9 @@ struct TileArgs {
     uint32_t* over_tiles;              // tiles to recompute in pass 2
     uint32_t qid_base;
     const uint32_t* qmap;              // optional reported query ids (else qid + qid_base)
+    const uint32_t* etraj;             // trajectory id per sorted entry position
+    const uint32_t* qtraj;             // trajectory id per query row
+    uint32_t excl;                     // exclude_same_trajectory
     Counters* ctr;
     uint32_t method;
     SubbinIndex sb;
@@ -121,6 +125,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             S.rstart[lane] = st.rstart;
             S.rcnt[lane] = st.rcnt;
             S.rind[lane] = st.rind;
+            S.qtraj[lane] = (a.excl && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
             S.qcount[lane] = 0;
             nlook = st.nlook;
         }
@@ -191,9 +196,12 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     const double2 st2 = __ldg(a.soa.st + p2), sx2 = __ldg(a.soa.sx + p2);
                     const double2 sy2 = __ldg(a.soa.sy + p2), sz2 = __ldg(a.soa.sz + p2);
                     double h0, h1;
-                    if (refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
+                    const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
+                    const bool x2 = a.excl && __ldg(a.etraj + p2) == S.qtraj[qi2];
+                    if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
                         stage_hit(S, qi1, p1, h0, h1, a.soa.eid);
-                    if (v2 && refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
+                    if (v2 && !x2 &&
+                        refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
                         stage_hit(S, qi2, p2, h0, h1, a.soa.eid);
                 }
             }

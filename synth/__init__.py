@@ -130,6 +130,8 @@ class Config:
     d: float               # headline distance
     d_sweep: tuple         # other distances used by tests / sweeps
     note: str
+    etraj: np.ndarray = None   # trajectory id of each entry segment
+    qtraj: np.ndarray = None   # trajectory id of each query segment
 
 
 CONFIG_NAMES = ("C0", "C1", "C2", "C3", "C4")
@@ -137,9 +139,18 @@ CONFIG_NAMES = ("C0", "C1", "C2", "C3", "C4")
 
 def _sample_query_trajectories(D: np.ndarray, ntraj: int, nseg: int,
                                nq_traj: int, seed: int) -> np.ndarray:
+    return _sample_with_ids(D, ntraj, nseg, nq_traj, seed)[0]
+
+
+def _sample_with_ids(D: np.ndarray, ntraj: int, nseg: int, nq_traj: int, seed: int):
     g = rng(seed)
     chosen = np.sort(g.choice(ntraj, size=nq_traj, replace=False))
-    return np.ascontiguousarray(D.reshape(ntraj, nseg, 8)[chosen].reshape(-1, 8))
+    Q = np.ascontiguousarray(D.reshape(ntraj, nseg, 8)[chosen].reshape(-1, 8))
+    return Q, np.repeat(chosen, nseg).astype(np.uint32)
+
+
+def _traj_ids(ntraj: int, nseg: int) -> np.ndarray:
+    return np.repeat(np.arange(ntraj, dtype=np.uint32), nseg)
 
 
 def make_config(name: str, rank: int = 0, scale: float = 1.0) -> Config:
@@ -160,7 +171,8 @@ def make_config(name: str, rank: int = 0, scale: float = 1.0) -> Config:
         Q = np.concatenate([segments_from_trajectories(t1, p1),
                             segments_from_trajectories(t2, p2)])
         return Config(name, D, Q, 0.05, (0.0, 0.01, 0.05, 0.2),
-                      "tiny random walks (P:L127 shape), unit cube")
+                      "tiny random walks (P:L127 shape), unit cube", _traj_ids(20, 100),
+                      np.repeat(np.array([1000, 1001], dtype=np.uint32), 100))
     if name in ("C1", "C4"):
         if name == "C1":
             n1, n2, nq_traj, seed = 2731, 2730, 52, 2
@@ -171,18 +183,20 @@ def make_config(name: str, rank: int = 0, scale: float = 1.0) -> Config:
         t, pos = galaxy(rng(seed), n1, n2, 193)
         D = segments_from_trajectories(t, pos)
         del t, pos
-        Q = _sample_query_trajectories(D, n1 + n2, 192, nq_traj, seed + 1000 + rank)
+        Q, qt = _sample_with_ids(D, n1 + n2, 192, nq_traj, seed + 1000 + rank)
         return Config(name, D, Q, 0.005, (0.001, 0.005, 0.02),
-                      "two-disk galaxy merger shape (P:L129), 193 synchronised samples")
+                      "two-disk galaxy merger shape (P:L129), 193 synchronised samples",
+                      _traj_ids(n1 + n2, 192), qt)
     if name == "C2":
         ntraj, nq_traj = max(2, int(21846 * scale)), max(1, int(521 * scale))
         side = (ntraj / 0.112) ** (1.0 / 3.0)   # density 0.112 pc^-3
         t, pos = random_walks(rng(3), ntraj, 193, side, 0.05, 100.0)
         D = segments_from_trajectories(t, pos)
         del t, pos
-        Q = _sample_query_trajectories(D, ntraj, 192, nq_traj, 3 + 1000 + rank)
+        Q, qt = _sample_with_ids(D, ntraj, 192, nq_traj, 3 + 1000 + rank)
         return Config(name, D, Q, 0.09, (0.03, 0.09, 0.5, 2.0, 8.0),
-                      "uniform dense random walks at 0.112 pc^-3 (P:L131)")
+                      "uniform dense random walks at 0.112 pc^-3 (P:L131)",
+                      _traj_ids(ntraj, 192), qt)
     if name == "C3":
         ntraj, nq_traj = max(2, int(10000 * scale)), max(1, int(250 * scale))
         t, pos = random_walks(rng(4), ntraj, 400, 1000.0, 1.0, 10000.0)
@@ -190,7 +204,8 @@ def make_config(name: str, rank: int = 0, scale: float = 1.0) -> Config:
         tq, pq = random_walks(rng(4 + 1000 + rank), nq_traj, 400, 1000.0, 1.0, 10000.0)
         Q = segments_from_trajectories(tq, pq)
         return Config(name, D, Q, 5.0, (1.0, 5.0, 20.0, 50.0),
-                      "sparse long-span random walks (P:L127 shape stretched)")
+                      "sparse long-span random walks (P:L127 shape stretched)",
+                      _traj_ids(ntraj, 399), _traj_ids(nq_traj, 399) + np.uint32(ntraj))
     # ---- paper-replica scenarios; sizes exactly as P:L127-P:L141
     if name == "S1":
         # Random: 2,500 random-walk trajectories x 400 timesteps = 997,500

@@ -334,3 +334,72 @@ def test_entry_ids_host_build(dts):
     idx = dts.build_index(c.D[perm], entry_ids=perm.astype(np.uint32))
     got = dts.search(idx, c.Q, c.d)
     assert got.tobytes() == ref.tobytes()
+
+
+# ------------------------------------------------ trajectory level (§8 f3)
+def test_exclude_same_trajectory(dts, oracle_mod):
+    """'any OTHER stellar trajectory': pairs of the same trajectory
+    are dropped; everything else is the oracle's result."""
+    import torch
+    c = synth.make_config("C2", scale=0.004)
+    d = 2.0
+    ora = oracle_mod.search(c.D, c.Q, d, threads=THREADS)
+    keep = c.qtraj[ora["query_id"]] != c.etraj[ora["entry_id"]]
+    assert (~keep).sum() >= c.Q.shape[0]            # the self pairs existed
+    ora = ora[keep]
+    for method in ("grid", "subbin"):
+        idx = dts.build_index(c.D, entry_traj=c.etraj, method=method)
+        got, _ = dts.search_ex(idx, c.Q, d, query_traj=c.qtraj, exclude_same_trajectory=True)
+        parity.compare(got, ora, c.D, c.Q, d, oracle_mod)
+        idxd = dts.build_index_device(torch.from_numpy(c.D).cuda(),
+                                      entry_traj=torch.from_numpy(c.etraj).cuda())
+        res, _ = dts.search_device(idxd, torch.from_numpy(c.Q).cuda(), d,
+                                   query_traj=torch.from_numpy(c.qtraj).cuda(),
+                                   exclude_same_trajectory=True)
+        assert res.numpy().tobytes() == got.tobytes()
+    with pytest.raises(dts.DTSError):
+        dts.search_ex(dts.build_index(c.D), c.Q, d, query_traj=c.qtraj,
+                      exclude_same_trajectory=True)
+
+
+def test_merge_trajectories_matches_oracle(dts, oracle_mod):
+    import torch
+    for name, scale, d in (("C0", 1.0, 0.2), ("C2", 0.004, 2.0)):
+        c = synth.make_config(name, scale=scale)
+        idx = dts.build_index_device(torch.from_numpy(c.D).cuda())
+        res, _ = dts.search_device(idx, torch.from_numpy(c.Q).cuda(), d)
+        seg = res.numpy()
+        m = dts.merge_trajectories_device(res, torch.from_numpy(c.qtraj).cuda(),
+                                          torch.from_numpy(c.etraj).cuda())
+        got = m.numpy()
+        ref = oracle_mod.merge_trajectory_pairs(seg, c.qtraj, c.etraj)
+        assert got.shape == ref.shape and got.shape[0] > 0
+        assert np.array_equal(got["query_traj"], ref["query_traj"])
+        assert np.array_equal(got["entry_traj"], ref["entry_traj"])
+        assert np.array_equal(got["t_start"], ref["t_start"])
+        assert np.array_equal(got["t_end"], ref["t_end"])
+        # and against the merge of the ORACLE's segment results
+        ora = oracle_mod.merge_trajectory_pairs(oracle_mod.search(c.D, c.Q, d, threads=THREADS),
+                                                c.qtraj, c.etraj)
+        assert got.shape == ora.shape
+        span = float(c.D[:, 4].max() - c.D[:, 0].min())
+        assert np.max(np.abs(got["t_start"] - ora["t_start"])) / span < 1e-9
+        assert np.max(np.abs(got["t_end"] - ora["t_end"])) / span < 1e-9
+
+
+def test_stationary_supernova_queries(dts, oracle_mod):
+    """Application (i) of P:L15: stars within d of a supernova -- a stationary
+    query point over a time window."""
+    c = synth.make_config("C2", scale=0.004)
+    g = synth.rng(21)
+    k = 40
+    P = c.D[g.choice(c.D.shape[0], size=k, replace=False)]
+    Q = np.zeros((k, 8))
+    Q[:, 0] = P[:, 0] - 0.3
+    Q[:, 4] = P[:, 0] + 2.7
+    Q[:, 1:4] = P[:, 1:4] + g.normal(0, 0.5, size=(k, 3))
+    Q[:, 5:8] = Q[:, 1:4]
+    for d in (0.5, 3.0):
+        got, info = run_and_compare(dts, oracle_mod, c.D, Q, d)
+        if d == 3.0:
+            assert info["common"] > 0

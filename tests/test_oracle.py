@@ -353,3 +353,16 @@ def test_paper_replica_shapes():
     assert synth.segment_count(2500, 400) == 997_500
     assert synth.segment_count(2 * 65536, 193) == 25_165_824
     assert synth.segment_count(65536, 193) == 12_582_912
+
+
+def test_merge_trajectory_pairs_hand_example(oracle_mod):
+    """Union of closed intervals per trajectory pair (P:L15 application):
+    touching pieces merge, gaps split, pairs stay separate."""
+    dt = oracle_mod.RESULT_DTYPE
+    res = np.array([(0, 0, 0.0, 1.0), (0, 1, 1.0, 2.0), (0, 2, 3.0, 4.0),
+                    (1, 0, 0.5, 0.7), (0, 3, 1.5, 1.8), (2, 1, 5.0, 5.0)], dtype=dt)
+    qtraj = [7, 7, 9]
+    etraj = [1, 1, 1, 2]
+    m = oracle_mod.merge_trajectory_pairs(res, qtraj, etraj)
+    got = [(int(r["query_traj"]), int(r["entry_traj"]), r["t_start"], r["t_end"]) for r in m]
+    assert got == [(7, 1, 0.0, 2.0), (7, 1, 3.0, 4.0), (7, 2, 1.5, 1.8), (9, 1, 5.0, 5.0)]
