@@ -255,6 +255,103 @@ dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_
     return h;
 }
 
+// Host query set streamed through the device in chunks (
+// the setting of the paper's prior work where Q does not fit on the GPU,
+// P:L28): while chunk i is searched on the caller's stream, chunk i+1 is
+// copied host -> device and the results of chunk i-1 device -> host on a
+// copy stream, into one growing pinned output buffer.  Chunks are contiguous
+// query-id ranges, so chunk-order concatenation is the canonical order.
+dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                             uint32_t qid_base, cudaStream_t s, size_t chunk,
+                             const uint32_t* dmap, const uint32_t* dtraj, bool excl,
+                             dts_search_stats* stats, size_t* out_count) {
+    cudaStream_t cs = nullptr;
+    DTS_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    cudaEvent_t h2d[2] = {nullptr, nullptr};
+    struct Pending {
+        dts_result* dev;
+        size_t n;
+    };
+    std::vector<Pending> pending;
+    dts_result* out = nullptr;
+    size_t cap = 0, used = 0;
+    dts_search_stats agg{};
+    if (stats) agg.time_kernels = stats->time_kernels;
+    auto cleanup = [&]() {
+        if (cs) cudaStreamSynchronize(cs);
+        for (auto& p : pending) cache_free(p.dev);
+        pending.clear();
+        for (auto& e : h2d) if (e) cudaEventDestroy(e);
+        if (cs) cudaStreamDestroy(cs);
+        cs = nullptr;
+    };
+    try {
+        for (auto& e : h2d) DTS_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+        DevBuf<dts_segment> qb0(chunk, s), qb1(chunk, s);
+        dts_segment* qb[2] = {qb0.p, qb1.p};
+        DTS_CUDA(cudaStreamSynchronize(s));          // buffers ready before the copy stream
+        const size_t nchunks = (nq + chunk - 1) / chunk;
+        auto issue_h2d = [&](size_t i) {
+            const size_t a = i * chunk, m = std::min(chunk, nq - a);
+            DTS_CUDA(cudaMemcpyAsync(qb[i & 1], Q + a, m * sizeof(dts_segment),
+                                     cudaMemcpyHostToDevice, cs));
+            DTS_CUDA(cudaEventRecord(h2d[i & 1], cs));
+        };
+        issue_h2d(0);
+        for (size_t i = 0; i < nchunks; ++i) {
+            const size_t a = i * chunk, m = std::min(chunk, nq - a);
+            DTS_CUDA(cudaStreamWaitEvent(s, h2d[i & 1], 0));
+            if (i + 1 < nchunks) issue_h2d(i + 1);   // buffer (i+1)&1 is free: search i-1 done
+            SearchOut so;
+            dts_search_stats cs_stats{};
+            cs_stats.time_kernels = agg.time_kernels;
+            search_device(index, qb[i & 1], m, d, qid_base + (uint32_t)a, s, &so, &cs_stats,
+                          ~0ull, dmap ? dmap + a : nullptr, dtraj ? dtraj + a : nullptr, excl);
+            if (so.count) {
+                if (used + so.count > cap) {          // grow the pinned output
+                    DTS_CUDA(cudaStreamSynchronize(cs));
+                    const size_t want = std::max(used + so.count,
+                                                 (size_t)((double)(used + so.count) *
+                                                          (double)nchunks / (double)(i + 1) * 1.2));
+                    dts_result* bigger = static_cast<dts_result*>(
+                        pinned_alloc(want * sizeof(dts_result)));
+                    if (used) std::memcpy(bigger, out, used * sizeof(dts_result));
+                    pinned_free(out);
+                    out = bigger;
+                    cap = want;
+                }
+                DTS_CUDA(cudaMemcpyAsync(out + used, so.results, so.count * sizeof(dts_result),
+                                         cudaMemcpyDeviceToHost, cs));
+                pending.push_back({so.results, so.count});
+                used += so.count;
+            }
+            agg.candidates += cs_stats.candidates;
+            agg.cell_lookups += cs_stats.cell_lookups;
+            agg.max_results_per_query =
+                std::max(agg.max_results_per_query, cs_stats.max_results_per_query);
+            agg.ms_prep += cs_stats.ms_prep;
+            agg.ms_count += cs_stats.ms_count;
+            agg.ms_scan += cs_stats.ms_scan;
+            agg.ms_scatter += cs_stats.ms_scatter;
+            agg.ms_canon += cs_stats.ms_canon;
+        }
+        DTS_CUDA(cudaStreamSynchronize(cs));
+    } catch (...) {
+        cleanup();
+        pinned_free(out);
+        throw;
+    }
+    cleanup();
+    agg.results = used;
+    if (stats) *stats = agg;
+    if (used == 0) {
+        pinned_free(out);
+        out = nullptr;
+    }
+    *out_count = used;
+    return out;
+}
+
 dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
                          uint32_t qid_base, cudaStream_t s, bool host, dts_result** out_results,
                          size_t* out_count, dts_search_stats* stats,
@@ -278,10 +375,6 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
         prepare_device(index->device);
         SearchOut so;
         if (host) {
-            DevBuf<dts_segment> dQ(nq, s);
-            if (nq)
-                DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment),
-                                         cudaMemcpyHostToDevice, s));
             DevBuf<uint32_t> dmap(qmap && nq ? nq : 0, s), dtraj(qtraj && nq ? nq : 0, s);
             if (dmap.p) {
                 DTS_CUDA(cudaMemcpyAsync(dmap.p, qmap, nq * sizeof(uint32_t),
@@ -291,6 +384,25 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
                 DTS_CUDA(cudaMemcpyAsync(dtraj.p, qtraj, nq * sizeof(uint32_t),
                                          cudaMemcpyHostToDevice, s));
             }
+            // large host query sets stream through the device in chunks
+            // (DTS_Q_CHUNK queries each, default 262144; 0 disables)
+            const char* ch_env = getenv("DTS_Q_CHUNK");
+            const size_t chunk = ch_env ? (size_t)std::strtoull(ch_env, nullptr, 10)
+                                        : (size_t)262144;
+            if (chunk > 0 && nq >= 2 * chunk) {
+                try {
+                    ret = search_pipelined(index, Q, nq, d, qid_base, s, chunk, dmap.p, dtraj.p,
+                                           excl, stats, &cnt);
+                    return;
+                } catch (ResultsTooLarge&) {
+                    // a chunk's results exceed the device: use the query-id
+                    // streaming below (all of Q resident)
+                }
+            }
+            DevBuf<dts_segment> dQ(nq, s);
+            if (nq)
+                DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment),
+                                         cudaMemcpyHostToDevice, s));
             // DTS_MAX_DEVICE_RESULTS caps the results held on the device at
             // once (testing knob for the streamed path; default: memory)
             const char* cap_env = getenv("DTS_MAX_DEVICE_RESULTS");

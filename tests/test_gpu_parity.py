@@ -403,3 +403,27 @@ def test_stationary_supernova_queries(dts, oracle_mod):
         got, info = run_and_compare(dts, oracle_mod, c.D, Q, d)
         if d == 3.0:
             assert info["common"] > 0
+
+
+# ------------------------------------------------ out-of-core Q (§8 f4)
+def test_pipelined_query_chunks_match(dts, oracle_mod, monkeypatch):
+    """Host query sets streamed through the device in chunks (H2D of the next
+    chunk and D2H of the previous results overlap the search) give the same
+    bytes as the one-shot search."""
+    c = synth.make_config("C2", scale=0.01)
+    idx = dts.build_index(c.D, entry_traj=c.etraj)
+    monkeypatch.setenv("DTS_Q_CHUNK", "0")
+    ref = dts.search(idx, c.Q, 2.0)
+    ref_x, _ = dts.search_ex(idx, c.Q, 2.0, query_traj=c.qtraj, exclude_same_trajectory=True,
+                             query_id_base=5)
+    for chunk in (97, 400, 1500):
+        monkeypatch.setenv("DTS_Q_CHUNK", str(chunk))
+        got = dts.search(idx, c.Q, 2.0)
+        assert got.tobytes() == ref.tobytes(), chunk
+        got_x, st = dts.search_ex(idx, c.Q, 2.0, query_traj=c.qtraj,
+                                  exclude_same_trajectory=True, query_id_base=5)
+        assert got_x.tobytes() == ref_x.tobytes(), chunk
+        assert st["results"] == ref_x.shape[0]
+    qs = np.arange(0, c.Q.shape[0], 37)
+    parity.compare(parity.restrict(ref, qs), oracle_mod.search_queries(c.D, c.Q, qs, 2.0),
+                   c.D, c.Q, 2.0, oracle_mod)
