@@ -124,9 +124,22 @@ __global__ void __launch_bounds__(BT) k_bounds_final(const Bounds* __restrict__ 
     block_reduce_write(b, out);
 }
 
+// Sorted (key, row) pairs, either packed -- a[p] = key << shift | row, when
+// key bits + row bits fit in 64 (a keys-only sort on the key bits then moves
+// 8 bytes per element instead of 12) -- or as separate arrays (ids != null).
+struct SortedKeys {
+    const unsigned long long* a;
+    int shift;
+    const uint32_t* ids;
+    __device__ __forceinline__ unsigned long long key(size_t p) const { return a[p] >> shift; }
+    __device__ __forceinline__ uint32_t row(size_t p) const {
+        return ids ? ids[p] : (uint32_t)(a[p] & ((1ull << shift) - 1ull));
+    }
+};
+
 __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size_t n, GridParams g,
                                             unsigned long long* __restrict__ keys,
-                                            uint32_t* __restrict__ ids) {
+                                            uint32_t* __restrict__ ids, int shift) {
     size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
     if (i >= n) return;
     double4 s0 = D[2 * i], s1 = D[2 * i + 1];
@@ -134,8 +147,13 @@ __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size
     int32_t cx = cell_of(g, 0, 0.5 * (s0.y + s1.y));
     int32_t cy = cell_of(g, 1, 0.5 * (s0.z + s1.z));
     int32_t cz = cell_of(g, 2, 0.5 * (s0.w + s1.w));
-    keys[i] = make_key(g, bin, cx, cy, cz);
-    ids[i] = (uint32_t)i;
+    const unsigned long long k = make_key(g, bin, cx, cy, cz);
+    if (ids) {
+        keys[i] = k;
+        ids[i] = (uint32_t)i;
+    } else {
+        keys[i] = (k << shift) | (unsigned long long)i;
+    }
 }
 
 __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
@@ -147,14 +165,14 @@ constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
 // Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
 __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
-                                              const uint32_t* __restrict__ ids, SegSoA soa) {
+                                              const SortedKeys sk, SegSoA soa) {
     const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
     uint32_t id[GATHER_ITEMS];
     double4 r0[GATHER_ITEMS], r1[GATHER_ITEMS];
 #pragma unroll
     for (int k = 0; k < GATHER_ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
-        id[k] = p < n ? __ldg(ids + p) : 0u;
+        id[k] = p < n ? sk.row(p) : 0u;
     }
 #pragma unroll
     for (int k = 0; k < GATHER_ITEMS; ++k) {
@@ -201,7 +219,7 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
 // [B_first, B_last] of P:L76, keys being bin-major) and the per-bin extent
 // [min t_start, max t_end] (B_start / B_end of P:L76) with warp-aggregated
 // atomics on order-preserving integer images of the times.
-__global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __restrict__ keys,
+__global__ void __launch_bounds__(BT) k_count_cells(const SortedKeys keys,
                                                    size_t n, GridParams g,
                                                    const double2* __restrict__ st,
                                                    uint32_t* __restrict__ bin_start,
@@ -215,8 +233,8 @@ __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __
     // the bin is recomputed with bin_of() from t_start exactly as k_keys did
     // (same inputs, same arithmetic), avoiding a 64-bit division of the key
     if (p < n) {
-        const unsigned long long k = keys[p];
-        f = (p == 0 || k != keys[p - 1]);
+        const unsigned long long k = keys.key(p);
+        f = (p == 0 || k != keys.key(p - 1));
         const double2 t = st[p];
         b = bin_of(g, t.x);
         const long long bp = p == 0 ? -1 : (long long)bin_of(g, st[p - 1].x);
@@ -268,15 +286,15 @@ __global__ void __launch_bounds__(BT) k_count_cells(const unsigned long long* __
     if (threadIdx.x == 0 && c) atomicAdd(count, (unsigned long long)c);
 }
 
-__global__ void __launch_bounds__(BT) k_insert(const unsigned long long* __restrict__ keys,
+__global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
                                               size_t n, HashTable ht) {
     size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
     if (p >= n) return;
-    unsigned long long k = keys[p];
-    if (p != 0 && keys[p - 1] == k) return;
+    unsigned long long k = keys.key(p);
+    if (p != 0 && keys.key(p - 1) == k) return;
     // the cell's run ends at the next key change (most cells hold 1-3 entries)
     size_t e = p + 1;
-    while (e < n && keys[e] == k) ++e;
+    while (e < n && keys.key(e) == k) ++e;
     const unsigned long long bmask = ht.mask >> 2;
     unsigned long long b = bucket_of(k >> 2, ht.log2cap);
     // try the slot matching the key's position in its group first: the (up
@@ -502,15 +520,26 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     for (int a = 0; a < 3; ++a) idx->max_ext[a] = hb.ext[a];
 
     // 3-4. keys + sort
-    DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
-    DevBuf<uint32_t> ids(n, s), ids_tmp(n, s);
-    k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p);
-    DTS_LAUNCH_CHECK();
     const unsigned long long max_key = (unsigned long long)g.m * g.cells_per_bin - 1ull;
     idx->key_bits = bits_for(max_key);
-    radix_sort_pairs(keys.p, ids.p, keys_tmp.p, ids_tmp.p, n, idx->key_bits, s);
-    keys_tmp.release();
-    ids_tmp.release();
+    const int row_bits = std::max(1, bits_for(n - 1));
+    const bool packed = row_bits + idx->key_bits <= 64;
+    DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
+    DevBuf<uint32_t> ids(packed ? 0 : n, s), ids_tmp(packed ? 0 : n, s);
+    k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p, row_bits);
+    DTS_LAUNCH_CHECK();
+    SortedKeys sk;
+    if (packed) {   // keys-only sort of the key bits; rows ride in the low bits
+        sk.a = radix_sort_keys(keys.p, keys_tmp.p, n, row_bits, row_bits + idx->key_bits, s);
+        sk.shift = row_bits;
+        sk.ids = nullptr;
+    } else {
+        radix_sort_pairs(keys.p, ids.p, keys_tmp.p, ids_tmp.p, n, idx->key_bits, s);
+        ids_tmp.release();
+        sk.a = keys.p;
+        sk.shift = 0;
+        sk.ids = ids.p;
+    }
 
     // 5. gather into the SoA layout
     const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
@@ -532,14 +561,13 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
-    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, ids.p,
-                                                                         idx->soa);
+    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, sk, idx->soa);
     DTS_LAUNCH_CHECK();
 
     // 6. non-empty cells -> hash table
     DevBuf<unsigned long long> ncell(1, s);
     DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
-    k_count_cells<<<grid_for(n), BT, 0, s>>>(keys.p, n, g, idx->soa.st, idx->bin_start, b0, b1,
+    k_count_cells<<<grid_for(n), BT, 0, s>>>(sk, n, g, idx->soa.st, idx->bin_start, b0, b1,
                                              ncell.p);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
@@ -554,13 +582,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     idx->ht.mask = (1ull << log2cap) - 1;
     idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
-    k_insert<<<grid_for(n), BT, 0, s>>>(keys.p, n, idx->ht);
+    k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
     DTS_LAUNCH_CHECK();
 
     // 7. GPUSpatioTemporal subbin arrays (DTS_METHOD_SUBBIN)
     idx->method = p.method;
     if (p.method == DTS_METHOD_SUBBIN) {
         keys.release();
+        keys_tmp.release();
         ids.release();
         build_subbins(idx, D, n, hb, p, s);
     }

@@ -197,6 +197,13 @@ void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size
 void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s);
 
+// Stable LSD radix sort of u64 keys on bits [lo, hi) only (keys-only: a
+// payload packed in the bits below lo rides along untouched; since the input
+// is in payload order, sorting on [lo, hi) equals a stable sort by the key).
+// Returns the buffer (keys or tmp) that holds the sorted keys.
+unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long* tmp, size_t n,
+                                    int lo, int hi, cudaStream_t s);
+
 int bits_for(unsigned long long max_value);
 
 // Device block cache (alloc.cu) for memory that outlives one API call.

@@ -188,7 +188,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         size_t idx = wbase + (size_t)i * 32 + lane;
         bool ok = idx < n;
         k[i] = ok ? keys[idx] : 0ull;
-        v[i] = ok ? vals[idx] : 0u;
+        v[i] = (ok && vals) ? vals[idx] : 0u;     // keys-only sorts pass vals == nullptr
         dig[i] = ok ? ((uint32_t)(k[i] >> shift) & (RADIX - 1)) : (uint32_t)RADIX;
     }
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -261,7 +261,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         const uint32_t dg = (uint32_t)(key >> shift) & (RADIX - 1);
         const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
         keys_out[dst] = key;
-        vals_out[dst] = sv[i];
+        if (vals_out) vals_out[dst] = sv[i];
     }
 }
 
@@ -277,6 +277,22 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
     DTS_LAUNCH_CHECK();
 }
 }  // namespace
+
+unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long* tmp, size_t n,
+                                    int lo, int hi, cudaStream_t s) {
+    if (n <= 1 || hi <= lo) return keys;
+    const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
+    const size_t ncount = (size_t)256 * ntiles;
+    DevBuf<uint32_t> counts(ncount, s), offs(ncount + 1, s);
+    unsigned long long *kin = keys, *kout = tmp;
+    for (int shift = lo; shift < hi; shift += 8) {
+        radix_pass<8>(kin, nullptr, kout, nullptr, n, shift, ntiles, counts.p, offs.p, s);
+        unsigned long long* t = kin;
+        kin = kout;
+        kout = t;
+    }
+    return kin;
+}
 
 void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
