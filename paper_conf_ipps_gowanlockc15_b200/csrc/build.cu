@@ -22,6 +22,7 @@
 //                     entry is in exactly one cell).
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 
 #include "internal.cuh"
 
@@ -523,7 +524,11 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     const unsigned long long max_key = (unsigned long long)g.m * g.cells_per_bin - 1ull;
     idx->key_bits = bits_for(max_key);
     const int row_bits = std::max(1, bits_for(n - 1));
-    const bool packed = row_bits + idx->key_bits <= 64;
+    static const bool allow_packed = [] {       // DTS_PACKED_SORT=0: (key, id) pairs
+        const char* e = getenv("DTS_PACKED_SORT");
+        return !(e && e[0] == '0');
+    }();
+    const bool packed = allow_packed && row_bits + idx->key_bits <= 64;
     DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
     DevBuf<uint32_t> ids(packed ? 0 : n, s), ids_tmp(packed ? 0 : n, s);
     k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p, row_bits);
