@@ -194,7 +194,16 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     const uint32_t lt_mask = (1u << lane) - 1u;
 #pragma unroll
     for (int i = 0; i < RS_ITEMS; ++i) {
-        uint32_t peers = __match_any_sync(0xffffffffu, dig[i]);
+        // lanes holding the same digit: BITS ballots (warp multi-split); the
+        // match.any instruction it replaces was the kernel's bottleneck
+        // (ncu: 33% of stall samples waiting on it)
+        uint32_t peers = __ballot_sync(0xffffffffu, dig[i] < (uint32_t)RADIX);
+#pragma unroll
+        for (int b = 0; b < BITS; ++b) {
+            const uint32_t bal = __ballot_sync(0xffffffffu, (dig[i] >> b) & 1u);
+            peers &= ((dig[i] >> b) & 1u) ? bal : ~bal;
+        }
+        if (dig[i] >= (uint32_t)RADIX) peers = 1u << lane;   // sentinel lanes: alone
         int leader = __ffs(peers) - 1;
         uint32_t old = 0;
         if (lane == leader) {
