@@ -1,0 +1,39 @@
+"""Small workloads through every kernel path, for compute-sanitizer
+(memcheck / racecheck / synccheck)."""
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import paper_conf_ipps_gowanlockc15_b200 as dts  # noqa: E402
+import synth  # noqa: E402
+
+c = synth.make_config("C0")
+for method in ("grid", "temporal", "subbin"):
+    idx = dts.build_index(c.D, method=method, entry_traj=c.etraj)
+    for d in (0.0, 0.05, 0.3):
+        dts.search(idx, c.Q, d)
+    dts.search_ex(idx, c.Q, 0.2, query_traj=c.qtraj, exclude_same_trajectory=True)
+    idx.free()
+# heavy output (recompute + radix canonicalisation path)
+g = np.random.default_rng(1)
+D = np.zeros((1500, 8))
+D[:, 4] = 1.0
+D[:, 1:4] = g.uniform(0, 0.02, size=(1500, 3))
+D[:, 5:8] = D[:, 1:4]
+Q = D[:20].copy()
+idx = dts.build_index(D)
+r = dts.search(idx, Q, 0.05)
+# device API, trajectory merge, canonicalise
+Dd = torch.from_numpy(c.D).cuda()
+Qd = torch.from_numpy(c.Q).cuda()
+idx = dts.build_index_device(Dd)
+res, _ = dts.search_device(idx, Qd, 0.2)
+m = dts.merge_trajectories_device(res, torch.from_numpy(c.qtraj).cuda(),
+                                  torch.from_numpy(c.etraj).cuda())
+t = res.tensor().clone()
+dts.canonicalize_device(t)
+print("sanitize workload ok", r.shape[0], res.count, m.count, flush=True)
