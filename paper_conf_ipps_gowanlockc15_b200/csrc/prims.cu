@@ -206,7 +206,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         if (dig[i] >= (uint32_t)RADIX) peers = 1u << lane;   // sentinel lanes: alone
         int leader = __ffs(peers) - 1;
         uint32_t old = 0;
-        if (lane == leader) {
+        if (lane == leader && dig[i] < (uint32_t)RADIX) {
             old = wcnt[warp][dig[i]];
             wcnt[warp][dig[i]] = old + __popc(peers);
         }
