@@ -595,10 +595,13 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         // DTS_TILE_OCC = 6 | 8: 85 or 64 registers per thread)
         static const int occ = [] {
             const char* e = getenv("DTS_TILE_OCC");
-            return (e && atoi(e) == 8) ? 8 : 6;
+            const int v = e ? atoi(e) : 6;
+            return (v == 5 || v == 7 || v == 8) ? v : 6;
         }();
         const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
         if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);
         else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);
         DTS_LAUNCH_CHECK();
     }
