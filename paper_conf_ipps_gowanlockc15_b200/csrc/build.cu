@@ -161,34 +161,39 @@ __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
 }
 
-constexpr int GATHER_ITEMS = 2;   // rows in flight per thread
-
-// Sorted position p <- original row ids[p]: GATHER_ITEMS positions per thread
+// Sorted position p <- original row ids[p]: ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first.
+// STREAM: evict-first loads of the read-once rows.  Variants are selectable
+// with DTS_GATHER=<items><s|n> for tuning (default 2n, measured best).
+template <int ITEMS, bool STREAM>
 __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
                                               const SortedKeys sk, SegSoA soa) {
-    const size_t base = (size_t)blockIdx.x * BT * GATHER_ITEMS + threadIdx.x;
-    uint32_t id[GATHER_ITEMS];
-    double4 r0[GATHER_ITEMS], r1[GATHER_ITEMS];
+    const size_t base = (size_t)blockIdx.x * BT * ITEMS + threadIdx.x;
+    uint32_t id[ITEMS];
+    double4 r0[ITEMS], r1[ITEMS];
 #pragma unroll
-    for (int k = 0; k < GATHER_ITEMS; ++k) {
+    for (int k = 0; k < ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
         id[k] = p < n ? sk.row(p) : 0u;
     }
 #pragma unroll
-    for (int k = 0; k < GATHER_ITEMS; ++k) {
+    for (int k = 0; k < ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
         if (p < n) {
-            // read-once rows: streaming (evict-first) loads
-            const double2* row = reinterpret_cast<const double2*>(D + 2 * (size_t)id[k]);
-            const double2 a0 = __ldcs(row), a1 = __ldcs(row + 1);
-            const double2 a2 = __ldcs(row + 2), a3 = __ldcs(row + 3);
-            r0[k] = make_double4(a0.x, a0.y, a1.x, a1.y);
-            r1[k] = make_double4(a2.x, a2.y, a3.x, a3.y);
+            if (STREAM) {
+                const double2* row = reinterpret_cast<const double2*>(D + 2 * (size_t)id[k]);
+                const double2 a0 = __ldcs(row), a1 = __ldcs(row + 1);
+                const double2 a2 = __ldcs(row + 2), a3 = __ldcs(row + 3);
+                r0[k] = make_double4(a0.x, a0.y, a1.x, a1.y);
+                r1[k] = make_double4(a2.x, a2.y, a3.x, a3.y);
+            } else {
+                r0[k] = D[2 * (size_t)id[k]];
+                r1[k] = D[2 * (size_t)id[k] + 1];
+            }
         }
     }
 #pragma unroll
-    for (int k = 0; k < GATHER_ITEMS; ++k) {
+    for (int k = 0; k < ITEMS; ++k) {
         const size_t p = base + (size_t)k * BT;
         if (p < n) {
             const double4 s0 = r0[k], s1 = r1[k];
@@ -566,7 +571,25 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
-    k_gather<<<grid_for((n + GATHER_ITEMS - 1) / GATHER_ITEMS), BT, 0, s>>>(D, n, sk, idx->soa);
+    {
+        static const int gv = [] {          // DTS_GATHER: 1n 2n 4n 1s 2s 4s
+            const char* e = getenv("DTS_GATHER");
+            if (!e || !e[0]) return 20;
+            const int items = e[0] - '0';
+            const int st = e[1] == 's' ? 1 : 0;
+            return ((items == 1 || items == 2 || items == 4) ? items : 2) * 10 + st;
+        }();
+        const int items = gv / 10;
+        const unsigned gb = grid_for((n + items - 1) / items);
+        switch (gv) {
+            case 10: k_gather<1, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+            case 11: k_gather<1, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+            case 21: k_gather<2, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+            case 40: k_gather<4, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+            case 41: k_gather<4, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+            default: k_gather<2, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
+        }
+    }
     DTS_LAUNCH_CHECK();
 
     // 6. non-empty cells -> hash table

@@ -592,7 +592,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
         const unsigned want = (ntiles + WW - 1) / WW;
         // CTAs per SM the kernel is register-bounded for (tuning knob
-        // DTS_TILE_OCC = 6 | 8: 85 or 64 registers per thread)
+        // DTS_TILE_OCC = 5..8: 102, 85, 73 or 64 registers per thread)
         static const int occ = [] {
             const char* e = getenv("DTS_TILE_OCC");
             // measured on C4 (one box, 20 steps): 5: 0.97 ms, 6: 1.00, 7: 0.86, 8: 0.92
