@@ -5,6 +5,7 @@
 // These implement the "radix sort and prefix scan" of the index builder
 // (BASELINE.json north_star) and the exclusive scan of
 // per-query result counts of the two-pass compaction (§8(a6)).
+#include <algorithm>
 #include <cstdlib>
 
 #include "internal.cuh"
@@ -160,11 +161,13 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_hist(const unsigned long long
 // warp-private digit counters; a cross-warp prefix per digit then orders the
 // chunks.  The tile is staged in digit order in shared memory and written
 // out with consecutive threads on consecutive output positions.
-template <int BITS>
+template <int BITS, bool VALS>
 __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ offsets, uint32_t ntiles,
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
+    // VALS = false: keys-only (packed) sort -- no value registers or staging,
+    // so more CTAs fit per SM to hide the key-load latency
     constexpr int RADIX = 1 << BITS;
     constexpr int DPT = RADIX / RS_THREADS;       // digits per thread (1 or 2)
     static_assert(DPT >= 1 && RADIX % RS_THREADS == 0, "RADIX must be a multiple of the CTA");
@@ -173,7 +176,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
     __shared__ uint32_t local_off[RADIX];
     __shared__ uint32_t warp_tot[RS_WARPS];
     __shared__ unsigned long long sk[RS_TILE];
-    __shared__ uint32_t sv[RS_TILE];
+    __shared__ uint32_t sv[VALS ? RS_TILE : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int j = lane; j < RADIX + 1; j += 32) wcnt[warp][j] = 0;
     for (int j = threadIdx.x; j < RADIX; j += RS_THREADS)
@@ -188,7 +191,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         size_t idx = wbase + (size_t)i * 32 + lane;
         bool ok = idx < n;
         k[i] = ok ? keys[idx] : 0ull;
-        v[i] = (ok && vals) ? vals[idx] : 0u;     // keys-only sorts pass vals == nullptr
+        v[i] = (VALS && ok) ? vals[idx] : 0u;
         dig[i] = ok ? ((uint32_t)(k[i] >> shift) & (RADIX - 1)) : (uint32_t)RADIX;
     }
     const uint32_t lt_mask = (1u << lane) - 1u;
@@ -257,7 +260,7 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         if (dig[i] < (uint32_t)RADIX) {
             const uint32_t lpos = local_off[dig[i]] + wcnt[warp][dig[i]] + rank[i];
             sk[lpos] = k[i];
-            sv[lpos] = v[i];
+            if (VALS) sv[lpos] = v[i];
         }
     }
     __syncthreads();
@@ -270,7 +273,234 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_scatter(
         const uint32_t dg = (uint32_t)(key >> shift) & (RADIX - 1);
         const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
         keys_out[dst] = key;
-        if (vals_out) vals_out[dst] = sv[i];
+        if (VALS) vals_out[dst] = sv[i];
+    }
+}
+
+// ------------------------------------------------------------ onesweep
+// One kernel per 8-bit pass.  Tiles take their ids in launch order from an
+// atomic counter, rank their keys as k_rs_scatter does, publish their digit
+// counts and find their global offsets by decoupled look-back over the
+// preceding tiles' published counts; the digit bases come from one histogram
+// of all passes computed up front (k_rs_hist_all, or fused into the kernel
+// that produced the keys).  A pass then reads and writes the keys once,
+// where hist + scan + scatter reads them twice and adds two launches.
+constexpr int OS_ITEMS = 12;
+constexpr int OS_TILE = RS_THREADS * OS_ITEMS;    // 3072 keys per tile
+constexpr uint32_t OS_AGG = 1u << 30;             // status word: count of this tile only
+constexpr uint32_t OS_PRE = 2u << 30;             // status word: inclusive prefix
+constexpr uint32_t OS_VAL = OS_AGG - 1u;
+constexpr int OS_LB = 8;                          // look-back window
+
+__device__ __forceinline__ uint32_t ld_relaxed(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_relaxed(uint32_t* p, uint32_t v) {
+    asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// Digit histograms of all passes (digits at bits lo + 8 p, p < npass) in one
+// read of the keys; hist[p * 256 + digit] is accumulated (caller zeroes it).
+__global__ void __launch_bounds__(RS_THREADS) k_rs_hist_all(const unsigned long long* __restrict__ keys,
+                                                            size_t n, int lo, int npass,
+                                                            uint32_t* __restrict__ hist) {
+    __shared__ uint32_t h[8 * 256];
+    for (int j = threadIdx.x; j < 8 * 256; j += RS_THREADS) h[j] = 0;
+    __syncthreads();
+    for (size_t i = (size_t)blockIdx.x * RS_THREADS + threadIdx.x; i < n;
+         i += (size_t)gridDim.x * RS_THREADS) {
+        const unsigned long long k = keys[i];
+        for (int p = 0; p < npass; ++p) atomicAdd(&h[p * 256 + ((k >> (lo + 8 * p)) & 255u)], 1u);
+    }
+    __syncthreads();
+    for (int j = threadIdx.x; j < npass * 256; j += RS_THREADS)
+        if (h[j]) atomicAdd(hist + j, h[j]);
+}
+
+// Exclusive scan of each pass's 256 digit counts, in place (one CTA per pass).
+__global__ void __launch_bounds__(RS_THREADS) k_rs_hist_scan(uint32_t* __restrict__ hist) {
+    uint32_t* h = hist + (size_t)blockIdx.x * 256;
+    const uint32_t c = h[threadIdx.x];
+    uint32_t total;
+    const uint32_t ex = block_exclusive_scan<uint32_t>(c, &total);
+    h[threadIdx.x] = ex;
+}
+
+template <bool VALS, int MINB>
+__global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
+    const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
+    int shift, const uint32_t* __restrict__ gbase, uint32_t* status, uint32_t* tile_ctr,
+    unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
+    constexpr int RADIX = 256;
+    static_assert(RADIX == RS_THREADS, "one digit per thread");
+    __shared__ uint32_t wcnt[RS_WARPS][RADIX + 1];
+    __shared__ uint32_t tile_base[RADIX];
+    __shared__ uint32_t local_off[RADIX];
+    __shared__ uint32_t warp_tot[RS_WARPS];
+    __shared__ uint32_t s_tile;
+    __shared__ unsigned long long sk[OS_TILE];
+    __shared__ uint32_t sv[VALS ? OS_TILE : 1];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
+    for (int j = lane; j < RADIX + 1; j += 32) wcnt[warp][j] = 0;
+    __syncthreads();
+    const uint32_t tile = s_tile;
+
+    // ---- load and rank (warp w owns a contiguous chunk of 32 * OS_ITEMS keys)
+    const size_t wbase = (size_t)tile * OS_TILE + (size_t)warp * (32 * OS_ITEMS);
+    unsigned long long k[OS_ITEMS];
+    uint32_t v[VALS ? OS_ITEMS : 1];
+    uint32_t dr[OS_ITEMS];                       // digit | rank << 9; digit RADIX: past the end
+#pragma unroll
+    for (int i = 0; i < OS_ITEMS; ++i) {
+        const size_t idx = wbase + (size_t)i * 32 + lane;
+        const bool ok = idx < n;
+        k[i] = ok ? keys[idx] : 0ull;
+        if (VALS) v[i] = ok ? vals[idx] : 0u;
+        dr[i] = ok ? ((uint32_t)(k[i] >> shift) & (RADIX - 1)) : (uint32_t)RADIX;
+    }
+    const uint32_t lt_mask = (1u << lane) - 1u;
+#pragma unroll
+    for (int i = 0; i < OS_ITEMS; ++i) {
+        const uint32_t dig = dr[i];
+        uint32_t peers = __ballot_sync(0xffffffffu, dig < (uint32_t)RADIX);
+#pragma unroll
+        for (int b = 0; b < 8; ++b) {
+            const uint32_t bal = __ballot_sync(0xffffffffu, (dig >> b) & 1u);
+            peers &= ((dig >> b) & 1u) ? bal : ~bal;
+        }
+        if (dig >= (uint32_t)RADIX) peers = 1u << lane;
+        const int leader = __ffs(peers) - 1;
+        uint32_t old = 0;
+        if (lane == leader && dig < (uint32_t)RADIX) {
+            old = wcnt[warp][dig];
+            wcnt[warp][dig] = old + __popc(peers);
+        }
+        old = __shfl_sync(0xffffffffu, old, leader);
+        dr[i] = dig | ((old + __popc(peers & lt_mask)) << 9);
+        __syncwarp();
+    }
+    __syncthreads();
+
+    // ---- thread t owns digit t: cross-warp prefix, then look-back
+    const int t = threadIdx.x;
+    uint32_t count = 0;
+#pragma unroll
+    for (int w = 0; w < RS_WARPS; ++w) {
+        const uint32_t c = wcnt[w][t];
+        wcnt[w][t] = count;
+        count += c;
+    }
+    uint32_t excl = 0;
+    uint32_t* mine = status + (size_t)tile * RADIX + t;
+    if (tile == 0) {
+        st_relaxed(mine, OS_PRE | count);
+    } else {
+        st_relaxed(mine, OS_AGG | count);
+        // windowed look-back: OS_LB predecessors per round trip (in the first
+        // wave every tile has only aggregates behind it; one tile per round
+        // trip would serialise the wave)
+        int32_t j = (int32_t)tile - 1;              // next predecessor to account for
+        bool done = false;
+        while (!done) {
+            uint32_t w[OS_LB];
+#pragma unroll
+            for (int q = 0; q < OS_LB; ++q)
+                w[q] = j - q >= 0 ? ld_relaxed(status + (size_t)(j - q) * RADIX + t) : OS_PRE;
+#pragma unroll
+            for (int q = 0; q < OS_LB; ++q) {
+                if (done) break;
+                if (w[q] == 0u) break;               // not published yet: poll again from j
+                excl += w[q] & OS_VAL;
+                --j;
+                if (w[q] & OS_PRE) done = true;
+            }
+        }
+        st_relaxed(mine, OS_PRE | (excl + count));
+    }
+    tile_base[t] = gbase[t] + excl;
+    {   // tile-local digit offsets
+        uint32_t inc = count;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += u;
+        }
+        if (lane == 31) warp_tot[warp] = inc;
+        __syncthreads();
+        uint32_t pre = 0;
+        for (int w = 0; w < warp; ++w) pre += warp_tot[w];
+        local_off[t] = pre + inc - count;
+    }
+    __syncthreads();
+    // ---- stage in digit order, write out coalesced
+#pragma unroll
+    for (int i = 0; i < OS_ITEMS; ++i) {
+        const uint32_t dig = dr[i] & 511u;
+        if (dig < (uint32_t)RADIX) {
+            const uint32_t lpos = local_off[dig] + wcnt[warp][dig] + (dr[i] >> 9);
+            sk[lpos] = k[i];
+            if (VALS) sv[lpos] = v[i];
+        }
+    }
+    __syncthreads();
+    const size_t tbase = (size_t)tile * OS_TILE;
+    const uint32_t tn = (uint32_t)min((size_t)OS_TILE, n - tbase);
+    for (uint32_t i = threadIdx.x; i < tn; i += RS_THREADS) {
+        const unsigned long long key = sk[i];
+        const uint32_t dg = (uint32_t)(key >> shift) & (RADIX - 1);
+        const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
+        keys_out[dst] = key;
+        if (VALS) vals_out[dst] = sv[i];
+    }
+}
+
+bool onesweep_enabled(size_t n) {
+    static const bool on = [] {                  // DTS_ONESWEEP=0: hist + scan + scatter
+        const char* e = getenv("DTS_ONESWEEP");
+        return !(e && e[0] == '0');
+    }();
+    return on && n < (size_t)OS_VAL;
+}
+
+// npass onesweep passes over digits at bits lo + 8 p; hist holds each pass's
+// exclusive digit bases (k_rs_hist_scan).  Returns the pass count's parity
+// buffers swapped: on return *kin / *vin hold the result.
+void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32_t** vin,
+                     uint32_t** vout, size_t n, int lo, int npass, const uint32_t* hist,
+                     cudaStream_t s) {
+    const uint32_t ntiles = (uint32_t)((n + OS_TILE - 1) / OS_TILE);
+    const size_t nstat = (size_t)ntiles * 256 + 32;
+    DevBuf<uint32_t> status(nstat, s);
+    for (int p = 0; p < npass; ++p) {
+        DTS_CUDA(cudaMemsetAsync(status.p, 0, nstat * sizeof(uint32_t), s));
+        uint32_t* ctr = status.p + (size_t)ntiles * 256;
+        static const int occ = [] {            // DTS_OS_OCC: CTAs/SM bound, keys-only
+            const char* e = getenv("DTS_OS_OCC");
+            const int v = e ? atoi(e) : 4;
+            return (v == 5 || v == 6) ? v : 4;
+        }();
+        if (*vin)
+            k_onesweep<true, 2><<<ntiles, RS_THREADS, 0, s>>>(*kin, *vin, n, lo + 8 * p,
+                                                             hist + 256 * p, status.p, ctr, *kout,
+                                                             *vout);
+        else if (occ == 5)
+            k_onesweep<false, 5><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
+                                                              hist + 256 * p, status.p, ctr,
+                                                              *kout, nullptr);
+        else if (occ == 6)
+            k_onesweep<false, 6><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
+                                                              hist + 256 * p, status.p, ctr,
+                                                              *kout, nullptr);
+        else
+            k_onesweep<false, 4><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
+                                                              hist + 256 * p, status.p, ctr,
+                                                              *kout, nullptr);
+        DTS_LAUNCH_CHECK();
+        std::swap(*kin, *kout);
+        std::swap(*vin, *vout);
     }
 }
 
@@ -282,7 +512,12 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
     k_rs_hist<BITS><<<ntiles, RS_THREADS, 0, s>>>(kin, n, shift, counts, ntiles);
     DTS_LAUNCH_CHECK();
     scan_exclusive_u32_to_u32(counts, offs, ncount, s);
-    k_rs_scatter<BITS><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs, ntiles, kout, vout);
+    if (vin)
+        k_rs_scatter<BITS, true><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs, ntiles,
+                                                               kout, vout);
+    else
+        k_rs_scatter<BITS, false><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, offs, ntiles,
+                                                                kout, vout);
     DTS_LAUNCH_CHECK();
 }
 }  // namespace
@@ -290,6 +525,20 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
 unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long* tmp, size_t n,
                                     int lo, int hi, cudaStream_t s) {
     if (n <= 1 || hi <= lo) return keys;
+    if (onesweep_enabled(n)) {
+        const int npass = (hi - lo + 7) / 8;
+        DevBuf<uint32_t> hist((size_t)npass * 256, s);
+        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)npass * 256 * sizeof(uint32_t), s));
+        const unsigned hb = (unsigned)std::min<size_t>((n + RS_THREADS - 1) / RS_THREADS, 148 * 8);
+        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, lo, npass, hist.p);
+        DTS_LAUNCH_CHECK();
+        k_rs_hist_scan<<<npass, RS_THREADS, 0, s>>>(hist.p);
+        DTS_LAUNCH_CHECK();
+        unsigned long long *kin = keys, *kout = tmp;
+        uint32_t *vin = nullptr, *vout = nullptr;
+        onesweep_passes(&kin, &kout, &vin, &vout, n, lo, npass, hist.p, s);
+        return kin;
+    }
     const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
     const size_t ncount = (size_t)256 * ntiles;
     DevBuf<uint32_t> counts(ncount, s), offs(ncount + 1, s);
@@ -306,6 +555,25 @@ unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long
 void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long long* keys_tmp,
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
     if (n <= 1 || nbits <= 0) return;
+    if (onesweep_enabled(n)) {
+        const int npass = (nbits + 7) / 8;
+        DevBuf<uint32_t> hist((size_t)npass * 256, s);
+        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)npass * 256 * sizeof(uint32_t), s));
+        const unsigned hb = (unsigned)std::min<size_t>((n + RS_THREADS - 1) / RS_THREADS, 148 * 8);
+        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, 0, npass, hist.p);
+        DTS_LAUNCH_CHECK();
+        k_rs_hist_scan<<<npass, RS_THREADS, 0, s>>>(hist.p);
+        DTS_LAUNCH_CHECK();
+        unsigned long long *kin = keys, *kout = keys_tmp;
+        uint32_t *vin = vals, *vout = vals_tmp;
+        onesweep_passes(&kin, &kout, &vin, &vout, n, 0, npass, hist.p, s);
+        if (npass & 1) {
+            DTS_CUDA(cudaMemcpyAsync(keys, kin, n * sizeof(unsigned long long),
+                                     cudaMemcpyDeviceToDevice, s));
+            DTS_CUDA(cudaMemcpyAsync(vals, vin, n * sizeof(uint32_t), cudaMemcpyDeviceToDevice, s));
+        }
+        return;
+    }
     // 8-bit digits: measured on C4 (35-bit keys) the 9-bit variant's 4 passes
     // cost more than 5 8-bit passes (45 KB of shared memory per CTA lowers
     // occupancy; 113 vs 80 us per pass at 20 M keys).  DTS_RADIX_BITS=9 opts in.

@@ -172,17 +172,28 @@ __device__ __forceinline__ Stencil make_stencil(const GridParams& g, const QStat
     // P:L76) does not overlap the query strictly: exact comparisons, so no
     // candidate is lost (on synchronised timesteps this removes the previous
     // step's bin, whose segments only touch the query at q.t0)
-    while (s.lb <= s.hb &&
-           !(__ldg(&bin_t0min[s.lb]) < q.t1 && __ldg(&bin_t1max[s.lb]) > q.t0)) ++s.lb;
-    while (s.hb >= s.lb &&
-           !(__ldg(&bin_t0min[s.hb]) < q.t1 && __ldg(&bin_t1max[s.hb]) > q.t0)) --s.hb;
+    // (the end bins' extents and the bin_start values the usual outcomes need
+    //  -- each end kept or moved by one bin -- are loaded together: one memory
+    //  round trip instead of three dependent ones)
+    const int32_t lb0 = s.lb, hb0 = s.hb;
+    double l0 = __ldg(&bin_t0min[lb0]), l1 = __ldg(&bin_t1max[lb0]);
+    double h0 = __ldg(&bin_t0min[hb0]), h1 = __ldg(&bin_t1max[hb0]);
+    const uint32_t bs_l0 = __ldg(&bin_start[lb0]), bs_l1 = __ldg(&bin_start[lb0 + 1]);
+    const uint32_t bs_h0 = __ldg(&bin_start[hb0]), bs_h1 = __ldg(&bin_start[hb0 + 1]);
+    while (s.lb <= s.hb && !(l0 < q.t1 && l1 > q.t0)) {
+        if (++s.lb <= s.hb) { l0 = __ldg(&bin_t0min[s.lb]); l1 = __ldg(&bin_t1max[s.lb]); }
+    }
     if (s.lb > s.hb) {
         s.lb = s.hb = 0;
         return s;
     }
+    while (s.hb > s.lb && !(h0 < q.t1 && h1 > q.t0)) {
+        if (--s.hb > s.lb) { h0 = __ldg(&bin_t0min[s.hb]); h1 = __ldg(&bin_t1max[s.hb]); }
+    }
     // the bins' contiguous entry range: GPUTemporal's E_k
-    const uint32_t b0 = __ldg(&bin_start[s.lb]);
-    const uint32_t T = __ldg(&bin_start[s.hb + 1]) - b0;
+    const uint32_t b0 = s.lb == lb0 ? bs_l0 : (s.lb == lb0 + 1 ? bs_l1 : __ldg(&bin_start[s.lb]));
+    const uint32_t b1 = s.hb == hb0 ? bs_h1 : (s.hb == hb0 - 1 ? bs_h0 : __ldg(&bin_start[s.hb + 1]));
+    const uint32_t T = b1 - b0;
     if (T == 0) return s;                                  // no entry in these bins
     s.mode = MODE_TEMPORAL;
     s.nlook = 1;
@@ -262,7 +273,9 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     const uint32_t r = loc % nzy;
     const int32_t cz = clo[2] + (int32_t)(r / (uint32_t)cn[1]);
     const int32_t cy = clo[1] + (int32_t)(r % (uint32_t)cn[1]);
-    if (!(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0)) return;
+    // interior bins only: the end bins were checked by make_stencil
+    if (bin != lb && bin != hb && !(__ldg(&bin_t0min[bin]) < qt1 && __ldg(&bin_t1max[bin]) > qt0))
+        return;
     const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
     const unsigned long long kend = key0 + (unsigned long long)cn[0];   // row keys [key0, kend)
     const ulonglong2* slots = reinterpret_cast<const ulonglong2*>(ht.slots);
@@ -311,7 +324,7 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
 // --------------------------------------------------------------- query prep
 __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uint32_t nq,
                                              GridParams g, unsigned long long* __restrict__ keys,
-                                             uint32_t* __restrict__ ids,
+                                             uint32_t* __restrict__ ids, int shift,
                                              Counters* __restrict__ ctr) {
     uint32_t i = blockIdx.x * PT + threadIdx.x;
     if (i >= nq) return;
@@ -334,8 +347,19 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
     if (!bad)
         key = make_key(g, bin_of(g, s0.x), cell_of(g, 0, 0.5 * (s0.y + s1.y)),
                        cell_of(g, 1, 0.5 * (s0.z + s1.z)), cell_of(g, 2, 0.5 * (s0.w + s1.w)));
-    keys[i] = key;
-    ids[i] = i;
+    if (ids) {
+        keys[i] = key;
+        ids[i] = i;
+    } else {                        // packed: (key, row) in one word, keys-only sort
+        keys[i] = (key << shift) | i;
+    }
+}
+
+__global__ void __launch_bounds__(PT) k_unpack_order(const unsigned long long* __restrict__ keys,
+                                                    uint32_t n, unsigned long long mask,
+                                                    uint32_t* __restrict__ order) {
+    const uint32_t i = blockIdx.x * PT + threadIdx.x;
+    if (i < n) order[i] = (uint32_t)(keys[i] & mask);
 }
 
 // ------------------------------------------------------------- block helpers
@@ -545,11 +569,23 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // ---- query prep: key + sort
     DevBuf<uint32_t> order(nq, s);
     {
+        // packed (key << row bits | row) keys-only sort when it fits 64 bits
+        const int row_bits = std::max(1, bits_for(nq - 1));
+        const bool packed = row_bits + idx->key_bits <= 64;
         DevBuf<unsigned long long> qk(nq, s), qk_tmp(nq, s);
-        DevBuf<uint32_t> order_tmp(nq, s);
-        k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p, order.p, ctr.p);
+        k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p,
+                                             packed ? nullptr : order.p, row_bits, ctr.p);
         DTS_LAUNCH_CHECK();
-        radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
+        if (packed) {
+            const unsigned long long* sorted =
+                radix_sort_keys(qk.p, qk_tmp.p, nq, row_bits, row_bits + idx->key_bits, s);
+            k_unpack_order<<<blocks(nq, PT), PT, 0, s>>>(sorted, (uint32_t)nq,
+                                                        (1ull << row_bits) - 1ull, order.p);
+            DTS_LAUNCH_CHECK();
+        } else {
+            DevBuf<uint32_t> order_tmp(nq, s);
+            radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
+        }
     }
     tm.mark();
 
@@ -599,11 +635,16 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             const int v = e ? atoi(e) : 7;
             return (v == 5 || v == 6 || v == 8) ? v : 7;
         }();
+        static const bool pf = [] {        // DTS_PREFETCH=1: L2 prefetch of the next
+            const char* e = getenv("DTS_PREFETCH");   // round's buckets (measured slower
+            return e && e[0] == '1';                 // on C4: 0.85 vs 0.81 ms)
+        }();
         const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
-        if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);
-        else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);
+        if (pf) k_wtile_count<7, true><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 8) k_wtile_count<8, false><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 7) k_wtile_count<7, false><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 5) k_wtile_count<5, false><<<grid, WT, 0, s>>>(ta);
+        else k_wtile_count<6, false><<<grid, WT, 0, s>>>(ta);
         DTS_LAUNCH_CHECK();
     }
     tm.mark();

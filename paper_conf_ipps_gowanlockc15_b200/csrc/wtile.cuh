@@ -28,7 +28,7 @@ struct WarpSmem {
     uint32_t rstart[WQ], rcnt[WQ], rind[WQ];   // single-run queries (temporal / subbin)
     uint32_t qtraj[WQ];                        // trajectory ids (exclude_same_trajectory)
     unsigned long long lkoff[WQ + 1];
-    unsigned long long hkey[WH];        // (query << 42) | (entry id << 10) | slot
+    unsigned long long hkey[WH];        // (query << 42) | (position, then entry id << 10) | slot
     double h0[WH], h1[WH];
     uint32_t nhit, over;
 };
@@ -68,13 +68,14 @@ __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
     return q;
 }
 
-__device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, double r0, double r1,
-                                          const uint32_t* __restrict__ eid) {
+// The hit is staged with its sorted position p; the entry ids of all the
+// tile's hits are looked up together before ranking (one round trip per tile
+// instead of a dependent load per hit).
+__device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, double r0, double r1) {
     atomicAdd(&S.qcount[qi], 1u);
     const uint32_t pos = atomicAdd(&S.nhit, 1u);
     if (pos < (uint32_t)WH) {
-        const uint32_t e = __ldg(eid + p);
-        S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)e << 10) | pos;
+        S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)p << 10) | pos;
         S.h0[pos] = r0;
         S.h1[pos] = r1;
     } else {
@@ -82,7 +83,32 @@ __device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, doubl
     }
 }
 
-template <int MINB>
+// L2 prefetch of the home bucket(s) of probe l of the tile (issued one round
+// ahead, so that the next round's bucket loads do not wait on DRAM).
+__device__ __forceinline__ void prefetch_probe(const WarpSmem& S, const GridParams& g,
+                                               const HashTable& ht, unsigned long long l) {
+    int qi = 0;
+#pragma unroll
+    for (int step = WQ / 2; step; step >>= 1)
+        if (S.lkoff[qi + step] <= l) qi += step;
+    if (S.mode[qi] != MODE_GRID) return;
+    const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
+    const uint32_t cn1 = (uint32_t)S.cn[1][qi];
+    const uint32_t nzy = cn1 * (uint32_t)S.cn[2][qi];
+    const int32_t bin = S.lb[qi] + (int32_t)(loc / nzy);
+    const uint32_t r = loc % nzy;
+    const unsigned long long key0 = make_key(g, bin, S.clo[0][qi], S.clo[1][qi] + (int32_t)(r % cn1),
+                                             S.clo[2][qi] + (int32_t)(r / cn1));
+    const unsigned long long g0 = key0 >> 2, g1 = (key0 + (unsigned long long)S.cn[0][qi] - 1) >> 2;
+    const CellSlot* b0 = ht.slots + 4 * bucket_of(g0, ht.log2cap);
+    asm volatile("prefetch.global.L2 [%0];" ::"l"(b0));
+    if (g1 != g0) {
+        const CellSlot* b1 = ht.slots + 4 * bucket_of(g1, ht.log2cap);
+        asm volatile("prefetch.global.L2 [%0];" ::"l"(b1));
+    }
+}
+
+template <int MINB, bool PF>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -147,6 +173,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             const unsigned long long l = r0 + lane;
             uint32_t start = 0, cnt = 0, ind = 0;
             int qi = 0;
+            if (PF && l + 32 < Ltot) prefetch_probe(S, g, a.ht, l + 32);
             if (l < Ltot) {
 #pragma unroll
                 for (int step = WQ / 2; step; step >>= 1)
@@ -199,10 +226,10 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
                     const bool x2 = a.excl && __ldg(a.etraj + p2) == S.qtraj[qi2];
                     if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
-                        stage_hit(S, qi1, p1, h0, h1, a.soa.eid);
+                        stage_hit(S, qi1, p1, h0, h1);
                     if (v2 && !x2 &&
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
-                        stage_hit(S, qi2, p2, h0, h1, a.soa.eid);
+                        stage_hit(S, qi2, p2, h0, h1);
                 }
             }
         }
@@ -224,6 +251,11 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 if (lane >= o) inc += u;
             }
             if (lane < WQ) S.qoff[lane] = inc - cnt;
+            for (uint32_t i = lane; i < nh; i += 32) {      // sorted position -> entry id
+                const unsigned long long k = S.hkey[i];
+                const uint32_t e = __ldg(a.soa.eid + (uint32_t)(k >> 10));
+                S.hkey[i] = (k & ~(0xffffffffull << 10)) | ((unsigned long long)e << 10);
+            }
             unsigned long long b = 0;
             if (lane == 0) b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
             b = __shfl_sync(0xffffffffu, b, 0);
