@@ -12,11 +12,11 @@
 //   3. k_keys         key = (bin of t_start, cell of the MBB midpoint), row-major
 //                     (bin, z, y, x) so that x-adjacent cells are adjacent runs.
 //   4. radix sort     stable (key, id): within a cell entries stay in id order.
-//   5. k_gather       sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz).
-//   6. k_count_cells / k_insert
-//                     bin offsets (B_first of P:L76), per-bin [min t_start,
-//                     max t_end] extents (B_start/B_end of P:L76) with
-//                     CTA-aggregated atomics, and non-empty cells ->
+//   5. k_gather_cells sorted SoA double2 streams (t0,t1) (x0,vx) (y0,vy) (z0,vz),
+//                     fused with: bin offsets (B_first of P:L76), per-bin
+//                     [min t_start, max t_end] extents (B_start/B_end of
+//                     P:L76) with CTA-aggregated atomics, non-empty cell count.
+//   6. k_insert       non-empty cells ->
 //                     open-addressing hash table key -> [start, end) (the role
 //                     of G and A of P:L44, with no duplicated ids since every
 //                     entry is in exactly one cell).
@@ -162,39 +162,67 @@ __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
 }
 
 // Sorted position p <- original row ids[p]: ITEMS positions per thread
-// (strided by the CTA so stores stay coalesced), all row loads issued first.
-// STREAM: evict-first loads of the read-once rows.  Variants are selectable
-// with DTS_GATHER=<items><s|n> for tuning (default 2n, measured best).
-template <int ITEMS, bool STREAM>
-__global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, size_t n,
-                                              const SortedKeys sk, SegSoA soa) {
-    const size_t base = (size_t)blockIdx.x * BT * ITEMS + threadIdx.x;
+// (strided by the CTA so stores stay coalesced), all row loads issued first;
+// the velocity form of each segment is written to the SoA streams.  Fused
+// with the per-cell / per-bin bookkeeping of the sorted order (the tile's
+// keys and bins are staged in shared memory with a one-element halo):
+//   * non-empty cells are counted (key change between p - 1 and p);
+//   * bin_start[0..m] (the entries of bin j are the sorted positions
+//     [bin_start[j], bin_start[j+1]): the index range [B_first, B_last] of
+//     P:L76, keys being bin-major);
+//   * per-bin extents [min t_start, max t_end] (B_start / B_end of P:L76) with
+//     one atomic pair per CTA when the tile lies in one bin (the common case:
+//     bins hold ~10^5 entries), per element otherwise, on order-preserving
+//     integer images of the times.
+// The bin is computed with bin_of() from t_start exactly as k_keys did (same
+// inputs, same arithmetic).
+template <int ITEMS>
+__global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restrict__ D, size_t n,
+                                                    const SortedKeys sk, SegSoA soa, GridParams g,
+                                                    uint32_t* __restrict__ bin_start,
+                                                    unsigned long long* __restrict__ bin_t0min,
+                                                    unsigned long long* __restrict__ bin_t1max,
+                                                    unsigned long long* __restrict__ count) {
+    constexpr int TILE = BT * ITEMS;
+    __shared__ unsigned long long s_key[TILE + 1];
+    __shared__ int32_t s_bin[TILE + 1];
+    __shared__ unsigned long long s_o0[BT / 32], s_o1[BT / 32];
+    __shared__ uint32_t s_cnt;
+    const size_t p0 = (size_t)blockIdx.x * TILE;
     uint32_t id[ITEMS];
     double4 r0[ITEMS], r1[ITEMS];
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
-        const size_t p = base + (size_t)k * BT;
-        id[k] = p < n ? sk.row(p) : 0u;
-    }
-#pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-        const size_t p = base + (size_t)k * BT;
+        const size_t p = p0 + (size_t)k * BT + threadIdx.x;
         if (p < n) {
-            if (STREAM) {
-                const double2* row = reinterpret_cast<const double2*>(D + 2 * (size_t)id[k]);
-                const double2 a0 = __ldcs(row), a1 = __ldcs(row + 1);
-                const double2 a2 = __ldcs(row + 2), a3 = __ldcs(row + 3);
-                r0[k] = make_double4(a0.x, a0.y, a1.x, a1.y);
-                r1[k] = make_double4(a2.x, a2.y, a3.x, a3.y);
-            } else {
-                r0[k] = D[2 * (size_t)id[k]];
-                r1[k] = D[2 * (size_t)id[k] + 1];
-            }
+            id[k] = sk.row(p);
+            s_key[1 + k * BT + threadIdx.x] = sk.key(p);
+        } else {
+            id[k] = 0u;
+        }
+    }
+    if (threadIdx.x == 0) {
+        s_cnt = 0;
+        if (p0 > 0) {                                  // halo: sorted position p0 - 1
+            s_key[0] = sk.key(p0 - 1);
+            s_bin[0] = bin_of(g, D[2 * (size_t)sk.row(p0 - 1)].x);
+        } else {
+            s_key[0] = ~0ull;
+            s_bin[0] = -1;
         }
     }
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
-        const size_t p = base + (size_t)k * BT;
+        const size_t p = p0 + (size_t)k * BT + threadIdx.x;
+        if (p < n) {
+            r0[k] = D[2 * (size_t)id[k]];
+            r1[k] = D[2 * (size_t)id[k] + 1];
+        }
+    }
+    unsigned long long o0 = ~0ull, o1 = 0ull;
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const size_t p = p0 + (size_t)k * BT + threadIdx.x;
         if (p < n) {
             const double4 s0 = r0[k], s1 = r1[k];
             const double dur = s1.x - s0.x;
@@ -203,8 +231,64 @@ __global__ void __launch_bounds__(BT) k_gather(const double4* __restrict__ D, si
             soa.sy[p] = make_double2(s0.z, velocity(s0.z, s1.z, dur));
             soa.sz[p] = make_double2(s0.w, velocity(s0.w, s1.w, dur));
             soa.eid[p] = id[k];
+            s_bin[1 + k * BT + threadIdx.x] = bin_of(g, s0.x);
+            const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);
+            o0 = a < o0 ? a : o0;
+            o1 = b > o1 ? b : o1;
         }
     }
+    __syncthreads();
+    const int32_t bfirst = s_bin[1];
+    bool one_bin = true;
+    uint32_t cells = 0;
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const int loc = k * BT + threadIdx.x;
+        const size_t p = p0 + (size_t)loc;
+        if (p < n) {
+            cells += (p == 0 || s_key[loc] != s_key[loc + 1]) ? 1u : 0u;
+            const int32_t bp = s_bin[loc], b = s_bin[loc + 1];
+            for (int32_t bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
+            if (p == n - 1)
+                for (int32_t bb = b + 1; bb <= g.m; ++bb) bin_start[bb] = (uint32_t)n;
+            one_bin = one_bin && b == bfirst;
+        }
+    }
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    cells = __reduce_add_sync(0xffffffffu, cells);
+    if (lane == 0 && cells) atomicAdd(&s_cnt, cells);
+    if (__syncthreads_and(one_bin)) {
+#pragma unroll
+        for (int off = 16; off; off >>= 1) {
+            const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
+            const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);
+            o0 = x < o0 ? x : o0;
+            o1 = y > o1 ? y : o1;
+        }
+        if (lane == 0) { s_o0[warp] = o0; s_o1[warp] = o1; }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int w = 1; w < BT / 32; ++w) {
+                o0 = s_o0[w] < o0 ? s_o0[w] : o0;
+                o1 = s_o1[w] > o1 ? s_o1[w] : o1;
+            }
+            atomicMin(&bin_t0min[bfirst], o0);
+            atomicMax(&bin_t1max[bfirst], o1);
+        }
+    } else {                                           // tile spans bins: per element
+#pragma unroll
+        for (int k = 0; k < ITEMS; ++k) {
+            const int loc = k * BT + threadIdx.x;
+            if (p0 + (size_t)loc < n) {
+                const int32_t b = s_bin[loc + 1];
+                const double2 t = soa.st[p0 + (size_t)loc];   // written above by this thread
+                atomicMin(&bin_t0min[b], ordered_bits(t.x));
+                atomicMax(&bin_t1max[b], ordered_bits(t.y));
+            }
+        }
+    }
+    __syncthreads();
+    if (threadIdx.x == 0 && s_cnt) atomicAdd(count, (unsigned long long)s_cnt);
 }
 
 __global__ void k_fill_u64(unsigned long long* __restrict__ a, size_t n, unsigned long long v) {
@@ -218,78 +302,6 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
         double v = from_ordered_bits(a[i]);
         a[i] = (unsigned long long)__double_as_longlong(v);
     }
-}
-
-// Counts non-empty cells, writes bin_start[0..m] (the entries of bin j are the
-// sorted positions [bin_start[j], bin_start[j+1]): the index range
-// [B_first, B_last] of P:L76, keys being bin-major) and the per-bin extent
-// [min t_start, max t_end] (B_start / B_end of P:L76) with warp-aggregated
-// atomics on order-preserving integer images of the times.
-__global__ void __launch_bounds__(BT) k_count_cells(const SortedKeys keys,
-                                                   size_t n, GridParams g,
-                                                   const double2* __restrict__ st,
-                                                   uint32_t* __restrict__ bin_start,
-                                                   unsigned long long* __restrict__ bin_t0min,
-                                                   unsigned long long* __restrict__ bin_t1max,
-                                                   unsigned long long* __restrict__ count) {
-    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    int f = 0;
-    long long b = -1;
-    unsigned long long o0 = ~0ull, o1 = 0ull;
-    // the bin is recomputed with bin_of() from t_start exactly as k_keys did
-    // (same inputs, same arithmetic), avoiding a 64-bit division of the key
-    if (p < n) {
-        const unsigned long long k = keys.key(p);
-        f = (p == 0 || k != keys.key(p - 1));
-        const double2 t = st[p];
-        b = bin_of(g, t.x);
-        const long long bp = p == 0 ? -1 : (long long)bin_of(g, st[p - 1].x);
-        for (long long bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
-        if (p == n - 1)
-            for (long long bb = b + 1; bb <= g.m; ++bb) bin_start[bb] = (uint32_t)n;
-        o0 = ordered_bits(t.x);
-        o1 = ordered_bits(t.y);
-    }
-    const int lane = threadIdx.x & 31;
-    // one atomic pair per CTA when the CTA's 256 sorted positions share a bin
-    // (the common case: bins hold ~10^5 entries), else per warp / per thread
-    const long long bfirst = bin_of(g, st[(size_t)blockIdx.x * BT].x);
-    if (__syncthreads_and(b == bfirst || b < 0)) {
-        __shared__ unsigned long long r0[BT / 32], r1[BT / 32];
-        for (int off = 16; off; off >>= 1) {
-            const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
-            const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);
-            o0 = x < o0 ? x : o0;
-            o1 = y > o1 ? y : o1;
-        }
-        if (lane == 0) { r0[threadIdx.x >> 5] = o0; r1[threadIdx.x >> 5] = o1; }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            for (int w = 1; w < BT / 32; ++w) {
-                o0 = r0[w] < o0 ? r0[w] : o0;
-                o1 = r1[w] > o1 ? r1[w] : o1;
-            }
-            atomicMin(&bin_t0min[bfirst], o0);
-            atomicMax(&bin_t1max[bfirst], o1);
-        }
-    } else if (const long long b0 = __shfl_sync(0xffffffffu, b, 0);
-               __all_sync(0xffffffffu, b == b0 || b < 0)) {
-        for (int off = 16; off; off >>= 1) {
-            const unsigned long long x = __shfl_xor_sync(0xffffffffu, o0, off);
-            const unsigned long long y = __shfl_xor_sync(0xffffffffu, o1, off);
-            o0 = x < o0 ? x : o0;
-            o1 = y > o1 ? y : o1;
-        }
-        if (lane == 0 && b0 >= 0) {
-            atomicMin(&bin_t0min[b0], o0);
-            atomicMax(&bin_t1max[b0], o1);
-        }
-    } else if (b >= 0) {
-        atomicMin(&bin_t0min[b], o0);
-        atomicMax(&bin_t1max[b], o1);
-    }
-    int c = __syncthreads_count(f);
-    if (threadIdx.x == 0 && c) atomicAdd(count, (unsigned long long)c);
 }
 
 __global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
@@ -571,35 +583,15 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
-    {
-        static const int gv = [] {          // DTS_GATHER: 1n 2n 4n 1s 2s 4s
-            const char* e = getenv("DTS_GATHER");
-            if (!e || !e[0]) return 20;
-            const int items = e[0] - '0';
-            const int st = e[1] == 's' ? 1 : 0;
-            return ((items == 1 || items == 2 || items == 4) ? items : 2) * 10 + st;
-        }();
-        const int items = gv / 10;
-        const unsigned gb = grid_for((n + items - 1) / items);
-        switch (gv) {
-            case 10: k_gather<1, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-            case 11: k_gather<1, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-            case 21: k_gather<2, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-            case 40: k_gather<4, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-            case 41: k_gather<4, true><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-            default: k_gather<2, false><<<gb, BT, 0, s>>>(D, n, sk, idx->soa); break;
-        }
-    }
-    DTS_LAUNCH_CHECK();
-
-    // 6. non-empty cells -> hash table
     DevBuf<unsigned long long> ncell(1, s);
     DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
-    k_count_cells<<<grid_for(n), BT, 0, s>>>(sk, n, g, idx->soa.st, idx->bin_start, b0, b1,
-                                             ncell.p);
+    k_gather_cells<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(D, n, sk, idx->soa, g, idx->bin_start,
+                                                           b0, b1, ncell.p);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
+
+    // 6. non-empty cells -> hash table
     unsigned long long hc = 0;
     DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
