@@ -215,7 +215,10 @@ def run_own(args):
         if world > 1:
             dts_dist.global_offset(res.count, rank, world)
         if stats_out is not None:
-            st["ms_build"] = idx.info()["ms_build"]
+            inf = idx.info()
+            st["ms_build"] = inf["ms_build"]
+            st["ms_phase"] = list(inf["ms_phase"])
+            st["index"] = inf
             stats_out.append(st)
         cnt = res.count
         res.free()
@@ -263,21 +266,48 @@ def run_own(args):
     ms_per_step = total_ms / args.steps
     value = world * nq / (ms_per_step * 1e-3)
 
-    # ---- dominant kernel roofline (pass 1 candidate streaming, events in-lib)
+    # ---- per-kernel rooflines (CUDA events in-lib, on the launching stream):
+    #      algorithmic bytes per launch / mean event time
     peak, peak_src = load_peaks()
     st0 = stats[-1]
     ms_count = statistics.mean(s["ms_count"] for s in stats)
     ms_scatter = statistics.mean(s["ms_scatter"] for s in stats)
     ms_build = statistics.mean(s["ms_build"] for s in stats)
+    ph = [statistics.mean(s["ms_phase"][i] for s in stats) for i in range(5)]
+    inf = st0["index"]
+    ncell_key = inf["bins"] * inf["grid"][0] * inf["grid"][1] * inf["grid"][2]
+    npass = (max(1, int(ncell_key - 1).bit_length()) + 7) // 8
+    ncells = inf["cells"]
     alg_bytes = st0["candidates"] * 64 + nq * (64 + 4) + st0["cell_lookups"] * 64
-    achieved = alg_bytes / (ms_count * 1e-3) / 1e9
-    traffic = None
+    traffic_all = {}
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(args.config, {}).get("k_wtile_count")
+            traffic_all = json.load(open(tf)).get(args.config, {})
         except (ValueError, AttributeError):
-            traffic = None
+            traffic_all = {}
+    kernels = [
+        # name, ms per launch-group, algorithmic bytes, model
+        ("k_wtile_count", ms_count, alg_bytes,
+         "64 B per candidate + 68 B per query + 64 B per hash-bucket probe"),
+        ("k_onesweep (entry sort)", ph[2], n * 8 + npass * n * 16,
+         f"8 B/key histogram read + {npass} passes x (8 B read + 8 B write) per key"),
+        ("k_gather_cells", ph[3], n * (8 + 64 + 68),
+         "8 B sorted key + 64 B record read + 68 B record/id write per entry"),
+        ("k_insert", ph[4], n * 8 + ncells * 16, "8 B key per entry + 16 B slot per cell"),
+        ("k_bounds", ph[0], n * 64, "64 B record read per entry"),
+        ("k_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
+         "(phase includes the host read-back of the bounds)"),
+    ]
+    kern = []
+    for name, ms, by, model in kernels:
+        a_gbs = by / (ms * 1e-3) / 1e9 if ms > 0 else None
+        kern.append({"kernel": name, "ms": ms, "bytes": int(by), "achieved_gbs": a_gbs,
+                     "frac": (a_gbs / peak) if a_gbs else None,
+                     "traffic": traffic_all.get(name.split()[0]), "bytes_model": model})
+    dom = max(kern, key=lambda k: k["ms"])
+    achieved = alg_bytes / (ms_count * 1e-3) / 1e9
+    traffic = traffic_all.get("k_wtile_count")
 
     # ---- e2e through the C ABI host entry points (pinned host buffers)
     e2e_val = None
@@ -322,7 +352,9 @@ def run_own(args):
                                "canonical sort (all SURVEY.md §8(a) rows), inputs resident in HBM",
                        "l2": "flushed between steps (256 MiB write outside the timed events)",
                        "parallelism": f"query-sharded x{world}, D replicated"},
-            "phases_ms": {"build": ms_build, "prep": statistics.mean(s["ms_prep"] for s in stats),
+            "phases_ms": {"build": ms_build, "build_bounds": ph[0], "build_keys": ph[1],
+                          "build_sort": ph[2], "build_gather": ph[3], "build_insert": ph[4],
+                          "prep": statistics.mean(s["ms_prep"] for s in stats),
                           "count_pass": ms_count, "scan": statistics.mean(s["ms_scan"] for s in stats),
                           "scatter_pass": ms_scatter,
                           "canon": statistics.mean(s["ms_canon"] for s in stats)},
@@ -331,12 +363,18 @@ def run_own(args):
                                     "the build, P:L135)"},
             "work": {"candidates_per_pass": st0["candidates"], "cell_lookups": st0["cell_lookups"],
                      "results_per_rank": results},
-            "roofline": {"bound": "hbm", "kernel": "k_wtile_count (pass 1: fused candidate streaming + "
-                         "fp64 refine)", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                         "frac": achieved / peak, "traffic": traffic,
-                         "peak_source": peak_src,
-                         "algorithmic_bytes": alg_bytes,
-                         "bytes_model": "64 B per candidate + 68 B per query + 64 B per hash-bucket probe"},
+            "roofline": {"bound": "hbm", "kernel": dom["kernel"], "achieved": dom["achieved_gbs"],
+                         "peak": peak, "unit": "GB/s", "frac": dom["frac"],
+                         "traffic": dom["traffic"], "peak_source": peak_src,
+                         "algorithmic_bytes": dom["bytes"], "ms": dom["ms"],
+                         "bytes_model": dom["bytes_model"],
+                         "note": "dominant kernel = largest device time of one step "
+                                 "(per-phase CUDA events); all kernels in roofline_kernels"},
+            "roofline_kernels": kern,
+            "roofline_search": {"bound": "hbm", "kernel": "k_wtile_count (pass 1: fused candidate "
+                                "streaming + fp64 refine)", "achieved": achieved, "peak": peak,
+                                "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                                "algorithmic_bytes": alg_bytes},
             "clocks": clk,
             "gpu_launches": int(launches),
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h2d),

@@ -225,6 +225,10 @@ typedef struct {
     uint32_t method;            /* dts_method of the index                   */
     uint32_t subbins[3];        /* v per dimension (SUBBIN), else 0          */
     uint64_t subbin_ids[3];     /* length of the X, Y, Z id arrays (SUBBIN)  */
+    float    ms_phase[5];       /* device time of the last build's phases (CUDA
+                                   events on the build stream): bounds, keys,
+                                   radix sort, gather (+ bins, cell count),
+                                   hash insert                               */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

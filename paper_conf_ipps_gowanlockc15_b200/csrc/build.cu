@@ -157,6 +157,99 @@ __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size
     }
 }
 
+// One non-empty cell into the bucketed open-addressing table: key -> [p, e).
+__device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long long k, uint32_t p,
+                                            uint32_t e) {
+    const unsigned long long bmask = ht.mask >> 2;
+    unsigned long long b = bucket_of(k >> 2, ht.log2cap);
+    // try the slot matching the key's position in its group first: the (up
+    // to) four x-adjacent cells sharing a home bucket then claim distinct
+    // slots without colliding on the same CAS
+    const int first = (int)(k & 3ull);
+    while (true) {
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            const int i = (first + j) & 3;
+            CellSlot& sl = ht.slots[4 * b + i];
+            const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
+            if (prev == EMPTY_KEY) {
+                sl.start = p;
+                sl.end = e;
+                return;
+            }
+        }
+        b = (b + 1) & bmask;
+    }
+}
+
+__global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
+                                              size_t n, HashTable ht) {
+    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
+    if (p >= n) return;
+    unsigned long long k = keys.key(p);
+    if (p != 0 && keys.key(p - 1) == k) return;
+    // the cell's run ends at the next key change (most cells hold 1-3 entries)
+    size_t e = p + 1;
+    while (e < n && keys.key(e) == k) ++e;
+    insert_cell(ht, k, (uint32_t)p, (uint32_t)e);
+}
+
+
+// ITEMS sorted positions per thread (strided by the grid so key loads stay
+// coalesced): the cell heads among them issue their first-choice CAS
+// together, so ITEMS atomics are in flight per thread instead of one; a head
+// that loses its first slot continues with insert_cell().
+template <int ITEMS>
+__global__ void __launch_bounds__(BT) k_insert_batched(const SortedKeys keys, size_t n,
+                                                      HashTable ht) {
+    const size_t stride = (size_t)gridDim.x * BT;
+    const size_t p0 = (size_t)blockIdx.x * BT + threadIdx.x;
+    unsigned long long k[ITEMS];
+    uint32_t e[ITEMS];
+    bool head[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+        const size_t p = p0 + (size_t)i * stride;
+        head[i] = false;
+        k[i] = 0;
+        e[i] = 0;
+        if (p < n) {
+            k[i] = keys.key(p);
+            head[i] = p == 0 || keys.key(p - 1) != k[i];
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+        if (head[i]) {   // the cell's run ends at the next key change
+            size_t q = p0 + (size_t)i * stride + 1;
+            while (q < n && keys.key(q) == k[i]) ++q;
+            e[i] = (uint32_t)q;
+        }
+    }
+    unsigned long long prev[ITEMS];
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+        prev[i] = 0;
+        if (head[i]) {
+            const unsigned long long b = bucket_of(k[i] >> 2, ht.log2cap);
+            prev[i] = atomicCAS(&ht.slots[4 * b + (k[i] & 3ull)].key, EMPTY_KEY, k[i]);
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < ITEMS; ++i) {
+        if (!head[i]) continue;
+        const uint32_t p = (uint32_t)(p0 + (size_t)i * stride);
+        if (prev[i] == EMPTY_KEY) {
+            const unsigned long long b = bucket_of(k[i] >> 2, ht.log2cap);
+            CellSlot& sl = ht.slots[4 * b + (k[i] & 3ull)];
+            sl.start = p;
+            sl.end = e[i];
+        } else {
+            insert_cell(ht, k[i], p, e[i]);
+        }
+    }
+}
+
 __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
 }
@@ -226,10 +319,10 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
         if (p < n) {
             const double4 s0 = r0[k], s1 = r1[k];
             const double dur = s1.x - s0.x;
-            soa.st[p] = make_double2(s0.x, s1.x);
-            soa.sx[p] = make_double2(s0.y, velocity(s0.y, s1.y, dur));
-            soa.sy[p] = make_double2(s0.z, velocity(s0.z, s1.z, dur));
-            soa.sz[p] = make_double2(s0.w, velocity(s0.w, s1.w, dur));
+            *soa.at(0, p) = make_double2(s0.x, s1.x);
+            *soa.at(1, p) = make_double2(s0.y, velocity(s0.y, s1.y, dur));
+            *soa.at(2, p) = make_double2(s0.z, velocity(s0.z, s1.z, dur));
+            *soa.at(3, p) = make_double2(s0.w, velocity(s0.w, s1.w, dur));
             soa.eid[p] = id[k];
             s_bin[1 + k * BT + threadIdx.x] = bin_of(g, s0.x);
             const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);
@@ -281,7 +374,7 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
             const int loc = k * BT + threadIdx.x;
             if (p0 + (size_t)loc < n) {
                 const int32_t b = s_bin[loc + 1];
-                const double2 t = soa.st[p0 + (size_t)loc];   // written above by this thread
+                const double2 t = *soa.at(0, p0 + (size_t)loc);   // written above by this thread
                 atomicMin(&bin_t0min[b], ordered_bits(t.x));
                 atomicMax(&bin_t1max[b], ordered_bits(t.y));
             }
@@ -304,36 +397,6 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
     }
 }
 
-__global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
-                                              size_t n, HashTable ht) {
-    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    if (p >= n) return;
-    unsigned long long k = keys.key(p);
-    if (p != 0 && keys.key(p - 1) == k) return;
-    // the cell's run ends at the next key change (most cells hold 1-3 entries)
-    size_t e = p + 1;
-    while (e < n && keys.key(e) == k) ++e;
-    const unsigned long long bmask = ht.mask >> 2;
-    unsigned long long b = bucket_of(k >> 2, ht.log2cap);
-    // try the slot matching the key's position in its group first: the (up
-    // to) four x-adjacent cells sharing a home bucket then claim distinct
-    // slots without colliding on the same CAS
-    const int first = (int)(k & 3ull);
-    while (true) {
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            const int i = (first + j) & 3;
-            CellSlot& sl = ht.slots[4 * b + i];
-            const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
-            if (prev == EMPTY_KEY) {
-                sl.start = (uint32_t)p;
-                sl.end = (uint32_t)e;
-                return;
-            }
-        }
-        b = (b + 1) & bmask;
-    }
-}
 
 inline unsigned grid_for(size_t n) { return (unsigned)((n + BT - 1) / BT); }
 
@@ -362,7 +425,7 @@ __global__ void __launch_bounds__(BT) k_sb_count(const double4* __restrict__ D,
 template <int A>
 __global__ void __launch_bounds__(BT) k_sb_emit(const double4* __restrict__ D,
                                                const uint32_t* __restrict__ eid,
-                                               const double2* __restrict__ st, size_t n,
+                                               const SegSoA soa, size_t n,
                                                SubbinIndex sb, GridParams g,
                                                const unsigned long long* __restrict__ off,
                                                unsigned long long* __restrict__ keys,
@@ -372,7 +435,7 @@ __global__ void __launch_bounds__(BT) k_sb_emit(const double4* __restrict__ D,
     const uint32_t i = eid[p];
     const double c0 = coord<A>(D[2 * (size_t)i]), c1 = coord<A>(D[2 * (size_t)i + 1]);
     const int32_t jlo = subbin_of(sb, A, fmin(c0, c1)), jhi = subbin_of(sb, A, fmax(c0, c1));
-    const unsigned long long bin = (unsigned long long)bin_of(g, st[p].x);
+    const unsigned long long bin = (unsigned long long)bin_of(g, soa.ld(0, p).x);
     unsigned long long o = off[p];
     for (int32_t j = jlo; j <= jhi; ++j, ++o) {
         keys[o] = (unsigned long long)j * (unsigned long long)g.m + bin;
@@ -446,13 +509,13 @@ static void build_subbins(dts_index* idx, const double4* D, size_t n, const Boun
         idx->sb_block[a] = blk;
         idx->sb_len[a] = len;
         if (a == 0)
-            k_sb_emit<0><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+            k_sb_emit<0><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa, n, sb, g,
                                                     off.p, keys.p, blk);
         else if (a == 1)
-            k_sb_emit<1><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+            k_sb_emit<1><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa, n, sb, g,
                                                     off.p, keys.p, blk);
         else
-            k_sb_emit<2><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa.st, n, sb, g,
+            k_sb_emit<2><<<grid_for(n), BT, 0, s>>>(D, idx->soa.eid, idx->soa, n, sb, g,
                                                     off.p, keys.p, blk);
         DTS_LAUNCH_CHECK();
         radix_sort_pairs(keys.p, blk, keys_tmp.p, vals_tmp.p, len, bits_for(nkeys - 1), s);
@@ -512,10 +575,12 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     idx->n = n;
     if (n == 0) return;
     const double4* D = reinterpret_cast<const double4*>(D_dev);
-    cudaEvent_t e0, e1;
-    DTS_CUDA(cudaEventCreate(&e0));
-    DTS_CUDA(cudaEventCreate(&e1));
-    DTS_CUDA(cudaEventRecord(e0, s));
+    // phase events: start, bounds, keys, sort, gather, insert (+ end)
+    cudaEvent_t ev[7];
+    for (auto& e : ev) DTS_CUDA(cudaEventCreate(&e));
+    int nev = 0;
+    auto mark = [&] { DTS_CUDA(cudaEventRecord(ev[nev++], s)); };
+    mark();
 
     // 1. bounds + validation
     const int np = (int)std::min<size_t>(grid_for(n), 148 * 8);
@@ -524,6 +589,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
     DTS_LAUNCH_CHECK();
+    mark();
     Bounds hb;
     DTS_CUDA(cudaMemcpyAsync(&hb, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
@@ -550,6 +616,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DevBuf<uint32_t> ids(packed ? 0 : n, s), ids_tmp(packed ? 0 : n, s);
     k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p, row_bits);
     DTS_LAUNCH_CHECK();
+    mark();
     SortedKeys sk;
     if (packed) {   // keys-only sort of the key bits; rows ride in the low bits
         sk.a = radix_sort_keys(keys.p, keys_tmp.p, n, row_bits, row_bits + idx->key_bits, s);
@@ -563,17 +630,21 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         sk.ids = ids.p;
     }
 
-    // 5. gather into the SoA layout
+    mark();
+    // 5. gather into the sorted record layout
     const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
     const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
     char* blk = nullptr;
     blk = static_cast<char*>(cache_alloc(bytes_soa + bytes_bins + 256));
     idx->block = blk;
-    idx->soa.st = reinterpret_cast<double2*>(blk);
-    idx->soa.sx = idx->soa.st + n;
-    idx->soa.sy = idx->soa.sx + n;
-    idx->soa.sz = idx->soa.sy + n;
-    idx->bin_t0min = reinterpret_cast<double*>(idx->soa.sz + n);
+    idx->soa.rec = reinterpret_cast<double2*>(blk);
+    static const bool aos = [] {              // DTS_LAYOUT=rec: 64-byte records
+        const char* e = getenv("DTS_LAYOUT");   // measured on C4: records cost
+        return e && e[0] == 'r';                // +0.08 ms gather, +0.02 ms search
+    }();
+    idx->soa.ss = aos ? 1 : n;
+    idx->soa.es = aos ? 4u : 1u;
+    idx->bin_t0min = reinterpret_cast<double*>(idx->soa.rec + 4 * n);
     idx->bin_t1max = idx->bin_t0min + g.m;
     idx->soa.eid = reinterpret_cast<uint32_t*>(idx->bin_t1max + g.m);
     idx->bin_start = idx->soa.eid + n;
@@ -583,6 +654,9 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b1, g.m, 0ull);
     DTS_LAUNCH_CHECK();
+    // 6. non-empty cells -> hash table of >= 2x as many slots (power of two)
+    // (measured: inserting from the gather, with the cells counted first,
+    //  costs 1.98 ms against 0.78 + 0.56 ms for gather + separate insert)
     DevBuf<unsigned long long> ncell(1, s);
     DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
     k_gather_cells<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(D, n, sk, idx->soa, g, idx->bin_start,
@@ -590,8 +664,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
-
-    // 6. non-empty cells -> hash table
+    mark();
     unsigned long long hc = 0;
     DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
@@ -602,8 +675,19 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     idx->ht.mask = (1ull << log2cap) - 1;
     idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
-    k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
+    // (measured on C4: 1 cell per thread 0.56 ms incl. the memset; batching
+    //  the first CAS of 2 / 4 / 8 cells: 0.59 / 0.70 / 0.91 ms)
+    static const int ins = [] {               // DTS_INSERT_ITEMS: 1 (k_insert), 2, 4, 8
+        const char* e = getenv("DTS_INSERT_ITEMS");
+        const int v = e ? atoi(e) : 1;
+        return (v == 2 || v == 4 || v == 8) ? v : 1;
+    }();
+    if (ins == 1) k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
+    else if (ins == 2) k_insert_batched<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(sk, n, idx->ht);
+    else if (ins == 4) k_insert_batched<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    else k_insert_batched<8><<<grid_for((n + 7) / 8), BT, 0, s>>>(sk, n, idx->ht);
     DTS_LAUNCH_CHECK();
+    mark();
 
     // 7. GPUSpatioTemporal subbin arrays (DTS_METHOD_SUBBIN)
     idx->method = p.method;
@@ -627,11 +711,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         DTS_LAUNCH_CHECK();
     }
 
-    DTS_CUDA(cudaEventRecord(e1, s));
-    DTS_CUDA(cudaEventSynchronize(e1));
-    DTS_CUDA(cudaEventElapsedTime(&idx->ms_build, e0, e1));
-    cudaEventDestroy(e0);
-    cudaEventDestroy(e1);
+    mark();
+    DTS_CUDA(cudaEventSynchronize(ev[nev - 1]));
+    DTS_CUDA(cudaEventElapsedTime(&idx->ms_build, ev[0], ev[nev - 1]));
+    for (int i = 0; i < 5; ++i) {
+        idx->ms_phase[i] = 0.f;
+        if (i + 1 < nev) cudaEventElapsedTime(&idx->ms_phase[i], ev[i], ev[i + 1]);
+    }
+    for (auto& e : ev) cudaEventDestroy(e);
 }
 
 }  // namespace dts

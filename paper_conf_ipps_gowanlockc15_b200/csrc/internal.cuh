@@ -77,12 +77,19 @@ struct DevBuf {
 // with v = (end - start) / (t_end - t_start) precomputed at build (0 for a
 // zero-duration segment, which can never overlap strictly in time).  The
 // position at time t is start + (t - t_start) * v.
+// Entry records in sorted order: four double2 "streams" k = 0..3 holding
+// (t0,t1) (x0,vx) (y0,vy) (z0,vz).  Stream k of position p is
+// rec[k * ss + p * es]: ss = n, es = 1 is the SoA layout (four arrays);
+// ss = 1, es = 4 the record layout (one 64-byte record per entry).
 struct SegSoA {
-    double2* st;
-    double2* sx;
-    double2* sy;
-    double2* sz;
+    double2* rec;
+    size_t ss;
+    uint32_t es;
     uint32_t* eid;   // caller's entry id of each sorted position
+#ifdef __CUDACC__
+    __device__ __forceinline__ double2* at(int k, size_t p) const { return rec + k * ss + p * es; }
+    __device__ __forceinline__ double2 ld(int k, size_t p) const { return __ldg(at(k, p)); }
+#endif
 };
 
 // Hash slot of one non-empty (bin, cell) key: entries [start, end) of the
@@ -226,6 +233,7 @@ struct dts_index {
     void* block = nullptr;         // single device allocation backing the arrays above
     double max_ext[3] = {0, 0, 0};
     float ms_build = 0.f;
+    float ms_phase[5] = {0, 0, 0, 0, 0};   // bounds, keys, sort, gather, insert
     int key_bits = 0;
     uint32_t method = 0;           // dts_method
     dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only

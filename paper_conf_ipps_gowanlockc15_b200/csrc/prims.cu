@@ -328,11 +328,12 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_hist_scan(uint32_t* __restric
     h[threadIdx.x] = ex;
 }
 
-template <bool VALS, int MINB>
+template <bool VALS, int MINB, int LB = OS_LB>
 __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ gbase, uint32_t* status, uint32_t* tile_ctr,
-    unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out) {
+    unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out,
+    uint32_t sleep_ns) {
     constexpr int RADIX = 256;
     static_assert(RADIX == RS_THREADS, "one digit per thread");
     __shared__ uint32_t wcnt[RS_WARPS][RADIX + 1];
@@ -372,14 +373,17 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
             peers &= ((dig >> b) & 1u) ? bal : ~bal;
         }
         if (dig >= (uint32_t)RADIX) peers = 1u << lane;
-        const int leader = __ffs(peers) - 1;
+        // the group's highest lane updates the counter: its rank below is
+        // the group size - 1 (one popc and one clz per key)
+        const uint32_t below = __popc(peers & lt_mask);
+        const int leader = 31 - __clz(peers);
         uint32_t old = 0;
         if (lane == leader && dig < (uint32_t)RADIX) {
             old = wcnt[warp][dig];
-            wcnt[warp][dig] = old + __popc(peers);
+            wcnt[warp][dig] = old + below + 1u;
         }
         old = __shfl_sync(0xffffffffu, old, leader);
-        dr[i] = dig | ((old + __popc(peers & lt_mask)) << 9);
+        dr[i] = dig | ((old + below) << 9);
         __syncwarp();
     }
     __syncthreads();
@@ -405,18 +409,26 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
         int32_t j = (int32_t)tile - 1;              // next predecessor to account for
         bool done = false;
         while (!done) {
-            uint32_t w[OS_LB];
+            uint32_t w[LB];
 #pragma unroll
-            for (int q = 0; q < OS_LB; ++q)
+            for (int q = 0; q < LB; ++q)
                 w[q] = j - q >= 0 ? ld_relaxed(status + (size_t)(j - q) * RADIX + t) : OS_PRE;
 #pragma unroll
-            for (int q = 0; q < OS_LB; ++q) {
-                if (done) break;
-                if (w[q] == 0u) break;               // not published yet: poll again from j
+            bool wait = false;
+#pragma unroll
+            for (int q = 0; q < LB; ++q) {
+                if (done || wait) break;
+                if (w[q] == 0u) {                    // not published yet: poll again from j
+                    wait = true;
+                    break;
+                }
                 excl += w[q] & OS_VAL;
                 --j;
                 if (w[q] & OS_PRE) done = true;
             }
+            // back off instead of spinning: polling loads and branches would
+            // take issue slots from the other CTAs' ranking and scatter
+            if (wait && sleep_ns) __nanosleep(sleep_ns);
         }
         st_relaxed(mine, OS_PRE | (excl + count));
     }
@@ -482,22 +494,40 @@ void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32
             const int v = e ? atoi(e) : 4;
             return (v == 5 || v == 6) ? v : 4;
         }();
+        static const uint32_t sleep_ns = [] {   // DTS_OS_SLEEP: look-back back-off (ns)
+            const char* e = getenv("DTS_OS_SLEEP");   // C4 entry sort, 5 passes: 0 ns
+            return e ? (uint32_t)atoi(e) : 256u;      // 0.984 ms, 32: 0.970, 128: 0.961,
+        }();                                          // 512: 0.957
+        // (measured on C4: window 8 0.936 ms, 16 1.03, 32 1.64 for the 5 passes)
+        static const int lb = [] {             // DTS_OS_LB: look-back window (8, 16, 32)
+            const char* e = getenv("DTS_OS_LB");
+            const int v = e ? atoi(e) : 8;
+            return (v == 16 || v == 32) ? v : 8;
+        }();
         if (*vin)
             k_onesweep<true, 2><<<ntiles, RS_THREADS, 0, s>>>(*kin, *vin, n, lo + 8 * p,
                                                              hist + 256 * p, status.p, ctr, *kout,
-                                                             *vout);
+                                                             *vout, sleep_ns);
+        else if (lb == 16)
+            k_onesweep<false, 4, 16><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
+                                                                  hist + 256 * p, status.p, ctr,
+                                                                  *kout, nullptr, sleep_ns);
+        else if (lb == 32)
+            k_onesweep<false, 4, 32><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
+                                                                  hist + 256 * p, status.p, ctr,
+                                                                  *kout, nullptr, sleep_ns);
         else if (occ == 5)
             k_onesweep<false, 5><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
                                                               hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr);
+                                                              *kout, nullptr, sleep_ns);
         else if (occ == 6)
             k_onesweep<false, 6><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
                                                               hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr);
+                                                              *kout, nullptr, sleep_ns);
         else
             k_onesweep<false, 4><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
                                                               hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr);
+                                                              *kout, nullptr, sleep_ns);
         DTS_LAUNCH_CHECK();
         std::swap(*kin, *kout);
         std::swap(*vin, *vout);
