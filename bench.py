@@ -276,7 +276,10 @@ def run_own(args):
     ph = [statistics.mean(s["ms_phase"][i] for s in stats) for i in range(5)]
     inf = st0["index"]
     ncell_key = inf["bins"] * inf["grid"][0] * inf["grid"][1] * inf["grid"][2]
-    npass = (max(1, int(ncell_key - 1).bit_length()) + 7) // 8
+    kbits = max(1, int(ncell_key - 1).bit_length())
+    npass = (kbits + 7) // 8                 # the library's digit plan: 9-bit digits
+    if npass > 1 and kbits <= 9 * (npass - 1):   # where they save a pass
+        npass -= 1
     ncells = inf["cells"]
     alg_bytes = st0["candidates"] * 64 + nq * (64 + 4) + st0["cell_lookups"] * 64
     traffic_all = {}

@@ -161,7 +161,7 @@ __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size
 __device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long long k, uint32_t p,
                                             uint32_t e) {
     const unsigned long long bmask = ht.mask >> 2;
-    unsigned long long b = bucket_of(k >> 2, ht.log2cap);
+    unsigned long long b = bucket_of(k >> 2, ht);
     // try the slot matching the key's position in its group first: the (up
     // to) four x-adjacent cells sharing a home bucket then claim distinct
     // slots without colliding on the same CAS
@@ -231,7 +231,7 @@ __global__ void __launch_bounds__(BT) k_insert_batched(const SortedKeys keys, si
     for (int i = 0; i < ITEMS; ++i) {
         prev[i] = 0;
         if (head[i]) {
-            const unsigned long long b = bucket_of(k[i] >> 2, ht.log2cap);
+            const unsigned long long b = bucket_of(k[i] >> 2, ht);
             prev[i] = atomicCAS(&ht.slots[4 * b + (k[i] & 3ull)].key, EMPTY_KEY, k[i]);
         }
     }
@@ -240,7 +240,7 @@ __global__ void __launch_bounds__(BT) k_insert_batched(const SortedKeys keys, si
         if (!head[i]) continue;
         const uint32_t p = (uint32_t)(p0 + (size_t)i * stride);
         if (prev[i] == EMPTY_KEY) {
-            const unsigned long long b = bucket_of(k[i] >> 2, ht.log2cap);
+            const unsigned long long b = bucket_of(k[i] >> 2, ht);
             CellSlot& sl = ht.slots[4 * b + (k[i] & 3ull)];
             sl.start = p;
             sl.end = e[i];
@@ -673,6 +673,11 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     while ((1ull << log2cap) < 2 * hc) ++log2cap;
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
+    static const int hblk = [] {              // DTS_HASH_BLOCK: log2 buckets per block
+        const char* e = getenv("DTS_HASH_BLOCK");
+        return e ? std::max(0, std::min(8, atoi(e))) : 0;
+    }();
+    idx->ht.blk = std::min(hblk, log2cap - 4);
     idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
     // (measured on C4: 1 cell per thread 0.56 ms incl. the memset; batching

@@ -120,6 +120,7 @@ struct HashTable {
     CellSlot* slots;
     unsigned long long mask;   // capacity - 1 (power of two)
     int log2cap;
+    int blk;                   // log2 of the buckets of a block (bucket_of)
 };
 
 // GPUSpatioTemporal subbins (P:L86-P:L92): per dimension a, v[a] subbins of
@@ -150,8 +151,13 @@ __device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double
 // sits in the first bucket, from its home on, that had a free slot when it
 // was inserted (no deletions), so a lookup stops at the first bucket holding
 // the key or a free slot -- almost always the home bucket.
-__device__ __forceinline__ unsigned long long bucket_of(unsigned long long group, int log2cap) {
-    return (group * 0x9E3779B97F4A7C15ull) >> (64 - (log2cap - 2));
+// With blk > 0, 2^blk consecutive groups keep consecutive home buckets (one
+// block of 2^blk x 64 bytes) and only the block is placed by the hash: the
+// build's inserts, in key order, then touch each block's lines together.
+__device__ __forceinline__ unsigned long long bucket_of(unsigned long long group,
+                                                        const HashTable& ht) {
+    const unsigned long long hi = group >> ht.blk, lo = group & ((1ull << ht.blk) - 1ull);
+    return (((hi * 0x9E3779B97F4A7C15ull) >> (64 - (ht.log2cap - 2 - ht.blk))) << ht.blk) | lo;
 }
 
 __device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {

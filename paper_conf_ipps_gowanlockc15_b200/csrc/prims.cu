@@ -301,41 +301,59 @@ __device__ __forceinline__ void st_relaxed(uint32_t* p, uint32_t v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// Digit histograms of all passes (digits at bits lo + 8 p, p < npass) in one
-// read of the keys; hist[p * 256 + digit] is accumulated (caller zeroes it).
+// Digit layout of a multi-pass sort: pass p sorts the digit of width
+// bits[p] (8 or 9) at bit shift[p]; its histogram is hist[p * 512 + digit].
+constexpr int OS_MAXPASS = 8;
+constexpr int OS_HSTRIDE = 512;
+struct PassPlan {
+    int npass;
+    int shift[OS_MAXPASS];
+    int bits[OS_MAXPASS];
+};
+
+// Digit histograms of all passes in one read of the keys (caller zeroes hist).
 __global__ void __launch_bounds__(RS_THREADS) k_rs_hist_all(const unsigned long long* __restrict__ keys,
-                                                            size_t n, int lo, int npass,
+                                                            size_t n, const PassPlan plan,
                                                             uint32_t* __restrict__ hist) {
-    __shared__ uint32_t h[8 * 256];
-    for (int j = threadIdx.x; j < 8 * 256; j += RS_THREADS) h[j] = 0;
+    __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += RS_THREADS) h[j] = 0;
     __syncthreads();
     for (size_t i = (size_t)blockIdx.x * RS_THREADS + threadIdx.x; i < n;
          i += (size_t)gridDim.x * RS_THREADS) {
         const unsigned long long k = keys[i];
-        for (int p = 0; p < npass; ++p) atomicAdd(&h[p * 256 + ((k >> (lo + 8 * p)) & 255u)], 1u);
+        for (int p = 0; p < plan.npass; ++p)
+            atomicAdd(&h[p * OS_HSTRIDE + ((k >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
     }
     __syncthreads();
-    for (int j = threadIdx.x; j < npass * 256; j += RS_THREADS)
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += RS_THREADS)
         if (h[j]) atomicAdd(hist + j, h[j]);
 }
 
-// Exclusive scan of each pass's 256 digit counts, in place (one CTA per pass).
+// Exclusive scan of each pass's (up to 512) digit counts, in place (one CTA
+// per pass, two digits per thread).
 __global__ void __launch_bounds__(RS_THREADS) k_rs_hist_scan(uint32_t* __restrict__ hist) {
-    uint32_t* h = hist + (size_t)blockIdx.x * 256;
-    const uint32_t c = h[threadIdx.x];
+    uint32_t* h = hist + (size_t)blockIdx.x * OS_HSTRIDE;
+    const uint32_t c0 = h[2 * threadIdx.x], c1 = h[2 * threadIdx.x + 1];
     uint32_t total;
-    const uint32_t ex = block_exclusive_scan<uint32_t>(c, &total);
-    h[threadIdx.x] = ex;
+    const uint32_t ex = block_exclusive_scan<uint32_t>(c0 + c1, &total);
+    h[2 * threadIdx.x] = ex;
+    h[2 * threadIdx.x + 1] = ex + c0;
 }
 
-template <bool VALS, int MINB, int LB = OS_LB>
+// One pass over a digit of RB bits (8: 256 digits, one per thread; 9: 512,
+// two per thread -- a 34-bit key then takes 9+9+8+8 instead of five 8-bit
+// passes).
+template <bool VALS, int MINB, int RB, int LB = OS_LB>
 __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ gbase, uint32_t* status, uint32_t* tile_ctr,
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out,
     uint32_t sleep_ns) {
-    constexpr int RADIX = 256;
-    static_assert(RADIX == RS_THREADS, "one digit per thread");
+    constexpr int RADIX = 1 << RB;
+    constexpr int DPT = RADIX / RS_THREADS;          // digits per thread
+    static_assert(DPT == 1 || DPT == 2, "8- or 9-bit digits");
+    constexpr uint32_t DMASK = RADIX - 1;
+    constexpr int RSH = RB + 1;                      // rank shift in dr (digit RADIX = sentinel)
     __shared__ uint32_t wcnt[RS_WARPS][RADIX + 1];
     __shared__ uint32_t tile_base[RADIX];
     __shared__ uint32_t local_off[RADIX];
@@ -353,14 +371,14 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const size_t wbase = (size_t)tile * OS_TILE + (size_t)warp * (32 * OS_ITEMS);
     unsigned long long k[OS_ITEMS];
     uint32_t v[VALS ? OS_ITEMS : 1];
-    uint32_t dr[OS_ITEMS];                       // digit | rank << 9; digit RADIX: past the end
+    uint32_t dr[OS_ITEMS];                       // digit | rank << RSH; digit RADIX: past the end
 #pragma unroll
     for (int i = 0; i < OS_ITEMS; ++i) {
         const size_t idx = wbase + (size_t)i * 32 + lane;
         const bool ok = idx < n;
         k[i] = ok ? keys[idx] : 0ull;
         if (VALS) v[i] = ok ? vals[idx] : 0u;
-        dr[i] = ok ? ((uint32_t)(k[i] >> shift) & (RADIX - 1)) : (uint32_t)RADIX;
+        dr[i] = ok ? ((uint32_t)(k[i] >> shift) & DMASK) : (uint32_t)RADIX;
     }
     const uint32_t lt_mask = (1u << lane) - 1u;
 #pragma unroll
@@ -368,7 +386,7 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
         const uint32_t dig = dr[i];
         uint32_t peers = __ballot_sync(0xffffffffu, dig < (uint32_t)RADIX);
 #pragma unroll
-        for (int b = 0; b < 8; ++b) {
+        for (int b = 0; b < RB; ++b) {
             const uint32_t bal = __ballot_sync(0xffffffffu, (dig >> b) & 1u);
             peers &= ((dig >> b) & 1u) ? bal : ~bal;
         }
@@ -383,58 +401,73 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
             wcnt[warp][dig] = old + below + 1u;
         }
         old = __shfl_sync(0xffffffffu, old, leader);
-        dr[i] = dig | ((old + below) << 9);
+        dr[i] = dig | ((old + below) << RSH);
         __syncwarp();
     }
     __syncthreads();
 
-    // ---- thread t owns digit t: cross-warp prefix, then look-back
+    // ---- thread t owns digits t*DPT .. t*DPT+DPT-1: cross-warp prefix, look-back
     const int t = threadIdx.x;
-    uint32_t count = 0;
+    uint32_t count[DPT], excl[DPT];
 #pragma unroll
-    for (int w = 0; w < RS_WARPS; ++w) {
-        const uint32_t c = wcnt[w][t];
-        wcnt[w][t] = count;
-        count += c;
+    for (int c = 0; c < DPT; ++c) {
+        const int dg = t * DPT + c;
+        uint32_t acc = 0;
+#pragma unroll
+        for (int w = 0; w < RS_WARPS; ++w) {
+            const uint32_t x = wcnt[w][dg];
+            wcnt[w][dg] = acc;
+            acc += x;
+        }
+        count[c] = acc;
+        excl[c] = 0;
     }
-    uint32_t excl = 0;
-    uint32_t* mine = status + (size_t)tile * RADIX + t;
+    uint32_t* mine = status + (size_t)tile * RADIX + t * DPT;
     if (tile == 0) {
-        st_relaxed(mine, OS_PRE | count);
+#pragma unroll
+        for (int c = 0; c < DPT; ++c) st_relaxed(mine + c, OS_PRE | count[c]);
     } else {
-        st_relaxed(mine, OS_AGG | count);
-        // windowed look-back: OS_LB predecessors per round trip (in the first
+#pragma unroll
+        for (int c = 0; c < DPT; ++c) st_relaxed(mine + c, OS_AGG | count[c]);
+        // windowed look-back: LB predecessors per round trip (in the first
         // wave every tile has only aggregates behind it; one tile per round
         // trip would serialise the wave)
-        int32_t j = (int32_t)tile - 1;              // next predecessor to account for
-        bool done = false;
-        while (!done) {
-            uint32_t w[LB];
 #pragma unroll
-            for (int q = 0; q < LB; ++q)
-                w[q] = j - q >= 0 ? ld_relaxed(status + (size_t)(j - q) * RADIX + t) : OS_PRE;
+        for (int c = 0; c < DPT; ++c) {
+            int32_t j = (int32_t)tile - 1;          // next predecessor to account for
+            bool done = false;
+            while (!done) {
+                uint32_t w[LB];
 #pragma unroll
-            bool wait = false;
+                for (int q = 0; q < LB; ++q)
+                    w[q] = j - q >= 0 ? ld_relaxed(status + (size_t)(j - q) * RADIX + t * DPT + c)
+                                      : OS_PRE;
+                bool wait = false;
 #pragma unroll
-            for (int q = 0; q < LB; ++q) {
-                if (done || wait) break;
-                if (w[q] == 0u) {                    // not published yet: poll again from j
-                    wait = true;
-                    break;
+                for (int q = 0; q < LB; ++q) {
+                    if (done || wait) break;
+                    if (w[q] == 0u) {                // not published yet: poll again from j
+                        wait = true;
+                        break;
+                    }
+                    excl[c] += w[q] & OS_VAL;
+                    --j;
+                    if (w[q] & OS_PRE) done = true;
                 }
-                excl += w[q] & OS_VAL;
-                --j;
-                if (w[q] & OS_PRE) done = true;
+                // back off instead of spinning: polling loads and branches
+                // would take issue slots from the other CTAs' ranking and scatter
+                if (wait && sleep_ns) __nanosleep(sleep_ns);
             }
-            // back off instead of spinning: polling loads and branches would
-            // take issue slots from the other CTAs' ranking and scatter
-            if (wait && sleep_ns) __nanosleep(sleep_ns);
+            st_relaxed(mine + c, OS_PRE | (excl[c] + count[c]));
         }
-        st_relaxed(mine, OS_PRE | (excl + count));
     }
-    tile_base[t] = gbase[t] + excl;
+#pragma unroll
+    for (int c = 0; c < DPT; ++c) tile_base[t * DPT + c] = gbase[t * DPT + c] + excl[c];
     {   // tile-local digit offsets
-        uint32_t inc = count;
+        uint32_t tc = 0;
+#pragma unroll
+        for (int c = 0; c < DPT; ++c) tc += count[c];
+        uint32_t inc = tc;
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
             const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
@@ -444,15 +477,20 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
         __syncthreads();
         uint32_t pre = 0;
         for (int w = 0; w < warp; ++w) pre += warp_tot[w];
-        local_off[t] = pre + inc - count;
+        pre += inc - tc;
+#pragma unroll
+        for (int c = 0; c < DPT; ++c) {
+            local_off[t * DPT + c] = pre;
+            pre += count[c];
+        }
     }
     __syncthreads();
     // ---- stage in digit order, write out coalesced
 #pragma unroll
     for (int i = 0; i < OS_ITEMS; ++i) {
-        const uint32_t dig = dr[i] & 511u;
+        const uint32_t dig = dr[i] & ((2u << RB) - 1u);
         if (dig < (uint32_t)RADIX) {
-            const uint32_t lpos = local_off[dig] + wcnt[warp][dig] + (dr[i] >> 9);
+            const uint32_t lpos = local_off[dig] + wcnt[warp][dig] + (dr[i] >> RSH);
             sk[lpos] = k[i];
             if (VALS) sv[lpos] = v[i];
         }
@@ -462,7 +500,7 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const uint32_t tn = (uint32_t)min((size_t)OS_TILE, n - tbase);
     for (uint32_t i = threadIdx.x; i < tn; i += RS_THREADS) {
         const unsigned long long key = sk[i];
-        const uint32_t dg = (uint32_t)(key >> shift) & (RADIX - 1);
+        const uint32_t dg = (uint32_t)(key >> shift) & DMASK;
         const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
         keys_out[dst] = key;
         if (VALS) vals_out[dst] = sv[i];
@@ -477,57 +515,69 @@ bool onesweep_enabled(size_t n) {
     return on && n < (size_t)OS_VAL;
 }
 
-// npass onesweep passes over digits at bits lo + 8 p; hist holds each pass's
-// exclusive digit bases (k_rs_hist_scan).  Returns the pass count's parity
-// buffers swapped: on return *kin / *vin hold the result.
+// Digit plan for key bits [lo, hi): as few passes as 9-bit digits allow,
+// 8-bit digits where they suffice (DTS_RADIX9=0: 8-bit digits only; key +
+// value sorts keep 8-bit digits: a 9-bit tile with values exceeds 48 KB).
+PassPlan plan_passes(int lo, int hi, bool allow9) {
+    static const bool r9 = [] {
+        const char* e = getenv("DTS_RADIX9");
+        return !(e && e[0] == '0');
+    }();
+    const int nb = hi - lo;
+    int np = (nb + 7) / 8;
+    int n9 = 0;
+    if (r9 && allow9 && np > 1 && nb <= 9 * (np - 1)) {
+        --np;
+        n9 = nb - 8 * np;                      // passes that need a 9th bit
+    }
+    PassPlan pl{};
+    pl.npass = np;
+    int sh = lo;
+    for (int p = 0; p < np; ++p) {
+        pl.bits[p] = p < n9 ? 9 : 8;
+        pl.shift[p] = sh;
+        sh += pl.bits[p];
+    }
+    return pl;
+}
+
+template <bool VALS, int MINB, int RB>
+void launch_onesweep(uint32_t ntiles, cudaStream_t s, const unsigned long long* kin,
+                     const uint32_t* vin, size_t n, int shift, const uint32_t* gbase,
+                     uint32_t* status, uint32_t* ctr, unsigned long long* kout, uint32_t* vout,
+                     uint32_t sleep_ns) {
+    k_onesweep<VALS, MINB, RB><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, gbase, status,
+                                                             ctr, kout, vout, sleep_ns);
+}
+
+// The plan's onesweep passes; hist holds each pass's exclusive digit bases
+// (k_rs_hist_scan).  On return *kin / *vin hold the result.
 void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32_t** vin,
-                     uint32_t** vout, size_t n, int lo, int npass, const uint32_t* hist,
+                     uint32_t** vout, size_t n, const PassPlan& plan, const uint32_t* hist,
                      cudaStream_t s) {
     const uint32_t ntiles = (uint32_t)((n + OS_TILE - 1) / OS_TILE);
-    const size_t nstat = (size_t)ntiles * 256 + 32;
+    const size_t nstat = (size_t)ntiles * OS_HSTRIDE + 32;
     DevBuf<uint32_t> status(nstat, s);
-    for (int p = 0; p < npass; ++p) {
-        DTS_CUDA(cudaMemsetAsync(status.p, 0, nstat * sizeof(uint32_t), s));
-        uint32_t* ctr = status.p + (size_t)ntiles * 256;
-        static const int occ = [] {            // DTS_OS_OCC: CTAs/SM bound, keys-only
-            const char* e = getenv("DTS_OS_OCC");
-            const int v = e ? atoi(e) : 4;
-            return (v == 5 || v == 6) ? v : 4;
-        }();
-        static const uint32_t sleep_ns = [] {   // DTS_OS_SLEEP: look-back back-off (ns)
-            const char* e = getenv("DTS_OS_SLEEP");   // C4 entry sort, 5 passes: 0 ns
-            return e ? (uint32_t)atoi(e) : 256u;      // 0.984 ms, 32: 0.970, 128: 0.961,
-        }();                                          // 512: 0.957
-        // (measured on C4: window 8 0.936 ms, 16 1.03, 32 1.64 for the 5 passes)
-        static const int lb = [] {             // DTS_OS_LB: look-back window (8, 16, 32)
-            const char* e = getenv("DTS_OS_LB");
-            const int v = e ? atoi(e) : 8;
-            return (v == 16 || v == 32) ? v : 8;
-        }();
-        if (*vin)
-            k_onesweep<true, 2><<<ntiles, RS_THREADS, 0, s>>>(*kin, *vin, n, lo + 8 * p,
-                                                             hist + 256 * p, status.p, ctr, *kout,
-                                                             *vout, sleep_ns);
-        else if (lb == 16)
-            k_onesweep<false, 4, 16><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
-                                                                  hist + 256 * p, status.p, ctr,
-                                                                  *kout, nullptr, sleep_ns);
-        else if (lb == 32)
-            k_onesweep<false, 4, 32><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
-                                                                  hist + 256 * p, status.p, ctr,
-                                                                  *kout, nullptr, sleep_ns);
-        else if (occ == 5)
-            k_onesweep<false, 5><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
-                                                              hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr, sleep_ns);
-        else if (occ == 6)
-            k_onesweep<false, 6><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
-                                                              hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr, sleep_ns);
-        else
-            k_onesweep<false, 4><<<ntiles, RS_THREADS, 0, s>>>(*kin, nullptr, n, lo + 8 * p,
-                                                              hist + 256 * p, status.p, ctr,
-                                                              *kout, nullptr, sleep_ns);
+    static const uint32_t sleep_ns = [] {   // DTS_OS_SLEEP: look-back back-off (ns)
+        const char* e = getenv("DTS_OS_SLEEP");   // C4 entry sort, 5 passes: 0 ns
+        return e ? (uint32_t)atoi(e) : 256u;      // 0.984 ms, 32: 0.970, 128: 0.961,
+    }();                                          // 512: 0.957 (look-back window 8:
+                                                  // 0.936, 16: 1.03, 32: 1.64)
+    for (int p = 0; p < plan.npass; ++p) {
+        const size_t used = (size_t)ntiles << plan.bits[p];
+        DTS_CUDA(cudaMemsetAsync(status.p, 0, (used + 32) * sizeof(uint32_t), s));
+        uint32_t* ctr = status.p + used;
+        const uint32_t* gb = hist + OS_HSTRIDE * p;
+        const int sh = plan.shift[p];
+        if (plan.bits[p] == 9) {
+            launch_onesweep<false, 3, 9>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
+                                              *kout, nullptr, sleep_ns);
+        } else {
+            if (*vin) launch_onesweep<true, 2, 8>(ntiles, s, *kin, *vin, n, sh, gb, status.p, ctr,
+                                                  *kout, *vout, sleep_ns);
+            else launch_onesweep<false, 4, 8>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
+                                              *kout, nullptr, sleep_ns);
+        }
         DTS_LAUNCH_CHECK();
         std::swap(*kin, *kout);
         std::swap(*vin, *vout);
@@ -556,17 +606,17 @@ unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long
                                     int lo, int hi, cudaStream_t s) {
     if (n <= 1 || hi <= lo) return keys;
     if (onesweep_enabled(n)) {
-        const int npass = (hi - lo + 7) / 8;
-        DevBuf<uint32_t> hist((size_t)npass * 256, s);
-        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)npass * 256 * sizeof(uint32_t), s));
+        const PassPlan plan = plan_passes(lo, hi, true);
+        DevBuf<uint32_t> hist((size_t)plan.npass * OS_HSTRIDE, s);
+        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)plan.npass * OS_HSTRIDE * sizeof(uint32_t), s));
         const unsigned hb = (unsigned)std::min<size_t>((n + RS_THREADS - 1) / RS_THREADS, 148 * 8);
-        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, lo, npass, hist.p);
+        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, plan, hist.p);
         DTS_LAUNCH_CHECK();
-        k_rs_hist_scan<<<npass, RS_THREADS, 0, s>>>(hist.p);
+        k_rs_hist_scan<<<plan.npass, RS_THREADS, 0, s>>>(hist.p);
         DTS_LAUNCH_CHECK();
         unsigned long long *kin = keys, *kout = tmp;
         uint32_t *vin = nullptr, *vout = nullptr;
-        onesweep_passes(&kin, &kout, &vin, &vout, n, lo, npass, hist.p, s);
+        onesweep_passes(&kin, &kout, &vin, &vout, n, plan, hist.p, s);
         return kin;
     }
     const uint32_t ntiles = (uint32_t)((n + RS_TILE - 1) / RS_TILE);
@@ -586,17 +636,18 @@ void radix_sort_pairs(unsigned long long* keys, uint32_t* vals, unsigned long lo
                       uint32_t* vals_tmp, size_t n, int nbits, cudaStream_t s) {
     if (n <= 1 || nbits <= 0) return;
     if (onesweep_enabled(n)) {
-        const int npass = (nbits + 7) / 8;
-        DevBuf<uint32_t> hist((size_t)npass * 256, s);
-        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)npass * 256 * sizeof(uint32_t), s));
+        const PassPlan plan = plan_passes(0, nbits, false);
+        const int npass = plan.npass;
+        DevBuf<uint32_t> hist((size_t)npass * OS_HSTRIDE, s);
+        DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)npass * OS_HSTRIDE * sizeof(uint32_t), s));
         const unsigned hb = (unsigned)std::min<size_t>((n + RS_THREADS - 1) / RS_THREADS, 148 * 8);
-        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, 0, npass, hist.p);
+        k_rs_hist_all<<<hb, RS_THREADS, 0, s>>>(keys, n, plan, hist.p);
         DTS_LAUNCH_CHECK();
         k_rs_hist_scan<<<npass, RS_THREADS, 0, s>>>(hist.p);
         DTS_LAUNCH_CHECK();
         unsigned long long *kin = keys, *kout = keys_tmp;
         uint32_t *vin = vals, *vout = vals_tmp;
-        onesweep_passes(&kin, &kout, &vin, &vout, n, 0, npass, hist.p, s);
+        onesweep_passes(&kin, &kout, &vin, &vout, n, plan, hist.p, s);
         if (npass & 1) {
             DTS_CUDA(cudaMemcpyAsync(keys, kin, n * sizeof(unsigned long long),
                                      cudaMemcpyDeviceToDevice, s));

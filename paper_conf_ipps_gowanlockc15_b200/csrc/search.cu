@@ -301,8 +301,8 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     for (unsigned long long gg = g0; gg <= g1; gg += 2) {
         // home buckets of two groups issued together (8 x 128-bit loads)
         const bool two = gg + 1 <= g1;
-        unsigned long long b0 = bucket_of(gg, ht.log2cap);
-        unsigned long long b1 = two ? bucket_of(gg + 1, ht.log2cap) : b0;
+        unsigned long long b0 = bucket_of(gg, ht);
+        unsigned long long b1 = two ? bucket_of(gg + 1, ht) : b0;
         probes += two ? 2u : 1u;
         bool e0 = scan_bucket(slots + 4 * b0);
         bool e1 = two ? scan_bucket(slots + 4 * b1) : true;

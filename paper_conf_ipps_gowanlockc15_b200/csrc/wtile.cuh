@@ -100,10 +100,10 @@ __device__ __forceinline__ void prefetch_probe(const WarpSmem& S, const GridPara
     const unsigned long long key0 = make_key(g, bin, S.clo[0][qi], S.clo[1][qi] + (int32_t)(r % cn1),
                                              S.clo[2][qi] + (int32_t)(r / cn1));
     const unsigned long long g0 = key0 >> 2, g1 = (key0 + (unsigned long long)S.cn[0][qi] - 1) >> 2;
-    const CellSlot* b0 = ht.slots + 4 * bucket_of(g0, ht.log2cap);
+    const CellSlot* b0 = ht.slots + 4 * bucket_of(g0, ht);
     asm volatile("prefetch.global.L2 [%0];" ::"l"(b0));
     if (g1 != g0) {
-        const CellSlot* b1 = ht.slots + 4 * bucket_of(g1, ht.log2cap);
+        const CellSlot* b1 = ht.slots + 4 * bucket_of(g1, ht);
         asm volatile("prefetch.global.L2 [%0];" ::"l"(b1));
     }
 }
