@@ -16,7 +16,7 @@
 // A tile whose hits exceed WH (or the global stage) is marked for the
 // count-then-scatter fallback of pass 2.
 
-constexpr int WQ = 16;                  // queries per warp tile
+constexpr int WQ = 16;                  // queries per warp tile (32: 1.42 ms on C4, 16: 0.82)
 constexpr int WH = 128;                 // staged hits per warp tile
 constexpr int WT = 128;                 // threads per CTA (4 independent warps)
 constexpr int WW = WT / 32;

@@ -12,6 +12,7 @@ import dts_parity as parity
 pytestmark = pytest.mark.gpu
 
 THREADS = max(1, min(32, os.cpu_count() or 1))
+REPO = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 @pytest.fixture(scope="module")
@@ -100,6 +101,42 @@ def test_index_parameter_invariance_and_determinism(dts, oracle_mod):
                                oracle_mod)
             assert got.tobytes() == ref.tobytes(), params
         idx.free()
+
+
+def test_radix_digit_plans_and_hash_blocks_invariant(dts, oracle_mod, monkeypatch):
+    """Same result bytes whatever digit plan the build's radix sort takes
+    (8-bit only, or 9-bit digits where they save a pass) and whatever block
+    placement the cell hash uses: both only change the index layout."""
+    c = synth.make_config("C1", scale=0.1)
+    ref = None
+    for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_BLOCK": "4"}):
+        # the toggles are read once per process: run each in a subprocess
+        import subprocess
+        import sys
+        code = ("import sys; sys.path[:0] = [%r, %r]; import numpy as np, synth, "
+                "paper_conf_ipps_gowanlockc15_b200 as m; c = synth.make_config('C1', scale=0.1); "
+                "i = m.build_index(c.D); r = m.search(i, c.Q, c.d); "
+                "sys.stdout.buffer.write(r.tobytes())" % (REPO, os.path.join(REPO, "tests")))
+        out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
+                             capture_output=True, timeout=600)
+        assert out.returncode == 0, out.stderr.decode()[-2000:]
+        if ref is None:
+            ref = out.stdout
+            got = np.frombuffer(ref, dtype=dts.RESULT_DTYPE)
+            parity.compare(got, oracle_mod.search(c.D, c.Q, c.d, threads=THREADS), c.D, c.Q,
+                           c.d, oracle_mod)
+        assert out.stdout == ref, env
+
+
+def test_build_phase_timings(dts):
+    c = synth.make_config("C1", scale=0.1)
+    idx = dts.build_index(c.D)
+    inf = idx.info()
+    ph = list(inf["ms_phase"])
+    assert len(ph) == 5 and all(x >= 0.0 for x in ph)
+    assert inf["ms_build"] > 0.0
+    assert sum(ph) <= inf["ms_build"] * 1.001 + 1e-3
+    idx.free()
 
 
 def test_device_api_matches_host_api(dts):
