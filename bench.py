@@ -293,15 +293,27 @@ def run_own(args):
         # name, ms per launch-group, algorithmic bytes, model
         ("k_wtile_count", ms_count, alg_bytes,
          "64 B per candidate + 68 B per query + 64 B per hash-bucket probe"),
-        ("k_onesweep (entry sort)", ph[2], n * 8 + npass * n * 16,
-         f"8 B/key histogram read + {npass} passes x (8 B read + 8 B write) per key"),
+        ("k_onesweep (entry sort)", ph[2],
+         (0 if inf.get("build_flags", 0) & 1 else n * 8) + npass * n * 16,
+         f"{npass} passes x (8 B read + 8 B write) per key"
+         + ("" if inf.get("build_flags", 0) & 1 else " + 8 B/key histogram read")),
         ("k_gather_cells", ph[3], n * (8 + 64 + 68),
          "8 B sorted key + 64 B record read + 68 B record/id write per entry"),
         ("k_insert", ph[4], n * 8 + ncells * 16, "8 B key per entry + 16 B slot per cell"),
-        ("k_bounds", ph[0], n * 64, "64 B record read per entry"),
-        ("k_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
-         "(phase includes the host read-back of the bounds)"),
     ]
+    if inf.get("build_flags", 0) & 1:
+        kernels += [
+            ("k_bounds_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
+             "(exact bounds, packed keys and all sort-pass digit counts in one read)"),
+            ("k_bounds_sample", ph[0], 65536 * 64, "64 B per sampled entry (2^16 sample; "
+             "phase includes the host read-back)"),
+        ]
+    else:
+        kernels += [
+            ("k_bounds", ph[0], n * 64, "64 B record read per entry"),
+            ("k_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
+             "(phase includes the host read-back of the bounds)"),
+        ]
     kern = []
     for name, ms, by, model in kernels:
         a_gbs = by / (ms * 1e-3) / 1e9 if ms > 0 else None

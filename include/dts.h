@@ -229,6 +229,10 @@ typedef struct {
                                    events on the build stream): bounds, keys,
                                    radix sort, gather (+ bins, cell count),
                                    hash insert                               */
+    uint32_t build_flags;       /* bit 0: grid from a strided sample of D and
+                                   one fused read of D for exact bounds, keys
+                                   and sort histograms (phase "bounds" is then
+                                   the sample, "keys" the fused pass)        */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

@@ -79,7 +79,8 @@ class IndexInfo(ctypes.Structure):
                 ("cell_width", ctypes.c_double * 3), ("max_extent", ctypes.c_double * 3),
                 ("max_duration", ctypes.c_double), ("ms_build", ctypes.c_float),
                 ("method", ctypes.c_uint32), ("subbins", ctypes.c_uint32 * 3),
-                ("subbin_ids", ctypes.c_uint64 * 3), ("ms_phase", ctypes.c_float * 5)]
+                ("subbin_ids", ctypes.c_uint64 * 3), ("ms_phase", ctypes.c_float * 5),
+                ("build_flags", ctypes.c_uint32)]
 
     def as_dict(self):
         out = {}

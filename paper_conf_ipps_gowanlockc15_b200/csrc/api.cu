@@ -565,6 +565,7 @@ dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
         r.max_duration = idx->gp.maxdur;
         r.ms_build = idx->ms_build;
         for (int i = 0; i < 5; ++i) r.ms_phase[i] = idx->ms_phase[i];
+        r.build_flags = idx->fused_keys ? 1u : 0u;
         r.method = idx->method;
         for (int a = 0; a < 3; ++a) {
             r.subbins[a] = idx->method == DTS_METHOD_SUBBIN ? (uint32_t)idx->sb.v[a] : 0u;

@@ -87,32 +87,49 @@ __device__ void block_reduce_write(Bounds& b, Bounds* out) {
 
 // Segment validity (readings c4, c8): finite coordinates and times,
 // t_end >= t_start, finite velocity.
+__device__ __forceinline__ void bounds_add(Bounds& b, const double4 s0, const double4 s1) {
+    // (t0,x0,y0,z0), (t1,x1,y1,z1)
+    const double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
+    bool fin = isfinite(s0.x) && isfinite(s1.x);
+    for (int a = 0; a < 3; ++a) fin = fin && isfinite(p0[a]) && isfinite(p1[a]);
+    if (!fin) { b.bad |= 1; return; }
+    if (s1.x < s0.x) { b.bad |= 2; return; }
+    const double dur = s1.x - s0.x;
+    b.tmin = fmin(b.tmin, s0.x);
+    b.tmax = fmax(b.tmax, s1.x);
+    b.maxdur = fmax(b.maxdur, dur);
+    b.absmax = fmax(b.absmax, fmax(fabs(s0.x), fabs(s1.x)));
+    for (int a = 0; a < 3; ++a) {
+        const double lo = fmin(p0[a], p1[a]), hi = fmax(p0[a], p1[a]);
+        b.lo[a] = fmin(b.lo[a], lo);
+        b.hi[a] = fmax(b.hi[a], hi);
+        const double e = hi - lo;
+        b.ext[a] = fmax(b.ext[a], e);
+        b.absmax = fmax(b.absmax, fmax(fabs(lo), fabs(hi)));
+        if (dur > 0.0 && !isfinite(e / dur)) b.bad |= 4;
+        if (!isfinite(e)) b.bad |= 4;
+    }
+}
+
 __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, size_t n,
                                               Bounds* __restrict__ partial) {
     Bounds b;
     bounds_init(b);
-    for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT) {
-        double4 s0 = D[2 * i], s1 = D[2 * i + 1];   // (t0,x0,y0,z0), (t1,x1,y1,z1)
-        double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
-        bool fin = isfinite(s0.x) && isfinite(s1.x);
-        for (int a = 0; a < 3; ++a) fin = fin && isfinite(p0[a]) && isfinite(p1[a]);
-        if (!fin) { b.bad |= 1; continue; }
-        if (s1.x < s0.x) { b.bad |= 2; continue; }
-        double dur = s1.x - s0.x;
-        b.tmin = fmin(b.tmin, s0.x);
-        b.tmax = fmax(b.tmax, s1.x);
-        b.maxdur = fmax(b.maxdur, dur);
-        b.absmax = fmax(b.absmax, fmax(fabs(s0.x), fabs(s1.x)));
-        for (int a = 0; a < 3; ++a) {
-            double lo = fmin(p0[a], p1[a]), hi = fmax(p0[a], p1[a]);
-            b.lo[a] = fmin(b.lo[a], lo);
-            b.hi[a] = fmax(b.hi[a], hi);
-            double e = hi - lo;
-            b.ext[a] = fmax(b.ext[a], e);
-            b.absmax = fmax(b.absmax, fmax(fabs(lo), fabs(hi)));
-            if (dur > 0.0 && !isfinite(e / dur)) b.bad |= 4;
-            if (!isfinite(e)) b.bad |= 4;
-        }
+    for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT)
+        bounds_add(b, D[2 * i], D[2 * i + 1]);
+    block_reduce_write(b, &partial[blockIdx.x]);
+}
+
+// Bounds of the S entries i = floor(j n / S), j < S: the provisional grid of
+// the fused bounds + keys pass (any grid gives the same results -- the
+// stencils use the exact extents; see build_index_device).
+__global__ void __launch_bounds__(BT) k_bounds_sample(const double4* __restrict__ D, size_t n,
+                                                     size_t S, Bounds* __restrict__ partial) {
+    Bounds b;
+    bounds_init(b);
+    for (size_t j = (size_t)blockIdx.x * BT + threadIdx.x; j < S; j += (size_t)gridDim.x * BT) {
+        const size_t i = (size_t)(((unsigned __int128)j * n) / S);
+        bounds_add(b, D[2 * i], D[2 * i + 1]);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
 }
@@ -155,6 +172,39 @@ __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size
     } else {
         keys[i] = (k << shift) | (unsigned long long)i;
     }
+}
+
+// One read of D for three things: the exact bounds and validation (as
+// k_bounds), the packed sort keys under the provisional grid g (as k_keys),
+// and the digit counts of every pass of the coming radix sort (as
+// k_rs_hist_all) -- the separate kernels read D twice and the keys once more.
+__global__ void __launch_bounds__(BT) k_bounds_keys(const double4* __restrict__ D, size_t n,
+                                                   GridParams g,
+                                                   unsigned long long* __restrict__ keys,
+                                                   int shift, const PassPlan plan,
+                                                   Bounds* __restrict__ partial,
+                                                   uint32_t* __restrict__ hist) {
+    __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT) h[j] = 0;
+    __syncthreads();
+    Bounds b;
+    bounds_init(b);
+    for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT) {
+        const double4 s0 = D[2 * i], s1 = D[2 * i + 1];
+        bounds_add(b, s0, s1);
+        const int32_t bin = bin_of(g, s0.x);
+        const int32_t cx = cell_of(g, 0, 0.5 * (s0.y + s1.y));
+        const int32_t cy = cell_of(g, 1, 0.5 * (s0.z + s1.z));
+        const int32_t cz = cell_of(g, 2, 0.5 * (s0.w + s1.w));
+        const unsigned long long v = (make_key(g, bin, cx, cy, cz) << shift) | (unsigned long long)i;
+        keys[i] = v;
+        for (int p = 0; p < plan.npass; ++p)
+            atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
+    }
+    block_reduce_write(b, &partial[blockIdx.x]);
+    __syncthreads();
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT)
+        if (h[j]) atomicAdd(hist + j, h[j]);
 }
 
 // One non-empty cell into the bucketed open-addressing table: key -> [p, e).
@@ -582,53 +632,131 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     auto mark = [&] { DTS_CUDA(cudaEventRecord(ev[nev++], s)); };
     mark();
 
-    // 1. bounds + validation
     const int np = (int)std::min<size_t>(grid_for(n), 148 * 8);
     DevBuf<Bounds> partial(np, s), total(1, s);
-    k_bounds<<<np, BT, 0, s>>>(D, n, partial.p);
-    DTS_LAUNCH_CHECK();
-    k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
-    DTS_LAUNCH_CHECK();
-    mark();
-    Bounds hb;
-    DTS_CUDA(cudaMemcpyAsync(&hb, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
-    DTS_CUDA(cudaStreamSynchronize(s));
-    if (hb.bad & 1) throw Error(DTS_EINVAL, "entry segment with a non-finite coordinate or time");
-    if (hb.bad & 2) throw Error(DTS_EINVAL, "entry segment with t_end < t_start");
-    if (hb.bad & 4) throw Error(DTS_EINVAL, "entry segment whose speed overflows fp64");
-
-    // 2. grid
-    GridParams g{};
-    choose_grid(hb, p, g);
-    idx->gp = g;
-    for (int a = 0; a < 3; ++a) idx->max_ext[a] = hb.ext[a];
-
-    // 3-4. keys + sort
-    const unsigned long long max_key = (unsigned long long)g.m * g.cells_per_bin - 1ull;
-    idx->key_bits = bits_for(max_key);
     const int row_bits = std::max(1, bits_for(n - 1));
     static const bool allow_packed = [] {       // DTS_PACKED_SORT=0: (key, id) pairs
         const char* e = getenv("DTS_PACKED_SORT");
         return !(e && e[0] == '0');
     }();
-    const bool packed = allow_packed && row_bits + idx->key_bits <= 64;
+    static const bool allow_fused = [] {        // DTS_FUSED_KEYS=0: bounds, then keys
+        const char* e = getenv("DTS_FUSED_KEYS");
+        return !(e && e[0] == '0');
+    }();
+    auto check = [](const Bounds& b) {
+        if (b.bad & 1) throw Error(DTS_EINVAL, "entry segment with a non-finite coordinate or time");
+        if (b.bad & 2) throw Error(DTS_EINVAL, "entry segment with t_end < t_start");
+        if (b.bad & 4) throw Error(DTS_EINVAL, "entry segment whose speed overflows fp64");
+    };
+    auto key_bits_of = [](const GridParams& g) {
+        return bits_for((unsigned long long)g.m * g.cells_per_bin - 1ull);
+    };
+    // pinned landing slot of the exact bounds (read while the sort runs)
+    static thread_local Bounds* hb_pinned = [] {
+        Bounds* q = nullptr;
+        DTS_CUDA(cudaMallocHost(&q, sizeof(Bounds)));
+        return q;
+    }();
+
+    Bounds hb;
+    GridParams g{};
     DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
-    DevBuf<uint32_t> ids(packed ? 0 : n, s), ids_tmp(packed ? 0 : n, s);
-    k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p, row_bits);
-    DTS_LAUNCH_CHECK();
-    mark();
+    DevBuf<uint32_t> ids(0, s), ids_tmp(0, s);
     SortedKeys sk;
-    if (packed) {   // keys-only sort of the key bits; rows ride in the low bits
-        sk.a = radix_sort_keys(keys.p, keys_tmp.p, n, row_bits, row_bits + idx->key_bits, s);
-        sk.shift = row_bits;
-        sk.ids = nullptr;
-    } else {
-        radix_sort_pairs(keys.p, ids.p, keys_tmp.p, ids_tmp.p, n, idx->key_bits, s);
-        ids_tmp.release();
-        sk.a = keys.p;
-        sk.shift = 0;
-        sk.ids = ids.p;
+    bool done = false;
+    if (allow_fused && allow_packed && radix_onesweep(n)) {
+        // 1. bounds of a strided sample -> provisional grid.  Any grid gives
+        //    the same results: the keys only group the entries, and every
+        //    query stencil is derived from the EXACT max extent and duration
+        //    (half_ext, maxdur set below), with cell_of/bin_of clamping
+        //    entries outside the sampled domain into the boundary cells and
+        //    bins, a monotone map, so the stencil stays a superset.
+        const size_t S = std::min<size_t>(n, (size_t)1 << 16);
+        const int nps = (int)std::min<size_t>(grid_for(S), 64);
+        k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p);
+        DTS_LAUNCH_CHECK();
+        k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
+        DTS_LAUNCH_CHECK();
+        mark();
+        Bounds hs;
+        DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        check(hs);
+        choose_grid(hs, p, g);
+        const int kb = key_bits_of(g);
+        if (row_bits + kb <= 64) {
+            // 2-3. exact bounds + keys + sort histograms in one read of D
+            const PassPlan plan = plan_passes(row_bits, row_bits + kb, true);
+            DevBuf<uint32_t> hist((size_t)plan.npass * OS_HSTRIDE, s);
+            DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)plan.npass * OS_HSTRIDE * 4, s));
+            k_bounds_keys<<<np, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p, hist.p);
+            DTS_LAUNCH_CHECK();
+            k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
+            DTS_LAUNCH_CHECK();
+            DTS_CUDA(cudaMemcpyAsync(hb_pinned, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
+            cudaEvent_t eb;
+            DTS_CUDA(cudaEventCreateWithFlags(&eb, cudaEventDisableTiming));
+            DTS_CUDA(cudaEventRecord(eb, s));
+            mark();
+            // 4. sort (enqueued before the host looks at the exact bounds)
+            sk.a = radix_sort_keys_hist(keys.p, keys_tmp.p, n, plan, hist.p, s);
+            sk.shift = row_bits;
+            sk.ids = nullptr;
+            DTS_CUDA(cudaEventSynchronize(eb));
+            cudaEventDestroy(eb);
+            hb = *hb_pinned;
+            check(hb);
+            // keep the provisional grid unless the sample missed the extents
+            // badly (cells or bins far narrower or wider than the exact rule
+            // gives: correct either way, only slower)
+            GridParams gf{};
+            choose_grid(hb, p, gf);
+            bool ok = g.b >= 0.75 * gf.b && g.b <= 1.5 * gf.b;
+            for (int a = 0; a < 3; ++a) ok = ok && g.w[a] >= 0.75 * gf.w[a] && g.w[a] <= 1.5 * gf.w[a];
+            if (ok) {
+                for (int a = 0; a < 3; ++a) g.half_ext[a] = 0.5 * hb.ext[a];
+                g.maxdur = hb.maxdur;
+                idx->key_bits = kb;
+                idx->fused_keys = true;
+                done = true;
+            }
+        }
     }
+    if (!done) {
+        // 1. exact bounds + validation, 2. grid, 3. keys, 4. sort
+        k_bounds<<<np, BT, 0, s>>>(D, n, partial.p);
+        DTS_LAUNCH_CHECK();
+        k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
+        DTS_LAUNCH_CHECK();
+        if (nev == 1) mark();
+        DTS_CUDA(cudaMemcpyAsync(&hb, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        check(hb);
+        g = GridParams{};
+        choose_grid(hb, p, g);
+        idx->key_bits = key_bits_of(g);
+        const bool packed = allow_packed && row_bits + idx->key_bits <= 64;
+        if (!packed) {
+            ids.alloc(n, s);
+            ids_tmp.alloc(n, s);
+        }
+        k_keys<<<grid_for(n), BT, 0, s>>>(D, n, g, keys.p, ids.p, row_bits);
+        DTS_LAUNCH_CHECK();
+        if (nev == 2) mark();
+        if (packed) {   // keys-only sort of the key bits; rows ride in the low bits
+            sk.a = radix_sort_keys(keys.p, keys_tmp.p, n, row_bits, row_bits + idx->key_bits, s);
+            sk.shift = row_bits;
+            sk.ids = nullptr;
+        } else {
+            radix_sort_pairs(keys.p, ids.p, keys_tmp.p, ids_tmp.p, n, idx->key_bits, s);
+            ids_tmp.release();
+            sk.a = keys.p;
+            sk.shift = 0;
+            sk.ids = ids.p;
+        }
+    }
+    idx->gp = g;
+    for (int a = 0; a < 3; ++a) idx->max_ext[a] = hb.ext[a];
 
     mark();
     // 5. gather into the sorted record layout

@@ -219,6 +219,26 @@ unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long
 
 int bits_for(unsigned long long max_value);
 
+// Digit layout of a multi-pass onesweep sort: pass p sorts the digit of width
+// bits[p] (8 or 9) at bit shift[p]; its histogram is hist[p * 512 + digit].
+constexpr int OS_MAXPASS = 8;
+constexpr int OS_HSTRIDE = 512;
+struct PassPlan {
+    int npass;
+    int shift[OS_MAXPASS];
+    int bits[OS_MAXPASS];
+};
+// As few passes as 9-bit digits allow for bits [lo, hi) (8-bit where enough).
+PassPlan plan_passes(int lo, int hi, bool allow9);
+// Whether n keys go through the onesweep sort (else hist + scan + scatter).
+bool radix_onesweep(size_t n);
+// Keys-only onesweep sort by the plan, with the per-pass digit counts
+// already accumulated in hist (npass x 512, e.g. by the kernel that wrote the
+// keys).  Returns the buffer (keys or tmp) holding the sorted keys.
+unsigned long long* radix_sort_keys_hist(unsigned long long* keys, unsigned long long* tmp,
+                                         size_t n, const PassPlan& plan, uint32_t* hist,
+                                         cudaStream_t s);
+
 // Device block cache (alloc.cu) for memory that outlives one API call.
 void* cache_alloc(size_t bytes);
 void cache_free(void* p);
@@ -240,6 +260,7 @@ struct dts_index {
     double max_ext[3] = {0, 0, 0};
     float ms_build = 0.f;
     float ms_phase[5] = {0, 0, 0, 0, 0};   // bounds, keys, sort, gather, insert
+    bool fused_keys = false;       // sampled grid + one-read bounds/keys/histograms
     int key_bits = 0;
     uint32_t method = 0;           // dts_method
     dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only

@@ -301,16 +301,6 @@ __device__ __forceinline__ void st_relaxed(uint32_t* p, uint32_t v) {
     asm volatile("st.relaxed.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
-// Digit layout of a multi-pass sort: pass p sorts the digit of width
-// bits[p] (8 or 9) at bit shift[p]; its histogram is hist[p * 512 + digit].
-constexpr int OS_MAXPASS = 8;
-constexpr int OS_HSTRIDE = 512;
-struct PassPlan {
-    int npass;
-    int shift[OS_MAXPASS];
-    int bits[OS_MAXPASS];
-};
-
 // Digit histograms of all passes in one read of the keys (caller zeroes hist).
 __global__ void __launch_bounds__(RS_THREADS) k_rs_hist_all(const unsigned long long* __restrict__ keys,
                                                             size_t n, const PassPlan plan,
@@ -518,6 +508,8 @@ bool onesweep_enabled(size_t n) {
 // Digit plan for key bits [lo, hi): as few passes as 9-bit digits allow,
 // 8-bit digits where they suffice (DTS_RADIX9=0: 8-bit digits only; key +
 // value sorts keep 8-bit digits: a 9-bit tile with values exceeds 48 KB).
+}  // namespace
+
 PassPlan plan_passes(int lo, int hi, bool allow9) {
     static const bool r9 = [] {
         const char* e = getenv("DTS_RADIX9");
@@ -541,6 +533,7 @@ PassPlan plan_passes(int lo, int hi, bool allow9) {
     return pl;
 }
 
+namespace {
 template <bool VALS, int MINB, int RB>
 void launch_onesweep(uint32_t ntiles, cudaStream_t s, const unsigned long long* kin,
                      const uint32_t* vin, size_t n, int shift, const uint32_t* gbase,
@@ -601,6 +594,19 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
     DTS_LAUNCH_CHECK();
 }
 }  // namespace
+
+unsigned long long* radix_sort_keys_hist(unsigned long long* keys, unsigned long long* tmp,
+                                         size_t n, const PassPlan& plan, uint32_t* hist,
+                                         cudaStream_t s) {
+    k_rs_hist_scan<<<plan.npass, RS_THREADS, 0, s>>>(hist);
+    DTS_LAUNCH_CHECK();
+    unsigned long long *kin = keys, *kout = tmp;
+    uint32_t *vin = nullptr, *vout = nullptr;
+    onesweep_passes(&kin, &kout, &vin, &vout, n, plan, hist, s);
+    return kin;
+}
+
+bool radix_onesweep(size_t n) { return onesweep_enabled(n); }
 
 unsigned long long* radix_sort_keys(unsigned long long* keys, unsigned long long* tmp, size_t n,
                                     int lo, int hi, cudaStream_t s) {
