@@ -88,27 +88,31 @@ __device__ void block_reduce_write(Bounds& b, Bounds* out) {
 // Segment validity (readings c4, c8): finite coordinates and times,
 // t_end >= t_start, finite velocity.
 __device__ __forceinline__ void bounds_add(Bounds& b, const double4 s0, const double4 s1) {
-    // (t0,x0,y0,z0), (t1,x1,y1,z1)
-    const double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
-    bool fin = isfinite(s0.x) && isfinite(s1.x);
-    for (int a = 0; a < 3; ++a) fin = fin && isfinite(p0[a]) && isfinite(p1[a]);
-    if (!fin) { b.bad |= 1; return; }
+    // (t0,x0,y0,z0), (t1,x1,y1,z1); v - v is 0 for a finite v and NaN
+    // otherwise, so one comparison checks all eight values
+    const double z = ((s0.x - s0.x) + (s1.x - s1.x)) + ((s0.y - s0.y) + (s1.y - s1.y)) +
+                     ((s0.z - s0.z) + (s1.z - s1.z)) + ((s0.w - s0.w) + (s1.w - s1.w));
+    if (!(z == 0.0)) { b.bad |= 1; return; }
     if (s1.x < s0.x) { b.bad |= 2; return; }
     const double dur = s1.x - s0.x;
     b.tmin = fmin(b.tmin, s0.x);
     b.tmax = fmax(b.tmax, s1.x);
     b.maxdur = fmax(b.maxdur, dur);
-    b.absmax = fmax(b.absmax, fmax(fabs(s0.x), fabs(s1.x)));
+    const double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
+    double emax = 0.0;
+#pragma unroll
     for (int a = 0; a < 3; ++a) {
         const double lo = fmin(p0[a], p1[a]), hi = fmax(p0[a], p1[a]);
         b.lo[a] = fmin(b.lo[a], lo);
         b.hi[a] = fmax(b.hi[a], hi);
         const double e = hi - lo;
         b.ext[a] = fmax(b.ext[a], e);
-        b.absmax = fmax(b.absmax, fmax(fabs(lo), fabs(hi)));
-        if (dur > 0.0 && !isfinite(e / dur)) b.bad |= 4;
-        if (!isfinite(e)) b.bad |= 4;
+        emax = fmax(emax, e);
     }
+    // speed |p1 - p0| / dur must be finite on every axis: an infinite extent,
+    // or (only possible for dur < 1) an overflowing quotient of the largest
+    // extent (division is monotone in the numerator)
+    if (!isfinite(emax) || (dur > 0.0 && dur < 1.0 && !isfinite(emax / dur))) b.bad |= 4;
 }
 
 __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, size_t n,
@@ -139,6 +143,12 @@ __global__ void __launch_bounds__(BT) k_bounds_final(const Bounds* __restrict__ 
     Bounds b;
     bounds_init(b);
     for (int i = threadIdx.x; i < np; i += BT) bounds_merge(b, partial[i]);
+    // max |coordinate or time| of the valid entries = max |bound| (the
+    // per-entry values need not be visited)
+    if (b.tmin <= b.tmax) {
+        b.absmax = fmax(fabs(b.tmin), fabs(b.tmax));
+        for (int a = 0; a < 3; ++a) b.absmax = fmax(b.absmax, fmax(fabs(b.lo[a]), fabs(b.hi[a])));
+    }
     block_reduce_write(b, out);
 }
 
@@ -370,9 +380,23 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
             const double4 s0 = r0[k], s1 = r1[k];
             const double dur = s1.x - s0.x;
             *soa.at(0, p) = make_double2(s0.x, s1.x);
-            *soa.at(1, p) = make_double2(s0.y, velocity(s0.y, s1.y, dur));
-            *soa.at(2, p) = make_double2(s0.z, velocity(s0.z, s1.z, dur));
-            *soa.at(3, p) = make_double2(s0.w, velocity(s0.w, s1.w, dur));
+            // one reciprocal instead of three divisions (a rounding-level
+            // change of v, reading c8); exact divisions when a product is
+            // not finite (subnormal durations, speeds near DBL_MAX), so v is
+            // finite whenever the validated quotient is
+            const double inv = dur > 0.0 ? 1.0 / dur : 0.0;
+            double vx, vy, vz;
+            vx = (s1.y - s0.y) * inv;
+            vy = (s1.z - s0.z) * inv;
+            vz = (s1.w - s0.w) * inv;
+            if (!(isfinite(vx) && isfinite(vy) && isfinite(vz))) {
+                vx = velocity(s0.y, s1.y, dur);
+                vy = velocity(s0.z, s1.z, dur);
+                vz = velocity(s0.w, s1.w, dur);
+            }
+            *soa.at(1, p) = make_double2(s0.y, vx);
+            *soa.at(2, p) = make_double2(s0.z, vy);
+            *soa.at(3, p) = make_double2(s0.w, vz);
             soa.eid[p] = id[k];
             s_bin[1 + k * BT + threadIdx.x] = bin_of(g, s0.x);
             const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);

@@ -128,6 +128,56 @@ def test_radix_digit_plans_and_hash_blocks_invariant(dts, oracle_mod, monkeypatc
         assert out.stdout == ref, env
 
 
+def _unsampled_positions(n, k):
+    """k positions that the build's 2^16-entry stride sample does not read."""
+    S = min(n, 1 << 16)
+    sampled = set((np.arange(S, dtype=np.uint64) * np.uint64(n) // np.uint64(S)).tolist())
+    out = [i for i in range(1, n) if i not in sampled][:k]
+    assert len(out) == k
+    return out
+
+
+@pytest.mark.parametrize("kind", ["long_segments", "far_outliers"])
+def test_sampled_grid_misses_outliers(dts, oracle_mod, kind):
+    """The build derives its grid from a strided sample of D; entries the
+    sample misses -- segments far longer than any sampled one (the grid is
+    then rebuilt from the exact bounds) or short segments far outside the
+    sampled domain (they clamp into the boundary cells) -- must still be
+    found, with the stencils taken from the exact extents."""
+    c = synth.make_config("C1", scale=0.2)
+    D = c.D.reshape(-1, 8).copy()
+    n = D.shape[0]
+    assert n > (1 << 16)
+    pos = _unsampled_positions(n, 6)
+    g = synth.rng(77)
+    for k, i in enumerate(pos):
+        t0 = float(g.uniform(0, 150))
+        if kind == "long_segments":      # 40 time units, 30 units of x travel
+            D[i] = [t0, -15.0 + k, 0.5, 0.0, t0 + 40.0, 15.0 + k, 0.5, 0.0]
+        else:                            # short segments 1e3 away
+            D[i] = [t0, 1000.0 + k, -800.0, 5.0, t0 + 1.0, 1000.01 + k, -800.0, 5.0]
+    # queries: the headline ones plus segments that cross each outlier
+    extra = []
+    for i in pos:
+        t0, x0, y0, z0, t1, x1, y1, z1 = D[i]
+        tm = 0.5 * (t0 + t1)
+        xm, ym, zm = 0.5 * (x0 + x1), 0.5 * (y0 + y1), 0.5 * (z0 + z1)
+        extra.append([tm - 0.5, xm, ym - 0.002, zm, tm + 0.5, xm, ym + 0.002, zm])
+    Q = np.concatenate([c.Q.reshape(-1, 8)[:400], np.array(extra)]).astype(np.float64)
+    idx = dts.build_index(D)
+    inf = idx.info()
+    got = dts.search(idx, Q, c.d)
+    ora = oracle_mod.search(D, Q, c.d, threads=THREADS)
+    info = parity.compare(got, ora, D, Q, c.d, oracle_mod)
+    hit = set(zip(got["query_id"].tolist(), got["entry_id"].tolist()))
+    for k, i in enumerate(pos):
+        assert (400 + k, i) in hit, (kind, k)
+    assert info["common"] >= len(pos)
+    if kind == "long_segments":          # exact extent, not the sample's
+        assert inf["max_extent"][0] >= 30.0
+    idx.free()
+
+
 def test_build_phase_timings(dts):
     c = synth.make_config("C1", scale=0.1)
     idx = dts.build_index(c.D)
