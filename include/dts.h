@@ -147,7 +147,12 @@ dts_status dts_build_index(const dts_segment* D, size_t n,
                            dts_index** out_index);
 
 /* Same, from device memory: D_dev points to n dts_segment records in device
- * memory of params->device, 16-byte aligned. Not retained after return. */
+ * memory of params->device, 16-byte aligned.  Validation errors are returned
+ * synchronously; the last build kernels may still run on cuda_stream when
+ * the call returns (stream-ordered, like a kernel launch), so D_dev and the
+ * params' device arrays must stay valid until the stream reaches that point
+ * (later work on the stream, or dts_index_get_info, which waits for it).
+ * Searches on other streams wait for the build by themselves. Not retained. */
 dts_status dts_build_index_device(const dts_segment* D_dev, size_t n,
                                   const dts_index_params* params,
                                   void* cuda_stream, dts_index** out_index);

@@ -106,6 +106,9 @@ void free_index_memory(dts_index* idx) {
     cudaSetDevice(idx->device);
     // blocks go back to the device cache (alloc.cu) for the next build
     cudaDeviceSynchronize();
+    for (int i = 0; i < idx->nev; ++i) cudaEventDestroy(idx->ev[i]);
+    idx->nev = 0;
+    idx->ready = nullptr;
     cache_free(idx->block);
     cache_free(idx->ht.slots);
     cache_free(idx->etraj);
@@ -188,6 +191,7 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
         } else {
             check_aligned(D, "D_dev");
             build_index_device(idx, D, n, p, s);
+            return;                 // asynchronous on s after validation (dts.h)
         }
         DTS_CUDA(cudaStreamSynchronize(s));
     });
@@ -552,6 +556,8 @@ void dts_free_index(dts_index* index) {
 dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
     return guarded([&] {
         if (!idx || !info) throw Error(DTS_EINVAL, "NULL argument");
+        cudaSetDevice(idx->device);
+        index_times(const_cast<dts_index*>(idx));
         dts_index_info r{};
         r.n = idx->n;
         r.cells = idx->n_cells;

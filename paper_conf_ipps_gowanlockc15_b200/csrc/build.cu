@@ -188,28 +188,50 @@ __global__ void __launch_bounds__(BT) k_keys(const double4* __restrict__ D, size
 // k_bounds), the packed sort keys under the provisional grid g (as k_keys),
 // and the digit counts of every pass of the coming radix sort (as
 // k_rs_hist_all) -- the separate kernels read D twice and the keys once more.
-__global__ void __launch_bounds__(BT) k_bounds_keys(const double4* __restrict__ D, size_t n,
-                                                   GridParams g,
-                                                   unsigned long long* __restrict__ keys,
-                                                   int shift, const PassPlan plan,
-                                                   Bounds* __restrict__ partial,
-                                                   uint32_t* __restrict__ hist) {
+__device__ __forceinline__ unsigned long long packed_key(const GridParams& g, const double4 s0,
+                                                         const double4 s1, int shift, size_t i) {
+    const int32_t bin = bin_of(g, s0.x);
+    const int32_t cx = cell_of(g, 0, 0.5 * (s0.y + s1.y));
+    const int32_t cy = cell_of(g, 1, 0.5 * (s0.z + s1.z));
+    const int32_t cz = cell_of(g, 2, 0.5 * (s0.w + s1.w));
+    return (make_key(g, bin, cx, cy, cz) << shift) | (unsigned long long)i;
+}
+
+__global__ void __launch_bounds__(BT, 3) k_bounds_keys(const double4* __restrict__ D, size_t n,
+                                                      GridParams g,
+                                                      unsigned long long* __restrict__ keys,
+                                                      int shift, const PassPlan plan,
+                                                      Bounds* __restrict__ partial,
+                                                      uint32_t* __restrict__ hist) {
     __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
     for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT) h[j] = 0;
     __syncthreads();
     Bounds b;
     bounds_init(b);
-    for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT) {
-        const double4 s0 = D[2 * i], s1 = D[2 * i + 1];
-        bounds_add(b, s0, s1);
-        const int32_t bin = bin_of(g, s0.x);
-        const int32_t cx = cell_of(g, 0, 0.5 * (s0.y + s1.y));
-        const int32_t cy = cell_of(g, 1, 0.5 * (s0.z + s1.z));
-        const int32_t cz = cell_of(g, 2, 0.5 * (s0.w + s1.w));
-        const unsigned long long v = (make_key(g, bin, cx, cy, cz) << shift) | (unsigned long long)i;
-        keys[i] = v;
+    auto count = [&](unsigned long long v) {
         for (int p = 0; p < plan.npass; ++p)
             atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
+    };
+    const size_t stride = (size_t)gridDim.x * BT;
+    size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
+    for (; i + stride < n; i += 2 * stride) {      // two entries in flight per thread
+        const size_t j = i + stride;
+        const double4 a0 = D[2 * i], a1 = D[2 * i + 1], c0 = D[2 * j], c1 = D[2 * j + 1];
+        bounds_add(b, a0, a1);
+        bounds_add(b, c0, c1);
+        const unsigned long long va = packed_key(g, a0, a1, shift, i);
+        const unsigned long long vc = packed_key(g, c0, c1, shift, j);
+        keys[i] = va;
+        keys[j] = vc;
+        count(va);
+        count(vc);
+    }
+    if (i < n) {
+        const double4 a0 = D[2 * i], a1 = D[2 * i + 1];
+        bounds_add(b, a0, a1);
+        const unsigned long long va = packed_key(g, a0, a1, shift, i);
+        keys[i] = va;
+        count(va);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
     __syncthreads();
@@ -650,8 +672,15 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     if (n == 0) return;
     const double4* D = reinterpret_cast<const double4*>(D_dev);
     // phase events: start, bounds, keys, sort, gather, insert (+ end)
-    cudaEvent_t ev[7];
-    for (auto& e : ev) DTS_CUDA(cudaEventCreate(&e));
+    // (kept in the index: the build returns without waiting for its last
+    //  kernels, the times are read by dts_index_get_info)
+    struct Events {
+        cudaEvent_t ev[7];
+        bool keep = false;
+        Events() { for (auto& e : ev) DTS_CUDA(cudaEventCreate(&e)); }
+        ~Events() { if (!keep) for (auto& e : ev) cudaEventDestroy(e); }
+    } evs;
+    cudaEvent_t* ev = evs.ev;
     int nev = 0;
     auto mark = [&] { DTS_CUDA(cudaEventRecord(ev[nev++], s)); };
     mark();
@@ -822,7 +851,11 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_CUDA(cudaStreamSynchronize(s));
     idx->n_cells = hc;
     int log2cap = 6;
-    while ((1ull << log2cap) < 2 * hc) ++log2cap;
+    static const double hload = [] {          // DTS_HASH_SLOTS: slots per cell (>= 1.1)
+        const char* e = getenv("DTS_HASH_SLOTS");
+        return e ? std::max(1.1, atof(e)) : 2.0;
+    }();
+    while ((double)(1ull << log2cap) < hload * (double)hc) ++log2cap;
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
     static const int hblk = [] {              // DTS_HASH_BLOCK: log2 buckets per block
@@ -869,13 +902,24 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     }
 
     mark();
-    DTS_CUDA(cudaEventSynchronize(ev[nev - 1]));
-    DTS_CUDA(cudaEventElapsedTime(&idx->ms_build, ev[0], ev[nev - 1]));
+    // no wait here: the last kernels may still run when the build returns;
+    // searches on other streams wait for `ready` (search_device), and the
+    // phase times are read on demand (index_times)
+    for (int i = 0; i < 7; ++i) idx->ev[i] = ev[i];
+    idx->nev = nev;
+    evs.keep = true;
+    idx->ready = ev[nev - 1];
+}
+
+void index_times(dts_index* idx) {
+    if (idx->nev == 0 || idx->timed) return;
+    DTS_CUDA(cudaEventSynchronize(idx->ev[idx->nev - 1]));
+    DTS_CUDA(cudaEventElapsedTime(&idx->ms_build, idx->ev[0], idx->ev[idx->nev - 1]));
     for (int i = 0; i < 5; ++i) {
         idx->ms_phase[i] = 0.f;
-        if (i + 1 < nev) cudaEventElapsedTime(&idx->ms_phase[i], ev[i], ev[i + 1]);
+        if (i + 1 < idx->nev) cudaEventElapsedTime(&idx->ms_phase[i], idx->ev[i], idx->ev[i + 1]);
     }
-    for (auto& e : ev) cudaEventDestroy(e);
+    idx->timed = true;
 }
 
 }  // namespace dts

@@ -261,6 +261,10 @@ struct dts_index {
     float ms_build = 0.f;
     float ms_phase[5] = {0, 0, 0, 0, 0};   // bounds, keys, sort, gather, insert
     bool fused_keys = false;       // sampled grid + one-read bounds/keys/histograms
+    cudaEvent_t ev[7] = {};        // build phase events (index_times)
+    int nev = 0;
+    bool timed = false;
+    cudaEvent_t ready = nullptr;   // end of the build (= ev[nev - 1])
     int key_bits = 0;
     uint32_t method = 0;           // dts_method
     dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only
@@ -272,6 +276,8 @@ struct dts_index {
 namespace dts {
 void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                         const dts_index_params& p, cudaStream_t s);
+// Waits for the end of the build and fills ms_build / ms_phase.
+void index_times(dts_index* idx);
 struct SearchOut {
     dts_result* results = nullptr;   // device, cudaMalloc'd (caller owns)
     size_t count = 0;

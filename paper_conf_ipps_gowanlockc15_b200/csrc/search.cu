@@ -550,6 +550,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         return;
     }
     const double4* Q = reinterpret_cast<const double4*>(Q_dev);
+    if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));   // build may still run
     DevBuf<Counters> ctr(1, s);
     DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
 
