@@ -277,6 +277,38 @@ __global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
 }
 
 
+// Tiled insert: the tile's keys (plus the one before) are staged in shared
+// memory, so a cell head finds its run's end there (global reads only for a
+// run that crosses the tile's end); then one CAS per cell as in k_insert.
+template <int ITEMS>
+__global__ void __launch_bounds__(BT) k_insert_tiled(const SortedKeys keys, size_t n,
+                                                    HashTable ht) {
+    constexpr int TILE = BT * ITEMS;
+    __shared__ unsigned long long s_key[TILE + 1];
+    const size_t p0 = (size_t)blockIdx.x * TILE;
+    const uint32_t tn = (uint32_t)min((size_t)TILE, n - p0);
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc < tn) s_key[1 + loc] = keys.key(p0 + loc);
+    }
+    if (threadIdx.x == 0) s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc >= tn) continue;
+        const unsigned long long key = s_key[1 + loc];
+        if (p0 + loc != 0 && s_key[loc] == key) continue;
+        uint32_t e = loc + 1;
+        while (e < tn && s_key[1 + e] == key) ++e;
+        size_t end = p0 + e;
+        if (e == tn)
+            while (end < n && keys.key(end) == key) ++end;
+        insert_cell(ht, key, (uint32_t)(p0 + loc), (uint32_t)end);
+    }
+}
+
 // ITEMS sorted positions per thread (strided by the grid so key loads stay
 // coalesced): the cell heads among them issue their first-choice CAS
 // together, so ITEMS atomics are in flight per thread instead of one; a head
@@ -379,8 +411,11 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
     if (threadIdx.x == 0) {
         s_cnt = 0;
         if (p0 > 0) {                                  // halo: sorted position p0 - 1
-            s_key[0] = sk.key(p0 - 1);
-            s_bin[0] = bin_of(g, D[2 * (size_t)sk.row(p0 - 1)].x);
+            // keys are bin-major (key = bin * cells_per_bin + cell), so the
+            // halo's bin needs no dependent load of its record
+            const unsigned long long hk = sk.key(p0 - 1);
+            s_key[0] = hk;
+            s_bin[0] = (int32_t)(hk / g.cells_per_bin);
         } else {
             s_key[0] = ~0ull;
             s_bin[0] = -1;
@@ -402,20 +437,13 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
             const double4 s0 = r0[k], s1 = r1[k];
             const double dur = s1.x - s0.x;
             *soa.at(0, p) = make_double2(s0.x, s1.x);
-            // one reciprocal instead of three divisions (a rounding-level
-            // change of v, reading c8); exact divisions when a product is
-            // not finite (subnormal durations, speeds near DBL_MAX), so v is
-            // finite whenever the validated quotient is
-            const double inv = dur > 0.0 ? 1.0 / dur : 0.0;
-            double vx, vy, vz;
-            vx = (s1.y - s0.y) * inv;
-            vy = (s1.z - s0.z) * inv;
-            vz = (s1.w - s0.w) * inv;
-            if (!(isfinite(vx) && isfinite(vy) && isfinite(vz))) {
-                vx = velocity(s0.y, s1.y, dur);
-                vy = velocity(s0.z, s1.z, dur);
-                vz = velocity(s0.w, s1.w, dur);
-            }
+            // three correctly rounded divisions, not one reciprocal and
+            // three products: equal ratios must give equal velocities, or a
+            // pair of coincident segments at d = 0 (no relative motion, the
+            // whole overlap within d) degenerates to a single instant
+            const double vx = velocity(s0.y, s1.y, dur);
+            const double vy = velocity(s0.z, s1.z, dur);
+            const double vz = velocity(s0.w, s1.w, dur);
             *soa.at(1, p) = make_double2(s0.y, vx);
             *soa.at(2, p) = make_double2(s0.z, vy);
             *soa.at(3, p) = make_double2(s0.w, vz);
@@ -865,14 +893,16 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     idx->ht.blk = std::min(hblk, log2cap - 4);
     idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
     DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
-    // (measured on C4: 1 cell per thread 0.56 ms incl. the memset; batching
-    //  the first CAS of 2 / 4 / 8 cells: 0.59 / 0.70 / 0.91 ms)
-    static const int ins = [] {               // DTS_INSERT_ITEMS: 1 (k_insert), 2, 4, 8
-        const char* e = getenv("DTS_INSERT_ITEMS");
-        const int v = e ? atoi(e) : 1;
-        return (v == 2 || v == 4 || v == 8) ? v : 1;
+    // (measured on C4, incl. the memset: tiled 0.550 ms, 1 cell per thread
+    //  with global key scans 0.565; batching the first CAS of 2 / 4 / 8
+    //  cells: 0.59 / 0.70 / 0.91 ms)
+    static const int ins = [] {               // DTS_INSERT_ITEMS: 0 tiled (k_insert_tiled),
+        const char* e = getenv("DTS_INSERT_ITEMS");   // 1 (k_insert), 2, 4, 8 batched
+        const int v = e ? atoi(e) : 0;
+        return (v == 0 || v == 2 || v == 4 || v == 8) ? v : 1;
     }();
-    if (ins == 1) k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
+    if (ins == 0) k_insert_tiled<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    else if (ins == 1) k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
     else if (ins == 2) k_insert_batched<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(sk, n, idx->ht);
     else if (ins == 4) k_insert_batched<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
     else k_insert_batched<8><<<grid_for((n + 7) / 8), BT, 0, s>>>(sk, n, idx->ht);
