@@ -20,7 +20,7 @@ __all__ = ["RESULT_DTYPE", "IndexParams", "Index", "DeviceResults", "DTSError",
            "lib_path", "load", "EXPORTED_SYMBOLS"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIB_PATH = os.path.join(_HERE, "libdts.so")
+_LIB_PATH = os.environ.get("DTS_LIB") or os.path.join(_HERE, "libdts.so")   # DTS_LIB: A/B builds
 
 RESULT_DTYPE = np.dtype([("query_id", "<u4"), ("entry_id", "<u4"),
                          ("t_start", "<f8"), ("t_end", "<f8")], align=True)

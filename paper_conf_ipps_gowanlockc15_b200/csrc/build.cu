@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, si
     Bounds b;
     bounds_init(b);
     for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT)
-        bounds_add(b, D[2 * i], D[2 * i + 1]);
+        bounds_add(b, ld256(D + 2 * i), ld256(D + 2 * i + 1));
     block_reduce_write(b, &partial[blockIdx.x]);
 }
 
@@ -216,7 +216,8 @@ __global__ void __launch_bounds__(BT, 3) k_bounds_keys(const double4* __restrict
     size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
     for (; i + stride < n; i += 2 * stride) {      // two entries in flight per thread
         const size_t j = i + stride;
-        const double4 a0 = D[2 * i], a1 = D[2 * i + 1], c0 = D[2 * j], c1 = D[2 * j + 1];
+        const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
+        const double4 c0 = ld256(D + 2 * j), c1 = ld256(D + 2 * j + 1);
         bounds_add(b, a0, a1);
         bounds_add(b, c0, c1);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
@@ -227,7 +228,7 @@ __global__ void __launch_bounds__(BT, 3) k_bounds_keys(const double4* __restrict
         count(vc);
     }
     if (i < n) {
-        const double4 a0 = D[2 * i], a1 = D[2 * i + 1];
+        const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
         bounds_add(b, a0, a1);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
         keys[i] = va;
@@ -408,14 +409,13 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
         if (p < n) {
             const double4 s0 = r0[k], s1 = r1[k];
             const double dur = s1.x - s0.x;
-            *soa.at(0, p) = make_double2(s0.x, s1.x);
             // three correctly rounded divisions, not one reciprocal and
             // three products: equal ratios must give equal velocities, or a
             // pair of coincident segments at d = 0 (no relative motion, the
             // whole overlap within d) degenerates to a single instant
-            *soa.at(1, p) = make_double2(s0.y, velocity(s0.y, s1.y, dur));
-            *soa.at(2, p) = make_double2(s0.z, velocity(s0.z, s1.z, dur));
-            *soa.at(3, p) = make_double2(s0.w, velocity(s0.w, s1.w, dur));
+            soa.store4(p, make_double2(s0.x, s1.x), make_double2(s0.y, velocity(s0.y, s1.y, dur)),
+                       make_double2(s0.z, velocity(s0.z, s1.z, dur)),
+                       make_double2(s0.w, velocity(s0.w, s1.w, dur)));
             soa.eid[p] = id[k];
             s_bin[1 + k * BT + threadIdx.x] = bin_of(g, s0.x);
             const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);
@@ -521,8 +521,8 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
     for (int k = 0; k < ITEMS; ++k) {
         const size_t p = p0 + (size_t)k * BT + threadIdx.x;
         if (p < n) {
-            r0[k] = D[2 * (size_t)id[k]];
-            r1[k] = D[2 * (size_t)id[k] + 1];
+            r0[k] = ld256(D + 2 * (size_t)id[k]);
+            r1[k] = ld256(D + 2 * (size_t)id[k] + 1);
         }
     }
     gather_tile<ITEMS>(n, p0, id, r0, r1, soa, g, bin_start, bin_t0min, bin_t1max, count, s_key,

@@ -89,6 +89,11 @@ struct SegSoA {
 #ifdef __CUDACC__
     __device__ __forceinline__ double2* at(int k, size_t p) const { return rec + k * ss + p * es; }
     __device__ __forceinline__ double2 ld(int k, size_t p) const { return __ldg(at(k, p)); }
+    // all four streams of position p (record layout: two 256-bit loads)
+    __device__ __forceinline__ void load4(size_t p, double2& st, double2& sx, double2& sy,
+                                          double2& sz) const;
+    __device__ __forceinline__ void store4(size_t p, double2 st, double2 sx, double2 sy,
+                                           double2 sz) const;
 #endif
 };
 
@@ -180,6 +185,52 @@ __device__ __forceinline__ unsigned long long make_key(const GridParams& g, int3
            ((unsigned long long)cz * (unsigned long long)g.nc[1] + (unsigned long long)cy) *
                (unsigned long long)g.nc[0] +
            (unsigned long long)cx;
+}
+
+// 256-bit read-only load (sm_100: LDG.E.256; one 32-byte sector per lane).
+__device__ __forceinline__ double4 ld256(const double4* p) {
+    double4 v;
+    asm("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%4];"
+                 : "=d"(v.x), "=d"(v.y), "=d"(v.z), "=d"(v.w) : "l"(p));
+    return v;
+}
+__device__ __forceinline__ ulonglong4 ld256u(const void* p) {
+    ulonglong4 v;
+    asm("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];"
+                 : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
+    return v;
+}
+
+__device__ __forceinline__ void SegSoA::load4(size_t p, double2& st, double2& sx, double2& sy,
+                                              double2& sz) const {
+    if (es == 4) {
+        const double4* r = reinterpret_cast<const double4*>(rec + 4 * p);
+        const double4 a = ld256(r), b = ld256(r + 1);
+        st = make_double2(a.x, a.y);
+        sx = make_double2(a.z, a.w);
+        sy = make_double2(b.x, b.y);
+        sz = make_double2(b.z, b.w);
+    } else {
+        st = ld(0, p);
+        sx = ld(1, p);
+        sy = ld(2, p);
+        sz = ld(3, p);
+    }
+}
+__device__ __forceinline__ void SegSoA::store4(size_t p, double2 st, double2 sx, double2 sy,
+                                               double2 sz) const {
+    if (es == 4) {
+        double* r = reinterpret_cast<double*>(rec + 4 * p);
+        asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r), "d"(st.x), "d"(st.y),
+                     "d"(sx.x), "d"(sx.y) : "memory");
+        asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r + 4), "d"(sy.x), "d"(sy.y),
+                     "d"(sz.x), "d"(sz.y) : "memory");
+    } else {
+        *at(0, p) = st;
+        *at(1, p) = sx;
+        *at(2, p) = sy;
+        *at(3, p) = sz;
+    }
 }
 
 // Monotone map of doubles to unsigned 64-bit integers (for atomic min/max).

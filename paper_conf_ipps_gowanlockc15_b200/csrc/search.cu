@@ -286,14 +286,17 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     // returns whether the bucket has a free slot (end of the chain)
     auto scan_bucket = [&](const ulonglong2* B) -> bool {
         bool empty = false;
+        // the 64-byte bucket as two 256-bit loads: slots (key, start | end << 32)
+        const ulonglong4 h0 = ld256u(B), h1 = ld256u(B + 2);
+        const unsigned long long kk[4] = {h0.x, h0.z, h1.x, h1.z};
+        const unsigned long long se[4] = {h0.y, h0.w, h1.y, h1.w};
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
-            const ulonglong2 s = __ldg(B + i);
-            if (s.x >= key0 && s.x < kend) {
-                first = min(first, (uint32_t)s.y);
-                last = max(last, (uint32_t)(s.y >> 32));
+            if (kk[i] - key0 < kend - key0) {      // key0 <= key < kend
+                first = min(first, (uint32_t)se[i]);
+                last = max(last, (uint32_t)(se[i] >> 32));
             }
-            empty |= (s.x == EMPTY_KEY);
+            empty |= (kk[i] == EMPTY_KEY);
         }
         return empty;
     };
@@ -440,9 +443,11 @@ __global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
                     if (s_excl[warp][j + step] <= t) j += step;
                 p = s_start[warp][j] + (uint32_t)(t - s_excl[warp][j]);
                 if (ind) p = __ldg(ind + p);
-                if (!(a.excl && __ldg(a.etraj + p) == qtraj))
-                    hit = refine(q, a.soa.ld(0, p), a.soa.ld(1, p), a.soa.ld(2, p),
-                                 a.soa.ld(3, p), d2, r0, r1);
+                if (!(a.excl && __ldg(a.etraj + p) == qtraj)) {
+                    double2 et, ex, ey, ez;
+                    a.soa.load4(p, et, ex, ey, ez);
+                    hit = refine(q, et, ex, ey, ez, d2, r0, r1);
+                }
             }
             const uint32_t bal = __ballot_sync(0xffffffffu, hit);
             if (hit) {

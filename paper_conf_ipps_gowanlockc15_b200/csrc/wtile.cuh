@@ -218,10 +218,9 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     if (i1) p1 = __ldg(sb_ids(a.sb, i1) + p1);   // subbin id array slot
                     if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + p2);
                     else if (!v2) p2 = p1;
-                    const double2 st1 = a.soa.ld(0, p1), sx1 = a.soa.ld(1, p1);
-                    const double2 sy1 = a.soa.ld(2, p1), sz1 = a.soa.ld(3, p1);
-                    const double2 st2 = a.soa.ld(0, p2), sx2 = a.soa.ld(1, p2);
-                    const double2 sy2 = a.soa.ld(2, p2), sz2 = a.soa.ld(3, p2);
+                    double2 st1, sx1, sy1, sz1, st2, sx2, sy2, sz2;
+                    a.soa.load4(p1, st1, sx1, sy1, sz1);
+                    a.soa.load4(p2, st2, sx2, sy2, sz2);
                     double h0, h1;
                     const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
                     const bool x2 = a.excl && __ldg(a.etraj + p2) == S.qtraj[qi2];
