@@ -869,9 +869,13 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     blk = static_cast<char*>(cache_alloc(bytes_soa + bytes_bins + 256));
     idx->block = blk;
     idx->soa.rec = reinterpret_cast<double2*>(blk);
-    static const bool aos = [] {              // DTS_LAYOUT=rec: 64-byte records
-        const char* e = getenv("DTS_LAYOUT");   // measured on C4: records cost
-        return e && e[0] == 'r';                // +0.08 ms gather, +0.02 ms search
+    // 64-byte records read and written as two 256-bit accesses (DTS_LAYOUT=
+    // soa: four 16-byte streams).  Measured on C4: records 0.759 ms gather,
+    // 0.742 ms pass 1; streams 0.765, 0.802 (with 128-bit accesses the
+    // records lost: 0.852 / 0.838 against 0.775 / 0.814)
+    static const bool aos = [] {
+        const char* e = getenv("DTS_LAYOUT");
+        return !(e && e[0] == 's');
     }();
     idx->soa.ss = aos ? 1 : n;
     idx->soa.es = aos ? 4u : 1u;
