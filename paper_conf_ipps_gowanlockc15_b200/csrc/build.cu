@@ -245,6 +245,7 @@ __device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long l
                                             uint32_t e) {
     const unsigned long long bmask = ht.mask >> 2;
     unsigned long long b = bucket_of(k >> 2, ht);
+    CellSlot* const slots = ht.cells();
     // try the slot matching the key's position in its group first: the (up
     // to) four x-adjacent cells sharing a home bucket then claim distinct
     // slots without colliding on the same CAS
@@ -253,7 +254,7 @@ __device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long l
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
             const int i = (first + j) & 3;
-            CellSlot& sl = ht.slots[4 * b + i];
+            CellSlot& sl = slots[4 * b + i];
             const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
             if (prev == EMPTY_KEY) {
                 sl.start = p;
@@ -265,17 +266,6 @@ __device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long l
     }
 }
 
-__global__ void __launch_bounds__(BT) k_insert(const SortedKeys keys,
-                                              size_t n, HashTable ht) {
-    size_t p = (size_t)blockIdx.x * BT + threadIdx.x;
-    if (p >= n) return;
-    unsigned long long k = keys.key(p);
-    if (p != 0 && keys.key(p - 1) == k) return;
-    // the cell's run ends at the next key change (most cells hold 1-3 entries)
-    size_t e = p + 1;
-    while (e < n && keys.key(e) == k) ++e;
-    insert_cell(ht, k, (uint32_t)p, (uint32_t)e);
-}
 
 
 // Tiled insert: the tile's keys (plus the one before) are staged in shared
@@ -310,60 +300,83 @@ __global__ void __launch_bounds__(BT) k_insert_tiled(const SortedKeys keys, size
     }
 }
 
-// ITEMS sorted positions per thread (strided by the grid so key loads stay
-// coalesced): the cell heads among them issue their first-choice CAS
-// together, so ITEMS atomics are in flight per thread instead of one; a head
-// that loses its first slot continues with insert_cell().
-template <int ITEMS>
-__global__ void __launch_bounds__(BT) k_insert_batched(const SortedKeys keys, size_t n,
-                                                      HashTable ht) {
-    const size_t stride = (size_t)gridDim.x * BT;
-    const size_t p0 = (size_t)blockIdx.x * BT + threadIdx.x;
-    unsigned long long k[ITEMS];
-    uint32_t e[ITEMS];
-    bool head[ITEMS];
+// Block slots (kind 1): the head of each block of 8 keys (the first sorted
+// entry with that key >> 3) walks the block's entries -- keys ascend, so the
+// offsets key & 7 come in order -- builds the 8 inclusive prefix counts and
+// claims one 32-byte slot.  One CAS per block instead of one per cell.
+__device__ __forceinline__ void insert_block(const HashTable& ht, unsigned long long blk,
+                                             uint32_t start, uint32_t big,
+                                             unsigned long long c_lo, unsigned long long c_hi) {
+    const unsigned long long bmask = ht.mask >> 1;
+    unsigned long long b = bucket_of(blk, ht);
+    BlockSlot* const slots = ht.blocks();
+    while (true) {
 #pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        const size_t p = p0 + (size_t)i * stride;
-        head[i] = false;
-        k[i] = 0;
-        e[i] = 0;
-        if (p < n) {
-            k[i] = keys.key(p);
-            head[i] = p == 0 || keys.key(p - 1) != k[i];
+        for (int i = 0; i < 2; ++i) {
+            BlockSlot& sl = slots[2 * b + i];
+            if (atomicCAS(&sl.key, EMPTY_KEY, blk) == EMPTY_KEY) {
+                sl.start = start;
+                sl.big = big;
+                unsigned long long* c = reinterpret_cast<unsigned long long*>(sl.cum);
+                c[0] = c_lo;
+                c[1] = c_hi;
+                return;
+            }
         }
-    }
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        if (head[i]) {   // the cell's run ends at the next key change
-            size_t q = p0 + (size_t)i * stride + 1;
-            while (q < n && keys.key(q) == k[i]) ++q;
-            e[i] = (uint32_t)q;
-        }
-    }
-    unsigned long long prev[ITEMS];
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        prev[i] = 0;
-        if (head[i]) {
-            const unsigned long long b = bucket_of(k[i] >> 2, ht);
-            prev[i] = atomicCAS(&ht.slots[4 * b + (k[i] & 3ull)].key, EMPTY_KEY, k[i]);
-        }
-    }
-#pragma unroll
-    for (int i = 0; i < ITEMS; ++i) {
-        if (!head[i]) continue;
-        const uint32_t p = (uint32_t)(p0 + (size_t)i * stride);
-        if (prev[i] == EMPTY_KEY) {
-            const unsigned long long b = bucket_of(k[i] >> 2, ht);
-            CellSlot& sl = ht.slots[4 * b + (k[i] & 3ull)];
-            sl.start = p;
-            sl.end = e[i];
-        } else {
-            insert_cell(ht, k[i], p, e[i]);
-        }
+        b = (b + 1) & bmask;
     }
 }
+
+template <int ITEMS>
+__global__ void __launch_bounds__(BT) k_insert_blocks(const SortedKeys keys, size_t n,
+                                                     HashTable ht) {
+    constexpr int TILE = BT * ITEMS;
+    __shared__ unsigned long long s_key[TILE + 1];
+    const size_t p0 = (size_t)blockIdx.x * TILE;
+    const uint32_t tn = (uint32_t)min((size_t)TILE, n - p0);
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc < tn) s_key[1 + loc] = keys.key(p0 + loc);
+    }
+    if (threadIdx.x == 0) s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
+    __syncthreads();
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc >= tn) continue;
+        const unsigned long long blk = s_key[1 + loc] >> 3;
+        if (p0 + loc != 0 && (s_key[loc] >> 3) == blk) continue;
+        // inclusive prefix counts per key offset, packed 4 x u16 per word
+        unsigned long long c_lo = 0, c_hi = 0;
+        uint32_t cnt = 0, j = 0;             // entries so far; next offset to fill
+        auto fill_to = [&](uint32_t jo) {    // offsets j .. jo-1 get the count so far
+            for (; j < jo; ++j) {
+                const unsigned long long v = (unsigned long long)min(cnt, 65535u);
+                if (j < 4) c_lo |= v << (16 * j);
+                else c_hi |= v << (16 * (j - 4));
+            }
+        };
+        size_t q = p0 + loc;
+        uint32_t e = loc;
+        while (true) {
+            unsigned long long kq;
+            if (e < tn) kq = s_key[1 + e];
+            else if (q < n) kq = keys.key(q);
+            else break;
+            if ((kq >> 3) != blk) break;
+            fill_to((uint32_t)(kq & 7ull));
+            ++cnt;
+            ++e;
+            ++q;
+        }
+        fill_to(8);
+        const uint32_t big = cnt > 65535u ? 1u : 0u;
+        if (big) c_lo = cnt;                  // the block as one run [start, start + cnt)
+        insert_block(ht, blk, (uint32_t)(p0 + loc), big, c_lo, c_hi);
+    }
+}
+
 
 __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
@@ -386,7 +399,7 @@ __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
 // inputs, same arithmetic).
 struct GatherSmem {
     unsigned long long s_o0[BT / 32], s_o1[BT / 32];
-    uint32_t s_cnt;
+    uint32_t s_cnt, s_blk;
 };
 
 // The tile's records are in registers (r0, r1 for rows id) and its keys in
@@ -426,13 +439,14 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
     __syncthreads();
     const int32_t bfirst = s_bin[1];
     bool one_bin = true;
-    uint32_t cells = 0;
+    uint32_t cells = 0, blks = 0;
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
         const int loc = k * BT + threadIdx.x;
         const size_t p = p0 + (size_t)loc;
         if (p < n) {
             cells += (p == 0 || s_key[loc] != s_key[loc + 1]) ? 1u : 0u;
+            blks += (p == 0 || (s_key[loc] >> 3) != (s_key[loc + 1] >> 3)) ? 1u : 0u;
             const int32_t bp = s_bin[loc], b = s_bin[loc + 1];
             for (int32_t bb = bp + 1; bb <= b; ++bb) bin_start[bb] = (uint32_t)p;
             if (p == n - 1)
@@ -442,7 +456,9 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
     }
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     cells = __reduce_add_sync(0xffffffffu, cells);
+    blks = __reduce_add_sync(0xffffffffu, blks);
     if (lane == 0 && cells) atomicAdd(&sm.s_cnt, cells);
+    if (lane == 0 && blks) atomicAdd(&sm.s_blk, blks);
     if (__syncthreads_and(one_bin)) {
 #pragma unroll
         for (int off = 16; off; off >>= 1) {
@@ -474,9 +490,11 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
         }
     }
     __syncthreads();
-    if (threadIdx.x == 0 && sm.s_cnt) {
+    if (threadIdx.x == 0 && sm.s_cnt) {         // count[0]: cells, count[1]: blocks of 8 keys
         atomicAdd(count, (unsigned long long)sm.s_cnt);
+        atomicAdd(count + 1, (unsigned long long)sm.s_blk);
         sm.s_cnt = 0;
+        sm.s_blk = 0;
     }
 }
 
@@ -506,6 +524,7 @@ __global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restric
     }
     if (threadIdx.x == 0) {
         sm.s_cnt = 0;
+        sm.s_blk = 0;
         if (p0 > 0) {                                  // halo: sorted position p0 - 1
             // keys are bin-major (key = bin * cells_per_bin + cell), so the
             // halo's bin needs no dependent load of its record
@@ -892,8 +911,8 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // 6. non-empty cells -> hash table of >= 2x as many slots (power of two)
     // (measured: inserting from the gather, with the cells counted first,
     //  costs 1.98 ms against 0.78 + 0.56 ms for gather + separate insert)
-    DevBuf<unsigned long long> ncell(1, s);
-    DTS_CUDA(cudaMemsetAsync(ncell.p, 0, sizeof(unsigned long long), s));
+    DevBuf<unsigned long long> ncell(2, s);       // cells, blocks of 8 keys
+    DTS_CUDA(cudaMemsetAsync(ncell.p, 0, 2 * sizeof(unsigned long long), s));
     // (a persistent variant that loads the next tile's keys while the
     //  current records are in flight measured 0.886 ms against 0.775 for one
     //  tile per CTA: fewer resident CTAs hide less of the row latency)
@@ -903,38 +922,37 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
     mark();
-    unsigned long long hc = 0;
-    DTS_CUDA(cudaMemcpyAsync(&hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
+    unsigned long long hc[2] = {0, 0};
+    DTS_CUDA(cudaMemcpyAsync(hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
-    idx->n_cells = hc;
-    int log2cap = 6;
-    static const double hload = [] {          // DTS_HASH_SLOTS: slots per cell (>= 1.1)
-        const char* e = getenv("DTS_HASH_SLOTS");
-        return e ? std::max(1.1, atof(e)) : 2.0;
+    idx->n_cells = hc[0];
+    // 6. the non-empty cells -> bucketed hash table.  Kind 1 (default): one
+    //    32-byte slot per block of 8 keys (prefix counts per cell), >= 3.3
+    //    slots per block; kind 0 (DTS_HASH_KIND=0): one 16-byte slot per
+    //    cell, >= 2 slots per cell.
+    static const int hkind = [] {
+        const char* e = getenv("DTS_HASH_KIND");
+        return (e && e[0] == '0') ? 0 : 1;
     }();
-    while ((double)(1ull << log2cap) < hload * (double)hc) ++log2cap;
+    static const double hload = [] {          // DTS_HASH_SLOTS: slots per item
+        const char* e = getenv("DTS_HASH_SLOTS");
+        return e ? std::max(1.1, atof(e)) : 0.0;
+    }();
+    const double per = hload > 0.0 ? hload : (hkind ? 3.3 : 2.0);
+    const double items = (double)(hkind ? hc[1] : hc[0]);
+    const size_t slot_bytes = hkind ? sizeof(BlockSlot) : sizeof(CellSlot);
+    int log2cap = 6;
+    while ((double)(1ull << log2cap) < per * items) ++log2cap;
+    idx->ht.kind = hkind;
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
-    static const int hblk = [] {              // DTS_HASH_BLOCK: log2 buckets per block
-        const char* e = getenv("DTS_HASH_BLOCK");
-        return e ? std::max(0, std::min(8, atoi(e))) : 0;
-    }();
-    idx->ht.blk = std::min(hblk, log2cap - 4);
-    idx->ht.slots = static_cast<CellSlot*>(cache_alloc(sizeof(CellSlot) << log2cap));
-    DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(CellSlot) << log2cap, s));
-    // (measured on C4, incl. the memset: tiled 0.550 ms, 1 cell per thread
-    //  with global key scans 0.565; batching the first CAS of 2 / 4 / 8
-    //  cells: 0.59 / 0.70 / 0.91 ms)
-    static const int ins = [] {               // DTS_INSERT_ITEMS: 0 tiled (k_insert_tiled),
-        const char* e = getenv("DTS_INSERT_ITEMS");   // 1 (k_insert), 2, 4, 8 batched
-        const int v = e ? atoi(e) : 0;
-        return (v == 0 || v == 2 || v == 4 || v == 8) ? v : 1;
-    }();
-    if (ins == 0) k_insert_tiled<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
-    else if (ins == 1) k_insert<<<grid_for(n), BT, 0, s>>>(sk, n, idx->ht);
-    else if (ins == 2) k_insert_batched<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(sk, n, idx->ht);
-    else if (ins == 4) k_insert_batched<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
-    else k_insert_batched<8><<<grid_for((n + 7) / 8), BT, 0, s>>>(sk, n, idx->ht);
+    idx->ht.slots = cache_alloc(slot_bytes << log2cap);
+    DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, slot_bytes << log2cap, s));
+    // (measured on C4 for cell slots, incl. the memset: tiled 0.550 ms; one
+    //  thread per entry with global key scans 0.565; batching the first CAS
+    //  of 2 / 4 / 8 cells 0.59 / 0.70 / 0.91 ms)
+    if (hkind) k_insert_blocks<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    else k_insert_tiled<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
     DTS_LAUNCH_CHECK();
     mark();
 

@@ -106,6 +106,20 @@ struct __align__(16) CellSlot {
 };
 static constexpr unsigned long long EMPTY_KEY = ~0ull;
 
+// Hash slot of one non-empty BLOCK of 8 consecutive keys (key >> 3): 8
+// x-adjacent cells of a row (a block may straddle two rows).  The block's
+// entries are the sorted positions [start, start + cum[7]); those of key
+// offset j are [start + cum[j-1], start + cum[j]) (cum[-1] = 0).  When the
+// block holds more than 65535 entries, big = 1, cum is unused and the block
+// is one run [start, end) with end = start + cum32 (exact superset: the
+// refinement filters).  32 bytes, one 256-bit load; two per 64-byte bucket.
+struct __align__(32) BlockSlot {
+    unsigned long long key;
+    uint32_t start;
+    uint32_t big;
+    uint16_t cum[8];
+};
+
 // Grid parameters (passed by value to kernels).
 struct GridParams {
     double tmin;        // temporal origin  (t_min of P:L76)
@@ -122,10 +136,13 @@ struct GridParams {
 };
 
 struct HashTable {
-    CellSlot* slots;
-    unsigned long long mask;   // capacity - 1 (power of two)
-    int log2cap;
-    int blk;                   // log2 of the buckets of a block (bucket_of)
+    void* slots;               // CellSlot (kind 0) or BlockSlot (kind 1)
+    unsigned long long mask;   // slots - 1 (power of two)
+    int log2cap;               // log2 of the slots
+    int kind;                  // 0: cells, 4 slots per bucket; 1: blocks, 2 per bucket
+    __host__ __device__ int log2bucket() const { return kind ? 1 : 2; }
+    __host__ __device__ CellSlot* cells() const { return static_cast<CellSlot*>(slots); }
+    __host__ __device__ BlockSlot* blocks() const { return static_cast<BlockSlot*>(slots); }
 };
 
 // GPUSpatioTemporal subbins (P:L86-P:L92): per dimension a, v[a] subbins of
@@ -149,20 +166,17 @@ __device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double
 }
 
 // ---------------------------------------------------------------- device helpers
-// Bucketed open addressing: a bucket is 4 slots (64 bytes, one line pair).
-// Keys are row-major with x fastest, so the four keys sharing k >> 2
-// (x-adjacent cells of one row) have the same home bucket: a stencil row of
-// three cells reads one or two buckets instead of three random slots.  A key
-// sits in the first bucket, from its home on, that had a free slot when it
-// was inserted (no deletions), so a lookup stops at the first bucket holding
-// the key or a free slot -- almost always the home bucket.
-// With blk > 0, 2^blk consecutive groups keep consecutive home buckets (one
-// block of 2^blk x 64 bytes) and only the block is placed by the hash: the
-// build's inserts, in key order, then touch each block's lines together.
+// Bucketed open addressing, 64-byte buckets.  Keys are row-major with x
+// fastest, so x-adjacent cells share a group: kind 0 hashes groups of 4 keys
+// (k >> 2) into buckets of four 16-byte cell slots; kind 1 hashes blocks of
+// 8 keys (k >> 3, one 32-byte slot per block) into buckets of two.  A stencil
+// row of three cells then reads one or two buckets.  An item sits in the
+// first bucket, from its home on, that had a free slot when it was inserted
+// (no deletions), so a lookup stops at the first bucket holding it or a
+// free slot -- almost always the home bucket.
 __device__ __forceinline__ unsigned long long bucket_of(unsigned long long group,
                                                         const HashTable& ht) {
-    const unsigned long long hi = group >> ht.blk, lo = group & ((1ull << ht.blk) - 1ull);
-    return (((hi * 0x9E3779B97F4A7C15ull) >> (64 - (ht.log2cap - 2 - ht.blk))) << ht.blk) | lo;
+    return (group * 0x9E3779B97F4A7C15ull) >> (64 - (ht.log2cap - ht.log2bucket()));
 }
 
 __device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {

@@ -278,9 +278,55 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
         return;
     const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
     const unsigned long long kend = key0 + (unsigned long long)cn[0];   // row keys [key0, kend)
+    uint32_t first = 0xffffffffu, last = 0;
+    if (ht.kind == 1) {
+        // blocks of 8 keys: the row's keys [key0, kend) lie in blocks
+        // key0 >> 3 .. (kend - 1) >> 3, each one 32-byte slot holding the
+        // prefix counts of its 8 cells; a bucket is two slots (64 bytes)
+        const BlockSlot* slots = ht.blocks();
+        const unsigned long long bmask = ht.mask >> 1;
+        for (unsigned long long blk = key0 >> 3; blk <= (kend - 1) >> 3; ++blk) {
+            unsigned long long b = bucket_of(blk, ht);
+            ++probes;
+            while (true) {
+                const ulonglong4 h0 = ld256u(slots + 2 * b), h1 = ld256u(slots + 2 * b + 1);
+                const bool m0 = h0.x == blk, m1 = h1.x == blk;
+                if (m0 || m1) {
+                    const ulonglong4 h = m0 ? h0 : h1;
+                    const uint32_t start = (uint32_t)h.y, big = (uint32_t)(h.y >> 32);
+                    const unsigned long long base = blk << 3;
+                    const uint32_t lo = (uint32_t)((key0 > base ? key0 : base) - base);
+                    const uint32_t hi = (uint32_t)(((kend - 1) < base + 7 ? (kend - 1) : base + 7) - base);
+                    uint32_t s0, s1;
+                    if (big) {                       // the whole block (superset)
+                        s0 = start;
+                        s1 = start + (uint32_t)h.z;
+                    } else {                         // cum[j]: 16 bits at word z (j < 4) or w
+                        const uint32_t c_lo = lo == 0 ? 0u
+                            : (uint32_t)(((lo - 1) < 4 ? h.z >> (16 * (lo - 1)) : h.w >> (16 * (lo - 5))) & 0xffffull);
+                        const uint32_t c_hi =
+                            (uint32_t)((hi < 4 ? h.z >> (16 * hi) : h.w >> (16 * (hi - 4))) & 0xffffull);
+                        s0 = start + c_lo;
+                        s1 = start + c_hi;
+                    }
+                    if (s1 > s0) {
+                        first = min(first, s0);
+                        last = max(last, s1);
+                    }
+                    break;
+                }
+                if (h0.x == EMPTY_KEY || h1.x == EMPTY_KEY) break;   // end of the chain
+                b = (b + 1) & bmask;
+            }
+        }
+        if (first != 0xffffffffu) {
+            start = first;
+            cnt = last - first;
+        }
+        return;
+    }
     const ulonglong2* slots = reinterpret_cast<const ulonglong2*>(ht.slots);
     const unsigned long long bmask = ht.mask >> 2;
-    uint32_t first = 0xffffffffu, last = 0;
     // any slot whose key lies in the row range contributes (a key met on
     // another group's chain is found twice; min/max make that harmless);
     // returns whether the bucket has a free slot (end of the chain)
@@ -650,16 +696,13 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             const int v = e ? atoi(e) : 7;
             return (v == 5 || v == 6 || v == 8) ? v : 7;
         }();
-        static const bool pf = [] {        // DTS_PREFETCH=1: L2 prefetch of the next
-            const char* e = getenv("DTS_PREFETCH");   // round's buckets (measured slower
-            return e && e[0] == '1';                 // on C4: 0.85 vs 0.81 ms)
-        }();
+        // (an L2 prefetch of the next round's buckets measured slower on C4:
+        //  0.85 vs 0.81 ms, and was removed)
         const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
-        if (pf) k_wtile_count<7, true><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 8) k_wtile_count<8, false><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 7) k_wtile_count<7, false><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 5) k_wtile_count<5, false><<<grid, WT, 0, s>>>(ta);
-        else k_wtile_count<6, false><<<grid, WT, 0, s>>>(ta);
+        if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
+        else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);
+        else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);
         DTS_LAUNCH_CHECK();
     }
     tm.mark();

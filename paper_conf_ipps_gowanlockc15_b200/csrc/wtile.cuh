@@ -83,32 +83,8 @@ __device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, doubl
     }
 }
 
-// L2 prefetch of the home bucket(s) of probe l of the tile (issued one round
-// ahead, so that the next round's bucket loads do not wait on DRAM).
-__device__ __forceinline__ void prefetch_probe(const WarpSmem& S, const GridParams& g,
-                                               const HashTable& ht, unsigned long long l) {
-    int qi = 0;
-#pragma unroll
-    for (int step = WQ / 2; step; step >>= 1)
-        if (S.lkoff[qi + step] <= l) qi += step;
-    if (S.mode[qi] != MODE_GRID) return;
-    const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
-    const uint32_t cn1 = (uint32_t)S.cn[1][qi];
-    const uint32_t nzy = cn1 * (uint32_t)S.cn[2][qi];
-    const int32_t bin = S.lb[qi] + (int32_t)(loc / nzy);
-    const uint32_t r = loc % nzy;
-    const unsigned long long key0 = make_key(g, bin, S.clo[0][qi], S.clo[1][qi] + (int32_t)(r % cn1),
-                                             S.clo[2][qi] + (int32_t)(r / cn1));
-    const unsigned long long g0 = key0 >> 2, g1 = (key0 + (unsigned long long)S.cn[0][qi] - 1) >> 2;
-    const CellSlot* b0 = ht.slots + 4 * bucket_of(g0, ht);
-    asm volatile("prefetch.global.L2 [%0];" ::"l"(b0));
-    if (g1 != g0) {
-        const CellSlot* b1 = ht.slots + 4 * bucket_of(g1, ht);
-        asm volatile("prefetch.global.L2 [%0];" ::"l"(b1));
-    }
-}
 
-template <int MINB, bool PF>
+template <int MINB>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -173,7 +149,6 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             const unsigned long long l = r0 + lane;
             uint32_t start = 0, cnt = 0, ind = 0;
             int qi = 0;
-            if (PF && l + 32 < Ltot) prefetch_probe(S, g, a.ht, l + 32);
             if (l < Ltot) {
 #pragma unroll
                 for (int step = WQ / 2; step; step >>= 1)

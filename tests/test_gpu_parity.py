@@ -103,13 +103,15 @@ def test_index_parameter_invariance_and_determinism(dts, oracle_mod):
         idx.free()
 
 
-def test_radix_digit_plans_and_hash_blocks_invariant(dts, oracle_mod, monkeypatch):
+def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     """Same result bytes whatever digit plan the build's radix sort takes
-    (8-bit only, or 9-bit digits where they save a pass) and whatever block
-    placement the cell hash uses: both only change the index layout."""
+    (8-bit only, or 9-bit digits where they save a pass), whichever hash
+    (cell slots or 8-key block slots) and record layout (64-byte records or
+    four 16-byte streams) the index uses: they only change the layout."""
     c = synth.make_config("C1", scale=0.1)
     ref = None
-    for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_BLOCK": "4"}):
+    for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_KIND": "0"},
+                {"DTS_HASH_KIND": "1"}, {"DTS_LAYOUT": "soa"}, {"DTS_FUSED_KEYS": "0"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
         import sys
