@@ -238,6 +238,10 @@ typedef struct {
                                    one fused read of D for exact bounds, keys
                                    and sort histograms (phase "bounds" is then
                                    the sample, "keys" the fused pass)        */
+    uint32_t hash_kind;         /* cell table: 0 one slot per cell, 1 one slot
+                                   per block of 8 consecutive cell keys      */
+    uint64_t hash_items;        /* slots in use (cells or blocks)            */
+    uint64_t hash_bytes;        /* table size in bytes                       */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

@@ -80,7 +80,8 @@ class IndexInfo(ctypes.Structure):
                 ("max_duration", ctypes.c_double), ("ms_build", ctypes.c_float),
                 ("method", ctypes.c_uint32), ("subbins", ctypes.c_uint32 * 3),
                 ("subbin_ids", ctypes.c_uint64 * 3), ("ms_phase", ctypes.c_float * 5),
-                ("build_flags", ctypes.c_uint32)]
+                ("build_flags", ctypes.c_uint32), ("hash_kind", ctypes.c_uint32),
+                ("hash_items", ctypes.c_uint64), ("hash_bytes", ctypes.c_uint64)]
 
     def as_dict(self):
         out = {}

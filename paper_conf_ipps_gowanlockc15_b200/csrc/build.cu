@@ -330,6 +330,11 @@ __device__ __forceinline__ void insert_block(const HashTable& ht, unsigned long 
 template <int ITEMS>
 __global__ void __launch_bounds__(BT) k_insert_blocks(const SortedKeys keys, size_t n,
                                                      HashTable ht) {
+    // warp w owns the tile positions [w * 32 * ITEMS, (w + 1) * 32 * ITEMS)
+    // in chunks of 32; the block heads of a chunk are processed one after
+    // the other by the whole warp, 32 entries of the block per step, the
+    // eight prefix counts taken with ballots (no lane walks a long block
+    // alone); then every head lane claims its slot
     constexpr int TILE = BT * ITEMS;
     __shared__ unsigned long long s_key[TILE + 1];
     const size_t p0 = (size_t)blockIdx.x * TILE;
@@ -341,39 +346,53 @@ __global__ void __launch_bounds__(BT) k_insert_blocks(const SortedKeys keys, siz
     }
     if (threadIdx.x == 0) s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
     __syncthreads();
-#pragma unroll
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    auto key_at = [&](uint32_t q) -> unsigned long long {   // tile position q (may be >= tn)
+        if (q < tn) return s_key[1 + q];
+        const size_t p = p0 + q;
+        return p < n ? keys.key(p) : ~0ull;
+    };
+#pragma unroll 1
     for (int k = 0; k < ITEMS; ++k) {
-        const uint32_t loc = k * BT + threadIdx.x;
-        if (loc >= tn) continue;
-        const unsigned long long blk = s_key[1 + loc] >> 3;
-        if (p0 + loc != 0 && (s_key[loc] >> 3) == blk) continue;
-        // inclusive prefix counts per key offset, packed 4 x u16 per word
-        unsigned long long c_lo = 0, c_hi = 0;
-        uint32_t cnt = 0, j = 0;             // entries so far; next offset to fill
-        auto fill_to = [&](uint32_t jo) {    // offsets j .. jo-1 get the count so far
-            for (; j < jo; ++j) {
-                const unsigned long long v = (unsigned long long)min(cnt, 65535u);
-                if (j < 4) c_lo |= v << (16 * j);
-                else c_hi |= v << (16 * (j - 4));
-            }
-        };
-        size_t q = p0 + loc;
-        uint32_t e = loc;
-        while (true) {
-            unsigned long long kq;
-            if (e < tn) kq = s_key[1 + e];
-            else if (q < n) kq = keys.key(q);
-            else break;
-            if ((kq >> 3) != blk) break;
-            fill_to((uint32_t)(kq & 7ull));
-            ++cnt;
-            ++e;
-            ++q;
+        const uint32_t cbase = (uint32_t)(warp * 32 * ITEMS + k * 32);
+        const uint32_t loc = cbase + lane;
+        bool head = false;
+        unsigned long long blk = 0;
+        if (loc < tn) {
+            blk = s_key[1 + loc] >> 3;
+            head = p0 + loc == 0 || (s_key[loc] >> 3) != blk;
         }
-        fill_to(8);
-        const uint32_t big = cnt > 65535u ? 1u : 0u;
-        if (big) c_lo = cnt;                  // the block as one run [start, start + cnt)
-        insert_block(ht, blk, (uint32_t)(p0 + loc), big, c_lo, c_hi);
+        uint32_t heads = __ballot_sync(0xffffffffu, head);
+        unsigned long long my_lo = 0, my_hi = 0;
+        uint32_t my_big = 0;
+        while (heads) {
+            const int h = __ffs(heads) - 1;
+            heads &= heads - 1;
+            const uint32_t hp = cbase + h;
+            const unsigned long long hb = __shfl_sync(0xffffffffu, blk, h);
+            uint32_t cum[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+            for (uint32_t q = hp;; q += 32) {
+                const unsigned long long kq = key_at(q + lane);
+                const bool in = (kq >> 3) == hb;
+                const uint32_t off = (uint32_t)(kq & 7ull);
+#pragma unroll
+                for (int j = 0; j < 8; ++j) cum[j] += __popc(__ballot_sync(0xffffffffu, in && off <= (uint32_t)j));
+                if (__ballot_sync(0xffffffffu, in) != 0xffffffffu) break;
+            }
+            if (lane == h) {
+                if (cum[7] > 65535u) {            // the block as one run [start, start + cum[7])
+                    my_big = 1;
+                    my_lo = cum[7];
+                } else {
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        my_lo |= (unsigned long long)cum[j] << (16 * j);
+                        my_hi |= (unsigned long long)cum[4 + j] << (16 * j);
+                    }
+                }
+            }
+        }
+        if (head) insert_block(ht, blk, (uint32_t)(p0 + loc), my_big, my_lo, my_hi);
     }
 }
 
@@ -944,6 +963,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     int log2cap = 6;
     while ((double)(1ull << log2cap) < per * items) ++log2cap;
     idx->ht.kind = hkind;
+    idx->hash_items = hkind ? hc[1] : hc[0];
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
     idx->ht.slots = cache_alloc(slot_bytes << log2cap);

@@ -326,6 +326,7 @@ struct dts_index {
     float ms_build = 0.f;
     float ms_phase[5] = {0, 0, 0, 0, 0};   // bounds, keys, sort, gather, insert
     bool fused_keys = false;       // sampled grid + one-read bounds/keys/histograms
+    unsigned long long hash_items = 0;
     cudaEvent_t ev[7] = {};        // build phase events (index_times)
     int nev = 0;
     bool timed = false;
