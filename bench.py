@@ -305,7 +305,7 @@ def run_own(args):
          + ("" if inf.get("build_flags", 0) & 1 else " + 8 B/key histogram read")),
         ("k_gather_cells", ph[3], n * (8 + 64 + 68),
          "8 B sorted key + 64 B record read + 68 B record/id write per entry"),
-        ("k_insert_blocks" if inf.get("hash_kind", 0) == 1 else "k_insert_tiled", ph[4],
+        ("k_insert_blocks_lane" if inf.get("hash_kind", 0) == 1 else "k_insert_tiled", ph[4],
          n * 8 + inf.get("hash_items", ncells) * (32 if inf.get("hash_kind", 0) == 1 else 16),
          "8 B key per entry + one slot per hash item (32 B per 8-key block, or 16 B per cell); "
          "phase includes the table memset"),

@@ -396,6 +396,99 @@ __global__ void __launch_bounds__(BT) k_insert_blocks(const SortedKeys keys, siz
     }
 }
 
+// Block slots, lane-parallel: every block head walks its own block in the
+// staged keys (blocks average ~4 entries on C4), counting the 8 key offsets
+// as bytes of one u64 (c += 1 << 8 * (key & 7)); one multiply by
+// 0x0101010101010101 then gives the 8 inclusive prefix counts.  A block
+// longer than WALK entries is queued and done by a whole warp with ballots
+// (as k_insert_blocks), so no lane walks a long block alone.
+template <int ITEMS, int WALK>
+__global__ void __launch_bounds__(BT) k_insert_blocks_lane(const SortedKeys keys, size_t n,
+                                                          HashTable ht) {
+    static_assert(WALK < 256, "byte counters");
+    constexpr int TILE = BT * ITEMS;
+    __shared__ unsigned long long s_key[TILE + 1];
+    __shared__ uint32_t s_long[TILE];
+    __shared__ uint32_t s_nlong;
+    const size_t p0 = (size_t)blockIdx.x * TILE;
+    const uint32_t tn = (uint32_t)min((size_t)TILE, n - p0);
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc < tn) s_key[1 + loc] = keys.key(p0 + loc);
+    }
+    if (threadIdx.x == 0) {
+        s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
+        s_nlong = 0;
+    }
+    __syncthreads();
+    auto key_at = [&](uint32_t q) -> unsigned long long {   // tile position q (may be >= tn)
+        if (q < tn) return s_key[1 + q];
+        const size_t p = p0 + q;
+        return p < n ? keys.key(p) : ~0ull;
+    };
+#pragma unroll
+    for (int k = 0; k < ITEMS; ++k) {
+        const uint32_t loc = k * BT + threadIdx.x;
+        if (loc >= tn) continue;
+        const unsigned long long blk = s_key[1 + loc] >> 3;
+        if (p0 + loc != 0 && (s_key[loc] >> 3) == blk) continue;
+        unsigned long long c = 0;
+        uint32_t q = loc;
+        int steps = 0;
+        unsigned long long kq = s_key[1 + loc];
+        do {
+            c += 1ull << (8 * (uint32_t)(kq & 7ull));
+            ++q;
+            ++steps;
+            kq = key_at(q);
+        } while ((kq >> 3) == blk && steps < WALK);
+        if ((kq >> 3) == blk) {                 // longer than WALK: warp path below
+            s_long[atomicAdd(&s_nlong, 1u)] = loc;
+            continue;
+        }
+        const unsigned long long pre = c * 0x0101010101010101ull;   // byte j = cum[j]
+        unsigned long long lo = 0, hi = 0;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            lo |= ((pre >> (8 * j)) & 0xFFull) << (16 * j);
+            hi |= ((pre >> (8 * (4 + j))) & 0xFFull) << (16 * j);
+        }
+        insert_block(ht, blk, (uint32_t)(p0 + loc), 0u, lo, hi);
+    }
+    __syncthreads();
+    const uint32_t nl = s_nlong;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (uint32_t w = warp; w < nl; w += BT / 32) {
+        const uint32_t hp = s_long[w];
+        const unsigned long long hb = s_key[1 + hp] >> 3;
+        uint32_t cum[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        for (uint32_t q = hp;; q += 32) {
+            const unsigned long long kq = key_at(q + lane);
+            const bool in = (kq >> 3) == hb;
+            const uint32_t off = (uint32_t)(kq & 7ull);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) cum[j] += __popc(__ballot_sync(0xffffffffu, in && off <= (uint32_t)j));
+            if (__ballot_sync(0xffffffffu, in) != 0xffffffffu) break;
+        }
+        if (lane == 0) {
+            unsigned long long lo = 0, hi = 0;
+            uint32_t big = 0;
+            if (cum[7] > 65535u) {
+                big = 1;
+                lo = cum[7];
+            } else {
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    lo |= (unsigned long long)cum[j] << (16 * j);
+                    hi |= (unsigned long long)cum[4 + j] << (16 * j);
+                }
+            }
+            insert_block(ht, hb, (uint32_t)(p0 + hp), big, lo, hi);
+        }
+    }
+}
+
 
 __device__ __forceinline__ double velocity(double p0, double p1, double dur) {
     return dur > 0.0 ? (p1 - p0) / dur : 0.0;
@@ -971,7 +1064,13 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // (measured on C4 for cell slots, incl. the memset: tiled 0.550 ms; one
     //  thread per entry with global key scans 0.565; batching the first CAS
     //  of 2 / 4 / 8 cells 0.59 / 0.70 / 0.91 ms)
-    if (hkind) k_insert_blocks<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    static const int iwalk = [] {             // DTS_INSERT_WALK=0: warp-cooperative heads
+        const char* e = getenv("DTS_INSERT_WALK");
+        return e ? atoi(e) : 1;
+    }();
+    if (hkind && iwalk)
+        k_insert_blocks_lane<4, 32><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    else if (hkind) k_insert_blocks<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
     else k_insert_tiled<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
     DTS_LAUNCH_CHECK();
     mark();
