@@ -197,7 +197,8 @@ __device__ __forceinline__ unsigned long long packed_key(const GridParams& g, co
     return (make_key(g, bin, cx, cy, cz) << shift) | (unsigned long long)i;
 }
 
-__global__ void __launch_bounds__(BT, 3) k_bounds_keys(const double4* __restrict__ D, size_t n,
+template <int MINB>
+__global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restrict__ D, size_t n,
                                                       GridParams g,
                                                       unsigned long long* __restrict__ keys,
                                                       int shift, const PassPlan plan,
@@ -208,9 +209,11 @@ __global__ void __launch_bounds__(BT, 3) k_bounds_keys(const double4* __restrict
     __syncthreads();
     Bounds b;
     bounds_init(b);
-    auto count = [&](unsigned long long v) {
-        for (int p = 0; p < plan.npass; ++p)
-            atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
+    auto count = [&](unsigned long long v) {    // unrolled: the plan stays in registers
+#pragma unroll
+        for (int p = 0; p < OS_MAXPASS; ++p)
+            if (p < plan.npass)
+                atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
     };
     const size_t stride = (size_t)gridDim.x * BT;
     size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
@@ -610,8 +613,8 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
     }
 }
 
-template <int ITEMS>
-__global__ void __launch_bounds__(BT, 4) k_gather_cells(const double4* __restrict__ D, size_t n,
+template <int ITEMS, int MINB = 4>
+__global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __restrict__ D, size_t n,
                                                     const SortedKeys sk, SegSoA soa, GridParams g,
                                                     uint32_t* __restrict__ bin_start,
                                                     unsigned long long* __restrict__ bin_t0min,
@@ -676,6 +679,16 @@ __global__ void k_ordered_to_double(unsigned long long* __restrict__ a, size_t n
 
 
 inline unsigned grid_for(size_t n) { return (unsigned)((n + BT - 1) / BT); }
+
+// SMs x resident CTAs of BT threads for kernel f on the current device (one
+// full wave for a grid-stride kernel).
+int resident_grid(const void* f) {
+    int dev = 0, sms = 0, occ = 0;
+    DTS_CUDA(cudaGetDevice(&dev));
+    DTS_CUDA(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    DTS_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, f, BT, 0));
+    return std::max(1, sms * std::max(1, occ));
+}
 
 // ---------------------------------------------------------- subbins (ST)
 // Coordinate A of a segment's start (row 0) / end (row 1).
@@ -923,9 +936,20 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             const PassPlan plan = plan_passes(row_bits, row_bits + kb, true);
             DevBuf<uint32_t> hist((size_t)plan.npass * OS_HSTRIDE, s);
             DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)plan.npass * OS_HSTRIDE * 4, s));
-            k_bounds_keys<<<np, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p, hist.p);
+            // grid-stride over D with exactly one wave of resident CTAs
+            // (np = 1184 CTAs at 3 per SM left the last of 2.67 waves 2/3 full)
+            static const int bk_minb = [] {     // DTS_BK_OCC: CTAs per SM (3: 0.321 ms on C4; 4 spills: 0.355)
+                const char* e = getenv("DTS_BK_OCC");
+                return (e && e[0] == '4') ? 4 : 3;
+            }();
+            const int npk = (int)std::min<size_t>((size_t)resident_grid(
+                bk_minb == 3 ? (const void*)k_bounds_keys<3> : (const void*)k_bounds_keys<4>), np);
+            if (bk_minb == 3)
+                k_bounds_keys<3><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p, hist.p);
+            else
+                k_bounds_keys<4><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p, hist.p);
             DTS_LAUNCH_CHECK();
-            k_bounds_final<<<1, BT, 0, s>>>(partial.p, np, total.p);
+            k_bounds_final<<<1, BT, 0, s>>>(partial.p, npk, total.p);
             DTS_LAUNCH_CHECK();
             DTS_CUDA(cudaMemcpyAsync(hb_pinned, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
             cudaEvent_t eb;
@@ -1028,8 +1052,19 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // (a persistent variant that loads the next tile's keys while the
     //  current records are in flight measured 0.886 ms against 0.775 for one
     //  tile per CTA: fewer resident CTAs hide less of the row latency)
-    k_gather_cells<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(D, n, sk, idx->soa, g, idx->bin_start,
-                                                           b0, b1, ncell.p);
+    static const int gvar = [] {        // DTS_GATHER (C4): 1 (1 entry/thread, 6 CTAs/SM) 0.761 ms,
+        const char* e = getenv("DTS_GATHER");   // 2 (2, 4: default) 0.751, 4 (4, 2) 0.751
+        return e ? atoi(e) : 2;
+    }();
+    if (gvar == 1)
+        k_gather_cells<1, 6><<<grid_for(n), BT, 0, s>>>(D, n, sk, idx->soa, g, idx->bin_start,
+                                                        b0, b1, ncell.p);
+    else if (gvar == 4)
+        k_gather_cells<4, 2><<<grid_for((n + 3) / 4), BT, 0, s>>>(D, n, sk, idx->soa, g,
+                                                                  idx->bin_start, b0, b1, ncell.p);
+    else
+        k_gather_cells<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(D, n, sk, idx->soa, g,
+                                                               idx->bin_start, b0, b1, ncell.p);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
