@@ -333,13 +333,14 @@ __global__ void __launch_bounds__(RS_THREADS) k_rs_hist_scan(uint32_t* __restric
 // One pass over a digit of RB bits (8: 256 digits, one per thread; 9: 512,
 // two per thread -- a 34-bit key then takes 9+9+8+8 instead of five 8-bit
 // passes).
-template <bool VALS, int MINB, int RB, int LB = OS_LB>
+template <bool VALS, int MINB, int RB, int ITEMS = OS_ITEMS, int LB = OS_LB>
 __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ gbase, uint32_t* status, uint32_t* tile_ctr,
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out,
     uint32_t sleep_ns) {
     constexpr int RADIX = 1 << RB;
+    constexpr int TILE = RS_THREADS * ITEMS;
     constexpr int DPT = RADIX / RS_THREADS;          // digits per thread
     static_assert(DPT == 1 || DPT == 2, "8- or 9-bit digits");
     constexpr uint32_t DMASK = RADIX - 1;
@@ -349,21 +350,21 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     __shared__ uint32_t local_off[RADIX];
     __shared__ uint32_t warp_tot[RS_WARPS];
     __shared__ uint32_t s_tile;
-    __shared__ unsigned long long sk[OS_TILE];
-    __shared__ uint32_t sv[VALS ? OS_TILE : 1];
+    __shared__ unsigned long long sk[TILE];
+    __shared__ uint32_t sv[VALS ? TILE : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
     for (int j = lane; j < RADIX + 1; j += 32) wcnt[warp][j] = 0;
     __syncthreads();
     const uint32_t tile = s_tile;
 
-    // ---- load and rank (warp w owns a contiguous chunk of 32 * OS_ITEMS keys)
-    const size_t wbase = (size_t)tile * OS_TILE + (size_t)warp * (32 * OS_ITEMS);
-    unsigned long long k[OS_ITEMS];
-    uint32_t v[VALS ? OS_ITEMS : 1];
-    uint32_t dr[OS_ITEMS];                       // digit | rank << RSH; digit RADIX: past the end
+    // ---- load and rank (warp w owns a contiguous chunk of 32 * ITEMS keys)
+    const size_t wbase = (size_t)tile * TILE + (size_t)warp * (32 * ITEMS);
+    unsigned long long k[ITEMS];
+    uint32_t v[VALS ? ITEMS : 1];
+    uint32_t dr[ITEMS];                       // digit | rank << RSH; digit RADIX: past the end
 #pragma unroll
-    for (int i = 0; i < OS_ITEMS; ++i) {
+    for (int i = 0; i < ITEMS; ++i) {
         const size_t idx = wbase + (size_t)i * 32 + lane;
         const bool ok = idx < n;
         k[i] = ok ? keys[idx] : 0ull;
@@ -372,7 +373,7 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     }
     const uint32_t lt_mask = (1u << lane) - 1u;
 #pragma unroll
-    for (int i = 0; i < OS_ITEMS; ++i) {
+    for (int i = 0; i < ITEMS; ++i) {
         const uint32_t dig = dr[i];
         uint32_t peers = __ballot_sync(0xffffffffu, dig < (uint32_t)RADIX);
 #pragma unroll
@@ -477,7 +478,7 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     __syncthreads();
     // ---- stage in digit order, write out coalesced
 #pragma unroll
-    for (int i = 0; i < OS_ITEMS; ++i) {
+    for (int i = 0; i < ITEMS; ++i) {
         const uint32_t dig = dr[i] & ((2u << RB) - 1u);
         if (dig < (uint32_t)RADIX) {
             const uint32_t lpos = local_off[dig] + wcnt[warp][dig] + (dr[i] >> RSH);
@@ -486,8 +487,8 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
         }
     }
     __syncthreads();
-    const size_t tbase = (size_t)tile * OS_TILE;
-    const uint32_t tn = (uint32_t)min((size_t)OS_TILE, n - tbase);
+    const size_t tbase = (size_t)tile * TILE;
+    const uint32_t tn = (uint32_t)min((size_t)TILE, n - tbase);
     for (uint32_t i = threadIdx.x; i < tn; i += RS_THREADS) {
         const unsigned long long key = sk[i];
         const uint32_t dg = (uint32_t)(key >> shift) & DMASK;
@@ -534,13 +535,30 @@ PassPlan plan_passes(int lo, int hi, bool allow9) {
 }
 
 namespace {
-template <bool VALS, int MINB, int RB>
+template <bool VALS, int MINB, int RB, int ITEMS = OS_ITEMS>
 void launch_onesweep(uint32_t ntiles, cudaStream_t s, const unsigned long long* kin,
                      const uint32_t* vin, size_t n, int shift, const uint32_t* gbase,
                      uint32_t* status, uint32_t* ctr, unsigned long long* kout, uint32_t* vout,
                      uint32_t sleep_ns) {
-    k_onesweep<VALS, MINB, RB><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, gbase, status,
-                                                             ctr, kout, vout, sleep_ns);
+    k_onesweep<VALS, MINB, RB, ITEMS><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, gbase,
+                                                                    status, ctr, kout, vout,
+                                                                    sleep_ns);
+}
+
+// Keys-only tile shapes (DTS_OS_SHAPE, A/B): 0 = 12 keys per thread for
+// both digit widths (3072-key tiles); 1 (default) = 16 (8-bit, 3 CTAs/SM)
+// and 13 (9-bit); 2 = 16 (8-bit, 4 CTAs/SM, spills) and 13 (9-bit).
+// Measured on the C4 entry sort (9+9+8+8): 0.834, 0.817, 0.828 ms.
+int os_shape() {
+    static const int v = [] {
+        const char* e = getenv("DTS_OS_SHAPE");
+        return e ? atoi(e) : 1;
+    }();
+    return v;
+}
+int os_items(int bits, bool vals) {
+    if (vals || os_shape() == 0) return OS_ITEMS;
+    return bits == 9 ? 13 : 16;
 }
 
 // The plan's onesweep passes; hist holds each pass's exclusive digit bases
@@ -548,8 +566,12 @@ void launch_onesweep(uint32_t ntiles, cudaStream_t s, const unsigned long long* 
 void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32_t** vin,
                      uint32_t** vout, size_t n, const PassPlan& plan, const uint32_t* hist,
                      cudaStream_t s) {
-    const uint32_t ntiles = (uint32_t)((n + OS_TILE - 1) / OS_TILE);
-    const size_t nstat = (size_t)ntiles * OS_HSTRIDE + 32;
+    uint32_t maxtiles = 0;
+    for (int p = 0; p < plan.npass; ++p) {
+        const uint32_t tile = RS_THREADS * os_items(plan.bits[p], *vin != nullptr);
+        maxtiles = std::max(maxtiles, (uint32_t)((n + tile - 1) / tile));
+    }
+    const size_t nstat = (size_t)maxtiles * OS_HSTRIDE + 32;
     DevBuf<uint32_t> status(nstat, s);
     static const uint32_t sleep_ns = [] {   // DTS_OS_SLEEP: look-back back-off (ns)
         const char* e = getenv("DTS_OS_SLEEP");   // C4 entry sort, 5 passes: 0 ns
@@ -557,17 +579,28 @@ void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32
     }();                                          // 512: 0.957 (look-back window 8:
                                                   // 0.936, 16: 1.03, 32: 1.64)
     for (int p = 0; p < plan.npass; ++p) {
+        const uint32_t tile = RS_THREADS * os_items(plan.bits[p], *vin != nullptr);
+        const uint32_t ntiles = (uint32_t)((n + tile - 1) / tile);
+        const int shape = *vin ? 0 : os_shape();
         const size_t used = (size_t)ntiles << plan.bits[p];
         DTS_CUDA(cudaMemsetAsync(status.p, 0, (used + 32) * sizeof(uint32_t), s));
         uint32_t* ctr = status.p + used;
         const uint32_t* gb = hist + OS_HSTRIDE * p;
         const int sh = plan.shift[p];
         if (plan.bits[p] == 9) {
-            launch_onesweep<false, 3, 9>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
+            if (shape) launch_onesweep<false, 3, 9, 13>(ntiles, s, *kin, nullptr, n, sh, gb,
+                                                        status.p, ctr, *kout, nullptr, sleep_ns);
+            else launch_onesweep<false, 3, 9>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
                                               *kout, nullptr, sleep_ns);
         } else {
             if (*vin) launch_onesweep<true, 2, 8>(ntiles, s, *kin, *vin, n, sh, gb, status.p, ctr,
                                                   *kout, *vout, sleep_ns);
+            else if (shape == 1)
+                launch_onesweep<false, 3, 8, 16>(ntiles, s, *kin, nullptr, n, sh, gb, status.p,
+                                                 ctr, *kout, nullptr, sleep_ns);
+            else if (shape == 2)
+                launch_onesweep<false, 4, 8, 16>(ntiles, s, *kin, nullptr, n, sh, gb, status.p,
+                                                 ctr, *kout, nullptr, sleep_ns);
             else launch_onesweep<false, 4, 8>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
                                               *kout, nullptr, sleep_ns);
         }
