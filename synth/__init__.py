@@ -291,3 +291,38 @@ def adversarial(seed: int, n: int = 50, nq: int = 50):
             D[i, 0] = Q[j, 4]
             D[i, 4] = D[i, 0] + 0.5
     return np.ascontiguousarray(D), np.ascontiguousarray(Q)
+
+
+def crowded(seed: int, big: int = 70000, clusters: int = 120, per_cluster: int = 50,
+            background: int = 3000, nq: int = 12):
+    """Crowded grid cells: `big` short segments inside one tiny box (one
+    8-cell hash block holding more than 65,535 entries), `clusters` boxes of
+    `per_cluster` segments (blocks longer than a warp), and `background`
+    short random segments in [0,1]^3, all over times in [0, 1]; queries cross
+    the big box, the clusters and empty space."""
+    g = rng(seed)
+
+    def box(n, c, r):
+        s = np.empty((n, 8))
+        s[:, 0] = g.uniform(0.0, 0.4, n)
+        s[:, 4] = s[:, 0] + g.uniform(0.2, 0.6, n)
+        s[:, 1:4] = c + g.uniform(-r, r, (n, 3))
+        s[:, 5:8] = c + g.uniform(-r, r, (n, 3))
+        return s
+
+    parts = [box(big, np.array([0.5, 0.5, 0.5]), 1e-4)]
+    for c in g.uniform(0.05, 0.95, (clusters, 3)):
+        parts.append(box(per_cluster, c, 2e-4))
+    bg = box(background, np.zeros(3), 0.0)
+    bg[:, 1:4] = g.uniform(0.0, 1.0, (background, 3))
+    bg[:, 5:8] = bg[:, 1:4] + g.uniform(-0.01, 0.01, (background, 3))
+    parts.append(bg)
+    D = np.concatenate(parts)
+    D = D[g.permutation(D.shape[0])]
+    Q = np.empty((nq, 8))
+    Q[:, 0] = g.uniform(0.0, 0.3, nq)
+    Q[:, 4] = Q[:, 0] + 0.5
+    a = np.concatenate([np.full((nq // 3, 3), 0.5), g.uniform(0.05, 0.95, (nq - nq // 3, 3))])
+    Q[:, 1:4] = a - 0.003
+    Q[:, 5:8] = a + 0.003
+    return np.ascontiguousarray(D), np.ascontiguousarray(Q)

@@ -111,7 +111,9 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     c = synth.make_config("C1", scale=0.1)
     ref = None
     for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_KIND": "0"},
-                {"DTS_HASH_KIND": "1"}, {"DTS_LAYOUT": "soa"}, {"DTS_FUSED_KEYS": "0"}):
+                {"DTS_HASH_KIND": "1"}, {"DTS_LAYOUT": "soa"}, {"DTS_FUSED_KEYS": "0"},
+                {"DTS_INSERT_WALK": "0"}, {"DTS_OS_SHAPE": "0"}, {"DTS_GATHER": "4"},
+                {"DTS_GATHER": "1"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
         import sys
@@ -128,6 +130,28 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
             parity.compare(got, oracle_mod.search(c.D, c.Q, c.d, threads=THREADS), c.D, c.Q,
                            c.d, oracle_mod)
         assert out.stdout == ref, env
+
+
+def test_crowded_cells(dts, oracle_mod):
+    """Blocks of 8 cells holding more than a warp's worth of entries (the
+    insert's warp path) and more than 65,535 (one run per block): parity with
+    the oracle, and the same bytes with warp-path-only inserts and with cell
+    slots."""
+    import subprocess
+    import sys
+    D, Q = synth.crowded(5)
+    d = 0.01
+    got, info = run_and_compare(dts, oracle_mod, D, Q, d)
+    assert info["common"] > 200000
+    code = ("import sys; sys.path[:0] = [%r, %r]; import synth, "
+            "paper_conf_ipps_gowanlockc15_b200 as m; D, Q = synth.crowded(5); "
+            "i = m.build_index(D); r = m.search(i, Q, %r); "
+            "sys.stdout.buffer.write(r.tobytes())" % (REPO, os.path.join(REPO, "tests"), d))
+    for env in ({"DTS_INSERT_WALK": "0"}, {"DTS_HASH_KIND": "0"}):
+        out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
+                             capture_output=True, timeout=600)
+        assert out.returncode == 0, out.stderr.decode()[-2000:]
+        assert out.stdout == got.tobytes(), env
 
 
 def _unsampled_positions(n, k):
