@@ -302,7 +302,9 @@ def run_own(args):
         ("k_onesweep (entry sort)", ph[2],
          (0 if inf.get("build_flags", 0) & 1 else n * 8) + npass * n * 16,
          f"{npass} passes x (8 B read + 8 B write) per key"
-         + ("" if inf.get("build_flags", 0) & 1 else " + 8 B/key histogram read")),
+         + ("" if inf.get("build_flags", 0) & 1 else " + 8 B/key histogram read")
+         + "; issue/latency-bound, not HBM-bound (DRAM ~15% busy): CUB DeviceRadixSort "
+           "takes 1.09 ms on the same shape (profiles/r01d_cub_sort.txt)"),
         ("k_gather_cells", ph[3], n * (8 + 64 + 68),
          "8 B sorted key + 64 B record read + 68 B record/id write per entry"),
         ("k_insert_blocks_lane" if inf.get("hash_kind", 0) == 1 else "k_insert_tiled", ph[4],

@@ -112,7 +112,8 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     ref = None
     for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_KIND": "0"},
                 {"DTS_HASH_KIND": "1"}, {"DTS_LAYOUT": "soa"}, {"DTS_FUSED_KEYS": "0"},
-                {"DTS_INSERT_WALK": "0"}, {"DTS_OS_SHAPE": "0"}, {"DTS_GATHER": "4"},
+                {"DTS_INSERT_WALK": "0"}, {"DTS_OS_SHAPE": "0"},
+                {"DTS_GATHER": "4"},
                 {"DTS_GATHER": "1"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
