@@ -826,6 +826,20 @@ static void build_subbins(dts_index* idx, const double4* D, size_t n, const Boun
 }
 
 // Host-side choice of the temporal bins and spatial cells.
+// DTS_CELL_SCALE="sx,sy,sz": cell widths times these factors (A/B knob;
+// any width gives the same results, the stencil covers as many cells as
+// it needs).
+static double cell_scale(int a) {
+    static const std::vector<double> f = [] {
+        std::vector<double> v{1.0, 1.0, 1.0};
+        const char* e = getenv("DTS_CELL_SCALE");
+        if (e) sscanf(e, "%lf,%lf,%lf", &v[0], &v[1], &v[2]);
+        for (double& x : v) if (!(x > 0.0) || !std::isfinite(x)) x = 1.0;
+        return v;
+    }();
+    return f[a];
+}
+
 static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g) {
     const double span_t = b.tmax - b.tmin;
     g.tmin = b.tmin;
@@ -849,6 +863,7 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
         // temporal and subbin methods use one cell per bin: the sort key is the
         // bin, so entries are grouped by t_start bin as in P:L76
         if (p.method != DTS_METHOD_GRID) w = std::max(span, 1.0) * 2.0;
+        else w *= cell_scale(a);
         w = std::max(w, span / (MAXC - 1.0));
         w = std::max(w, 1e-12 * b.absmax);
         if (!(w > 0.0) || !std::isfinite(w)) w = 1.0;
