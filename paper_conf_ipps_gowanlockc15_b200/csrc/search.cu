@@ -699,7 +699,18 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         // (an L2 prefetch of the next round's buckets measured slower on C4:
         //  0.85 vs 0.81 ms, and was removed)
         const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
-        if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
+        // DTS_WTILE_TMA=32: candidate records staged by TMA bulk copies in
+        // chunks of 32 (record layout, grid and temporal methods)
+        static const int tma = [] {
+            const char* e = getenv("DTS_WTILE_TMA");
+            return e ? atoi(e) : 0;
+        }();
+        const bool tma_ok = idx->soa.es == 4 && idx->method != DTS_METHOD_SUBBIN;
+        if (tma_ok && tma == 32) {
+            const int o = occ >= 7 ? 6 : occ;
+            if (o == 6) k_wtile_count<6, true, 32><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(ta);
+            else k_wtile_count<5, true, 32><<<std::min<unsigned>(want, nsm * 5), WT, 0, s>>>(ta);
+        } else if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
         else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
         else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);
         else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);

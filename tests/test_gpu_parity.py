@@ -148,7 +148,7 @@ def test_crowded_cells(dts, oracle_mod):
             "paper_conf_ipps_gowanlockc15_b200 as m; D, Q = synth.crowded(5); "
             "i = m.build_index(D); r = m.search(i, Q, %r); "
             "sys.stdout.buffer.write(r.tobytes())" % (REPO, os.path.join(REPO, "tests"), d))
-    for env in ({"DTS_INSERT_WALK": "0"}, {"DTS_HASH_KIND": "0"}):
+    for env in ({"DTS_INSERT_WALK": "0"}, {"DTS_HASH_KIND": "0"}, {"DTS_WTILE_TMA": "32"}):
         out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
                              capture_output=True, timeout=600)
         assert out.returncode == 0, out.stderr.decode()[-2000:]
