@@ -21,11 +21,26 @@ constexpr int WH = 128;                 // staged hits per warp tile
 constexpr int WT = 128;                 // threads per CTA (4 independent warps)
 constexpr int WW = WT / 32;
 
+// Query record as read by the refinement: (t0,t1) (x0,vx) (y0,vy) (z0,vz)
+// in four 16-byte words (four LDS.128 per candidate instead of eight
+// LDS.64), padded to 80 bytes so that queries 2 apart do not share banks.
+constexpr int QREC = 5;
+
+// A query's stencil as read by a probe lane: 64 bytes, four LDS.128.
+struct __align__(16) QStencil {
+    int32_t lb, hb;
+    uint32_t mode, rind;
+    int32_t clo[3];
+    uint32_t rstart;                   // single-run queries (temporal / subbin)
+    int32_t cn[3];
+    uint32_t rcnt;
+};
+
 struct WarpSmem {
-    double qt0[WQ], qt1[WQ], qx0[WQ], qvx[WQ], qy0[WQ], qvy[WQ], qz0[WQ], qvz[WQ];
-    int32_t lb[WQ], hb[WQ], clo[3][WQ], cn[3][WQ];
-    uint32_t qid[WQ], mode[WQ], qcount[WQ], qoff[WQ];
-    uint32_t rstart[WQ], rcnt[WQ], rind[WQ];   // single-run queries (temporal / subbin)
+    double2 qrec[WQ][QREC];
+    double qt0[WQ], qt1[WQ];
+    QStencil qs[WQ];
+    uint32_t qid[WQ], qcount[WQ], qoff[WQ];
     uint32_t qtraj[WQ];                        // trajectory ids (exclude_same_trajectory)
     unsigned long long lkoff[WQ + 1];
     unsigned long long hkey[WH];        // (query << 42) | (position, then entry id << 10) | slot
@@ -61,10 +76,11 @@ struct TileArgs {
 
 __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
     QState q;
-    q.t0 = S.qt0[qi]; q.t1 = S.qt1[qi];
-    q.x0 = S.qx0[qi]; q.vx = S.qvx[qi];
-    q.y0 = S.qy0[qi]; q.vy = S.qvy[qi];
-    q.z0 = S.qz0[qi]; q.vz = S.qvz[qi];
+    const double2 a = S.qrec[qi][0], b = S.qrec[qi][1], c = S.qrec[qi][2], e = S.qrec[qi][3];
+    q.t0 = a.x; q.t1 = a.y;
+    q.x0 = b.x; q.vx = b.y;
+    q.y0 = c.x; q.vy = c.y;
+    q.z0 = e.x; q.vz = e.y;
     return q;
 }
 
@@ -168,17 +184,18 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             const Stencil st = make_stencil(g, q, qlo, qhi, d, live, a.bin_start, a.bin_t0min,
                                             a.bin_t1max, a.method, a.sb);
             S.qt0[lane] = q.t0; S.qt1[lane] = q.t1;
-            S.qx0[lane] = q.x0; S.qvx[lane] = q.vx;
-            S.qy0[lane] = q.y0; S.qvy[lane] = q.vy;
-            S.qz0[lane] = q.z0; S.qvz[lane] = q.vz;
-            S.lb[lane] = st.lb; S.hb[lane] = st.hb;
+            S.qrec[lane][0] = make_double2(q.t0, q.t1);
+            S.qrec[lane][1] = make_double2(q.x0, q.vx);
+            S.qrec[lane][2] = make_double2(q.y0, q.vy);
+            S.qrec[lane][3] = make_double2(q.z0, q.vz);
+            QStencil qs;
+            qs.lb = st.lb; qs.hb = st.hb;
+            qs.mode = st.mode; qs.rind = st.rind;
 #pragma unroll
-            for (int ax = 0; ax < 3; ++ax) { S.clo[ax][lane] = st.clo[ax]; S.cn[ax][lane] = st.cn[ax]; }
+            for (int ax = 0; ax < 3; ++ax) { qs.clo[ax] = st.clo[ax]; qs.cn[ax] = st.cn[ax]; }
+            qs.rstart = st.rstart; qs.rcnt = st.rcnt;
+            S.qs[lane] = qs;
             S.qid[lane] = qid;
-            S.mode[lane] = st.mode;
-            S.rstart[lane] = st.rstart;
-            S.rcnt[lane] = st.rcnt;
-            S.rind[lane] = st.rind;
             S.qtraj[lane] = (a.excl && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
             S.qcount[lane] = 0;
             nlook = st.nlook;
@@ -206,12 +223,11 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 for (int step = WQ / 2; step; step >>= 1)
                     if (S.lkoff[qi + step] <= l) qi += step;
                 const uint32_t loc = (uint32_t)(l - S.lkoff[qi]);
-                const int32_t clo[3] = {S.clo[0][qi], S.clo[1][qi], S.clo[2][qi]};
-                const int32_t cn[3] = {S.cn[0][qi], S.cn[1][qi], S.cn[2][qi]};
-                resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, S.mode[qi], S.lb[qi],
-                        S.hb[qi], clo, cn, S.qt0[qi], S.qt1[qi], loc, S.rstart[qi], S.rcnt[qi],
+                const QStencil qs = S.qs[qi];
+                resolve(g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, qs.mode, qs.lb,
+                        qs.hb, qs.clo, qs.cn, S.qt0[qi], S.qt1[qi], loc, qs.rstart, qs.rcnt,
                         start, cnt, n_probe);
-                ind = S.rind[qi];
+                ind = qs.rind;
             }
             unsigned long long incl = cnt;
 #pragma unroll
@@ -273,27 +289,42 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     }
                     __syncwarp();
                 }
-            } else
+            } else {
+            // per run: the position delta start - excl (mod 2^32: a candidate's
+            // position p = t + delta fits 32 bits even when the round's total
+            // does not) and (query | method index << 8), one 32-bit shuffle
+            // each; the run search shuffles 32-bit prefixes when the total fits
+            const uint32_t delta = start - (uint32_t)excl;
+            const uint32_t qind = (uint32_t)qi | (ind << 8);
+            const bool narrow = total <= 0xffffffffull;
+            const uint32_t incl32 = (uint32_t)incl;
             for (unsigned long long base = 0; base < total; base += 64) {
                 const unsigned long long t1 = base + lane, t2 = t1 + 32;
                 int j1 = 0, j2 = 0;
+                if (narrow) {
+                    const uint32_t u1 = (uint32_t)t1, u2 = (uint32_t)t2;
 #pragma unroll
-                for (int step = 16; step; step >>= 1) {
-                    if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
-                    if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
+                    for (int step = 16; step; step >>= 1) {
+                        if (__shfl_sync(0xffffffffu, incl32, j1 + step - 1) <= u1) j1 += step;
+                        if (__shfl_sync(0xffffffffu, incl32, j2 + step - 1) <= u2) j2 += step;
+                    }
+                } else {
+#pragma unroll
+                    for (int step = 16; step; step >>= 1) {
+                        if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
+                        if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
+                    }
                 }
-                const uint32_t s1 = __shfl_sync(0xffffffffu, start, j1);
-                const uint32_t s2 = __shfl_sync(0xffffffffu, start, j2);
-                const unsigned long long e1 = __shfl_sync(0xffffffffu, excl, j1);
-                const unsigned long long e2 = __shfl_sync(0xffffffffu, excl, j2);
-                const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
-                const int qi2 = __shfl_sync(0xffffffffu, qi, j2);
-                const uint32_t i1 = __shfl_sync(0xffffffffu, ind, j1);
-                const uint32_t i2 = __shfl_sync(0xffffffffu, ind, j2);
+                const uint32_t dl1 = __shfl_sync(0xffffffffu, delta, j1);
+                const uint32_t dl2 = __shfl_sync(0xffffffffu, delta, j2);
+                const uint32_t qx1 = __shfl_sync(0xffffffffu, qind, j1);
+                const uint32_t qx2 = __shfl_sync(0xffffffffu, qind, j2);
+                const int qi1 = (int)(qx1 & 0xffu), qi2 = (int)(qx2 & 0xffu);
+                const uint32_t i1 = qx1 >> 8, i2 = qx2 >> 8;
                 const bool v1 = t1 < total, v2 = t2 < total;
                 if (v1) {
-                    uint32_t p1 = s1 + (uint32_t)(t1 - e1);
-                    uint32_t p2 = v2 ? s2 + (uint32_t)(t2 - e2) : p1;
+                    uint32_t p1 = (uint32_t)t1 + dl1;
+                    uint32_t p2 = v2 ? (uint32_t)t2 + dl2 : p1;
                     if (i1) p1 = __ldg(sb_ids(a.sb, i1) + p1);   // subbin id array slot
                     if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + p2);
                     else if (!v2) p2 = p1;
@@ -309,6 +340,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
                         stage_hit(S, qi2, p2, h0, h1);
                 }
+            }
             }
         }
         __syncwarp();
