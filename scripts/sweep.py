@@ -59,6 +59,9 @@ def main():
     ap.add_argument("--configs", nargs="+", default=["C1", "C2", "C3"])
     ap.add_argument("--methods", nargs="+", default=["grid", "temporal", "subbin"])
     ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--dmax", type=float, default=None,
+                    help="skip distances above this (S2 at d = 5 has 7.5e9 results: 180 GB "
+                         "of host memory)")
     ap.add_argument("--out", default=None)
     a = ap.parse_args()
     out = open(a.out, "a") if a.out else None
@@ -69,6 +72,8 @@ def main():
         for method in a.methods:
             built = {}
             for d in c.d_sweep:
+                if a.dmax is not None and d > a.dmax:
+                    continue
                 key = d if method == "grid" else None
                 if key not in built:
                     for k in list(built):
