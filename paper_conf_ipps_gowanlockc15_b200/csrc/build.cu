@@ -124,15 +124,21 @@ __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, si
     block_reduce_write(b, &partial[blockIdx.x]);
 }
 
-// Bounds of the S entries i = floor(j n / S), j < S: the provisional grid of
-// the fused bounds + keys pass (any grid gives the same results -- the
-// stencils use the exact extents; see build_index_device).
+// Bounds of S entries, one per stride [floor(j n / S), floor((j+1) n / S)),
+// at a hashed offset inside it (a fixed offset aliases with periodic inputs:
+// trajectory-major D with a stride that is a multiple of the segments per
+// trajectory samples one time step only): the provisional grid of the fused
+// bounds + keys pass (any grid gives the same results -- the stencils use
+// the exact extents; see build_index_device).
 __global__ void __launch_bounds__(BT) k_bounds_sample(const double4* __restrict__ D, size_t n,
                                                      size_t S, Bounds* __restrict__ partial) {
     Bounds b;
     bounds_init(b);
     for (size_t j = (size_t)blockIdx.x * BT + threadIdx.x; j < S; j += (size_t)gridDim.x * BT) {
-        const size_t i = (size_t)(((unsigned __int128)j * n) / S);
+        const size_t i0 = (size_t)(((unsigned __int128)j * n) / S);
+        const size_t i1 = (size_t)(((unsigned __int128)(j + 1) * n) / S);
+        const unsigned long long h = (j + 1) * 0x9E3779B97F4A7C15ull;
+        const size_t i = i0 + (i1 > i0 ? (size_t)((h >> 32) % (i1 - i0)) : 0);
         bounds_add(b, D[2 * i], D[2 * i + 1]);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
@@ -994,6 +1000,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             choose_grid(hb, p, gf);
             bool ok = g.b >= 0.75 * gf.b && g.b <= 1.5 * gf.b;
             for (int a = 0; a < 3; ++a) ok = ok && g.w[a] >= 0.75 * gf.w[a] && g.w[a] <= 1.5 * gf.w[a];
+            // ... or missed part of the domain: entries beyond the sampled
+            // domain are clamped into the boundary bins / cells, which then
+            // hold far more than their share (a sample of one time step
+            // made two bins of 193 on a trajectory-major input)
+            ok = ok && hb.tmin >= g.tmin - g.b && hb.tmax <= g.tmin + (double)g.m * g.b + g.b;
+            for (int a = 0; a < 3; ++a)
+                ok = ok && hb.lo[a] >= g.o[a] - g.w[a] &&
+                     hb.hi[a] <= g.o[a] + (double)g.nc[a] * g.w[a] + g.w[a];
             if (ok) {
                 for (int a = 0; a < 3; ++a) g.half_ext[a] = 0.5 * hb.ext[a];
                 g.maxdur = hb.maxdur;

@@ -155,10 +155,21 @@ def test_crowded_cells(dts, oracle_mod):
         assert out.stdout == got.tobytes(), env
 
 
+def _sampled_positions(n):
+    """The rows the build's 2^16-entry sample reads: one per stride
+    [j n / S, (j+1) n / S), at a hashed offset (k_bounds_sample)."""
+    S = min(n, 1 << 16)
+    out = []
+    for j in range(S):
+        i0, i1 = j * n // S, (j + 1) * n // S
+        h = ((j + 1) * 0x9E3779B97F4A7C15) & 0xFFFFFFFFFFFFFFFF
+        out.append(i0 + ((h >> 32) % (i1 - i0) if i1 > i0 else 0))
+    return out
+
+
 def _unsampled_positions(n, k):
     """k positions that the build's 2^16-entry stride sample does not read."""
-    S = min(n, 1 << 16)
-    sampled = set((np.arange(S, dtype=np.uint64) * np.uint64(n) // np.uint64(S)).tolist())
+    sampled = set(_sampled_positions(n))
     out = [i for i in range(1, n) if i not in sampled][:k]
     assert len(out) == k
     return out
@@ -170,7 +181,9 @@ def test_sampled_grid_misses_outliers(dts, oracle_mod, kind):
     sample misses -- segments far longer than any sampled one (the grid is
     then rebuilt from the exact bounds) or short segments far outside the
     sampled domain (they clamp into the boundary cells) -- must still be
-    found, with the stencils taken from the exact extents."""
+    found, with the stencils taken from the exact extents (the grid is
+    rebuilt from the exact bounds when the sample missed part of the
+    domain)."""
     c = synth.make_config("C1", scale=0.2)
     D = c.D.reshape(-1, 8).copy()
     n = D.shape[0]
@@ -203,6 +216,33 @@ def test_sampled_grid_misses_outliers(dts, oracle_mod, kind):
     if kind == "long_segments":          # exact extent, not the sample's
         assert inf["max_extent"][0] >= 30.0
     idx.free()
+
+
+def test_periodic_input_sample_not_aliased(dts, oracle_mod):
+    """Trajectory-major D whose sample stride is a multiple of the segments
+    per trajectory (4 here, as 192 is for the paper's S2 shape): a sample at
+    a fixed offset per stride would see one time step and build two bins;
+    the hashed offsets (and the domain check on the provisional grid) give
+    one bin per time step.  Results match the oracle either way."""
+    g = synth.rng(11)
+    ntraj, nseg = 1 << 16, 4
+    t = np.arange(nseg + 1, dtype=np.float64)
+    pos = np.cumsum(g.normal(0, 0.01, (ntraj, nseg + 1, 3)), axis=1) + g.uniform(0, 1, (ntraj, 1, 3))
+    D = np.empty((ntraj, nseg, 8))
+    D[:, :, 0] = t[:-1]
+    D[:, :, 4] = t[1:]
+    D[:, :, 1:4] = pos[:, :-1]
+    D[:, :, 5:8] = pos[:, 1:]
+    D = np.ascontiguousarray(D.reshape(-1, 8))
+    Q = np.ascontiguousarray(D[::2621][:100].copy())
+    idx = dts.build_index(D)
+    inf = idx.info()
+    assert inf["bins"] >= nseg, inf
+    got = dts.search(idx, Q, 0.003)
+    idx.free()
+    ora = oracle_mod.search(D, Q, 0.003, threads=THREADS)
+    info = parity.compare(got, ora, D, Q, 0.003, oracle_mod)
+    assert info["common"] >= Q.shape[0]
 
 
 def test_build_phase_timings(dts):
