@@ -156,15 +156,9 @@ def test_crowded_cells(dts, oracle_mod):
 
 
 def _sampled_positions(n):
-    """The rows the build's 2^16-entry sample reads: one per stride
-    [j n / S, (j+1) n / S), at a hashed offset (k_bounds_sample)."""
+    """The rows the build's 2^16-entry sample reads: j n / S (k_bounds_sample)."""
     S = min(n, 1 << 16)
-    out = []
-    for j in range(S):
-        i0, i1 = j * n // S, (j + 1) * n // S
-        h = ((j + 1) * 0x9E3779B97F4A7C15) & 0xFFFFFFFFFFFFFFFF
-        out.append(i0 + ((h >> 32) % (i1 - i0) if i1 > i0 else 0))
-    return out
+    return [j * n // S for j in range(S)]
 
 
 def _unsampled_positions(n, k):
@@ -220,10 +214,11 @@ def test_sampled_grid_misses_outliers(dts, oracle_mod, kind):
 
 def test_periodic_input_sample_not_aliased(dts, oracle_mod):
     """Trajectory-major D whose sample stride is a multiple of the segments
-    per trajectory (4 here, as 192 is for the paper's S2 shape): a sample at
-    a fixed offset per stride would see one time step and build two bins;
-    the hashed offsets (and the domain check on the provisional grid) give
-    one bin per time step.  Results match the oracle either way."""
+    per trajectory (4 here, as 192 is for the paper's S2 shape): the strided
+    sample sees one time step and would build two bins; the exact time range
+    (from the fused keys pass) lies well outside the sampled one, so the
+    build redoes the keys with the exact grid, one bin per time step.  Results match the
+    oracle either way."""
     g = synth.rng(11)
     ntraj, nseg = 1 << 16, 4
     t = np.arange(nseg + 1, dtype=np.float64)
