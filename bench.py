@@ -155,7 +155,9 @@ def run_reference(args):
     cores = host_cores()
     times = []
     last_sample = ""
-    per_step_s = args.ref_step_seconds
+    # the whole --steps K --warmup W run stays within ~--ref-budget-seconds
+    per_step_s = max(0.5, min(args.ref_step_seconds,
+                              args.ref_budget_seconds / max(1, args.steps + args.warmup)))
     for i in range(args.warmup + args.steps):
         v, cores, sample = oracle_rate(cfg, per_step_s, seed=500 + i)
         if i >= args.warmup:
@@ -437,6 +439,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
+    ap.add_argument("--ref-budget-seconds", type=float, default=150.0,
+                    help="reference arm: oracle seconds for the whole run (per-step samples "
+                         "shrink with --steps + --warmup)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
