@@ -159,6 +159,31 @@ __global__ void __launch_bounds__(BT) k_bounds_final(const Bounds* __restrict__ 
     block_reduce_write(b, out);
 }
 
+// Occupancy of the sample's bounding box: the midpoints of the S strided
+// sample rows marked in a 32^3 bitmap over [lo, hi] (bounds read from the
+// device).  The fraction of marked cells estimates how much of the box the
+// data fills (C4's galaxy: 5%; C3's random walks: 60%).
+constexpr int OCC_RES = 32;
+__global__ void __launch_bounds__(BT) k_sample_occupancy(const double4* __restrict__ D, size_t n,
+                                                        size_t S, const Bounds* __restrict__ bnd,
+                                                        uint32_t* __restrict__ bitmap) {
+    const Bounds b = *bnd;
+    for (size_t j = (size_t)blockIdx.x * BT + threadIdx.x; j < S; j += (size_t)gridDim.x * BT) {
+        const size_t i = (size_t)(((unsigned __int128)j * n) / S);
+        const double4 s0 = D[2 * i], s1 = D[2 * i + 1];
+        const double mid[3] = {0.5 * (s0.y + s1.y), 0.5 * (s0.z + s1.z), 0.5 * (s0.w + s1.w)};
+        uint32_t cell = 0;
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            const double span = b.hi[a] - b.lo[a];
+            double f = span > 0.0 ? (mid[a] - b.lo[a]) / span * OCC_RES : 0.0;
+            int c = (f > 0.0) ? (int)fmin(f, (double)(OCC_RES - 1)) : 0;
+            cell = cell * OCC_RES + (uint32_t)c;
+        }
+        atomicOr(&bitmap[cell >> 5], 1u << (cell & 31u));
+    }
+}
+
 // Sorted (key, row) pairs, either packed -- a[p] = key << shift | row, when
 // key bits + row bits fit in 64 (a keys-only sort on the key bits then moves
 // 8 bytes per element instead of 12) -- or as separate arrays (ids != null).
@@ -848,7 +873,8 @@ static double cell_scale(int a) {
     return f[a];
 }
 
-static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g) {
+static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g, size_t n,
+                        double occ) {
     const double span_t = b.tmax - b.tmin;
     g.tmin = b.tmin;
     g.maxdur = b.maxdur;
@@ -879,6 +905,28 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
         g.w[a] = w;
         g.half_ext[a] = 0.5 * b.ext[a];
         g.nc[a] = (int32_t)std::min(std::floor(span / w) + 1.0, MAXC);
+    }
+    // sparse data: cap the cells per bin at 512 x the entries per bin per
+    // occupied fraction of the box (C3, 384 entries per bin in a 1000^3
+    // cube, had 12.7 M cells per bin: 96 row probes per query, nearly all
+    // empty); clustered or dense data (C4: 26 cells per such entry) are left
+    // alone.  Widths only grow, so the E + d lower bound still holds.
+    static const double dcap = [] {          // DTS_DENSITY_CAP: 0 disables
+        const char* e = getenv("DTS_DENSITY_CAP");
+        return e ? atof(e) : 512.0;
+    }();
+    if (p.method == DTS_METHOD_GRID && p.cells_per_dim == 0 && occ > 0.0 && dcap > 0.0 && n > 0) {
+        const double nb = (double)n / (double)g.m;
+        const double cap = std::max(64.0, dcap * nb / occ);
+        const double prod = (double)g.nc[0] * g.nc[1] * g.nc[2];
+        if (prod > cap) {
+            const double f = std::cbrt(prod / cap);
+            for (int a = 0; a < 3; ++a) {
+                const double span = b.hi[a] - b.lo[a];
+                g.w[a] *= f;
+                g.nc[a] = (int32_t)std::min(std::floor(span / g.w[a]) + 1.0, MAXC);
+            }
+        }
     }
     // keep the key space below 2^62: coarsen the finest axis until it fits
     while ((double)g.m * g.nc[0] * g.nc[1] * g.nc[2] >= 4.6e18) {
@@ -945,6 +993,27 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DevBuf<uint32_t> ids(0, s), ids_tmp(0, s);
     SortedKeys sk;
     bool done = false;
+    // sample occupancy of the bounding box (choose_grid's density cap)
+    double occ = -1.0;
+    DevBuf<uint32_t> occ_bits(OCC_RES * OCC_RES * OCC_RES / 32, s);
+    static thread_local uint32_t* occ_host = [] {
+        uint32_t* q = nullptr;
+        DTS_CUDA(cudaMallocHost(&q, OCC_RES * OCC_RES * OCC_RES / 8));
+        return q;
+    }();
+    auto occ_launch = [&](size_t S, const Bounds* bnd) {
+        DTS_CUDA(cudaMemsetAsync(occ_bits.p, 0, OCC_RES * OCC_RES * OCC_RES / 8, s));
+        const int nb = (int)std::min<size_t>(std::max<size_t>(grid_for(S) / 4, 1), 592);
+        k_sample_occupancy<<<nb, BT, 0, s>>>(D, n, S, bnd, occ_bits.p);
+        DTS_LAUNCH_CHECK();
+        DTS_CUDA(cudaMemcpyAsync(occ_host, occ_bits.p, OCC_RES * OCC_RES * OCC_RES / 8,
+                                 cudaMemcpyDeviceToHost, s));
+    };
+    auto occ_fraction = [&]() {
+        size_t c = 0;
+        for (int i = 0; i < OCC_RES * OCC_RES * OCC_RES / 32; ++i) c += __builtin_popcount(occ_host[i]);
+        return (double)c / (double)(OCC_RES * OCC_RES * OCC_RES);
+    };
     if (allow_fused && allow_packed && radix_onesweep(n)) {
         // 1. bounds of a strided sample -> provisional grid.  Any grid gives
         //    the same results: the keys only group the entries, and every
@@ -962,12 +1031,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         DTS_LAUNCH_CHECK();
         k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
         DTS_LAUNCH_CHECK();
+        occ_launch(S, total.p);
         mark();
         Bounds hs;
         DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         check(hs);
-        choose_grid(hs, p, g);
+        occ = occ_fraction();
+        choose_grid(hs, p, g, n, occ);
         const int kb = key_bits_of(g);
         if (row_bits + kb <= 64) {
             // 2-3. exact bounds + keys + sort histograms in one read of D
@@ -1008,7 +1079,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             // badly (cells or bins far narrower or wider than the exact rule
             // gives: correct either way, only slower)
             GridParams gf{};
-            choose_grid(hb, p, gf);
+            choose_grid(hb, p, gf, n, occ);
             bool ok = g.b >= 0.75 * gf.b && g.b <= 1.5 * gf.b;
             for (int a = 0; a < 3; ++a) ok = ok && g.w[a] >= 0.75 * gf.w[a] && g.w[a] <= 1.5 * gf.w[a];
             // ... or missed more than a tenth of the time range: entries
@@ -1040,7 +1111,12 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         DTS_CUDA(cudaStreamSynchronize(s));
         check(hb);
         g = GridParams{};
-        choose_grid(hb, p, g);
+        if (occ < 0.0) {            // no sample taken yet: the strided sample's occupancy
+            occ_launch(std::min<size_t>(n, (size_t)1 << 16), total.p);
+            DTS_CUDA(cudaStreamSynchronize(s));
+            occ = occ_fraction();
+        }
+        choose_grid(hb, p, g, n, occ);
         idx->key_bits = key_bits_of(g);
         const bool packed = allow_packed && row_bits + idx->key_bits <= 64;
         if (!packed) {
