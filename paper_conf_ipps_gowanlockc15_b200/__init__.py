@@ -12,6 +12,7 @@ from __future__ import annotations
 
 import ctypes
 import os
+import weakref
 
 import numpy as np
 
@@ -291,13 +292,22 @@ def build_index_device(D_dev, n: int = None, device: int = 0, temporal_bins: int
     return Index(h.value, device)
 
 
-def _host_results(ptr, count) -> np.ndarray:
-    if count == 0:
-        return np.empty(0, dtype=RESULT_DTYPE)
-    out = np.empty(count, dtype=RESULT_DTYPE)
-    ctypes.memmove(out.ctypes.data, ptr, count * RESULT_DTYPE.itemsize)
+def _free_results(ptr: int) -> None:
     load().dts_free_results(ctypes.c_void_p(ptr))
-    return out
+
+
+def _host_results(ptr, count) -> np.ndarray:
+    """The library's pinned result array as a numpy array, without a copy
+    (copying 0.8 GB of results into fresh pageable memory took longer than
+    the search): dts_free_results runs when the array and every view of it
+    are gone."""
+    if count == 0:
+        if ptr:
+            _free_results(ptr)
+        return np.empty(0, dtype=RESULT_DTYPE)
+    buf = (ctypes.c_char * (count * RESULT_DTYPE.itemsize)).from_address(ptr)
+    weakref.finalize(buf, _free_results, ptr)
+    return np.frombuffer(buf, dtype=RESULT_DTYPE, count=count)
 
 
 def search_ex(index: Index, Q, d: float, query_id_base: int = 0, stream=None,
