@@ -576,3 +576,26 @@ def test_pipelined_query_chunks_match(dts, oracle_mod, monkeypatch):
     qs = np.arange(0, c.Q.shape[0], 37)
     parity.compare(parity.restrict(ref, qs), oracle_mod.search_queries(c.D, c.Q, qs, 2.0),
                    c.D, c.Q, 2.0, oracle_mod)
+
+
+def test_host_results_zero_copy_lifetime(dts, oracle_mod):
+    """dts_search's host results are a numpy view of the library's pinned
+    array: a view taken from them stays valid after the array itself is gone
+    and other searches reuse the library's pinned-buffer cache."""
+    import gc
+    c = synth.make_config("C0")
+    idx = dts.build_index(c.D)
+    res = dts.search(idx, c.Q, c.d)
+    want = res.copy()
+    view = res[["query_id", "entry_id"]][::2]
+    tail = res["t_end"][1:]
+    del res
+    gc.collect()
+    for _ in range(5):                       # churn the pinned cache
+        r = dts.search(idx, c.Q[::-1].copy(), 0.2)
+        del r
+        gc.collect()
+    assert np.array_equal(view["query_id"], want["query_id"][::2])
+    assert np.array_equal(view["entry_id"], want["entry_id"][::2])
+    assert np.array_equal(tail, want["t_end"][1:])
+    idx.free()
