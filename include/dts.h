@@ -152,7 +152,9 @@ dts_status dts_build_index(const dts_segment* D, size_t n,
  * the call returns (stream-ordered, like a kernel launch), so D_dev and the
  * params' device arrays must stay valid until the stream reaches that point
  * (later work on the stream, or dts_index_get_info, which waits for it).
- * Searches on other streams wait for the build by themselves. Not retained. */
+ * Searches on other streams wait for the build by themselves, after their
+ * query preparation (which needs only the grid chosen at build time), so that
+ * preparation overlaps the build's tail. Not retained. */
 dts_status dts_build_index_device(const dts_segment* D_dev, size_t n,
                                   const dts_index_params* params,
                                   void* cuda_stream, dts_index** out_index);

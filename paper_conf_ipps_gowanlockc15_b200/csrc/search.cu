@@ -601,7 +601,6 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         return;
     }
     const double4* Q = reinterpret_cast<const double4*>(Q_dev);
-    if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));   // build may still run
     DevBuf<Counters> ctr(1, s);
     DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
 
@@ -664,6 +663,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
         }
     }
+    // the build may still run (dts_build_index_device returns once its last
+    // kernels are enqueued): the query prep above needs only the grid
+    // parameters, so on another stream it overlaps the build's tail; pass 1
+    // reads the index and waits for it here (inside the prep phase's events,
+    // so ms_count times pass 1 alone)
+    if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));
     tm.mark();
 
     // ---- pass 1: warp tiles, count + staging
