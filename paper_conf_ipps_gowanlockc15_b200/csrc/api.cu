@@ -116,6 +116,8 @@ void free_index_memory(dts_index* idx) {
     for (int a = 0; a < 3; ++a) {
         cache_free(idx->sb_block[a]);
         idx->sb_block[a] = nullptr;
+        cache_free(idx->sb_rec[a]);
+        idx->sb_rec[a] = nullptr;
     }
     idx->block = nullptr;
     idx->ht.slots = nullptr;

@@ -806,6 +806,21 @@ __global__ void __launch_bounds__(BT) k_sb_dir(const unsigned long long* __restr
 // entries: per dimension, (subbin, bin) keys for every overlap, a stable
 // radix sort (positions stay ascending inside a chunk) and a directory of
 // chunk offsets.
+// rec[j] = the record at sorted position ids[j] (two 256-bit accesses).
+__global__ void __launch_bounds__(BT) k_sb_gather_rec(double4* __restrict__ rec, const SegSoA soa,
+                                                     const uint32_t* __restrict__ ids,
+                                                     unsigned long long len) {
+    const unsigned long long j = (unsigned long long)blockIdx.x * BT + threadIdx.x;
+    if (j >= len) return;
+    double2 st, sx, sy, sz;
+    soa.load4(__ldg(ids + j), st, sx, sy, sz);
+    double* r = reinterpret_cast<double*>(rec + 2 * j);
+    asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r), "d"(st.x), "d"(st.y),
+                 "d"(sx.x), "d"(sx.y) : "memory");
+    asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r + 4), "d"(sy.x), "d"(sy.y),
+                 "d"(sz.x), "d"(sz.y) : "memory");
+}
+
 static void build_subbins(dts_index* idx, const double4* D, size_t n, const Bounds& hb,
                           const dts_index_params& p, cudaStream_t s) {
     const GridParams& g = idx->gp;
@@ -854,6 +869,16 @@ static void build_subbins(dts_index* idx, const double4* D, size_t n, const Boun
         DTS_LAUNCH_CHECK();
         sb.ids[a] = blk;
         sb.dir[a] = blk + len;
+        // the records of the id array, in its order (B200 layout choice: the
+        // paper's X/Y/Z arrays hold ids; a copy of the 64-byte records
+        // per dimension turns each candidate into a contiguous read)
+        double4* rec = static_cast<double4*>(cache_alloc((size_t)len * 2 * sizeof(double4) + 64));
+        idx->sb_rec[a] = rec;
+        if (len) {
+            k_sb_gather_rec<<<grid_for(len), BT, 0, s>>>(rec, idx->soa, blk, len);
+            DTS_LAUNCH_CHECK();
+        }
+        sb.rec[a] = rec;
         DTS_CUDA(cudaStreamSynchronize(s));
     }
 }

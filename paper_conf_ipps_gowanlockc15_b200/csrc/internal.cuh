@@ -156,6 +156,10 @@ struct SubbinIndex {
     int32_t m;
     const uint32_t* ids[3];
     const uint32_t* dir[3];
+    // the entry records of ids[a], in the same order (64 bytes per slot, two
+    // 256-bit loads): a subbin chunk streams its candidates contiguously
+    // instead of one dependent random record read per id
+    const double4* rec[3];
 };
 
 __device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double x) {
@@ -335,6 +339,7 @@ struct dts_index {
     uint32_t method = 0;           // dts_method
     dts::SubbinIndex sb{};         // DTS_METHOD_SUBBIN only
     uint32_t* sb_block[3] = {nullptr, nullptr, nullptr};   // ids + dir per dimension
+    double4* sb_rec[3] = {nullptr, nullptr, nullptr};      // records of ids, per dimension
     uint64_t sb_len[3] = {0, 0, 0};
     uint32_t* etraj = nullptr;     // trajectory id per sorted position (optional)
 };

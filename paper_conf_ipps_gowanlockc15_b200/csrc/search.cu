@@ -247,6 +247,18 @@ __device__ __forceinline__ const uint32_t* sb_ids(const SubbinIndex& sb, uint32_
     return ind == 1 ? sb.ids[0] : (ind == 2 ? sb.ids[1] : sb.ids[2]);
 }
 
+// The record at slot j of the subbin array of dimension ind - 1 (its copy
+// in id order, SubbinIndex::rec).
+__device__ __forceinline__ void sb_load(const SubbinIndex& sb, uint32_t ind, uint32_t j,
+                                        double2& st, double2& sx, double2& sy, double2& sz) {
+    const double4* r = (ind == 1 ? sb.rec[0] : (ind == 2 ? sb.rec[1] : sb.rec[2])) + 2 * (size_t)j;
+    const double4 a = ld256(r), b = ld256(r + 1);
+    st = make_double2(a.x, a.y);
+    sx = make_double2(a.z, a.w);
+    sy = make_double2(b.x, b.y);
+    sz = make_double2(b.z, b.w);
+}
+
 // Resolve probe `loc` of a query's stencil into one entry run [start,
 // start+cnt).  A grid probe is a stencil ROW (bin, cz, cy) over the cells
 // cx in [clo0, clo0 + cn0): keys are row-major with x fastest, so the
@@ -731,6 +743,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             const int o = occ >= 7 ? 6 : occ;
             if (o == 6) k_wtile_count<6, true, 32><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(ta);
             else k_wtile_count<5, true, 32><<<std::min<unsigned>(want, nsm * 5), WT, 0, s>>>(ta);
+        } else if (idx->method == DTS_METHOD_SUBBIN) {
+            k_wtile_count<7, false, 32, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
         } else if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
         else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
         else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);

@@ -142,7 +142,9 @@ struct WarpStage {
     unsigned long long bar[2];
 };
 
-template <int MINB, bool TMA = false, int CH = 32>
+// SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
+// temporal methods compile without that indirection.
+template <int MINB, bool TMA = false, int CH = 32, bool SB = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     __shared__ __align__(128) WarpStage<TMA ? CH : 1> STG[TMA ? WW : 1];
@@ -320,17 +322,21 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 const uint32_t qx1 = __shfl_sync(0xffffffffu, qind, j1);
                 const uint32_t qx2 = __shfl_sync(0xffffffffu, qind, j2);
                 const int qi1 = (int)(qx1 & 0xffu), qi2 = (int)(qx2 & 0xffu);
-                const uint32_t i1 = qx1 >> 8, i2 = qx2 >> 8;
+                const uint32_t i1 = SB ? qx1 >> 8 : 0u, i2 = SB ? qx2 >> 8 : 0u;
                 const bool v1 = t1 < total, v2 = t2 < total;
                 if (v1) {
                     uint32_t p1 = (uint32_t)t1 + dl1;
                     uint32_t p2 = v2 ? (uint32_t)t2 + dl2 : p1;
-                    if (i1) p1 = __ldg(sb_ids(a.sb, i1) + p1);   // subbin id array slot
-                    if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + p2);
+                    const uint32_t i2v = v2 ? i2 : i1;
+                    const uint32_t sl1 = p1, sl2 = p2;      // subbin slots (when i != 0)
+                    if (i1) p1 = __ldg(sb_ids(a.sb, i1) + sl1);   // id -> sorted position
+                    if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + sl2);
                     else if (!v2) p2 = p1;
                     double2 st1, sx1, sy1, sz1, st2, sx2, sy2, sz2;
-                    a.soa.load4(p1, st1, sx1, sy1, sz1);
-                    a.soa.load4(p2, st2, sx2, sy2, sz2);
+                    if (i1) sb_load(a.sb, i1, sl1, st1, sx1, sy1, sz1);   // contiguous copy
+                    else a.soa.load4(p1, st1, sx1, sy1, sz1);
+                    if (i2v) sb_load(a.sb, i2v, v2 ? sl2 : sl1, st2, sx2, sy2, sz2);
+                    else a.soa.load4(p2, st2, sx2, sy2, sz2);
                     double h0, h1;
                     const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
                     const bool x2 = a.excl && __ldg(a.etraj + p2) == S.qtraj[qi2];
