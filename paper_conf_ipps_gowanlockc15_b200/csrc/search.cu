@@ -645,7 +645,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             const char* e = getenv("DTS_QSORT_MIN");
             return e ? (size_t)atoll(e) : ((size_t)1 << 18);
         }();
-        const bool sort_q = nq >= qsort_min;
+        // (the temporal and subbin methods always sort: their one-run queries
+        // are grouped by identical run inside a tile, which needs neighbours)
+        const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID;
         DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q ? nq : 0, s);
         k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p,
                                              (packed && sort_q) ? nullptr : order.p, row_bits,
@@ -744,7 +746,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             if (o == 6) k_wtile_count<6, true, 32><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(ta);
             else k_wtile_count<5, true, 32><<<std::min<unsigned>(want, nsm * 5), WT, 0, s>>>(ta);
         } else if (idx->method == DTS_METHOD_SUBBIN) {
-            k_wtile_count<7, false, 32, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
+            k_wtile_count<7, false, 32, true, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
+        } else if (idx->method == DTS_METHOD_TEMPORAL) {
+            k_wtile_count<7, false, 32, false, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
         } else if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
         else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
         else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);

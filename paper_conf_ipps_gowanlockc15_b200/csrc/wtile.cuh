@@ -143,8 +143,11 @@ struct WarpStage {
 };
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
-// temporal methods compile without that indirection.
-template <int MINB, bool TMA = false, int CH = 32, bool SB = false>
+// temporal methods compile without that indirection.  GROUP: one-run
+// queries (temporal / subbin methods) streamed per group of identical runs
+// (step 1a); the grid method compiles without it (its rare one-run
+// fallback queries go through the probe rounds).
+template <int MINB, bool TMA = false, int CH = 32, bool SB = false, bool GROUP = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     __shared__ __align__(128) WarpStage<TMA ? CH : 1> STG[TMA ? WW : 1];
@@ -173,6 +176,8 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
 
         // ---- 0: queries, stencils, probe offsets
         unsigned long long nlook = 0;
+        bool single = false;                 // one-run query (temporal / subbin / fallback)
+        uint32_t rs = 0, rc = 0, ri = 0;
         const uint32_t sp = wt * WQ + lane;
         if (lane < WQ) {
             QState q{};
@@ -201,6 +206,13 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             S.qtraj[lane] = (a.excl && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
             S.qcount[lane] = 0;
             nlook = st.nlook;
+            if (GROUP && st.mode == MODE_TEMPORAL && st.rcnt > 0) {   // streamed in 1a
+                single = true;
+                nlook = 0;
+                rs = st.rstart;
+                rc = st.rcnt;
+                ri = st.rind;
+            }
         }
         if (lane == 0) { S.nhit = 0; S.over = 0; S.lkoff[0] = 0; }
         {
@@ -214,6 +226,45 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         }
         __syncwarp();
         const unsigned long long Ltot = S.lkoff[WQ];
+
+        // ---- 1a: one-run queries grouped by identical run (sorted neighbours
+        //      usually share their bins, or their subbin chunk): each
+        //      candidate of a run is loaded once and refined against every
+        //      query of the group, instead of once per query
+        for (uint32_t smask = GROUP ? __ballot_sync(0xffffffffu, single) : 0u; smask;) {
+            const int ld = __ffs(smask) - 1;
+            const uint32_t lrs = __shfl_sync(0xffffffffu, rs, ld);
+            const uint32_t lrc = __shfl_sync(0xffffffffu, rc, ld);
+            const uint32_t lri = __shfl_sync(0xffffffffu, ri, ld);
+            const uint32_t members =
+                __ballot_sync(0xffffffffu, single && rs == lrs && rc == lrc && ri == lri);
+            smask &= ~members;
+            n_cand += (unsigned long long)__popc(members) * lrc;
+            for (uint32_t base = 0; base < lrc; base += 32) {
+                const uint32_t t = base + lane;
+                if (t >= lrc) continue;
+                const uint32_t slot = lrs + t;
+                uint32_t p = slot;
+                double2 st, sx, sy, sz;
+                if (SB && lri) {
+                    sb_load(a.sb, lri, slot, st, sx, sy, sz);
+                    p = ~0u;                             // id looked up on a hit only
+                    if (a.excl) p = __ldg(sb_ids(a.sb, lri) + slot);
+                } else {
+                    a.soa.load4(p, st, sx, sy, sz);
+                }
+                const uint32_t et = a.excl ? __ldg(a.etraj + p) : 0u;
+                for (uint32_t mm = members; mm; mm &= mm - 1) {
+                    const int qi = __ffs(mm) - 1;
+                    double h0, h1;
+                    if (a.excl && et == S.qtraj[qi]) continue;
+                    if (refine(smem_query(S, qi), st, sx, sy, sz, d2, h0, h1)) {
+                        if (p == ~0u) p = __ldg(sb_ids(a.sb, lri) + slot);
+                        stage_hit(S, qi, p, h0, h1);
+                    }
+                }
+            }
+        }
 
         // ---- 1: rounds of 32 row probes, flattened, candidates two per lane
         for (unsigned long long r0 = 0; r0 < Ltot; r0 += 32) {
