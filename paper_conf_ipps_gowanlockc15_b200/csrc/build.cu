@@ -899,7 +899,8 @@ static double cell_scale(int a) {
 }
 
 static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& g, size_t n,
-                        double occ) {
+                        double occ, bool* capped = nullptr) {
+    if (capped) *capped = false;
     const double span_t = b.tmax - b.tmin;
     g.tmin = b.tmin;
     g.maxdur = b.maxdur;
@@ -931,20 +932,21 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
         g.half_ext[a] = 0.5 * b.ext[a];
         g.nc[a] = (int32_t)std::min(std::floor(span / w) + 1.0, MAXC);
     }
-    // sparse data: cap the cells per bin at 512 x the entries per bin per
+    // sparse data: cap the cells per bin at 1024 x the entries per bin per
     // occupied fraction of the box (C3, 384 entries per bin in a 1000^3
     // cube, had 12.7 M cells per bin: 96 row probes per query, nearly all
     // empty); clustered or dense data (C4: 26 cells per such entry) are left
     // alone.  Widths only grow, so the E + d lower bound still holds.
     static const double dcap = [] {          // DTS_DENSITY_CAP: 0 disables
         const char* e = getenv("DTS_DENSITY_CAP");
-        return e ? atof(e) : 512.0;
+        return e ? atof(e) : 1024.0;
     }();
     if (p.method == DTS_METHOD_GRID && p.cells_per_dim == 0 && occ > 0.0 && dcap > 0.0 && n > 0) {
         const double nb = (double)n / (double)g.m;
         const double cap = std::max(64.0, dcap * nb / occ);
         const double prod = (double)g.nc[0] * g.nc[1] * g.nc[2];
         if (prod > cap) {
+            if (capped) *capped = true;
             const double f = std::cbrt(prod / cap);
             for (int a = 0; a < 3; ++a) {
                 const double span = b.hi[a] - b.lo[a];
@@ -1056,14 +1058,22 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         DTS_LAUNCH_CHECK();
         k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
         DTS_LAUNCH_CHECK();
-        occ_launch(S, total.p);
         mark();
         Bounds hs;
         DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         check(hs);
-        occ = occ_fraction();
-        choose_grid(hs, p, g, n, occ);
+        // the occupancy only matters when even a full box would be capped
+        // (C3); dense or clustered data (C4, C2, S3) skip its kernel
+        bool capped = false;
+        choose_grid(hs, p, g, n, 1.0, &capped);
+        occ = 1.0;
+        if (capped) {
+            occ_launch(S, total.p);
+            DTS_CUDA(cudaStreamSynchronize(s));
+            occ = occ_fraction();
+            choose_grid(hs, p, g, n, occ);
+        }
         const int kb = key_bits_of(g);
         if (row_bits + kb <= 64) {
             // 2-3. exact bounds + keys + sort histograms in one read of D
@@ -1137,9 +1147,15 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         check(hb);
         g = GridParams{};
         if (occ < 0.0) {            // no sample taken yet: the strided sample's occupancy
-            occ_launch(std::min<size_t>(n, (size_t)1 << 16), total.p);
-            DTS_CUDA(cudaStreamSynchronize(s));
-            occ = occ_fraction();
+            bool capped = false;
+            choose_grid(hb, p, g, n, 1.0, &capped);
+            occ = 1.0;
+            if (capped) {
+                occ_launch(std::min<size_t>(n, (size_t)1 << 16), total.p);
+                DTS_CUDA(cudaStreamSynchronize(s));
+                occ = occ_fraction();
+            }
+            g = GridParams{};
         }
         choose_grid(hb, p, g, n, occ);
         idx->key_bits = key_bits_of(g);
