@@ -351,11 +351,10 @@ __device__ __forceinline__ void insert_block(const HashTable& ht, unsigned long 
         for (int i = 0; i < 2; ++i) {
             BlockSlot& sl = slots[2 * b + i];
             if (atomicCAS(&sl.key, EMPTY_KEY, blk) == EMPTY_KEY) {
-                sl.start = start;
-                sl.big = big;
-                unsigned long long* c = reinterpret_cast<unsigned long long*>(sl.cum);
-                c[0] = c_lo;
-                c[1] = c_hi;
+                // the rest of the slot in two stores: (start, big), cum[0..7]
+                *reinterpret_cast<unsigned long long*>(&sl.start) =
+                    (unsigned long long)start | ((unsigned long long)big << 32);
+                *reinterpret_cast<ulonglong2*>(sl.cum) = make_ulonglong2(c_lo, c_hi);
                 return;
             }
         }
