@@ -599,3 +599,30 @@ def test_host_results_zero_copy_lifetime(dts, oracle_mod):
     assert np.array_equal(view["entry_id"], want["entry_id"][::2])
     assert np.array_equal(tail, want["t_end"][1:])
     idx.free()
+
+
+def test_density_cap_invariant(dts, oracle_mod):
+    """Sparse data (C3-shaped: a few hundred entries per bin in a 1000^3
+    cube) gets coarser cells from the density cap; the result bytes are the
+    same as with the plain E + d grid (DTS_DENSITY_CAP=0) and match the
+    oracle."""
+    import subprocess
+    import sys
+    c = synth.make_config("C3", scale=0.05)
+    code = ("import sys; sys.path[:0] = [%r, %r]; import synth, "
+            "paper_conf_ipps_gowanlockc15_b200 as m; c = synth.make_config('C3', scale=0.05); "
+            "i = m.build_index(c.D); sys.stderr.write(repr(i.info()['grid'])); "
+            "r = m.search(i, c.Q, c.d); sys.stdout.buffer.write(r.tobytes())"
+            % (REPO, os.path.join(REPO, "tests")))
+    outs, grids = [], []
+    for env in ({}, {"DTS_DENSITY_CAP": "0"}):
+        out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
+                             capture_output=True, timeout=600)
+        assert out.returncode == 0, out.stderr.decode()[-2000:]
+        outs.append(out.stdout)
+        grids.append(out.stderr.decode()[-60:])
+    assert outs[0] == outs[1], grids
+    assert grids[0] != grids[1], grids          # the cap did change the grid
+    got = np.frombuffer(outs[0], dtype=dts.RESULT_DTYPE)
+    parity.compare(got, oracle_mod.search(c.D, c.Q, c.d, threads=THREADS), c.D, c.Q, c.d,
+                   oracle_mod)
