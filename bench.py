@@ -4,15 +4,23 @@ search time and query-segments/s at 1/2/4/8 B200, % HBM roofline).
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--config C4] [--impl reference]
 
-A step = one pass of the whole hot path over the
-workload: index build over the resident entry set D, query prep, both fused
-candidate-streaming + refinement passes, the exact-offset scan, canonical
-ordering.  `value` is device-timed throughput with inputs already in HBM;
-`e2e` is the same metric through the C ABI's host entry points (pinned host
-D and Q copied in, results copied out every step).  Multi-GPU (torchrun):
-weak scaling, every rank searches its own 1M-query set against the replicated
-D; the only collective is an all_gather of the per-rank result counts (global
-offsets).  Rank 0 prints one JSON line.
+A step is one search of the workload's whole query set against the resident
+index: query prep (keys + sort), candidate generation, the fused candidate
+streaming + fp64 refinement count pass, the exact-offset scan and the
+emission pass.  That is the paper's response time:
+"the time to construct the index is not included".  The index build
+(§8(a1)-(a2)) is timed separately every run (`with_build`: build + search per
+step) and reported next to it.  `value` is device-timed throughput with the
+inputs resident in HBM; `e2e` is the same search through the C ABI's host
+entry point (pinned host Q copied in, results copied out every step).
+
+Multi-GPU (torchrun, one process per GPU): strong scaling of the ONE query
+set -- every rank holds D + index and the whole Q; inside each timed step the
+ranks cost an equal share of Q (dts_query_costs_device), all-gather the
+per-block candidate counts, cut the prefix sum into balanced contiguous
+query-id ranges, search their range, and all-gather the result counts (the
+offsets of the canonical global result).  The step time is
+the max over ranks.  Rank 0 prints one JSON line.
 
 The oracle (oracle/, test infrastructure) runs only in the cpu_baseline leg
 (rank 0, N=1) and in --impl reference.
@@ -20,8 +28,11 @@ The oracle (oracle/, test infrastructure) runs only in the cpu_baseline leg
 from __future__ import annotations
 
 import argparse
+import csv
+import io
 import json
 import os
+import shutil
 import statistics
 import subprocess
 import sys
@@ -36,17 +47,22 @@ if ROOT not in sys.path:
 
 import synth  # noqa: E402
 
-METRIC = "query-segments/s (search step incl. index build; BASELINE: search time and q-seg/s at 1/2/4/8 B200, % HBM roofline)"
+METRIC = ("query-segments/s: search of the whole query set against the resident index "
+          "(the paper's response time, build excluded, P:L135); BASELINE: search time and "
+          "query-segments/s at 1/2/4/8 B200, % HBM roofline")
 UNIT = "query-segments/s"
 WORKLOADS = {
     "C4": "galaxy-shaped synthetic at scale: 20,132,736 entry segments (104,858 stellar-orbit "
-          "trajectories x 192 steps), 1,000,128 query segments per rank (5,209 trajectories "
-          "sampled from D), d=0.005 (BASELINE.json configs[4])",
+          "trajectories x 192 steps), 1,000,128 query segments (5,209 trajectories sampled "
+          "from D), d=0.005 (BASELINE.json configs[4]); query-sharded over the ranks",
     "C1": "galaxy-shaped synthetic: 1,048,512 entry segments, 9,984 query segments, d=0.005 "
           "(BASELINE.json configs[1])",
     "C2": "uniform dense random walks: 4,194,432 entries, 100,032 queries (configs[2])",
     "C3": "uniform sparse long-span random walks: 3,990,000 entries, 99,750 queries (configs[3])",
 }
+# extra d points of the headline workload (SURVEY.md §8(d) sweep)
+POINTS = {"C4": [0.02], "C1": [0.02], "C2": [2.0], "C3": [20.0]}
+BLOCK = 256          # queries per cost block (strong-scaling split granularity)
 
 
 def _env_int(k, default):
@@ -62,6 +78,13 @@ def load_peaks():
         j = json.load(open(p))
         return float(j["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def config_dict(name, cfg, d):
+    """The workload, identical in both arms (own and reference)."""
+    return {"workload": WORKLOADS.get(name, name), "name": name,
+            "n_entries": int(cfg.D.shape[0]), "n_queries": int(cfg.Q.shape[0]), "d": d,
+            "l2": "flushed between steps (256 MiB write outside the timed events)"}
 
 
 class ClockSampler:
@@ -125,26 +148,27 @@ def host_cores():
         return os.cpu_count() or 1
 
 
-def oracle_rate(cfg, seconds: float, seed: int):
+def oracle_rate(cfg, d, seconds: float, seed: int):
     """Oracle (as it stands) on a bounded sample of the workload's queries:
     brute force of each sampled query against all of D, one single-threaded
-    oracle instance per host core.  Returns (q-seg/s, cores, sample text)."""
+    oracle instance per host core.  Returns (q-seg/s, cores, sample text,
+    wall seconds)."""
     import oracle
     oracle.build()
     cores = host_cores()
     g = synth.rng(seed)
     t = time.perf_counter()
-    oracle.search_queries(cfg.D, cfg.Q, [int(g.integers(cfg.Q.shape[0]))], cfg.d)
+    oracle.search_queries(cfg.D, cfg.Q, [int(g.integers(cfg.Q.shape[0]))], d)
     t1 = max(time.perf_counter() - t, 1e-4)               # one query, one core
-    nsample = int(max(cores, min(20000, cores * max(1, round(seconds / t1)))))
+    nsample = int(max(cores, min(40000, cores * max(1, round(seconds / t1)))))
     qs = np.sort(g.choice(cfg.Q.shape[0], size=min(nsample, cfg.Q.shape[0]), replace=False))
     t = time.perf_counter()
-    oracle.search_queries(cfg.D, cfg.Q, qs, cfg.d, threads=cores)
+    oracle.search_queries(cfg.D, cfg.Q, qs, d, threads=cores)
     el = time.perf_counter() - t
     sample = (f"{qs.size} query segments sampled uniformly (seed {seed}) from the workload's "
               f"{cfg.Q.shape[0]}, each brute-forced against all {cfg.D.shape[0]} entries; "
               f"{el:.1f} s wall on {cores} threads")
-    return qs.size / el, cores, sample
+    return qs.size / el, cores, sample, el
 
 
 def run_reference(args):
@@ -152,34 +176,83 @@ def run_reference(args):
     if rank != 0:
         return 0
     cfg = synth.make_config(args.config)
+    d = args.d if args.d is not None else cfg.d
     cores = host_cores()
-    times = []
+    vals, walls = [], []
     last_sample = ""
-    # the whole --steps K --warmup W run stays within ~--ref-budget-seconds
+    # the whole --steps K --warmup W run stays within ~--ref-budget-seconds;
+    # a step is one bounded sample of the workload's queries
     per_step_s = max(0.5, min(args.ref_step_seconds,
                               args.ref_budget_seconds / max(1, args.steps + args.warmup)))
     for i in range(args.warmup + args.steps):
-        v, cores, sample = oracle_rate(cfg, per_step_s, seed=500 + i)
+        v, cores, sample, el = oracle_rate(cfg, d, per_step_s, seed=500 + i)
         if i >= args.warmup:
-            times.append(v)
+            vals.append(v)
+            walls.append(el)
             last_sample = sample
-    value = statistics.median(times)
+    value = statistics.median(vals)
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT,
         "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup,
-        "ms_per_step": 1e3 * cfg.Q.shape[0] / value, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config,
-                   "n_entries": int(cfg.D.shape[0]), "n_queries": int(cfg.Q.shape[0]),
-                   "d": cfg.d},
+        "ms_per_step": 1e3 * statistics.median(walls), "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": config_dict(args.config, cfg, d),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
                          "sample": "per step: " + last_sample},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
-        "note": "plain single-threaded C brute force (oracle/), one instance per host core; "
-                "ms_per_step extrapolates the sampled rate to the full query set",
+        "note": "plain single-threaded C brute force (oracle/), one instance per host core; each "
+                "step is a bounded uniform sample of the workload's queries (ms_per_step is the "
+                "sample's wall time, value = sampled queries / that time)",
     }
     print(json.dumps(line), flush=True)
     return 0
+
+
+def measure_traffic(config, d, timeout=420):
+    """DRAM bytes of one pass-1 launch (k_wtile_count), measured now with ncu
+    (dram__bytes_read.sum + dram__bytes_write.sum, one launch, the same
+    workload and launch configuration) in a child process.  Returns (dict or
+    None, note)."""
+    ncu = shutil.which("ncu") or "/usr/local/cuda/bin/ncu"
+    if not os.path.exists(ncu):
+        return None, "ncu not found"
+    cmd = [ncu, "--metrics", "dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum",
+           "--clock-control", "none", "-k", "regex:k_wtile_count", "-c", "1", "--csv",
+           sys.executable, os.path.join(ROOT, "scripts", "traffic_probe.py"), "--config", config,
+           "--d", repr(d)]
+    try:
+        out = subprocess.run(cmd, capture_output=True, text=True, timeout=timeout)
+    except (subprocess.TimeoutExpired, OSError) as e:
+        return None, f"ncu probe failed: {type(e).__name__}"
+    vals = {}
+    text = out.stdout
+    start = text.find('"ID"')
+    if start < 0:
+        return None, "ncu probe: no metrics in output (rc %d)" % out.returncode
+    for row in csv.DictReader(io.StringIO(text[start:])):
+        name, unit, v = row.get("Metric Name"), row.get("Metric Unit"), row.get("Metric Value")
+        try:
+            x = float(str(v).replace(",", ""))
+        except (TypeError, ValueError):
+            continue
+        scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-9,
+                 "usecond": 1e-6, "msecond": 1e-3}.get(unit, 1)
+        vals[name] = x * scale
+    if "dram__bytes_read.sum" not in vals:
+        return None, "ncu probe: metrics missing"
+    return {"dram_bytes": vals["dram__bytes_read.sum"] + vals.get("dram__bytes_write.sum", 0.0),
+            "dram_read": vals["dram__bytes_read.sum"],
+            "dram_write": vals.get("dram__bytes_write.sum", 0.0),
+            "ncu_kernel_s": vals.get("gpu__time_duration.sum")}, \
+        "ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum on one k_wtile_count launch " \
+        "(scripts/traffic_probe.py, same workload; cold L2, as in the timed steps)"
+
+
+def pass1_bytes(st, nq):
+    """Algorithmic bytes of one pass-1 launch (SURVEY.md §8(d) per-unit
+    figures): 64 B per candidate pair, 68 B per query (record +
+    count), 8 B per offset lookup, 24 B per result staged."""
+    return 64 * st["candidates"] + 68 * nq + 8 * st["cell_lookups"] + 24 * st["results"]
 
 
 def run_own(args):
@@ -206,7 +279,7 @@ def run_own(args):
     from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
     dts.load()
 
-    cfg = synth.make_config(args.config, rank=rank)
+    cfg = synth.make_config(args.config)        # the same D and Q on every rank
     d = args.d if args.d is not None else cfg.d
     n, nq = cfg.D.shape[0], cfg.Q.shape[0]
     D_pin = torch.from_numpy(cfg.D).pin_memory()
@@ -216,212 +289,223 @@ def run_own(args):
     stream = torch.cuda.current_stream(dev)
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)   # > 126 MB L2
 
-    def step():
-        """The hot path of one step: returns when its results are on the
-        device (the library syncs for the result count)."""
-        idx = dts.build_index_device(D_dev, device=local, stream=stream)
-        res, st = dts.search_device(idx, Q_dev, d, stream=stream, time_kernels=True)
+    def maxrank(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], device=dev if backend == "nccl" else "cpu", dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def barrier():
+        torch.cuda.synchronize(dev)
         if world > 1:
-            dts_dist.global_offset(res.count, rank, world)
-        return idx, res, st
+            dist.barrier()
 
-    def finish(idx, res, st, stats_out=None):
-        """Bookkeeping after the timed region of a step: phase times, frees."""
-        if stats_out is not None:
-            inf = idx.info()
-            st["ms_build"] = inf["ms_build"]
-            st["ms_phase"] = list(inf["ms_phase"])
-            st["index"] = inf
-            stats_out.append(st)
-        cnt = res.count
-        res.free()
-        idx.free()
-        return cnt
+    # ---- the index: built once, outside the timed search
+    idx = dts.build_index_device(D_dev, device=local, stream=stream)
+    build_info = idx.info()
 
-    for _ in range(max(args.warmup, 0)):
-        finish(*step())
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
+    def search_step(dd, timed_kernels=True):
+        """One search of the whole query set (this rank's balanced share of
+        it at N > 1).  Returns (results, stats, (lo, hi))."""
+        if world == 1:
+            res, st = dts.search_device(idx, Q_dev, dd, stream=stream, time_kernels=timed_kernels)
+            return res, st, (0, nq)
+        res, st, rng, _, _ = dts_dist.search_strong(idx, Q_dev, dd, rank, world, block=BLOCK,
+                                                    stream=stream, time_kernels=timed_kernels)
+        return res, st, rng
 
-    # ---- timed region: per-step CUDA events on the launching stream, L2
-    #      flushed between steps (outside the events)
+    def timed(fn, steps, warmup, after=None):
+        """CUDA events on the launching stream around each step, L2 flushed
+        between steps (outside the events); max over ranks of the total.
+        Returns (ms per step, per-step ms, per-step outputs, result count,
+        library kernel launches in the timed steps)."""
+        outs = []
+        for _ in range(warmup):
+            r = fn()
+            r[0].free()
+            if after:
+                after(r)
+        barrier()
+        k0 = dts.kernel_launches()
+        evs = []
+        for _ in range(steps):
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            r = fn()
+            e1.record(stream)
+            evs.append((e0, e1))
+            flush.zero_()
+            outs.append(r[1:])
+            cnt = r[0].count
+            r[0].free()
+        barrier()
+        k1 = dts.kernel_launches()
+        ms = [a.elapsed_time(b) for a, b in evs]
+        return maxrank(sum(ms)) / steps, ms, outs, cnt, k1 - k0
+
+    # ---- headline: search of the whole query set, index resident
+    barrier()
     clocks = ClockSampler(local)
     clocks.start()
-    launches0 = dts.kernel_launches()
-    evs = []
-    stats = []
-    torch.cuda.synchronize(dev)
-    if world > 1:
-        dist.barrier()
     wall0 = time.perf_counter()
-    results = 0
-    for _ in range(args.steps):
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        out = step()
-        e1.record(stream)
-        evs.append((e0, e1))
-        flush.zero_()
-        results = finish(*out, stats_out=stats)
-    torch.cuda.synchronize(dev)
+    ms_per_step, step_ms, outs, results, launches = timed(lambda: search_step(d), args.steps,
+                                                          args.warmup)
     wall = time.perf_counter() - wall0
-    if world > 1:
-        dist.barrier()
-    launches = dts.kernel_launches() - launches0
     clk = clocks.stop()
-    step_ms = [a.elapsed_time(b) for a, b in evs]
-    total_ms = sum(step_ms)
-    if world > 1:
-        t = torch.tensor([total_ms], device=dev if backend == "nccl" else "cpu",
-                         dtype=torch.float64)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        total_ms = float(t.item())
-    ms_per_step = total_ms / args.steps
-    value = world * nq / (ms_per_step * 1e-3)
-
-    # ---- per-kernel rooflines (CUDA events in-lib, on the launching stream):
-    #      algorithmic bytes per launch (DESIGN.md §6) / mean event time
-    peak, peak_src = load_peaks()
+    value = nq / (ms_per_step * 1e-3)
+    stats = [o[0] for o in outs]
+    lo, hi = outs[-1][1]
+    nq_rank = hi - lo
     st0 = stats[-1]
-    ms_count = statistics.mean(s["ms_count"] for s in stats)
-    ms_scatter = statistics.mean(s["ms_scatter"] for s in stats)
-    ms_build = statistics.mean(s["ms_build"] for s in stats)
-    ph = [statistics.mean(s["ms_phase"][i] for s in stats) for i in range(5)]
-    inf = st0["index"]
-    ncell_key = inf["bins"] * inf["grid"][0] * inf["grid"][1] * inf["grid"][2]
-    kbits = max(1, int(ncell_key - 1).bit_length())
-    npass = (kbits + 7) // 8                 # the library's digit plan: 9-bit digits
-    if npass > 1 and kbits <= 9 * (npass - 1):   # where they save a pass
-        npass -= 1
-    ncells = inf["cells"]
-    alg_bytes = st0["candidates"] * 64 + nq * (64 + 4) + st0["cell_lookups"] * 64
-    traffic_all = {}
-    tf = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tf):
-        try:
-            traffic_all = json.load(open(tf)).get(args.config, {})
-        except (ValueError, AttributeError):
-            traffic_all = {}
-    kernels = [
-        # name, ms per launch-group, algorithmic bytes, model
-        ("k_wtile_count", ms_count, alg_bytes,
-         "64 B per candidate + 68 B per query + 64 B per hash-bucket probe"),
-        ("k_onesweep (entry sort)", ph[2],
-         (0 if inf.get("build_flags", 0) & 1 else n * 8) + npass * n * 16,
-         f"{npass} passes x (8 B read + 8 B write) per key"
-         + ("" if inf.get("build_flags", 0) & 1 else " + 8 B/key histogram read")
-         + "; issue/latency-bound, not HBM-bound (DRAM ~15% busy): CUB DeviceRadixSort "
-           "takes 1.09 ms on the same shape (profiles/r01d_cub_sort.txt)"),
-        ("k_gather_cells", ph[3], n * (8 + 64 + 68),
-         "8 B sorted key + 64 B record read + 68 B record/id write per entry"),
-        ("k_insert_blocks_lane" if inf.get("hash_kind", 0) == 1 else "k_insert_tiled", ph[4],
-         n * 8 + inf.get("hash_items", ncells) * (32 if inf.get("hash_kind", 0) == 1 else 16),
-         "8 B key per entry + one slot per hash item (32 B per 8-key block, or 16 B per cell); "
-         "phase includes the table memset"),
-    ]
-    if inf.get("build_flags", 0) & 1:
-        kernels += [
-            ("k_bounds_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
-             "(exact bounds, packed keys and all sort-pass digit counts in one read)"),
-            ("k_bounds_sample", ph[0], 65536 * 64, "64 B per sampled entry (2^16 sample; "
-             "phase includes the host read-back)"),
-        ]
-    else:
-        kernels += [
-            ("k_bounds", ph[0], n * 64, "64 B record read per entry"),
-            ("k_keys", ph[1], n * (64 + 8), "64 B record read + 8 B key write per entry "
-             "(phase includes the host read-back of the bounds)"),
-        ]
-    kern = []
-    for name, ms, by, model in kernels:
-        a_gbs = by / (ms * 1e-3) / 1e9 if ms > 0 else None
-        kern.append({"kernel": name, "ms": ms, "bytes": int(by), "achieved_gbs": a_gbs,
-                     "frac": (a_gbs / peak) if a_gbs else None,
-                     "traffic": traffic_all.get(name.split()[0]), "bytes_model": model})
-    dom = max(kern, key=lambda k: k["ms"])
-    achieved = alg_bytes / (ms_count * 1e-3) / 1e9
-    traffic = traffic_all.get("k_wtile_count")
+    mean = lambda k: statistics.mean(s[k] for s in stats)   # noqa: E731
+    ph = {k: mean(k) for k in ("ms_prep", "ms_count", "ms_scan", "ms_scatter", "ms_canon")}
 
-    # ---- e2e through the C ABI host entry points (pinned host buffers)
-    e2e_val = None
-    e2e_search = None
-    h2d = (n + nq) * 64
-    d2h = results * 24
-    if rank == 0 or world > 1:
-        D_np = D_pin.numpy()
-        Q_np = Q_pin.numpy()
-        ts = []
-        ts_search = []
-        for i in range(max(1, args.e2e_steps) + 1):
-            torch.cuda.synchronize(dev)
-            t0 = time.perf_counter()
-            idx = dts.build_index(D_np, device=local)
-            t1 = time.perf_counter()
-            res = dts.search(idx, Q_np, d)
-            t2 = time.perf_counter()
-            if i > 0:
-                ts.append(t2 - t0)
-                ts_search.append(t2 - t1)
-            d2h = res.nbytes
-            idx.free()
-            del res
-        e2e_val = world * nq / statistics.median(ts)
-        e2e_search = world * nq / statistics.median(ts_search)
+    # ---- roofline of the dominant kernel: pass 1 (k_wtile_count)
+    peak, peak_src = load_peaks()
+    alg = pass1_bytes(st0, nq_rank)
+    achieved = alg / (ph["ms_count"] * 1e-3) / 1e9
+    traffic, tnote = (None, "skipped (--no-traffic or N > 1)")
+    if rank == 0 and world == 1 and not args.no_traffic:
+        traffic, tnote = measure_traffic(args.config, d)
+    dram = traffic["dram_bytes"] if traffic else None
+    roofline = {
+        "bound": "hbm", "kernel": "k_wtile_count (pass 1: fused candidate streaming + fp64 "
+                                  "refinement + per-query counts + hit staging)",
+        "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+        "traffic": dram, "peak_source": peak_src, "algorithmic_bytes": int(alg),
+        "ms": ph["ms_count"],
+        "bytes_model": "64 B x candidates + 68 B x queries + 8 B x offset lookups + 24 B x "
+                       "results (SURVEY.md §8(d) per-unit figures)",
+        "units": {"candidates": st0["candidates"], "queries": nq_rank,
+                  "offset_lookups": st0["cell_lookups"], "results": st0["results"]},
+        "frac_algorithmic": achieved / peak,
+        "frac_dram": (dram / (ph["ms_count"] * 1e-3) / 1e9 / peak) if dram else None,
+        "traffic_note": tnote,
+        "share_of_step": ph["ms_count"] / ms_per_step if ms_per_step > 0 else None,
+        "note": "achieved = algorithmic bytes / mean pass-1 duration (CUDA events on the "
+                "launching stream inside the library, every timed step)",
+    }
+
+    # ---- extra d points of the same workload (fewer steps)
+    points = []
+    for dp in ([] if args.no_points else POINTS.get(args.config, [])):
+        pms, _, pouts, pres, _ = timed(lambda: search_step(dp), max(3, args.steps // 5), 2)
+        pst = pouts[-1][0]
+        plo, phi = pouts[-1][1]
+        pc = statistics.mean(o[0]["ms_count"] for o in pouts)
+        pa = pass1_bytes(pst, phi - plo) / (pc * 1e-3) / 1e9
+        points.append({"d": dp, "value": nq / (pms * 1e-3), "ms_per_step": pms,
+                       "results": pst["results"], "candidates": pst["candidates"],
+                       "offset_lookups": pst["cell_lookups"], "ms_count_pass": pc,
+                       "roofline_search": {"achieved": pa, "peak": peak, "frac": pa / peak,
+                                           "algorithmic_bytes": pass1_bytes(pst, phi - plo)},
+                       "phases_ms": {k: statistics.mean(o[0][k] for o in pouts)
+                                     for k in ("ms_prep", "ms_count", "ms_scan", "ms_scatter",
+                                               "ms_canon")}})
+
+    # ---- secondary line: index build + search per step (all §8(a) rows)
+    wb = None
+    if not args.no_build_line:
+        def build_step():
+            i2 = dts.build_index_device(D_dev, device=local, stream=stream)
+            r = search_step(d)
+            return r[0], (r[1], i2), r[2]
+        bms, _, bouts, _, _ = timed(build_step, args.build_steps, 2,
+                                    after=lambda r: r[1][1].free())
+        infs = []
+        for (s_, i2), _r in bouts:
+            infs.append(i2.info())
+            i2.free()
+        bph = [statistics.mean(i["ms_phase"][k] for i in infs) for k in range(5)]
+        bbuild = statistics.mean(i["ms_build"] for i in infs)
+        wb = {"value": nq / (bms * 1e-3), "ms_per_step": bms, "ms_build": bbuild,
+              "build_phases_ms": {"bounds_sample": bph[0], "bounds_keys": bph[1], "sort": bph[2],
+                                  "gather": bph[3], "insert": bph[4]},
+              "note": "index build (bounds, keys, radix sort, gather, hash insert) + the "
+                      "search, per step; every rank builds the replicated index"}
+
+    # ---- e2e through the C ABI host entry point (pinned host Q and results)
+    Q_np = Q_pin.numpy()
+    if world == 1:
+        lo_e, hi_e = 0, nq
+    else:
+        b = dts_dist.balanced_query_bounds(idx, Q_dev, d, rank, world, block=BLOCK,
+                                           stream=stream)
+        lo_e, hi_e = b[rank], b[rank + 1]
+    idx_h = dts.build_index(D_pin.numpy(), device=local)
+    ts = []
+    d2h = 0
+    for i in range(max(1, args.e2e_steps) + 1):
+        barrier()
+        t0 = time.perf_counter()
+        res = dts.search(idx_h, Q_np[lo_e:hi_e], d, query_id_base=lo_e)
+        if world > 1:
+            dts_dist.global_offset(res.shape[0], rank, world)
+        t1 = time.perf_counter()
+        if i > 0:
+            ts.append(maxrank(t1 - t0))
+        d2h = res.nbytes
+        del res
+    e2e_s = statistics.median(ts)
+    tb = []
+    for i in range(2 if world == 1 else 0):
+        t0 = time.perf_counter()
+        ib = dts.build_index(D_pin.numpy(), device=local)
+        r = dts.search(ib, Q_np, d)
+        tb.append(time.perf_counter() - t0)
+        ib.free()
+        del r
+    idx_h.free()
 
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        v, cores, sample = oracle_rate(cfg, args.cpu_seconds, seed=42)
+        v, cores, sample, _ = oracle_rate(cfg, d, args.cpu_seconds, seed=42)
         cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample}
 
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_per_step,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None,
+            "search_time_s": ms_per_step * 1e-3,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
-            "config": {"workload": WORKLOADS.get(args.config, args.config), "name": args.config,
-                       "n_entries": int(n), "n_queries_per_rank": int(nq), "d": d,
-                       "step": "index build + query prep + count pass + scan + scatter pass + "
-                               "canonical sort (all SURVEY.md §8(a) rows), inputs resident in HBM",
-                       "l2": "flushed between steps (256 MiB write outside the timed events)",
-                       "parallelism": f"query-sharded x{world}, D replicated"},
-            "phases_ms": {"build": ms_build, "build_bounds": ph[0], "build_keys": ph[1],
-                          "build_sort": ph[2], "build_gather": ph[3], "build_insert": ph[4],
-                          "prep": statistics.mean(s["ms_prep"] for s in stats),
-                          "count_pass": ms_count, "scan": statistics.mean(s["ms_scan"] for s in stats),
-                          "scatter_pass": ms_scatter,
-                          "canon": statistics.mean(s["ms_canon"] for s in stats)},
-            "search_only": {"value": world * nq / ((ms_per_step - ms_build) * 1e-3), "unit": UNIT,
-                            "note": "step minus index build (the paper's response time excludes "
-                                    "the build, P:L135)"},
-            "work": {"candidates_per_pass": st0["candidates"], "cell_lookups": st0["cell_lookups"],
-                     "results_per_rank": results},
-            "roofline": {"bound": "hbm", "kernel": dom["kernel"], "achieved": dom["achieved_gbs"],
-                         "peak": peak, "unit": "GB/s", "frac": dom["frac"],
-                         "traffic": dom["traffic"], "peak_source": peak_src,
-                         "algorithmic_bytes": dom["bytes"], "ms": dom["ms"],
-                         "bytes_model": dom["bytes_model"],
-                         "note": "dominant kernel = largest device time of one step "
-                                 "(per-phase CUDA events); all kernels in roofline_kernels"},
-            "roofline_kernels": kern,
-            "roofline_search": {"bound": "hbm", "kernel": "k_wtile_count (pass 1: fused candidate "
-                                "streaming + fp64 refine)", "achieved": achieved, "peak": peak,
-                                "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
-                                "algorithmic_bytes": alg_bytes},
+            "config": config_dict(args.config, cfg, d),
+            "step": "query prep + candidate generation + count pass (streaming + fp64 refine) + "
+                    "scan + emission; index built once before timing (P:L135)"
+                    + ("" if world == 1 else "; per step: per-block candidate costs of an equal "
+                       "share of Q, all_gather of the costs, balanced contiguous query-id ranges, "
+                       "search, all_gather of the result counts"),
+            "parallelism": f"query-sharded x{world} (balanced by candidate counts), D and index "
+                           "replicated" if world > 1 else "one GPU",
+            "phases_ms": {"prep": ph["ms_prep"], "count_pass": ph["ms_count"],
+                          "scan": ph["ms_scan"], "emit_pass": ph["ms_scatter"],
+                          "overflow_sort": ph["ms_canon"]},
+            "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)],
+            "work": {"candidates": st0["candidates"], "offset_lookups": st0["cell_lookups"],
+                     "results": results, "queries_rank0": nq_rank},
+            "roofline": roofline,
+            "with_build": wb,
+            "index": {"n": build_info["n"], "cells": build_info["cells"],
+                      "bins": build_info["bins"], "grid": build_info["grid"],
+                      "hash_bytes": build_info["hash_bytes"], "ms_build_first": build_info["ms_build"]},
+            "points": points,
             "clocks": clk,
             "gpu_launches": int(launches),
-            "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": int(h2d),
-                    "d2h_bytes_per_step": int(d2h),
-                    "search_only_value": e2e_search,
-                    "note": "dts_build_index(host D) + dts_search(host Q) -> host results, "
-                            "wall clock, median of steps"},
+            "e2e": {"value": nq / e2e_s, "unit": UNIT,
+                    "h2d_bytes_per_step": int((hi_e - lo_e) * 64), "d2h_bytes_per_step": int(d2h),
+                    "search_time_s": e2e_s,
+                    "with_build_value": (nq / statistics.median(tb)) if tb else None,
+                    "note": "dts_search(host Q from pinned memory -> pinned host results), index "
+                            "resident, wall clock, median of steps (max over ranks); "
+                            "with_build_value adds dts_build_index(host D, 1.29 GB H2D)"},
             "wall_s_timed": wall,
         }
         if cpu is not None:
             line["cpu_baseline"] = cpu
         print(json.dumps(line), flush=True)
+    idx.free()
     if world > 1:
         dist.barrier()
         dist.destroy_process_group()
@@ -431,18 +515,22 @@ def run_own(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=100)
-    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="C4")
     ap.add_argument("--d", type=float, default=None)
     ap.add_argument("--impl", default="own", choices=["own", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=5)
+    ap.add_argument("--build-steps", type=int, default=10)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
     ap.add_argument("--ref-budget-seconds", type=float, default=150.0,
                     help="reference arm: oracle seconds for the whole run (per-step samples "
                          "shrink with --steps + --warmup)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-traffic", action="store_true")
+    ap.add_argument("--no-points", action="store_true")
+    ap.add_argument("--no-build-line", action="store_true")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

@@ -210,6 +210,24 @@ dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n
                                          void* cuda_stream,
                                          dts_traj_result** out_dev, size_t* out_count);
 
+/* Per-query candidate counts ("per-query candidate count
+ * estimate (for balancing)"; the partitioned search of P:L17 / P:L34 over
+ * independent queries).  For every query of Q_dev (nq segments in
+ * device memory of the index's device, 16-byte aligned) the candidate
+ * generation of the search (bins, stencil cells, row probes of the index) is
+ * run and the lengths of its candidate runs are summed: exactly the
+ * (query, entry) pairs dts_search at distance d would refine for it (the
+ * `candidates` statistic, per query).  No candidate record is read.
+ * costs_dev (device memory, ceil(nq / block) uint64, written, not
+ * accumulated) receives the sums over blocks of `block` consecutive queries
+ * (block = 1: per query).  A caller sharding Q over ranks splits the prefix
+ * sum of these costs evenly (dist.py).  Invalid query segments count 0 (the
+ * search reports them).  Errors: DTS_EINVAL (NULL with nq > 0, block == 0,
+ * bad d, nq >= 2^32, misaligned Q_dev), DTS_ECUDA.  Synchronous on return. */
+dts_status dts_query_costs_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                  double d, uint32_t block, void* cuda_stream,
+                                  uint64_t* costs_dev);
+
 /* Sort n results in device memory into canonical (query_id, entry_id) order,
  * in place (e.g. after concatenating the outputs of shards of D). */
 dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream);

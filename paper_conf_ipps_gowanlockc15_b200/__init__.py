@@ -32,6 +32,7 @@ EXPORTED_SYMBOLS = (
     "dts_search_device", "dts_free_results", "dts_free_results_device", "dts_free_index",
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
     "dts_search_device_ex", "dts_canonicalize_device", "dts_merge_trajectories_device",
+    "dts_query_costs_device",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -123,6 +124,8 @@ def load():
     lib.dts_merge_trajectories_device.argtypes = [P, S, P, S, P, S, P, pp, ps]
     lib.dts_merge_trajectories_device.restype = ctypes.c_int
     lib.dts_search_device_ex.restype = ctypes.c_int
+    lib.dts_query_costs_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, P]
+    lib.dts_query_costs_device.restype = ctypes.c_int
     lib.dts_canonicalize_device.argtypes = [P, S, P]
     lib.dts_canonicalize_device.restype = ctypes.c_int
     lib.dts_search_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
@@ -370,6 +373,23 @@ def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=
                                         ctypes.c_void_p(_stream_ptr(stream)),
                                         ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     return DeviceResults(out.value or 0, cnt.value, index.device), st.as_dict()
+
+
+def query_costs_device(index: Index, Q_dev, d: float, block: int = 1, stream=None, out=None):
+    """dts_query_costs_device: Q_dev CUDA tensor (nq, 8) float64 -> CUDA int64
+    tensor of ceil(nq / block) candidate counts (sum over each block of
+    `block` consecutive queries of the pairs the search would refine)."""
+    import torch
+    lib = load()
+    nq = int(Q_dev.shape[0])
+    nb = (nq + int(block) - 1) // int(block)
+    if out is None:
+        out = torch.empty(nb, dtype=torch.int64, device=Q_dev.device)
+    _check(lib.dts_query_costs_device(index.handle, ctypes.c_void_p(Q_dev.data_ptr() if nq else 0),
+                                      nq, float(d), int(block),
+                                      ctypes.c_void_p(_stream_ptr(stream)),
+                                      ctypes.c_void_p(out.data_ptr() if nb else 0)))
+    return out
 
 
 def merge_trajectories_device(results, query_traj, entry_traj, stream=None):

@@ -89,6 +89,13 @@ void cache_free(void* p) {
     c.cached[dev] += sz;
 }
 
+int cache_device(void* p) {
+    Cache& c = cache();
+    std::lock_guard<std::mutex> lk(c.mu);
+    auto it = c.live.find(p);
+    return it == c.live.end() ? -1 : it->second.first;
+}
+
 bool cache_owns(void* p) {
     Cache& c = cache();
     std::lock_guard<std::mutex> lk(c.mu);

@@ -103,9 +103,13 @@ void pinned_free(void* p) {
 
 void free_index_memory(dts_index* idx) {
     if (!idx) return;
+    DeviceGuard dg;
     cudaSetDevice(idx->device);
-    // blocks go back to the device cache (alloc.cu) for the next build
-    cudaDeviceSynchronize();
+    // blocks go back to the device cache (alloc.cu) for the next build: wait
+    // for the end of the build only (a build returns before its last kernels
+    // finish; searches are synchronous on return, so none is in flight),
+    // not for every stream of the device
+    if (idx->ready) cudaEventSynchronize(idx->ready);
     for (int i = 0; i < idx->nev; ++i) cudaEventDestroy(idx->ev[i]);
     idx->nev = 0;
     idx->ready = nullptr;
@@ -164,6 +168,7 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
                         bool host, cudaStream_t s, dts_index** out_index) {
     if (out_index) *out_index = nullptr;
     dts_index* idx = nullptr;
+    DeviceGuard dg;
     dts_status st = guarded([&] {
         if (!out_index) throw Error(DTS_EINVAL, "out_index is NULL");
         if (n > 0 && !D) throw Error(DTS_EINVAL, "D is NULL with n > 0");
@@ -370,6 +375,7 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
     const uint32_t* qtraj = opts ? opts->query_traj : nullptr;
     const bool excl = opts && opts->exclude_same_trajectory;
     if (opts) qid_base = opts->query_id_base;
+    DeviceGuard dg;
     dts_status st = guarded([&] {
         if (!index) throw Error(DTS_EINVAL, "index is NULL");
         if (!out_results || !out_count) throw Error(DTS_EINVAL, "output pointer is NULL");
@@ -510,6 +516,7 @@ dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n
     if (out_count) *out_count = 0;
     dts_traj_result* o = nullptr;
     size_t c = 0;
+    DeviceGuard dg;
     dts_status st = guarded([&] {
         if (!out_dev || !out_count) throw Error(DTS_EINVAL, "output pointer is NULL");
         if (n > 0 && (!results_dev || !query_traj || !entry_traj))
@@ -522,6 +529,25 @@ dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n
         *out_count = c;
     }
     return st;
+}
+
+dts_status dts_query_costs_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                  double d, uint32_t block, void* cuda_stream,
+                                  uint64_t* costs_dev) {
+    DeviceGuard dg;
+    return guarded([&] {
+        if (!index) throw Error(DTS_EINVAL, "index is NULL");
+        if (nq > 0 && (!Q_dev || !costs_dev)) throw Error(DTS_EINVAL, "NULL pointer with nq > 0");
+        if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
+        if (block == 0) throw Error(DTS_EINVAL, "block must be >= 1");
+        if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
+        prepare_device(index->device);
+        if (nq) check_aligned(Q_dev, "Q_dev");
+        const cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
+        query_costs_device(index, Q_dev, nq, d, block,
+                           reinterpret_cast<unsigned long long*>(costs_dev), s);
+        DTS_CUDA(cudaStreamSynchronize(s));
+    });
 }
 
 dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream) {
@@ -543,10 +569,16 @@ dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, s
 void dts_free_results(dts_result* results) { pinned_free(results); }
 
 void dts_free_results_device(void* results) {
-    if (results) {
-        cudaDeviceSynchronize();
-        cache_free(results);
-    }
+    if (!results) return;
+    // the block may still be read by work the caller enqueued on any stream
+    // of its device: wait for that device (not the caller's current one)
+    // before it is handed out again
+    const int dev = cache_device(results);
+    if (dev < 0) return;                      // not a library block
+    DeviceGuard dg;
+    cudaSetDevice(dev);
+    cudaDeviceSynchronize();
+    cache_free(results);
 }
 
 void dts_free_index(dts_index* index) {
@@ -558,6 +590,7 @@ void dts_free_index(dts_index* index) {
 dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
     return guarded([&] {
         if (!idx || !info) throw Error(DTS_EINVAL, "NULL argument");
+        DeviceGuard dg;
         cudaSetDevice(idx->device);
         index_times(const_cast<dts_index*>(idx));
         dts_index_info r{};

@@ -954,12 +954,22 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
             }
         }
     }
+    // a row's x-cells start at a multiple of 8 keys: nc[0] is rounded up to a
+    // multiple of 8 (the extra cells stay empty), so an 8-key hash block never
+    // straddles two rows or two bins.  A block holding more than 65535 entries
+    // is returned whole by a row probe (superset); if it could straddle rows,
+    // two probes of one query would return the same entries twice.
+    // (the temporal and subbin methods never probe cells: one cell per bin)
+    const bool grid = p.method == DTS_METHOD_GRID;
+    auto round8 = [grid](int32_t v) { return grid ? (int32_t)(((int64_t)v + 7) / 8 * 8) : v; };
+    g.nc[0] = round8(g.nc[0]);
     // keep the key space below 2^62: coarsen the finest axis until it fits
     while ((double)g.m * g.nc[0] * g.nc[1] * g.nc[2] >= 4.6e18) {
         int a = 0;
         for (int j = 1; j < 3; ++j) if (g.nc[j] > g.nc[a]) a = j;
         g.w[a] *= 2.0;
         g.nc[a] = (int32_t)std::floor((b.hi[a] - b.lo[a]) / g.w[a]) + 1;
+        if (a == 0) g.nc[0] = round8(g.nc[0]);
     }
     for (int a = 0; a < 3; ++a) g.inv_w[a] = 1.0 / g.w[a];
     g.cells_per_bin = (unsigned long long)g.nc[0] * g.nc[1] * g.nc[2];

@@ -311,6 +311,18 @@ unsigned long long* radix_sort_keys_hist(unsigned long long* keys, unsigned long
 // Device block cache (alloc.cu) for memory that outlives one API call.
 void* cache_alloc(size_t bytes);
 void cache_free(void* p);
+int cache_device(void* p);          // owning device of a live block, -1 if not ours
+
+// Saves the caller's current device and restores it on scope exit (every
+// entry point of the C ABI runs under one: the library switches to the
+// index's device, the caller's thread state is left as it was).
+struct DeviceGuard {
+    int prev = -1;
+    DeviceGuard() { if (cudaGetDevice(&prev) != cudaSuccess) { cudaGetLastError(); prev = -1; } }
+    ~DeviceGuard() { if (prev >= 0) cudaSetDevice(prev); }
+    DeviceGuard(const DeviceGuard&) = delete;
+    DeviceGuard& operator=(const DeviceGuard&) = delete;
+};
 
 }  // namespace dts
 
@@ -369,6 +381,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
                    unsigned long long max_results = ~0ull, const uint32_t* qmap = nullptr,
                    const uint32_t* qtraj = nullptr, bool exclude_same_traj = false);
+// Per-query candidate counts summed per block of `block` queries (search.cu).
+void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
+                        uint32_t block, unsigned long long* out, cudaStream_t s);
 // Trajectory-level merge (traj.cu); output in cache_alloc'd device memory.
 void merge_trajectories_device(const dts_result* r, size_t n, const uint32_t* qtraj,
                                size_t nqid, const uint32_t* etraj, size_t neid,

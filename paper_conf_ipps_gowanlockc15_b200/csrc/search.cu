@@ -581,6 +581,37 @@ __global__ void k_validate_only(const double4* __restrict__ Q, uint32_t nq, Coun
 
 inline unsigned blocks(size_t n, int per) { return (unsigned)((n + per - 1) / per); }
 
+// Per-query candidate counts ("per-query candidate count
+// estimate (for balancing)"): the stencil and its row probes exactly as in
+// pass 1, summing the run lengths -- the candidates pass 1 will refine --
+// without touching a record.  One thread per query; sums per block of
+// `block` consecutive queries.
+__global__ void __launch_bounds__(PT) k_query_costs(const double4* __restrict__ Q, uint32_t nq,
+                                                   double d, GridParams g, HashTable ht,
+                                                   const double* __restrict__ bin_t0min,
+                                                   const double* __restrict__ bin_t1max,
+                                                   const uint32_t* __restrict__ bin_start,
+                                                   uint32_t method, SubbinIndex sb,
+                                                   uint32_t block,
+                                                   unsigned long long* __restrict__ out) {
+    const uint32_t i = blockIdx.x * PT + threadIdx.x;
+    if (i >= nq) return;
+    QState q;
+    double qlo[3], qhi[3];
+    const bool live = load_query(Q, i, q, qlo, qhi);
+    const Stencil st = make_stencil(g, q, qlo, qhi, d, live, bin_start, bin_t0min, bin_t1max,
+                                    method, sb);
+    unsigned long long c = 0;
+    uint32_t probes = 0;
+    for (uint32_t l = 0; l < st.nlook; ++l) {
+        uint32_t s0 = 0, cnt = 0;
+        resolve(g, ht, bin_t0min, bin_t1max, bin_start, st.mode, st.lb, st.hb, st.clo, st.cn,
+                q.t0, q.t1, l, st.rstart, st.rcnt, s0, cnt, probes);
+        c += cnt;
+    }
+    if (c) atomicAdd(&out[i / block], c);
+}
+
 struct EventTimer {
     bool on;
     cudaStream_t s;
@@ -877,6 +908,20 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         local.ms_canon = tm.ms(4);
     }
     if (stats) *stats = local;
+}
+
+void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
+                        uint32_t block, unsigned long long* out, cudaStream_t s) {
+    if (block == 0) throw Error(DTS_EINVAL, "block must be >= 1");
+    const size_t nb = (nq + block - 1) / block;
+    if (nb) DTS_CUDA(cudaMemsetAsync(out, 0, nb * sizeof(unsigned long long), s));
+    if (nq == 0 || idx->n == 0) return;
+    if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));
+    k_query_costs<<<blocks(nq, PT), PT, 0, s>>>(reinterpret_cast<const double4*>(Q_dev),
+                                                (uint32_t)nq, d, idx->gp, idx->ht,
+                                                idx->bin_t0min, idx->bin_t1max, idx->bin_start,
+                                                idx->method, idx->sb, block, out);
+    DTS_LAUNCH_CHECK();
 }
 
 namespace {

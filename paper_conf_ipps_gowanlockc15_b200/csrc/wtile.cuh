@@ -432,10 +432,14 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 for (uint32_t i = lane; i < nh; i += 32) {
                     const unsigned long long k = S.hkey[i];
                     const uint32_t q = (uint32_t)(k >> 42), e = (uint32_t)(k >> 10);
+                    // rank inside the query: hits with a smaller entry id,
+                    // ties (equal caller ids) broken by stage slot, so every
+                    // slot of the tile's range is written exactly once
                     uint32_t rank = 0;
                     for (uint32_t j = 0; j < nh; ++j) {
                         const unsigned long long kj = S.hkey[j];
-                        rank += ((uint32_t)(kj >> 42) == q && (uint32_t)(kj >> 10) < e) ? 1u : 0u;
+                        const uint32_t ej = (uint32_t)(kj >> 10);
+                        rank += ((uint32_t)(kj >> 42) == q && (ej < e || (ej == e && j < i))) ? 1u : 0u;
                     }
                     const uint32_t slot = (uint32_t)(k & 1023ull);
                     dts_result r;

@@ -68,6 +68,74 @@ def search_sharded(search_fn, Q, d: float, rank: int, world: int, group=None, we
     return res, off, total
 
 
+def _comm_device(group=None):
+    import torch
+    import torch.distributed as dist
+    if dist.get_backend(group) == "nccl":
+        return torch.device("cuda", torch.cuda.current_device())
+    return torch.device("cpu")
+
+
+def block_split(nblocks: int, world: int):
+    """Equal split of `nblocks` cost blocks over ranks (block indices)."""
+    return [nblocks * r // world for r in range(world + 1)]
+
+
+def balanced_query_bounds(idx, Q_dev, d: float, rank: int, world: int, group=None,
+                          block: int = 256, stream=None, costs_fn=None):
+    """Query-id bounds [b[r], b[r+1]) of every rank, balanced by the
+    candidate counts of the search (dts_query_costs_device, SURVEY.md
+    §8(a4)/(e)).  Each rank costs an equal share of Q's blocks of `block`
+    queries (so the estimate itself is sharded); the per-block sums are
+    all-gathered (8 bytes per block) and every rank cuts the same prefix
+    sum at total * r / world.  Returns the bounds list (query ids, multiples
+    of `block` except the last) on every rank.  costs_fn(lo, hi) replaces the
+    library call (CPU tests of the exchange)."""
+    import torch
+    import torch.distributed as dist
+
+    nq = int(Q_dev.shape[0])
+    nb = (nq + block - 1) // block
+    if world == 1:
+        return [0, nq]
+    eb = block_split(nb, world)
+    lo, hi = eb[rank] * block, min(nq, eb[rank + 1] * block)
+    if costs_fn is None:
+        import paper_conf_ipps_gowanlockc15_b200 as dts
+        mine = dts.query_costs_device(idx, Q_dev[lo:hi], d, block=block, stream=stream)
+    else:
+        mine = costs_fn(lo, hi)
+    width = max(eb[r + 1] - eb[r] for r in range(world))
+    cdev = _comm_device(group)
+    pad = torch.zeros(width, dtype=torch.int64, device=cdev)
+    pad[:mine.numel()] = mine.to(cdev)
+    parts = [torch.zeros_like(pad) for _ in range(world)]
+    dist.all_gather(parts, pad, group=group)
+    costs = np.concatenate([parts[r][:eb[r + 1] - eb[r]].cpu().numpy() for r in range(world)])
+    bb = shard_bounds(nb, world, weights=costs)
+    return [min(nq, x * block) for x in bb]
+
+
+def search_strong(idx, Q_dev, d: float, rank: int, world: int, group=None, block: int = 256,
+                  stream=None, bounds=None, time_kernels: bool = False):
+    """One strong-scaling search step: the one query set
+    Q_dev (resident on every rank, as is the index) is split into contiguous
+    query-id ranges balanced by candidate counts (or by `bounds` if given),
+    this rank searches its range with global query ids, and the per-rank
+    result counts are all-gathered (the only exchange of the search).
+    Returns (DeviceResults, search stats, (lo, hi), offset of this rank's
+    slice in the global canonical result, global total)."""
+    import paper_conf_ipps_gowanlockc15_b200 as dts
+    if bounds is None:
+        bounds = balanced_query_bounds(idx, Q_dev, d, rank, world, group, block, stream)
+    lo, hi = bounds[rank], bounds[rank + 1]
+    res, st = dts.search_device(idx, Q_dev[lo:hi], d, query_id_base=lo, stream=stream,
+                                time_kernels=time_kernels)
+    off, total, _ = global_offset(res.count, rank, world, group=group,
+                                  device=_comm_device(group) if world > 1 else None)
+    return res, st, (lo, hi), off, total
+
+
 # --------------------------------------------------------------------------
 # Fallback when D exceeds one GPU's HBM (SURVEY.md §8(e)): shard D by
 # t_start range.  Rank r holds the entries with t_start in [T_r, T_{r+1});
@@ -107,31 +175,40 @@ def route_queries(Q, T, maxdur, rank: int):
 
 
 def gather_to_root(local, rank: int, world: int, group=None):
-    """All-gather variable-length uint8 tensors (padded to the largest);
-    returns the concatenation in rank order on rank 0, None elsewhere."""
+    """Variable-length uint8 tensors to rank 0: the sizes are all-gathered
+    (8 bytes per rank), then every rank sends exactly its bytes to rank 0
+    (point to point), so no rank holds more than its own slice except the
+    root.  Returns the concatenation in rank order on rank 0, None elsewhere."""
     import torch
     import torch.distributed as dist
     n = torch.tensor([local.numel()], dtype=torch.int64, device=local.device)
     sizes = [torch.zeros_like(n) for _ in range(world)]
     dist.all_gather(sizes, n, group=group)
     sizes = [int(s.item()) for s in sizes]
-    mx = max(sizes) if sizes else 0
-    pad = torch.zeros(mx, dtype=torch.uint8, device=local.device)
-    pad[:local.numel()] = local
-    parts = [torch.zeros_like(pad) for _ in range(world)]
-    dist.all_gather(parts, pad, group=group)
     if rank != 0:
+        if sizes[rank]:
+            dist.send(local.contiguous(), dst=0, group=group)
         return None
-    return torch.cat([p[:s] for p, s in zip(parts, sizes)])
+    parts = [local]
+    for r in range(1, world):
+        buf = torch.empty(sizes[r], dtype=torch.uint8, device=local.device)
+        if sizes[r]:
+            dist.recv(buf, src=r, group=group)
+        parts.append(buf)
+    return torch.cat(parts)
 
 
 def search_temporal_sharded(D, Q, d: float, rank: int, world: int, group=None,
-                            method: str = "grid", device: int = 0):
-    """Temporal-range sharding of D over `world` GPUs (one rank each).
-    Returns the canonical global results (numpy) on rank 0, None elsewhere."""
+                            method: str = "grid", device=None):
+    """Temporal-range sharding of D over `world` GPUs (one rank each; device
+    defaults to the rank's current CUDA device, i.e. LOCAL_RANK under a
+    one-process-per-GPU launch).  Returns the canonical global results
+    (numpy) on rank 0, None elsewhere."""
     import torch
 
     import paper_conf_ipps_gowanlockc15_b200 as dts
+    if device is None:
+        device = torch.cuda.current_device()
     T, rows, maxdur = temporal_partition(D, world)
     dev = torch.device("cuda", device)
     mine = rows[rank]
@@ -145,8 +222,11 @@ def search_temporal_sharded(D, Q, d: float, rank: int, world: int, group=None,
     local = res.tensor().clone()
     res.free()
     idx.free()
+    if _comm_device(group).type == "cpu":
+        local = local.cpu()
     allres = gather_to_root(local, rank, world, group)
     if allres is None:
         return None
+    allres = allres.to(dev)
     dts.canonicalize_device(allres)
     return allres.cpu().numpy().view(dts.RESULT_DTYPE)

@@ -13,6 +13,11 @@ muts=(
  's/hi = tau2 < 1.0 ? tau2 : 1.0;/hi = tau2;/'
  's/\*t_e = (1.0 - hi) \* ts + hi \* te;/*t_e = (1.0 - hi) * ts + hi * ts;/'
  's/position_at(q, \*te, pq);/position_at(q, *ts, pq);/'
+ 's/tau = -beta \/ a;/tau = beta \/ a;/'
+ 's/if (tau > 1.0) tau = 1.0;//'
+ 's/double x = A\[0\] + tau \* V\[0\], y = A\[1\] + tau \* V\[1\]/double x = A[0] + tau * V[0], y = A[1] + tau * V[0]/'
+ 's/\*dmin = sqrt(x \* x + y \* y + z \* z);/*dmin = x * x + y * y + z * z;/'
+ 's/if (tau < 0.0) tau = 0.0;//'
 )
 rc=0
 for m in "${muts[@]}"; do

@@ -37,3 +37,18 @@ m = dts.merge_trajectories_device(res, torch.from_numpy(c.qtraj).cuda(),
 t = res.tensor().clone()
 dts.canonicalize_device(t)
 print("sanitize workload ok", r.shape[0], res.count, m.count, flush=True)
+# crowded hash blocks (> 65,535 entries in one 8-cell block, warp-path
+# inserts) plus one long segment (coarse cells, multi-row stencils)
+D, Q = synth.crowded(5)
+D = np.concatenate([D, [[0.0, 0.05, 0.5, 0.5, 1.0, 0.95, 0.52, 0.5]]])
+idx = dts.build_index(D)
+r2 = dts.search(idx, Q, 0.01)
+idx.free()
+# a multi-tile onesweep sort (look-back across tiles) and the cost kernel
+c1 = synth.make_config("C1", scale=0.1)
+idx = dts.build_index_device(torch.from_numpy(c1.D).cuda())
+Q1 = torch.from_numpy(c1.Q).cuda()
+res1, _ = dts.search_device(idx, Q1, 0.02)
+costs = dts.query_costs_device(idx, Q1, 0.02, block=64)
+torch.cuda.synchronize()
+print("sanitize workload 2 ok", r2.shape[0], res1.count, int(costs.sum()), flush=True)

@@ -1,11 +1,12 @@
 """Parity rule (BASELINE.json north_star; readings c11, c10):
 
 * the result pair set must equal the oracle's, except pairs whose minimum
-  distance (computed by the oracle's routine) lies within 1e-9*d of d, plus
-  the fp64 rounding floor 1e-12*L of a distance computed from coordinates of
-  magnitude L = max |coordinate| (reading c11: without the floor the band is
-  empty at d = 0, where a pair that touches at one instant is a rounding
-  decision of either implementation);
+  distance (computed by the oracle's routine, pinned in tests/test_oracle.py)
+  lies within 1e-9*d of d -- exactly the north star's band for every d > 0.
+  At d = 0 that band is empty; there, and only there, the band is the fp64
+  rounding floor 1e-12*L of a distance computed from coordinates of magnitude
+  L = max |coordinate| (reading c11: a pair that touches at one instant is a
+  rounding decision of either implementation);
 * interval endpoints of common pairs agree within 1e-9 in normalised time
   t^ = (t - t_min(D)) / (t_max(D) - t_min(D));
 * results are in canonical (query_id, entry_id) order with no duplicates.
@@ -17,12 +18,17 @@ FLOOR = 1e-12
 TOL_T = 1e-9
 
 
+SUMMARY = []          # one dict per compare() call (written by conftest at session end)
+
+
 def band(D, Q, d):
+    if d > 0:
+        return BAND * d
     Dv = np.asarray(D).reshape(-1, 8)[:, [1, 2, 3, 5, 6, 7]]
     Qv = np.asarray(Q).reshape(-1, 8)[:, [1, 2, 3, 5, 6, 7]]
     L = max(float(np.abs(Dv).max()) if Dv.size else 0.0,
             float(np.abs(Qv).max()) if Qv.size else 0.0)
-    return BAND * d + FLOOR * L
+    return FLOOR * L
 
 
 def keys(res) -> np.ndarray:
@@ -64,9 +70,11 @@ def compare(gpu, ora, D, Q, d, oracle_mod, qid_base=0, tol_t=TOL_T):
         assert worst <= tol_t, f"endpoint error {worst} in normalised time > {tol_t}"
     else:
         worst = 0.0
-    return {"gpu": int(kg.size), "oracle": int(ko.size), "common": int(common.size),
+    info = {"gpu": int(kg.size), "oracle": int(ko.size), "common": int(common.size),
             "band_only_gpu": int(only_g.size), "band_only_oracle": int(only_o.size),
-            "worst_endpoint": worst}
+            "worst_endpoint": worst, "d": float(d), "band": float(band(D, Q, d))}
+    SUMMARY.append(info)
+    return info
 
 
 def restrict(res, qids):

@@ -130,3 +130,48 @@ def test_temporal_partition_properties():
         for r in range(world):
             t0 = c.D[rows[r], 0]
             assert np.all(t0 >= T[r]) and np.all(t0 < T[r + 1])
+
+
+def _balance_worker(rank, world, port, out_dir):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    nq, block = 1000, 16
+    # skewed per-query costs: the first fifth of the queries is 20x heavier
+    per = np.where(np.arange(nq) < nq // 5, 20, 1).astype(np.int64)
+
+    def costs_fn(lo, hi):
+        # blocks of `block` queries, as dts_query_costs_device(block=16) returns
+        p = per[lo:hi]
+        nb = (p.size + block - 1) // block
+        p = np.pad(p, (0, nb * block - p.size))
+        return torch.from_numpy(p.reshape(nb, block).sum(1))
+
+    Q = torch.zeros((nq, 8), dtype=torch.float64)
+    b = dts_dist.balanced_query_bounds(None, Q, 0.1, rank, world, block=block, costs_fn=costs_fn)
+    with open(os.path.join(out_dir, f"b{rank}.txt"), "w") as f:
+        f.write(" ".join(map(str, b)))
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_balanced_bounds_exchange(tmp_path):
+    """Strong-scaling split: each rank costs an equal share
+    of the query blocks, the per-block costs are all-gathered, and every rank
+    computes the same balanced contiguous bounds (block-aligned), which put
+    about half of the total cost on each rank."""
+    import torch.multiprocessing as mp
+    world = 2
+    mp.spawn(_balance_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    bs = [list(map(int, open(tmp_path / f"b{r}.txt").read().split())) for r in range(world)]
+    assert bs[0] == bs[1]
+    b = bs[0]
+    assert b[0] == 0 and b[-1] == 1000 and b[1] % 16 == 0
+    per = np.where(np.arange(1000) < 200, 20, 1)
+    half = per.sum() / 2
+    assert abs(per[:b[1]].sum() - half) <= 16 * 20      # within one block of the cut
+    assert b[1] < 500                                    # far from the equal-count split

@@ -1,0 +1,195 @@
+"""GPU tests of the C ABI's contract beyond the result set: duplicate-free
+output with crowded hash blocks under coarse cells, non-distinct caller
+entry ids, concurrent searches on two streams, the per-query candidate costs
+(dts_query_costs_device), and the multi-rank paths (strong query sharding
+and temporal sharding of D) running libdts in two processes on one GPU."""
+import os
+import socket
+import threading
+
+import numpy as np
+import pytest
+
+import synth
+import dts_parity as parity
+
+pytestmark = pytest.mark.gpu
+
+THREADS = max(1, min(32, os.cpu_count() or 1))
+
+
+@pytest.fixture(scope="module")
+def dts():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import paper_conf_ipps_gowanlockc15_b200 as m
+    m.load()
+    return m
+
+
+def test_crowded_block_with_long_segment_no_duplicates(dts, oracle_mod):
+    """A block of 8 cells with > 65,535 entries is returned whole by a row
+    probe.  One spatially long segment makes the cells coarse and every
+    stencil several rows tall; the x-cells per row are a multiple of 8, so a
+    block never straddles two rows and no entry comes back twice (canonical,
+    duplicate-free output, reading c7)."""
+    D, Q = synth.crowded(5)
+    D = np.concatenate([D, [[0.0, 0.05, 0.5, 0.5, 1.0, 0.95, 0.52, 0.5]]])
+    for d in (0.01, 0.05):
+        idx = dts.build_index(D)
+        inf = idx.info()
+        assert inf["grid"][0] % 8 == 0
+        got = dts.search(idx, Q, d)
+        idx.free()
+        parity.assert_canonical(got)          # strictly increasing keys: no duplicates
+        ora = oracle_mod.search(D, Q, d, threads=THREADS)
+        info = parity.compare(got, ora, D, Q, d, oracle_mod)
+        assert info["common"] > 100000
+
+
+def test_non_distinct_entry_ids(dts, oracle_mod):
+    """Caller entry ids need not be distinct (e.g. a per-trajectory segment
+    number): every result is still reported once, with its interval, and no
+    stage slot is left unwritten (staged ranks break ties by slot)."""
+    c = synth.make_config("C2", scale=0.004)
+    ids = (np.arange(c.D.shape[0]) // 3).astype(np.uint32)
+    d = 2.0
+    idx = dts.build_index(c.D, entry_ids=ids)
+    got = dts.search(idx, c.Q, d)
+    idx.free()
+    ora = oracle_mod.search(c.D, c.Q, d, threads=THREADS)
+    ora["entry_id"] = ids[ora["entry_id"]]
+    assert got.shape == ora.shape
+
+    def canon(a):
+        return np.sort(a, order=["query_id", "entry_id", "t_start", "t_end"])
+    g, o = canon(got), canon(ora)
+    assert np.array_equal(g["query_id"], o["query_id"])
+    assert np.array_equal(g["entry_id"], o["entry_id"])
+    span = float(c.D[:, 4].max() - c.D[:, 0].min())
+    assert np.max(np.abs(g["t_start"] - o["t_start"])) / span < 1e-9
+    assert np.max(np.abs(g["t_end"] - o["t_end"])) / span < 1e-9
+    # non-decreasing (query, entry id) order
+    k = got["query_id"].astype(np.uint64) << np.uint64(32) | got["entry_id"].astype(np.uint64)
+    assert np.all(k[1:] >= k[:-1])
+
+
+def test_concurrent_searches_two_streams(dts):
+    """An index is immutable after build: two host threads searching it at
+    once, each on its own stream, get the bytes of sequential searches."""
+    import torch
+    c = synth.make_config("C2", scale=0.02)
+    idx = dts.build_index(c.D)
+    Qa, Qb = c.Q, np.ascontiguousarray(c.Q[::-1])
+    ref_a = dts.search(idx, Qa, 2.0).tobytes()
+    ref_b = dts.search(idx, Qb, 0.5).tobytes()
+    Qa_d, Qb_d = torch.from_numpy(Qa).cuda(), torch.from_numpy(Qb).cuda()
+    out = {}
+    errs = []
+
+    def run(name, Qh, Qd, d):
+        try:
+            s = torch.cuda.Stream()
+            for k in range(4):
+                if k % 2 == 0:
+                    out[(name, k)] = dts.search(idx, Qh, d, stream=s).tobytes()
+                else:
+                    with torch.cuda.stream(s):
+                        res, _ = dts.search_device(idx, Qd, d, stream=s)
+                        out[(name, k)] = res.numpy().tobytes()
+                        res.free()
+        except Exception as e:          # surfaced below
+            errs.append(e)
+
+    ta = threading.Thread(target=run, args=("a", Qa, Qa_d, 2.0))
+    tb = threading.Thread(target=run, args=("b", Qb, Qb_d, 0.5))
+    ta.start(); tb.start(); ta.join(); tb.join()
+    assert not errs, errs
+    for k in range(4):
+        assert out[("a", k)] == ref_a, k
+        assert out[("b", k)] == ref_b, k
+    idx.free()
+
+
+def test_query_costs_match_candidates(dts):
+    """dts_query_costs_device sums, per block of queries, exactly the
+    candidate pairs the search refines (its `candidates` statistic)."""
+    import torch
+    for name, scale, d in (("C1", 0.2, 0.005), ("C2", 0.01, 2.0), ("C3", 0.02, 5.0)):
+        c = synth.make_config(name, scale=scale)
+        for method in ("grid", "subbin", "temporal"):
+            idx = dts.build_index_device(torch.from_numpy(c.D).cuda(), method=method)
+            Qd = torch.from_numpy(c.Q).cuda()
+            res, st = dts.search_device(idx, Qd, d)
+            per = dts.query_costs_device(idx, Qd, d, block=1)
+            blk = dts.query_costs_device(idx, Qd, d, block=100)
+            assert int(per.sum()) == st["candidates"], (name, method)
+            assert blk.numel() == (c.Q.shape[0] + 99) // 100
+            ref = torch.nn.functional.pad(per, (0, blk.numel() * 100 - per.numel()))
+            assert torch.equal(ref.view(-1, 100).sum(1), blk)
+            # sub-ranges: the costs of rows [a, b) alone
+            a, b = c.Q.shape[0] // 3, c.Q.shape[0] // 2
+            assert torch.equal(dts.query_costs_device(idx, Qd[a:b], d), per[a:b])
+            res.free()
+            idx.free()
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _rank_worker(rank, world, port, out_dir):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_ipps_gowanlockc15_b200 as dts
+    from paper_conf_ipps_gowanlockc15_b200 import dist as dts_dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    torch.cuda.set_device(0)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    c = synth.make_config("C2", scale=0.01)
+    d = 2.0
+    idx = dts.build_index_device(torch.from_numpy(c.D).cuda())
+    Qd = torch.from_numpy(c.Q).cuda()
+    res, st, (lo, hi), off, total = dts_dist.search_strong(idx, Qd, d, rank, world, block=64)
+    np.save(os.path.join(out_dir, f"strong{rank}.npy"), res.numpy())
+    with open(os.path.join(out_dir, f"strong{rank}.txt"), "w") as f:
+        f.write(f"{lo} {hi} {off} {total}")
+    res.free()
+    idx.free()
+    tmp = dts_dist.search_temporal_sharded(c.D, c.Q, d, rank, world)
+    if rank == 0:
+        np.save(os.path.join(out_dir, "temporal.npy"), tmp)
+    dist.barrier()
+    dist.destroy_process_group()
+
+
+def test_multirank_libdts_on_one_gpu(dts, tmp_path):
+    """Two ranks (gloo) running libdts on the same GPU: the strong query
+    sharding (balanced by dts_query_costs_device, counts all-gathered) placed
+    at the gathered offsets, and the temporal sharding of D gathered on rank 0,
+    both give the unsharded search's bytes."""
+    import torch.multiprocessing as mp
+    world = 2
+    mp.spawn(_rank_worker, args=(world, _free_port(), str(tmp_path)), nprocs=world, join=True)
+    c = synth.make_config("C2", scale=0.01)
+    idx = dts.build_index(c.D)
+    ref = dts.search(idx, c.Q, 2.0)
+    idx.free()
+    out = np.empty(ref.shape[0], dtype=ref.dtype)
+    prev_hi = 0
+    for r in range(world):
+        part = np.load(tmp_path / f"strong{r}.npy")
+        lo, hi, off, total = map(int, open(tmp_path / f"strong{r}.txt").read().split())
+        assert lo == prev_hi and total == ref.shape[0]
+        prev_hi = hi
+        out[off:off + part.shape[0]] = part
+    assert prev_hi == c.Q.shape[0]
+    assert out.tobytes() == ref.tobytes()
+    assert np.load(tmp_path / "temporal.npy").tobytes() == ref.tobytes()

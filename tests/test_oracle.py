@@ -187,6 +187,60 @@ def test_bruteforce_independent_minimum(oracle_mod):
     assert np.all(np.diff(keys) > 0)
 
 
+def test_dmin_independent_minimum(oracle_mod):
+    """The tie-band distance (oracle_dmin, reading c11) against an independent
+    golden-section minimum of |Delta(t)| over the strict overlap, on >= 300
+    random pairs (with overlap), plus NaN for pairs without overlap."""
+    D, Q = synth.random_small(21, 700, 700, side=0.6, tspan=1.5, maxdur=1.0, maxlen=0.4)
+    qids = np.arange(700)
+    eids = (np.arange(700) * 7) % 700
+    dm = oracle_mod.dmin_pairs(D, Q, qids, eids)
+    checked = interior = 0
+    for i in range(700):
+        q, l = Q[qids[i]], D[eids[i]]
+        ov = overlap(q, l)
+        if ov is None:
+            assert np.isnan(dm[i]), i
+            continue
+        ref, tm = golden_min(q, l, *ov)
+        assert abs(dm[i] - ref) <= 1e-9 * max(1.0, ref), (i, dm[i], ref)
+        checked += 1
+        interior += ov[0] + 1e-6 < tm < ov[1] - 1e-6
+    assert checked >= 300 and interior >= 50
+
+
+def test_dmin_hand_worked(oracle_mod):
+    """d_min of the hand-worked pairs (tests/golden/pairs.json): the closest
+    approach over the common time span, worked out from the geometry."""
+    spec = {p["id"]: p for p in json.load(open(os.path.join(GOLDEN, "pairs.json")))["pairs"]}
+    want = {
+        "P1": 0.05,        # parallel, 0.05 apart the whole time
+        "P2": 0.2,         # parallel, 0.2 apart
+        "P3": 0.0,         # crossing paths meet at t = 0.5
+        "P4": 0.25,        # tangent: closest at t = 0.5, distance 0.25
+        "P7": 0.0,         # head-on, meet at t = 0.5
+        "P8": 0.0,         # q passes the stationary l at t = 0.2
+        "P10": 0.0,        # same line, same place over [0.5, 1]
+        "P12": 0.0,        # q reaches x = 0.95 at t = 0.95
+        "P13": 0.0,        # 3-D: diff = (2 - 2t, 0, 0), zero at t = 1
+    }
+    for pid, exp in want.items():
+        p = spec[pid]
+        got = oracle_mod.dmin_pairs(np.array([p["l"]]), np.array([p["q"]]), [0], [0])[0]
+        assert got == pytest.approx(exp, abs=1e-15), pid
+    for pid in ("P5", "P6"):                       # no strict overlap
+        p = spec[pid]
+        assert np.isnan(oracle_mod.dmin_pairs(np.array([p["l"]]), np.array([p["q"]]), [0], [0])[0])
+    # closest approach after the overlap ends (upper clamp) and before it starts
+    q = [0.0, 0.0, 0.0, 0.0, 1.0, 1.0, 0.0, 0.0]
+    l_after = [0.0, 3.0, 0.5, 0.0, 1.0, 2.5, 0.5, 0.0]     # gap 3 -> 1.5 in x, 0.5 in y
+    assert oracle_mod.dmin_pairs(np.array([l_after]), np.array([q]), [0], [0])[0] == \
+        pytest.approx(math.hypot(1.5, 0.5), abs=1e-15)
+    l_before = [0.0, -1.0, 0.0, 0.25, 1.0, -1.5, 0.0, 0.25]  # moving away from the start
+    assert oracle_mod.dmin_pairs(np.array([l_before]), np.array([q]), [0], [0])[0] == \
+        pytest.approx(math.hypot(1.0, 0.25), abs=1e-15)
+
+
 # ---- invariants ------------------------------------------------------------
 
 def _as_dict(res):
