@@ -301,6 +301,11 @@ def run_own(args):
         if world > 1:
             dist.barrier()
 
+    # clocks sampled over every timed region of the run (the headline's alone
+    # lasts ~20 ms, shorter than nvidia-smi's 100 ms sampling period)
+    clocks = ClockSampler(local)
+    clocks.start()
+
     # ---- the index: built once, outside the timed search
     idx = dts.build_index_device(D_dev, device=local, stream=stream)
     build_info = idx.info()
@@ -337,7 +342,7 @@ def run_own(args):
             e1.record(stream)
             evs.append((e0, e1))
             flush.zero_()
-            outs.append(r[1:])
+            outs.append(r[1:] if after is None else after(r))
             cnt = r[0].count
             r[0].free()
         barrier()
@@ -347,13 +352,10 @@ def run_own(args):
 
     # ---- headline: search of the whole query set, index resident
     barrier()
-    clocks = ClockSampler(local)
-    clocks.start()
     wall0 = time.perf_counter()
     ms_per_step, step_ms, outs, results, launches = timed(lambda: search_step(d), args.steps,
                                                           args.warmup)
     wall = time.perf_counter() - wall0
-    clk = clocks.stop()
     value = nq / (ms_per_step * 1e-3)
     stats = [o[0] for o in outs]
     lo, hi = outs[-1][1]
@@ -412,12 +414,13 @@ def run_own(args):
             i2 = dts.build_index_device(D_dev, device=local, stream=stream)
             r = search_step(d)
             return r[0], (r[1], i2), r[2]
-        bms, _, bouts, _, _ = timed(build_step, args.build_steps, 2,
-                                    after=lambda r: r[1][1].free())
-        infs = []
-        for (s_, i2), _r in bouts:
-            infs.append(i2.info())
+
+        def build_after(r):          # outside the events: phase times, free the index
+            i2 = r[1][1]
+            inf = i2.info()
             i2.free()
+            return inf
+        bms, _, infs, _, _ = timed(build_step, args.build_steps, 2, after=build_after)
         bph = [statistics.mean(i["ms_phase"][k] for i in infs) for k in range(5)]
         bbuild = statistics.mean(i["ms_build"] for i in infs)
         wb = {"value": nq / (bms * 1e-3), "ms_per_step": bms, "ms_build": bbuild,
@@ -425,6 +428,9 @@ def run_own(args):
                                   "gather": bph[3], "insert": bph[4]},
               "note": "index build (bounds, keys, radix sort, gather, hash insert) + the "
                       "search, per step; every rank builds the replicated index"}
+
+    clk = clocks.stop()
+    clk["window"] = "from the index build through the with_build steps (all device work)"
 
     # ---- e2e through the C ABI host entry point (pinned host Q and results)
     Q_np = Q_pin.numpy()

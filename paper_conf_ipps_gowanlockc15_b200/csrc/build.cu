@@ -648,8 +648,6 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
     if (threadIdx.x == 0 && sm.s_cnt) {         // count[0]: cells, count[1]: blocks of 8 keys
         atomicAdd(count, (unsigned long long)sm.s_cnt);
         atomicAdd(count + 1, (unsigned long long)sm.s_blk);
-        sm.s_cnt = 0;
-        sm.s_blk = 0;
     }
 }
 

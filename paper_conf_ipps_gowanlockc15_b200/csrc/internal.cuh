@@ -354,6 +354,9 @@ struct dts_index {
     double4* sb_rec[3] = {nullptr, nullptr, nullptr};      // records of ids, per dimension
     uint64_t sb_len[3] = {0, 0, 0};
     uint32_t* etraj = nullptr;     // trajectory id per sorted position (optional)
+    // spill-buffer size hint (records): the largest output a search of this
+    // index has produced after its spill buffer filled (search.cu)
+    mutable std::atomic<unsigned long long> spill_hint{0};
 };
 
 namespace dts {

@@ -50,11 +50,14 @@ struct Counters {                       // device-side statistics / flags
     unsigned long long candidates;
     unsigned long long lookups;
     unsigned long long staged;          // staging slots reserved
+    unsigned long long spilled;         // spill slots reserved (may exceed the buffer)
+    unsigned long long spill_valid;     // first spill slot not written (~0: all written)
     unsigned int max_count;
-    unsigned int n_over;                // tiles recomputed in pass 2
+    unsigned int n_over;                // tiles re-run (spill buffer full)
+    unsigned int n_spill;               // tiles whose hits were spilled
+    unsigned int n_big;                 // spilled queries longer than a CTA sort
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
-    unsigned int pad;
 };
 
 // Query in the velocity form used by the refinement.
@@ -426,108 +429,10 @@ __global__ void __launch_bounds__(PT) k_unpack_order(const unsigned long long* _
 // ------------------------------------------------------------- block helpers
 #include "wtile.cuh"
 
-// -------------------------------- fallback: warp-per-query scatter (pass 2)
-struct PassArgs {
-    const double4* Q;
-    const uint32_t* order;
-    uint32_t nq;
-    double d;
-    GridParams g;
-    SegSoA soa;
-    HashTable ht;
-    const double* bin_t0min;
-    const double* bin_t1max;
-    const uint32_t* bin_start;
-    const unsigned long long* offsets;
-    const uint32_t* tiles;         // tiles to process (TQ sorted positions each)
-    dts_result* out;
-    uint32_t qid_base;
-    uint32_t method;
-    SubbinIndex sb;
-    const uint32_t* etraj;
-    const uint32_t* qtraj;
-    uint32_t excl;
-};
-
-// Warp w of CTA b processes sorted position tiles[b / (TQ/PW)]*TQ + ...; the
-// warp's lanes probe 32 stencil cells at a time, a warp scan flattens the
-// runs, lanes stream 32 candidates at a time and write hits at the query's
-// exact offset + ballot rank (deterministic order, sorted afterwards).
-__global__ void __launch_bounds__(PT) k_pass_scatter(const PassArgs a) {
-    __shared__ uint32_t s_start[PW][32];
-    __shared__ uint32_t s_excl[PW][32];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    constexpr int CTAS_PER_TILE = TQ / PW;
-    const uint32_t tile = a.tiles[blockIdx.x / CTAS_PER_TILE];
-    const uint32_t sq = tile * TQ + (blockIdx.x % CTAS_PER_TILE) * PW + warp;
-    if (sq >= a.nq) return;
-    const uint32_t qid = a.order[sq];
-    QState q;
-    double qlo[3], qhi[3];
-    const bool live = load_query(a.Q, qid, q, qlo, qhi);
-    const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start, a.bin_t0min,
-                                    a.bin_t1max, a.method, a.sb);
-    const uint32_t* ind = st.rind ? sb_ids(a.sb, st.rind) : nullptr;   // subbin id array
-    const uint32_t qtraj = a.excl ? __ldg(a.qtraj + qid) : 0u;
-    const double d2 = a.d * a.d;
-    unsigned long long out_pos = a.offsets[qid];
-    uint32_t dummy = 0;
-    for (uint32_t c0 = 0; c0 < st.nlook; c0 += 32) {
-        const uint32_t c = c0 + lane;
-        uint32_t start = 0, cnt = 0;
-        if (c < st.nlook)
-            resolve(a.g, a.ht, a.bin_t0min, a.bin_t1max, a.bin_start, st.mode, st.lb, st.hb,
-                    st.clo, st.cn, q.t0, q.t1, c, st.rstart, st.rcnt, start, cnt, dummy);
-        unsigned long long incl = cnt;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
-            if (lane >= o) incl += u;
-        }
-        const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
-        __syncwarp();
-        s_start[warp][lane] = start;
-        s_excl[warp][lane] = (uint32_t)(incl - cnt);   // < 2^32: runs of one query
-        __syncwarp();
-        for (unsigned long long base = 0; base < total; base += 32) {
-            const unsigned long long t = base + lane;
-            bool hit = false;
-            double r0 = 0.0, r1 = 0.0;
-            uint32_t p = 0;
-            if (t < total) {
-                int j = 0;
-#pragma unroll
-                for (int step = 16; step; step >>= 1)
-                    if (s_excl[warp][j + step] <= t) j += step;
-                p = s_start[warp][j] + (uint32_t)(t - s_excl[warp][j]);
-                if (ind) p = __ldg(ind + p);
-                if (!(a.excl && __ldg(a.etraj + p) == qtraj)) {
-                    double2 et, ex, ey, ez;
-                    a.soa.load4(p, et, ex, ey, ez);
-                    hit = refine(q, et, ex, ey, ez, d2, r0, r1);
-                }
-            }
-            const uint32_t bal = __ballot_sync(0xffffffffu, hit);
-            if (hit) {
-                dts_result rr;
-                rr.query_id = qid;                  // local id; mapped by k_place_over
-                rr.entry_id = __ldg(a.soa.eid + p);
-                rr.t_start = r0;
-                rr.t_end = r1;
-                a.out[out_pos + __popc(bal & ((1u << lane) - 1u))] = rr;
-            }
-            out_pos += __popc(bal);
-        }
-    }
-}
-
-// ------------------------------------------------------ canonical order
-// Fallback tiles (staging overflowed): their queries' results were written
-// by k_pass_scatter into a compact buffer, query q at cover_off[q] .. + count
-// (cover_off = exclusive scan, in query-id order, of the counts of those
-// queries only).  One device-wide stable radix sort by (query, entry id)
-// puts them in canonical order; k_place_over copies each to its exact final
-// offset.  Cost is linear in the number of such results.
+// ------------------------------------------------------ re-run bookkeeping
+// Tiles re-run after the spill buffer filled: cover[q] = counts[q] for their
+// queries (their records in the first spill buffer are stale; the scan of
+// cover sizes the re-run's exact spill buffer).
 __global__ void __launch_bounds__(PT) k_mark_over(const uint32_t* __restrict__ tiles,
                                                  const uint32_t* __restrict__ order, uint32_t nq,
                                                  const uint32_t* __restrict__ counts,
@@ -538,34 +443,6 @@ __global__ void __launch_bounds__(PT) k_mark_over(const uint32_t* __restrict__ t
         const uint32_t q = order[sp];
         cover[q] = counts[q];
     }
-}
-
-__global__ void __launch_bounds__(PT) k_keys_over(const dts_result* __restrict__ raw,
-                                                 unsigned long long n,
-                                                 unsigned long long* __restrict__ keys,
-                                                 uint32_t* __restrict__ vals) {
-    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
-    if (k >= n) return;
-    const dts_result r = raw[k];
-    keys[k] = ((unsigned long long)r.query_id << 32) | r.entry_id;
-    vals[k] = (uint32_t)k;
-}
-
-__global__ void __launch_bounds__(PT) k_place_over(const unsigned long long* __restrict__ keys,
-                                                  const uint32_t* __restrict__ vals,
-                                                  unsigned long long n,
-                                                  const unsigned long long* __restrict__ cover_off,
-                                                  const unsigned long long* __restrict__ offsets,
-                                                  const dts_result* __restrict__ raw,
-                                                  const uint32_t* __restrict__ qmap,
-                                                  uint32_t qid_base,
-                                                  dts_result* __restrict__ out) {
-    const unsigned long long k = (unsigned long long)blockIdx.x * PT + threadIdx.x;
-    if (k >= n) return;
-    const uint32_t q = (uint32_t)(keys[k] >> 32);
-    dts_result r = raw[vals[k]];
-    r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
-    out[offsets[q] + (k - cover_off[q])] = r;
 }
 
 __global__ void k_validate_only(const double4* __restrict__ Q, uint32_t nq, Counters* ctr) {
@@ -716,13 +593,25 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));
     tm.mark();
 
-    // ---- pass 1: warp tiles, count + staging
+    // ---- pass 1: warp tiles, count + staging (spilling output-heavy tiles)
     const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
     const unsigned long long stage_cap = 4ull * nq + (1ull << 20);
-    DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s);
+    // spill buffer: sized from the largest output this index has seen (a
+    // repeated output-heavy search spills without re-runs), at least 8
+    // records per query
+    // (DTS_SPILL_CAP: a fixed capacity, testing knob for the re-run path)
+    static const long long spill_env = [] {
+        const char* e = getenv("DTS_SPILL_CAP");
+        return e ? atoll(e) : -1ll;
+    }();
+    const unsigned long long spill_cap = spill_env >= 0 ? (unsigned long long)spill_env
+        : std::max<unsigned long long>(8ull * nq + (1ull << 20),
+                                       idx->spill_hint.load(std::memory_order_relaxed));
+    DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s), spill_tiles(ntiles, s);
     DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s);
-    DevBuf<dts_result> stage(stage_cap, s);
-    TileArgs ta;
+    DevBuf<dts_result> stage(stage_cap, s), spill(std::max<unsigned long long>(spill_cap, 1), s);
+    DTS_CUDA(cudaMemsetAsync(&ctr.p->spill_valid, 0xFF, sizeof(unsigned long long), s));
+    TileArgs ta{};
     ta.Q = Q;
     ta.order = order.p;
     ta.nq = (uint32_t)nq;
@@ -738,6 +627,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.stage_cap = stage_cap;
     ta.tile_base = tile_base.p;
     ta.over_tiles = over_tiles.p;
+    ta.spill_tiles = spill_tiles.p;
+    ta.spill = spill.p;
+    ta.spill_cap = spill_cap;
+    ta.tile_list = nullptr;
+    ta.n_list = 0;
+    ta.spill_all = 0;
     ta.qid_base = qid_base;
     ta.qmap = qmap;
     ta.etraj = idx->etraj;
@@ -749,43 +644,32 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.ctr = ctr.p;
     ta.method = idx->method;
     ta.sb = idx->sb;
+    int nsm = 148;
     {
-        int dev = 0, nsm = 148;
+        int dev = 0;
         cudaGetDevice(&dev);
         cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-        const unsigned want = (ntiles + WW - 1) / WW;
-        // CTAs per SM the kernel is register-bounded for (tuning knob
-        // DTS_TILE_OCC = 5..8: 102, 85, 73 or 64 registers per thread)
-        static const int occ = [] {
-            const char* e = getenv("DTS_TILE_OCC");
-            // measured on C4 (one box, 20 steps): 5: 0.97 ms, 6: 1.00, 7: 0.86, 8: 0.92
-            const int v = e ? atoi(e) : 7;
-            return (v == 5 || v == 6 || v == 8) ? v : 7;
-        }();
-        // (an L2 prefetch of the next round's buckets measured slower on C4:
-        //  0.85 vs 0.81 ms, and was removed)
-        const unsigned grid = std::min<unsigned>(want, (unsigned)(nsm * occ));
-        // DTS_WTILE_TMA=32: candidate records staged by TMA bulk copies in
-        // chunks of 32 (record layout, grid and temporal methods)
-        static const int tma = [] {
-            const char* e = getenv("DTS_WTILE_TMA");
-            return e ? atoi(e) : 0;
-        }();
-        const bool tma_ok = idx->soa.es == 4 && idx->method != DTS_METHOD_SUBBIN;
-        if (tma_ok && tma == 32) {
-            const int o = occ >= 7 ? 6 : occ;
-            if (o == 6) k_wtile_count<6, true, 32><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(ta);
-            else k_wtile_count<5, true, 32><<<std::min<unsigned>(want, nsm * 5), WT, 0, s>>>(ta);
-        } else if (idx->method == DTS_METHOD_SUBBIN) {
-            k_wtile_count<7, false, 32, true, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
-        } else if (idx->method == DTS_METHOD_TEMPORAL) {
-            k_wtile_count<7, false, 32, false, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(ta);
-        } else if (occ == 8) k_wtile_count<8><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 7) k_wtile_count<7><<<grid, WT, 0, s>>>(ta);
-        else if (occ == 5) k_wtile_count<5><<<grid, WT, 0, s>>>(ta);
-        else k_wtile_count<6><<<grid, WT, 0, s>>>(ta);
-        DTS_LAUNCH_CHECK();
     }
+    // CTAs per SM the grid kernel is register-bounded for (DTS_TILE_OCC =
+    // 6..8: 85, 73 or 64 registers per thread; measured on C4 (one box, 20
+    // steps): 6: 1.00 ms, 7: 0.86, 8: 0.92)
+    static const int occ = [] {
+        const char* e = getenv("DTS_TILE_OCC");
+        const int v = e ? atoi(e) : 7;
+        return (v == 6 || v == 8) ? v : 7;
+    }();
+    auto launch_pass1 = [&](const TileArgs& args, uint32_t tiles) {
+        const unsigned want = (tiles + WW - 1) / WW;
+        if (idx->method == DTS_METHOD_SUBBIN)
+            k_wtile_count<7, true, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
+        else if (idx->method == DTS_METHOD_TEMPORAL)
+            k_wtile_count<7, false, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
+        else if (occ == 8) k_wtile_count<8><<<std::min<unsigned>(want, nsm * 8), WT, 0, s>>>(args);
+        else if (occ == 6) k_wtile_count<6><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(args);
+        else k_wtile_count<7><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
+        DTS_LAUNCH_CHECK();
+    };
+    launch_pass1(ta, ntiles);
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
     tm.mark();
@@ -805,10 +689,15 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     local.cell_lookups = h.c.lookups;
     local.results = h.total;
     local.max_results_per_query = h.c.max_count;
+    if (h.c.n_over) {
+        // the spill buffer filled: size the next search's from this output
+        unsigned long long want = h.total + (1ull << 20), cur = idx->spill_hint.load();
+        while (cur < want && !idx->spill_hint.compare_exchange_weak(cur, want)) {}
+    }
 
     // ---- results that do not fit the device: report the per-query counts
     //      so a host caller can stream the search in query chunks
-    const double per = h.c.n_over ? 24.0 + 48.0 : 24.0;   // fin (+ raw, keys, vals, tmp)
+    const double per = h.c.n_over ? 24.0 + 24.0 : 24.0;   // fin (+ the re-run's spill)
     // (cudaMemGetInfo is slow and jittery -- ms -- so it is asked only when
     //  the results are large enough to matter)
     if (h.total > 0 && ((double)h.total * per > 1e9 || h.total > max_results)) {
@@ -833,58 +722,97 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                                                              offsets.p, tile_base.p, stage.p,
                                                              fin);
             DTS_LAUNCH_CHECK();
-            // ---- overflowed tiles: recompute (count-then-scatter) into a
-            //      compact buffer, then one radix sort by (query, entry id)
-            if (h.c.n_over) {
-                DevBuf<uint32_t> cover(nq, s);
-                DevBuf<unsigned long long> cover_off(nq + 1, s);
-                DTS_CUDA(cudaMemsetAsync(cover.p, 0, nq * sizeof(uint32_t), s));
-                k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq,
-                                                      counts.p, cover.p);
-                DTS_LAUNCH_CHECK();
-                scan_exclusive_u32_to_u64(cover.p, cover_off.p, nq, s);
+            tm.mark();
+            if (h.c.n_spill || h.c.n_over) {
+                DevBuf<uint32_t> cursor(nq, s), cover(h.c.n_over ? nq : 0, s);
+                DTS_CUDA(cudaMemsetAsync(cursor.p, 0, nq * sizeof(uint32_t), s));
+                DevBuf<dts_result> spill2(0, s);
                 unsigned long long n_raw = 0;
-                DTS_CUDA(cudaMemcpyAsync(&n_raw, cover_off.p + nq, sizeof(n_raw),
+                if (h.c.n_over) {
+                    // ---- tiles that found the spill buffer full: pass 1
+                    //      again over those tiles only, every hit spilled
+                    //      into a buffer of exactly their result count
+                    DevBuf<unsigned long long> cover_off(nq + 1, s);
+                    DTS_CUDA(cudaMemsetAsync(cover.p, 0, nq * sizeof(uint32_t), s));
+                    k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq,
+                                                          counts.p, cover.p);
+                    DTS_LAUNCH_CHECK();
+                    scan_exclusive_u32_to_u64(cover.p, cover_off.p, nq, s);
+                    DTS_CUDA(cudaMemcpyAsync(&n_raw, cover_off.p + nq, sizeof(n_raw),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                    spill2.alloc(std::max<unsigned long long>(n_raw, 1), s);
+                    DevBuf<Counters> ctr2(1, s);
+                    DTS_CUDA(cudaMemsetAsync(ctr2.p, 0, sizeof(Counters), s));
+                    DTS_CUDA(cudaMemsetAsync(&ctr2.p->spill_valid, 0xFF, 8, s));
+                    TileArgs tb = ta;
+                    tb.ctr = ctr2.p;
+                    tb.spill = spill2.p;
+                    tb.spill_cap = n_raw;
+                    tb.tile_list = over_tiles.p;
+                    tb.n_list = h.c.n_over;
+                    tb.spill_all = 1;
+                    launch_pass1(tb, h.c.n_over);
+                }
+                // ---- spilled records to their query segments, then each
+                //      segment sorted by entry id
+                const unsigned long long n1 = std::min(std::min(h.c.spilled, spill_cap),
+                                                       h.c.spill_valid);
+                if (n1) {
+                    k_spill_place<<<blocks(n1, 256), 256, 0, s>>>(
+                        spill.p, n1, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p, qmap,
+                        qid_base, fin);
+                    DTS_LAUNCH_CHECK();
+                }
+                if (n_raw) {
+                    k_spill_place<<<blocks(n_raw, 256), 256, 0, s>>>(
+                        spill2.p, n_raw, nullptr, offsets.p, cursor.p, qmap, qid_base, fin);
+                    DTS_LAUNCH_CHECK();
+                }
+                DevBuf<uint32_t> bigc(nq, s);
+                DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
+                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, sizeof(unsigned int), s));
+                if (h.c.n_spill) {
+                    k_seg_sort<<<h.c.n_spill * WQ, SEG_T, 0, s>>>(spill_tiles.p, order.p,
+                                                                 (uint32_t)nq, counts.p,
+                                                                 offsets.p, fin, bigc.p, ctr.p);
+                    DTS_LAUNCH_CHECK();
+                }
+                if (h.c.n_over) {
+                    k_seg_sort<<<h.c.n_over * WQ, SEG_T, 0, s>>>(over_tiles.p, order.p,
+                                                                (uint32_t)nq, counts.p,
+                                                                offsets.p, fin, bigc.p, ctr.p);
+                    DTS_LAUNCH_CHECK();
+                }
+                unsigned int n_big = 0;
+                DTS_CUDA(cudaMemcpyAsync(&n_big, &ctr.p->n_big, sizeof(n_big),
                                          cudaMemcpyDeviceToHost, s));
                 DTS_CUDA(cudaStreamSynchronize(s));
-                DevBuf<dts_result> raw(n_raw, s);
-                PassArgs pa;
-                pa.Q = Q;
-                pa.order = order.p;
-                pa.nq = (uint32_t)nq;
-                pa.d = d;
-                pa.g = idx->gp;
-                pa.soa = idx->soa;
-                pa.ht = idx->ht;
-                pa.bin_t0min = idx->bin_t0min;
-                pa.bin_t1max = idx->bin_t1max;
-                pa.bin_start = idx->bin_start;
-                pa.offsets = cover_off.p;          // compact positions
-                pa.tiles = over_tiles.p;
-                pa.out = raw.p;
-                pa.qid_base = qid_base;
-                pa.method = idx->method;
-                pa.sb = idx->sb;
-                pa.etraj = ta.etraj;
-                pa.qtraj = ta.qtraj;
-                pa.excl = ta.excl;
-                const unsigned nb = h.c.n_over * (TQ / PW);
-                k_pass_scatter<<<nb, PT, 0, s>>>(pa);
-                DTS_LAUNCH_CHECK();
-                tm.mark();
-                if (n_raw >= (1ull << 32))
-                    throw Error(DTS_ENOTSUP, "more than 2^32 results in recomputed tiles");
-                DevBuf<unsigned long long> k1(n_raw, s), k2(n_raw, s);
-                DevBuf<uint32_t> v1(n_raw, s), v2(n_raw, s);
-                k_keys_over<<<blocks(n_raw, PT), PT, 0, s>>>(raw.p, n_raw, k1.p, v1.p);
-                DTS_LAUNCH_CHECK();
-                radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, n_raw, 32 + bits_for(nq - 1), s);
-                k_place_over<<<blocks(n_raw, PT), PT, 0, s>>>(k1.p, v1.p, n_raw, cover_off.p,
-                                                             offsets.p, raw.p, qmap, qid_base,
-                                                             fin);
-                DTS_LAUNCH_CHECK();
-            } else {
-                tm.mark();
+                if (n_big) {
+                    // ---- segments longer than a CTA sort: one device-wide
+                    //      radix sort by (query, entry id) over those only
+                    DevBuf<unsigned long long> bigoff(nq + 1, s);
+                    scan_exclusive_u32_to_u64(bigc.p, bigoff.p, nq, s);
+                    unsigned long long nb = 0;
+                    DTS_CUDA(cudaMemcpyAsync(&nb, bigoff.p + nq, sizeof(nb),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                    if (nb >= (1ull << 32))
+                        throw Error(DTS_ENOTSUP, "more than 2^32 results in long segments");
+                    DevBuf<unsigned long long> k1(nb, s), k2(nb, s);
+                    DevBuf<uint32_t> v1(nb, s), v2(nb, s);
+                    DevBuf<dts_result> tmp(nb, s);
+                    k_big_keys<<<blocks((size_t)nq * 32, 256), 256, 0, s>>>(
+                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, fin, k1.p, v1.p);
+                    DTS_LAUNCH_CHECK();
+                    radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, nb, 32 + bits_for(nq - 1), s);
+                    k_big_gather<<<blocks(nb, 256), 256, 0, s>>>(k1.p, v1.p, nb, bigoff.p,
+                                                                offsets.p, fin, tmp.p);
+                    DTS_LAUNCH_CHECK();
+                    k_big_place<<<blocks(nb, 256), 256, 0, s>>>(k1.p, nb, bigoff.p, offsets.p,
+                                                               tmp.p, fin);
+                    DTS_LAUNCH_CHECK();
+                }
             }
             tm.mark();
             DTS_CUDA(cudaStreamSynchronize(s));

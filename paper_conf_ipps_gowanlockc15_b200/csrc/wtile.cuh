@@ -9,17 +9,24 @@
 //      count; a shuffle scan gives the tile's probe offsets;
 //   1. rounds of 32 row probes (one per lane) -> runs; a shuffle scan flattens
 //      them; lanes stream the candidates two at a time and refine them;
-//      hits go to the warp's shared-memory stage (query, entry id, interval);
+//      hits go to the warp's shared-memory stage (query, position, interval);
 //   2. per-query counts are written; each staged hit's rank inside its query
 //      is counted against the other staged hits (ordering by entry id), and
 //      the tile's hits are written to the global stage in canonical order.
-// A tile whose hits exceed WH (or the global stage) is marked for the
-// count-then-scatter fallback of pass 2.
+// Output-heavy tiles: whenever the shared stage could overflow in the next
+// step (more than WH - 64 hits), the warp flushes it to a global spill buffer
+// (one atomic per flush; hits as final records with the local query id) and
+// goes on; after the scan the spilled records are placed at their query's
+// offsets and each such query's segment is sorted by entry id (k_spill_place,
+// k_seg_sort).  No candidate is streamed twice.  Only a tile that finds the
+// spill buffer full is re-run (pass 1 again over the listed tiles, spilling
+// every hit into an exactly sized second buffer).
 
 constexpr int WQ = 16;                  // queries per warp tile (32: 1.42 ms on C4, 16: 0.82)
 constexpr int WH = 128;                 // staged hits per warp tile
 constexpr int WT = 128;                 // threads per CTA (4 independent warps)
 constexpr int WW = WT / 32;
+constexpr unsigned long long SPILLED = NONE - 2;   // tile_base of a spilled tile
 
 // Query record as read by the refinement: (t0,t1) (x0,vx) (y0,vy) (z0,vz)
 // in four 16-byte words (four LDS.128 per candidate instead of eight
@@ -45,7 +52,7 @@ struct WarpSmem {
     unsigned long long lkoff[WQ + 1];
     unsigned long long hkey[WH];        // (query << 42) | (position, then entry id << 10) | slot
     double h0[WH], h1[WH];
-    uint32_t nhit, over;
+    uint32_t nhit, over, spilled;
 };
 
 struct TileArgs {
@@ -62,8 +69,15 @@ struct TileArgs {
     uint32_t* counts;                  // per query id
     dts_result* stage;                 // staged hits (tile-contiguous, canonical inside)
     unsigned long long stage_cap;
-    unsigned long long* tile_base;     // per warp tile: first staged slot, NONE-1 empty, NONE redo
-    uint32_t* over_tiles;              // tiles to recompute in pass 2
+    unsigned long long* tile_base;     // per warp tile: first staged slot, NONE-1 empty,
+                                       // SPILLED spilled, NONE re-run
+    uint32_t* over_tiles;              // tiles to re-run (spill buffer full)
+    uint32_t* spill_tiles;             // tiles whose hits went to the spill buffer
+    dts_result* spill;                 // spilled hits (query_id = LOCAL query id)
+    unsigned long long spill_cap;
+    const uint32_t* tile_list;         // re-run: the tiles to process (else 0..ntiles-1)
+    uint32_t n_list;
+    uint32_t spill_all;                // re-run: every hit is spilled
     uint32_t qid_base;
     const uint32_t* qmap;              // optional reported query ids (else qid + qid_base)
     const uint32_t* etraj;             // trajectory id per sorted entry position
@@ -86,9 +100,11 @@ __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
 
 // The hit is staged with its sorted position p; the entry ids of all the
 // tile's hits are looked up together before ranking (one round trip per tile
-// instead of a dependent load per hit).
+// instead of a dependent load per hit).  A tile that is to be re-run only
+// counts.
 __device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, double r0, double r1) {
     atomicAdd(&S.qcount[qi], 1u);
+    if (S.over) return;
     const uint32_t pos = atomicAdd(&S.nhit, 1u);
     if (pos < (uint32_t)WH) {
         S.hkey[pos] = ((unsigned long long)qi << 42) | ((unsigned long long)p << 10) | pos;
@@ -99,80 +115,71 @@ __device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, doubl
     }
 }
 
+// Warp-uniform: the shared stage's hits -> the global spill buffer as
+// records (local query id, entry id, interval); one atomic per flush.  A
+// flush that finds the buffer full marks the tile for a re-run and records
+// the first invalid slot (records from there on are not placed).
+__device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int lane) {
+    __syncwarp();
+    const uint32_t nh = min(S.nhit, (uint32_t)WH);
+    if (nh == 0 || S.over) return;
+    unsigned long long b = 0;
+    if (lane == 0) b = atomicAdd(&a.ctr->spilled, (unsigned long long)nh);
+    b = __shfl_sync(0xffffffffu, b, 0);
+    if (b + nh > a.spill_cap) {
+        if (lane == 0) {
+            atomicMin(&a.ctr->spill_valid, b);
+            S.over = 1u;
+        }
+        __syncwarp();
+        return;
+    }
+    for (uint32_t i = lane; i < nh; i += 32) {
+        const unsigned long long k = S.hkey[i];
+        dts_result r;
+        r.query_id = S.qid[(uint32_t)(k >> 42)];
+        r.entry_id = __ldg(a.soa.eid + (uint32_t)(k >> 10));
+        r.t_start = S.h0[i];
+        r.t_end = S.h1[i];
+        a.spill[b + i] = r;
+    }
+    __syncwarp();
+    if (lane == 0) {
+        S.nhit = 0;
+        S.spilled = 1u;
+    }
+    __syncwarp();
+}
 
-// ---- TMA bulk staging of candidate records (sm_90+: cp.async.bulk)
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-    return (uint32_t)__cvta_generic_to_shared(p);
+// Flush when the next step (at most `step_max` hits) could overflow the stage.
+__device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int lane,
+                                            uint32_t step_max) {
+    __syncwarp();
+    if (S.nhit > (uint32_t)WH - step_max) flush_spill(S, a, lane);
 }
-__device__ __forceinline__ void mbar_init(unsigned long long* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count)
-                 : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
-                 "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(unsigned long long* bar, uint32_t parity) {
-    asm volatile(
-        "{\n"
-        ".reg .pred p;\n"
-        "WAIT_%=:\n"
-        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
-        "@!p bra WAIT_%=;\n"
-        "}\n" ::"r"(smem_u32(bar)), "r"(parity) : "memory");
-}
-// global -> shared bulk copy of `bytes` (multiple of 16, both 16-B aligned),
-// completion counted on the mbarrier
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes,
-                                         unsigned long long* bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
-        ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-
-// Per-warp double buffer of CH candidate records (64 B each) filled by the
-// TMA engine: the candidate stream no longer goes through the LSU/L1
-// (whose wavefronts run at ~70% of peak in the LDG version).
-template <int CH>
-struct WarpStage {
-    double4 rec[2][CH][2];
-    unsigned long long bar[2];
-};
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
 // temporal methods compile without that indirection.  GROUP: one-run
 // queries (temporal / subbin methods) streamed per group of identical runs
 // (step 1a); the grid method compiles without it (its rare one-run
 // fallback queries go through the probe rounds).
-template <int MINB, bool TMA = false, int CH = 32, bool SB = false, bool GROUP = false>
+template <int MINB, bool SB = false, bool GROUP = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
-    __shared__ __align__(128) WarpStage<TMA ? CH : 1> STG[TMA ? WW : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     WarpSmem& S = SW[warp];
     const GridParams& g = a.g;
     const double d = a.d, d2 = d * d;
-    const uint32_t ntiles = (a.nq + WQ - 1) / WQ;
+    const uint32_t ntiles = a.tile_list ? a.n_list : (a.nq + WQ - 1) / WQ;
     unsigned long long n_cand = 0;
     uint32_t n_probe = 0;
-    uint32_t phase[2] = {0u, 0u};
-    if (TMA) {
-        if (lane == 0) {
-            mbar_init(&STG[warp].bar[0], 1);
-            mbar_init(&STG[warp].bar[1], 1);
-            asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        }
-        __syncwarp();
-    }
 
     while (true) {
-        uint32_t wt = 0;
-        if (lane == 0) wt = atomicAdd(&a.ctr->work, 1u);
-        wt = __shfl_sync(0xffffffffu, wt, 0);
-        if (wt >= ntiles) break;
+        uint32_t wi = 0;
+        if (lane == 0) wi = atomicAdd(&a.ctr->work, 1u);
+        wi = __shfl_sync(0xffffffffu, wi, 0);
+        if (wi >= ntiles) break;
+        const uint32_t wt = a.tile_list ? a.tile_list[wi] : wi;
 
         // ---- 0: queries, stencils, probe offsets
         unsigned long long nlook = 0;
@@ -214,7 +221,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 ri = st.rind;
             }
         }
-        if (lane == 0) { S.nhit = 0; S.over = 0; S.lkoff[0] = 0; }
+        if (lane == 0) { S.nhit = 0; S.over = 0; S.spilled = 0; S.lkoff[0] = 0; }
         {
             unsigned long long inc = nlook;
 #pragma unroll
@@ -230,7 +237,8 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         // ---- 1a: one-run queries grouped by identical run (sorted neighbours
         //      usually share their bins, or their subbin chunk): each
         //      candidate of a run is loaded once and refined against every
-        //      query of the group, instead of once per query
+        //      query of the group, instead of once per query; at most 32
+        //      hits per (candidate chunk, query) step
         for (uint32_t smask = GROUP ? __ballot_sync(0xffffffffu, single) : 0u; smask;) {
             const int ld = __ffs(smask) - 1;
             const uint32_t lrs = __shfl_sync(0xffffffffu, rs, ld);
@@ -242,26 +250,29 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             n_cand += (unsigned long long)__popc(members) * lrc;
             for (uint32_t base = 0; base < lrc; base += 32) {
                 const uint32_t t = base + lane;
-                if (t >= lrc) continue;
-                const uint32_t slot = lrs + t;
+                const bool valid = t < lrc;
+                const uint32_t slot = lrs + (valid ? t : 0u);
                 uint32_t p = slot;
-                double2 st, sx, sy, sz;
-                if (SB && lri) {
-                    sb_load(a.sb, lri, slot, st, sx, sy, sz);
-                    p = ~0u;                             // id looked up on a hit only
-                    if (a.excl) p = __ldg(sb_ids(a.sb, lri) + slot);
-                } else {
-                    a.soa.load4(p, st, sx, sy, sz);
+                double2 st = make_double2(0, 0), sx = st, sy = st, sz = st;
+                if (valid) {
+                    if (SB && lri) {
+                        sb_load(a.sb, lri, slot, st, sx, sy, sz);
+                        p = ~0u;                             // id looked up on a hit only
+                        if (a.excl) p = __ldg(sb_ids(a.sb, lri) + slot);
+                    } else {
+                        a.soa.load4(p, st, sx, sy, sz);
+                    }
                 }
-                const uint32_t et = a.excl ? __ldg(a.etraj + p) : 0u;
+                const uint32_t et = (a.excl && valid) ? __ldg(a.etraj + p) : 0u;
                 for (uint32_t mm = members; mm; mm &= mm - 1) {
                     const int qi = __ffs(mm) - 1;
                     double h0, h1;
-                    if (a.excl && et == S.qtraj[qi]) continue;
-                    if (refine(smem_query(S, qi), st, sx, sy, sz, d2, h0, h1)) {
+                    if (valid && !(a.excl && et == S.qtraj[qi]) &&
+                        refine(smem_query(S, qi), st, sx, sy, sz, d2, h0, h1)) {
                         if (p == ~0u) p = __ldg(sb_ids(a.sb, lri) + slot);
                         stage_hit(S, qi, p, h0, h1);
                     }
+                    maybe_flush(S, a, lane, 32u);
                 }
             }
         }
@@ -291,58 +302,6 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
             const unsigned long long excl = incl - cnt;
             n_cand += total;
-            if (TMA) {
-                // chunks of CH candidates: chunk c+1's runs are copied into
-                // the other buffer while chunk c is refined.  Lane j copies
-                // the piece of its run j that falls in the chunk.
-                WarpStage<TMA ? CH : 1>& W = STG[warp];
-                const unsigned long long nch = (total + CH - 1) / CH;
-                auto issue = [&](unsigned long long c) {
-                    const int bsel = (int)(c & 1ull);
-                    const unsigned long long cb = c * CH;
-                    const unsigned long long ce = min(cb + (unsigned long long)CH, total);
-                    fence_proxy_async();        // our reads of this buffer precede the copy
-                    if (lane == 0) mbar_expect_tx(&W.bar[bsel], (uint32_t)((ce - cb) * 64));
-                    __syncwarp();
-                    const unsigned long long lo = max(excl, cb), hi = min(incl, ce);
-                    if (hi > lo)
-                        bulk_g2s(&W.rec[bsel][lo - cb][0],
-                                 a.soa.rec + 4 * ((size_t)start + (size_t)(lo - excl)),
-                                 (uint32_t)((hi - lo) * 64), &W.bar[bsel]);
-                };
-                if (nch) issue(0);    // (an empty round issues nothing: every
-                                      //  expect_tx must be matched by a wait)
-                for (unsigned long long c = 0; c < nch; ++c) {
-                    if (c + 1 < nch) issue(c + 1);
-                    const int bsel = (int)(c & 1ull);
-                    mbar_wait(&W.bar[bsel], phase[bsel]);
-                    phase[bsel] ^= 1u;
-                    const unsigned long long cb = c * CH;
-#pragma unroll
-                    for (int h = 0; h < CH / 32; ++h) {
-                        const unsigned long long t1 = cb + lane + 32 * h;
-                        int j1 = 0;
-#pragma unroll
-                        for (int step = 16; step; step >>= 1)
-                            if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
-                        const uint32_t s1 = __shfl_sync(0xffffffffu, start, j1);
-                        const unsigned long long e1 = __shfl_sync(0xffffffffu, excl, j1);
-                        const int qi1 = __shfl_sync(0xffffffffu, qi, j1);
-                        if (t1 < total) {
-                            const uint32_t p1 = s1 + (uint32_t)(t1 - e1);
-                            const double4 r0 = W.rec[bsel][lane + 32 * h][0];
-                            const double4 r1 = W.rec[bsel][lane + 32 * h][1];
-                            double h0, h1;
-                            const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
-                            if (!x1 && refine(smem_query(S, qi1), make_double2(r0.x, r0.y),
-                                              make_double2(r0.z, r0.w), make_double2(r1.x, r1.y),
-                                              make_double2(r1.z, r1.w), d2, h0, h1))
-                                stage_hit(S, qi1, p1, h0, h1);
-                        }
-                    }
-                    __syncwarp();
-                }
-            } else {
             // per run: the position delta start - excl (mod 2^32: a candidate's
             // position p = t + delta fits 32 bits even when the round's total
             // does not) and (query | method index << 8), one 32-bit shuffle
@@ -397,20 +356,29 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
                         stage_hit(S, qi2, p2, h0, h1);
                 }
-            }
+                maybe_flush(S, a, lane, 64u);
             }
         }
         __syncwarp();
 
-        // ---- 2: counts, canonical staging
-        const uint32_t nh = S.nhit;
+        // ---- 2: counts; canonical staging, or the last spill flush
         const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
         if (lane < WQ && sp < a.nq) {
             a.counts[S.qid[lane]] = cnt;
             if (cnt) atomicMax(&a.ctr->max_count, cnt);
         }
+        if (a.spill_all || S.spilled) flush_spill(S, a, lane);
+        __syncwarp();
+        const uint32_t nh = S.nhit;
         bool over = S.over != 0u;
-        if (!over && nh > 0) {
+        if (a.spill_all) {
+            // re-run: every hit is in the spill buffer (exactly sized)
+        } else if (!over && S.spilled) {
+            if (lane == 0) {
+                a.tile_base[wt] = SPILLED;
+                a.spill_tiles[atomicAdd(&a.ctr->n_spill, 1u)] = wt;
+            }
+        } else if (!over && nh > 0) {
             uint32_t inc = cnt;
 #pragma unroll
             for (int o = 1; o < 32; o <<= 1) {
@@ -454,12 +422,9 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         } else if (!over && lane == 0) {
             a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
         }
-        if (over) {
-            if (lane == 0) {
-                a.tile_base[wt] = NONE;
-                const uint32_t slot = atomicAdd(&a.ctr->n_over, 1u);
-                a.over_tiles[slot] = wt;
-            }
+        if (over && !a.spill_all && lane == 0) {
+            a.tile_base[wt] = NONE;
+            a.over_tiles[atomicAdd(&a.ctr->n_over, 1u)] = wt;
         }
         __syncwarp();
     }
@@ -486,7 +451,7 @@ __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ 
     const uint32_t wt = blockIdx.x * WW + warp;
     if (wt >= ntiles) return;
     const unsigned long long tb = tile_base[wt];
-    if (tb >= NONE - 1) return;                      // recomputed or empty tile
+    if (tb >= SPILLED) return;                       // spilled, re-run or empty tile
     const uint32_t sp = wt * WQ + lane;
     uint32_t cnt = 0;
     unsigned long long off = 0;
@@ -513,4 +478,132 @@ __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ 
         const uint32_t e = __shfl_sync(0xffffffffu, excl, q);
         if (i < nh) out[o + (i - e)] = stage[tb + i];
     }
+}
+
+// ------------------------------------------- spilled tiles: place + sort
+// Spilled records (query_id = local query id) go to their query's segment
+// [offsets[q], offsets[q] + counts[q]) in arrival order; records of queries
+// whose tile was re-run (cover[q] != 0) are stale and skipped.
+__global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restrict__ sp,
+                                                    unsigned long long n,
+                                                    const uint32_t* __restrict__ cover,
+                                                    const unsigned long long* __restrict__ offsets,
+                                                    uint32_t* __restrict__ cursor,
+                                                    const uint32_t* __restrict__ qmap,
+                                                    uint32_t qid_base,
+                                                    dts_result* __restrict__ out) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
+    if (k >= n) return;
+    dts_result r = sp[k];
+    const uint32_t q = r.query_id;
+    if (cover && cover[q]) return;
+    const unsigned long long pos = offsets[q] + atomicAdd(&cursor[q], 1u);
+    r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
+    out[pos] = r;
+}
+
+// One CTA per (listed tile, query slot): the query's segment (at most
+// SEG_CAP records) is loaded into shared memory, its (entry id, arrival
+// slot) keys are bitonic-sorted, and the records are written back in entry
+// id order (canonical; equal caller ids keep an unspecified order).  Longer
+// segments are flagged in bigc for the device-wide sort.
+constexpr int SEG_T = 128;
+constexpr int SEG_CAP = 1024;
+__global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__ tiles,
+                                                   const uint32_t* __restrict__ order,
+                                                   uint32_t nq,
+                                                   const uint32_t* __restrict__ counts,
+                                                   const unsigned long long* __restrict__ offsets,
+                                                   dts_result* __restrict__ out,
+                                                   uint32_t* __restrict__ bigc,
+                                                   Counters* __restrict__ ctr) {
+    __shared__ unsigned long long key[SEG_CAP];
+    __shared__ dts_result rec[SEG_CAP];
+    const uint32_t sp = tiles[blockIdx.x / WQ] * WQ + blockIdx.x % WQ;
+    if (sp >= nq) return;
+    const uint32_t q = order[sp];
+    const uint32_t c = counts[q];
+    if (c <= 1) return;
+    if (c > (uint32_t)SEG_CAP) {
+        if (threadIdx.x == 0) {
+            bigc[q] = c;
+            atomicAdd(&ctr->n_big, 1u);
+        }
+        return;
+    }
+    dts_result* seg = out + offsets[q];
+    uint32_t N = 2;
+    while (N < c) N <<= 1;
+    for (uint32_t i = threadIdx.x; i < N; i += SEG_T) {
+        if (i < c) {
+            const dts_result r = seg[i];
+            rec[i] = r;
+            key[i] = ((unsigned long long)r.entry_id << 32) | i;
+        } else {
+            key[i] = ~0ull;
+        }
+    }
+    __syncthreads();
+    for (uint32_t k = 2; k <= N; k <<= 1) {
+        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
+            for (uint32_t i = threadIdx.x; i < N; i += SEG_T) {
+                const uint32_t l = i ^ j;
+                if (l > i) {
+                    const unsigned long long a = key[i], b = key[l];
+                    const bool up = (i & k) == 0;
+                    if ((a > b) == up) {
+                        key[i] = b;
+                        key[l] = a;
+                    }
+                }
+            }
+            __syncthreads();
+        }
+    }
+    for (uint32_t i = threadIdx.x; i < c; i += SEG_T) seg[i] = rec[(uint32_t)(key[i] & 0xffffffffull)];
+}
+
+// Segments longer than SEG_CAP: (query, entry id) keys and their positions.
+__global__ void __launch_bounds__(256) k_big_keys(uint32_t nq, const uint32_t* __restrict__ bigc,
+                                                 const unsigned long long* __restrict__ bigoff,
+                                                 const unsigned long long* __restrict__ offsets,
+                                                 const dts_result* __restrict__ out,
+                                                 unsigned long long* __restrict__ keys,
+                                                 uint32_t* __restrict__ vals) {
+    const uint32_t warp = (blockIdx.x * 256 + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+    if (warp >= nq) return;
+    const uint32_t c = bigc[warp];
+    if (!c) return;
+    const unsigned long long o = offsets[warp], b = bigoff[warp];
+    for (uint32_t i = lane; i < c; i += 32) {
+        keys[b + i] = ((unsigned long long)warp << 32) | out[o + i].entry_id;
+        vals[b + i] = (uint32_t)(b + i);
+    }
+}
+
+__global__ void __launch_bounds__(256) k_big_gather(const unsigned long long* __restrict__ keys,
+                                                   const uint32_t* __restrict__ vals,
+                                                   unsigned long long n,
+                                                   const unsigned long long* __restrict__ bigoff,
+                                                   const unsigned long long* __restrict__ offsets,
+                                                   const dts_result* __restrict__ in,
+                                                   dts_result* __restrict__ tmp) {
+    // tmp[k] = the record of sorted element k, read from its old place
+    const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
+    if (k >= n) return;
+    const uint32_t q = (uint32_t)(keys[k] >> 32);
+    const unsigned long long src = vals[k];            // flat index before the sort
+    tmp[k] = in[offsets[q] + (src - bigoff[q])];
+}
+
+__global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __restrict__ keys,
+                                                  unsigned long long n,
+                                                  const unsigned long long* __restrict__ bigoff,
+                                                  const unsigned long long* __restrict__ offsets,
+                                                  const dts_result* __restrict__ tmp,
+                                                  dts_result* __restrict__ out) {
+    const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
+    if (k >= n) return;
+    const uint32_t q = (uint32_t)(keys[k] >> 32);
+    out[offsets[q] + (k - bigoff[q])] = tmp[k];
 }

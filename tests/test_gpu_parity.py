@@ -445,6 +445,59 @@ def test_heavy_output_recompute_path(dts, oracle_mod):
         assert info["common"] > 1000
 
 
+def test_spill_paths_same_bytes(dts, oracle_mod):
+    """Output-heavy tiles spill their hits (no re-stream); with the spill
+    buffer forced small (DTS_SPILL_CAP) tiles find it full and are re-run
+    into an exactly sized buffer, and with it forced to 0 every spilling
+    tile is re-run.  Same bytes every way, oracle parity, including queries
+    with more results than one CTA sorts (device-wide sort of long
+    segments)."""
+    import subprocess
+    import sys
+    code = ("import sys; sys.path[:0] = [%r, %r]; import numpy as np, synth, "
+            "paper_conf_ipps_gowanlockc15_b200 as m\n"
+            "c = synth.make_config('C2', scale=0.004)\n"
+            "g = np.random.default_rng(5); n = 4000\n"
+            "D = np.zeros((n, 8)); D[:, 4] = 1.0\n"
+            "D[:, 1:4] = g.uniform(0, 0.01, (n, 3)); D[:, 5:8] = D[:, 1:4]\n"
+            "Q = np.array([[0.0, 0, 0, 0, 1.0, 0.005, 0.005, 0.005]] * 3)\n"
+            "out = [m.search(m.build_index(c.D), c.Q, d).tobytes() for d in (2.0, 8.0)]\n"
+            "out.append(m.search(m.build_index(D), Q, 0.05).tobytes())\n"
+            "sys.stdout.buffer.write(b''.join(len(o).to_bytes(8, 'little') + o for o in out))"
+            % (REPO, os.path.join(REPO, "tests")))
+
+    def split(buf):
+        parts, k = [], 0
+        while k < len(buf):
+            n = int.from_bytes(buf[k:k + 8], "little")
+            parts.append(buf[k + 8:k + 8 + n])
+            k += 8 + n
+        return parts
+    runs = []
+    for env in ({}, {"DTS_SPILL_CAP": "1000"}, {"DTS_SPILL_CAP": "0"}):
+        out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
+                             capture_output=True, timeout=900)
+        assert out.returncode == 0, out.stderr.decode()[-3000:]
+        runs.append(split(out.stdout))
+    assert runs[0] == runs[1] == runs[2]
+    c = synth.make_config("C2", scale=0.004)
+    for k, d in enumerate((2.0, 8.0)):
+        got = np.frombuffer(runs[0][k], dtype=dts.RESULT_DTYPE)
+        info = parity.compare(got, oracle_mod.search(c.D, c.Q, d, threads=THREADS), c.D, c.Q, d,
+                              oracle_mod)
+        assert info["common"] > 20 * c.Q.shape[0]
+    g = np.random.default_rng(5)
+    n = 4000
+    D = np.zeros((n, 8))
+    D[:, 4] = 1.0
+    D[:, 1:4] = g.uniform(0, 0.01, (n, 3))
+    D[:, 5:8] = D[:, 1:4]
+    Q = np.array([[0.0, 0, 0, 0, 1.0, 0.005, 0.005, 0.005]] * 3)
+    got = np.frombuffer(runs[0][2], dtype=dts.RESULT_DTYPE)
+    info = parity.compare(got, oracle_mod.search(D, Q, 0.05), D, Q, 0.05, oracle_mod)
+    assert info["common"] == 3 * n              # three queries with 4,000 results each
+
+
 @pytest.mark.parametrize("world", [2, 3])
 def test_temporal_shards_on_one_gpu_match_unsharded(dts, world):
     """SURVEY §4 'multi-GPU without a cluster': the temporal-range shards of D
