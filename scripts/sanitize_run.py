@@ -52,3 +52,9 @@ res1, _ = dts.search_device(idx, Q1, 0.02)
 costs = dts.query_costs_device(idx, Q1, 0.02, block=64)
 torch.cuda.synchronize()
 print("sanitize workload 2 ok", r2.shape[0], res1.count, int(costs.sum()), flush=True)
+# spill path (output-heavy tiles), re-run path is exercised by DTS_SPILL_CAP in the tests
+c2 = synth.make_config("C2", scale=0.004)
+idx = dts.build_index(c2.D)
+r3 = dts.search(idx, c2.Q, 8.0)
+idx.free()
+print("sanitize workload 3 ok", r3.shape[0], flush=True)
