@@ -976,6 +976,7 @@ static void choose_grid(const Bounds& b, const dts_index_params& p, GridParams& 
 void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                         const dts_index_params& p, cudaStream_t s) {
     idx->n = n;
+    idx->eid_bits = p.entry_ids ? 32 : std::max(1, bits_for(n ? n - 1 : 0));
     if (n == 0) return;
     const double4* D = reinterpret_cast<const double4*>(D_dev);
     // phase events: start, bounds, keys, sort, gather, insert (+ end)

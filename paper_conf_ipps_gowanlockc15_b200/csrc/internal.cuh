@@ -357,6 +357,7 @@ struct dts_index {
     // spill-buffer size hint (records): the largest output a search of this
     // index has produced after its spill buffer filled (search.cu)
     mutable std::atomic<unsigned long long> spill_hint{0};
+    int eid_bits = 32;             // bits of the largest reported entry id
 };
 
 namespace dts {

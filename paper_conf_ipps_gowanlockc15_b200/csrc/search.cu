@@ -797,20 +797,23 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     DTS_CUDA(cudaMemcpyAsync(&nb, bigoff.p + nq, sizeof(nb),
                                              cudaMemcpyDeviceToHost, s));
                     DTS_CUDA(cudaStreamSynchronize(s));
-                    if (nb >= (1ull << 32))
-                        throw Error(DTS_ENOTSUP, "more than 2^32 results in long segments");
+                    // key bits: query, entry id (caller ids: 32 bits), slot
+                    const int qb = bits_for(nq - 1), eb = idx->eid_bits;
+                    const int sb = std::max(1, bits_for((unsigned long long)h.c.max_count - 1));
+                    if (qb + eb + sb > 64)
+                        throw Error(DTS_ENOTSUP, "long result segments: sort key exceeds 64 bits");
                     DevBuf<unsigned long long> k1(nb, s), k2(nb, s);
-                    DevBuf<uint32_t> v1(nb, s), v2(nb, s);
                     DevBuf<dts_result> tmp(nb, s);
                     k_big_keys<<<blocks((size_t)nq * 32, 256), 256, 0, s>>>(
-                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, fin, k1.p, v1.p);
+                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, fin, eb, sb, k1.p);
                     DTS_LAUNCH_CHECK();
-                    radix_sort_pairs(k1.p, v1.p, k2.p, v2.p, nb, 32 + bits_for(nq - 1), s);
-                    k_big_gather<<<blocks(nb, 256), 256, 0, s>>>(k1.p, v1.p, nb, bigoff.p,
-                                                                offsets.p, fin, tmp.p);
+                    const unsigned long long* sk =
+                        radix_sort_keys(k1.p, k2.p, nb, sb, sb + eb + qb, s);
+                    k_big_gather<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, offsets.p, fin,
+                                                                tmp.p);
                     DTS_LAUNCH_CHECK();
-                    k_big_place<<<blocks(nb, 256), 256, 0, s>>>(k1.p, nb, bigoff.p, offsets.p,
-                                                               tmp.p, fin);
+                    k_big_place<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, bigoff.p,
+                                                               offsets.p, tmp.p, fin);
                     DTS_LAUNCH_CHECK();
                 }
             }

@@ -563,47 +563,46 @@ __global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__
     for (uint32_t i = threadIdx.x; i < c; i += SEG_T) seg[i] = rec[(uint32_t)(key[i] & 0xffffffffull)];
 }
 
-// Segments longer than SEG_CAP: (query, entry id) keys and their positions.
+// Segments longer than SEG_CAP: one device-wide keys-only radix sort of
+// packed keys (query << (eb + sb) | entry id << sb | slot in segment) on the
+// (query, entry id) bits; the slot rides in the low bits.  One warp per query.
 __global__ void __launch_bounds__(256) k_big_keys(uint32_t nq, const uint32_t* __restrict__ bigc,
                                                  const unsigned long long* __restrict__ bigoff,
                                                  const unsigned long long* __restrict__ offsets,
-                                                 const dts_result* __restrict__ out,
-                                                 unsigned long long* __restrict__ keys,
-                                                 uint32_t* __restrict__ vals) {
+                                                 const dts_result* __restrict__ out, int eb, int sb,
+                                                 unsigned long long* __restrict__ keys) {
     const uint32_t warp = (blockIdx.x * 256 + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (warp >= nq) return;
     const uint32_t c = bigc[warp];
     if (!c) return;
     const unsigned long long o = offsets[warp], b = bigoff[warp];
-    for (uint32_t i = lane; i < c; i += 32) {
-        keys[b + i] = ((unsigned long long)warp << 32) | out[o + i].entry_id;
-        vals[b + i] = (uint32_t)(b + i);
-    }
+    const unsigned long long qk = (unsigned long long)warp << (eb + sb);
+    for (uint32_t i = lane; i < c; i += 32)
+        keys[b + i] = qk | ((unsigned long long)out[o + i].entry_id << sb) | i;
 }
 
+// tmp[k] = the record of sorted element k (read from its place in its segment)
 __global__ void __launch_bounds__(256) k_big_gather(const unsigned long long* __restrict__ keys,
-                                                   const uint32_t* __restrict__ vals,
-                                                   unsigned long long n,
-                                                   const unsigned long long* __restrict__ bigoff,
+                                                   unsigned long long n, int eb, int sb,
                                                    const unsigned long long* __restrict__ offsets,
                                                    const dts_result* __restrict__ in,
                                                    dts_result* __restrict__ tmp) {
-    // tmp[k] = the record of sorted element k, read from its old place
     const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
     if (k >= n) return;
-    const uint32_t q = (uint32_t)(keys[k] >> 32);
-    const unsigned long long src = vals[k];            // flat index before the sort
-    tmp[k] = in[offsets[q] + (src - bigoff[q])];
+    const unsigned long long key = keys[k];
+    const uint32_t q = (uint32_t)(key >> (eb + sb));
+    const unsigned long long slot = key & ((1ull << sb) - 1ull);
+    tmp[k] = in[offsets[q] + slot];
 }
 
 __global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __restrict__ keys,
-                                                  unsigned long long n,
+                                                  unsigned long long n, int eb, int sb,
                                                   const unsigned long long* __restrict__ bigoff,
                                                   const unsigned long long* __restrict__ offsets,
                                                   const dts_result* __restrict__ tmp,
                                                   dts_result* __restrict__ out) {
     const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
     if (k >= n) return;
-    const uint32_t q = (uint32_t)(keys[k] >> 32);
+    const uint32_t q = (uint32_t)(keys[k] >> (eb + sb));
     out[offsets[q] + (k - bigoff[q])] = tmp[k];
 }

@@ -21,19 +21,25 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--points", nargs="+", default=["C2:8", "S2:1", "C2:2"])
 ap.add_argument("--reps", type=int, default=5)
 ap.add_argument("--method", default="grid")
+ap.add_argument("--no-hint", action="store_true", help="grid sized without d_hint = d")
 a = ap.parse_args()
 cache = {}
 for pt in a.points:
     name, d = pt.split(":")
     d = float(d)
-    if name not in cache:
+    key = (name, None if a.no_hint else d)
+    if key not in cache:
+        for v in cache.values():
+            v[2].free()
         cache.clear()
         torch.cuda.empty_cache()
         c = synth.make_config(name)
         Dd = torch.from_numpy(c.D).cuda()
         Qd = torch.from_numpy(c.Q).cuda()
-        cache[name] = (c, Qd, dts.build_index_device(Dd, method=a.method), Dd)
-    c, Qd, idx, _ = cache[name]
+        # as scripts/sweep.py: the grid sized for the d searched (d_hint = d)
+        cache[key] = (c, Qd, dts.build_index_device(Dd, method=a.method,
+                                                    d_hint=0.0 if a.no_hint else d), Dd)
+    c, Qd, idx, _ = cache[key]
     s = torch.cuda.current_stream()
     for _ in range(2):
         r, st = dts.search_device(idx, Qd, d, stream=s, time_kernels=True)

@@ -485,7 +485,8 @@ def test_spill_paths_same_bytes(dts, oracle_mod):
         got = np.frombuffer(runs[0][k], dtype=dts.RESULT_DTYPE)
         info = parity.compare(got, oracle_mod.search(c.D, c.Q, d, threads=THREADS), c.D, c.Q, d,
                               oracle_mod)
-        assert info["common"] > 20 * c.Q.shape[0]
+        if d == 8.0:                            # hundreds of results per query: spills
+            assert info["common"] > 20 * c.Q.shape[0]
     g = np.random.default_rng(5)
     n = 4000
     D = np.zeros((n, 8))
