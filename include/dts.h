@@ -258,9 +258,9 @@ typedef struct {
                                    one fused read of D for exact bounds, keys
                                    and sort histograms (phase "bounds" is then
                                    the sample, "keys" the fused pass)        */
-    uint32_t hash_kind;         /* cell table: 0 one slot per cell, 1 one slot
-                                   per block of 8 consecutive cell keys      */
-    uint64_t hash_items;        /* slots in use (cells or blocks)            */
+    uint32_t hash_kind;         /* cell table: 1 = one 32-byte slot per block
+                                   of 8 consecutive cell keys (the only kind) */
+    uint64_t hash_items;        /* slots in use (blocks)                     */
     uint64_t hash_bytes;        /* table size in bytes                       */
 } dts_index_info;
 

@@ -276,67 +276,7 @@ __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restr
         if (h[j]) atomicAdd(hist + j, h[j]);
 }
 
-// One non-empty cell into the bucketed open-addressing table: key -> [p, e).
-__device__ __forceinline__ void insert_cell(const HashTable& ht, unsigned long long k, uint32_t p,
-                                            uint32_t e) {
-    const unsigned long long bmask = ht.mask >> 2;
-    unsigned long long b = bucket_of(k >> 2, ht);
-    CellSlot* const slots = ht.cells();
-    // try the slot matching the key's position in its group first: the (up
-    // to) four x-adjacent cells sharing a home bucket then claim distinct
-    // slots without colliding on the same CAS
-    const int first = (int)(k & 3ull);
-    while (true) {
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            const int i = (first + j) & 3;
-            CellSlot& sl = slots[4 * b + i];
-            const unsigned long long prev = atomicCAS(&sl.key, EMPTY_KEY, k);
-            if (prev == EMPTY_KEY) {
-                sl.start = p;
-                sl.end = e;
-                return;
-            }
-        }
-        b = (b + 1) & bmask;
-    }
-}
-
-
-
-// Tiled insert: the tile's keys (plus the one before) are staged in shared
-// memory, so a cell head finds its run's end there (global reads only for a
-// run that crosses the tile's end); then one CAS per cell as in k_insert.
-template <int ITEMS>
-__global__ void __launch_bounds__(BT) k_insert_tiled(const SortedKeys keys, size_t n,
-                                                    HashTable ht) {
-    constexpr int TILE = BT * ITEMS;
-    __shared__ unsigned long long s_key[TILE + 1];
-    const size_t p0 = (size_t)blockIdx.x * TILE;
-    const uint32_t tn = (uint32_t)min((size_t)TILE, n - p0);
-#pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-        const uint32_t loc = k * BT + threadIdx.x;
-        if (loc < tn) s_key[1 + loc] = keys.key(p0 + loc);
-    }
-    if (threadIdx.x == 0) s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
-    __syncthreads();
-#pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-        const uint32_t loc = k * BT + threadIdx.x;
-        if (loc >= tn) continue;
-        const unsigned long long key = s_key[1 + loc];
-        if (p0 + loc != 0 && s_key[loc] == key) continue;
-        uint32_t e = loc + 1;
-        while (e < tn && s_key[1 + e] == key) ++e;
-        size_t end = p0 + e;
-        if (e == tn)
-            while (end < n && keys.key(end) == key) ++end;
-        insert_cell(ht, key, (uint32_t)(p0 + loc), (uint32_t)end);
-    }
-}
-
-// Block slots (kind 1): the head of each block of 8 keys (the first sorted
+// Block slots: the head of each block of 8 keys (the first sorted
 // entry with that key >> 3) walks the block's entries -- keys ascend, so the
 // offsets key & 7 come in order -- builds the 8 inclusive prefix counts and
 // claims one 32-byte slot.  One CAS per block instead of one per cell.
@@ -359,75 +299,6 @@ __device__ __forceinline__ void insert_block(const HashTable& ht, unsigned long 
             }
         }
         b = (b + 1) & bmask;
-    }
-}
-
-template <int ITEMS>
-__global__ void __launch_bounds__(BT) k_insert_blocks(const SortedKeys keys, size_t n,
-                                                     HashTable ht) {
-    // warp w owns the tile positions [w * 32 * ITEMS, (w + 1) * 32 * ITEMS)
-    // in chunks of 32; the block heads of a chunk are processed one after
-    // the other by the whole warp, 32 entries of the block per step, the
-    // eight prefix counts taken with ballots (no lane walks a long block
-    // alone); then every head lane claims its slot
-    constexpr int TILE = BT * ITEMS;
-    __shared__ unsigned long long s_key[TILE + 1];
-    const size_t p0 = (size_t)blockIdx.x * TILE;
-    const uint32_t tn = (uint32_t)min((size_t)TILE, n - p0);
-#pragma unroll
-    for (int k = 0; k < ITEMS; ++k) {
-        const uint32_t loc = k * BT + threadIdx.x;
-        if (loc < tn) s_key[1 + loc] = keys.key(p0 + loc);
-    }
-    if (threadIdx.x == 0) s_key[0] = p0 > 0 ? keys.key(p0 - 1) : ~0ull;
-    __syncthreads();
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    auto key_at = [&](uint32_t q) -> unsigned long long {   // tile position q (may be >= tn)
-        if (q < tn) return s_key[1 + q];
-        const size_t p = p0 + q;
-        return p < n ? keys.key(p) : ~0ull;
-    };
-#pragma unroll 1
-    for (int k = 0; k < ITEMS; ++k) {
-        const uint32_t cbase = (uint32_t)(warp * 32 * ITEMS + k * 32);
-        const uint32_t loc = cbase + lane;
-        bool head = false;
-        unsigned long long blk = 0;
-        if (loc < tn) {
-            blk = s_key[1 + loc] >> 3;
-            head = p0 + loc == 0 || (s_key[loc] >> 3) != blk;
-        }
-        uint32_t heads = __ballot_sync(0xffffffffu, head);
-        unsigned long long my_lo = 0, my_hi = 0;
-        uint32_t my_big = 0;
-        while (heads) {
-            const int h = __ffs(heads) - 1;
-            heads &= heads - 1;
-            const uint32_t hp = cbase + h;
-            const unsigned long long hb = __shfl_sync(0xffffffffu, blk, h);
-            uint32_t cum[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-            for (uint32_t q = hp;; q += 32) {
-                const unsigned long long kq = key_at(q + lane);
-                const bool in = (kq >> 3) == hb;
-                const uint32_t off = (uint32_t)(kq & 7ull);
-#pragma unroll
-                for (int j = 0; j < 8; ++j) cum[j] += __popc(__ballot_sync(0xffffffffu, in && off <= (uint32_t)j));
-                if (__ballot_sync(0xffffffffu, in) != 0xffffffffu) break;
-            }
-            if (lane == h) {
-                if (cum[7] > 65535u) {            // the block as one run [start, start + cum[7])
-                    my_big = 1;
-                    my_lo = cum[7];
-                } else {
-#pragma unroll
-                    for (int j = 0; j < 4; ++j) {
-                        my_lo |= (unsigned long long)cum[j] << (16 * j);
-                        my_hi |= (unsigned long long)cum[4 + j] << (16 * j);
-                    }
-                }
-            }
-        }
-        if (head) insert_block(ht, blk, (uint32_t)(p0 + loc), my_big, my_lo, my_hi);
     }
 }
 
@@ -638,7 +509,7 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
             const int loc = k * BT + threadIdx.x;
             if (p0 + (size_t)loc < n) {
                 const int32_t b = s_bin[loc + 1];
-                const double2 t = *soa.at(0, p0 + (size_t)loc);   // written above by this thread
+                const double2 t = *soa.at(p0 + (size_t)loc);   // written above by this thread
                 atomicMin(&bin_t0min[b], ordered_bits(t.x));
                 atomicMax(&bin_t1max[b], ordered_bits(t.y));
             }
@@ -763,7 +634,7 @@ __global__ void __launch_bounds__(BT) k_sb_emit(const double4* __restrict__ D,
     const uint32_t i = eid[p];
     const double c0 = coord<A>(D[2 * (size_t)i]), c1 = coord<A>(D[2 * (size_t)i + 1]);
     const int32_t jlo = subbin_of(sb, A, fmin(c0, c1)), jhi = subbin_of(sb, A, fmax(c0, c1));
-    const unsigned long long bin = (unsigned long long)bin_of(g, soa.ld(0, p).x);
+    const unsigned long long bin = (unsigned long long)bin_of(g, __ldg(soa.at(p)).x);
     unsigned long long o = off[p];
     for (int32_t j = jlo; j <= jhi; ++j, ++o) {
         keys[o] = (unsigned long long)j * (unsigned long long)g.m + bin;
@@ -1198,16 +1069,6 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     blk = static_cast<char*>(cache_alloc(bytes_soa + bytes_bins + 256));
     idx->block = blk;
     idx->soa.rec = reinterpret_cast<double2*>(blk);
-    // 64-byte records read and written as two 256-bit accesses (DTS_LAYOUT=
-    // soa: four 16-byte streams).  Measured on C4: records 0.759 ms gather,
-    // 0.742 ms pass 1; streams 0.765, 0.802 (with 128-bit accesses the
-    // records lost: 0.852 / 0.838 against 0.775 / 0.814)
-    static const bool aos = [] {
-        const char* e = getenv("DTS_LAYOUT");
-        return !(e && e[0] == 's');
-    }();
-    idx->soa.ss = aos ? 1 : n;
-    idx->soa.es = aos ? 4u : 1u;
     idx->bin_t0min = reinterpret_cast<double*>(idx->soa.rec + 4 * n);
     idx->bin_t1max = idx->bin_t0min + g.m;
     idx->soa.eid = reinterpret_cast<uint32_t*>(idx->bin_t1max + g.m);
@@ -1247,44 +1108,25 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     DTS_CUDA(cudaMemcpyAsync(hc, ncell.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
     idx->n_cells = hc[0];
-    // 6. the non-empty cells -> bucketed hash table.  Kind 1 (default): one
-    //    32-byte slot per block of 8 keys (prefix counts per cell), >= 3.3
-    //    slots per block; kind 0 (DTS_HASH_KIND=0): one 16-byte slot per
-    //    cell, >= 2 slots per cell.
-    static const int hkind = [] {
-        const char* e = getenv("DTS_HASH_KIND");
-        return (e && e[0] == '0') ? 0 : 1;
-    }();
-    static const double hload = [] {          // DTS_HASH_SLOTS: slots per item
+    // 6. the non-empty blocks of 8 keys -> bucketed hash table, one 32-byte
+    //    slot per block (prefix counts per cell), >= 3.3 slots per block
+    //    (1.6: insert 0.487 ms, pass 1 0.711 on C4, against 0.435, 0.651)
+    static const double hload = [] {          // DTS_HASH_SLOTS: slots per block
         const char* e = getenv("DTS_HASH_SLOTS");
-        return e ? std::max(1.1, atof(e)) : 0.0;
+        return e ? std::max(1.1, atof(e)) : 3.3;
     }();
-    const double per = hload > 0.0 ? hload : (hkind ? 3.3 : 2.0);
-    const double items = (double)(hkind ? hc[1] : hc[0]);
-    const size_t slot_bytes = hkind ? sizeof(BlockSlot) : sizeof(CellSlot);
+    const double items = (double)hc[1];
     int log2cap = 6;
-    while ((double)(1ull << log2cap) < per * items) ++log2cap;
-    idx->ht.kind = hkind;
-    idx->hash_items = hkind ? hc[1] : hc[0];
+    while ((double)(1ull << log2cap) < hload * items) ++log2cap;
+    idx->hash_items = hc[1];
     idx->ht.log2cap = log2cap;
     idx->ht.mask = (1ull << log2cap) - 1;
-    idx->ht.slots = cache_alloc(slot_bytes << log2cap);
-    DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, slot_bytes << log2cap, s));
-    // (measured on C4 for cell slots, incl. the memset: tiled 0.550 ms; one
-    //  thread per entry with global key scans 0.565; batching the first CAS
-    //  of 2 / 4 / 8 cells 0.59 / 0.70 / 0.91 ms)
-    static const int iwalk = [] {             // DTS_INSERT_WALK=0: warp-cooperative heads
-        const char* e = getenv("DTS_INSERT_WALK");
-        return e ? atoi(e) : 1;
-    }();
-    // (a walk-free variant -- CTA max-scan of the head positions, per-block
-    //  offset counters by shared-memory atomics -- measured 0.507 ms against
-    //  0.435 for the lane walks: the insert is bound by the CAS round trips
-    //  into the 512 MB table, which the walks overlap)
-    if (hkind && iwalk)
-        k_insert_blocks_lane<4, 32><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
-    else if (hkind) k_insert_blocks<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
-    else k_insert_tiled<4><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    idx->ht.slots = cache_alloc(sizeof(BlockSlot) << log2cap);
+    DTS_CUDA(cudaMemsetAsync(idx->ht.slots, 0xFF, sizeof(BlockSlot) << log2cap, s));
+    // lane-parallel walks of the staged keys, warp path past 32 entries
+    // (warp-cooperative heads for every block: 0.736 ms on C4; one CAS per
+    // cell into cell slots: 0.56 ms; these lane walks: 0.435)
+    k_insert_blocks_lane<4, 32><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
     DTS_LAUNCH_CHECK();
     mark();
 

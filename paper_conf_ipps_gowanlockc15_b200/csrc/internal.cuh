@@ -71,25 +71,20 @@ struct DevBuf {
 };
 
 // ---------------------------------------------------------------- layout
-// Entry segments in the index live in key order as four 16-byte streams
-// (SoA, one 128-bit load each):
-//   st = (t_start, t_end)   sx = (x_start, vx)   sy = (y_start, vy)   sz = (z_start, vz)
-// with v = (end - start) / (t_end - t_start) precomputed at build (0 for a
-// zero-duration segment, which can never overlap strictly in time).  The
-// position at time t is start + (t - t_start) * v.
-// Entry records in sorted order: four double2 "streams" k = 0..3 holding
-// (t0,t1) (x0,vx) (y0,vy) (z0,vz).  Stream k of position p is
-// rec[k * ss + p * es]: ss = n, es = 1 is the SoA layout (four arrays);
-// ss = 1, es = 4 the record layout (one 64-byte record per entry).
+// Entry segments in the index live in key order as one 64-byte record each,
+//   (t_start, t_end, x_start, vx, y_start, vy, z_start, vz),
+// read and written as two 256-bit accesses, with v = (end - start) /
+// (t_end - t_start) precomputed at build (0 for a zero-duration segment,
+// which can never overlap strictly in time).  The position at time t is
+// start + (t - t_start) * v.  (Four 16-byte double2 streams instead were
+// measured slower on C4 in round 1: gather 0.765 vs 0.759 ms, pass 1 0.802
+// vs 0.742.)
 struct SegSoA {
-    double2* rec;
-    size_t ss;
-    uint32_t es;
+    double2* rec;    // 4 double2 per sorted position
     uint32_t* eid;   // caller's entry id of each sorted position
 #ifdef __CUDACC__
-    __device__ __forceinline__ double2* at(int k, size_t p) const { return rec + k * ss + p * es; }
-    __device__ __forceinline__ double2 ld(int k, size_t p) const { return __ldg(at(k, p)); }
-    // all four streams of position p (record layout: two 256-bit loads)
+    __device__ __forceinline__ const double2* at(size_t p) const { return rec + 4 * p; }
+    // the record of sorted position p (two 256-bit loads)
     __device__ __forceinline__ void load4(size_t p, double2& st, double2& sx, double2& sy,
                                           double2& sz) const;
     __device__ __forceinline__ void store4(size_t p, double2 st, double2 sx, double2 sy,
@@ -97,13 +92,6 @@ struct SegSoA {
 #endif
 };
 
-// Hash slot of one non-empty (bin, cell) key: entries [start, end) of the
-// sorted arrays.  16 bytes, one 128-bit load.
-struct __align__(16) CellSlot {
-    unsigned long long key;
-    uint32_t start;
-    uint32_t end;
-};
 static constexpr unsigned long long EMPTY_KEY = ~0ull;
 
 // Hash slot of one non-empty BLOCK of 8 consecutive keys (key >> 3): 8
@@ -136,12 +124,10 @@ struct GridParams {
 };
 
 struct HashTable {
-    void* slots;               // CellSlot (kind 0) or BlockSlot (kind 1)
+    void* slots;               // BlockSlot, 2 per 64-byte bucket
     unsigned long long mask;   // slots - 1 (power of two)
     int log2cap;               // log2 of the slots
-    int kind;                  // 0: cells, 4 slots per bucket; 1: blocks, 2 per bucket
-    __host__ __device__ int log2bucket() const { return kind ? 1 : 2; }
-    __host__ __device__ CellSlot* cells() const { return static_cast<CellSlot*>(slots); }
+    __host__ __device__ int log2bucket() const { return 1; }
     __host__ __device__ BlockSlot* blocks() const { return static_cast<BlockSlot*>(slots); }
 };
 
@@ -171,10 +157,11 @@ __device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double
 
 // ---------------------------------------------------------------- device helpers
 // Bucketed open addressing, 64-byte buckets.  Keys are row-major with x
-// fastest, so x-adjacent cells share a group: kind 0 hashes groups of 4 keys
-// (k >> 2) into buckets of four 16-byte cell slots; kind 1 hashes blocks of
-// 8 keys (k >> 3, one 32-byte slot per block) into buckets of two.  A stencil
-// row of three cells then reads one or two buckets.  An item sits in the
+// fastest, so x-adjacent cells share a block: blocks of 8 keys (k >> 3, one
+// 32-byte slot per block) are hashed into buckets of two slots.  A stencil
+// row of three cells then reads one or two buckets.  (One 16-byte slot per
+// cell, four per bucket, measured slower in round 1: insert 0.56 vs 0.44 ms,
+// pass 1 0.80 vs 0.65 ms on C4.)  An item sits in the
 // first bucket, from its home on, that had a free slot when it was inserted
 // (no deletions), so a lookup stops at the first bucket holding it or a
 // free slot -- almost always the home bucket.
@@ -221,34 +208,20 @@ __device__ __forceinline__ ulonglong4 ld256u(const void* p) {
 
 __device__ __forceinline__ void SegSoA::load4(size_t p, double2& st, double2& sx, double2& sy,
                                               double2& sz) const {
-    if (es == 4) {
-        const double4* r = reinterpret_cast<const double4*>(rec + 4 * p);
-        const double4 a = ld256(r), b = ld256(r + 1);
-        st = make_double2(a.x, a.y);
-        sx = make_double2(a.z, a.w);
-        sy = make_double2(b.x, b.y);
-        sz = make_double2(b.z, b.w);
-    } else {
-        st = ld(0, p);
-        sx = ld(1, p);
-        sy = ld(2, p);
-        sz = ld(3, p);
-    }
+    const double4* r = reinterpret_cast<const double4*>(rec + 4 * p);
+    const double4 a = ld256(r), b = ld256(r + 1);
+    st = make_double2(a.x, a.y);
+    sx = make_double2(a.z, a.w);
+    sy = make_double2(b.x, b.y);
+    sz = make_double2(b.z, b.w);
 }
 __device__ __forceinline__ void SegSoA::store4(size_t p, double2 st, double2 sx, double2 sy,
                                                double2 sz) const {
-    if (es == 4) {
-        double* r = reinterpret_cast<double*>(rec + 4 * p);
-        asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r), "d"(st.x), "d"(st.y),
-                     "d"(sx.x), "d"(sx.y) : "memory");
-        asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r + 4), "d"(sy.x), "d"(sy.y),
-                     "d"(sz.x), "d"(sz.y) : "memory");
-    } else {
-        *at(0, p) = st;
-        *at(1, p) = sx;
-        *at(2, p) = sy;
-        *at(3, p) = sz;
-    }
+    double* r = reinterpret_cast<double*>(rec + 4 * p);
+    asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r), "d"(st.x), "d"(st.y),
+                 "d"(sx.x), "d"(sx.y) : "memory");
+    asm volatile("st.global.v4.f64 [%0], {%1,%2,%3,%4};" ::"l"(r + 4), "d"(sy.x), "d"(sy.y),
+                 "d"(sz.x), "d"(sz.y) : "memory");
 }
 
 // Monotone map of doubles to unsigned 64-bit integers (for atomic min/max).

@@ -294,89 +294,44 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     const unsigned long long key0 = make_key(g, bin, clo[0], cy, cz);
     const unsigned long long kend = key0 + (unsigned long long)cn[0];   // row keys [key0, kend)
     uint32_t first = 0xffffffffu, last = 0;
-    if (ht.kind == 1) {
-        // blocks of 8 keys: the row's keys [key0, kend) lie in blocks
-        // key0 >> 3 .. (kend - 1) >> 3, each one 32-byte slot holding the
-        // prefix counts of its 8 cells; a bucket is two slots (64 bytes)
-        const BlockSlot* slots = ht.blocks();
-        const unsigned long long bmask = ht.mask >> 1;
-        for (unsigned long long blk = key0 >> 3; blk <= (kend - 1) >> 3; ++blk) {
-            unsigned long long b = bucket_of(blk, ht);
-            ++probes;
-            while (true) {
-                const ulonglong4 h0 = ld256u(slots + 2 * b), h1 = ld256u(slots + 2 * b + 1);
-                const bool m0 = h0.x == blk, m1 = h1.x == blk;
-                if (m0 || m1) {
-                    const ulonglong4 h = m0 ? h0 : h1;
-                    const uint32_t start = (uint32_t)h.y, big = (uint32_t)(h.y >> 32);
-                    const unsigned long long base = blk << 3;
-                    const uint32_t lo = (uint32_t)((key0 > base ? key0 : base) - base);
-                    const uint32_t hi = (uint32_t)(((kend - 1) < base + 7 ? (kend - 1) : base + 7) - base);
-                    uint32_t s0, s1;
-                    if (big) {                       // the whole block (superset)
-                        s0 = start;
-                        s1 = start + (uint32_t)h.z;
-                    } else {                         // cum[j]: 16 bits at word z (j < 4) or w
-                        const uint32_t c_lo = lo == 0 ? 0u
-                            : (uint32_t)(((lo - 1) < 4 ? h.z >> (16 * (lo - 1)) : h.w >> (16 * (lo - 5))) & 0xffffull);
-                        const uint32_t c_hi =
-                            (uint32_t)((hi < 4 ? h.z >> (16 * hi) : h.w >> (16 * (hi - 4))) & 0xffffull);
-                        s0 = start + c_lo;
-                        s1 = start + c_hi;
-                    }
-                    if (s1 > s0) {
-                        first = min(first, s0);
-                        last = max(last, s1);
-                    }
-                    break;
+    // blocks of 8 keys: the row's keys [key0, kend) lie in blocks
+    // key0 >> 3 .. (kend - 1) >> 3 of this row only (nc[0] is a multiple of
+    // 8), each one 32-byte slot holding the prefix counts of its 8 cells; a
+    // bucket is two slots (64 bytes)
+    const BlockSlot* slots = ht.blocks();
+    const unsigned long long bmask = ht.mask >> 1;
+    for (unsigned long long blk = key0 >> 3; blk <= (kend - 1) >> 3; ++blk) {
+        unsigned long long b = bucket_of(blk, ht);
+        ++probes;
+        while (true) {
+            const ulonglong4 h0 = ld256u(slots + 2 * b), h1 = ld256u(slots + 2 * b + 1);
+            const bool m0 = h0.x == blk, m1 = h1.x == blk;
+            if (m0 || m1) {
+                const ulonglong4 h = m0 ? h0 : h1;
+                const uint32_t bstart = (uint32_t)h.y, big = (uint32_t)(h.y >> 32);
+                const unsigned long long base = blk << 3;
+                const uint32_t lo = (uint32_t)((key0 > base ? key0 : base) - base);
+                const uint32_t hi = (uint32_t)(((kend - 1) < base + 7 ? (kend - 1) : base + 7) - base);
+                uint32_t s0, s1;
+                if (big) {                       // the whole block (superset)
+                    s0 = bstart;
+                    s1 = bstart + (uint32_t)h.z;
+                } else {                         // cum[j]: 16 bits at word z (j < 4) or w
+                    const uint32_t c_lo = lo == 0 ? 0u
+                        : (uint32_t)(((lo - 1) < 4 ? h.z >> (16 * (lo - 1)) : h.w >> (16 * (lo - 5))) & 0xffffull);
+                    const uint32_t c_hi =
+                        (uint32_t)((hi < 4 ? h.z >> (16 * hi) : h.w >> (16 * (hi - 4))) & 0xffffull);
+                    s0 = bstart + c_lo;
+                    s1 = bstart + c_hi;
                 }
-                if (h0.x == EMPTY_KEY || h1.x == EMPTY_KEY) break;   // end of the chain
-                b = (b + 1) & bmask;
+                if (s1 > s0) {
+                    first = min(first, s0);
+                    last = max(last, s1);
+                }
+                break;
             }
-        }
-        if (first != 0xffffffffu) {
-            start = first;
-            cnt = last - first;
-        }
-        return;
-    }
-    const ulonglong2* slots = reinterpret_cast<const ulonglong2*>(ht.slots);
-    const unsigned long long bmask = ht.mask >> 2;
-    // any slot whose key lies in the row range contributes (a key met on
-    // another group's chain is found twice; min/max make that harmless);
-    // returns whether the bucket has a free slot (end of the chain)
-    auto scan_bucket = [&](const ulonglong2* B) -> bool {
-        bool empty = false;
-        // the 64-byte bucket as two 256-bit loads: slots (key, start | end << 32)
-        const ulonglong4 h0 = ld256u(B), h1 = ld256u(B + 2);
-        const unsigned long long kk[4] = {h0.x, h0.z, h1.x, h1.z};
-        const unsigned long long se[4] = {h0.y, h0.w, h1.y, h1.w};
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-            if (kk[i] - key0 < kend - key0) {      // key0 <= key < kend
-                first = min(first, (uint32_t)se[i]);
-                last = max(last, (uint32_t)(se[i] >> 32));
-            }
-            empty |= (kk[i] == EMPTY_KEY);
-        }
-        return empty;
-    };
-    const unsigned long long g0 = key0 >> 2, g1 = (kend - 1) >> 2;
-    for (unsigned long long gg = g0; gg <= g1; gg += 2) {
-        // home buckets of two groups issued together (8 x 128-bit loads)
-        const bool two = gg + 1 <= g1;
-        unsigned long long b0 = bucket_of(gg, ht);
-        unsigned long long b1 = two ? bucket_of(gg + 1, ht) : b0;
-        probes += two ? 2u : 1u;
-        bool e0 = scan_bucket(slots + 4 * b0);
-        bool e1 = two ? scan_bucket(slots + 4 * b1) : true;
-        while (!e0) {                                    // overflow chains (rare)
-            b0 = (b0 + 1) & bmask;
-            e0 = scan_bucket(slots + 4 * b0);
-        }
-        while (!e1) {
-            b1 = (b1 + 1) & bmask;
-            e1 = scan_bucket(slots + 4 * b1);
+            if (h0.x == EMPTY_KEY || h1.x == EMPTY_KEY) break;   // end of the chain
+            b = (b + 1) & bmask;
         }
     }
     if (first != 0xffffffffu) {
@@ -754,34 +709,35 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     tb.spill_all = 1;
                     launch_pass1(tb, h.c.n_over);
                 }
-                // ---- spilled records to their query segments, then each
-                //      segment sorted by entry id
+                // ---- spilled records to their query segments of a scratch
+                //      mirror of the output, then each segment sorted by
+                //      entry id into the output
+                DevBuf<dts_result> raw(h.total, s);
                 const unsigned long long n1 = std::min(std::min(h.c.spilled, spill_cap),
                                                        h.c.spill_valid);
                 if (n1) {
                     k_spill_place<<<blocks(n1, 256), 256, 0, s>>>(
-                        spill.p, n1, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p, qmap,
-                        qid_base, fin);
+                        spill.p, n1, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p, raw.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (n_raw) {
                     k_spill_place<<<blocks(n_raw, 256), 256, 0, s>>>(
-                        spill2.p, n_raw, nullptr, offsets.p, cursor.p, qmap, qid_base, fin);
+                        spill2.p, n_raw, nullptr, offsets.p, cursor.p, raw.p);
                     DTS_LAUNCH_CHECK();
                 }
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
                 DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, sizeof(unsigned int), s));
                 if (h.c.n_spill) {
-                    k_seg_sort<<<h.c.n_spill * WQ, SEG_T, 0, s>>>(spill_tiles.p, order.p,
-                                                                 (uint32_t)nq, counts.p,
-                                                                 offsets.p, fin, bigc.p, ctr.p);
+                    k_seg_sort<<<h.c.n_spill * WQ, SEG_T, 0, s>>>(
+                        spill_tiles.p, order.p, (uint32_t)nq, counts.p, offsets.p, raw.p, qmap,
+                        qid_base, fin, bigc.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
-                    k_seg_sort<<<h.c.n_over * WQ, SEG_T, 0, s>>>(over_tiles.p, order.p,
-                                                                (uint32_t)nq, counts.p,
-                                                                offsets.p, fin, bigc.p, ctr.p);
+                    k_seg_sort<<<h.c.n_over * WQ, SEG_T, 0, s>>>(
+                        over_tiles.p, order.p, (uint32_t)nq, counts.p, offsets.p, raw.p, qmap,
+                        qid_base, fin, bigc.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 unsigned int n_big = 0;
@@ -790,7 +746,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 DTS_CUDA(cudaStreamSynchronize(s));
                 if (n_big) {
                     // ---- segments longer than a CTA sort: one device-wide
-                    //      radix sort by (query, entry id) over those only
+                    //      keys-only radix sort over those only
                     DevBuf<unsigned long long> bigoff(nq + 1, s);
                     scan_exclusive_u32_to_u64(bigc.p, bigoff.p, nq, s);
                     unsigned long long nb = 0;
@@ -803,17 +759,14 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     if (qb + eb + sb > 64)
                         throw Error(DTS_ENOTSUP, "long result segments: sort key exceeds 64 bits");
                     DevBuf<unsigned long long> k1(nb, s), k2(nb, s);
-                    DevBuf<dts_result> tmp(nb, s);
                     k_big_keys<<<blocks((size_t)nq * 32, 256), 256, 0, s>>>(
-                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, fin, eb, sb, k1.p);
+                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, raw.p, eb, sb, k1.p);
                     DTS_LAUNCH_CHECK();
                     const unsigned long long* sk =
                         radix_sort_keys(k1.p, k2.p, nb, sb, sb + eb + qb, s);
-                    k_big_gather<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, offsets.p, fin,
-                                                                tmp.p);
-                    DTS_LAUNCH_CHECK();
                     k_big_place<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, bigoff.p,
-                                                               offsets.p, tmp.p, fin);
+                                                               offsets.p, raw.p, qmap, qid_base,
+                                                               fin);
                     DTS_LAUNCH_CHECK();
                 }
             }

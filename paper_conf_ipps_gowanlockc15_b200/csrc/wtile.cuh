@@ -482,48 +482,58 @@ __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ 
 
 // ------------------------------------------- spilled tiles: place + sort
 // Spilled records (query_id = local query id) go to their query's segment
-// [offsets[q], offsets[q] + counts[q]) in arrival order; records of queries
-// whose tile was re-run (cover[q] != 0) are stale and skipped.
+// [offsets[q], offsets[q] + counts[q]) of `raw` (a scratch mirror of the
+// output), in arrival order: one atomic per (warp, query) group
+// (__match_any_sync), not per record.  Records of queries whose tile was
+// re-run (cover[q] != 0) are stale and skipped.
 __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restrict__ sp,
                                                     unsigned long long n,
                                                     const uint32_t* __restrict__ cover,
                                                     const unsigned long long* __restrict__ offsets,
                                                     uint32_t* __restrict__ cursor,
-                                                    const uint32_t* __restrict__ qmap,
-                                                    uint32_t qid_base,
-                                                    dts_result* __restrict__ out) {
+                                                    dts_result* __restrict__ raw) {
     const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
-    if (k >= n) return;
-    dts_result r = sp[k];
-    const uint32_t q = r.query_id;
-    if (cover && cover[q]) return;
-    const unsigned long long pos = offsets[q] + atomicAdd(&cursor[q], 1u);
-    r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
-    out[pos] = r;
+    const int lane = threadIdx.x & 31;
+    dts_result r;
+    bool live = k < n;
+    if (live) {
+        r = sp[k];
+        if (cover && cover[r.query_id]) live = false;
+    }
+    const uint32_t q = live ? r.query_id : 0xffffffffu;
+    const uint32_t grp = __match_any_sync(0xffffffffu, q);
+    if (!live) return;
+    const int leader = __ffs(grp) - 1;
+    uint32_t base = 0;
+    if (lane == leader) base = atomicAdd(&cursor[q], (uint32_t)__popc(grp));
+    base = __shfl_sync(grp, base, leader);
+    raw[offsets[q] + base + __popc(grp & ((1u << lane) - 1u))] = r;
 }
 
-// One CTA per (listed tile, query slot): the query's segment (at most
-// SEG_CAP records) is loaded into shared memory, its (entry id, arrival
-// slot) keys are bitonic-sorted, and the records are written back in entry
-// id order (canonical; equal caller ids keep an unspecified order).  Longer
-// segments are flagged in bigc for the device-wide sort.
-constexpr int SEG_T = 128;
-constexpr int SEG_CAP = 1024;
+// One CTA per (listed tile, query slot): the (entry id, slot) keys of the
+// query's segment of `raw` (at most SEG_CAP) are bitonic-sorted in shared
+// memory and the records gathered into the output in entry id order, with
+// the reported query id (canonical; equal caller ids keep an unspecified
+// order).  Longer segments are flagged in bigc for the device-wide sort.
+constexpr int SEG_T = 256;
+constexpr int SEG_CAP = 4096;
 __global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__ tiles,
                                                    const uint32_t* __restrict__ order,
                                                    uint32_t nq,
                                                    const uint32_t* __restrict__ counts,
                                                    const unsigned long long* __restrict__ offsets,
+                                                   const dts_result* __restrict__ raw,
+                                                   const uint32_t* __restrict__ qmap,
+                                                   uint32_t qid_base,
                                                    dts_result* __restrict__ out,
                                                    uint32_t* __restrict__ bigc,
                                                    Counters* __restrict__ ctr) {
     __shared__ unsigned long long key[SEG_CAP];
-    __shared__ dts_result rec[SEG_CAP];
     const uint32_t sp = tiles[blockIdx.x / WQ] * WQ + blockIdx.x % WQ;
     if (sp >= nq) return;
     const uint32_t q = order[sp];
     const uint32_t c = counts[q];
-    if (c <= 1) return;
+    if (c == 0) return;
     if (c > (uint32_t)SEG_CAP) {
         if (threadIdx.x == 0) {
             bigc[q] = c;
@@ -531,18 +541,13 @@ __global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__
         }
         return;
     }
-    dts_result* seg = out + offsets[q];
-    uint32_t N = 2;
+    const unsigned long long off = offsets[q];
+    const dts_result* seg = raw + off;
+    const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
+    uint32_t N = 1;
     while (N < c) N <<= 1;
-    for (uint32_t i = threadIdx.x; i < N; i += SEG_T) {
-        if (i < c) {
-            const dts_result r = seg[i];
-            rec[i] = r;
-            key[i] = ((unsigned long long)r.entry_id << 32) | i;
-        } else {
-            key[i] = ~0ull;
-        }
-    }
+    for (uint32_t i = threadIdx.x; i < N; i += SEG_T)
+        key[i] = i < c ? (((unsigned long long)seg[i].entry_id << 32) | i) : ~0ull;
     __syncthreads();
     for (uint32_t k = 2; k <= N; k <<= 1) {
         for (uint32_t j = k >> 1; j > 0; j >>= 1) {
@@ -560,7 +565,11 @@ __global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__
             __syncthreads();
         }
     }
-    for (uint32_t i = threadIdx.x; i < c; i += SEG_T) seg[i] = rec[(uint32_t)(key[i] & 0xffffffffull)];
+    for (uint32_t i = threadIdx.x; i < c; i += SEG_T) {
+        dts_result r = seg[(uint32_t)(key[i] & 0xffffffffull)];
+        r.query_id = qrep;
+        out[off + i] = r;
+    }
 }
 
 // Segments longer than SEG_CAP: one device-wide keys-only radix sort of
@@ -581,28 +590,22 @@ __global__ void __launch_bounds__(256) k_big_keys(uint32_t nq, const uint32_t* _
         keys[b + i] = qk | ((unsigned long long)out[o + i].entry_id << sb) | i;
 }
 
-// tmp[k] = the record of sorted element k (read from its place in its segment)
-__global__ void __launch_bounds__(256) k_big_gather(const unsigned long long* __restrict__ keys,
-                                                   unsigned long long n, int eb, int sb,
-                                                   const unsigned long long* __restrict__ offsets,
-                                                   const dts_result* __restrict__ in,
-                                                   dts_result* __restrict__ tmp) {
+// out[k-th place of its segment] = raw[slot] of sorted element k, with the
+// reported query id
+__global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __restrict__ keys,
+                                                  unsigned long long n, int eb, int sb,
+                                                  const unsigned long long* __restrict__ bigoff,
+                                                  const unsigned long long* __restrict__ offsets,
+                                                  const dts_result* __restrict__ raw,
+                                                  const uint32_t* __restrict__ qmap,
+                                                  uint32_t qid_base,
+                                                  dts_result* __restrict__ out) {
     const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
     if (k >= n) return;
     const unsigned long long key = keys[k];
     const uint32_t q = (uint32_t)(key >> (eb + sb));
     const unsigned long long slot = key & ((1ull << sb) - 1ull);
-    tmp[k] = in[offsets[q] + slot];
-}
-
-__global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __restrict__ keys,
-                                                  unsigned long long n, int eb, int sb,
-                                                  const unsigned long long* __restrict__ bigoff,
-                                                  const unsigned long long* __restrict__ offsets,
-                                                  const dts_result* __restrict__ tmp,
-                                                  dts_result* __restrict__ out) {
-    const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
-    if (k >= n) return;
-    const uint32_t q = (uint32_t)(keys[k] >> (eb + sb));
-    out[offsets[q] + (k - bigoff[q])] = tmp[k];
+    dts_result r = raw[offsets[q] + slot];
+    r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
+    out[offsets[q] + (k - bigoff[q])] = r;
 }

@@ -105,16 +105,16 @@ def test_index_parameter_invariance_and_determinism(dts, oracle_mod):
 
 def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     """Same result bytes whatever digit plan the build's radix sort takes
-    (8-bit only, or 9-bit digits where they save a pass), whichever hash
-    (cell slots or 8-key block slots) and record layout (64-byte records or
-    four 16-byte streams) the index uses: they only change the layout."""
+    (8-bit only, or 9-bit digits where they save a pass), whichever grid
+    source (sampled + fused keys pass, or exact bounds first), hash load,
+    gather shape and pass-1 occupancy the index and search use: they only
+    change the layout and the schedule."""
     c = synth.make_config("C1", scale=0.1)
     ref = None
-    for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_KIND": "0"},
-                {"DTS_HASH_KIND": "1"}, {"DTS_LAYOUT": "soa"}, {"DTS_FUSED_KEYS": "0"},
-                {"DTS_INSERT_WALK": "0"}, {"DTS_OS_SHAPE": "0"},
-                {"DTS_GATHER": "4"},
-                {"DTS_GATHER": "1"}):
+    for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_SLOTS": "1.2"},
+                {"DTS_FUSED_KEYS": "0"}, {"DTS_OS_SHAPE": "0"}, {"DTS_GATHER": "4"},
+                {"DTS_GATHER": "1"}, {"DTS_TILE_OCC": "6"}, {"DTS_TILE_OCC": "8"},
+                {"DTS_QSORT_MIN": "0"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
         import sys
@@ -136,8 +136,8 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
 def test_crowded_cells(dts, oracle_mod):
     """Blocks of 8 cells holding more than a warp's worth of entries (the
     insert's warp path) and more than 65,535 (one run per block): parity with
-    the oracle, and the same bytes with warp-path-only inserts and with cell
-    slots."""
+    the oracle, and the same bytes with a denser hash table, the exact-bounds
+    grid and sorted queries."""
     import subprocess
     import sys
     D, Q = synth.crowded(5)
@@ -148,7 +148,7 @@ def test_crowded_cells(dts, oracle_mod):
             "paper_conf_ipps_gowanlockc15_b200 as m; D, Q = synth.crowded(5); "
             "i = m.build_index(D); r = m.search(i, Q, %r); "
             "sys.stdout.buffer.write(r.tobytes())" % (REPO, os.path.join(REPO, "tests"), d))
-    for env in ({"DTS_INSERT_WALK": "0"}, {"DTS_HASH_KIND": "0"}, {"DTS_WTILE_TMA": "32"}):
+    for env in ({"DTS_HASH_SLOTS": "1.2"}, {"DTS_FUSED_KEYS": "0"}, {"DTS_QSORT_MIN": "0"}):
         out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
                              capture_output=True, timeout=600)
         assert out.returncode == 0, out.stderr.decode()[-2000:]
