@@ -615,13 +615,22 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     }();
     auto launch_pass1 = [&](const TileArgs& args, uint32_t tiles) {
         const unsigned want = (tiles + WW - 1) / WW;
-        if (idx->method == DTS_METHOD_SUBBIN)
-            k_wtile_count<7, true, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
-        else if (idx->method == DTS_METHOD_TEMPORAL)
-            k_wtile_count<7, false, true><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
-        else if (occ == 8) k_wtile_count<8><<<std::min<unsigned>(want, nsm * 8), WT, 0, s>>>(args);
-        else if (occ == 6) k_wtile_count<6><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(args);
-        else k_wtile_count<7><<<std::min<unsigned>(want, nsm * 7), WT, 0, s>>>(args);
+        const unsigned g7 = std::min<unsigned>(want, nsm * 7);
+        if (args.excl) {                  // exclude_same_trajectory instantiations
+            if (idx->method == DTS_METHOD_SUBBIN) k_wtile_count<7, true, true, true><<<g7, WT, 0, s>>>(args);
+            else if (idx->method == DTS_METHOD_TEMPORAL) k_wtile_count<7, false, true, true><<<g7, WT, 0, s>>>(args);
+            else k_wtile_count<7, false, false, true><<<g7, WT, 0, s>>>(args);
+        } else if (idx->method == DTS_METHOD_SUBBIN) {
+            k_wtile_count<7, true, true><<<g7, WT, 0, s>>>(args);
+        } else if (idx->method == DTS_METHOD_TEMPORAL) {
+            k_wtile_count<7, false, true><<<g7, WT, 0, s>>>(args);
+        } else if (occ == 8) {
+            k_wtile_count<8><<<std::min<unsigned>(want, nsm * 8), WT, 0, s>>>(args);
+        } else if (occ == 6) {
+            k_wtile_count<6><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(args);
+        } else {
+            k_wtile_count<7><<<g7, WT, 0, s>>>(args);
+        }
         DTS_LAUNCH_CHECK();
     };
     launch_pass1(ta, ntiles);

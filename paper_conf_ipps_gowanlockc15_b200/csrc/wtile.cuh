@@ -52,6 +52,8 @@ struct WarpSmem {
     unsigned long long lkoff[WQ + 1];
     unsigned long long hkey[WH];        // (query << 42) | (position, then entry id << 10) | slot
     double h0[WH], h1[WH];
+    uint2 run[32];                      // a probe round's non-empty runs, compacted:
+                                        // (position delta, query | method index << 8)
     uint32_t nhit, over, spilled;
 };
 
@@ -162,8 +164,9 @@ __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int 
 // temporal methods compile without that indirection.  GROUP: one-run
 // queries (temporal / subbin methods) streamed per group of identical runs
 // (step 1a); the grid method compiles without it (its rare one-run
-// fallback queries go through the probe rounds).
-template <int MINB, bool SB = false, bool GROUP = false>
+// fallback queries go through the probe rounds).  EXCL: exclude pairs of
+// the same trajectory (compiled out of the plain search).
+template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -210,7 +213,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             qs.rstart = st.rstart; qs.rcnt = st.rcnt;
             S.qs[lane] = qs;
             S.qid[lane] = qid;
-            S.qtraj[lane] = (a.excl && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
+            S.qtraj[lane] = (EXCL && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
             S.qcount[lane] = 0;
             nlook = st.nlook;
             if (GROUP && st.mode == MODE_TEMPORAL && st.rcnt > 0) {   // streamed in 1a
@@ -258,16 +261,16 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     if (SB && lri) {
                         sb_load(a.sb, lri, slot, st, sx, sy, sz);
                         p = ~0u;                             // id looked up on a hit only
-                        if (a.excl) p = __ldg(sb_ids(a.sb, lri) + slot);
+                        if (EXCL) p = __ldg(sb_ids(a.sb, lri) + slot);
                     } else {
                         a.soa.load4(p, st, sx, sy, sz);
                     }
                 }
-                const uint32_t et = (a.excl && valid) ? __ldg(a.etraj + p) : 0u;
+                const uint32_t et = (EXCL && valid) ? __ldg(a.etraj + p) : 0u;
                 for (uint32_t mm = members; mm; mm &= mm - 1) {
                     const int qi = __ffs(mm) - 1;
                     double h0, h1;
-                    if (valid && !(a.excl && et == S.qtraj[qi]) &&
+                    if (valid && !(EXCL && et == S.qtraj[qi]) &&
                         refine(smem_query(S, qi), st, sx, sy, sz, d2, h0, h1)) {
                         if (p == ~0u) p = __ldg(sb_ids(a.sb, lri) + slot);
                         stage_hit(S, qi, p, h0, h1);
@@ -302,42 +305,40 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
             const unsigned long long excl = incl - cnt;
             n_cand += total;
-            // per run: the position delta start - excl (mod 2^32: a candidate's
-            // position p = t + delta fits 32 bits even when the round's total
-            // does not) and (query | method index << 8), one 32-bit shuffle
-            // each; the run search shuffles 32-bit prefixes when the total fits
-            const uint32_t delta = start - (uint32_t)excl;
-            const uint32_t qind = (uint32_t)qi | (ind << 8);
-            const bool narrow = total <= 0xffffffffull;
-            const uint32_t incl32 = (uint32_t)incl;
+            // the round's non-empty runs, compacted into shared memory:
+            // (position delta start - excl mod 2^32, query | method index <<
+            // 8); a candidate t lies in run r = (non-empty runs starting at
+            // or before t) - 1, counted with one OR-reduction of the run
+            // starts per 32 candidates -- no per-candidate search
+            const bool ne = cnt > 0;
+            const uint32_t lt = (1u << lane) - 1u;
+            if (ne) {
+                const uint32_t ci = __popc(__ballot_sync(0xffffffffu, ne) & lt);
+                S.run[ci] = make_uint2(start - (uint32_t)excl, (uint32_t)qi | (ind << 8));
+            } else {
+                __ballot_sync(0xffffffffu, ne);
+            }
+            __syncwarp();
+            uint32_t before = 0;          // non-empty runs starting before `base`
             for (unsigned long long base = 0; base < total; base += 64) {
+                const unsigned long long d1 = excl - base, d2 = d1 - 32;
+                const uint32_t m1 = __reduce_or_sync(0xffffffffu, (ne && excl >= base && d1 < 32)
+                                                                      ? 1u << (uint32_t)d1 : 0u);
+                const uint32_t m2 = __reduce_or_sync(
+                    0xffffffffu, (ne && excl >= base + 32 && d2 < 32) ? 1u << (uint32_t)d2 : 0u);
+                const uint32_t r1 = min(before + __popc(m1 & (lt | (1u << lane))) - 1u, 31u);
+                before += __popc(m1);
+                const uint32_t r2 = min(before + __popc(m2 & (lt | (1u << lane))) - 1u, 31u);
+                before += __popc(m2);
                 const unsigned long long t1 = base + lane, t2 = t1 + 32;
-                int j1 = 0, j2 = 0;
-                if (narrow) {
-                    const uint32_t u1 = (uint32_t)t1, u2 = (uint32_t)t2;
-#pragma unroll
-                    for (int step = 16; step; step >>= 1) {
-                        if (__shfl_sync(0xffffffffu, incl32, j1 + step - 1) <= u1) j1 += step;
-                        if (__shfl_sync(0xffffffffu, incl32, j2 + step - 1) <= u2) j2 += step;
-                    }
-                } else {
-#pragma unroll
-                    for (int step = 16; step; step >>= 1) {
-                        if (__shfl_sync(0xffffffffu, incl, j1 + step - 1) <= t1) j1 += step;
-                        if (__shfl_sync(0xffffffffu, incl, j2 + step - 1) <= t2) j2 += step;
-                    }
-                }
-                const uint32_t dl1 = __shfl_sync(0xffffffffu, delta, j1);
-                const uint32_t dl2 = __shfl_sync(0xffffffffu, delta, j2);
-                const uint32_t qx1 = __shfl_sync(0xffffffffu, qind, j1);
-                const uint32_t qx2 = __shfl_sync(0xffffffffu, qind, j2);
-                const int qi1 = (int)(qx1 & 0xffu), qi2 = (int)(qx2 & 0xffu);
-                const uint32_t i1 = SB ? qx1 >> 8 : 0u, i2 = SB ? qx2 >> 8 : 0u;
                 const bool v1 = t1 < total, v2 = t2 < total;
                 if (v1) {
-                    uint32_t p1 = (uint32_t)t1 + dl1;
-                    uint32_t p2 = v2 ? (uint32_t)t2 + dl2 : p1;
-                    const uint32_t i2v = v2 ? i2 : i1;
+                    const uint2 ru1 = S.run[r1];
+                    const uint2 ru2 = v2 ? S.run[r2] : ru1;
+                    const int qi1 = (int)(ru1.y & 0xffu), qi2 = (int)(ru2.y & 0xffu);
+                    const uint32_t i1 = SB ? ru1.y >> 8 : 0u, i2 = SB ? ru2.y >> 8 : 0u;
+                    uint32_t p1 = (uint32_t)t1 + ru1.x;
+                    uint32_t p2 = v2 ? (uint32_t)t2 + ru2.x : p1;
                     const uint32_t sl1 = p1, sl2 = p2;      // subbin slots (when i != 0)
                     if (i1) p1 = __ldg(sb_ids(a.sb, i1) + sl1);   // id -> sorted position
                     if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + sl2);
@@ -345,11 +346,11 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     double2 st1, sx1, sy1, sz1, st2, sx2, sy2, sz2;
                     if (i1) sb_load(a.sb, i1, sl1, st1, sx1, sy1, sz1);   // contiguous copy
                     else a.soa.load4(p1, st1, sx1, sy1, sz1);
-                    if (i2v) sb_load(a.sb, i2v, v2 ? sl2 : sl1, st2, sx2, sy2, sz2);
+                    if (i2) sb_load(a.sb, i2, sl2, st2, sx2, sy2, sz2);
                     else a.soa.load4(p2, st2, sx2, sy2, sz2);
                     double h0, h1;
-                    const bool x1 = a.excl && __ldg(a.etraj + p1) == S.qtraj[qi1];
-                    const bool x2 = a.excl && __ldg(a.etraj + p2) == S.qtraj[qi2];
+                    const bool x1 = EXCL && __ldg(a.etraj + p1) == S.qtraj[qi1];
+                    const bool x2 = EXCL && __ldg(a.etraj + p2) == S.qtraj[qi2];
                     if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
                         stage_hit(S, qi1, p1, h0, h1);
                     if (v2 && !x2 &&
