@@ -312,12 +312,9 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             // starts per 32 candidates -- no per-candidate search
             const bool ne = cnt > 0;
             const uint32_t lt = (1u << lane) - 1u;
-            if (ne) {
-                const uint32_t ci = __popc(__ballot_sync(0xffffffffu, ne) & lt);
-                S.run[ci] = make_uint2(start - (uint32_t)excl, (uint32_t)qi | (ind << 8));
-            } else {
-                __ballot_sync(0xffffffffu, ne);
-            }
+            const uint32_t nemask = __ballot_sync(0xffffffffu, ne);
+            if (ne) S.run[__popc(nemask & lt)] = make_uint2(start - (uint32_t)excl,
+                                                            (uint32_t)qi | (ind << 8));
             __syncwarp();
             uint32_t before = 0;          // non-empty runs starting before `base`
             for (unsigned long long base = 0; base < total; base += 64) {
