@@ -318,11 +318,12 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             __syncwarp();
             uint32_t before = 0;          // non-empty runs starting before `base`
             for (unsigned long long base = 0; base < total; base += 64) {
-                const unsigned long long d1 = excl - base, d2 = d1 - 32;
-                const uint32_t m1 = __reduce_or_sync(0xffffffffu, (ne && excl >= base && d1 < 32)
-                                                                      ? 1u << (uint32_t)d1 : 0u);
+                // run-start offsets inside the two 32-candidate halves
+                const unsigned long long o1 = excl - base, o2 = o1 - 32;
+                const uint32_t m1 = __reduce_or_sync(0xffffffffu, (ne && excl >= base && o1 < 32)
+                                                                      ? 1u << (uint32_t)o1 : 0u);
                 const uint32_t m2 = __reduce_or_sync(
-                    0xffffffffu, (ne && excl >= base + 32 && d2 < 32) ? 1u << (uint32_t)d2 : 0u);
+                    0xffffffffu, (ne && excl >= base + 32 && o2 < 32) ? 1u << (uint32_t)o2 : 0u);
                 const uint32_t r1 = min(before + __popc(m1 & (lt | (1u << lane))) - 1u, 31u);
                 before += __popc(m1);
                 const uint32_t r2 = min(before + __popc(m2 & (lt | (1u << lane))) - 1u, 31u);
