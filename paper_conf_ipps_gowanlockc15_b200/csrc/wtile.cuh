@@ -402,11 +402,15 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     // rank inside the query: hits with a smaller entry id,
                     // ties (equal caller ids) broken by stage slot, so every
                     // slot of the tile's range is written exactly once
+                    // (a query with one staged hit -- most of them on the
+                    // galaxy workloads -- has rank 0)
                     uint32_t rank = 0;
-                    for (uint32_t j = 0; j < nh; ++j) {
-                        const unsigned long long kj = S.hkey[j];
-                        const uint32_t ej = (uint32_t)(kj >> 10);
-                        rank += ((uint32_t)(kj >> 42) == q && (ej < e || (ej == e && j < i))) ? 1u : 0u;
+                    if (S.qcount[q] > 1u) {
+                        for (uint32_t j = 0; j < nh; ++j) {
+                            const unsigned long long kj = S.hkey[j];
+                            const uint32_t ej = (uint32_t)(kj >> 10);
+                            rank += ((uint32_t)(kj >> 42) == q && (ej < e || (ej == e && j < i))) ? 1u : 0u;
+                        }
                     }
                     const uint32_t slot = (uint32_t)(k & 1023ull);
                     dts_result r;
