@@ -197,6 +197,44 @@ dts_status dts_search_device_ex(const dts_index* index,
                                 dts_result** out_results_dev, size_t* out_count,
                                 dts_search_stats* stats);         /* may be NULL */
 
+/* Count-only search (P:L32's result set, counted, not materialised): the
+ * number of results of every query of Q (host, copied) at distance d, with
+ * the same options as dts_search_ex (query_ids / query_id_base do not
+ * matter for counting).  counts: host array of nq uint32 (may be NULL);
+ * *total: the sum.  Runs the candidate generation and fp64 refinement of the
+ * search without keeping any hit, so it works for
+ * any result size (S2 at d = 5: 7.5e9 results, the paper's largest).
+ * Errors as dts_search_ex.  Synchronous. */
+dts_status dts_search_count(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                            const dts_search_options* opts, void* cuda_stream,
+                            uint32_t* counts, uint64_t* total, dts_search_stats* stats);
+
+/* dts_search_count on device Q (16-byte aligned); counts_dev: device array of
+ * nq uint32 (may be NULL); option pointers in device memory. */
+dts_status dts_search_count_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                   double d, const dts_search_options* opts, void* cuda_stream,
+                                   uint32_t* counts_dev, uint64_t* total,
+                                   dts_search_stats* stats);
+
+/* Receives one chunk of results (library-owned pinned memory, valid only
+ * during the call); return 0 to continue, nonzero to stop the search. */
+typedef int (*dts_result_callback)(const dts_result* results, size_t count, void* user);
+
+/* Streamed search of host Q for result sets larger than device or host
+ * memory -- the paper processes Q incrementally when its result buffer
+ * fills: a count pass, then contiguous query-id chunks of
+ * at most chunk_results results (0 = auto, from free device memory; a single
+ * query with more results is one chunk) are searched and handed to callback
+ * in canonical (query_id, entry_id) order, so the concatenation of all
+ * chunks is exactly dts_search_ex's output.  Options as dts_search_ex (host
+ * pointers).  stats->results = results delivered.  Errors as dts_search_ex;
+ * DTS_EINVAL for a NULL callback.  Synchronous; the callback runs on the
+ * calling thread. */
+dts_status dts_search_stream(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                             const dts_search_options* opts, uint64_t chunk_results,
+                             dts_result_callback callback, void* user, void* cuda_stream,
+                             dts_search_stats* stats);
+
 /* Trajectory-level results from segment-level ones, all in device memory:
  * every result (q, l, [t_s, t_e]) is mapped to (query_traj[q], entry_traj[l])
  * (query_traj indexed by reported query id, n_query_ids entries; entry_traj by

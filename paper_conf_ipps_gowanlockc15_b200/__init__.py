@@ -32,7 +32,8 @@ EXPORTED_SYMBOLS = (
     "dts_search_device", "dts_free_results", "dts_free_results_device", "dts_free_index",
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
     "dts_search_device_ex", "dts_canonicalize_device", "dts_merge_trajectories_device",
-    "dts_query_costs_device",
+    "dts_query_costs_device", "dts_search_count", "dts_search_count_device",
+    "dts_search_stream",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -59,6 +60,10 @@ class SearchOptions(ctypes.Structure):
 
 
 METHODS = {"grid": 0, "temporal": 1, "subbin": 2}
+
+# int callback(const dts_result* results, size_t count, void* user)
+RESULT_CALLBACK = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t,
+                                   ctypes.c_void_p)
 
 TRAJ_DTYPE = np.dtype([("query_traj", "<u4"), ("entry_traj", "<u4"),
                        ("t_start", "<f8"), ("t_end", "<f8")], align=True)
@@ -124,6 +129,19 @@ def load():
     lib.dts_merge_trajectories_device.argtypes = [P, S, P, S, P, S, P, pp, ps]
     lib.dts_merge_trajectories_device.restype = ctypes.c_int
     lib.dts_search_device_ex.restype = ctypes.c_int
+    lib.dts_search_count.argtypes = [P, P, S, ctypes.c_double, ctypes.POINTER(SearchOptions), P,
+                                     P, ctypes.POINTER(ctypes.c_uint64),
+                                     ctypes.POINTER(SearchStats)]
+    lib.dts_search_count.restype = ctypes.c_int
+    lib.dts_search_count_device.argtypes = [P, P, S, ctypes.c_double,
+                                            ctypes.POINTER(SearchOptions), P, P,
+                                            ctypes.POINTER(ctypes.c_uint64),
+                                            ctypes.POINTER(SearchStats)]
+    lib.dts_search_count_device.restype = ctypes.c_int
+    lib.dts_search_stream.argtypes = [P, P, S, ctypes.c_double, ctypes.POINTER(SearchOptions),
+                                      ctypes.c_uint64, RESULT_CALLBACK, P, P,
+                                      ctypes.POINTER(SearchStats)]
+    lib.dts_search_stream.restype = ctypes.c_int
     lib.dts_query_costs_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, P]
     lib.dts_query_costs_device.restype = ctypes.c_int
     lib.dts_canonicalize_device.argtypes = [P, S, P]
@@ -373,6 +391,86 @@ def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=
                                         ctypes.c_void_p(_stream_ptr(stream)),
                                         ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
     return DeviceResults(out.value or 0, cnt.value, index.device), st.as_dict()
+
+
+def _options(query_id_base=0, query_ids=None, query_traj=None, exclude_same_trajectory=False):
+    return SearchOptions(int(query_id_base), query_ids, query_traj,
+                         1 if exclude_same_trajectory else 0)
+
+
+def search_count(index: Index, Q, d: float, query_traj=None,
+                 exclude_same_trajectory: bool = False, stream=None, time_kernels=False):
+    """dts_search_count: host Q -> (total, per-query counts uint32 array, stats)."""
+    lib = load()
+    Q = _segments(Q)
+    qtraj = _u32_host(query_traj, Q.shape[0], "query_traj")
+    opts = _options(0, None, qtraj.ctypes.data if qtraj is not None else None,
+                    exclude_same_trajectory)
+    counts = np.empty(Q.shape[0], dtype=np.uint32)
+    total = ctypes.c_uint64()
+    st = SearchStats()
+    st.time_kernels = 1 if time_kernels else 0
+    _check(lib.dts_search_count(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
+                                float(d), ctypes.byref(opts),
+                                ctypes.c_void_p(_stream_ptr(stream)),
+                                counts.ctypes.data if Q.size else None, ctypes.byref(total),
+                                ctypes.byref(st)))
+    return int(total.value), counts, st.as_dict()
+
+
+def search_count_device(index: Index, Q_dev, d: float, counts_out=None, stream=None,
+                        time_kernels=False):
+    """dts_search_count_device: CUDA Q -> (total, CUDA int32 counts tensor, stats)."""
+    import torch
+    lib = load()
+    nq = int(Q_dev.shape[0])
+    if counts_out is None:
+        counts_out = torch.empty(nq, dtype=torch.int32, device=Q_dev.device)
+    total = ctypes.c_uint64()
+    st = SearchStats()
+    st.time_kernels = 1 if time_kernels else 0
+    opts = _options()
+    _check(lib.dts_search_count_device(index.handle, ctypes.c_void_p(Q_dev.data_ptr() if nq else 0),
+                                       nq, float(d), ctypes.byref(opts),
+                                       ctypes.c_void_p(_stream_ptr(stream)),
+                                       ctypes.c_void_p(counts_out.data_ptr() if nq else 0),
+                                       ctypes.byref(total), ctypes.byref(st)))
+    return int(total.value), counts_out, st.as_dict()
+
+
+def search_stream(index: Index, Q, d: float, callback, chunk_results: int = 0,
+                  query_id_base: int = 0, query_ids=None, query_traj=None,
+                  exclude_same_trajectory: bool = False, stream=None):
+    """dts_search_stream: host Q; `callback(chunk)` receives each chunk of
+    results in canonical order as a numpy structured view of library memory,
+    valid only during the call (copy what must outlive it); returning True
+    stops the search.  Returns the stats dict."""
+    lib = load()
+    Q = _segments(Q)
+    qids = _u32_host(query_ids, Q.shape[0], "query_ids")
+    qtraj = _u32_host(query_traj, Q.shape[0], "query_traj")
+    opts = _options(query_id_base, qids.ctypes.data if qids is not None else None,
+                    qtraj.ctypes.data if qtraj is not None else None, exclude_same_trajectory)
+    errors = []
+
+    def trampoline(ptr, count, _user):
+        try:
+            buf = (ctypes.c_char * (count * RESULT_DTYPE.itemsize)).from_address(ptr)
+            stop = callback(np.frombuffer(buf, dtype=RESULT_DTYPE, count=count))
+            return 1 if stop else 0
+        except BaseException as e:          # surfaced after the call
+            errors.append(e)
+            return 1
+
+    cb = RESULT_CALLBACK(trampoline)
+    st = SearchStats()
+    rc = lib.dts_search_stream(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
+                               float(d), ctypes.byref(opts), int(chunk_results), cb, None,
+                               ctypes.c_void_p(_stream_ptr(stream)), ctypes.byref(st))
+    if errors:
+        raise errors[0]
+    _check(rc)
+    return st.as_dict()
 
 
 def query_costs_device(index: Index, Q_dev, d: float, block: int = 1, stream=None, out=None):

@@ -466,6 +466,120 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
     return st;
 }
 
+// Count-only search of host or device Q: per-query counts (device buffer,
+// optional copy out) and the total.
+void count_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                  const dts_search_options* opts, cudaStream_t s, bool host_q,
+                  uint32_t* counts_host, uint32_t* counts_dev_out, uint64_t* total,
+                  dts_search_stats* stats) {
+    const uint32_t* qtraj = opts ? opts->query_traj : nullptr;
+    const bool excl = opts && opts->exclude_same_trajectory;
+    DevBuf<dts_segment> dQ(host_q ? nq : 0, s);
+    DevBuf<uint32_t> dtraj(host_q && qtraj && nq ? nq : 0, s), cnt(nq, s);
+    const dts_segment* Qd = Q;
+    if (host_q && nq) {
+        DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment), cudaMemcpyHostToDevice, s));
+        Qd = dQ.p;
+        if (qtraj) {
+            DTS_CUDA(cudaMemcpyAsync(dtraj.p, qtraj, nq * sizeof(uint32_t),
+                                     cudaMemcpyHostToDevice, s));
+            qtraj = dtraj.p;
+        }
+    }
+    SearchOut so;
+    search_device(index, Qd, nq, d, 0, s, &so, stats, ~0ull, nullptr, qtraj, excl, true,
+                  counts_dev_out ? counts_dev_out : cnt.p);
+    if (counts_host && nq) {
+        DTS_CUDA(cudaMemcpyAsync(counts_host, counts_dev_out ? counts_dev_out : cnt.p,
+                                 nq * sizeof(uint32_t), cudaMemcpyDeviceToHost, s));
+    }
+    DTS_CUDA(cudaStreamSynchronize(s));
+    *total = so.count;
+}
+
+// Streamed search of host Q: a count pass plans contiguous query-id chunks of
+// at most `chunk_results` results; each chunk is searched, copied to a pinned
+// buffer and handed to the callback in canonical order (chunk-order
+// concatenation is the canonical order).  Results never exist in full
+// anywhere: the paper's incremental processing of Q.
+void stream_common(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                   const dts_search_options* opts, uint64_t chunk_results,
+                   dts_result_callback cb, void* user, cudaStream_t s,
+                   dts_search_stats* stats) {
+    const uint32_t qid_base = opts ? opts->query_id_base : 0;
+    const uint32_t* qmap_h = opts ? opts->query_ids : nullptr;
+    const uint32_t* qtraj_h = opts ? opts->query_traj : nullptr;
+    const bool excl = opts && opts->exclude_same_trajectory;
+    DevBuf<dts_segment> dQ(nq, s);
+    DevBuf<uint32_t> dmap(qmap_h && nq ? nq : 0, s), dtraj(qtraj_h && nq ? nq : 0, s);
+    if (nq) DTS_CUDA(cudaMemcpyAsync(dQ.p, Q, nq * sizeof(dts_segment), cudaMemcpyHostToDevice, s));
+    if (dmap.p) DTS_CUDA(cudaMemcpyAsync(dmap.p, qmap_h, nq * 4, cudaMemcpyHostToDevice, s));
+    if (dtraj.p) DTS_CUDA(cudaMemcpyAsync(dtraj.p, qtraj_h, nq * 4, cudaMemcpyHostToDevice, s));
+    std::vector<uint32_t> counts(nq);
+    DevBuf<uint32_t> dcnt(nq, s);
+    dts_search_stats cst{};
+    SearchOut so;
+    search_device(index, dQ.p, nq, d, 0, s, &so, &cst, ~0ull, nullptr, dtraj.p, excl, true,
+                  dcnt.p);
+    if (nq) {
+        DTS_CUDA(cudaMemcpyAsync(counts.data(), dcnt.p, nq * 4, cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+    }
+    if (chunk_results == 0) {
+        size_t free_b = 0, total_b = 0;
+        DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
+        chunk_results = std::max<uint64_t>(1, std::min<uint64_t>(uint64_t(1) << 27,
+                                                                 (uint64_t)(0.25 * free_b / 96.0)));
+    }
+    // pinned landing buffer: the largest chunk (a single query may exceed
+    // chunk_results; it is then a chunk of its own)
+    uint64_t biggest = 0;
+    {
+        size_t a = 0;
+        while (a < nq) {
+            size_t b = a;
+            uint64_t acc = 0;
+            while (b < nq && (b == a || acc + counts[b] <= chunk_results)) acc += counts[b++];
+            biggest = std::max(biggest, acc);
+            a = b;
+        }
+    }
+    dts_result* hbuf = nullptr;
+    if (biggest) hbuf = static_cast<dts_result*>(pinned_alloc(biggest * sizeof(dts_result)));
+    dts_search_stats agg = cst;
+    agg.results = 0;
+    try {
+        size_t a = 0;
+        while (a < nq) {
+            size_t b = a;
+            uint64_t acc = 0;
+            while (b < nq && (b == a || acc + counts[b] <= chunk_results)) acc += counts[b++];
+            if (acc) {
+                SearchOut co;
+                search_device(index, dQ.p + a, b - a, d, qid_base + (uint32_t)a, s, &co, nullptr,
+                              ~0ull, dmap.p ? dmap.p + a : nullptr, dtraj.p ? dtraj.p + a : nullptr,
+                              excl);
+                if (co.count != acc) {
+                    cache_free(co.results);
+                    throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
+                }
+                DTS_CUDA(cudaMemcpyAsync(hbuf, co.results, acc * sizeof(dts_result),
+                                         cudaMemcpyDeviceToHost, s));
+                DTS_CUDA(cudaStreamSynchronize(s));
+                cache_free(co.results);
+                agg.results += acc;
+                if (cb(hbuf, (size_t)acc, user) != 0) break;      // the caller stops early
+            }
+            a = b;
+        }
+    } catch (...) {
+        pinned_free(hbuf);
+        throw;
+    }
+    pinned_free(hbuf);
+    if (stats) *stats = agg;
+}
+
 }  // namespace
 }  // namespace dts
 
@@ -529,6 +643,62 @@ dts_status dts_merge_trajectories_device(const dts_result* results_dev, size_t n
         *out_count = c;
     }
     return st;
+}
+
+dts_status dts_search_count(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                            const dts_search_options* opts, void* cuda_stream,
+                            uint32_t* counts, uint64_t* total, dts_search_stats* stats) {
+    if (total) *total = 0;
+    DeviceGuard dg;
+    return guarded([&] {
+        if (!index) throw Error(DTS_EINVAL, "index is NULL");
+        if (!total) throw Error(DTS_EINVAL, "total is NULL");
+        if (nq > 0 && !Q) throw Error(DTS_EINVAL, "Q is NULL with nq > 0");
+        if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
+        if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
+        prepare_device(index->device);
+        count_common(index, Q, nq, d, opts, static_cast<cudaStream_t>(cuda_stream), true, counts,
+                     nullptr, total, stats);
+    });
+}
+
+dts_status dts_search_count_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                   double d, const dts_search_options* opts, void* cuda_stream,
+                                   uint32_t* counts_dev, uint64_t* total,
+                                   dts_search_stats* stats) {
+    if (total) *total = 0;
+    DeviceGuard dg;
+    return guarded([&] {
+        if (!index) throw Error(DTS_EINVAL, "index is NULL");
+        if (!total) throw Error(DTS_EINVAL, "total is NULL");
+        if (nq > 0 && !Q_dev) throw Error(DTS_EINVAL, "Q_dev is NULL with nq > 0");
+        if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
+        if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
+        prepare_device(index->device);
+        if (nq) check_aligned(Q_dev, "Q_dev");
+        count_common(index, Q_dev, nq, d, opts, static_cast<cudaStream_t>(cuda_stream), false,
+                     nullptr, counts_dev, total, stats);
+    });
+}
+
+dts_status dts_search_stream(const dts_index* index, const dts_segment* Q, size_t nq, double d,
+                             const dts_search_options* opts, uint64_t chunk_results,
+                             dts_result_callback callback, void* user, void* cuda_stream,
+                             dts_search_stats* stats) {
+    DeviceGuard dg;
+    return guarded([&] {
+        if (!index) throw Error(DTS_EINVAL, "index is NULL");
+        if (!callback) throw Error(DTS_EINVAL, "callback is NULL");
+        if (nq > 0 && !Q) throw Error(DTS_EINVAL, "Q is NULL with nq > 0");
+        if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
+        const uint32_t base = opts ? opts->query_id_base : 0;
+        if ((uint64_t)base + nq > (uint64_t(1) << 32))
+            throw Error(DTS_EINVAL, "query_id_base + nq exceeds 2^32");
+        if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
+        prepare_device(index->device);
+        stream_common(index, Q, nq, d, opts, chunk_results, callback, user,
+                      static_cast<cudaStream_t>(cuda_stream), stats);
+    });
 }
 
 dts_status dts_query_costs_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,

@@ -357,7 +357,8 @@ struct ResultsTooLarge : Error {
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
                    unsigned long long max_results = ~0ull, const uint32_t* qmap = nullptr,
-                   const uint32_t* qtraj = nullptr, bool exclude_same_traj = false);
+                   const uint32_t* qtraj = nullptr, bool exclude_same_traj = false,
+                   bool count_only = false, uint32_t* counts_out = nullptr);
 // Per-query candidate counts summed per block of `block` queries (search.cu).
 void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                         uint32_t block, unsigned long long* out, cudaStream_t s);

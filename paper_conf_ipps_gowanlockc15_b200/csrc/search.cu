@@ -466,7 +466,8 @@ struct EventTimer {
 void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                    uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
                    unsigned long long max_results, const uint32_t* qmap,
-                   const uint32_t* qtraj, bool exclude_same_traj) {
+                   const uint32_t* qtraj, bool exclude_same_traj, bool count_only,
+                   uint32_t* counts_out) {
     out->results = nullptr;
     out->count = 0;
     dts_search_stats local{};
@@ -486,6 +487,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         DTS_CUDA(cudaMemcpyAsync(&hc, ctr.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         if (hc.bad) throw Error(DTS_EINVAL, "invalid query segment (non-finite or t_end < t_start)");
+        if (count_only && counts_out) {
+            DTS_CUDA(cudaMemsetAsync(counts_out, 0, nq * sizeof(uint32_t), s));
+            DTS_CUDA(cudaStreamSynchronize(s));
+        }
         if (stats) *stats = local;
         return;
     }
@@ -588,6 +593,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.tile_list = nullptr;
     ta.n_list = 0;
     ta.spill_all = 0;
+    ta.count_only = count_only ? 1u : 0u;
     ta.qid_base = qid_base;
     ta.qmap = qmap;
     ta.etraj = idx->etraj;
@@ -653,6 +659,22 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     local.cell_lookups = h.c.lookups;
     local.results = h.total;
     local.max_results_per_query = h.c.max_count;
+    if (count_only) {                   // counts and total only (dts_search_count)
+        if (counts_out && nq)
+            DTS_CUDA(cudaMemcpyAsync(counts_out, counts.p, nq * sizeof(uint32_t),
+                                     cudaMemcpyDefault, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        out->count = (size_t)h.total;
+        tm.mark();
+        tm.mark();
+        if (local.time_kernels) {
+            local.ms_prep = tm.ms(0);
+            local.ms_count = tm.ms(1);
+            local.ms_scan = tm.ms(2);
+        }
+        if (stats) *stats = local;
+        return;
+    }
     if (h.c.n_over) {
         // the spill buffer filled: size the next search's from this output
         unsigned long long want = h.total + (1ull << 20), cur = idx->spill_hint.load();

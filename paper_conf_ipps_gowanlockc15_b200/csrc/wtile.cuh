@@ -80,6 +80,7 @@ struct TileArgs {
     const uint32_t* tile_list;         // re-run: the tiles to process (else 0..ntiles-1)
     uint32_t n_list;
     uint32_t spill_all;                // re-run: every hit is spilled
+    uint32_t count_only;               // per-query counts only (no hit is kept)
     uint32_t qid_base;
     const uint32_t* qmap;              // optional reported query ids (else qid + qid_base)
     const uint32_t* etraj;             // trajectory id per sorted entry position
@@ -224,7 +225,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 ri = st.rind;
             }
         }
-        if (lane == 0) { S.nhit = 0; S.over = 0; S.spilled = 0; S.lkoff[0] = 0; }
+        if (lane == 0) { S.nhit = 0; S.over = a.count_only; S.spilled = 0; S.lkoff[0] = 0; }
         {
             unsigned long long inc = nlook;
 #pragma unroll
@@ -425,7 +426,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         } else if (!over && lane == 0) {
             a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
         }
-        if (over && !a.spill_all && lane == 0) {
+        if (over && !a.spill_all && !a.count_only && lane == 0) {
             a.tile_base[wt] = NONE;
             a.over_tiles[atomicAdd(&a.ctr->n_over, 1u)] = wt;
         }

@@ -193,3 +193,43 @@ def test_multirank_libdts_on_one_gpu(dts, tmp_path):
     assert prev_hi == c.Q.shape[0]
     assert out.tobytes() == ref.tobytes()
     assert np.load(tmp_path / "temporal.npy").tobytes() == ref.tobytes()
+
+
+def test_search_count_and_stream(dts, oracle_mod):
+    """Count-only search (per-query counts, total) and the streamed search
+    (canonical chunks through a callback) agree with the materialised
+    search byte for byte; a query with more results than a chunk is a chunk
+    of its own; the callback can stop the search."""
+    import torch
+    c = synth.make_config("C2", scale=0.01)
+    idx = dts.build_index(c.D, entry_traj=c.etraj)
+    for d, excl in ((2.0, False), (8.0, False), (2.0, True)):
+        kw = dict(query_traj=c.qtraj, exclude_same_trajectory=True) if excl else {}
+        ref, _ = dts.search_ex(idx, c.Q, d, **kw)
+        total, counts, st = dts.search_count(idx, c.Q, d, **kw)
+        assert total == ref.shape[0] == int(counts.sum())
+        assert np.array_equal(counts, np.bincount(ref["query_id"], minlength=c.Q.shape[0]))
+        chunks = []
+        st = dts.search_stream(idx, c.Q, d, lambda ch: chunks.append(ch.copy()),
+                               chunk_results=max(1, int(counts.max()) // 2),
+                               query_id_base=0, **kw)
+        got = np.concatenate(chunks)
+        assert got.tobytes() == ref.tobytes()
+        assert st["results"] == ref.shape[0]
+        assert max(ch.shape[0] for ch in chunks) <= max(int(counts.max()), int(counts.max()) // 2)
+    # device count, and an early stop after the first chunk
+    idd = dts.build_index_device(torch.from_numpy(c.D).cuda())
+    total_d, counts_d, _ = dts.search_count_device(idd, torch.from_numpy(c.Q).cuda(), 2.0)
+    ref = dts.search(idx, c.Q, 2.0)
+    assert total_d == ref.shape[0]
+    assert np.array_equal(counts_d.cpu().numpy().astype(np.uint32),
+                          np.bincount(ref["query_id"], minlength=c.Q.shape[0]))
+    seen = []
+    dts.search_stream(idx, c.Q, 2.0, lambda ch: seen.append(ch.shape[0]) or True, chunk_results=50)
+    assert len(seen) == 1
+    # oracle parity of the streamed output on a sample
+    qs = np.arange(0, c.Q.shape[0], 23)
+    parity.compare(parity.restrict(ref, qs), oracle_mod.search_queries(c.D, c.Q, qs, 2.0),
+                   c.D, c.Q, 2.0, oracle_mod)
+    idx.free()
+    idd.free()
