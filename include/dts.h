@@ -85,7 +85,13 @@ typedef struct {
     uint32_t temporal_bins;     /* m of P:L76; 0 = bin width = max segment duration    */
     uint32_t cells_per_dim;     /* grid resolution cap per axis; 0 = from extents     */
     double   d_hint;            /* typical search distance, sizes grid cells; 0 = none */
-    uint64_t mem_budget_bytes;  /* reserved (0 = free HBM)                             */
+    uint64_t mem_budget_bytes;  /* device bytes the index may use (0 = no limit).  When
+                                   dts_build_index's estimate for D (~310 B per entry)
+                                   exceeds it, D is split by t_start into temporal
+                                   shards kept in pinned host memory, each indexed on
+                                   the device in turn at search time; results are the
+                                   same.  Ignored by
+                                   dts_build_index_device (D is already resident).   */
     uint32_t method;            /* dts_method                                          */
     uint32_t subbins;           /* v of P:L87 per dimension (SUBBIN); 0 = 16, always
                                    capped so a subbin is wider than the largest
@@ -300,6 +306,8 @@ typedef struct {
                                    of 8 consecutive cell keys (the only kind) */
     uint64_t hash_items;        /* slots in use (blocks)                     */
     uint64_t hash_bytes;        /* table size in bytes                       */
+    uint32_t shards;            /* temporal shards on the host (mem_budget_bytes
+                                   exceeded), 0 for an index resident on the device */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

@@ -88,7 +88,8 @@ class IndexInfo(ctypes.Structure):
                 ("method", ctypes.c_uint32), ("subbins", ctypes.c_uint32 * 3),
                 ("subbin_ids", ctypes.c_uint64 * 3), ("ms_phase", ctypes.c_float * 5),
                 ("build_flags", ctypes.c_uint32), ("hash_kind", ctypes.c_uint32),
-                ("hash_items", ctypes.c_uint64), ("hash_bytes", ctypes.c_uint64)]
+                ("hash_items", ctypes.c_uint64), ("hash_bytes", ctypes.c_uint64),
+                ("shards", ctypes.c_uint32)]
 
     def as_dict(self):
         out = {}
@@ -181,10 +182,11 @@ def _segments(a) -> np.ndarray:
 
 
 def _params(device=0, temporal_bins=0, cells_per_dim=0, d_hint=0.0, method="grid",
-            subbins=0, entry_ids_ptr=None, entry_traj_ptr=None) -> IndexParams:
+            subbins=0, entry_ids_ptr=None, entry_traj_ptr=None,
+            mem_budget_bytes=0) -> IndexParams:
     m = METHODS[method] if isinstance(method, str) else int(method)
-    return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint), 0,
-                       m, int(subbins), entry_ids_ptr, entry_traj_ptr)
+    return IndexParams(int(device), int(temporal_bins), int(cells_per_dim), float(d_hint),
+                       int(mem_budget_bytes), m, int(subbins), entry_ids_ptr, entry_traj_ptr)
 
 
 def _u32_host(a, n, what):
@@ -279,16 +281,17 @@ class DeviceResults:
 
 def build_index(D, device: int = 0, temporal_bins: int = 0, cells_per_dim: int = 0,
                 d_hint: float = 0.0, method="grid", subbins: int = 0,
-                entry_ids=None, entry_traj=None) -> Index:
+                entry_ids=None, entry_traj=None, mem_budget_bytes: int = 0) -> Index:
     """dts_build_index: D is host (n, 8) float64 (copied); entry_ids /
-    entry_traj: optional host uint32 reported ids / trajectory ids per row."""
+    entry_traj: optional host uint32 reported ids / trajectory ids per row;
+    mem_budget_bytes: device budget (over it: temporal shards on the host)."""
     lib = load()
     D = _segments(D)
     ids = _u32_host(entry_ids, D.shape[0], "entry_ids")
     traj = _u32_host(entry_traj, D.shape[0], "entry_traj")
     p = _params(device, temporal_bins, cells_per_dim, d_hint, method, subbins,
                 ids.ctypes.data if ids is not None else None,
-                traj.ctypes.data if traj is not None else None)
+                traj.ctypes.data if traj is not None else None, mem_budget_bytes)
     h = ctypes.c_void_p()
     _check(lib.dts_build_index(D.ctypes.data if D.size else None, D.shape[0], ctypes.byref(p),
                                ctypes.byref(h)))

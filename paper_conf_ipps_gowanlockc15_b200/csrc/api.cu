@@ -19,6 +19,29 @@ std::atomic<unsigned long long> g_launches{0};
 static thread_local std::string g_err;
 void set_last_error(const std::string& msg) { g_err = msg; }
 
+// Device memory of an index back to the device cache (alloc.cu): waits for
+// the end of the build only (a build returns before its last kernels finish;
+// searches are synchronous on return, so none is in flight), not for every
+// stream of the device.
+void free_index_arrays(dts_index* idx) {
+    if (idx->ready) cudaEventSynchronize(idx->ready);
+    for (int i = 0; i < idx->nev; ++i) cudaEventDestroy(idx->ev[i]);
+    idx->nev = 0;
+    idx->ready = nullptr;
+    cache_free(idx->block);
+    cache_free(idx->ht.slots);
+    cache_free(idx->etraj);
+    idx->etraj = nullptr;
+    for (int a = 0; a < 3; ++a) {
+        cache_free(idx->sb_block[a]);
+        idx->sb_block[a] = nullptr;
+        cache_free(idx->sb_rec[a]);
+        idx->sb_rec[a] = nullptr;
+    }
+    idx->block = nullptr;
+    idx->ht.slots = nullptr;
+}
+
 namespace {
 
 std::mutex g_mu;
@@ -105,26 +128,9 @@ void free_index_memory(dts_index* idx) {
     if (!idx) return;
     DeviceGuard dg;
     cudaSetDevice(idx->device);
-    // blocks go back to the device cache (alloc.cu) for the next build: wait
-    // for the end of the build only (a build returns before its last kernels
-    // finish; searches are synchronous on return, so none is in flight),
-    // not for every stream of the device
-    if (idx->ready) cudaEventSynchronize(idx->ready);
-    for (int i = 0; i < idx->nev; ++i) cudaEventDestroy(idx->ev[i]);
-    idx->nev = 0;
-    idx->ready = nullptr;
-    cache_free(idx->block);
-    cache_free(idx->ht.slots);
-    cache_free(idx->etraj);
-    idx->etraj = nullptr;
-    for (int a = 0; a < 3; ++a) {
-        cache_free(idx->sb_block[a]);
-        idx->sb_block[a] = nullptr;
-        cache_free(idx->sb_rec[a]);
-        idx->sb_rec[a] = nullptr;
-    }
-    idx->block = nullptr;
-    idx->ht.slots = nullptr;
+    free_index_arrays(idx);
+    ooc_free(idx->ooc);
+    idx->ooc = nullptr;
 }
 
 dts_index_params defaults() {
@@ -179,6 +185,13 @@ dts_status build_common(const dts_segment* D, size_t n, const dts_index_params* 
         idx = new dts_index();
         idx->device = p.device;
         if (n == 0) return;
+        if (host && p.mem_budget_bytes && index_bytes_estimate(n) > p.mem_budget_bytes) {
+            // D (and its index) exceed the budget: temporal shards in pinned
+            // host memory, indexed one at a time at search time (ooc.cu)
+            ooc_build(idx, D, n, p, s);
+            DTS_CUDA(cudaStreamSynchronize(s));
+            return;
+        }
         if (host) {
             DevBuf<dts_segment> dD(n, s);
             DevBuf<uint32_t> dmap(p.entry_ids ? n : 0, s);
@@ -765,6 +778,7 @@ dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
         index_times(const_cast<dts_index*>(idx));
         dts_index_info r{};
         r.n = idx->n;
+        r.shards = idx->ooc ? (uint32_t)idx->ooc->shards.size() : 0u;
         r.cells = idx->n_cells;
         r.bins = (uint32_t)idx->gp.m;
         for (int a = 0; a < 3; ++a) {

@@ -299,6 +299,22 @@ struct DeviceGuard {
 
 }  // namespace dts
 
+namespace dts {
+// Temporal shards of an entry database larger than the device budget (ooc.cu).
+struct OocShard {
+    size_t n = 0;
+    double t0min = 0, t1max = 0;   // min t_start, max t_end of the shard's entries
+};
+struct OocIndex {
+    dts_segment* D_h = nullptr;    // pinned, shards contiguous
+    uint32_t* ids_h = nullptr;     // pinned, reported entry id per row
+    uint32_t* traj_h = nullptr;    // pinned, trajectory id per row (optional)
+    std::vector<OocShard> shards;
+    std::vector<size_t> off;       // first row of each shard
+    dts_index_params p{};          // parameters of the per-shard builds
+};
+}  // namespace dts
+
 // The opaque index (definition shared by build.cu, search.cu and api.cu).
 struct dts_index {
     int device = 0;
@@ -331,6 +347,7 @@ struct dts_index {
     // index has produced after its spill buffer filled (search.cu)
     mutable std::atomic<unsigned long long> spill_hint{0};
     int eid_bits = 32;             // bits of the largest reported entry id
+    dts::OocIndex* ooc = nullptr;  // set: D lives in pinned host temporal shards
 };
 
 namespace dts {
@@ -368,4 +385,15 @@ void merge_trajectories_device(const dts_result* r, size_t n, const uint32_t* qt
                                cudaStream_t s, dts_traj_result** out, size_t* count);
 // Sort results in device memory by (query_id, entry_id), in place.
 void canonicalize_device(dts_result* r, size_t n, cudaStream_t s);
+// Device memory of an index (after its build has finished) back to the cache.
+void free_index_arrays(dts_index* idx);
+// Entry databases larger than the budget (ooc.cu).
+uint64_t index_bytes_estimate(size_t n);
+void ooc_build(dts_index* idx, const dts_segment* D_host, size_t n, const dts_index_params& p,
+               cudaStream_t s);
+void ooc_free(OocIndex* o);
+void ooc_search(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
+                uint32_t qid_base, cudaStream_t s, SearchOut* out, dts_search_stats* stats,
+                const uint32_t* qmap, const uint32_t* qtraj, bool excl, bool count_only,
+                uint32_t* counts_out);
 }  // namespace dts

@@ -476,6 +476,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         if (stats) *stats = local;
         return;
     }
+    if (idx->ooc) {              // D in temporal shards on the host (ooc.cu)
+        ooc_search(idx, Q_dev, nq, d, qid_base, s, out, stats, qmap, qtraj, exclude_same_traj,
+                   count_only, counts_out);
+        return;
+    }
     const double4* Q = reinterpret_cast<const double4*>(Q_dev);
     DevBuf<Counters> ctr(1, s);
     DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
@@ -828,6 +833,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                         uint32_t block, unsigned long long* out, cudaStream_t s) {
     if (block == 0) throw Error(DTS_EINVAL, "block must be >= 1");
+    if (idx->ooc) throw Error(DTS_ENOTSUP, "query costs of an index over temporal shards");
     const size_t nb = (nq + block - 1) / block;
     if (nb) DTS_CUDA(cudaMemsetAsync(out, 0, nb * sizeof(unsigned long long), s));
     if (nq == 0 || idx->n == 0) return;

@@ -233,3 +233,36 @@ def test_search_count_and_stream(dts, oracle_mod):
                    c.D, c.Q, 2.0, oracle_mod)
     idx.free()
     idd.free()
+
+
+@pytest.mark.parametrize("budget_mb", [70, 66])
+def test_mem_budget_temporal_shards(dts, oracle_mod, budget_mb):
+    """An index over the device budget (mem_budget_bytes) keeps D in temporal
+    shards on the host and indexes them one at a time at search time
+    (SURVEY.md §8(e) fallback): same bytes as the resident index for the
+    plain, trajectory-excluding, count-only and streamed searches."""
+    c = synth.make_config("C2", scale=0.01)
+    ref_idx = dts.build_index(c.D, entry_traj=c.etraj)
+    idx = dts.build_index(c.D, entry_traj=c.etraj, mem_budget_bytes=budget_mb << 20)
+    inf = idx.info()
+    assert inf["shards"] >= 2, inf
+    assert ref_idx.info()["shards"] == 0
+    for d in (0.5, 2.0, 8.0):
+        ref = dts.search(ref_idx, c.Q, d, query_id_base=3)
+        got = dts.search(idx, c.Q, d, query_id_base=3)
+        assert got.tobytes() == ref.tobytes(), d
+    kw = dict(query_traj=c.qtraj, exclude_same_trajectory=True)
+    ref, _ = dts.search_ex(ref_idx, c.Q, 2.0, **kw)
+    got, _ = dts.search_ex(idx, c.Q, 2.0, **kw)
+    assert got.tobytes() == ref.tobytes()
+    total, counts, _ = dts.search_count(idx, c.Q, 2.0)
+    rt, rc, _ = dts.search_count(ref_idx, c.Q, 2.0)
+    assert total == rt and np.array_equal(counts, rc)
+    chunks = []
+    dts.search_stream(idx, c.Q, 2.0, lambda ch: chunks.append(ch.copy()), chunk_results=5000)
+    assert np.concatenate(chunks).tobytes() == dts.search(ref_idx, c.Q, 2.0).tobytes()
+    qs = np.arange(0, c.Q.shape[0], 29)
+    parity.compare(parity.restrict(dts.search(idx, c.Q, 2.0), qs),
+                   oracle_mod.search_queries(c.D, c.Q, qs, 2.0), c.D, c.Q, 2.0, oracle_mod)
+    idx.free()
+    ref_idx.free()
