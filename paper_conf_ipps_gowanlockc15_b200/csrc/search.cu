@@ -689,9 +689,16 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // ---- results that do not fit the device: report the per-query counts
     //      so a host caller can stream the search in query chunks
     const double per = h.c.n_over ? 24.0 + 24.0 : 24.0;   // fin (+ the re-run's spill)
-    // (cudaMemGetInfo is slow and jittery -- ms -- so it is asked only when
-    //  the results are large enough to matter)
-    if (h.total > 0 && ((double)h.total * per > 1e9 || h.total > max_results)) {
+    // (cudaMemGetInfo is slow and jittery -- up to 15 ms measured on S2 at
+    //  d = 1 with 30 GB of pool memory mapped -- so it is asked only when the
+    //  results could take more than a quarter of the device's memory)
+    static const double dev_bytes = [] {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceProp pr;
+        return cudaGetDeviceProperties(&pr, dev) == cudaSuccess ? (double)pr.totalGlobalMem : 0.0;
+    }();
+    if (h.total > 0 && ((double)h.total * per > 0.25 * dev_bytes || h.total > max_results)) {
         size_t free_b = 0, total_b = 0;
         DTS_CUDA(cudaMemGetInfo(&free_b, &total_b));
         if ((double)h.total * per > 0.8 * (double)free_b || h.total > max_results) {
