@@ -206,10 +206,22 @@ __device__ __forceinline__ ulonglong4 ld256u(const void* p) {
     return v;
 }
 
+// Both 256-bit halves of a record, issued together: `volatile` keeps the
+// compiler from sinking the second load behind the refinement's temporal
+// test (it did: one more dependent memory round trip per candidate).
+__device__ __forceinline__ void ld512v(const double4* p, double4& a, double4& b) {
+    asm volatile("ld.global.nc.v4.f64 {%0,%1,%2,%3}, [%8];\n\t"
+                 "ld.global.nc.v4.f64 {%4,%5,%6,%7}, [%8+32];"
+                 : "=d"(a.x), "=d"(a.y), "=d"(a.z), "=d"(a.w), "=d"(b.x), "=d"(b.y), "=d"(b.z),
+                   "=d"(b.w)
+                 : "l"(p));
+}
+
 __device__ __forceinline__ void SegSoA::load4(size_t p, double2& st, double2& sx, double2& sy,
                                               double2& sz) const {
     const double4* r = reinterpret_cast<const double4*>(rec + 4 * p);
-    const double4 a = ld256(r), b = ld256(r + 1);
+    double4 a, b;
+    ld512v(r, a, b);
     st = make_double2(a.x, a.y);
     sx = make_double2(a.z, a.w);
     sy = make_double2(b.x, b.y);

@@ -83,9 +83,12 @@ struct Stencil {
 __device__ __forceinline__ bool refine(const QState& q, const double2 st, const double2 sx,
                                        const double2 sy, const double2 sz, const double d2,
                                        double& t_out0, double& t_out1) {
+    // the temporal and the "outside and not approaching" rejections are
+    // taken together, after the whole record is used: a branch on the
+    // temporal test alone let ptxas sink the record's second 32-byte load
+    // behind it (one more dependent memory round trip per candidate)
     const double ts = fmax(q.t0, st.x);
     const double te = fmin(q.t1, st.y);
-    if (!(ts < te)) return false;
     const double dq = ts - q.t0, de = ts - st.x;
     const double ax = fma(de, sx.y, sx.x) - fma(dq, q.vx, q.x0);
     const double ay = fma(de, sy.y, sy.x) - fma(dq, q.vy, q.y0);
@@ -93,7 +96,8 @@ __device__ __forceinline__ bool refine(const QState& q, const double2 st, const 
     const double wx = sx.y - q.vx, wy = sy.y - q.vy, wz = sz.y - q.vz;
     const double cc = fma(ax, ax, fma(ay, ay, fma(az, az, -d2)));
     const double bb = fma(ax, wx, fma(ay, wy, az * wz));
-    if (cc > 0.0 && bb >= 0.0) return false;          // outside and not approaching
+    if (!(ts < te) || (cc > 0.0 && bb >= 0.0)) return false;   // no strict overlap, or
+                                                                // outside and not approaching
     const double aa = fma(wx, wx, fma(wy, wy, wz * wz));
     const double L = te - ts;
     double lo, hi;
