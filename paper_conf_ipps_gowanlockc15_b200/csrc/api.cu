@@ -409,14 +409,17 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
                 DTS_CUDA(cudaMemcpyAsync(dtraj.p, qtraj, nq * sizeof(uint32_t),
                                          cudaMemcpyHostToDevice, s));
             }
-            // large host query sets stream through the device in chunks
-            // (DTS_Q_CHUNK queries each, default 2^21 = 128 MB of segments;
-            // 0 disables).  Measured on C4: at 1 M queries four 256 K chunks
-            // are slower than one shot (per-search fixed costs), so only
-            // query sets of >= 2 chunks are pipelined.
+            // large host query sets stream through the device in chunks:
+            // chunk i's H2D overlaps search i-1 and its results' D2H search
+            // i+1 (DTS_Q_CHUNK queries per chunk; 0 disables).  Default: from
+            // 2^19 queries, chunks of max(2^18, nq / 4).  Measured on C4 (1 M
+            // queries, index resident, host API): one shot 2.37 ms; chunks of
+            // 131072: 2.83; 262144: 2.18; 333376: 2.25; 500064: 2.23.
             const char* ch_env = getenv("DTS_Q_CHUNK");
             const size_t chunk = ch_env ? (size_t)std::strtoull(ch_env, nullptr, 10)
-                                        : (size_t)1 << 21;
+                                        : (nq >= ((size_t)1 << 19)
+                                               ? std::max<size_t>((size_t)1 << 18, (nq + 3) / 4)
+                                               : 0);
             if (chunk > 0 && nq >= 2 * chunk) {
                 try {
                     ret = search_pipelined(index, Q, nq, d, qid_base, s, chunk, dmap.p, dtraj.p,
