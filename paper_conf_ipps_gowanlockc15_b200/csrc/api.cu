@@ -796,7 +796,7 @@ dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
         r.build_flags = idx->fused_keys ? 1u : 0u;
         r.hash_kind = 1u;
         r.hash_items = idx->hash_items;
-        r.hash_bytes = idx->ht.slots ? (uint64_t)(idx->ht.mask + 1) * sizeof(dts::BlockSlot) : 0;
+        r.hash_bytes = idx->ht.slots ? (uint64_t)idx->ht.nslots() * sizeof(dts::BlockSlot) : 0;
         r.method = idx->method;
         for (int a = 0; a < 3; ++a) {
             r.subbins[a] = idx->method == DTS_METHOD_SUBBIN ? (uint32_t)idx->sb.v[a] : 0u;

@@ -125,10 +125,9 @@ struct GridParams {
 
 struct HashTable {
     void* slots;               // BlockSlot, 2 per 64-byte bucket
-    unsigned long long mask;   // slots - 1 (power of two)
-    int log2cap;               // log2 of the slots
-    __host__ __device__ int log2bucket() const { return 1; }
+    unsigned long long nbuckets;   // buckets (any count: not a power of two)
     __host__ __device__ BlockSlot* blocks() const { return static_cast<BlockSlot*>(slots); }
+    __host__ __device__ unsigned long long nslots() const { return 2ull * nbuckets; }
 };
 
 // GPUSpatioTemporal subbins (P:L86-P:L92): per dimension a, v[a] subbins of
@@ -165,9 +164,18 @@ __device__ __forceinline__ int32_t subbin_of(const SubbinIndex& s, int a, double
 // first bucket, from its home on, that had a free slot when it was inserted
 // (no deletions), so a lookup stops at the first bucket holding it or a
 // free slot -- almost always the home bucket.
+// Home bucket: a Fibonacci hash of the block key mapped onto [0, nbuckets)
+// by a multiply-shift range reduction (the table is sized to the load
+// factor exactly, not rounded up to a power of two: with power-of-two sizes
+// the same load target gave anywhere from 3.3 to 6.6 slots per block).
 __device__ __forceinline__ unsigned long long bucket_of(unsigned long long group,
                                                         const HashTable& ht) {
-    return (group * 0x9E3779B97F4A7C15ull) >> (64 - (ht.log2cap - ht.log2bucket()));
+    const unsigned long long h = (group * 0x9E3779B97F4A7C15ull) >> 32;   // 32 mixed bits
+    return (h * ht.nbuckets) >> 32;
+}
+__device__ __forceinline__ unsigned long long next_bucket(unsigned long long b,
+                                                          const HashTable& ht) {
+    return b + 1 == ht.nbuckets ? 0ull : b + 1;
 }
 
 __device__ __forceinline__ int32_t bin_of(const GridParams& g, double t) {

@@ -303,7 +303,6 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
     // 8), each one 32-byte slot holding the prefix counts of its 8 cells; a
     // bucket is two slots (64 bytes)
     const BlockSlot* slots = ht.blocks();
-    const unsigned long long bmask = ht.mask >> 1;
     for (unsigned long long blk = key0 >> 3; blk <= (kend - 1) >> 3; ++blk) {
         unsigned long long b = bucket_of(blk, ht);
         ++probes;
@@ -335,7 +334,7 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
                 break;
             }
             if (h0.x == EMPTY_KEY || h1.x == EMPTY_KEY) break;   // end of the chain
-            b = (b + 1) & bmask;
+            b = next_bucket(b, ht);
         }
     }
     if (first != 0xffffffffu) {

@@ -20,6 +20,7 @@ agg = collections.defaultdict(list)
 for r in rows: agg[(r["config"], r["d"], r["lib"])].append(r)
 for k in sorted(agg):
     v = agg[k]
-    print(k, "search %.4f count %.4f prep %.4f emit %.4f canon %.4f" % tuple(
-        min(x[f] for x in v) for f in ("search_ms", "count_ms", "prep_ms", "emit_ms", "canon_ms")))
+    print(k, "search %.4f count %.4f prep %.4f emit %.4f canon %.4f build %.4f" % tuple(
+        min(x.get(f, 0) for x in v) for f in ("search_ms", "count_ms", "prep_ms", "emit_ms", "canon_ms", "build_ms")),
+        "insert %.4f" % min(x.get("build_phases", [0]*5)[4] for x in v))
 PY

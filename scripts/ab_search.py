@@ -37,8 +37,13 @@ for pt in a.points:
         c = synth.make_config(name)
         Dd = torch.from_numpy(c.D).cuda()
         Qd = torch.from_numpy(c.Q).cuda()
+        # build twice (the first maps fresh pages); phases of the second
+        i0 = dts.build_index_device(Dd, d_hint=hint)
+        i0.info()
+        i0.free()
         cache[key] = (Qd, dts.build_index_device(Dd, d_hint=hint), Dd)
     Qd, idx, _ = cache[key]
+    binf = idx.info()
     s = torch.cuda.current_stream()
     for _ in range(3):
         r, st = dts.search_device(idx, Qd, d, stream=s, time_kernels=True)
@@ -61,4 +66,6 @@ for pt in a.points:
                       "prep_ms": statistics.median(x["ms_prep"] for x in sts),
                       "emit_ms": statistics.median(x["ms_scatter"] for x in sts),
                       "canon_ms": statistics.median(x["ms_canon"] for x in sts),
-                      "results": n, "candidates": sts[-1]["candidates"]}), flush=True)
+                      "results": n, "candidates": sts[-1]["candidates"],
+                      "build_ms": binf["ms_build"], "build_phases": binf["ms_phase"],
+                      "hash_bytes": binf["hash_bytes"]}), flush=True)
