@@ -308,6 +308,9 @@ typedef struct {
     uint64_t hash_bytes;        /* table size in bytes                       */
     uint32_t shards;            /* temporal shards on the host (mem_budget_bytes
                                    exceeded), 0 for an index resident on the device */
+    uint64_t outlier_rows;      /* entries filed as copies along their path (extent
+                                   or duration above 8x the mean; grid method) */
+    uint64_t outlier_copies;    /* their copies (n counts them)               */
 } dts_index_info;
 
 dts_status dts_index_get_info(const dts_index* index, dts_index_info* info);

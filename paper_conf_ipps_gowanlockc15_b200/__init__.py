@@ -89,7 +89,8 @@ class IndexInfo(ctypes.Structure):
                 ("subbin_ids", ctypes.c_uint64 * 3), ("ms_phase", ctypes.c_float * 5),
                 ("build_flags", ctypes.c_uint32), ("hash_kind", ctypes.c_uint32),
                 ("hash_items", ctypes.c_uint64), ("hash_bytes", ctypes.c_uint64),
-                ("shards", ctypes.c_uint32)]
+                ("shards", ctypes.c_uint32), ("outlier_rows", ctypes.c_uint64),
+                ("outlier_copies", ctypes.c_uint64)]
 
     def as_dict(self):
         out = {}

@@ -32,6 +32,9 @@ void free_index_arrays(dts_index* idx) {
     cache_free(idx->ht.slots);
     cache_free(idx->etraj);
     idx->etraj = nullptr;
+    cache_free(idx->out_block);
+    idx->out_block = nullptr;
+    idx->out = dts::OutlierIndex{};
     for (int a = 0; a < 3; ++a) {
         cache_free(idx->sb_block[a]);
         idx->sb_block[a] = nullptr;
@@ -782,6 +785,8 @@ dts_status dts_index_get_info(const dts_index* idx, dts_index_info* info) {
         dts_index_info r{};
         r.n = idx->n;
         r.shards = idx->ooc ? (uint32_t)idx->ooc->shards.size() : 0u;
+        r.outlier_rows = idx->n_outliers;
+        r.outlier_copies = idx->n_copies;
         r.cells = idx->n_cells;
         r.bins = (uint32_t)idx->gp.m;
         for (int a = 0; a < 3; ++a) {

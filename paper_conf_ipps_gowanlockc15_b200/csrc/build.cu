@@ -32,18 +32,30 @@ namespace {
 struct Bounds {
     double tmin, tmax;
     double lo[3], hi[3];
-    double ext[3];
-    double maxdur;
+    double ext[3];             // max extent per axis (outliers excluded when thresholds apply)
+    double maxdur;             // max duration (idem)
     double absmax;
+    double sext[3], sdur;      // sums of extents and durations (sample means)
+    unsigned long long cnt;    // valid entries added
+    unsigned long long nout;   // outliers (extent or duration above the thresholds)
     int bad;
+};
+
+// Outlier thresholds (build.cu header of internal.cuh "outliers"): an entry
+// whose extent exceeds ext[a] on some axis or whose duration exceeds dur.
+struct Thresh {
+    double ext[3], dur;
+    int on;
 };
 
 constexpr int BT = 256;
 
 __device__ __forceinline__ void bounds_init(Bounds& b) {
     b.tmin = INFINITY; b.tmax = -INFINITY;
-    for (int a = 0; a < 3; ++a) { b.lo[a] = INFINITY; b.hi[a] = -INFINITY; b.ext[a] = 0.0; }
-    b.maxdur = 0.0; b.absmax = 0.0; b.bad = 0;
+    for (int a = 0; a < 3; ++a) {
+        b.lo[a] = INFINITY; b.hi[a] = -INFINITY; b.ext[a] = 0.0; b.sext[a] = 0.0;
+    }
+    b.maxdur = 0.0; b.absmax = 0.0; b.sdur = 0.0; b.cnt = 0; b.nout = 0; b.bad = 0;
 }
 
 __device__ __forceinline__ void bounds_merge(Bounds& b, const Bounds& o) {
@@ -53,22 +65,28 @@ __device__ __forceinline__ void bounds_merge(Bounds& b, const Bounds& o) {
         b.ext[a] = fmax(b.ext[a], o.ext[a]);
     }
     b.maxdur = fmax(b.maxdur, o.maxdur); b.absmax = fmax(b.absmax, o.absmax);
+    for (int a = 0; a < 3; ++a) b.sext[a] += o.sext[a];
+    b.sdur += o.sdur; b.cnt += o.cnt; b.nout += o.nout;
     b.bad |= o.bad;
 }
 
+// Field by field (shuffle, then merge): no second Bounds held in registers.
 __device__ __forceinline__ void bounds_shfl(Bounds& b, int off) {
-    Bounds o;
-    o.tmin = __shfl_xor_sync(0xffffffffu, b.tmin, off);
-    o.tmax = __shfl_xor_sync(0xffffffffu, b.tmax, off);
+    const unsigned F = 0xffffffffu;
+    b.tmin = fmin(b.tmin, __shfl_xor_sync(F, b.tmin, off));
+    b.tmax = fmax(b.tmax, __shfl_xor_sync(F, b.tmax, off));
     for (int a = 0; a < 3; ++a) {
-        o.lo[a] = __shfl_xor_sync(0xffffffffu, b.lo[a], off);
-        o.hi[a] = __shfl_xor_sync(0xffffffffu, b.hi[a], off);
-        o.ext[a] = __shfl_xor_sync(0xffffffffu, b.ext[a], off);
+        b.lo[a] = fmin(b.lo[a], __shfl_xor_sync(F, b.lo[a], off));
+        b.hi[a] = fmax(b.hi[a], __shfl_xor_sync(F, b.hi[a], off));
+        b.ext[a] = fmax(b.ext[a], __shfl_xor_sync(F, b.ext[a], off));
+        b.sext[a] += __shfl_xor_sync(F, b.sext[a], off);
     }
-    o.maxdur = __shfl_xor_sync(0xffffffffu, b.maxdur, off);
-    o.absmax = __shfl_xor_sync(0xffffffffu, b.absmax, off);
-    o.bad = __shfl_xor_sync(0xffffffffu, b.bad, off);
-    bounds_merge(b, o);
+    b.maxdur = fmax(b.maxdur, __shfl_xor_sync(F, b.maxdur, off));
+    b.absmax = fmax(b.absmax, __shfl_xor_sync(F, b.absmax, off));
+    b.sdur += __shfl_xor_sync(F, b.sdur, off);
+    b.cnt += __shfl_xor_sync(F, b.cnt, off);
+    b.nout += __shfl_xor_sync(F, b.nout, off);
+    b.bad |= __shfl_xor_sync(F, b.bad, off);
 }
 
 __device__ void block_reduce_write(Bounds& b, Bounds* out) {
@@ -86,18 +104,34 @@ __device__ void block_reduce_write(Bounds& b, Bounds* out) {
 }
 
 // Segment validity (readings c4, c8): finite coordinates and times,
-// t_end >= t_start, finite velocity.
-__device__ __forceinline__ void bounds_add(Bounds& b, const double4 s0, const double4 s1) {
+// t_end >= t_start, finite velocity.  With thresholds, an outlier counts in
+// the domain (time range, spatial bounds) but not in the max extent and
+// duration that size the grid and the stencils; returns whether the entry
+// is an outlier.
+__device__ __forceinline__ bool is_outlier(const Thresh& th, const double4 s0, const double4 s1) {
+    return th.on && (fabs(s1.y - s0.y) > th.ext[0] || fabs(s1.z - s0.z) > th.ext[1] ||
+                     fabs(s1.w - s0.w) > th.ext[2] || s1.x - s0.x > th.dur);
+}
+
+template <bool SUMS = true>
+__device__ __forceinline__ bool bounds_add(Bounds& b, const double4 s0, const double4 s1,
+                                           const Thresh& th) {
     // (t0,x0,y0,z0), (t1,x1,y1,z1); v - v is 0 for a finite v and NaN
     // otherwise, so one comparison checks all eight values
     const double z = ((s0.x - s0.x) + (s1.x - s1.x)) + ((s0.y - s0.y) + (s1.y - s1.y)) +
                      ((s0.z - s0.z) + (s1.z - s1.z)) + ((s0.w - s0.w) + (s1.w - s1.w));
-    if (!(z == 0.0)) { b.bad |= 1; return; }
-    if (s1.x < s0.x) { b.bad |= 2; return; }
+    if (!(z == 0.0)) { b.bad |= 1; return false; }
+    if (s1.x < s0.x) { b.bad |= 2; return false; }
+    const bool outl = is_outlier(th, s0, s1);
     const double dur = s1.x - s0.x;
     b.tmin = fmin(b.tmin, s0.x);
     b.tmax = fmax(b.tmax, s1.x);
-    b.maxdur = fmax(b.maxdur, dur);
+    if (!outl) b.maxdur = fmax(b.maxdur, dur);
+    if (SUMS) {
+        b.sdur += dur;
+        b.cnt += 1;
+    }
+    b.nout += outl ? 1ull : 0ull;
     const double p0[3] = {s0.y, s0.z, s0.w}, p1[3] = {s1.y, s1.z, s1.w};
     double emax = 0.0;
 #pragma unroll
@@ -106,13 +140,15 @@ __device__ __forceinline__ void bounds_add(Bounds& b, const double4 s0, const do
         b.lo[a] = fmin(b.lo[a], lo);
         b.hi[a] = fmax(b.hi[a], hi);
         const double e = hi - lo;
-        b.ext[a] = fmax(b.ext[a], e);
+        if (SUMS) b.sext[a] += e;
+        if (!outl) b.ext[a] = fmax(b.ext[a], e);
         emax = fmax(emax, e);
     }
     // speed |p1 - p0| / dur must be finite on every axis: an infinite extent,
     // or (only possible for dur < 1) an overflowing quotient of the largest
     // extent (division is monotone in the numerator)
     if (!isfinite(emax) || (dur > 0.0 && dur < 1.0 && !isfinite(emax / dur))) b.bad |= 4;
+    return outl;
 }
 
 __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, size_t n,
@@ -120,7 +156,7 @@ __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, si
     Bounds b;
     bounds_init(b);
     for (size_t i = (size_t)blockIdx.x * BT + threadIdx.x; i < n; i += (size_t)gridDim.x * BT)
-        bounds_add(b, ld256(D + 2 * i), ld256(D + 2 * i + 1));
+        bounds_add(b, ld256(D + 2 * i), ld256(D + 2 * i + 1), Thresh{{0, 0, 0}, 0, 0});
     block_reduce_write(b, &partial[blockIdx.x]);
 }
 
@@ -135,12 +171,13 @@ __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, si
 // hashes the 8-cell blocks less evenly -- a Fibonacci hash spreads the
 // arithmetic progressions of the old grid's block keys better than random.)
 __global__ void __launch_bounds__(BT) k_bounds_sample(const double4* __restrict__ D, size_t n,
-                                                     size_t S, Bounds* __restrict__ partial) {
+                                                     size_t S, Bounds* __restrict__ partial,
+                                                     Thresh th) {
     Bounds b;
     bounds_init(b);
     for (size_t j = (size_t)blockIdx.x * BT + threadIdx.x; j < S; j += (size_t)gridDim.x * BT) {
         const size_t i = (size_t)(((unsigned __int128)j * n) / S);
-        bounds_add(b, D[2 * i], D[2 * i + 1]);
+        bounds_add(b, D[2 * i], D[2 * i + 1], th);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
 }
@@ -230,13 +267,31 @@ __device__ __forceinline__ unsigned long long packed_key(const GridParams& g, co
     return (make_key(g, bin, cx, cy, cz) << shift) | (unsigned long long)i;
 }
 
-template <int MINB>
+// Outliers (thresholds th): bit of the row in orows, row appended to olist
+// (capacity ocap; ocount may exceed it: the build then drops outlier filing).
+struct OutlierOut {
+    uint32_t* orows;
+    uint32_t* olist;
+    unsigned int* ocount;
+    unsigned int ocap;
+};
+
+__device__ __forceinline__ void note_outlier(const OutlierOut& oo, size_t i) {
+    atomicOr(&oo.orows[i >> 5], 1u << (i & 31));
+    const unsigned int k = atomicAdd(oo.ocount, 1u);
+    if (k < oo.ocap) oo.olist[k] = (uint32_t)i;
+}
+
+// OUT: thresholds on (outliers flagged and listed), one entry per thread
+// step; else two in flight and no outlier code (its registers spilled)
+template <int MINB, bool OUT>
 __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restrict__ D, size_t n,
                                                       GridParams g,
                                                       unsigned long long* __restrict__ keys,
                                                       int shift, const PassPlan plan,
                                                       Bounds* __restrict__ partial,
-                                                      uint32_t* __restrict__ hist) {
+                                                      uint32_t* __restrict__ hist, Thresh th,
+                                                      OutlierOut oo) {
     __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
     for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT) h[j] = 0;
     __syncthreads();
@@ -250,12 +305,22 @@ __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restr
     };
     const size_t stride = (size_t)gridDim.x * BT;
     size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
+    const Thresh thr = OUT ? th : Thresh{{0, 0, 0}, 0, 0};
+    if (OUT) {
+        for (; i < n; i += stride) {
+            const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
+            if (bounds_add<false>(b, a0, a1, thr)) note_outlier(oo, i);
+            const unsigned long long va = packed_key(g, a0, a1, shift, i);
+            keys[i] = va;
+            count(va);
+        }
+    }
     for (; i + stride < n; i += 2 * stride) {      // two entries in flight per thread
         const size_t j = i + stride;
         const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
         const double4 c0 = ld256(D + 2 * j), c1 = ld256(D + 2 * j + 1);
-        bounds_add(b, a0, a1);
-        bounds_add(b, c0, c1);
+        bounds_add<false>(b, a0, a1, thr);
+        bounds_add<false>(b, c0, c1, thr);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
         const unsigned long long vc = packed_key(g, c0, c1, shift, j);
         keys[i] = va;
@@ -265,12 +330,88 @@ __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restr
     }
     if (i < n) {
         const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
-        bounds_add(b, a0, a1);
+        bounds_add<false>(b, a0, a1, thr);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
         keys[i] = va;
         count(va);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
+    __syncthreads();
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT)
+        if (h[j]) atomicAdd(hist + j, h[j]);
+}
+
+// The record of row i of D as the search sees it (velocity form, the same
+// arithmetic as the gather).
+__device__ __forceinline__ double velocity(double p0, double p1, double dur) {
+    return dur > 0.0 ? (p1 - p0) / dur : 0.0;
+}
+__device__ __forceinline__ ORec orec_of(const double4* __restrict__ D, size_t i) {
+    const double4 s0 = D[2 * i], s1 = D[2 * i + 1];
+    const double dur = s1.x - s0.x;
+    ORec o;
+    o.t0 = s0.x;
+    o.t1 = s1.x;
+    o.x[0] = s0.y; o.x[1] = s0.z; o.x[2] = s0.w;
+    o.v[0] = velocity(s0.y, s1.y, dur);
+    o.v[1] = velocity(s0.z, s1.z, dur);
+    o.v[2] = velocity(s0.w, s1.w, dur);
+    return o;
+}
+
+// Copies of each listed outlier (cells of its sub-slice boxes, every bin of
+// its time span); counts[i] saturates at OUT_MAX (the build then drops
+// outlier filing).
+constexpr unsigned int OUT_MAX = 1u << 20;
+__global__ void __launch_bounds__(BT) k_outlier_count(const double4* __restrict__ D,
+                                                     const uint32_t* __restrict__ olist,
+                                                     uint32_t nout, GridParams g,
+                                                     uint32_t* __restrict__ counts) {
+    const uint32_t i = blockIdx.x * BT + threadIdx.x;
+    if (i >= nout) return;
+    const ORec o = orec_of(D, olist[i]);
+    const int32_t jo0 = bin_of(g, o.t0), jo1 = bin_of(g, o.t1);
+    unsigned long long c = 0;
+    for (int32_t j = jo0; j <= jo1 && c < OUT_MAX; ++j)
+        outlier_boxes(g, o, j, jo0, jo1, [&](const int32_t lo[3], const int32_t hi[3]) {
+            c += (unsigned long long)(hi[0] - lo[0] + 1) * (unsigned long long)(hi[1] - lo[1] + 1) *
+                 (unsigned long long)(hi[2] - lo[2] + 1);
+        });
+    counts[i] = (uint32_t)min(c, (unsigned long long)OUT_MAX);
+}
+
+// Packed keys (cell key << shift | row) of the copies at keys[off[i] ..],
+// with their digit counts added to the sort's histograms.
+__global__ void __launch_bounds__(BT) k_outlier_emit(const double4* __restrict__ D,
+                                                    const uint32_t* __restrict__ olist,
+                                                    uint32_t nout, GridParams g,
+                                                    const unsigned long long* __restrict__ off,
+                                                    unsigned long long* __restrict__ keys, int shift,
+                                                    const PassPlan plan,
+                                                    uint32_t* __restrict__ hist) {
+    __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
+    for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT) h[j] = 0;
+    __syncthreads();
+    const uint32_t i = blockIdx.x * BT + threadIdx.x;
+    if (i < nout) {
+        const uint32_t row = olist[i];
+        const ORec o = orec_of(D, row);
+        const int32_t jo0 = bin_of(g, o.t0), jo1 = bin_of(g, o.t1);
+        unsigned long long k = off[i];
+        for (int32_t j = jo0; j <= jo1; ++j)
+            outlier_boxes(g, o, j, jo0, jo1, [&](const int32_t lo[3], const int32_t hi[3]) {
+                for (int32_t cz = lo[2]; cz <= hi[2]; ++cz)
+                    for (int32_t cy = lo[1]; cy <= hi[1]; ++cy)
+                        for (int32_t cx = lo[0]; cx <= hi[0]; ++cx) {
+                            const unsigned long long v =
+                                (make_key(g, j, cx, cy, cz) << shift) | (unsigned long long)row;
+                            keys[k++] = v;
+                            for (int p = 0; p < plan.npass; ++p)
+                                atomicAdd(&h[p * OS_HSTRIDE +
+                                             ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
+                        }
+            });
+    }
     __syncthreads();
     for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += BT)
         if (h[j]) atomicAdd(hist + j, h[j]);
@@ -403,10 +544,6 @@ __global__ void __launch_bounds__(BT) k_insert_blocks_lane(const SortedKeys keys
 // continue past the tile: its head walks the global keys beyond (positions
 // before the tile's first head belong to the previous tile's last block and
 // are counted by that walk).
-__device__ __forceinline__ double velocity(double p0, double p1, double dur) {
-    return dur > 0.0 ? (p1 - p0) / dur : 0.0;
-}
-
 // Sorted position p <- original row ids[p]: ITEMS positions per thread
 // (strided by the CTA so stores stay coalesced), all row loads issued first;
 // the velocity form of each segment is written to the SoA streams.  Fused
@@ -901,6 +1038,17 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     Bounds hb;
     GridParams g{};
     DevBuf<unsigned long long> keys(n, s), keys_tmp(n, s);
+    // long-segment outliers (internal.cuh "outliers"): rows flagged by the
+    // fused pass, filed as copies along their path; nt = sorted positions
+    static const bool outliers_on = [] {     // DTS_OUTLIERS=0: plain filing
+        const char* e = getenv("DTS_OUTLIERS");
+        return !(e && e[0] == '0');
+    }();
+    Thresh th{{0, 0, 0}, 0, 0};
+    DevBuf<uint32_t> orows(0, s), olist(0, s);
+    DevBuf<unsigned int> ocount(0, s);
+    size_t nt = n;
+    unsigned long long n_out = 0;
     DevBuf<uint32_t> ids(0, s), ids_tmp(0, s);
     SortedKeys sk;
     bool done = false;
@@ -938,15 +1086,31 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         }();
         const size_t S = std::min<size_t>(n, (size_t)1 << slog);
         const int nps = (int)std::min<size_t>(std::max<size_t>(grid_for(S) / 4, 1), 592);
-        k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p);
+        k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, Thresh{{0, 0, 0}, 0, 0});
         DTS_LAUNCH_CHECK();
         k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
         DTS_LAUNCH_CHECK();
-        mark();
         Bounds hs;
         DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         check(hs);
+        // outlier thresholds (grid method): 8x the sample's mean extent per
+        // axis and mean duration, at least a thousandth of the sample's span;
+        // the sample's bounds are then taken again without the outliers
+        if (outliers_on && p.method == DTS_METHOD_GRID && hs.cnt > 0) {
+            const double c = (double)hs.cnt;
+            for (int a = 0; a < 3; ++a)
+                th.ext[a] = std::max(8.0 * hs.sext[a] / c, 1e-3 * (hs.hi[a] - hs.lo[a]));
+            th.dur = std::max(8.0 * hs.sdur / c, 1e-3 * (hs.tmax - hs.tmin));
+            th.on = 1;
+            k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, th);
+            DTS_LAUNCH_CHECK();
+            k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
+            DTS_LAUNCH_CHECK();
+            DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaStreamSynchronize(s));
+        }
+        mark();
         // the occupancy only matters when even a full box would be capped
         // (C3); dense or clustered data (C4, C2, S3) skip its kernel
         bool capped = false;
@@ -971,13 +1135,25 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                 return (e && e[0] == '4') ? 4 : 3;
             }();
             const int npk = (int)std::min<size_t>((size_t)resident_grid(
-                bk_minb == 3 ? (const void*)k_bounds_keys<3> : (const void*)k_bounds_keys<4>), np);
-            if (bk_minb == 3)
-                k_bounds_keys<3><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p,
-                                                    hist.p);
+                bk_minb == 3 ? (const void*)k_bounds_keys<3, false> : (const void*)k_bounds_keys<4, false>), np);
+            OutlierOut oo{};
+            if (th.on) {
+                orows.alloc(n / 32 + 1, s);
+                olist.alloc(std::min<size_t>(n, (size_t)(n / 64) + 4096), s);
+                ocount.alloc(1, s);
+                DTS_CUDA(cudaMemsetAsync(orows.p, 0, (n / 32 + 1) * 4, s));
+                DTS_CUDA(cudaMemsetAsync(ocount.p, 0, 4, s));
+                oo = OutlierOut{orows.p, olist.p, ocount.p, (unsigned int)olist.n};
+            }
+            if (th.on)
+                k_bounds_keys<3, true><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan,
+                                                          partial.p, hist.p, th, oo);
+            else if (bk_minb == 3)
+                k_bounds_keys<3, false><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan,
+                                                           partial.p, hist.p, th, oo);
             else
-                k_bounds_keys<4><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan, partial.p,
-                                                    hist.p);
+                k_bounds_keys<4, false><<<npk, BT, 0, s>>>(D, n, g, keys.p, row_bits, plan,
+                                                           partial.p, hist.p, th, oo);
             DTS_LAUNCH_CHECK();
             k_bounds_final<<<1, BT, 0, s>>>(partial.p, npk, total.p);
             DTS_LAUNCH_CHECK();
@@ -986,10 +1162,49 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             DTS_CUDA(cudaEventCreateWithFlags(&eb, cudaEventDisableTiming));
             DTS_CUDA(cudaEventRecord(eb, s));
             mark();
+            bool drop_outliers = false;
+            if (th.on) {
+                // outliers found: their copies join the keys before the sort
+                // (the host needs their number first)
+                DTS_CUDA(cudaEventSynchronize(eb));
+                const unsigned long long nout = hb_pinned->b.nout;
+                if (nout > (unsigned long long)olist.n) {
+                    drop_outliers = true;          // too many to be outliers: plain filing
+                } else if (nout > 0) {
+                    DevBuf<uint32_t> cnt(nout, s);
+                    DevBuf<unsigned long long> off(nout + 1, s);
+                    k_outlier_count<<<grid_for(nout), BT, 0, s>>>(D, olist.p, (uint32_t)nout, g,
+                                                                  cnt.p);
+                    DTS_LAUNCH_CHECK();
+                    scan_exclusive_u32_to_u64(cnt.p, off.p, nout, s);
+                    unsigned long long ncp = 0;
+                    DTS_CUDA(cudaMemcpyAsync(&ncp, off.p + nout, 8, cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                    if (ncp > std::min<unsigned long long>(n / 2 + 1024, 1ull << 27) ||
+                        n + ncp >= (1ull << 32)) {
+                        drop_outliers = true;
+                    } else {
+                        DevBuf<unsigned long long> k2(n + ncp, s), k2t(n + ncp, s);
+                        DTS_CUDA(cudaMemcpyAsync(k2.p, keys.p, n * 8, cudaMemcpyDeviceToDevice, s));
+                        k_outlier_emit<<<grid_for(nout), BT, 0, s>>>(D, olist.p, (uint32_t)nout, g,
+                                                                     off.p, k2.p + n, row_bits,
+                                                                     plan, hist.p);
+                        DTS_LAUNCH_CHECK();
+                        keys.release();
+                        keys_tmp.release();
+                        keys.p = k2.detach(); keys.n = n + ncp; keys.s = s;
+                        keys_tmp.p = k2t.detach(); keys_tmp.n = n + ncp; keys_tmp.s = s;
+                        nt = n + ncp;
+                        n_out = nout;
+                    }
+                }
+            }
             // 4. sort (enqueued before the host looks at the exact bounds)
-            sk.a = radix_sort_keys_hist(keys.p, keys_tmp.p, n, plan, hist.p, s);
-            sk.shift = row_bits;
-            sk.ids = nullptr;
+            if (!drop_outliers) {
+                sk.a = radix_sort_keys_hist(keys.p, keys_tmp.p, nt, plan, hist.p, s);
+                sk.shift = row_bits;
+                sk.ids = nullptr;
+            }
             DTS_CUDA(cudaEventSynchronize(eb));
             cudaEventDestroy(eb);
             hb = hb_pinned->b;
@@ -1010,12 +1225,15 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                 const double slack = g.b * std::max(1.0, 0.1 * (double)g.m);
                 ok = ok && hb.tmin >= g.tmin - slack && hb.tmax <= g.tmin + (double)g.m * g.b + slack;
             }
-            if (ok) {
+            if (ok && !drop_outliers) {
                 for (int a = 0; a < 3; ++a) g.half_ext[a] = 0.5 * hb.ext[a];
                 g.maxdur = hb.maxdur;
                 idx->key_bits = kb;
                 idx->fused_keys = true;
                 done = true;
+            } else {
+                nt = n;                         // the exact path files every entry once
+                n_out = 0;
             }
         }
     }
@@ -1068,16 +1286,16 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
 
     mark();
     // 5. gather into the sorted record layout
-    const size_t bytes_soa = n * (4 * sizeof(double2) + sizeof(uint32_t));
+    const size_t bytes_soa = nt * (4 * sizeof(double2) + sizeof(uint32_t));
     const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
     char* blk = nullptr;
     blk = static_cast<char*>(cache_alloc(bytes_soa + bytes_bins + 256));
     idx->block = blk;
     idx->soa.rec = reinterpret_cast<double2*>(blk);
-    idx->bin_t0min = reinterpret_cast<double*>(idx->soa.rec + 4 * n);
+    idx->bin_t0min = reinterpret_cast<double*>(idx->soa.rec + 4 * nt);
     idx->bin_t1max = idx->bin_t0min + g.m;
     idx->soa.eid = reinterpret_cast<uint32_t*>(idx->bin_t1max + g.m);
-    idx->bin_start = idx->soa.eid + n;
+    idx->bin_start = idx->soa.eid + nt;
     unsigned long long* b0 = reinterpret_cast<unsigned long long*>(idx->bin_t0min);
     unsigned long long* b1 = reinterpret_cast<unsigned long long*>(idx->bin_t1max);
     k_fill_u64<<<grid_for(g.m), BT, 0, s>>>(b0, g.m, ~0ull);
@@ -1097,13 +1315,13 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         return e ? atoi(e) : 2;
     }();
     if (gvar == 1)
-        k_gather_cells<1, 6><<<grid_for(n), BT, 0, s>>>(D, n, sk, idx->soa, g, idx->bin_start,
+        k_gather_cells<1, 6><<<grid_for(nt), BT, 0, s>>>(D, nt, sk, idx->soa, g, idx->bin_start,
                                                         b0, b1, ncell.p);
     else if (gvar == 4)
-        k_gather_cells<4, 2><<<grid_for((n + 3) / 4), BT, 0, s>>>(D, n, sk, idx->soa, g,
+        k_gather_cells<4, 2><<<grid_for((nt + 3) / 4), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                   idx->bin_start, b0, b1, ncell.p);
     else
-        k_gather_cells<2><<<grid_for((n + 1) / 2), BT, 0, s>>>(D, n, sk, idx->soa, g,
+        k_gather_cells<2><<<grid_for((nt + 1) / 2), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                idx->bin_start, b0, b1, ncell.p);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
@@ -1135,8 +1353,23 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // lane-parallel walks of the staged keys, warp path past 32 entries
     // (warp-cooperative heads for every block: 0.736 ms on C4; one CAS per
     // cell into cell slots: 0.56 ms; these lane walks: 0.435)
-    k_insert_blocks_lane<4, 32><<<grid_for((n + 3) / 4), BT, 0, s>>>(sk, n, idx->ht);
+    k_insert_blocks_lane<4, 32><<<grid_for((nt + 3) / 4), BT, 0, s>>>(sk, nt, idx->ht);
     DTS_LAUNCH_CHECK();
+    // outliers: the sorted packed keys (cell key << shift | row) and the row
+    // bitmap stay with the index for the search's canonical-copy test
+    idx->n = nt;
+    idx->n_outliers = n_out;
+    idx->n_copies = nt - n;
+    if (n_out) {
+        const size_t kb8 = nt * sizeof(unsigned long long), rb = (n / 32 + 1) * sizeof(uint32_t);
+        char* ob = static_cast<char*>(cache_alloc(kb8 + rb + 64));
+        idx->out_block = ob;
+        DTS_CUDA(cudaMemcpyAsync(ob, sk.a, kb8, cudaMemcpyDeviceToDevice, s));
+        DTS_CUDA(cudaMemcpyAsync(ob + kb8, orows.p, rb, cudaMemcpyDeviceToDevice, s));
+        idx->out.okeys = reinterpret_cast<const unsigned long long*>(ob);
+        idx->out.orows = reinterpret_cast<const uint32_t*>(ob + kb8);
+        idx->out.shift = sk.shift;
+    }
     mark();
 
     // 7. GPUSpatioTemporal subbin arrays (DTS_METHOD_SUBBIN)
@@ -1150,14 +1383,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
 
     // 8. trajectory ids in sorted order (params.entry_traj, device memory here)
     if (p.entry_traj) {
-        idx->etraj = static_cast<uint32_t*>(cache_alloc(n * sizeof(uint32_t)));
-        k_gather_u32<<<grid_for(n), BT, 0, s>>>(idx->etraj, p.entry_traj, idx->soa.eid, n);
+        idx->etraj = static_cast<uint32_t*>(cache_alloc(nt * sizeof(uint32_t)));
+        k_gather_u32<<<grid_for(nt), BT, 0, s>>>(idx->etraj, p.entry_traj, idx->soa.eid, nt);
         DTS_LAUNCH_CHECK();
     }
 
     // 9. reported entry ids of a shard (params.entry_ids, device memory here)
     if (p.entry_ids) {
-        k_map_ids<<<grid_for(n), BT, 0, s>>>(idx->soa.eid, n, p.entry_ids);
+        k_map_ids<<<grid_for(nt), BT, 0, s>>>(idx->soa.eid, nt, p.entry_ids);
         DTS_LAUNCH_CHECK();
     }
 

@@ -200,6 +200,57 @@ __device__ __forceinline__ unsigned long long make_key(const GridParams& g, int3
            (unsigned long long)cx;
 }
 
+// ---------------------------------------------------------------- outliers
+// Entries far longer in space or time than the rest ("outliers": extent or
+// duration above 8x the sample mean) are not filed by MBB midpoint -- their
+// extent would widen every query's stencil and their duration every
+// query's bin range.  Each is filed instead as copies along its path: for
+// every bin j its time overlaps, the time inside the bin is cut into S
+// sub-slices of about one cell of travel, and the copy keys are the cells of
+// each sub-slice's box.  A query meets the copies in its stencil; the search
+// keeps a hit on a copy only from the canonical copy: the least key among the
+// sub-slice boxes of the first probed bin whose boxes meet the query's
+// stencil (outlier_canonical in search.cu).  Build and search derive the
+// boxes with this one function from the same record values, so they agree
+// bit for bit.
+struct ORec {
+    double t0, t1;
+    double x[3], v[3];   // velocity form: position at t = x + (t - t0) v
+};
+
+template <typename F>
+__device__ __forceinline__ void outlier_boxes(const GridParams& g, const ORec& o, int32_t j,
+                                              int32_t jo0, int32_t jo1, F&& f) {
+    const double eps = 1e-12 * (fabs(g.tmin) + fabs(o.t0) + fabs(o.t1) + g.b);
+    const double ts = (j == jo0) ? o.t0 : fmax(o.t0, g.tmin + (double)j * g.b - eps);
+    const double te = (j == jo1) ? o.t1 : fmin(o.t1, g.tmin + (double)(j + 1) * g.b + eps);
+    double cross = 0.0;
+#pragma unroll
+    for (int a = 0; a < 3; ++a) cross = fmax(cross, fabs(o.v[a]) * (te - ts) * g.inv_w[a]);
+    const int S = (int)fmin(64.0, fmax(1.0, ceil(cross)));
+    for (int k = 0; k < S; ++k) {
+        const double ta = ts + (te - ts) * (double)k / (double)S;
+        const double tb = (k + 1 == S) ? te : ts + (te - ts) * (double)(k + 1) / (double)S;
+        int32_t lo[3], hi[3];
+#pragma unroll
+        for (int a = 0; a < 3; ++a) {
+            const double pa = o.x[a] + (ta - o.t0) * o.v[a];
+            const double pb = o.x[a] + (tb - o.t0) * o.v[a];
+            const double sl = 1e-12 * (fabs(pa) + fabs(pb) + g.w[a]);
+            lo[a] = cell_of(g, a, fmin(pa, pb) - sl);
+            hi[a] = cell_of(g, a, fmax(pa, pb) + sl);
+        }
+        f(lo, hi);
+    }
+}
+
+// Outlier state of an index (device pointers; okeys == NULL: no outliers).
+struct OutlierIndex {
+    const unsigned long long* okeys;   // sorted packed keys (key << shift | row) per position
+    const uint32_t* orows;             // bitmap over rows of D: 1 = outlier
+    int shift;
+};
+
 // 256-bit read-only load (sm_100: LDG.E.256; one 32-byte sector per lane).
 __device__ __forceinline__ double4 ld256(const double4* p) {
     double4 v;
@@ -367,6 +418,9 @@ struct dts_index {
     // index has produced after its spill buffer filled (search.cu)
     mutable std::atomic<unsigned long long> spill_hint{0};
     int eid_bits = 32;             // bits of the largest reported entry id
+    dts::OutlierIndex out{};       // long-segment copies (build.cu), okeys NULL if none
+    void* out_block = nullptr;     // backing memory of out (cache)
+    unsigned long long n_outliers = 0, n_copies = 0;
     dts::OocIndex* ooc = nullptr;  // set: D lives in pinned host temporal shards
 };
 

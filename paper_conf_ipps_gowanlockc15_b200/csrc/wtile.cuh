@@ -89,6 +89,7 @@ struct TileArgs {
     Counters* ctr;
     uint32_t method;
     SubbinIndex sb;
+    OutlierIndex out;                  // long-segment copies (okeys NULL: none)
 };
 
 __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
@@ -118,11 +119,107 @@ __device__ __forceinline__ void stage_hit(WarpSmem& S, int qi, uint32_t p, doubl
     }
 }
 
+// A hit on position p counts unless p holds a copy of an outlier that is not
+// the query's canonical copy (internal.cuh "outliers"): the least key among
+// the sub-slice boxes of the first bin the query probes whose boxes meet its
+// stencil box (the whole grid for a query that scans its bins' full range).
+// A pair within d is met in that bin and cell by construction, and copies
+// with equal packed keys (a repeated cell, or the midpoint filing) keep the
+// first position only: exactly one copy of each outlier yields the hit.
+struct OutlierArgs {                  // what the canonical-copy test reads
+    OutlierIndex out;
+    SegSoA soa;
+    const double* bin_t0min;
+    const double* bin_t1max;
+};
+
+__device__ __forceinline__ bool outlier_keep(const OutlierArgs& a, const GridParams& g,
+                                             const WarpSmem& S, int qi, uint32_t p) {
+    const unsigned long long pk = __ldg(a.out.okeys + p);
+    const uint32_t row = (uint32_t)(pk & ((1ull << a.out.shift) - 1ull));
+    if (!((__ldg(a.out.orows + (row >> 5)) >> (row & 31u)) & 1u)) return true;   // not an outlier
+    if (p > 0 && __ldg(a.out.okeys + p - 1) == pk) return false;                // repeated copy
+    const unsigned long long key = pk >> a.out.shift;
+    const QStencil qs = S.qs[qi];
+    double2 st, sx, sy, sz;
+    a.soa.load4(p, st, sx, sy, sz);
+    ORec o;
+    o.t0 = st.x; o.t1 = st.y;
+    o.x[0] = sx.x; o.x[1] = sy.x; o.x[2] = sz.x;
+    o.v[0] = sx.y; o.v[1] = sy.y; o.v[2] = sz.y;
+    const int32_t jo0 = bin_of(g, o.t0), jo1 = bin_of(g, o.t1);
+    int32_t blo[3], bhi[3];
+    for (int ax = 0; ax < 3; ++ax) {
+        const bool grid = qs.mode == MODE_GRID;
+        blo[ax] = grid ? qs.clo[ax] : 0;
+        bhi[ax] = grid ? qs.clo[ax] + qs.cn[ax] - 1 : g.nc[ax] - 1;
+    }
+    const double qt0 = S.qt0[qi], qt1 = S.qt1[qi];
+    for (int32_t j = max(qs.lb, jo0); j <= min(qs.hb, jo1); ++j) {
+        // interior bins a row probe skips (extent not overlapping the query)
+        if (qs.mode == MODE_GRID && j != qs.lb && j != qs.hb &&
+            !(__ldg(&a.bin_t0min[j]) < qt1 && __ldg(&a.bin_t1max[j]) > qt0))
+            continue;
+        unsigned long long best = ~0ull;
+        outlier_boxes(g, o, j, jo0, jo1, [&](const int32_t lo[3], const int32_t hi[3]) {
+            const int32_t cx = max(lo[0], blo[0]), cy = max(lo[1], blo[1]), cz = max(lo[2], blo[2]);
+            if (cx <= min(hi[0], bhi[0]) && cy <= min(hi[1], bhi[1]) && cz <= min(hi[2], bhi[2])) {
+                const unsigned long long k = make_key(g, j, cx, cy, cz);
+                best = k < best ? k : best;
+            }
+        });
+        if (best != ~0ull) return best == key;
+    }
+    return false;
+}
+
+// Warp-uniform, only for indexes with outliers: drop the staged hits on
+// non-canonical outlier copies (outlier_keep) and compact the stage; the
+// query counts are corrected.  Runs where register pressure is low (before
+// a flush and at the tile's end), not in the candidate loop.
+__device__ __forceinline__ void filter_outlier_hits(WarpSmem& S, const OutlierArgs& a,
+                                                   const GridParams& g, int lane) {
+    __syncwarp();
+    const uint32_t nh = min(S.nhit, (uint32_t)WH);
+    uint32_t kept = 0;
+    for (uint32_t b0 = 0; b0 < nh; b0 += 32) {
+        const uint32_t i = b0 + lane;
+        bool keep = false;
+        unsigned long long k = 0;
+        double r0 = 0.0, r1 = 0.0;
+        if (i < nh) {
+            k = S.hkey[i];
+            r0 = S.h0[i];
+            r1 = S.h1[i];
+            const int qi = (int)(k >> 42);
+            keep = outlier_keep(a, g, S, qi, (uint32_t)(k >> 10));
+            if (!keep) atomicSub(&S.qcount[qi], 1u);
+        }
+        const uint32_t bal = __ballot_sync(0xffffffffu, keep);
+        __syncwarp();
+        if (keep) {                               // compact in place (targets <= sources)
+            const uint32_t dst = kept + __popc(bal & ((1u << lane) - 1u));
+            S.hkey[dst] = (k & ~1023ull) | dst;
+            S.h0[dst] = r0;
+            S.h1[dst] = r1;
+        }
+        kept += __popc(bal);
+        __syncwarp();
+    }
+    if (lane == 0) S.nhit = kept;
+    __syncwarp();
+}
+
 // Warp-uniform: the shared stage's hits -> the global spill buffer as
 // records (local query id, entry id, interval); one atomic per flush.  A
 // flush that finds the buffer full marks the tile for a re-run and records
 // the first invalid slot (records from there on are not placed).
+template <bool OUT>
 __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int lane) {
+    if constexpr (OUT) {
+        if (!S.over)
+            filter_outlier_hits(S, OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g, lane);
+    }
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
     if (nh == 0 || S.over) return;
@@ -155,10 +252,11 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
 }
 
 // Flush when the next step (at most `step_max` hits) could overflow the stage.
+template <bool OUT>
 __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int lane,
                                             uint32_t step_max) {
     __syncwarp();
-    if (S.nhit > (uint32_t)WH - step_max) flush_spill(S, a, lane);
+    if (S.nhit > (uint32_t)WH - step_max) flush_spill<OUT>(S, a, lane);
 }
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
@@ -166,8 +264,9 @@ __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int 
 // queries (temporal / subbin methods) streamed per group of identical runs
 // (step 1a); the grid method compiles without it (its rare one-run
 // fallback queries go through the probe rounds).  EXCL: exclude pairs of
-// the same trajectory (compiled out of the plain search).
-template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false>
+// the same trajectory (compiled out of the plain search).  OUT: the index
+// has long-segment copies (the canonical-copy filter of the hits).
+template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false, bool OUT = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -276,7 +375,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         if (p == ~0u) p = __ldg(sb_ids(a.sb, lri) + slot);
                         stage_hit(S, qi, p, h0, h1);
                     }
-                    maybe_flush(S, a, lane, 32u);
+                    maybe_flush<OUT>(S, a, lane, 32u);
                 }
             }
         }
@@ -356,18 +455,23 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
                         stage_hit(S, qi2, p2, h0, h1);
                 }
-                maybe_flush(S, a, lane, 64u);
+                maybe_flush<OUT>(S, a, lane, 64u);
             }
         }
         __syncwarp();
 
         // ---- 2: counts; canonical staging, or the last spill flush
+        if constexpr (OUT) {
+            if (!S.over && !a.count_only)
+                filter_outlier_hits(S, OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g,
+                                    lane);
+        }
         const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
         if (lane < WQ && sp < a.nq) {
             a.counts[S.qid[lane]] = cnt;
             if (cnt) atomicMax(&a.ctr->max_count, cnt);
         }
-        if (a.spill_all || S.spilled) flush_spill(S, a, lane);
+        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane);
         __syncwarp();
         const uint32_t nh = S.nhit;
         bool over = S.over != 0u;

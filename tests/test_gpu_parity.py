@@ -207,8 +207,11 @@ def test_sampled_grid_misses_outliers(dts, oracle_mod, kind):
     for k, i in enumerate(pos):
         assert (400 + k, i) in hit, (kind, k)
     assert info["common"] >= len(pos)
-    if kind == "long_segments":          # exact extent, not the sample's
-        assert inf["max_extent"][0] >= 30.0
+    if kind == "long_segments":
+        # filed as copies along their path (outliers: extent far above the
+        # sample's mean), so the grid keeps the short segments' extent;
+        # without outlier filing the exact extent sizes the grid instead
+        assert inf["outlier_rows"] >= 6 or inf["max_extent"][0] >= 30.0, inf
     idx.free()
 
 
