@@ -22,6 +22,7 @@
 //                     entry is in exactly one cell).
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
 #include <cstdlib>
 
 #include "internal.cuh"
@@ -576,7 +577,7 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
                                             unsigned long long* __restrict__ bin_t1max,
                                             unsigned long long* __restrict__ count,
                                             const unsigned long long* s_key, int32_t* s_bin,
-                                            GatherSmem& sm) {
+                                            GatherSmem& sm, bool key_bins) {
     unsigned long long o0 = ~0ull, o1 = 0ull;
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
@@ -592,7 +593,11 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
                        make_double2(s0.z, velocity(s0.z, s1.z, dur)),
                        make_double2(s0.w, velocity(s0.w, s1.w, dur)));
             soa.eid[p] = id[k];
-            s_bin[1 + k * BT + threadIdx.x] = bin_of(g, s0.x);
+            // (with outlier copies a position's bin is its key's: a copy is
+            // filed in every bin its time spans, not only its start's)
+            s_bin[1 + k * BT + threadIdx.x] =
+                key_bins ? (int32_t)(s_key[1 + k * BT + threadIdx.x] / g.cells_per_bin)
+                         : bin_of(g, s0.x);
             const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);
             o0 = a < o0 ? a : o0;
             o1 = b > o1 ? b : o1;
@@ -664,7 +669,8 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
                                                     uint32_t* __restrict__ bin_start,
                                                     unsigned long long* __restrict__ bin_t0min,
                                                     unsigned long long* __restrict__ bin_t1max,
-                                                    unsigned long long* __restrict__ count) {
+                                                    unsigned long long* __restrict__ count,
+                                                    int key_bins) {
     constexpr int TILE = BT * ITEMS;
     __shared__ unsigned long long s_key[TILE + 1];
     __shared__ int32_t s_bin[TILE + 1];
@@ -705,7 +711,7 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
         }
     }
     gather_tile<ITEMS>(n, p0, id, r0, r1, soa, g, bin_start, bin_t0min, bin_t1max, count, s_key,
-                       s_bin, sm);
+                       s_bin, sm, key_bins != 0);
 }
 
 
@@ -1003,7 +1009,8 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     } evs;
     cudaEvent_t* ev = evs.ev;
     int nev = 0;
-    auto mark = [&] { DTS_CUDA(cudaEventRecord(ev[nev++], s)); };
+    // (at most 7 marks; a retried phase keeps its first mark)
+    auto mark = [&] { if (nev < 7) DTS_CUDA(cudaEventRecord(ev[nev++], s)); };
     mark();
 
     const int np = (int)std::min<size_t>(grid_for(n), 148 * 8);
@@ -1122,6 +1129,10 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             occ = occ_fraction();
             choose_grid(hs, p, g, n, occ);
         }
+        // the fused pass; a second attempt with the exact grid when the
+        // sample's grid was far off (the exact path below would drop the
+        // outlier filing)
+        for (int attempt = 0; attempt < 2 && !done; ++attempt) {
         const int kb = key_bits_of(g);
         if (row_bits + kb <= 64) {
             // 2-3. exact bounds + keys + sort histograms in one read of D
@@ -1161,7 +1172,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             cudaEvent_t eb;
             DTS_CUDA(cudaEventCreateWithFlags(&eb, cudaEventDisableTiming));
             DTS_CUDA(cudaEventRecord(eb, s));
-            mark();
+            if (attempt == 0) mark();
             bool drop_outliers = false;
             if (th.on) {
                 // outliers found: their copies join the keys before the sort
@@ -1180,7 +1191,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                     unsigned long long ncp = 0;
                     DTS_CUDA(cudaMemcpyAsync(&ncp, off.p + nout, 8, cudaMemcpyDeviceToHost, s));
                     DTS_CUDA(cudaStreamSynchronize(s));
-                    if (ncp > std::min<unsigned long long>(n / 2 + 1024, 1ull << 27) ||
+                    if (ncp > std::min<unsigned long long>(8ull * n + (1ull << 20), 1ull << 27) ||
                         n + ncp >= (1ull << 32)) {
                         drop_outliers = true;
                     } else {
@@ -1225,6 +1236,13 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                 const double slack = g.b * std::max(1.0, 0.1 * (double)g.m);
                 ok = ok && hb.tmin >= g.tmin - slack && hb.tmax <= g.tmin + (double)g.m * g.b + slack;
             }
+            static const bool dbg = getenv("DTS_DEBUG_BUILD") != nullptr;
+            if (dbg)
+                fprintf(stderr, "[dts build] n=%zu th.on=%d th=(%g %g %g | %g) nout=%llu nt=%zu "
+                                "drop=%d ok=%d g.b=%g gf.b=%g g.w=(%g %g %g) gf.w=(%g %g %g)\n",
+                        n, th.on, th.ext[0], th.ext[1], th.ext[2], th.dur,
+                        (unsigned long long)hb.nout, nt, (int)drop_outliers, (int)ok, g.b, gf.b,
+                        g.w[0], g.w[1], g.w[2], gf.w[0], gf.w[1], gf.w[2]);
             if (ok && !drop_outliers) {
                 for (int a = 0; a < 3; ++a) g.half_ext[a] = 0.5 * hb.ext[a];
                 g.maxdur = hb.maxdur;
@@ -1232,9 +1250,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                 idx->fused_keys = true;
                 done = true;
             } else {
-                nt = n;                         // the exact path files every entry once
+                nt = n;                         // start over (or the exact path below)
                 n_out = 0;
+                if (drop_outliers || !th.on) break;
+                g = gf;                         // retry once with the exact (main) grid
             }
+        } else {
+            break;
+        }
         }
     }
     if (!done) {
@@ -1316,13 +1339,15 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     }();
     if (gvar == 1)
         k_gather_cells<1, 6><<<grid_for(nt), BT, 0, s>>>(D, nt, sk, idx->soa, g, idx->bin_start,
-                                                        b0, b1, ncell.p);
+                                                        b0, b1, ncell.p, n_out ? 1 : 0);
     else if (gvar == 4)
         k_gather_cells<4, 2><<<grid_for((nt + 3) / 4), BT, 0, s>>>(D, nt, sk, idx->soa, g,
-                                                                  idx->bin_start, b0, b1, ncell.p);
+                                                                  idx->bin_start, b0, b1, ncell.p,
+                                                                  n_out ? 1 : 0);
     else
         k_gather_cells<2><<<grid_for((nt + 1) / 2), BT, 0, s>>>(D, nt, sk, idx->soa, g,
-                                                               idx->bin_start, b0, b1, ncell.p);
+                                                               idx->bin_start, b0, b1, ncell.p,
+                                                               n_out ? 1 : 0);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
