@@ -577,8 +577,10 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
                                             unsigned long long* __restrict__ bin_t1max,
                                             unsigned long long* __restrict__ count,
                                             const unsigned long long* s_key, int32_t* s_bin,
-                                            GatherSmem& sm, bool key_bins) {
+                                            GatherSmem& sm, bool key_bins,
+                                            const uint32_t* __restrict__ orows) {
     unsigned long long o0 = ~0ull, o1 = 0ull;
+    unsigned long long e0[ITEMS], e1[ITEMS];   // time extent each position gives its bin
 #pragma unroll
     for (int k = 0; k < ITEMS; ++k) {
         const size_t p = p0 + (size_t)k * BT + threadIdx.x;
@@ -595,12 +597,23 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
             soa.eid[p] = id[k];
             // (with outlier copies a position's bin is its key's: a copy is
             // filed in every bin its time spans, not only its start's)
-            s_bin[1 + k * BT + threadIdx.x] =
-                key_bins ? (int32_t)(s_key[1 + k * BT + threadIdx.x] / g.cells_per_bin)
-                         : bin_of(g, s0.x);
-            const unsigned long long a = ordered_bits(s0.x), b = ordered_bits(s1.x);
+            const int32_t bk = key_bins ? (int32_t)(s_key[1 + k * BT + threadIdx.x] / g.cells_per_bin)
+                                        : bin_of(g, s0.x);
+            s_bin[1 + k * BT + threadIdx.x] = bk;
+            double ta = s0.x, tb = s1.x;
+            if (orows && ((__ldg(orows + (id[k] >> 5)) >> (id[k] & 31u)) & 1u)) {
+                // an outlier's copy stands for its time inside this bin only
+                if (bk != bin_of(g, s0.x)) ta = fmax(ta, g.tmin + (double)bk * g.b);
+                if (bk != bin_of(g, s1.x)) tb = fmin(tb, g.tmin + (double)(bk + 1) * g.b);
+            }
+            const unsigned long long a = ordered_bits(ta), b = ordered_bits(tb);
+            e0[k] = a;
+            e1[k] = b;
             o0 = a < o0 ? a : o0;
             o1 = b > o1 ? b : o1;
+        } else {
+            e0[k] = ~0ull;
+            e1[k] = 0ull;
         }
     }
     __syncthreads();
@@ -650,9 +663,8 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
             const int loc = k * BT + threadIdx.x;
             if (p0 + (size_t)loc < n) {
                 const int32_t b = s_bin[loc + 1];
-                const double2 t = *soa.at(p0 + (size_t)loc);   // written above by this thread
-                atomicMin(&bin_t0min[b], ordered_bits(t.x));
-                atomicMax(&bin_t1max[b], ordered_bits(t.y));
+                atomicMin(&bin_t0min[b], e0[k]);
+                atomicMax(&bin_t1max[b], e1[k]);
             }
         }
     }
@@ -670,7 +682,8 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
                                                     unsigned long long* __restrict__ bin_t0min,
                                                     unsigned long long* __restrict__ bin_t1max,
                                                     unsigned long long* __restrict__ count,
-                                                    int key_bins) {
+                                                    int key_bins,
+                                                    const uint32_t* __restrict__ orows) {
     constexpr int TILE = BT * ITEMS;
     __shared__ unsigned long long s_key[TILE + 1];
     __shared__ int32_t s_bin[TILE + 1];
@@ -711,7 +724,7 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
         }
     }
     gather_tile<ITEMS>(n, p0, id, r0, r1, soa, g, bin_start, bin_t0min, bin_t1max, count, s_key,
-                       s_bin, sm, key_bins != 0);
+                       s_bin, sm, key_bins != 0, orows);
 }
 
 
@@ -1339,15 +1352,17 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     }();
     if (gvar == 1)
         k_gather_cells<1, 6><<<grid_for(nt), BT, 0, s>>>(D, nt, sk, idx->soa, g, idx->bin_start,
-                                                        b0, b1, ncell.p, n_out ? 1 : 0);
+                                                        b0, b1, ncell.p, n_out ? 1 : 0, n_out ? orows.p : nullptr);
     else if (gvar == 4)
         k_gather_cells<4, 2><<<grid_for((nt + 3) / 4), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                   idx->bin_start, b0, b1, ncell.p,
-                                                                  n_out ? 1 : 0);
+                                                                  n_out ? 1 : 0,
+                                                                  n_out ? orows.p : nullptr);
     else
         k_gather_cells<2><<<grid_for((nt + 1) / 2), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                idx->bin_start, b0, b1, ncell.p,
-                                                               n_out ? 1 : 0);
+                                                               n_out ? 1 : 0,
+                                                               n_out ? orows.p : nullptr);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
