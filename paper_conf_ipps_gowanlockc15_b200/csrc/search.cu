@@ -632,8 +632,14 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         const unsigned want = (tiles + WW - 1) / WW;
         const unsigned g7 = std::min<unsigned>(want, nsm * 7);
         if (args.out.okeys) {             // the index holds long-segment copies
-            if (args.excl) k_wtile_count<7, false, false, true, true><<<g7, WT, 0, s>>>(args);
-            else k_wtile_count<7, false, false, false, true><<<g7, WT, 0, s>>>(args);
+            if (args.count_only) {
+                if (args.excl) k_wtile_count<7, false, false, true, true, true><<<g7, WT, 0, s>>>(args);
+                else k_wtile_count<7, false, false, false, true, true><<<g7, WT, 0, s>>>(args);
+            } else if (args.excl) {
+                k_wtile_count<7, false, false, true, true><<<g7, WT, 0, s>>>(args);
+            } else {
+                k_wtile_count<7, false, false, false, true><<<g7, WT, 0, s>>>(args);
+            }
         } else if (args.excl) {           // exclude_same_trajectory instantiations
             if (idx->method == DTS_METHOD_SUBBIN) k_wtile_count<7, true, true, true><<<g7, WT, 0, s>>>(args);
             else if (idx->method == DTS_METHOD_TEMPORAL) k_wtile_count<7, false, true, true><<<g7, WT, 0, s>>>(args);

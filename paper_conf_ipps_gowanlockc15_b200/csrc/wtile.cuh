@@ -251,6 +251,22 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
     __syncwarp();
 }
 
+// A hit of the probe rounds: staged; in count-only mode on an index with
+// outlier copies, checked against the canonical copy right away (nothing is
+// staged to be filtered later).
+template <bool OUT, bool CNT>
+__device__ __forceinline__ void record_hit(WarpSmem& S, const TileArgs& a, int qi, uint32_t p,
+                                           double r0, double r1) {
+    if constexpr (OUT && CNT) {
+        {
+            if (outlier_keep(OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g, S, qi, p))
+                atomicAdd(&S.qcount[qi], 1u);
+            return;
+        }
+    }
+    stage_hit(S, qi, p, r0, r1);
+}
+
 // Flush when the next step (at most `step_max` hits) could overflow the stage.
 template <bool OUT>
 __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int lane,
@@ -265,8 +281,10 @@ __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int 
 // (step 1a); the grid method compiles without it (its rare one-run
 // fallback queries go through the probe rounds).  EXCL: exclude pairs of
 // the same trajectory (compiled out of the plain search).  OUT: the index
-// has long-segment copies (the canonical-copy filter of the hits).
-template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false, bool OUT = false>
+// has long-segment copies (the canonical-copy filter of the hits); CNT:
+// count-only search on such an index (the filter applied at each hit).
+template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false, bool OUT = false,
+          bool CNT = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -450,10 +468,10 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     const bool x1 = EXCL && __ldg(a.etraj + p1) == S.qtraj[qi1];
                     const bool x2 = EXCL && __ldg(a.etraj + p2) == S.qtraj[qi2];
                     if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
-                        stage_hit(S, qi1, p1, h0, h1);
+                        record_hit<OUT, CNT>(S, a, qi1, p1, h0, h1);
                     if (v2 && !x2 &&
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
-                        stage_hit(S, qi2, p2, h0, h1);
+                        record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1);
                 }
                 maybe_flush<OUT>(S, a, lane, 64u);
             }
