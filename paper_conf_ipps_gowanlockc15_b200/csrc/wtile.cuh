@@ -177,8 +177,10 @@ __device__ __forceinline__ bool outlier_keep(const OutlierArgs& a, const GridPar
 // non-canonical outlier copies (outlier_keep) and compact the stage; the
 // query counts are corrected.  Runs where register pressure is low (before
 // a flush and at the tile's end), not in the candidate loop.
-__device__ __forceinline__ void filter_outlier_hits(WarpSmem& S, const OutlierArgs& a,
-                                                   const GridParams& g, int lane) {
+__device__ __noinline__ void filter_outlier_hits(WarpSmem& S, const OutlierArgs* __restrict__ ap,
+                                                const GridParams* __restrict__ gp, int lane) {
+    const GridParams& g = *gp;
+    const OutlierArgs& a = *ap;
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
     uint32_t kept = 0;
@@ -215,10 +217,11 @@ __device__ __forceinline__ void filter_outlier_hits(WarpSmem& S, const OutlierAr
 // flush that finds the buffer full marks the tile for a re-run and records
 // the first invalid slot (records from there on are not placed).
 template <bool OUT>
-__device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int lane) {
+__device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int lane,
+                                            const OutlierArgs* oa = nullptr,
+                                            const GridParams* og = nullptr) {
     if constexpr (OUT) {
-        if (!S.over)
-            filter_outlier_hits(S, OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g, lane);
+        if (!S.over) filter_outlier_hits(S, oa, og, lane);
     }
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
@@ -270,9 +273,10 @@ __device__ __forceinline__ void record_hit(WarpSmem& S, const TileArgs& a, int q
 // Flush when the next step (at most `step_max` hits) could overflow the stage.
 template <bool OUT>
 __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int lane,
-                                            uint32_t step_max) {
+                                            uint32_t step_max, const OutlierArgs* oa = nullptr,
+                                            const GridParams* og = nullptr) {
     __syncwarp();
-    if (S.nhit > (uint32_t)WH - step_max) flush_spill<OUT>(S, a, lane);
+    if (S.nhit > (uint32_t)WH - step_max) flush_spill<OUT>(S, a, lane, oa, og);
 }
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
@@ -287,6 +291,18 @@ template <int MINB, bool SB = false, bool GROUP = false, bool EXCL = false, bool
           bool CNT = false>
 __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     __shared__ WarpSmem SW[WW];
+    // the grid and the outlier arrays in shared memory for the (out-of-line)
+    // canonical-copy filter: passing the kernel parameters' address would
+    // copy all of them to the stack
+    __shared__ GridParams s_g[OUT ? 1 : 1];
+    __shared__ OutlierArgs s_oa[OUT ? 1 : 1];
+    if (OUT) {
+        if (threadIdx.x == 0) {
+            s_g[0] = a.g;
+            s_oa[0] = OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max};
+        }
+        __syncthreads();
+    }
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     WarpSmem& S = SW[warp];
     const GridParams& g = a.g;
@@ -393,7 +409,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         if (p == ~0u) p = __ldg(sb_ids(a.sb, lri) + slot);
                         stage_hit(S, qi, p, h0, h1);
                     }
-                    maybe_flush<OUT>(S, a, lane, 32u);
+                    maybe_flush<OUT>(S, a, lane, 32u, s_oa, s_g);
                 }
             }
         }
@@ -473,7 +489,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
                         record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1);
                 }
-                maybe_flush<OUT>(S, a, lane, 64u);
+                maybe_flush<OUT>(S, a, lane, 64u, s_oa, s_g);
             }
         }
         __syncwarp();
@@ -481,15 +497,14 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         // ---- 2: counts; canonical staging, or the last spill flush
         if constexpr (OUT) {
             if (!S.over && !a.count_only)
-                filter_outlier_hits(S, OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g,
-                                    lane);
+                filter_outlier_hits(S, s_oa, s_g, lane);
         }
         const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
         if (lane < WQ && sp < a.nq) {
             a.counts[S.qid[lane]] = cnt;
             if (cnt) atomicMax(&a.ctr->max_count, cnt);
         }
-        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane);
+        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane, s_oa, s_g);
         __syncwarp();
         const uint32_t nh = S.nhit;
         bool over = S.over != 0u;
