@@ -578,7 +578,8 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
                                             unsigned long long* __restrict__ count,
                                             const unsigned long long* s_key, int32_t* s_bin,
                                             GatherSmem& sm, bool key_bins,
-                                            const uint32_t* __restrict__ orows) {
+                                            const uint32_t* __restrict__ orows,
+                                            uint32_t* __restrict__ obits) {
     unsigned long long o0 = ~0ull, o1 = 0ull;
     unsigned long long e0[ITEMS], e1[ITEMS];   // time extent each position gives its bin
 #pragma unroll
@@ -601,10 +602,17 @@ __device__ __forceinline__ void gather_tile(size_t n, size_t p0, const uint32_t 
                                         : bin_of(g, s0.x);
             s_bin[1 + k * BT + threadIdx.x] = bk;
             double ta = s0.x, tb = s1.x;
-            if (orows && ((__ldg(orows + (id[k] >> 5)) >> (id[k] & 31u)) & 1u)) {
+            const bool copy = orows && ((__ldg(orows + (id[k] >> 5)) >> (id[k] & 31u)) & 1u);
+            if (copy) {
                 // an outlier's copy stands for its time inside this bin only
                 if (bk != bin_of(g, s0.x)) ta = fmax(ta, g.tmin + (double)bk * g.b);
                 if (bk != bin_of(g, s1.x)) tb = fmin(tb, g.tmin + (double)(bk + 1) * g.b);
+            }
+            // bitmap of the positions holding copies (32 consecutive
+            // positions per warp and k: one ballot, one word)
+            if (obits) {
+                const uint32_t w = __ballot_sync(__activemask(), copy);
+                if ((threadIdx.x & 31) == 0) obits[p >> 5] = w;
             }
             const unsigned long long a = ordered_bits(ta), b = ordered_bits(tb);
             e0[k] = a;
@@ -683,7 +691,8 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
                                                     unsigned long long* __restrict__ bin_t1max,
                                                     unsigned long long* __restrict__ count,
                                                     int key_bins,
-                                                    const uint32_t* __restrict__ orows) {
+                                                    const uint32_t* __restrict__ orows,
+                                                    uint32_t* __restrict__ obits) {
     constexpr int TILE = BT * ITEMS;
     __shared__ unsigned long long s_key[TILE + 1];
     __shared__ int32_t s_bin[TILE + 1];
@@ -724,7 +733,7 @@ __global__ void __launch_bounds__(BT, MINB) k_gather_cells(const double4* __rest
         }
     }
     gather_tile<ITEMS>(n, p0, id, r0, r1, soa, g, bin_start, bin_t0min, bin_t1max, count, s_key,
-                       s_bin, sm, key_bins != 0, orows);
+                       s_bin, sm, key_bins != 0, orows, obits);
 }
 
 
@@ -1321,6 +1330,20 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     for (int a = 0; a < 3; ++a) idx->max_ext[a] = hb.ext[a];
 
     mark();
+    // outliers: the sorted packed keys (cell key << shift | row) and a bitmap
+    // of the positions holding copies stay with the index for the search's
+    // canonical-copy test
+    uint32_t* obits = nullptr;
+    if (n_out) {
+        const size_t kb8 = nt * sizeof(unsigned long long), rb = (nt / 32 + 1) * sizeof(uint32_t);
+        char* ob = static_cast<char*>(cache_alloc(kb8 + rb + 64));
+        idx->out_block = ob;
+        obits = reinterpret_cast<uint32_t*>(ob + kb8);
+        DTS_CUDA(cudaMemsetAsync(obits, 0, rb, s));
+        idx->out.okeys = reinterpret_cast<const unsigned long long*>(ob);
+        idx->out.obits = obits;
+        idx->out.shift = sk.shift;
+    }
     // 5. gather into the sorted record layout
     const size_t bytes_soa = nt * (4 * sizeof(double2) + sizeof(uint32_t));
     const size_t bytes_bins = 2 * (size_t)g.m * sizeof(double) + ((size_t)g.m + 1) * 4 + 16;
@@ -1352,17 +1375,17 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     }();
     if (gvar == 1)
         k_gather_cells<1, 6><<<grid_for(nt), BT, 0, s>>>(D, nt, sk, idx->soa, g, idx->bin_start,
-                                                        b0, b1, ncell.p, n_out ? 1 : 0, n_out ? orows.p : nullptr);
+                                                        b0, b1, ncell.p, n_out ? 1 : 0, n_out ? orows.p : nullptr, obits);
     else if (gvar == 4)
         k_gather_cells<4, 2><<<grid_for((nt + 3) / 4), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                   idx->bin_start, b0, b1, ncell.p,
                                                                   n_out ? 1 : 0,
-                                                                  n_out ? orows.p : nullptr);
+                                                                  n_out ? orows.p : nullptr, obits);
     else
         k_gather_cells<2><<<grid_for((nt + 1) / 2), BT, 0, s>>>(D, nt, sk, idx->soa, g,
                                                                idx->bin_start, b0, b1, ncell.p,
                                                                n_out ? 1 : 0,
-                                                               n_out ? orows.p : nullptr);
+                                                               n_out ? orows.p : nullptr, obits);
     DTS_LAUNCH_CHECK();
     k_ordered_to_double<<<grid_for(2 * (size_t)g.m), BT, 0, s>>>(b0, 2 * (size_t)g.m);
     DTS_LAUNCH_CHECK();
@@ -1395,21 +1418,12 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
     // cell into cell slots: 0.56 ms; these lane walks: 0.435)
     k_insert_blocks_lane<4, 32><<<grid_for((nt + 3) / 4), BT, 0, s>>>(sk, nt, idx->ht);
     DTS_LAUNCH_CHECK();
-    // outliers: the sorted packed keys (cell key << shift | row) and the row
-    // bitmap stay with the index for the search's canonical-copy test
     idx->n = nt;
     idx->n_outliers = n_out;
     idx->n_copies = nt - n;
-    if (n_out) {
-        const size_t kb8 = nt * sizeof(unsigned long long), rb = (n / 32 + 1) * sizeof(uint32_t);
-        char* ob = static_cast<char*>(cache_alloc(kb8 + rb + 64));
-        idx->out_block = ob;
-        DTS_CUDA(cudaMemcpyAsync(ob, sk.a, kb8, cudaMemcpyDeviceToDevice, s));
-        DTS_CUDA(cudaMemcpyAsync(ob + kb8, orows.p, rb, cudaMemcpyDeviceToDevice, s));
-        idx->out.okeys = reinterpret_cast<const unsigned long long*>(ob);
-        idx->out.orows = reinterpret_cast<const uint32_t*>(ob + kb8);
-        idx->out.shift = sk.shift;
-    }
+    if (n_out)
+        DTS_CUDA(cudaMemcpyAsync(idx->out_block, sk.a, nt * sizeof(unsigned long long),
+                                 cudaMemcpyDeviceToDevice, s));
     mark();
 
     // 7. GPUSpatioTemporal subbin arrays (DTS_METHOD_SUBBIN)

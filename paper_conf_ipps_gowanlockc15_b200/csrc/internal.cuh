@@ -247,7 +247,7 @@ __device__ __forceinline__ void outlier_boxes(const GridParams& g, const ORec& o
 // Outlier state of an index (device pointers; okeys == NULL: no outliers).
 struct OutlierIndex {
     const unsigned long long* okeys;   // sorted packed keys (key << shift | row) per position
-    const uint32_t* orows;             // bitmap over rows of D: 1 = outlier
+    const uint32_t* obits;             // bitmap over sorted positions: 1 = an outlier's copy
     int shift;
 };
 

@@ -133,14 +133,18 @@ struct OutlierArgs {                  // what the canonical-copy test reads
     const double* bin_t1max;
 };
 
-__device__ __forceinline__ bool outlier_keep(const OutlierArgs& a, const GridParams& g,
-                                             const WarpSmem& S, int qi, uint32_t p) {
+// Whether the copy at position p is the query's canonical copy of its
+// outlier.  Out of line: called for hits on outlier copies only.
+__device__ __noinline__ bool outlier_canonical(const OutlierArgs* __restrict__ ap,
+                                               const GridParams* __restrict__ gp,
+                                               const QStencil* __restrict__ qsp, double qt0,
+                                               double qt1, uint32_t p) {
+    const OutlierArgs& a = *ap;
+    const GridParams& g = *gp;
     const unsigned long long pk = __ldg(a.out.okeys + p);
-    const uint32_t row = (uint32_t)(pk & ((1ull << a.out.shift) - 1ull));
-    if (!((__ldg(a.out.orows + (row >> 5)) >> (row & 31u)) & 1u)) return true;   // not an outlier
     if (p > 0 && __ldg(a.out.okeys + p - 1) == pk) return false;                // repeated copy
     const unsigned long long key = pk >> a.out.shift;
-    const QStencil qs = S.qs[qi];
+    const QStencil qs = *qsp;
     double2 st, sx, sy, sz;
     a.soa.load4(p, st, sx, sy, sz);
     ORec o;
@@ -154,7 +158,6 @@ __device__ __forceinline__ bool outlier_keep(const OutlierArgs& a, const GridPar
         blo[ax] = grid ? qs.clo[ax] : 0;
         bhi[ax] = grid ? qs.clo[ax] + qs.cn[ax] - 1 : g.nc[ax] - 1;
     }
-    const double qt0 = S.qt0[qi], qt1 = S.qt1[qi];
     for (int32_t j = max(qs.lb, jo0); j <= min(qs.hb, jo1); ++j) {
         // interior bins a row probe skips (extent not overlapping the query)
         if (qs.mode == MODE_GRID && j != qs.lb && j != qs.hb &&
@@ -173,14 +176,17 @@ __device__ __forceinline__ bool outlier_keep(const OutlierArgs& a, const GridPar
     return false;
 }
 
-// Warp-uniform, only for indexes with outliers: drop the staged hits on
-// non-canonical outlier copies (outlier_keep) and compact the stage; the
-// query counts are corrected.  Runs where register pressure is low (before
-// a flush and at the tile's end), not in the candidate loop.
-__device__ __noinline__ void filter_outlier_hits(WarpSmem& S, const OutlierArgs* __restrict__ ap,
-                                                const GridParams* __restrict__ gp, int lane) {
-    const GridParams& g = *gp;
-    const OutlierArgs& a = *ap;
+__device__ __forceinline__ bool is_copy(const OutlierIndex& out, uint32_t p) {
+    return (__ldg(out.obits + (p >> 5)) >> (p & 31u)) & 1u;
+}
+
+// Warp-uniform, only for indexes with outliers: every staged hit's entry id
+// and copy flag are loaded together (one round trip, as the plain path's id
+// lookup); hits on copies that are not the query's canonical copy are
+// dropped, the stage compacted, the query counts corrected, and the kept
+// hits' positions replaced by their entry ids (hkey then holds entry ids).
+__device__ __forceinline__ void filter_resolve_ids(WarpSmem& S, const OutlierArgs* oa,
+                                                   const GridParams* og, int lane) {
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
     uint32_t kept = 0;
@@ -189,19 +195,25 @@ __device__ __noinline__ void filter_outlier_hits(WarpSmem& S, const OutlierArgs*
         bool keep = false;
         unsigned long long k = 0;
         double r0 = 0.0, r1 = 0.0;
+        uint32_t e = 0;
         if (i < nh) {
             k = S.hkey[i];
             r0 = S.h0[i];
             r1 = S.h1[i];
-            const int qi = (int)(k >> 42);
-            keep = outlier_keep(a, g, S, qi, (uint32_t)(k >> 10));
-            if (!keep) atomicSub(&S.qcount[qi], 1u);
+            const uint32_t p = (uint32_t)(k >> 10);
+            e = __ldg(oa->soa.eid + p);
+            keep = true;
+            if (is_copy(oa->out, p)) {
+                const int qi = (int)(k >> 42);
+                keep = outlier_canonical(oa, og, &S.qs[qi], S.qt0[qi], S.qt1[qi], p);
+                if (!keep) atomicSub(&S.qcount[qi], 1u);
+            }
         }
         const uint32_t bal = __ballot_sync(0xffffffffu, keep);
         __syncwarp();
         if (keep) {                               // compact in place (targets <= sources)
             const uint32_t dst = kept + __popc(bal & ((1u << lane) - 1u));
-            S.hkey[dst] = (k & ~1023ull) | dst;
+            S.hkey[dst] = (k & (0xFull << 42)) | ((unsigned long long)e << 10) | dst;
             S.h0[dst] = r0;
             S.h1[dst] = r1;
         }
@@ -221,7 +233,7 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
                                             const OutlierArgs* oa = nullptr,
                                             const GridParams* og = nullptr) {
     if constexpr (OUT) {
-        if (!S.over) filter_outlier_hits(S, oa, og, lane);
+        if (!S.over) filter_resolve_ids(S, oa, og, lane);
     }
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
@@ -241,7 +253,7 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
         const unsigned long long k = S.hkey[i];
         dts_result r;
         r.query_id = S.qid[(uint32_t)(k >> 42)];
-        r.entry_id = __ldg(a.soa.eid + (uint32_t)(k >> 10));
+        r.entry_id = OUT ? (uint32_t)(k >> 10) : __ldg(a.soa.eid + (uint32_t)(k >> 10));
         r.t_start = S.h0[i];
         r.t_end = S.h1[i];
         a.spill[b + i] = r;
@@ -259,13 +271,13 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
 // staged to be filtered later).
 template <bool OUT, bool CNT>
 __device__ __forceinline__ void record_hit(WarpSmem& S, const TileArgs& a, int qi, uint32_t p,
-                                           double r0, double r1) {
+                                           double r0, double r1, const OutlierArgs* oa,
+                                           const GridParams* og) {
     if constexpr (OUT && CNT) {
-        {
-            if (outlier_keep(OutlierArgs{a.out, a.soa, a.bin_t0min, a.bin_t1max}, a.g, S, qi, p))
-                atomicAdd(&S.qcount[qi], 1u);
-            return;
-        }
+        if (!is_copy(a.out, p) ||
+            outlier_canonical(oa, og, &S.qs[qi], S.qt0[qi], S.qt1[qi], p))
+            atomicAdd(&S.qcount[qi], 1u);
+        return;
     }
     stage_hit(S, qi, p, r0, r1);
 }
@@ -484,10 +496,10 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                     const bool x1 = EXCL && __ldg(a.etraj + p1) == S.qtraj[qi1];
                     const bool x2 = EXCL && __ldg(a.etraj + p2) == S.qtraj[qi2];
                     if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
-                        record_hit<OUT, CNT>(S, a, qi1, p1, h0, h1);
+                        record_hit<OUT, CNT>(S, a, qi1, p1, h0, h1, s_oa, s_g);
                     if (v2 && !x2 &&
                         refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
-                        record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1);
+                        record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1, s_oa, s_g);
                 }
                 maybe_flush<OUT>(S, a, lane, 64u, s_oa, s_g);
             }
@@ -495,9 +507,11 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         __syncwarp();
 
         // ---- 2: counts; canonical staging, or the last spill flush
+        // (OUT: the stage's ids are resolved, and its hits on non-canonical
+        //  copies dropped, by the flush below or right here)
         if constexpr (OUT) {
-            if (!S.over && !a.count_only)
-                filter_outlier_hits(S, s_oa, s_g, lane);
+            if (!S.over && !a.count_only && !(a.spill_all || S.spilled))
+                filter_resolve_ids(S, s_oa, s_g, lane);
         }
         const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
         if (lane < WQ && sp < a.nq) {
@@ -523,10 +537,12 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                 if (lane >= o) inc += u;
             }
             if (lane < WQ) S.qoff[lane] = inc - cnt;
-            for (uint32_t i = lane; i < nh; i += 32) {      // sorted position -> entry id
-                const unsigned long long k = S.hkey[i];
-                const uint32_t e = __ldg(a.soa.eid + (uint32_t)(k >> 10));
-                S.hkey[i] = (k & ~(0xffffffffull << 10)) | ((unsigned long long)e << 10);
+            if (!OUT) {
+                for (uint32_t i = lane; i < nh; i += 32) {  // sorted position -> entry id
+                    const unsigned long long k = S.hkey[i];
+                    const uint32_t e = __ldg(a.soa.eid + (uint32_t)(k >> 10));
+                    S.hkey[i] = (k & ~(0xffffffffull << 10)) | ((unsigned long long)e << 10);
+                }
             }
             unsigned long long b = 0;
             if (lane == 0) b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
