@@ -231,9 +231,10 @@ __device__ __forceinline__ void filter_resolve_ids(WarpSmem& S, const OutlierArg
 template <bool OUT>
 __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int lane,
                                             const OutlierArgs* oa = nullptr,
-                                            const GridParams* og = nullptr) {
+                                            const GridParams* og = nullptr,
+                                            bool resolved = false) {
     if constexpr (OUT) {
-        if (!S.over) filter_resolve_ids(S, oa, og, lane);
+        if (!S.over && !resolved) filter_resolve_ids(S, oa, og, lane);
     }
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
@@ -508,17 +509,16 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
 
         // ---- 2: counts; canonical staging, or the last spill flush
         // (OUT: the stage's ids are resolved, and its hits on non-canonical
-        //  copies dropped, by the flush below or right here)
+        //  copies dropped, before the counts are read)
         if constexpr (OUT) {
-            if (!S.over && !a.count_only && !(a.spill_all || S.spilled))
-                filter_resolve_ids(S, s_oa, s_g, lane);
+            if (!S.over && !a.count_only) filter_resolve_ids(S, s_oa, s_g, lane);
         }
         const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
         if (lane < WQ && sp < a.nq) {
             a.counts[S.qid[lane]] = cnt;
             if (cnt) atomicMax(&a.ctr->max_count, cnt);
         }
-        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane, s_oa, s_g);
+        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane, s_oa, s_g, true);
         __syncwarp();
         const uint32_t nh = S.nhit;
         bool over = S.over != 0u;
