@@ -106,7 +106,7 @@ __device__ void block_reduce_write(Bounds& b, Bounds* out) {
 
 // Segment validity (readings c4, c8): finite coordinates and times,
 // t_end >= t_start, finite velocity.  With thresholds, an outlier counts in
-// the domain (time range, spatial bounds) but not in the max extent and
+// the time range but not in the spatial bounds, the max extent and the
 // duration that size the grid and the stencils; returns whether the entry
 // is an outlier.
 __device__ __forceinline__ bool is_outlier(const Thresh& th, const double4 s0, const double4 s1) {
@@ -138,11 +138,15 @@ __device__ __forceinline__ bool bounds_add(Bounds& b, const double4 s0, const do
 #pragma unroll
     for (int a = 0; a < 3; ++a) {
         const double lo = fmin(p0[a], p1[a]), hi = fmax(p0[a], p1[a]);
-        b.lo[a] = fmin(b.lo[a], lo);
-        b.hi[a] = fmax(b.hi[a], hi);
         const double e = hi - lo;
         if (SUMS) b.sext[a] += e;
-        if (!outl) b.ext[a] = fmax(b.ext[a], e);
+        if (!outl) {
+            // the grid's domain is the main entries' (an outlier's copies
+            // clamp into the boundary cells like any point outside it)
+            b.lo[a] = fmin(b.lo[a], lo);
+            b.hi[a] = fmax(b.hi[a], hi);
+            b.ext[a] = fmax(b.ext[a], e);
+        }
         emax = fmax(emax, e);
     }
     // speed |p1 - p0| / dur must be finite on every axis: an infinite extent,
