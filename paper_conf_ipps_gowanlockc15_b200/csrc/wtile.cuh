@@ -185,7 +185,7 @@ __device__ __forceinline__ bool is_copy(const OutlierIndex& out, uint32_t p) {
 // lookup); hits on copies that are not the query's canonical copy are
 // dropped, the stage compacted, the query counts corrected, and the kept
 // hits' positions replaced by their entry ids (hkey then holds entry ids).
-__device__ __forceinline__ void filter_resolve_ids(WarpSmem& S, const OutlierArgs* oa,
+__device__ __noinline__ void filter_resolve_ids(WarpSmem& S, const OutlierArgs* oa,
                                                    const GridParams* og, int lane) {
     __syncwarp();
     const uint32_t nh = min(S.nhit, (uint32_t)WH);
