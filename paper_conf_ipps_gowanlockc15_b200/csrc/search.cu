@@ -563,7 +563,14 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 
     // ---- pass 1: warp tiles, count + staging (spilling output-heavy tiles)
     const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
-    const unsigned long long stage_cap = 4ull * nq + (1ull << 20);
+    // (DTS_STAGE_CAP: a fixed staging capacity, testing knob for the re-run
+    //  of tiles that find the stage full)
+    static const long long stage_env = [] {
+        const char* e = getenv("DTS_STAGE_CAP");
+        return e ? atoll(e) : -1ll;
+    }();
+    unsigned long long stage_cap = stage_env >= 0 ? (unsigned long long)stage_env
+                                                  : 4ull * nq + (1ull << 20);
     // spill buffer: sized from the largest output this index has seen (a
     // repeated output-heavy search spills without re-runs), at least 8
     // records per query
@@ -572,7 +579,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         const char* e = getenv("DTS_SPILL_CAP");
         return e ? atoll(e) : -1ll;
     }();
-    const unsigned long long spill_cap = spill_env >= 0 ? (unsigned long long)spill_env
+    unsigned long long spill_cap = spill_env >= 0 ? (unsigned long long)spill_env
         : std::max<unsigned long long>(8ull * nq + (1ull << 20),
                                        idx->spill_hint.load(std::memory_order_relaxed));
     DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s), spill_tiles(ntiles, s);
@@ -658,6 +665,55 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         DTS_LAUNCH_CHECK();
     };
     launch_pass1(ta, ntiles);
+    if (ta.out.okeys && !count_only) {
+        // ---- long-segment copies: spilled records carry sorted positions
+        //      and their tiles' counts include hits on non-canonical copies;
+        //      both are fixed before the scan (k_spill_filter).  A tile that
+        //      overflowed a buffer (counts unfiltered, or hits not kept)
+        //      sends pass 1 round again, the overflowed buffer sized by the
+        //      sum of the counts (an upper bound of what it must hold).
+        Counters c1;
+        DTS_CUDA(cudaMemcpyAsync(&c1, ctr.p, sizeof(c1), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        if (c1.n_over) {
+            scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
+            unsigned long long bound = 0;
+            DTS_CUDA(cudaMemcpyAsync(&bound, offsets.p + nq, sizeof(bound),
+                                     cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaStreamSynchronize(s));
+            if (c1.staged > stage_cap) {
+                stage_cap = std::max(stage_cap, bound);
+                stage.alloc(stage_cap, s);
+                ta.stage = stage.p;
+                ta.stage_cap = stage_cap;
+            }
+            if (c1.spill_valid != ~0ull) {
+                spill_cap = std::max(spill_cap, bound);
+                spill.alloc(std::max<unsigned long long>(spill_cap, 1), s);
+                ta.spill = spill.p;
+                ta.spill_cap = spill_cap;
+                unsigned long long want = bound + (1ull << 20), cur = idx->spill_hint.load();
+                while (cur < want && !idx->spill_hint.compare_exchange_weak(cur, want)) {}
+            }
+            DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
+            DTS_CUDA(cudaMemsetAsync(&ctr.p->spill_valid, 0xFF, sizeof(unsigned long long), s));
+            launch_pass1(ta, ntiles);
+            DTS_CUDA(cudaMemcpyAsync(&c1, ctr.p, sizeof(c1), cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaStreamSynchronize(s));
+            if (c1.n_over) throw Error(DTS_EINTERNAL, "pass 1 overflowed buffers sized by its counts");
+        }
+        const unsigned long long n1 = std::min(c1.spilled, spill_cap);
+        if (n1) {
+            k_spill_filter<<<(unsigned)std::min<unsigned long long>(blocks(n1, 128), nsm * 8ull), 128,
+                             0, s>>>(ta, n1, spill.p);
+            DTS_LAUNCH_CHECK();
+        }
+        if (c1.n_spill) {
+            k_spill_max<<<blocks((size_t)c1.n_spill * WQ, 128), 128, 0, s>>>(
+                spill_tiles.p, c1.n_spill, order.p, (uint32_t)nq, counts.p, ctr.p);
+            DTS_LAUNCH_CHECK();
+        }
+    }
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
     tm.mark();

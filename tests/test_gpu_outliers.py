@@ -132,3 +132,52 @@ def test_random_sets_with_long_segments(dts, oracle_mod):
         parity.compare(got, ora, D, Q, d, oracle_mod)
         total_long += int(inf["outlier_rows"])
     assert total_long > 100                              # the copies path was exercised
+
+
+def test_output_heavy_with_long_segments_all_buffer_paths(dts, oracle_mod):
+    """Output-heavy tiles on an index with copies: spilled records carry
+    sorted positions and are resolved and filtered after pass 1
+    (k_spill_filter); with the spill or the staging buffer forced small
+    (DTS_SPILL_CAP, DTS_STAGE_CAP) pass 1 goes round again with buffers sized
+    by its counts.  Same bytes every way, = plain filing, = the oracle."""
+    code = ("import sys; sys.path[:0] = [%r, %r]; import numpy as np, "
+            "paper_conf_ipps_gowanlockc15_b200 as m\n"
+            "D = np.load(sys.argv[1]); Q = np.load(sys.argv[2])\n"
+            "i = m.build_index(D); inf = i.info()\n"
+            "import os\n"
+            "if os.environ.get('DTS_OUTLIERS') != '0': assert inf['outlier_rows'] >= 20, inf\n"
+            "r = m.search(i, Q, 0.01); assert m.search_count(i, Q, 0.01)[0] == r.shape[0]\n"
+            "sys.stdout.buffer.write(r.tobytes())" % (REPO, os.path.join(REPO, "tests")))
+    g = np.random.default_rng(17)
+    n = 3000
+    D = np.zeros((n, 8))
+    D[:, 4] = 1.0
+    D[:, 1:4] = g.uniform(0, 0.05, (n, 3))
+    D[:, 5:8] = D[:, 1:4] + g.uniform(-0.002, 0.002, (n, 3))
+    L = np.zeros((24, 8))                     # 30 units of travel across the cube
+    L[:, 4] = 1.0
+    L[:, 1], L[:, 5] = -15.0, 15.0
+    L[:, [2, 3]] = g.uniform(0, 0.05, (24, 2))
+    L[:, [6, 7]] = L[:, [2, 3]]
+    L[::3, 5:8] = L[::3, 1:4] + [30.0, 0.02, -0.01]
+    D = np.ascontiguousarray(np.concatenate([D, L]))
+    Q = np.ascontiguousarray(D[g.choice(n, 300, replace=False)])
+    import tempfile
+    outs = []
+    with tempfile.TemporaryDirectory() as td:
+        np.save(os.path.join(td, "D.npy"), D)
+        np.save(os.path.join(td, "Q.npy"), Q)
+        for env in ({}, {"DTS_SPILL_CAP": "1000"}, {"DTS_SPILL_CAP": "0"},
+                    {"DTS_STAGE_CAP": "0"}, {"DTS_OUTLIERS": "0"}):
+            out = subprocess.run([sys.executable, "-c", code, os.path.join(td, "D.npy"),
+                                  os.path.join(td, "Q.npy")], env={**os.environ, **env},
+                                 capture_output=True, timeout=900)
+            assert out.returncode == 0, (env, out.stderr.decode()[-3000:])
+            outs.append(out.stdout)
+    assert all(o == outs[0] for o in outs[1:])
+    got = np.frombuffer(outs[0], dtype=dts.RESULT_DTYPE)
+    parity.assert_canonical(got)
+    info = parity.compare(got, oracle_mod.search(D, Q, 0.01, threads=THREADS), D, Q, 0.01,
+                          oracle_mod)
+    assert info["common"] > 30 * Q.shape[0]                   # output-heavy: tiles spill
+    assert np.isin(got["entry_id"], np.arange(n, D.shape[0])).sum() > 100   # copies hit
