@@ -19,3 +19,4 @@ for tool in memcheck racecheck synccheck; do
 done
 fi
 TAG=$TAG KERNELS="${KERNELS:-k_wtile_count}" bash scripts/gpu_prof.sh
+echo "== outliers"; timeout 900 python scripts/outlier_bench.py --plain --reps 20 > gpurun_out/${TAG}_outliers.jsonl 2> gpurun_out/${TAG}_outliers.err; echo "outliers rc=$?"; cut -c1-160 gpurun_out/${TAG}_outliers.jsonl

@@ -58,3 +58,32 @@ idx = dts.build_index(c2.D)
 r3 = dts.search(idx, c2.Q, 8.0)
 idx.free()
 print("sanitize workload 3 ok", r3.shape[0], flush=True)
+# long-segment outliers: copies, canonical filter in staged tiles, spilled
+# records filtered after pass 1 (k_spill_filter), count-only filter
+g = np.random.default_rng(17)
+n = 3000
+D = np.zeros((n, 8))
+D[:, 4] = 1.0
+D[:, 1:4] = g.uniform(0, 0.05, (n, 3))
+D[:, 5:8] = D[:, 1:4] + g.uniform(-0.002, 0.002, (n, 3))
+L = np.zeros((24, 8))
+L[:, 4] = 1.0
+L[:, 1], L[:, 5] = -15.0, 15.0
+L[:, [2, 3]] = g.uniform(0, 0.05, (24, 2))
+L[:, [6, 7]] = L[:, [2, 3]]
+D = np.ascontiguousarray(np.concatenate([D, L]))
+Q = np.ascontiguousarray(D[g.choice(n, 300, replace=False)])
+idx = dts.build_index(D)
+assert idx.info()["outlier_rows"] >= 20
+r4 = dts.search(idx, Q, 0.01)
+tot4 = dts.search_count(idx, Q, 0.01)[0]
+idx.free()
+# temporal shards in host memory (mem_budget_bytes), streamed results
+c5 = synth.make_config("C2", scale=0.01)
+idx = dts.build_index(c5.D, mem_budget_bytes=70 << 20)
+assert idx.info()["shards"] >= 2
+r5 = dts.search(idx, c5.Q, 2.0)
+chunks = []
+dts.search_stream(idx, c5.Q, 2.0, lambda a: chunks.append(a.shape[0]), chunk_results=5000)
+idx.free()
+print("sanitize workload 4 ok", r4.shape[0], tot4, r5.shape[0], sum(chunks), flush=True)
