@@ -44,7 +44,9 @@ def build(force: bool = False, verbose: bool = False) -> str:
     objs = []
     for src in sources():
         obj = os.path.join(objdir, os.path.basename(src) + ".o")
-        cmd = [NVCC, *FLAGS, "-I", INCLUDE, "-c", src, "-o", obj]
+        # DTS_NVCC_EXTRA: extra flags (A/B builds of compile-time variants)
+        extra = os.environ.get("DTS_NVCC_EXTRA", "").split()
+        cmd = [NVCC, *FLAGS, *extra, "-I", INCLUDE, "-c", src, "-o", obj]
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             sys.stderr.write(r.stdout + r.stderr)

@@ -56,6 +56,7 @@ struct Counters {                       // device-side statistics / flags
     unsigned int n_over;                // tiles re-run (spill buffer full)
     unsigned int n_spill;               // tiles whose hits were spilled
     unsigned int n_big;                 // spilled queries longer than a CTA sort
+    unsigned int n_mid;                 // spilled queries for the CTA sort
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
 };
@@ -633,7 +634,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     static const int occ = [] {
         const char* e = getenv("DTS_TILE_OCC");
         const int v = e ? atoi(e) : 7;
-        return (v == 6 || v == 8) ? v : 7;
+        return (v == 5 || v == 6 || v == 8) ? v : 7;
     }();
     auto launch_pass1 = [&](const TileArgs& args, uint32_t tiles) {
         const unsigned want = (tiles + WW - 1) / WW;
@@ -657,6 +658,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             k_wtile_count<7, false, true><<<g7, WT, 0, s>>>(args);
         } else if (occ == 8) {
             k_wtile_count<8><<<std::min<unsigned>(want, nsm * 8), WT, 0, s>>>(args);
+        } else if (occ == 5) {
+            k_wtile_count<5><<<std::min<unsigned>(want, nsm * 5), WT, 0, s>>>(args);
         } else if (occ == 6) {
             k_wtile_count<6><<<std::min<unsigned>(want, nsm * 6), WT, 0, s>>>(args);
         } else {
@@ -839,23 +842,32 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 }
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
-                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, sizeof(unsigned int), s));
+                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 2 * sizeof(unsigned int), s));
+                const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * WQ;
+                DevBuf<uint32_t> mid_list(nslots, s);
+                const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
-                    k_seg_sort<<<h.c.n_spill * WQ, SEG_T, 0, s>>>(
-                        spill_tiles.p, order.p, (uint32_t)nq, counts.p, offsets.p, raw.p, qmap,
-                        qid_base, fin, bigc.p, ctr.p);
+                    k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * WQ, 4), 128, 0, s>>>(
+                        spill_tiles.p, h.c.n_spill * WQ, order.p, (uint32_t)nq, counts.p,
+                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, bigc.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
-                    k_seg_sort<<<h.c.n_over * WQ, SEG_T, 0, s>>>(
-                        over_tiles.p, order.p, (uint32_t)nq, counts.p, offsets.p, raw.p, qmap,
-                        qid_base, fin, bigc.p, ctr.p);
+                    k_seg_sort_warp<<<blocks((size_t)h.c.n_over * WQ, 4), 128, 0, s>>>(
+                        over_tiles.p, h.c.n_over * WQ, order.p, (uint32_t)nq, counts.p,
+                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, bigc.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
-                unsigned int n_big = 0;
-                DTS_CUDA(cudaMemcpyAsync(&n_big, &ctr.p->n_big, sizeof(n_big),
+                unsigned int nbm[2] = {0, 0};                // n_big, n_mid
+                DTS_CUDA(cudaMemcpyAsync(nbm, &ctr.p->n_big, sizeof(nbm),
                                          cudaMemcpyDeviceToHost, s));
                 DTS_CUDA(cudaStreamSynchronize(s));
+                const unsigned int n_big = nbm[0];
+                if (nbm[1]) {
+                    k_seg_sort<<<nbm[1], SEG_T, 0, s>>>(mid_list.p, counts.p, offsets.p, raw.p,
+                                                        qmap, qid_base, fin);
+                    DTS_LAUNCH_CHECK();
+                }
                 if (n_big) {
                     // ---- segments longer than a CTA sort: one device-wide
                     //      keys-only radix sort over those only

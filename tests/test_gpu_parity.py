@@ -332,18 +332,34 @@ def test_empty_inputs(dts):
 
 
 def test_huge_result_segment(dts, oracle_mod):
-    """One query with > 4096 results exercises the radix-sorted segment path."""
+    """Spilled queries of every segment-sort size class in one tile: 300
+    results (a warp), 2,000 (a 256-thread CTA), 6,000 (a 1024-thread CTA)
+    and 17,000 (device-wide radix sort of long segments), with the entries
+    of each cluster in shuffled order."""
     g = synth.rng(77)
-    n = 6000
-    D = np.zeros((n, 8))
-    D[:, 0] = 0.0
-    D[:, 4] = 1.0
-    D[:, 1:4] = g.uniform(0, 0.01, size=(n, 3))
-    D[:, 5:8] = D[:, 1:4]
-    D = D[g.permutation(n)]
-    Q = np.array([[0.0, 0, 0, 0, 1.0, 0.005, 0.005, 0.005], [0.0, 0.5, 0.5, 0.5, 1.0, 1, 1, 1]])
+    parts = []
+    for k, m in enumerate((17000, 6000, 2000, 300)):
+        P = np.zeros((m, 8))
+        P[:, 4] = 1.0
+        P[:, 1:4] = k + g.uniform(0, 0.01, size=(m, 3))
+        P[:, 5:8] = P[:, 1:4]
+        parts.append(P)
+    D = np.concatenate(parts)
+    D = D[g.permutation(D.shape[0])]
+    Q = np.array([[0.0, k + 0.005, k + 0.005, k + 0.005, 1.0, k + 0.005, k + 0.005, k + 0.005]
+                  for k in range(4)] + [[0.0, 0.5, 0.5, 0.5, 1.0, 0.6, 0.6, 0.6]])
     got, info = run_and_compare(dts, oracle_mod, D, Q, 0.05)
-    assert info["common"] > 4096
+    assert np.array_equal(np.bincount(got["query_id"], minlength=5), [17000, 6000, 2000, 300, 0])
+    # caller entry ids over all 32 bits (four radix passes in the warp sort)
+    ids = ((g.permutation(D.shape[0]).astype(np.uint64) * 2654435761 + 12345) % (1 << 32)).astype(np.uint32)
+    idx = dts.build_index(D, entry_ids=ids)
+    got2 = dts.search(idx, Q, 0.05)
+    idx.free()
+    assert np.array_equal(got2["query_id"], got["query_id"])
+    for qi in range(4):
+        e = got2["entry_id"][got2["query_id"] == qi]
+        assert np.all(np.diff(e.astype(np.int64)) > 0)                 # canonical order
+        assert np.array_equal(np.sort(e), np.sort(ids[got["entry_id"][got["query_id"] == qi]]))
 
 
 def test_invalid_inputs_raise(dts):
