@@ -56,7 +56,8 @@ struct Counters {                       // device-side statistics / flags
     unsigned int n_over;                // tiles re-run (spill buffer full)
     unsigned int n_spill;               // tiles whose hits were spilled
     unsigned int n_big;                 // spilled queries longer than a CTA sort
-    unsigned int n_mid;                 // spilled queries for the CTA sort
+    unsigned int n_mid, n_large;        // spilled queries for the CTA sorts
+    unsigned int n_skew;                // ... whose ids cluster (radix sort)
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
 };
@@ -842,32 +843,65 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 }
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
-                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 2 * sizeof(unsigned int), s));
+                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 4 * sizeof(unsigned int), s));
                 const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * WQ;
-                DevBuf<uint32_t> mid_list(nslots, s);
+                DevBuf<uint32_t> mid_list(nslots, s), large_list(nslots, s);
                 const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * WQ, 4), 128, 0, s>>>(
                         spill_tiles.p, h.c.n_spill * WQ, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, bigc.p, ctr.p);
+                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, large_list.p, bigc.p,
+                        ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_over * WQ, 4), 128, 0, s>>>(
                         over_tiles.p, h.c.n_over * WQ, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, bigc.p, ctr.p);
+                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, large_list.p, bigc.p,
+                        ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
-                unsigned int nbm[2] = {0, 0};                // n_big, n_mid
+                unsigned int nbm[4] = {0, 0, 0, 0};   // n_big, n_mid, n_large, n_skew
                 DTS_CUDA(cudaMemcpyAsync(nbm, &ctr.p->n_big, sizeof(nbm),
                                          cudaMemcpyDeviceToHost, s));
                 DTS_CUDA(cudaStreamSynchronize(s));
-                const unsigned int n_big = nbm[0];
+                static const bool smem_ok = [] {
+                    return cudaFuncSetAttribute(k_seg_radix<1024, 16, 1>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_CAP * 8) == cudaSuccess &&
+                           cudaFuncSetAttribute(k_seg_bucket<1024, 16, 1>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_CAP * 12) == cudaSuccess &&
+                           cudaFuncSetAttribute(k_seg_bucket<512, 8, 2>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_MID * 12) == cudaSuccess;
+                }();
+                if (!smem_ok) throw Error(DTS_ECUDA, "segment sort: shared memory size refused");
+                DevBuf<uint32_t> skew_list(nbm[1] + nbm[2], s);
                 if (nbm[1]) {
-                    k_seg_sort<<<nbm[1], SEG_T, 0, s>>>(mid_list.p, counts.p, offsets.p, raw.p,
-                                                        qmap, qid_base, fin);
+                    k_seg_bucket<512, 8, 2><<<nbm[1], 512, SEG_MID * 12, s>>>(
+                        mid_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, fin,
+                        skew_list.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
+                if (nbm[2]) {
+                    k_seg_bucket<1024, 16, 1><<<nbm[2], 1024, SEG_CAP * 12, s>>>(
+                        large_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, fin,
+                        skew_list.p, ctr.p);
+                    DTS_LAUNCH_CHECK();
+                }
+                unsigned int n_skew = 0;
+                if (nbm[1] + nbm[2]) {
+                    DTS_CUDA(cudaMemcpyAsync(&n_skew, &ctr.p->n_skew, sizeof(n_skew),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                }
+                if (n_skew) {
+                    k_seg_radix<1024, 16, 1><<<n_skew, 1024, SEG_CAP * 8, s>>>(
+                        skew_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, eb, fin);
+                    DTS_LAUNCH_CHECK();
+                }
+                const unsigned int n_big = nbm[0];
                 if (n_big) {
                     // ---- segments longer than a CTA sort: one device-wide
                     //      keys-only radix sort over those only

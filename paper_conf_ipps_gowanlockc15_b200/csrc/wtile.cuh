@@ -729,8 +729,51 @@ __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restric
 // bitonic sorts up to 16,384 records lost to the device-wide radix sort
 // (canonicalisation 44 ms vs 39).
 constexpr int SEGW_CAP = 512;
-constexpr int SEG_CAP = 4096;
-constexpr int SEG_T = 256;
+constexpr int SEG_MID = 4096;                  // k_seg_radix<8>
+constexpr int SEG_CAP = 16384;                 // k_seg_radix<32>
+
+// A segment's (entry id << 32 | slot) keys into shared memory, and the
+// records gathered in key order into the output: UNR independent loads in
+// flight per thread (a plain loop waits for each load before its store).
+template <int UNR>
+__device__ __forceinline__ void seg_keys_load(unsigned long long* key, const dts_result* seg,
+                                              uint32_t c, uint32_t t, uint32_t nt) {
+    for (uint32_t b = t; b < c; b += nt * UNR) {
+        uint32_t e[UNR];
+#pragma unroll
+        for (int j = 0; j < UNR; ++j) {
+            const uint32_t i = b + (uint32_t)j * nt;
+            e[j] = i < c ? seg[i].entry_id : 0u;
+        }
+#pragma unroll
+        for (int j = 0; j < UNR; ++j) {
+            const uint32_t i = b + (uint32_t)j * nt;
+            if (i < c) key[i] = ((unsigned long long)e[j] << 32) | i;
+        }
+    }
+}
+
+template <int UNR>
+__device__ __forceinline__ void seg_gather(const unsigned long long* key, const dts_result* seg,
+                                           uint32_t c, uint32_t qrep, dts_result* out, uint32_t t,
+                                           uint32_t nt) {
+    for (uint32_t b = t; b < c; b += nt * UNR) {
+        dts_result r[UNR];
+#pragma unroll
+        for (int j = 0; j < UNR; ++j) {
+            const uint32_t i = b + (uint32_t)j * nt;
+            if (i < c) r[j] = seg[(uint32_t)(key[i] & 0xffffffffull)];
+        }
+#pragma unroll
+        for (int j = 0; j < UNR; ++j) {
+            const uint32_t i = b + (uint32_t)j * nt;
+            if (i < c) {
+                r[j].query_id = qrep;
+                out[i] = r[j];
+            }
+        }
+    }
+}
 
 struct SegWarpSmem {
     unsigned long long buf[2][SEGW_CAP];
@@ -748,6 +791,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
                                                       uint32_t qid_base, int eb,
                                                       dts_result* __restrict__ out,
                                                       uint32_t* __restrict__ mid_list,
+                                                      uint32_t* __restrict__ large_list,
                                                       uint32_t* __restrict__ bigc,
                                                       Counters* __restrict__ ctr) {
     __shared__ SegWarpSmem SWS[4];
@@ -761,8 +805,10 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     if (c == 0) return;
     if (c > (uint32_t)SEGW_CAP) {
         if (lane == 0) {
-            if (c <= (uint32_t)SEG_CAP) {
+            if (c <= (uint32_t)SEG_MID) {
                 mid_list[atomicAdd(&ctr->n_mid, 1u)] = q;
+            } else if (c <= (uint32_t)SEG_CAP) {
+                large_list[atomicAdd(&ctr->n_large, 1u)] = q;
             } else {
                 bigc[q] = c;
                 atomicAdd(&ctr->n_big, 1u);
@@ -773,8 +819,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     SegWarpSmem& S = SWS[warp];
     const unsigned long long off = offsets[q];
     const dts_result* seg = raw + off;
-    for (uint32_t i = lane; i < c; i += 32)
-        S.buf[0][i] = ((unsigned long long)seg[i].entry_id << 32) | i;
+    seg_keys_load<8>(S.buf[0], seg, c, lane, 32);
     const uint32_t lt = (1u << lane) - 1u;
     int cur = 0;
     for (int sh = 32; sh < 32 + eb; sh += 8, cur ^= 1) {
@@ -823,56 +868,208 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
             __syncwarp();
         }
     }
-    const unsigned long long* R = S.buf[cur];
+    __syncwarp();
     const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
-    for (uint32_t i = lane; i < c; i += 32) {
-        dts_result r = seg[(uint32_t)(R[i] & 0xffffffffull)];
-        r.query_id = qrep;
-        out[off + i] = r;
-    }
+    seg_gather<4>(S.buf[cur], seg, c, qrep, out + off, lane, 32);
 }
 
-// One CTA per listed query (SEGW_CAP < count <= SEG_CAP): the (entry id,
-// slot) keys bitonic-sorted in shared memory.
-__global__ void __launch_bounds__(SEG_T) k_seg_sort(const uint32_t* __restrict__ list,
-                                                   const uint32_t* __restrict__ counts,
-                                                   const unsigned long long* __restrict__ offsets,
-                                                   const dts_result* __restrict__ raw,
-                                                   const uint32_t* __restrict__ qmap,
-                                                   uint32_t qid_base,
-                                                   dts_result* __restrict__ out) {
-    __shared__ unsigned long long key[SEG_CAP];
+// One CTA of SEGC_T threads per listed query (SEGW_CAP < count <= SEGC_T *
+// ITEMS): an LSD radix sort of the (entry id << 32 | slot) keys over the
+// entry id bits, 8 bits per pass, the keys in one shared-memory buffer
+// between passes.  Per pass a warp ranks its contiguous range of keys
+// (ballot multisplit, ITEMS keys per lane kept in registers with their
+// ranks), the per-warp digit counts are scanned across warps and digits,
+// and every key is stored at its stable position (all keys are in
+// registers by then, so the buffer is overwritten in place).
+template <int SEGC_T, int ITEMS, int MINB>
+__global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __restrict__ list,
+                                                        const uint32_t* __restrict__ counts,
+                                                        const unsigned long long* __restrict__ offsets,
+                                                        const dts_result* __restrict__ raw,
+                                                        const uint32_t* __restrict__ qmap,
+                                                        uint32_t qid_base, int eb,
+                                                        dts_result* __restrict__ out) {
+    constexpr int SEGC_W = SEGC_T / 32;
+    extern __shared__ unsigned long long sbuf[];        // SEGC_T * ITEMS keys
+    __shared__ uint32_t wcnt[SEGC_W][257];
+    __shared__ uint32_t wtot[8];
     const uint32_t q = list[blockIdx.x];
     const uint32_t c = counts[q];
     const unsigned long long off = offsets[q];
     const dts_result* seg = raw + off;
-    const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
-    uint32_t N = 1;
-    while (N < c) N <<= 1;
-    for (uint32_t i = threadIdx.x; i < N; i += SEG_T)
-        key[i] = i < c ? (((unsigned long long)seg[i].entry_id << 32) | i) : ~0ull;
-    __syncthreads();
-    for (uint32_t k = 2; k <= N; k <<= 1) {
-        for (uint32_t j = k >> 1; j > 0; j >>= 1) {
-            for (uint32_t i = threadIdx.x; i < N; i += SEG_T) {
-                const uint32_t l = i ^ j;
-                if (l > i) {
-                    const unsigned long long a = key[i], b = key[l];
-                    const bool up = (i & k) == 0;
-                    if ((a > b) == up) {
-                        key[i] = b;
-                        key[l] = a;
-                    }
-                }
+    const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    seg_keys_load<8>(sbuf, seg, c, t, SEGC_T);
+    const uint32_t lt = (1u << lane) - 1u;
+    const uint32_t wbase = warp * 32u * ITEMS;
+    for (int sh = 32; sh < 32 + eb; sh += 8) {
+        for (uint32_t j = lane; j < 257; j += 32) wcnt[warp][j] = 0;
+        __syncthreads();
+        unsigned long long k[ITEMS];
+        uint32_t rk[ITEMS / 2];                      // two 16-bit ranks per word
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t p = wbase + (uint32_t)i * 32u + lane;
+            const bool valid = p < c;
+            k[i] = valid ? sbuf[p] : 0ull;
+            const uint32_t dig = valid ? ((uint32_t)(k[i] >> sh) & 255u) : 256u;
+            uint32_t peers = 0xffffffffu;
+#pragma unroll
+            for (int b = 0; b < 9; ++b) {
+                const uint32_t bal = __ballot_sync(0xffffffffu, (dig >> b) & 1u);
+                peers &= ((dig >> b) & 1u) ? bal : ~bal;
             }
-            __syncthreads();
+            const uint32_t base = wcnt[warp][dig];
+            __syncwarp();
+            if (lane == 31u - __clz(peers)) wcnt[warp][dig] = base + __popc(peers);
+            const uint32_t r = base + __popc(peers & lt);
+            rk[i / 2] = (i & 1) ? (rk[i / 2] | (r << 16)) : r;
+            __syncwarp();
+        }
+        __syncthreads();
+        // digit d (thread d < 256): counts of the warps before -> per-warp
+        // base, then an exclusive scan of the digit totals
+        uint32_t tot = 0;
+        if (t < 256) {
+#pragma unroll
+            for (int w = 0; w < SEGC_W; ++w) {
+                const uint32_t x = wcnt[w][t];
+                wcnt[w][t] = tot;
+                tot += x;
+            }
+        }
+        uint32_t inc = tot;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= (uint32_t)o) inc += u;
+        }
+        if (t < 256 && lane == 31) wtot[warp] = inc;
+        __syncthreads();
+        if (t < 256) {
+            uint32_t pre = inc - tot;
+            for (uint32_t w = 0; w < warp; ++w) pre += wtot[w];
+#pragma unroll
+            for (int w = 0; w < SEGC_W; ++w) wcnt[w][t] += pre;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int i = 0; i < ITEMS; ++i) {
+            const uint32_t p = wbase + (uint32_t)i * 32u + lane;
+            if (p < c)
+                sbuf[wcnt[warp][(uint32_t)(k[i] >> sh) & 255u] + ((rk[i / 2] >> (16 * (i & 1))) & 0xffffu)] = k[i];
+        }
+        __syncthreads();
+    }
+    const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
+    seg_gather<4>(sbuf, seg, c, qrep, out + off, t, SEGC_T);
+}
+
+// One CTA of T threads per listed query (SEGW_CAP < count <= CAP): a
+// counting sort on the high bits of (entry id - the segment's least id)
+// into about one bucket per record (shared-memory atomics, no ranking
+// ballots), then an insertion sort of each bucket by one thread.  A segment
+// whose ids cluster (a bucket over SEGB_MAX records) is sorted by the
+// ballot-ranked radix sort instead (queued on skew_list).  Measured on S2 at
+// d = 1 (292 M records in segments of 4,097-16,384): the radix sort's
+// ballot multisplit (9 ballots per key per 8-bit pass) took 13.0 ms.
+constexpr int SEGB_MAX = 32;
+
+template <int T, int ITEMS, int MINB>
+__global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restrict__ list,
+                                                       const uint32_t* __restrict__ counts,
+                                                       const unsigned long long* __restrict__ offsets,
+                                                       const dts_result* __restrict__ raw,
+                                                       const uint32_t* __restrict__ qmap,
+                                                       uint32_t qid_base,
+                                                       dts_result* __restrict__ out,
+                                                       uint32_t* __restrict__ skew_list,
+                                                       Counters* __restrict__ ctr) {
+    constexpr uint32_t CAP = (uint32_t)T * ITEMS;
+    extern __shared__ unsigned long long bbuf[];        // CAP keys, then CAP bucket counters
+    uint32_t* cnt = reinterpret_cast<uint32_t*>(bbuf + CAP);
+    __shared__ uint32_t s_min, s_max, s_bmax, s_wsum[T / 32];
+    const uint32_t q = list[blockIdx.x];
+    const uint32_t c = counts[q];
+    const unsigned long long off = offsets[q];
+    const dts_result* seg = raw + off;
+    const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    if (t == 0) { s_min = ~0u; s_max = 0u; s_bmax = 0u; }
+    // ---- the segment's ids, held in registers (slot t + j*T), and their range
+    uint32_t e[ITEMS];
+    uint32_t mn = ~0u, mx = 0u;
+#pragma unroll
+    for (int j = 0; j < ITEMS; ++j) {
+        const uint32_t i = t + (uint32_t)j * T;
+        e[j] = i < c ? seg[i].entry_id : 0u;
+    }
+#pragma unroll
+    for (int j = 0; j < ITEMS; ++j) {
+        if (t + (uint32_t)j * T < c) { mn = min(mn, e[j]); mx = max(mx, e[j]); }
+    }
+    mn = __reduce_min_sync(0xffffffffu, mn);
+    mx = __reduce_max_sync(0xffffffffu, mx);
+    uint32_t nb = 32;
+    while (nb < c) nb <<= 1;
+    for (uint32_t i = t; i < nb; i += T) cnt[i] = 0;
+    __syncthreads();
+    if (lane == 0) { atomicMin(&s_min, mn); atomicMax(&s_max, mx); }
+    __syncthreads();
+    mn = s_min;
+    const uint32_t span = s_max - mn;
+    const int sbits = span ? 32 - __clz(span) : 0;
+    const int lnb = 31 - __clz(nb);
+    const int sh = sbits > lnb ? sbits - lnb : 0;
+    // ---- bucket counts
+#pragma unroll
+    for (int j = 0; j < ITEMS; ++j)
+        if (t + (uint32_t)j * T < c) atomicAdd(&cnt[(e[j] - mn) >> sh], 1u);
+    __syncthreads();
+    // ---- exclusive scan of the counters (nb / T per thread, consecutive)
+    const uint32_t per = (nb + T - 1) / T, b0 = t * per;
+    uint32_t sum = 0, bmax = 0;
+    for (uint32_t j = 0; j < per; ++j) {
+        if (b0 + j < nb) { const uint32_t x = cnt[b0 + j]; sum += x; bmax = max(bmax, x); }
+    }
+    bmax = __reduce_max_sync(0xffffffffu, bmax);
+    uint32_t inc = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= (uint32_t)o) inc += u;
+    }
+    if (lane == 31) s_wsum[warp] = inc;
+    if (lane == 0) atomicMax(&s_bmax, bmax);
+    __syncthreads();
+    if (s_bmax > (uint32_t)SEGB_MAX) {              // clustered ids: the radix sort
+        if (t == 0) skew_list[atomicAdd(&ctr->n_skew, 1u)] = q;
+        return;
+    }
+    uint32_t run = inc - sum;
+    for (uint32_t w = 0; w < warp; ++w) run += s_wsum[w];
+    for (uint32_t j = 0; j < per; ++j) {
+        if (b0 + j < nb) { const uint32_t x = cnt[b0 + j]; cnt[b0 + j] = run; run += x; }
+    }
+    __syncthreads();
+    // ---- scatter into the buckets (cnt[b] ends at the end of bucket b)
+#pragma unroll
+    for (int j = 0; j < ITEMS; ++j) {
+        const uint32_t i = t + (uint32_t)j * T;
+        if (i < c) bbuf[atomicAdd(&cnt[(e[j] - mn) >> sh], 1u)] = ((unsigned long long)e[j] << 32) | i;
+    }
+    __syncthreads();
+    // ---- each bucket sorted by one thread (insertion sort, <= SEGB_MAX keys)
+    for (uint32_t b = t; b < nb; b += T) {
+        const uint32_t lo = b ? cnt[b - 1] : 0u, hi = cnt[b];
+        for (uint32_t i = lo + 1; i < hi; ++i) {
+            const unsigned long long k = bbuf[i];
+            uint32_t j = i;
+            while (j > lo && bbuf[j - 1] > k) { bbuf[j] = bbuf[j - 1]; --j; }
+            bbuf[j] = k;
         }
     }
-    for (uint32_t i = threadIdx.x; i < c; i += SEG_T) {
-        dts_result r = seg[(uint32_t)(key[i] & 0xffffffffull)];
-        r.query_id = qrep;
-        out[off + i] = r;
-    }
+    __syncthreads();
+    const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
+    seg_gather<4>(bbuf, seg, c, qrep, out + off, t, T);
 }
 
 // Segments longer than SEG_CAP: one device-wide keys-only radix sort of

@@ -360,6 +360,19 @@ def test_huge_result_segment(dts, oracle_mod):
         e = got2["entry_id"][got2["query_id"] == qi]
         assert np.all(np.diff(e.astype(np.int64)) > 0)                 # canonical order
         assert np.array_equal(np.sort(e), np.sort(ids[got["entry_id"][got["query_id"] == qi]]))
+    # clustered ids (one far id per query widens the id range): the bucket
+    # sort's buckets overflow and those segments go to the radix sort
+    ids3 = np.arange(D.shape[0], dtype=np.uint32)
+    for qi in (1, 2):
+        ids3[got["entry_id"][got["query_id"] == qi][7]] = 4_000_000_000 + qi
+    idx = dts.build_index(D, entry_ids=ids3)
+    got3 = dts.search(idx, Q, 0.05)
+    idx.free()
+    assert np.array_equal(got3["query_id"], got["query_id"])
+    for qi in range(4):
+        e = got3["entry_id"][got3["query_id"] == qi]
+        assert np.all(np.diff(e.astype(np.int64)) > 0)
+        assert np.array_equal(np.sort(e), np.sort(ids3[got["entry_id"][got["query_id"] == qi]]))
 
 
 def test_invalid_inputs_raise(dts):
