@@ -177,7 +177,8 @@ __global__ void __launch_bounds__(BT) k_bounds(const double4* __restrict__ D, si
 // arithmetic progressions of the old grid's block keys better than random.)
 __global__ void __launch_bounds__(BT) k_bounds_sample(const double4* __restrict__ D, size_t n,
                                                      size_t S, Bounds* __restrict__ partial,
-                                                     Thresh th) {
+                                                     const Thresh* __restrict__ thp) {
+    const Thresh th = thp ? *thp : Thresh{{0, 0, 0}, 0, 0};
     Bounds b;
     bounds_init(b);
     for (size_t j = (size_t)blockIdx.x * BT + threadIdx.x; j < S; j += (size_t)gridDim.x * BT) {
@@ -185,6 +186,26 @@ __global__ void __launch_bounds__(BT) k_bounds_sample(const double4* __restrict_
         bounds_add(b, D[2 * i], D[2 * i + 1], th);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
+}
+
+// Outlier thresholds from the sample's bounds (grid method): 8x the mean
+// extent per axis and the mean duration, at least a thousandth of the
+// sample's span (on the device: the second sample pass follows without a
+// host round trip).
+struct SampleOut {
+    Bounds b;          // the sample's bounds without the outliers
+    Thresh th;
+};
+__global__ void k_thresh(const Bounds* __restrict__ b, Thresh* __restrict__ th) {
+    const Bounds x = *b;
+    Thresh t{{0, 0, 0}, 0, 0};
+    if (x.cnt > 0 && !x.bad) {
+        const double c = (double)x.cnt;
+        for (int a = 0; a < 3; ++a) t.ext[a] = fmax(8.0 * x.sext[a] / c, 1e-3 * (x.hi[a] - x.lo[a]));
+        t.dur = fmax(8.0 * x.sdur / c, 1e-3 * (x.tmax - x.tmin));
+        t.on = 1;
+    }
+    *th = t;
 }
 
 __global__ void __launch_bounds__(BT) k_bounds_final(const Bounds* __restrict__ partial, int np,
@@ -287,8 +308,9 @@ __device__ __forceinline__ void note_outlier(const OutlierOut& oo, size_t i) {
     if (k < oo.ocap) oo.olist[k] = (uint32_t)i;
 }
 
-// OUT: thresholds on (outliers flagged and listed), one entry per thread
-// step; else two in flight and no outlier code (its registers spilled)
+// OUT: thresholds on (outliers flagged and listed); two entries in flight
+// per thread step either way (one at a time with outliers measured 0.416 ms
+// on C4 against 0.32 without)
 template <int MINB, bool OUT>
 __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restrict__ D, size_t n,
                                                       GridParams g,
@@ -311,34 +333,28 @@ __global__ void __launch_bounds__(BT, MINB) k_bounds_keys(const double4* __restr
     const size_t stride = (size_t)gridDim.x * BT;
     size_t i = (size_t)blockIdx.x * BT + threadIdx.x;
     const Thresh thr = OUT ? th : Thresh{{0, 0, 0}, 0, 0};
-    if (OUT) {
-        for (; i < n; i += stride) {
-            const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
-            if (bounds_add<false>(b, a0, a1, thr)) note_outlier(oo, i);
-            const unsigned long long va = packed_key(g, a0, a1, shift, i);
-            keys[i] = va;
-            count(va);
-        }
-    }
     for (; i + stride < n; i += 2 * stride) {      // two entries in flight per thread
         const size_t j = i + stride;
         const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
         const double4 c0 = ld256(D + 2 * j), c1 = ld256(D + 2 * j + 1);
-        bounds_add<false>(b, a0, a1, thr);
-        bounds_add<false>(b, c0, c1, thr);
+        const bool oa = bounds_add<false>(b, a0, a1, thr);
+        const bool oc = bounds_add<false>(b, c0, c1, thr);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
         const unsigned long long vc = packed_key(g, c0, c1, shift, j);
         keys[i] = va;
         keys[j] = vc;
         count(va);
         count(vc);
+        if (OUT && oa) note_outlier(oo, i);
+        if (OUT && oc) note_outlier(oo, j);
     }
     if (i < n) {
         const double4 a0 = ld256(D + 2 * i), a1 = ld256(D + 2 * i + 1);
-        bounds_add<false>(b, a0, a1, thr);
+        const bool oa = bounds_add<false>(b, a0, a1, thr);
         const unsigned long long va = packed_key(g, a0, a1, shift, i);
         keys[i] = va;
         count(va);
+        if (OUT && oa) note_outlier(oo, i);
     }
     block_reduce_write(b, &partial[blockIdx.x]);
     __syncthreads();
@@ -1119,30 +1135,39 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         }();
         const size_t S = std::min<size_t>(n, (size_t)1 << slog);
         const int nps = (int)std::min<size_t>(std::max<size_t>(grid_for(S) / 4, 1), 592);
-        k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, Thresh{{0, 0, 0}, 0, 0});
-        DTS_LAUNCH_CHECK();
-        k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
-        DTS_LAUNCH_CHECK();
-        Bounds hs;
-        DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
-        DTS_CUDA(cudaStreamSynchronize(s));
-        check(hs);
-        // outlier thresholds (grid method): 8x the sample's mean extent per
-        // axis and mean duration, at least a thousandth of the sample's span;
-        // the sample's bounds are then taken again without the outliers
-        if (outliers_on && p.method == DTS_METHOD_GRID && hs.cnt > 0) {
-            const double c = (double)hs.cnt;
-            for (int a = 0; a < 3; ++a)
-                th.ext[a] = std::max(8.0 * hs.sext[a] / c, 1e-3 * (hs.hi[a] - hs.lo[a]));
-            th.dur = std::max(8.0 * hs.sdur / c, 1e-3 * (hs.tmax - hs.tmin));
-            th.on = 1;
-            k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, th);
-            DTS_LAUNCH_CHECK();
-            k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, total.p);
-            DTS_LAUNCH_CHECK();
-            DTS_CUDA(cudaMemcpyAsync(&hs, total.p, sizeof(Bounds), cudaMemcpyDeviceToHost, s));
-            DTS_CUDA(cudaStreamSynchronize(s));
+        const bool want_out = outliers_on && p.method == DTS_METHOD_GRID;
+        // the outlier list's buffers do not depend on the sample: allocated
+        // before the host waits for it
+        if (want_out) {
+            orows.alloc(n / 32 + 1, s);
+            olist.alloc(std::min<size_t>(n, (size_t)(n / 64) + 4096), s);
+            ocount.alloc(1, s);
+            DTS_CUDA(cudaMemsetAsync(orows.p, 0, (n / 32 + 1) * 4, s));
+            DTS_CUDA(cudaMemsetAsync(ocount.p, 0, 4, s));
         }
+        DevBuf<SampleOut> so(1, s);
+        k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, nullptr);
+        DTS_LAUNCH_CHECK();
+        k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, want_out ? total.p : &so.p->b);
+        DTS_LAUNCH_CHECK();
+        if (want_out) {
+            // thresholds on the device, then the sample's bounds without the
+            // outliers; one host round trip for both
+            k_thresh<<<1, 1, 0, s>>>(total.p, &so.p->th);
+            DTS_LAUNCH_CHECK();
+            k_bounds_sample<<<nps, BT, 0, s>>>(D, n, S, partial.p, &so.p->th);
+            DTS_LAUNCH_CHECK();
+            k_bounds_final<<<1, BT, 0, s>>>(partial.p, nps, &so.p->b);
+            DTS_LAUNCH_CHECK();
+        } else {
+            DTS_CUDA(cudaMemsetAsync(&so.p->th, 0, sizeof(Thresh), s));
+        }
+        SampleOut hso;
+        DTS_CUDA(cudaMemcpyAsync(&hso, so.p, sizeof(SampleOut), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        Bounds hs = hso.b;
+        check(hs);
+        th = hso.th;
         mark();
         // the occupancy only matters when even a full box would be capped
         // (C3); dense or clustered data (C4, C2, S3) skip its kernel
@@ -1150,7 +1175,7 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
         choose_grid(hs, p, g, n, 1.0, &capped);
         occ = 1.0;
         if (capped) {
-            occ_launch(S, total.p);
+            occ_launch(S, &so.p->b);
             DTS_CUDA(cudaStreamSynchronize(s));
             occ = occ_fraction();
             choose_grid(hs, p, g, n, occ);
@@ -1175,11 +1200,10 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                 bk_minb == 3 ? (const void*)k_bounds_keys<3, false> : (const void*)k_bounds_keys<4, false>), np);
             OutlierOut oo{};
             if (th.on) {
-                orows.alloc(n / 32 + 1, s);
-                olist.alloc(std::min<size_t>(n, (size_t)(n / 64) + 4096), s);
-                ocount.alloc(1, s);
-                DTS_CUDA(cudaMemsetAsync(orows.p, 0, (n / 32 + 1) * 4, s));
-                DTS_CUDA(cudaMemsetAsync(ocount.p, 0, 4, s));
+                if (attempt > 0) {                    // the first attempt's marks
+                    DTS_CUDA(cudaMemsetAsync(orows.p, 0, (n / 32 + 1) * 4, s));
+                    DTS_CUDA(cudaMemsetAsync(ocount.p, 0, 4, s));
+                }
                 oo = OutlierOut{orows.p, olist.p, ocount.p, (unsigned int)olist.n};
             }
             if (th.on)
@@ -1199,6 +1223,14 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
             DTS_CUDA(cudaEventCreateWithFlags(&eb, cudaEventDisableTiming));
             DTS_CUDA(cudaEventRecord(eb, s));
             if (attempt == 0) mark();
+            // 4. sort, enqueued before the host looks at the outlier count
+            //    and the exact bounds (with outliers the keys and their copies
+            //    are sorted again below, from a snapshot of the digit counts)
+            DevBuf<uint32_t> hist0(th.on ? (size_t)plan.npass * OS_HSTRIDE : 0, s);
+            if (th.on)
+                DTS_CUDA(cudaMemcpyAsync(hist0.p, hist.p, (size_t)plan.npass * OS_HSTRIDE * 4,
+                                         cudaMemcpyDeviceToDevice, s));
+            unsigned long long* sorted = radix_sort_keys_hist(keys.p, keys_tmp.p, n, plan, hist.p, s);
             bool drop_outliers = false;
             if (th.on) {
                 // outliers found: their copies join the keys before the sort
@@ -1222,10 +1254,11 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                         drop_outliers = true;
                     } else {
                         DevBuf<unsigned long long> k2(n + ncp, s), k2t(n + ncp, s);
-                        DTS_CUDA(cudaMemcpyAsync(k2.p, keys.p, n * 8, cudaMemcpyDeviceToDevice, s));
+                        // (the keys in any order: the sort's result is unique)
+                        DTS_CUDA(cudaMemcpyAsync(k2.p, sorted, n * 8, cudaMemcpyDeviceToDevice, s));
                         k_outlier_emit<<<grid_for(nout), BT, 0, s>>>(D, olist.p, (uint32_t)nout, g,
                                                                      off.p, k2.p + n, row_bits,
-                                                                     plan, hist.p);
+                                                                     plan, hist0.p);
                         DTS_LAUNCH_CHECK();
                         keys.release();
                         keys_tmp.release();
@@ -1233,12 +1266,12 @@ void build_index_device(dts_index* idx, const dts_segment* D_dev, size_t n,
                         keys_tmp.p = k2t.detach(); keys_tmp.n = n + ncp; keys_tmp.s = s;
                         nt = n + ncp;
                         n_out = nout;
+                        sorted = radix_sort_keys_hist(keys.p, keys_tmp.p, nt, plan, hist0.p, s);
                     }
                 }
             }
-            // 4. sort (enqueued before the host looks at the exact bounds)
             if (!drop_outliers) {
-                sk.a = radix_sort_keys_hist(keys.p, keys_tmp.p, nt, plan, hist.p, s);
+                sk.a = sorted;
                 sk.shift = row_bits;
                 sk.ids = nullptr;
             }
