@@ -46,16 +46,20 @@ int main() {
     for (size_t i = 0; i < n; ++i) perm[i] = (uint32_t)i;
     std::mt19937_64 g(1);
     std::shuffle(perm.begin(), perm.end(), g);
-    // "bucketed" permutation: runs of 8 consecutive targets (a radix pass's scatter)
-    std::vector<uint32_t> bperm(n);
-    {
-        std::vector<uint32_t> runs(n / 8);
+    // permutations made of runs of R consecutive targets in random order
+    auto runs_perm = [&](size_t R) {
+        std::vector<uint32_t> pr(n), runs(n / R);
         for (size_t i = 0; i < runs.size(); ++i) runs[i] = (uint32_t)i;
         std::shuffle(runs.begin(), runs.end(), g);
-        for (size_t i = 0; i < n; ++i) bperm[i] = i / 8 < runs.size() ? runs[i / 8] * 8 + (i % 8) : (uint32_t)i;
-    }
-    R4 *D, *out; uint32_t *dp, *dbp, *pos; uint4* fl;
+        for (size_t i = 0; i < n; ++i) pr[i] = i / R < runs.size() ? runs[i / R] * R + (i % R) : (uint32_t)i;
+        return pr;
+    };
+    std::vector<uint32_t> bperm = runs_perm(8), p2 = runs_perm(2), p4 = runs_perm(4);
+    R4 *D, *out; uint32_t *dp, *dbp, *pos, *d2, *d4; uint4* fl;
     cudaMalloc(&D, n * 64); cudaMalloc(&out, n * 64); cudaMalloc(&dp, n * 4); cudaMalloc(&dbp, n * 4); cudaMalloc(&pos, n * 4);
+    cudaMalloc(&d2, n * 4); cudaMalloc(&d4, n * 4);
+    cudaMemcpy(d2, p2.data(), n * 4, cudaMemcpyHostToDevice);
+    cudaMemcpy(d4, p4.data(), n * 4, cudaMemcpyHostToDevice);
     const size_t nf = (256u << 20) / 16; cudaMalloc(&fl, nf * 16);
     cudaMemset(D, 1, n * 64);
     cudaMemcpy(dp, perm.data(), n * 4, cudaMemcpyHostToDevice);
@@ -79,6 +83,8 @@ int main() {
     run("scatter 64B random", [&] { k_scatter<<<G, T>>>(D, dp, out, n); }, n * 132.0);
     run("scatter 64B runs of 8", [&] { k_scatter<<<G, T>>>(D, dbp, out, n); }, n * 132.0);
     run("gather 64B runs of 8", [&] { k_gather<<<G, T>>>(D, dbp, out, n); }, n * 132.0);
+    run("gather 64B runs of 4", [&] { k_gather<<<G, T>>>(D, d4, out, n); }, n * 132.0);
+    run("gather 64B runs of 2", [&] { k_gather<<<G, T>>>(D, d2, out, n); }, n * 132.0);
     run("scatter u32 random", [&] { k_scatter_u32<<<G, T>>>(dp, pos, n); }, n * 8.0);
     run("scatter u32 runs of 8", [&] { k_scatter_u32<<<G, T>>>(dbp, pos, n); }, n * 8.0);
     cudaError_t e = cudaDeviceSynchronize();
