@@ -1,5 +1,6 @@
 """Summarise an ncu launch-list CSV (gpu__time_duration per launch): per-kernel
-totals for the last `--steps` steps' worth of launches."""
+totals of the last search call (from its query-key kernel on), or of the
+last `frac` of the launches when the list has no search."""
 import collections
 import csv
 import sys
@@ -17,6 +18,9 @@ for r in rows:
         data.append(dict(zip(hdr, r)))
 agg = collections.OrderedDict()
 start = int(len(data) * (1 - frac))
+qk = [i for i, r in enumerate(data) if "k_qkeys" in r["Kernel Name"]]
+if qk:
+    start = qk[-1]
 for r in data[start:]:
     name = r["Kernel Name"].split("(")[0].replace("(anonymous namespace)::", "")[:48]
     v = float(r["Metric Value"])
