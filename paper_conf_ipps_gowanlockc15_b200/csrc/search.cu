@@ -525,7 +525,22 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         }();
         // (the temporal and subbin methods always sort: their one-run queries
         // are grouped by identical run inside a tile, which needs neighbours)
-        const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID;
+        // ... and output-heavy grid searches sort too: expected candidates
+        // per query (entries per non-empty cell x stencil cells) over
+        // DTS_QSORT_WORK (default 1024): neighbouring queries then share
+        // their rows in L1/L2 (C2 at d = 8, 100 k queries: pass 1 3.72 ->
+        // 3.11 ms sorted; at d = 2, ~40 candidates per query, sorting costs
+        // more than it saves)
+        static const double qsort_work = [] {
+            const char* e = getenv("DTS_QSORT_WORK");
+            return e ? atof(e) : 1024.0;
+        }();
+        double work = idx->n_cells ? (double)idx->n / (double)idx->n_cells : 0.0;
+        for (int a = 0; a < 3; ++a)
+            work *= std::floor(2.0 * (d + idx->gp.half_ext[a]) / idx->gp.w[a]) + 2.0;
+        work *= std::floor(idx->gp.maxdur / idx->gp.b) + 2.0;          // bins a query spans
+        const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID ||
+                            (idx->method == DTS_METHOD_GRID && work >= qsort_work);
         DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q ? nq : 0, s);
         k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p,
                                              (packed && sort_q) ? nullptr : order.p, row_bits,
