@@ -56,7 +56,7 @@ struct Counters {                       // device-side statistics / flags
     unsigned int n_over;                // tiles re-run (spill buffer full)
     unsigned int n_spill;               // tiles whose hits were spilled
     unsigned int n_big;                 // spilled queries longer than a CTA sort
-    unsigned int n_mid, n_large;        // spilled queries for the CTA sorts
+    unsigned int n_cls[3];              // spilled queries for the CTA sorts, by size class
     unsigned int n_skew;                // ... whose ids cluster (radix sort)
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
@@ -843,40 +843,46 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 // ---- spilled records to their query segments of a scratch
                 //      mirror of the output, then each segment sorted by
                 //      entry id into the output
-                DevBuf<dts_result> raw(h.total, s);
+                // keys (entry id << 32 | spill index) placed by query, then
+                // sorted; the records gathered from the spill buffers
+                DevBuf<unsigned long long> rkeys(h.total, s);
                 const unsigned long long n1 = std::min(std::min(h.c.spilled, spill_cap),
                                                        h.c.spill_valid);
+                if (n1 + n_raw >= (1ull << 32))
+                    throw Error(DTS_ENOTSUP, "more than 2^32 spilled results in one search call");
+                const SpillSrc src{spill.p, n1, spill2.p};
                 if (n1) {
                     k_spill_place<<<blocks(n1, 256), 256, 0, s>>>(
-                        spill.p, n1, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p, raw.p);
+                        spill.p, n1, 0u, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p,
+                        rkeys.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (n_raw) {
                     k_spill_place<<<blocks(n_raw, 256), 256, 0, s>>>(
-                        spill2.p, n_raw, nullptr, offsets.p, cursor.p, raw.p);
+                        spill2.p, n_raw, (uint32_t)n1, nullptr, offsets.p, cursor.p, rkeys.p);
                     DTS_LAUNCH_CHECK();
                 }
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
-                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 4 * sizeof(unsigned int), s));
+                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 5 * sizeof(unsigned int), s));
                 const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * WQ;
-                DevBuf<uint32_t> mid_list(nslots, s), large_list(nslots, s);
+                DevBuf<uint32_t> lists(3 * nslots, s);
                 const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * WQ, 4), 128, 0, s>>>(
                         spill_tiles.p, h.c.n_spill * WQ, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, large_list.p, bigc.p,
+                        offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
                         ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_over * WQ, 4), 128, 0, s>>>(
                         over_tiles.p, h.c.n_over * WQ, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, raw.p, qmap, qid_base, eb, fin, mid_list.p, large_list.p, bigc.p,
+                        offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
                         ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
-                unsigned int nbm[4] = {0, 0, 0, 0};   // n_big, n_mid, n_large, n_skew
+                unsigned int nbm[5] = {0, 0, 0, 0, 0};   // n_big, n_cls[3], n_skew
                 DTS_CUDA(cudaMemcpyAsync(nbm, &ctr.p->n_big, sizeof(nbm),
                                          cudaMemcpyDeviceToHost, s));
                 DTS_CUDA(cudaStreamSynchronize(s));
@@ -887,33 +893,42 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                            cudaFuncSetAttribute(k_seg_bucket<1024, 16, 1>,
                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                 SEG_CAP * 12) == cudaSuccess &&
+                           cudaFuncSetAttribute(k_seg_bucket<512, 16, 2>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_MID2 * 12) == cudaSuccess &&
                            cudaFuncSetAttribute(k_seg_bucket<512, 8, 2>,
                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
                                                 SEG_MID * 12) == cudaSuccess;
                 }();
                 if (!smem_ok) throw Error(DTS_ECUDA, "segment sort: shared memory size refused");
-                DevBuf<uint32_t> skew_list(nbm[1] + nbm[2], s);
+                DevBuf<uint32_t> skew_list(nbm[1] + nbm[2] + nbm[3], s);
                 if (nbm[1]) {
                     k_seg_bucket<512, 8, 2><<<nbm[1], 512, SEG_MID * 12, s>>>(
-                        mid_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, fin,
+                        lists.p, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, fin,
                         skew_list.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (nbm[2]) {
-                    k_seg_bucket<1024, 16, 1><<<nbm[2], 1024, SEG_CAP * 12, s>>>(
-                        large_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, fin,
+                    k_seg_bucket<512, 16, 2><<<nbm[2], 512, SEG_MID2 * 12, s>>>(
+                        lists.p + nslots, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, fin,
                         skew_list.p, ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
+                if (nbm[3]) {
+                    k_seg_bucket<1024, 16, 1><<<nbm[3], 1024, SEG_CAP * 12, s>>>(
+                        lists.p + 2 * nslots, counts.p, offsets.p, rkeys.p, src, qmap, qid_base,
+                        fin, skew_list.p, ctr.p);
+                    DTS_LAUNCH_CHECK();
+                }
                 unsigned int n_skew = 0;
-                if (nbm[1] + nbm[2]) {
+                if (nbm[1] + nbm[2] + nbm[3]) {
                     DTS_CUDA(cudaMemcpyAsync(&n_skew, &ctr.p->n_skew, sizeof(n_skew),
                                              cudaMemcpyDeviceToHost, s));
                     DTS_CUDA(cudaStreamSynchronize(s));
                 }
                 if (n_skew) {
                     k_seg_radix<1024, 16, 1><<<n_skew, 1024, SEG_CAP * 8, s>>>(
-                        skew_list.p, counts.p, offsets.p, raw.p, qmap, qid_base, eb, fin);
+                        skew_list.p, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, eb, fin);
                     DTS_LAUNCH_CHECK();
                 }
                 const unsigned int n_big = nbm[0];
@@ -933,12 +948,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                         throw Error(DTS_ENOTSUP, "long result segments: sort key exceeds 64 bits");
                     DevBuf<unsigned long long> k1(nb, s), k2(nb, s);
                     k_big_keys<<<blocks((size_t)nq * 32, 256), 256, 0, s>>>(
-                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, raw.p, eb, sb, k1.p);
+                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, rkeys.p, eb, sb, k1.p);
                     DTS_LAUNCH_CHECK();
                     const unsigned long long* sk =
                         radix_sort_keys(k1.p, k2.p, nb, sb, sb + eb + qb, s);
                     k_big_place<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, bigoff.p,
-                                                               offsets.p, raw.p, qmap, qid_base,
+                                                               offsets.p, rkeys.p, src, qmap, qid_base,
                                                                fin);
                     DTS_LAUNCH_CHECK();
                 }

@@ -687,33 +687,47 @@ __global__ void __launch_bounds__(128) k_spill_max(const uint32_t* __restrict__ 
 }
 
 // ------------------------------------------- spilled tiles: place + sort
-// Spilled records (query_id = local query id) go to their query's segment
-// [offsets[q], offsets[q] + counts[q]) of `raw` (a scratch mirror of the
-// output), in arrival order: one atomic per (warp, query) group
-// (__match_any_sync), not per record.  Records of queries whose tile was
-// re-run (cover[q] != 0) are stale and skipped.
+// The spilled records: the first spill buffer, then the re-run's (index
+// space [0, na) then [na, na + nb)).
+struct SpillSrc {
+    const dts_result* a;
+    unsigned long long na;
+    const dts_result* b;
+    __device__ __forceinline__ dts_result at(uint32_t i) const { return i < na ? a[i] : b[i - na]; }
+};
+
+// Each live spilled record's key (entry id << 32 | its spill index) goes to
+// its query's segment [offsets[q], offsets[q] + counts[q]) of `rkeys`, in
+// arrival order: one atomic per (warp, query) group (__match_any_sync), not
+// per record.  Records of queries whose tile was re-run (cover[q] != 0) are
+// stale and skipped, and so are records the outlier filter dropped.  (Keys,
+// 8 bytes, instead of the 24-byte records: the sorts read them contiguously
+// and gather each record once, from the spill buffer.)
 __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restrict__ sp,
-                                                    unsigned long long n,
+                                                    unsigned long long n, uint32_t base_idx,
                                                     const uint32_t* __restrict__ cover,
                                                     const unsigned long long* __restrict__ offsets,
                                                     uint32_t* __restrict__ cursor,
-                                                    dts_result* __restrict__ raw) {
+                                                    unsigned long long* __restrict__ rkeys) {
     const unsigned long long k = (unsigned long long)blockIdx.x * 256 + threadIdx.x;
     const int lane = threadIdx.x & 31;
-    dts_result r;
+    uint32_t q = 0xffffffffu, e = 0;
     bool live = k < n;
     if (live) {
-        r = sp[k];
-        if (r.query_id == DROPPED || (cover && cover[r.query_id])) live = false;
+        const uint2 qe = *reinterpret_cast<const uint2*>(sp + k);   // (query_id, entry_id)
+        q = qe.x;
+        e = qe.y;
+        if (q == DROPPED || (cover && cover[q])) live = false;
     }
-    const uint32_t q = live ? r.query_id : 0xffffffffu;
+    if (!live) q = 0xffffffffu;
     const uint32_t grp = __match_any_sync(0xffffffffu, q);
     if (!live) return;
     const int leader = __ffs(grp) - 1;
     uint32_t base = 0;
     if (lane == leader) base = atomicAdd(&cursor[q], (uint32_t)__popc(grp));
     base = __shfl_sync(grp, base, leader);
-    raw[offsets[q] + base + __popc(grp & ((1u << lane) - 1u))] = r;
+    rkeys[offsets[q] + base + __popc(grp & ((1u << lane) - 1u))] =
+        ((unsigned long long)e << 32) | (uint32_t)(base_idx + k);
 }
 
 // Spilled queries' segments of `raw` sorted by entry id into the output,
@@ -729,32 +743,34 @@ __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restric
 // bitonic sorts up to 16,384 records lost to the device-wide radix sort
 // (canonicalisation 44 ms vs 39).
 constexpr int SEGW_CAP = 512;
-constexpr int SEG_MID = 4096;                  // k_seg_radix<8>
-constexpr int SEG_CAP = 16384;                 // k_seg_radix<32>
+constexpr int SEG_MID = 4096;                  // k_seg_bucket<512, 8>: 4 CTAs per SM
+constexpr int SEG_MID2 = 8192;                 // k_seg_bucket<512, 16>: 2 CTAs per SM
+constexpr int SEG_CAP = 16384;                 // k_seg_bucket<1024, 16>: 1 CTA per SM
 
-// A segment's (entry id << 32 | slot) keys into shared memory, and the
-// records gathered in key order into the output: UNR independent loads in
-// flight per thread (a plain loop waits for each load before its store).
+// A segment's (entry id << 32 | spill index) keys into shared memory, and
+// the records gathered in key order into the output: UNR independent loads
+// in flight per thread (a plain loop waits for each load before its store).
 template <int UNR>
-__device__ __forceinline__ void seg_keys_load(unsigned long long* key, const dts_result* seg,
-                                              uint32_t c, uint32_t t, uint32_t nt) {
+__device__ __forceinline__ void seg_keys_load(unsigned long long* key,
+                                              const unsigned long long* rk, uint32_t c,
+                                              uint32_t t, uint32_t nt) {
     for (uint32_t b = t; b < c; b += nt * UNR) {
-        uint32_t e[UNR];
+        unsigned long long e[UNR];
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
             const uint32_t i = b + (uint32_t)j * nt;
-            e[j] = i < c ? seg[i].entry_id : 0u;
+            e[j] = i < c ? rk[i] : 0ull;
         }
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
             const uint32_t i = b + (uint32_t)j * nt;
-            if (i < c) key[i] = ((unsigned long long)e[j] << 32) | i;
+            if (i < c) key[i] = e[j];
         }
     }
 }
 
 template <int UNR>
-__device__ __forceinline__ void seg_gather(const unsigned long long* key, const dts_result* seg,
+__device__ __forceinline__ void seg_gather(const unsigned long long* key, const SpillSrc& src,
                                            uint32_t c, uint32_t qrep, dts_result* out, uint32_t t,
                                            uint32_t nt) {
     for (uint32_t b = t; b < c; b += nt * UNR) {
@@ -762,7 +778,7 @@ __device__ __forceinline__ void seg_gather(const unsigned long long* key, const 
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
             const uint32_t i = b + (uint32_t)j * nt;
-            if (i < c) r[j] = seg[(uint32_t)(key[i] & 0xffffffffull)];
+            if (i < c) r[j] = src.at((uint32_t)(key[i] & 0xffffffffull));
         }
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
@@ -786,12 +802,13 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
                                                       uint32_t nq,
                                                       const uint32_t* __restrict__ counts,
                                                       const unsigned long long* __restrict__ offsets,
-                                                      const dts_result* __restrict__ raw,
+                                                      const unsigned long long* __restrict__ rkeys,
+                                                      const SpillSrc src,
                                                       const uint32_t* __restrict__ qmap,
                                                       uint32_t qid_base, int eb,
                                                       dts_result* __restrict__ out,
-                                                      uint32_t* __restrict__ mid_list,
-                                                      uint32_t* __restrict__ large_list,
+                                                      uint32_t* __restrict__ lists,   // 3 x lstride
+                                                      size_t lstride,
                                                       uint32_t* __restrict__ bigc,
                                                       Counters* __restrict__ ctr) {
     __shared__ SegWarpSmem SWS[4];
@@ -805,10 +822,9 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     if (c == 0) return;
     if (c > (uint32_t)SEGW_CAP) {
         if (lane == 0) {
-            if (c <= (uint32_t)SEG_MID) {
-                mid_list[atomicAdd(&ctr->n_mid, 1u)] = q;
-            } else if (c <= (uint32_t)SEG_CAP) {
-                large_list[atomicAdd(&ctr->n_large, 1u)] = q;
+            if (c <= (uint32_t)SEG_CAP) {
+                const int k = c <= (uint32_t)SEG_MID ? 0 : (c <= (uint32_t)SEG_MID2 ? 1 : 2);
+                lists[(size_t)k * lstride + atomicAdd(&ctr->n_cls[k], 1u)] = q;
             } else {
                 bigc[q] = c;
                 atomicAdd(&ctr->n_big, 1u);
@@ -818,8 +834,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     }
     SegWarpSmem& S = SWS[warp];
     const unsigned long long off = offsets[q];
-    const dts_result* seg = raw + off;
-    seg_keys_load<8>(S.buf[0], seg, c, lane, 32);
+    seg_keys_load<8>(S.buf[0], rkeys + off, c, lane, 32);
     const uint32_t lt = (1u << lane) - 1u;
     int cur = 0;
     for (int sh = 32; sh < 32 + eb; sh += 8, cur ^= 1) {
@@ -870,7 +885,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     }
     __syncwarp();
     const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
-    seg_gather<4>(S.buf[cur], seg, c, qrep, out + off, lane, 32);
+    seg_gather<4>(S.buf[cur], src, c, qrep, out + off, lane, 32);
 }
 
 // One CTA of SEGC_T threads per listed query (SEGW_CAP < count <= SEGC_T *
@@ -885,7 +900,8 @@ template <int SEGC_T, int ITEMS, int MINB>
 __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __restrict__ list,
                                                         const uint32_t* __restrict__ counts,
                                                         const unsigned long long* __restrict__ offsets,
-                                                        const dts_result* __restrict__ raw,
+                                                        const unsigned long long* __restrict__ rkeys,
+                                                      const SpillSrc src,
                                                         const uint32_t* __restrict__ qmap,
                                                         uint32_t qid_base, int eb,
                                                         dts_result* __restrict__ out) {
@@ -896,9 +912,8 @@ __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __re
     const uint32_t q = list[blockIdx.x];
     const uint32_t c = counts[q];
     const unsigned long long off = offsets[q];
-    const dts_result* seg = raw + off;
     const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
-    seg_keys_load<8>(sbuf, seg, c, t, SEGC_T);
+    seg_keys_load<8>(sbuf, rkeys + off, c, t, SEGC_T);
     const uint32_t lt = (1u << lane) - 1u;
     const uint32_t wbase = warp * 32u * ITEMS;
     for (int sh = 32; sh < 32 + eb; sh += 8) {
@@ -961,7 +976,7 @@ __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __re
         __syncthreads();
     }
     const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
-    seg_gather<4>(sbuf, seg, c, qrep, out + off, t, SEGC_T);
+    seg_gather<4>(sbuf, src, c, qrep, out + off, t, SEGC_T);
 }
 
 // One CTA of T threads per listed query (SEGW_CAP < count <= CAP): a
@@ -978,7 +993,8 @@ template <int T, int ITEMS, int MINB>
 __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restrict__ list,
                                                        const uint32_t* __restrict__ counts,
                                                        const unsigned long long* __restrict__ offsets,
-                                                       const dts_result* __restrict__ raw,
+                                                       const unsigned long long* __restrict__ rkeys,
+                                                      const SpillSrc src,
                                                        const uint32_t* __restrict__ qmap,
                                                        uint32_t qid_base,
                                                        dts_result* __restrict__ out,
@@ -991,20 +1007,22 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
     const uint32_t q = list[blockIdx.x];
     const uint32_t c = counts[q];
     const unsigned long long off = offsets[q];
-    const dts_result* seg = raw + off;
+    const unsigned long long* rk = rkeys + off;
     const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
     if (t == 0) { s_min = ~0u; s_max = 0u; s_bmax = 0u; }
-    // ---- the segment's ids, held in registers (slot t + j*T), and their range
-    uint32_t e[ITEMS];
+    // ---- the segment's keys (entry id << 32 | spill index), held in
+    //      registers (slot t + j*T), and the range of their ids
+    unsigned long long kk[ITEMS];
     uint32_t mn = ~0u, mx = 0u;
 #pragma unroll
     for (int j = 0; j < ITEMS; ++j) {
         const uint32_t i = t + (uint32_t)j * T;
-        e[j] = i < c ? seg[i].entry_id : 0u;
+        kk[j] = i < c ? rk[i] : 0ull;
     }
 #pragma unroll
     for (int j = 0; j < ITEMS; ++j) {
-        if (t + (uint32_t)j * T < c) { mn = min(mn, e[j]); mx = max(mx, e[j]); }
+        const uint32_t e = (uint32_t)(kk[j] >> 32);
+        if (t + (uint32_t)j * T < c) { mn = min(mn, e); mx = max(mx, e); }
     }
     mn = __reduce_min_sync(0xffffffffu, mn);
     mx = __reduce_max_sync(0xffffffffu, mx);
@@ -1022,7 +1040,7 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
     // ---- bucket counts
 #pragma unroll
     for (int j = 0; j < ITEMS; ++j)
-        if (t + (uint32_t)j * T < c) atomicAdd(&cnt[(e[j] - mn) >> sh], 1u);
+        if (t + (uint32_t)j * T < c) atomicAdd(&cnt[((uint32_t)(kk[j] >> 32) - mn) >> sh], 1u);
     __syncthreads();
     // ---- exclusive scan of the counters (nb / T per thread, consecutive)
     const uint32_t per = (nb + T - 1) / T, b0 = t * per;
@@ -1054,7 +1072,7 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
 #pragma unroll
     for (int j = 0; j < ITEMS; ++j) {
         const uint32_t i = t + (uint32_t)j * T;
-        if (i < c) bbuf[atomicAdd(&cnt[(e[j] - mn) >> sh], 1u)] = ((unsigned long long)e[j] << 32) | i;
+        if (i < c) bbuf[atomicAdd(&cnt[((uint32_t)(kk[j] >> 32) - mn) >> sh], 1u)] = kk[j];
     }
     __syncthreads();
     // ---- each bucket sorted by one thread (insertion sort, <= SEGB_MAX keys)
@@ -1069,7 +1087,7 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
     }
     __syncthreads();
     const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
-    seg_gather<4>(bbuf, seg, c, qrep, out + off, t, T);
+    seg_gather<4>(bbuf, src, c, qrep, out + off, t, T);
 }
 
 // Segments longer than SEG_CAP: one device-wide keys-only radix sort of
@@ -1078,7 +1096,8 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
 __global__ void __launch_bounds__(256) k_big_keys(uint32_t nq, const uint32_t* __restrict__ bigc,
                                                  const unsigned long long* __restrict__ bigoff,
                                                  const unsigned long long* __restrict__ offsets,
-                                                 const dts_result* __restrict__ out, int eb, int sb,
+                                                 const unsigned long long* __restrict__ rkeys,
+                                                 int eb, int sb,
                                                  unsigned long long* __restrict__ keys) {
     const uint32_t warp = (blockIdx.x * 256 + threadIdx.x) >> 5, lane = threadIdx.x & 31;
     if (warp >= nq) return;
@@ -1087,16 +1106,17 @@ __global__ void __launch_bounds__(256) k_big_keys(uint32_t nq, const uint32_t* _
     const unsigned long long o = offsets[warp], b = bigoff[warp];
     const unsigned long long qk = (unsigned long long)warp << (eb + sb);
     for (uint32_t i = lane; i < c; i += 32)
-        keys[b + i] = qk | ((unsigned long long)out[o + i].entry_id << sb) | i;
+        keys[b + i] = qk | ((rkeys[o + i] >> 32) << sb) | i;
 }
 
-// out[k-th place of its segment] = raw[slot] of sorted element k, with the
-// reported query id
+// out[k-th place of its segment] = the spilled record of its segment's key
+// at the slot of sorted element k, with the reported query id
 __global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __restrict__ keys,
                                                   unsigned long long n, int eb, int sb,
                                                   const unsigned long long* __restrict__ bigoff,
                                                   const unsigned long long* __restrict__ offsets,
-                                                  const dts_result* __restrict__ raw,
+                                                  const unsigned long long* __restrict__ rkeys,
+                                                  const SpillSrc src,
                                                   const uint32_t* __restrict__ qmap,
                                                   uint32_t qid_base,
                                                   dts_result* __restrict__ out) {
@@ -1105,7 +1125,7 @@ __global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __r
     const unsigned long long key = keys[k];
     const uint32_t q = (uint32_t)(key >> (eb + sb));
     const unsigned long long slot = key & ((1ull << sb) - 1ull);
-    dts_result r = raw[offsets[q] + slot];
+    dts_result r = src.at((uint32_t)(rkeys[offsets[q] + slot] & 0xffffffffull));
     r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
     out[offsets[q] + (k - bigoff[q])] = r;
 }
