@@ -712,3 +712,24 @@ def test_density_cap_invariant(dts, oracle_mod):
     got = np.frombuffer(outs[0], dtype=dts.RESULT_DTYPE)
     parity.compare(got, oracle_mod.search(c.D, c.Q, c.d, threads=THREADS), c.D, c.Q, c.d,
                    oracle_mod)
+
+
+def test_segment_sort_class_boundaries(dts, oracle_mod):
+    """Spilled queries with exactly 512 / 513 / 4096 / 4097 / 8192 / 8193 /
+    16384 / 16385 results: each side of every segment-sort size boundary
+    (warp radix, three bucket-sort CTA sizes, device-wide radix)."""
+    g = synth.rng(91)
+    sizes = (512, 513, 4096, 4097, 8192, 8193, 16384, 16385)
+    parts = []
+    for k, m in enumerate(sizes):
+        P = np.zeros((m, 8))
+        P[:, 4] = 1.0
+        P[:, 1:4] = 2.0 * k + g.uniform(0, 0.01, size=(m, 3))
+        P[:, 5:8] = P[:, 1:4] + g.uniform(-0.001, 0.001, size=(m, 3))
+        parts.append(P)
+    D = np.concatenate(parts)
+    D = D[g.permutation(D.shape[0])]
+    Q = np.array([[0.0, 2.0 * k + 0.005, 2.0 * k + 0.005, 2.0 * k + 0.005, 1.0,
+                   2.0 * k + 0.005, 2.0 * k + 0.005, 2.0 * k + 0.005] for k in range(len(sizes))])
+    got, info = run_and_compare(dts, oracle_mod, D, Q, 0.05)
+    assert np.array_equal(np.bincount(got["query_id"], minlength=len(sizes)), sizes)
