@@ -347,10 +347,13 @@ PassPlan plan_passes(int lo, int hi, bool allow9);
 bool radix_onesweep(size_t n);
 // Keys-only onesweep sort by the plan, with the per-pass digit counts
 // already accumulated in hist (npass x 512, e.g. by the kernel that wrote the
-// keys).  Returns the buffer (keys or tmp) holding the sorted keys.
+// keys).  Returns the buffer (keys or tmp) holding the sorted keys; with
+// rows_out the last pass writes only (key & row_mask) of each sorted key
+// there (a packed (key, row) sort that only needs the order) and returns NULL.
 unsigned long long* radix_sort_keys_hist(unsigned long long* keys, unsigned long long* tmp,
                                          size_t n, const PassPlan& plan, uint32_t* hist,
-                                         cudaStream_t s);
+                                         cudaStream_t s, uint32_t* rows_out = nullptr,
+                                         unsigned long long row_mask = 0);
 
 // Device block cache (alloc.cu) for memory that outlives one API call.
 void* cache_alloc(size_t bytes);

@@ -338,7 +338,7 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
     const unsigned long long* __restrict__ keys, const uint32_t* __restrict__ vals, size_t n,
     int shift, const uint32_t* __restrict__ gbase, uint32_t* status, uint32_t* tile_ctr,
     unsigned long long* __restrict__ keys_out, uint32_t* __restrict__ vals_out,
-    uint32_t sleep_ns) {
+    uint32_t sleep_ns, uint32_t* __restrict__ rows_out, unsigned long long row_mask) {
     constexpr int RADIX = 1 << RB;
     constexpr int TILE = RS_THREADS * ITEMS;
     constexpr int DPT = RADIX / RS_THREADS;          // digits per thread
@@ -493,7 +493,8 @@ __global__ void __launch_bounds__(RS_THREADS, MINB) k_onesweep(
         const unsigned long long key = sk[i];
         const uint32_t dg = (uint32_t)(key >> shift) & DMASK;
         const uint32_t dst = tile_base[dg] + (i - local_off[dg]);
-        keys_out[dst] = key;
+        if (rows_out) rows_out[dst] = (uint32_t)(key & row_mask);   // last pass: rows only
+        else keys_out[dst] = key;
         if (VALS) vals_out[dst] = sv[i];
     }
 }
@@ -539,10 +540,11 @@ template <bool VALS, int MINB, int RB, int ITEMS = OS_ITEMS>
 void launch_onesweep(uint32_t ntiles, cudaStream_t s, const unsigned long long* kin,
                      const uint32_t* vin, size_t n, int shift, const uint32_t* gbase,
                      uint32_t* status, uint32_t* ctr, unsigned long long* kout, uint32_t* vout,
-                     uint32_t sleep_ns) {
+                     uint32_t sleep_ns, uint32_t* rows_out = nullptr,
+                     unsigned long long row_mask = 0) {
     k_onesweep<VALS, MINB, RB, ITEMS><<<ntiles, RS_THREADS, 0, s>>>(kin, vin, n, shift, gbase,
                                                                     status, ctr, kout, vout,
-                                                                    sleep_ns);
+                                                                    sleep_ns, rows_out, row_mask);
 }
 
 // Keys-only tile shapes (DTS_OS_SHAPE, A/B): 0 = 12 keys per thread for
@@ -565,7 +567,8 @@ int os_items(int bits, bool vals) {
 // (k_rs_hist_scan).  On return *kin / *vin hold the result.
 void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32_t** vin,
                      uint32_t** vout, size_t n, const PassPlan& plan, const uint32_t* hist,
-                     cudaStream_t s) {
+                     cudaStream_t s, uint32_t* rows_out = nullptr,
+                     unsigned long long row_mask = 0) {
     uint32_t maxtiles = 0;
     for (int p = 0; p < plan.npass; ++p) {
         const uint32_t tile = RS_THREADS * os_items(plan.bits[p], *vin != nullptr);
@@ -587,22 +590,23 @@ void onesweep_passes(unsigned long long** kin, unsigned long long** kout, uint32
         uint32_t* ctr = status.p + used;
         const uint32_t* gb = hist + OS_HSTRIDE * p;
         const int sh = plan.shift[p];
+        uint32_t* ro = (p == plan.npass - 1 && !*vin) ? rows_out : nullptr;
         if (plan.bits[p] == 9) {
             if (shape) launch_onesweep<false, 3, 9, 13>(ntiles, s, *kin, nullptr, n, sh, gb,
-                                                        status.p, ctr, *kout, nullptr, sleep_ns);
+                                                        status.p, ctr, *kout, nullptr, sleep_ns, ro, row_mask);
             else launch_onesweep<false, 3, 9>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
-                                              *kout, nullptr, sleep_ns);
+                                              *kout, nullptr, sleep_ns, ro, row_mask);
         } else {
             if (*vin) launch_onesweep<true, 2, 8>(ntiles, s, *kin, *vin, n, sh, gb, status.p, ctr,
                                                   *kout, *vout, sleep_ns);
             else if (shape == 1)
                 launch_onesweep<false, 3, 8, 16>(ntiles, s, *kin, nullptr, n, sh, gb, status.p,
-                                                 ctr, *kout, nullptr, sleep_ns);
+                                                 ctr, *kout, nullptr, sleep_ns, ro, row_mask);
             else if (shape == 2)
                 launch_onesweep<false, 4, 8, 16>(ntiles, s, *kin, nullptr, n, sh, gb, status.p,
-                                                 ctr, *kout, nullptr, sleep_ns);
+                                                 ctr, *kout, nullptr, sleep_ns, ro, row_mask);
             else launch_onesweep<false, 4, 8>(ntiles, s, *kin, nullptr, n, sh, gb, status.p, ctr,
-                                              *kout, nullptr, sleep_ns);
+                                              *kout, nullptr, sleep_ns, ro, row_mask);
         }
         DTS_LAUNCH_CHECK();
         std::swap(*kin, *kout);
@@ -630,13 +634,14 @@ void radix_pass(const unsigned long long* kin, const uint32_t* vin, unsigned lon
 
 unsigned long long* radix_sort_keys_hist(unsigned long long* keys, unsigned long long* tmp,
                                          size_t n, const PassPlan& plan, uint32_t* hist,
-                                         cudaStream_t s) {
+                                         cudaStream_t s, uint32_t* rows_out,
+                                         unsigned long long row_mask) {
     k_rs_hist_scan<<<plan.npass, RS_THREADS, 0, s>>>(hist);
     DTS_LAUNCH_CHECK();
     unsigned long long *kin = keys, *kout = tmp;
     uint32_t *vin = nullptr, *vout = nullptr;
-    onesweep_passes(&kin, &kout, &vin, &vout, n, plan, hist, s);
-    return kin;
+    onesweep_passes(&kin, &kout, &vin, &vout, n, plan, hist, s, rows_out, row_mask);
+    return rows_out ? nullptr : kin;
 }
 
 bool radix_onesweep(size_t n) { return onesweep_enabled(n); }

@@ -346,36 +346,59 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
 }
 
 // --------------------------------------------------------------- query prep
+// Query keys (grid-stride), validation, and -- for the packed keys-only sort
+// -- the digit counts of every pass of its plan (hist != NULL; one pass over
+// the keys fewer than a separate histogram kernel).
 __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uint32_t nq,
                                              GridParams g, unsigned long long* __restrict__ keys,
                                              uint32_t* __restrict__ ids, int shift,
-                                             Counters* __restrict__ ctr) {
-    uint32_t i = blockIdx.x * PT + threadIdx.x;
-    if (i >= nq) return;
-    const double4 s0 = Q[2 * (size_t)i], s1 = Q[2 * (size_t)i + 1];
-    const double c[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
-    unsigned bad = 0;
+                                             Counters* __restrict__ ctr, const PassPlan plan,
+                                             uint32_t* __restrict__ hist) {
+    __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
+    if (hist) {
+        for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += PT) h[j] = 0;
+        __syncthreads();
+    }
+    unsigned bad_all = 0;
+    for (uint32_t i = blockIdx.x * PT + threadIdx.x; i < nq; i += gridDim.x * PT) {
+        const double4 s0 = Q[2 * (size_t)i], s1 = Q[2 * (size_t)i + 1];
+        const double c[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
+        unsigned bad = 0;
 #pragma unroll
-    for (int k = 0; k < 8; ++k) if (!isfinite(c[k])) bad |= 1;
-    if (!bad && s1.x < s0.x) bad |= 2;
-    if (!bad) {
-        const double dur = s1.x - s0.x;
+        for (int k = 0; k < 8; ++k) if (!isfinite(c[k])) bad |= 1;
+        if (!bad && s1.x < s0.x) bad |= 2;
+        if (!bad) {
+            const double dur = s1.x - s0.x;
 #pragma unroll
-        for (int a = 1; a < 4; ++a) {
-            double e = fabs(c[4 + a] - c[a]);
-            if (!isfinite(e) || (dur > 0.0 && !isfinite(e / dur))) bad |= 4;
+            for (int a = 1; a < 4; ++a) {
+                double e = fabs(c[4 + a] - c[a]);
+                if (!isfinite(e) || (dur > 0.0 && !isfinite(e / dur))) bad |= 4;
+            }
+        }
+        bad_all |= bad;
+        unsigned long long key = 0;
+        if (!bad)
+            key = make_key(g, bin_of(g, s0.x), cell_of(g, 0, 0.5 * (s0.y + s1.y)),
+                           cell_of(g, 1, 0.5 * (s0.z + s1.z)), cell_of(g, 2, 0.5 * (s0.w + s1.w)));
+        if (ids) {
+            keys[i] = key;
+            ids[i] = i;
+        } else {                        // packed: (key, row) in one word, keys-only sort
+            const unsigned long long v = (key << shift) | i;
+            keys[i] = v;
+            if (hist) {
+#pragma unroll
+                for (int p = 0; p < OS_MAXPASS; ++p)
+                    if (p < plan.npass)
+                        atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
+            }
         }
     }
-    if (bad) atomicOr(&ctr->bad, bad);
-    unsigned long long key = 0;
-    if (!bad)
-        key = make_key(g, bin_of(g, s0.x), cell_of(g, 0, 0.5 * (s0.y + s1.y)),
-                       cell_of(g, 1, 0.5 * (s0.z + s1.z)), cell_of(g, 2, 0.5 * (s0.w + s1.w)));
-    if (ids) {
-        keys[i] = key;
-        ids[i] = i;
-    } else {                        // packed: (key, row) in one word, keys-only sort
-        keys[i] = (key << shift) | i;
+    if (bad_all) atomicOr(&ctr->bad, bad_all);
+    if (hist) {
+        __syncthreads();
+        for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += PT)
+            if (h[j]) atomicAdd(hist + j, h[j]);
     }
 }
 
@@ -507,6 +530,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 
     EventTimer tm(local.time_kernels != 0, s);
     tm.mark();
+    static const int nsm_prep = [] {
+        int dev = 0, v = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+        return v;
+    }();
     // ---- query prep: key + sort
     DevBuf<uint32_t> order(nq, s);
     {
@@ -542,24 +571,34 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID ||
                             (idx->method == DTS_METHOD_GRID && work >= qsort_work);
         DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q ? nq : 0, s);
-        k_qkeys<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, idx->gp, qk.p,
-                                             (packed && sort_q) ? nullptr : order.p, row_bits,
-                                             ctr.p);
+        static const int drop = [] {           // DTS_QSORT_DROP: low key bits left unsorted
+            const char* e = getenv("DTS_QSORT_DROP");
+            return e ? std::max(0, std::min(24, atoi(e))) : -1;
+        }();
+        // the order only serves locality: by default only the key's top 16
+        // bits (bin and the slowest cell axis) are sorted, two radix passes
+        // (C4, 34-bit keys: all but key_bits % 8 = 2 bits, four passes: prep
+        // 0.122 ms, pass 1 0.618; top 24 bits: 0.104, 0.616; top 16: 0.084,
+        // 0.617).  The packed sort's digit counts come from k_qkeys and its
+        // last pass writes the order itself.
+        const int dr = drop >= 0 ? drop : std::max(0, idx->key_bits - 16);
+        const int lo = row_bits + std::min(dr, std::max(0, idx->key_bits - 8));
+        const bool fused = sort_q && packed && radix_onesweep(nq) && nq > 1 &&
+                           row_bits + idx->key_bits > lo;
+        const PassPlan plan = fused ? plan_passes(lo, row_bits + idx->key_bits, true) : PassPlan{};
+        DevBuf<uint32_t> hist(fused ? (size_t)plan.npass * OS_HSTRIDE : 0, s);
+        if (fused)
+            DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)plan.npass * OS_HSTRIDE * 4, s));
+        k_qkeys<<<(unsigned)std::min<size_t>(blocks(nq, PT), (size_t)nsm_prep * 8), PT, 0, s>>>(
+            Q, (uint32_t)nq, idx->gp, qk.p, (packed && sort_q) ? nullptr : order.p, row_bits,
+            ctr.p, plan, fused ? hist.p : nullptr);
         DTS_LAUNCH_CHECK();
         if (!sort_q) {
             // order = identity (written by k_qkeys)
+        } else if (fused) {
+            radix_sort_keys_hist(qk.p, qk_tmp.p, nq, plan, hist.p, s, order.p,
+                                 (1ull << row_bits) - 1ull);
         } else if (packed) {
-            static const int drop = [] {       // DTS_QSORT_DROP: low key bits left unsorted
-                const char* e = getenv("DTS_QSORT_DROP");
-                return e ? std::max(0, std::min(24, atoi(e))) : -1;
-            }();
-            // the order only serves locality: by default only the key's top
-            // 16 bits (bin and the slowest cell axis) are sorted, two radix
-            // passes (C4, 34-bit keys: all but key_bits % 8 = 2 bits, four
-            // passes: prep 0.122 ms, pass 1 0.618; top 24 bits: 0.104,
-            // 0.616; top 16: 0.084, 0.617)
-            const int dr = drop >= 0 ? drop : std::max(0, idx->key_bits - 16);
-            const int lo = row_bits + std::min(dr, std::max(0, idx->key_bits - 8));
             const unsigned long long* sorted =
                 radix_sort_keys(qk.p, qk_tmp.p, nq, lo, row_bits + idx->key_bits, s);
             k_unpack_order<<<blocks(nq, PT), PT, 0, s>>>(sorted, (uint32_t)nq,
