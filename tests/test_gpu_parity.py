@@ -733,3 +733,13 @@ def test_segment_sort_class_boundaries(dts, oracle_mod):
                    2.0 * k + 0.005, 2.0 * k + 0.005, 2.0 * k + 0.005] for k in range(len(sizes))])
     got, info = run_and_compare(dts, oracle_mod, D, Q, 0.05)
     assert np.array_equal(np.bincount(got["query_id"], minlength=len(sizes)), sizes)
+
+
+@pytest.mark.parametrize("nq", [4096, 8192, 8193, 12287])
+def test_query_counts_at_scan_tile_edges(dts, oracle_mod, nq):
+    """Query sets of whole and partial single-pass scan tiles (4,096 counts):
+    exact offsets and the total at the tile edges (C0, queries repeated)."""
+    c = synth.make_config("C0")
+    Q = np.ascontiguousarray(np.resize(c.Q, (nq, 8)))
+    got, info = run_and_compare(dts, oracle_mod, c.D, Q, 0.2)
+    assert info["common"] > 0
