@@ -121,96 +121,10 @@ void scan_exclusive(const Tin* in, Tout* out, size_t n, cudaStream_t s) {
 void scan_exclusive_u32_to_u32(const uint32_t* in, uint32_t* out, size_t n, cudaStream_t s) {
     scan_exclusive<uint32_t, uint32_t>(in, out, n, s);
 }
-// Single-pass exclusive scan (u32 -> u64, out[n] = total) by decoupled
-// look-back: tiles of LB_TILE values take ids in launch order, publish their
-// aggregate, then their inclusive prefix once the predecessors' are known
-// (status word: 2 flag bits | 62-bit value).  One launch instead of the
-// reduce / scan / downsweep chain (C4's 1 M per-query counts: 3 launches and
-// two pool allocations, 21 us, before).
-namespace {
-constexpr int LB_ITEMS = 16;
-constexpr int LB_TILE = SCAN_THREADS * LB_ITEMS;               // 4096
-constexpr unsigned long long LB_AGG = 1ull << 62, LB_PRE = 2ull << 62;
-constexpr unsigned long long LB_VAL = LB_AGG - 1ull;
-
-__device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long* p) {
-    unsigned long long v;
-    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_relaxed64(unsigned long long* p, unsigned long long v) {
-    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
-}
-
-__global__ void __launch_bounds__(SCAN_THREADS) k_scan_lookback(const uint32_t* __restrict__ in,
-                                                               size_t n,
-                                                               unsigned long long* status,
-                                                               unsigned int* tile_ctr,
-                                                               unsigned long long* __restrict__ out) {
-    __shared__ unsigned int s_tile;
-    __shared__ unsigned long long s_prefix;
-    if (threadIdx.x == 0) s_tile = atomicAdd(tile_ctr, 1u);
-    __syncthreads();
-    const unsigned int tile = s_tile;
-    const size_t base = (size_t)tile * LB_TILE + (size_t)threadIdx.x * LB_ITEMS;
-    uint32_t v[LB_ITEMS];
-    unsigned long long sum = 0;
-#pragma unroll
-    for (int i = 0; i < LB_ITEMS; ++i) {
-        const size_t idx = base + i;
-        v[i] = idx < n ? in[idx] : 0u;
-        sum += v[i];
-    }
-    unsigned long long total;
-    unsigned long long run = block_exclusive_scan<unsigned long long>(sum, &total);
-    if (threadIdx.x == 0) {
-        unsigned long long excl = 0;
-        if (tile == 0) {
-            st_relaxed64(status + tile, LB_PRE | total);
-        } else {
-            st_relaxed64(status + tile, LB_AGG | total);
-            int j = (int)tile - 1;
-            while (true) {
-                const unsigned long long w = ld_relaxed64(status + j);
-                if (w == 0ull) continue;                   // not published yet
-                excl += w & LB_VAL;
-                if (w & LB_PRE) break;
-                --j;
-            }
-            st_relaxed64(status + tile, LB_PRE | (excl + total));
-        }
-        s_prefix = excl;
-    }
-    __syncthreads();
-    run += s_prefix;
-#pragma unroll
-    for (int i = 0; i < LB_ITEMS; ++i) {
-        const size_t idx = base + i;
-        if (idx < n) out[idx] = run;
-        run += v[i];
-    }
-    if (base <= n - 1 && n - 1 < base + LB_ITEMS) out[n] = run;   // the thread of the last value
-}
-}  // namespace
-
 void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size_t n,
                                cudaStream_t s) {
-    static const bool lookback = [] {            // DTS_SCAN_LOOKBACK=0: reduce/scan/down
-        const char* e = getenv("DTS_SCAN_LOOKBACK");
-        return !(e && e[0] == '0');
-    }();
-    if (!lookback || n <= (size_t)SCAN_TILE) {
-        scan_exclusive<uint32_t, unsigned long long>(in, out, n, s);
-        return;
-    }
-    const size_t nt = (n + LB_TILE - 1) / LB_TILE;
-    DevBuf<unsigned long long> status(nt + 1, s);
-    DTS_CUDA(cudaMemsetAsync(status.p, 0, (nt + 1) * sizeof(unsigned long long), s));
-    k_scan_lookback<<<(unsigned)nt, SCAN_THREADS, 0, s>>>(
-        in, n, status.p, reinterpret_cast<unsigned int*>(status.p + nt), out);
-    DTS_LAUNCH_CHECK();
+    scan_exclusive<uint32_t, unsigned long long>(in, out, n, s);
 }
-
 // ============================================================== radix sort
 namespace {
 constexpr int RS_THREADS = 256;

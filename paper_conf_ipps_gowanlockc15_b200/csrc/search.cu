@@ -776,6 +776,33 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
     tm.mark();
 
+    // pass 2 launched before the host learns the total, into a buffer sized
+    // by this index's previous result count: a repeated search of one index
+    // then has no host round trip between the scan and the copy (a buffer
+    // that turns out too small is freed and pass 2 launched again)
+    struct SpecOut {
+        dts_result* p = nullptr;
+        cudaStream_t s = nullptr;
+        ~SpecOut() {
+            if (p) {
+                cudaStreamSynchronize(s);
+                cache_free(p);
+            }
+        }
+    } spec;
+    spec.s = s;
+    const unsigned long long hint = count_only ? 0ull : idx->result_hint.load();
+    static const bool spec_on = [] {          // DTS_SPEC_EMIT=0: off
+        const char* e = getenv("DTS_SPEC_EMIT");
+        return !(e && e[0] == '0');
+    }();
+    if (spec_on && hint > 0) {
+        spec.p = static_cast<dts_result*>(cache_alloc(hint * sizeof(dts_result)));
+        k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
+                                                         offsets.p, tile_base.p, stage.p, spec.p,
+                                                         hint);
+        DTS_LAUNCH_CHECK();
+    }
     struct {
         Counters c;
         unsigned long long total;
@@ -784,6 +811,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     DTS_CUDA(cudaMemcpyAsync(&h.total, offsets.p + nq, sizeof(unsigned long long),
                              cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaStreamSynchronize(s));
+    if (!count_only) idx->result_hint.store(h.total + h.total / 8 + 4096);
     if (h.c.bad & 1) throw Error(DTS_EINVAL, "query segment with a non-finite coordinate or time");
     if (h.c.bad & 2) throw Error(DTS_EINVAL, "query segment with t_end < t_start");
     if (h.c.bad & 4) throw Error(DTS_EINVAL, "query segment whose speed overflows fp64");
@@ -840,13 +868,28 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 
     if (h.total > 0) {
         dts_result* fin = nullptr;
-        fin = static_cast<dts_result*>(cache_alloc(h.total * sizeof(dts_result)));
+        bool emitted = false;
+        if (spec.p && h.total <= hint) {        // the speculative pass 2 holds it all
+            fin = spec.p;
+            spec.p = nullptr;
+            emitted = true;
+        } else {
+            if (spec.p) {
+                DTS_CUDA(cudaStreamSynchronize(s));
+                cache_free(spec.p);
+                spec.p = nullptr;
+            }
+            fin = static_cast<dts_result*>(cache_alloc(h.total * sizeof(dts_result)));
+        }
         try {
             // ---- pass 2: staged tiles are copied to their exact offsets
-            k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
-                                                             offsets.p, tile_base.p, stage.p,
-                                                             fin);
-            DTS_LAUNCH_CHECK();
+            if (!emitted) {
+                k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq,
+                                                                 counts.p, offsets.p,
+                                                                 tile_base.p, stage.p, fin,
+                                                                 h.total);
+                DTS_LAUNCH_CHECK();
+            }
             tm.mark();
             if (h.c.n_spill || h.c.n_over) {
                 DevBuf<uint32_t> cursor(nq, s), cover(h.c.n_over ? nq : 0, s);

@@ -597,13 +597,16 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
 
 // ------------------------------------------------------ pass 2: emission
 // One warp per warp tile: the tile's staged hits are contiguous and grouped
-// by query in canonical order; copy each query's group to its exact offset.
+// by query in canonical order; copy each query's group to its exact offset
+// (positions from cap on are not written: a speculative launch into a
+// buffer that turned out too small is discarded).
 __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ order, uint32_t nq,
                                                   const uint32_t* __restrict__ counts,
                                                   const unsigned long long* __restrict__ offsets,
                                                   const unsigned long long* __restrict__ tile_base,
                                                   const dts_result* __restrict__ stage,
-                                                  dts_result* __restrict__ out) {
+                                                  dts_result* __restrict__ out,
+                                                  unsigned long long cap) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t ntiles = (nq + WQ - 1) / WQ;
     const uint32_t wt = blockIdx.x * WW + warp;
@@ -634,7 +637,7 @@ __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ 
             if (__shfl_sync(0xffffffffu, incl, q + step - 1) <= i) q += step;
         const unsigned long long o = __shfl_sync(0xffffffffu, off, q);
         const uint32_t e = __shfl_sync(0xffffffffu, excl, q);
-        if (i < nh) out[o + (i - e)] = stage[tb + i];
+        if (i < nh && o + (i - e) < cap) out[o + (i - e)] = stage[tb + i];
     }
 }
 

@@ -743,3 +743,23 @@ def test_query_counts_at_scan_tile_edges(dts, oracle_mod, nq):
     Q = np.ascontiguousarray(np.resize(c.Q, (nq, 8)))
     got, info = run_and_compare(dts, oracle_mod, c.D, Q, 0.2)
     assert info["common"] > 0
+
+
+def test_repeated_searches_speculative_pass2(dts, oracle_mod):
+    """Pass 2 of a repeated search of one index is launched before the total
+    is known, into a buffer sized by the previous result count; a larger
+    output falls back to an exact buffer.  Growing and shrinking outputs on
+    one index give the bytes of a fresh index's search."""
+    c = synth.make_config("C1", scale=0.1)
+    idx = dts.build_index(c.D)
+    seq = (0.005, 0.02, 0.02, 0.05, 0.005, 0.05, 0.001)
+    got = [dts.search(idx, c.Q, d).tobytes() for d in seq]
+    idx.free()
+    for d, g in zip(seq, got):
+        fresh = dts.build_index(c.D)
+        assert g == dts.search(fresh, c.Q, d).tobytes(), d
+        fresh.free()
+    r = np.frombuffer(got[3], dtype=dts.RESULT_DTYPE)
+    qs = np.arange(0, c.Q.shape[0], 7)
+    parity.compare(parity.restrict(r, qs), oracle_mod.search_queries(c.D, c.Q, qs, 0.05),
+                   c.D, c.Q, 0.05, oracle_mod)
