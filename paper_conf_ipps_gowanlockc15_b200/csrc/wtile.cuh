@@ -290,6 +290,162 @@ __device__ __forceinline__ void maybe_flush(WarpSmem& S, const TileArgs& a, int 
     if (S.nhit > (uint32_t)WH - step_max) flush_spill<OUT>(S, a, lane);
 }
 
+// One probe round's runs (lane: [start, start + cnt) of query qi, subbin
+// array ind - 1 or sorted positions when 0), flattened and streamed two
+// candidates per lane; hits staged (or spilled).
+template <bool SB, bool EXCL, bool OUT, bool CNT>
+__device__ __forceinline__ void stream_round(WarpSmem& S, const TileArgs& a, int lane,
+                                             uint32_t start, uint32_t cnt, int qi, uint32_t ind,
+                                             double d2, unsigned long long& n_cand,
+                                             const OutlierArgs* s_oa, const GridParams* s_g) {
+    unsigned long long incl = cnt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
+        if (lane >= o) incl += u;
+    }
+    const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
+    const unsigned long long excl = incl - cnt;
+    n_cand += total;
+    // the round's non-empty runs, compacted into shared memory:
+    // (position delta start - excl mod 2^32, query | method index <<
+    // 8); a candidate t lies in run r = (non-empty runs starting at
+    // or before t) - 1, counted with one OR-reduction of the run
+    // starts per 32 candidates -- no per-candidate search
+    const bool ne = cnt > 0;
+    const uint32_t lt = (1u << lane) - 1u;
+    const uint32_t nemask = __ballot_sync(0xffffffffu, ne);
+    if (ne) S.run[__popc(nemask & lt)] = make_uint2(start - (uint32_t)excl,
+                                                    (uint32_t)qi | (ind << 8));
+    __syncwarp();
+    uint32_t before = 0;          // non-empty runs starting before `base`
+    for (unsigned long long base = 0; base < total; base += 64) {
+        // run-start offsets inside the two 32-candidate halves
+        const unsigned long long o1 = excl - base, o2 = o1 - 32;
+        const uint32_t m1 = __reduce_or_sync(0xffffffffu, (ne && excl >= base && o1 < 32)
+                                                              ? 1u << (uint32_t)o1 : 0u);
+        const uint32_t m2 = __reduce_or_sync(
+            0xffffffffu, (ne && excl >= base + 32 && o2 < 32) ? 1u << (uint32_t)o2 : 0u);
+        const uint32_t r1 = min(before + __popc(m1 & (lt | (1u << lane))) - 1u, 31u);
+        before += __popc(m1);
+        const uint32_t r2 = min(before + __popc(m2 & (lt | (1u << lane))) - 1u, 31u);
+        before += __popc(m2);
+        const unsigned long long t1 = base + lane, t2 = t1 + 32;
+        const bool v1 = t1 < total, v2 = t2 < total;
+        if (v1) {
+            const uint2 ru1 = S.run[r1];
+            const uint2 ru2 = v2 ? S.run[r2] : ru1;
+            const int qi1 = (int)(ru1.y & 0xffu), qi2 = (int)(ru2.y & 0xffu);
+            const uint32_t i1 = SB ? ru1.y >> 8 : 0u, i2 = SB ? ru2.y >> 8 : 0u;
+            uint32_t p1 = (uint32_t)t1 + ru1.x;
+            uint32_t p2 = v2 ? (uint32_t)t2 + ru2.x : p1;
+            const uint32_t sl1 = p1, sl2 = p2;      // subbin slots (when i != 0)
+            if (i1) p1 = __ldg(sb_ids(a.sb, i1) + sl1);   // id -> sorted position
+            if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + sl2);
+            else if (!v2) p2 = p1;
+            double2 st1, sx1, sy1, sz1, st2, sx2, sy2, sz2;
+            if (i1) sb_load(a.sb, i1, sl1, st1, sx1, sy1, sz1);   // contiguous copy
+            else a.soa.load4(p1, st1, sx1, sy1, sz1);
+            if (i2) sb_load(a.sb, i2, sl2, st2, sx2, sy2, sz2);
+            else a.soa.load4(p2, st2, sx2, sy2, sz2);
+            double h0, h1;
+            const bool x1 = EXCL && __ldg(a.etraj + p1) == S.qtraj[qi1];
+            const bool x2 = EXCL && __ldg(a.etraj + p2) == S.qtraj[qi2];
+            if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
+                record_hit<OUT, CNT>(S, a, qi1, p1, h0, h1, s_oa, s_g);
+            if (v2 && !x2 &&
+                refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
+                record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1, s_oa, s_g);
+        }
+        maybe_flush<OUT>(S, a, lane, 64u);
+    }
+}
+
+// Step 2 of a tile: counts; canonical staging, or the last spill flush.
+template <bool OUT>
+__device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int lane, uint32_t wt,
+                                            uint32_t sp, const OutlierArgs* s_oa,
+                                            const GridParams* s_g) {
+    // (OUT: a staged tile's ids are resolved, and its hits on
+    //  non-canonical copies dropped, before the counts are read; a
+    //  spilled tile's counts are corrected by k_spill_filter, and their
+    //  maximum taken by k_spill_max after it)
+    if constexpr (OUT) {
+        if (!S.over && !a.count_only && !S.spilled && !a.spill_all)
+            filter_resolve_ids(S, s_oa, s_g, lane);
+    }
+    const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
+    if (lane < WQ && sp < a.nq) {
+        a.counts[S.qid[lane]] = cnt;
+        if (cnt && !(OUT && S.spilled)) atomicMax(&a.ctr->max_count, cnt);
+    }
+    if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane);
+    __syncwarp();
+    const uint32_t nh = S.nhit;
+    bool over = S.over != 0u;
+    if (a.spill_all) {
+        // re-run: every hit is in the spill buffer (exactly sized)
+    } else if (!over && S.spilled) {
+        if (lane == 0) {
+            a.tile_base[wt] = SPILLED;
+            a.spill_tiles[atomicAdd(&a.ctr->n_spill, 1u)] = wt;
+        }
+    } else if (!over && nh > 0) {
+        uint32_t inc = cnt;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+            if (lane >= o) inc += u;
+        }
+        if (lane < WQ) S.qoff[lane] = inc - cnt;
+        if (!OUT) {
+            for (uint32_t i = lane; i < nh; i += 32) {  // sorted position -> entry id
+                const unsigned long long k = S.hkey[i];
+                const uint32_t e = __ldg(a.soa.eid + (uint32_t)(k >> 10));
+                S.hkey[i] = (k & ~(0xffffffffull << 10)) | ((unsigned long long)e << 10);
+            }
+        }
+        unsigned long long b = 0;
+        if (lane == 0) b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
+        b = __shfl_sync(0xffffffffu, b, 0);
+        over = b + nh > a.stage_cap;
+        __syncwarp();
+        if (!over) {
+            for (uint32_t i = lane; i < nh; i += 32) {
+                const unsigned long long k = S.hkey[i];
+                const uint32_t q = (uint32_t)(k >> 42), e = (uint32_t)(k >> 10);
+                // rank inside the query: hits with a smaller entry id,
+                // ties (equal caller ids) broken by stage slot, so every
+                // slot of the tile's range is written exactly once
+                // (a query with one staged hit -- most of them on the
+                // galaxy workloads -- has rank 0)
+                uint32_t rank = 0;
+                if (S.qcount[q] > 1u) {
+                    for (uint32_t j = 0; j < nh; ++j) {
+                        const unsigned long long kj = S.hkey[j];
+                        const uint32_t ej = (uint32_t)(kj >> 10);
+                        rank += ((uint32_t)(kj >> 42) == q && (ej < e || (ej == e && j < i))) ? 1u : 0u;
+                    }
+                }
+                const uint32_t slot = (uint32_t)(k & 1023ull);
+                dts_result r;
+                r.query_id = a.qmap ? __ldg(a.qmap + S.qid[q]) : S.qid[q] + a.qid_base;
+                r.entry_id = e;
+                r.t_start = S.h0[slot];
+                r.t_end = S.h1[slot];
+                a.stage[b + S.qoff[q] + rank] = r;
+            }
+            if (lane == 0) a.tile_base[wt] = b;
+        }
+    } else if (!over && lane == 0) {
+        a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
+    }
+    if (over && !a.spill_all && !a.count_only && lane == 0) {
+        a.tile_base[wt] = NONE;
+        a.over_tiles[atomicAdd(&a.ctr->n_over, 1u)] = wt;
+    }
+}
+
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
 // temporal methods compile without that indirection.  GROUP: one-run
 // queries (temporal / subbin methods) streamed per group of identical runs
@@ -441,149 +597,11 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
                         start, cnt, n_probe);
                 ind = qs.rind;
             }
-            unsigned long long incl = cnt;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const unsigned long long u = __shfl_up_sync(0xffffffffu, incl, o);
-                if (lane >= o) incl += u;
-            }
-            const unsigned long long total = __shfl_sync(0xffffffffu, incl, 31);
-            const unsigned long long excl = incl - cnt;
-            n_cand += total;
-            // the round's non-empty runs, compacted into shared memory:
-            // (position delta start - excl mod 2^32, query | method index <<
-            // 8); a candidate t lies in run r = (non-empty runs starting at
-            // or before t) - 1, counted with one OR-reduction of the run
-            // starts per 32 candidates -- no per-candidate search
-            const bool ne = cnt > 0;
-            const uint32_t lt = (1u << lane) - 1u;
-            const uint32_t nemask = __ballot_sync(0xffffffffu, ne);
-            if (ne) S.run[__popc(nemask & lt)] = make_uint2(start - (uint32_t)excl,
-                                                            (uint32_t)qi | (ind << 8));
-            __syncwarp();
-            uint32_t before = 0;          // non-empty runs starting before `base`
-            for (unsigned long long base = 0; base < total; base += 64) {
-                // run-start offsets inside the two 32-candidate halves
-                const unsigned long long o1 = excl - base, o2 = o1 - 32;
-                const uint32_t m1 = __reduce_or_sync(0xffffffffu, (ne && excl >= base && o1 < 32)
-                                                                      ? 1u << (uint32_t)o1 : 0u);
-                const uint32_t m2 = __reduce_or_sync(
-                    0xffffffffu, (ne && excl >= base + 32 && o2 < 32) ? 1u << (uint32_t)o2 : 0u);
-                const uint32_t r1 = min(before + __popc(m1 & (lt | (1u << lane))) - 1u, 31u);
-                before += __popc(m1);
-                const uint32_t r2 = min(before + __popc(m2 & (lt | (1u << lane))) - 1u, 31u);
-                before += __popc(m2);
-                const unsigned long long t1 = base + lane, t2 = t1 + 32;
-                const bool v1 = t1 < total, v2 = t2 < total;
-                if (v1) {
-                    const uint2 ru1 = S.run[r1];
-                    const uint2 ru2 = v2 ? S.run[r2] : ru1;
-                    const int qi1 = (int)(ru1.y & 0xffu), qi2 = (int)(ru2.y & 0xffu);
-                    const uint32_t i1 = SB ? ru1.y >> 8 : 0u, i2 = SB ? ru2.y >> 8 : 0u;
-                    uint32_t p1 = (uint32_t)t1 + ru1.x;
-                    uint32_t p2 = v2 ? (uint32_t)t2 + ru2.x : p1;
-                    const uint32_t sl1 = p1, sl2 = p2;      // subbin slots (when i != 0)
-                    if (i1) p1 = __ldg(sb_ids(a.sb, i1) + sl1);   // id -> sorted position
-                    if (v2 && i2) p2 = __ldg(sb_ids(a.sb, i2) + sl2);
-                    else if (!v2) p2 = p1;
-                    double2 st1, sx1, sy1, sz1, st2, sx2, sy2, sz2;
-                    if (i1) sb_load(a.sb, i1, sl1, st1, sx1, sy1, sz1);   // contiguous copy
-                    else a.soa.load4(p1, st1, sx1, sy1, sz1);
-                    if (i2) sb_load(a.sb, i2, sl2, st2, sx2, sy2, sz2);
-                    else a.soa.load4(p2, st2, sx2, sy2, sz2);
-                    double h0, h1;
-                    const bool x1 = EXCL && __ldg(a.etraj + p1) == S.qtraj[qi1];
-                    const bool x2 = EXCL && __ldg(a.etraj + p2) == S.qtraj[qi2];
-                    if (!x1 && refine(smem_query(S, qi1), st1, sx1, sy1, sz1, d2, h0, h1))
-                        record_hit<OUT, CNT>(S, a, qi1, p1, h0, h1, s_oa, s_g);
-                    if (v2 && !x2 &&
-                        refine(smem_query(S, qi2), st2, sx2, sy2, sz2, d2, h0, h1))
-                        record_hit<OUT, CNT>(S, a, qi2, p2, h0, h1, s_oa, s_g);
-                }
-                maybe_flush<OUT>(S, a, lane, 64u);
-            }
+            stream_round<SB, EXCL, OUT, CNT>(S, a, lane, start, cnt, qi, ind, d2, n_cand, s_oa, s_g);
         }
         __syncwarp();
 
-        // ---- 2: counts; canonical staging, or the last spill flush
-        // (OUT: a staged tile's ids are resolved, and its hits on
-        //  non-canonical copies dropped, before the counts are read; a
-        //  spilled tile's counts are corrected by k_spill_filter, and their
-        //  maximum taken by k_spill_max after it)
-        if constexpr (OUT) {
-            if (!S.over && !a.count_only && !S.spilled && !a.spill_all)
-                filter_resolve_ids(S, s_oa, s_g, lane);
-        }
-        const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
-        if (lane < WQ && sp < a.nq) {
-            a.counts[S.qid[lane]] = cnt;
-            if (cnt && !(OUT && S.spilled)) atomicMax(&a.ctr->max_count, cnt);
-        }
-        if (a.spill_all || S.spilled) flush_spill<OUT>(S, a, lane);
-        __syncwarp();
-        const uint32_t nh = S.nhit;
-        bool over = S.over != 0u;
-        if (a.spill_all) {
-            // re-run: every hit is in the spill buffer (exactly sized)
-        } else if (!over && S.spilled) {
-            if (lane == 0) {
-                a.tile_base[wt] = SPILLED;
-                a.spill_tiles[atomicAdd(&a.ctr->n_spill, 1u)] = wt;
-            }
-        } else if (!over && nh > 0) {
-            uint32_t inc = cnt;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
-                if (lane >= o) inc += u;
-            }
-            if (lane < WQ) S.qoff[lane] = inc - cnt;
-            if (!OUT) {
-                for (uint32_t i = lane; i < nh; i += 32) {  // sorted position -> entry id
-                    const unsigned long long k = S.hkey[i];
-                    const uint32_t e = __ldg(a.soa.eid + (uint32_t)(k >> 10));
-                    S.hkey[i] = (k & ~(0xffffffffull << 10)) | ((unsigned long long)e << 10);
-                }
-            }
-            unsigned long long b = 0;
-            if (lane == 0) b = atomicAdd(&a.ctr->staged, (unsigned long long)nh);
-            b = __shfl_sync(0xffffffffu, b, 0);
-            over = b + nh > a.stage_cap;
-            __syncwarp();
-            if (!over) {
-                for (uint32_t i = lane; i < nh; i += 32) {
-                    const unsigned long long k = S.hkey[i];
-                    const uint32_t q = (uint32_t)(k >> 42), e = (uint32_t)(k >> 10);
-                    // rank inside the query: hits with a smaller entry id,
-                    // ties (equal caller ids) broken by stage slot, so every
-                    // slot of the tile's range is written exactly once
-                    // (a query with one staged hit -- most of them on the
-                    // galaxy workloads -- has rank 0)
-                    uint32_t rank = 0;
-                    if (S.qcount[q] > 1u) {
-                        for (uint32_t j = 0; j < nh; ++j) {
-                            const unsigned long long kj = S.hkey[j];
-                            const uint32_t ej = (uint32_t)(kj >> 10);
-                            rank += ((uint32_t)(kj >> 42) == q && (ej < e || (ej == e && j < i))) ? 1u : 0u;
-                        }
-                    }
-                    const uint32_t slot = (uint32_t)(k & 1023ull);
-                    dts_result r;
-                    r.query_id = a.qmap ? __ldg(a.qmap + S.qid[q]) : S.qid[q] + a.qid_base;
-                    r.entry_id = e;
-                    r.t_start = S.h0[slot];
-                    r.t_end = S.h1[slot];
-                    a.stage[b + S.qoff[q] + rank] = r;
-                }
-                if (lane == 0) a.tile_base[wt] = b;
-            }
-        } else if (!over && lane == 0) {
-            a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
-        }
-        if (over && !a.spill_all && !a.count_only && lane == 0) {
-            a.tile_base[wt] = NONE;
-            a.over_tiles[atomicAdd(&a.ctr->n_over, 1u)] = wt;
-        }
+        tile_finish<OUT>(S, a, lane, wt, sp, s_oa, s_g);
         __syncwarp();
     }
 
