@@ -310,7 +310,7 @@ def run_own(args):
     idx = dts.build_index_device(D_dev, device=local, stream=stream)
     build_info = idx.info()
 
-    def search_step(dd, timed_kernels=True):
+    def search_step(dd, timed_kernels="defer"):
         """One search of the whole query set (this rank's balanced share of
         it at N > 1).  Returns (results, stats, (lo, hi))."""
         if world == 1:
@@ -357,7 +357,10 @@ def run_own(args):
                                                           args.warmup)
     wall = time.perf_counter() - wall0
     value = nq / (ms_per_step * 1e-3)
-    stats = [o[0] for o in outs]
+    # the library recorded each step's phase events on the launching stream
+    # ("defer": their elapsed times are read here, after the timed region,
+    # so that reading them is not part of any step)
+    stats = [dts.read_times(o[0]) for o in outs]
     lo, hi = outs[-1][1]
     nq_rank = hi - lo
     st0 = stats[-1]
@@ -394,6 +397,7 @@ def run_own(args):
     points = []
     for dp in ([] if args.no_points else POINTS.get(args.config, [])):
         pms, _, pouts, pres, _ = timed(lambda: search_step(dp), max(3, args.steps // 5), 2)
+        pouts = [(dts.read_times(o[0]), o[1]) for o in pouts]
         pst = pouts[-1][0]
         plo, phi = pouts[-1][1]
         pc = statistics.mean(o[0]["ms_count"] for o in pouts)

@@ -134,13 +134,25 @@ typedef struct {
     uint64_t cell_lookups;      /* (bin, cell) probes issued per pass                   */
     uint64_t results;           /* results returned                                     */
     uint32_t max_results_per_query;
-    uint32_t time_kernels;      /* in: nonzero = record CUDA-event times below        */
+    uint32_t time_kernels;      /* in: 1 = record CUDA-event phase times below and read
+                                   them before returning; 2 = record them only (read
+                                   later by dts_search_read_times, so that the call
+                                   returns as soon as its results are ready)          */
     float    ms_prep;           /* query keys + sort                                    */
     float    ms_count;          /* pass 1 (fused candidate streaming + refine, count)   */
     float    ms_scan;           /* exclusive scan of per-query counts                   */
     float    ms_scatter;        /* pass 2 (fused streaming + refine, scatter)           */
     float    ms_canon;          /* per-query sort by entry id                           */
+    uint32_t timer_slot;        /* out (time_kernels == 2): the call's event set        */
 } dts_search_stats;
+
+/* The phase times of a search made with time_kernels == 2: fills ms_* of
+ * *stats from the event set named by stats->timer_slot (waits for those
+ * events).  Event sets live per calling thread and device, 1024 of them
+ * recycled in call order: call from the searching thread, with its device
+ * current, within 1024 timed searches.  DTS_EINVAL for a recycled or unknown
+ * slot. */
+dts_status dts_search_read_times(dts_search_stats* stats);
 
 typedef struct dts_index dts_index;   /* opaque; owns the device copy of D + index */
 

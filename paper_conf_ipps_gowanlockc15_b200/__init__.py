@@ -33,7 +33,7 @@ EXPORTED_SYMBOLS = (
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
     "dts_search_device_ex", "dts_canonicalize_device", "dts_merge_trajectories_device",
     "dts_query_costs_device", "dts_search_count", "dts_search_count_device",
-    "dts_search_stream",
+    "dts_search_stream", "dts_search_read_times",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -74,7 +74,8 @@ class SearchStats(ctypes.Structure):
                 ("results", ctypes.c_uint64), ("max_results_per_query", ctypes.c_uint32),
                 ("time_kernels", ctypes.c_uint32), ("ms_prep", ctypes.c_float),
                 ("ms_count", ctypes.c_float), ("ms_scan", ctypes.c_float),
-                ("ms_scatter", ctypes.c_float), ("ms_canon", ctypes.c_float)]
+                ("ms_scatter", ctypes.c_float), ("ms_canon", ctypes.c_float),
+                ("timer_slot", ctypes.c_uint32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -146,6 +147,8 @@ def load():
     lib.dts_search_stream.restype = ctypes.c_int
     lib.dts_query_costs_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, P]
     lib.dts_query_costs_device.restype = ctypes.c_int
+    lib.dts_search_read_times.argtypes = [ctypes.POINTER(SearchStats)]
+    lib.dts_search_read_times.restype = ctypes.c_int
     lib.dts_canonicalize_device.argtypes = [P, S, P]
     lib.dts_canonicalize_device.restype = ctypes.c_int
     lib.dts_search_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, pp, ps,
@@ -350,7 +353,7 @@ def search_ex(index: Index, Q, d: float, query_id_base: int = 0, stream=None,
     out = ctypes.c_void_p()
     cnt = ctypes.c_size_t()
     st = SearchStats()
-    st.time_kernels = 1 if time_kernels else 0
+    st.time_kernels = _timing_mode(time_kernels)
     _check(lib.dts_search_ex(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
                              float(d), ctypes.byref(opts), ctypes.c_void_p(_stream_ptr(stream)),
                              ctypes.byref(out), ctypes.byref(cnt), ctypes.byref(st)))
@@ -369,6 +372,22 @@ def search(index: Index, Q, d: float, query_id_base: int = 0, stream=None) -> np
     return _host_results(out.value, cnt.value)
 
 
+def _timing_mode(time_kernels) -> int:
+    """time_kernels: False/0 off, True/1 phase times read before the call
+    returns, "defer"/2 recorded only (read later by read_times)."""
+    if time_kernels == "defer":
+        return 2
+    return int(time_kernels) if time_kernels in (0, 1, 2) else (1 if time_kernels else 0)
+
+
+def read_times(stats: dict) -> dict:
+    """dts_search_read_times: the phase times of a search made with
+    time_kernels="defer" (same thread), as a new stats dict."""
+    st = SearchStats(**{k: stats[k] for k, _ in SearchStats._fields_})
+    _check(load().dts_search_read_times(ctypes.byref(st)))
+    return st.as_dict()
+
+
 def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=None,
                   n: int = None, time_kernels: bool = False, query_ids=None, query_traj=None,
                   exclude_same_trajectory: bool = False):
@@ -382,7 +401,7 @@ def search_device(index: Index, Q_dev, d: float, query_id_base: int = 0, stream=
     out = ctypes.c_void_p()
     cnt = ctypes.c_size_t()
     st = SearchStats()
-    st.time_kernels = 1 if time_kernels else 0
+    st.time_kernels = _timing_mode(time_kernels)
     if query_ids is None and query_traj is None and not exclude_same_trajectory:
         _check(lib.dts_search_device(index.handle, ctypes.c_void_p(ptr), n, float(d),
                                      int(query_id_base), ctypes.c_void_p(_stream_ptr(stream)),
@@ -413,7 +432,7 @@ def search_count(index: Index, Q, d: float, query_traj=None,
     counts = np.empty(Q.shape[0], dtype=np.uint32)
     total = ctypes.c_uint64()
     st = SearchStats()
-    st.time_kernels = 1 if time_kernels else 0
+    st.time_kernels = _timing_mode(time_kernels)
     _check(lib.dts_search_count(index.handle, Q.ctypes.data if Q.size else None, Q.shape[0],
                                 float(d), ctypes.byref(opts),
                                 ctypes.c_void_p(_stream_ptr(stream)),
@@ -432,7 +451,7 @@ def search_count_device(index: Index, Q_dev, d: float, counts_out=None, stream=N
         counts_out = torch.empty(nq, dtype=torch.int32, device=Q_dev.device)
     total = ctypes.c_uint64()
     st = SearchStats()
-    st.time_kernels = 1 if time_kernels else 0
+    st.time_kernels = _timing_mode(time_kernels)
     opts = _options()
     _check(lib.dts_search_count_device(index.handle, ctypes.c_void_p(Q_dev.data_ptr() if nq else 0),
                                        nq, float(d), ctypes.byref(opts),

@@ -755,6 +755,13 @@ dts_status dts_search_device(const dts_index* index, const dts_segment* Q_dev, s
                          out_count, stats);
 }
 
+dts_status dts_search_read_times(dts_search_stats* stats) {
+    return guarded([&] {
+        if (!stats) throw Error(DTS_EINVAL, "stats is NULL");
+        search_read_times(stats);
+    });
+}
+
 void dts_free_results(dts_result* results) { pinned_free(results); }
 
 void dts_free_results_device(void* results) {

@@ -7,6 +7,9 @@
 #include <stdint.h>
 
 #include <atomic>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <stdexcept>
 #include <string>
@@ -15,6 +18,37 @@
 #include "../../include/dts.h"
 
 namespace dts {
+
+// ------------------------------------------------------------ host trace
+// Host timeline of one call (DTS_TRACE=1: one line on stderr per call, the
+// microseconds from the call's entry to each mark); a diagnostic of the
+// per-call host cost, off by default.
+struct HostTrace {
+    static bool enabled() {
+        static const bool on = [] {
+            const char* e = std::getenv("DTS_TRACE");
+            return e && e[0] == '1';
+        }();
+        return on;
+    }
+    const char* tag;
+    bool on = enabled();
+    int k = 0;
+    const char* what[16];
+    std::chrono::steady_clock::time_point t0 = std::chrono::steady_clock::now(), t[16];
+    explicit HostTrace(const char* name) : tag(name) {}
+    void mark(const char* w) {
+        if (on && k < 16) { what[k] = w; t[k++] = std::chrono::steady_clock::now(); }
+    }
+    ~HostTrace() {
+        if (!on) return;
+        std::fprintf(stderr, "[dts trace] %s", tag);
+        for (int i = 0; i < k; ++i)
+            std::fprintf(stderr, " %s=%.1f", what[i],
+                         std::chrono::duration<double, std::micro>(t[i] - t0).count());
+        std::fprintf(stderr, "\n");
+    }
+};
 
 // ---------------------------------------------------------------- errors
 struct Error : std::runtime_error {
@@ -457,6 +491,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                    const uint32_t* qtraj = nullptr, bool exclude_same_traj = false,
                    bool count_only = false, uint32_t* counts_out = nullptr);
 // Per-query candidate counts summed per block of `block` queries (search.cu).
+void search_read_times(dts_search_stats* stats);
 void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
                         uint32_t block, unsigned long long* out, cudaStream_t s);
 // Trajectory-level merge (traj.cu); output in cache_alloc'd device memory.

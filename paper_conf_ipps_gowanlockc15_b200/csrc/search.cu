@@ -402,6 +402,64 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
     }
 }
 
+// Query order for the grid method ("query segments in Q are sorted by
+// non-decreasing t_start"): the top QSB bits of the packed key -- the time
+// bin and the top spatial bit on C4 -- in one counting-sort pass.  Each CTA
+// takes the exclusive digit bases from k_qkeys' histogram, counts its tile
+// in shared memory (the atomics' return values are the ranks), reserves its
+// per-digit ranges with one global atomic per digit present, and writes the
+// rows.  The order inside a digit is unspecified: it only groups queries
+// for locality (results are canonical whatever the order).
+constexpr int QS_ITEMS = 8;
+__global__ void __launch_bounds__(PT) k_qscatter(const unsigned long long* __restrict__ keys,
+                                                uint32_t nq, int shift, int bits,
+                                                const uint32_t* __restrict__ hist,
+                                                uint32_t* __restrict__ cursor,
+                                                unsigned long long row_mask,
+                                                uint32_t* __restrict__ order) {
+    __shared__ uint32_t base[OS_HSTRIDE], lcnt[OS_HSTRIDE], wsum[PT / 32];
+    const uint32_t nd = 1u << bits, t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    // exclusive bases of the digits (nd <= 512: two per thread)
+    const uint32_t h0 = 2 * t < nd ? hist[2 * t] : 0u, h1 = 2 * t + 1 < nd ? hist[2 * t + 1] : 0u;
+    uint32_t inc = h0 + h1;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, inc, o);
+        if (lane >= (uint32_t)o) inc += u;
+    }
+    if (lane == 31) wsum[warp] = inc;
+    lcnt[2 * t] = 0;
+    lcnt[2 * t + 1] = 0;
+    __syncthreads();
+    uint32_t pre = inc - h0 - h1;
+    for (uint32_t w = 0; w < warp; ++w) pre += wsum[w];
+    base[2 * t] = pre;
+    base[2 * t + 1] = pre + h0;
+    const uint32_t i0 = blockIdx.x * (PT * QS_ITEMS) + t;
+    unsigned long long k[QS_ITEMS];
+    uint32_t r[QS_ITEMS];
+#pragma unroll
+    for (int j = 0; j < QS_ITEMS; ++j) {
+        const uint32_t i = i0 + (uint32_t)j * PT;
+        k[j] = i < nq ? keys[i] : 0ull;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < QS_ITEMS; ++j) {
+        const uint32_t i = i0 + (uint32_t)j * PT;
+        if (i < nq) r[j] = atomicAdd(&lcnt[(uint32_t)(k[j] >> shift) & (nd - 1u)], 1u);
+    }
+    __syncthreads();
+    for (uint32_t dg = t; dg < nd; dg += PT)
+        if (lcnt[dg]) base[dg] += atomicAdd(&cursor[dg], lcnt[dg]);
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < QS_ITEMS; ++j) {
+        const uint32_t i = i0 + (uint32_t)j * PT;
+        if (i < nq) order[base[(uint32_t)(k[j] >> shift) & (nd - 1u)] + r[j]] = (uint32_t)(k[j] & row_mask);
+    }
+}
+
 __global__ void __launch_bounds__(PT) k_unpack_order(const unsigned long long* __restrict__ keys,
                                                     uint32_t n, unsigned long long mask,
                                                     uint32_t* __restrict__ order) {
@@ -472,21 +530,56 @@ __global__ void __launch_bounds__(PT) k_query_costs(const double4* __restrict__ 
     if (c) atomicAdd(&out[i / block], c);
 }
 
+// Phase events of one search (time_kernels): sets of six events per thread
+// and device, created on first use and recycled in call order (creating
+// and destroying them per call cost host time on the call's critical path).
+// Mode 2 leaves the elapsed-time reads to dts_search_read_times, after the
+// caller's timed region.
+constexpr uint32_t TIMER_SETS = 1024;
+struct TimerRing {
+    cudaEvent_t ev[TIMER_SETS][6];
+    bool made[TIMER_SETS] = {false};
+    uint32_t next = 0;            // calls so far (slot = next % TIMER_SETS)
+    int k[TIMER_SETS] = {0};      // events recorded per set
+};
+TimerRing& timer_ring(int dev) {
+    static thread_local TimerRing* rings[64] = {nullptr};
+    if (dev < 0 || dev >= 64) throw Error(DTS_ENOTSUP, "device ordinal >= 64");
+    if (!rings[dev]) rings[dev] = new TimerRing();
+    return *rings[dev];
+}
+
 struct EventTimer {
     bool on;
     cudaStream_t s;
-    cudaEvent_t ev[6];
-    int k = 0;
+    cudaEvent_t* ev = nullptr;
+    int* k = nullptr;
+    uint32_t handle = 0;
+    int k0 = 0;
     EventTimer(bool enable, cudaStream_t st) : on(enable), s(st) {
-        if (on) for (auto& e : ev) DTS_CUDA(cudaEventCreate(&e));
+        if (!on) {
+            k = &k0;
+            return;
+        }
+        int dev = 0;
+        DTS_CUDA(cudaGetDevice(&dev));
+        TimerRing& r = timer_ring(dev);
+        handle = r.next++;
+        const uint32_t i = handle % TIMER_SETS;
+        if (!r.made[i]) {
+            for (auto& e : r.ev[i]) DTS_CUDA(cudaEventCreate(&e));
+            r.made[i] = true;
+        }
+        ev = r.ev[i];
+        k = &r.k[i];
+        *k = 0;
     }
-    void mark() { if (on && k < 6) DTS_CUDA(cudaEventRecord(ev[k++], s)); }
+    void mark() { if (on && *k < 6) DTS_CUDA(cudaEventRecord(ev[(*k)++], s)); }
     float ms(int i) {
         float t = 0.f;
-        if (on && i + 1 < k) cudaEventElapsedTime(&t, ev[i], ev[i + 1]);
+        if (on && i + 1 < *k) cudaEventElapsedTime(&t, ev[i], ev[i + 1]);
         return t;
     }
-    ~EventTimer() { if (on) for (auto& e : ev) cudaEventDestroy(e); }
 };
 
 }  // namespace
@@ -497,9 +590,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                    const uint32_t* qtraj, bool exclude_same_traj, bool count_only,
                    uint32_t* counts_out) {
     out->results = nullptr;
+    HostTrace tr("search");
     out->count = 0;
     dts_search_stats local{};
     if (stats) local.time_kernels = stats->time_kernels;
+    local.timer_slot = 0xffffffffu;               // set when phase events are recorded
     if (nq == 0) {
         if (stats) *stats = local;
         return;
@@ -512,6 +607,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     const double4* Q = reinterpret_cast<const double4*>(Q_dev);
     DevBuf<Counters> ctr(1, s);
     DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
+    tr.mark("ctr");
 
     if (idx->n == 0) {   // empty index: validate only
         k_validate_only<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, ctr.p);
@@ -570,7 +666,6 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         work *= std::floor(idx->gp.maxdur / idx->gp.b) + 2.0;          // bins a query spans
         const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID ||
                             (idx->method == DTS_METHOD_GRID && work >= qsort_work);
-        DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q ? nq : 0, s);
         static const int drop = [] {           // DTS_QSORT_DROP: low key bits left unsorted
             const char* e = getenv("DTS_QSORT_DROP");
             return e ? std::max(0, std::min(24, atoi(e))) : -1;
@@ -581,19 +676,36 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         // 0.122 ms, pass 1 0.618; top 24 bits: 0.104, 0.616; top 16: 0.084,
         // 0.617).  The packed sort's digit counts come from k_qkeys and its
         // last pass writes the order itself.
+        // grid method: the top 9 key bits (the bin) in one counting
+        // pass (k_qscatter; DTS_QSORT_DROP selects the multi-pass sort);
+        // C4: pass 1 0.577 -> 0.565 ms (queries of one bin
+        // in their given order load the memory system more evenly than
+        // cell-sorted ones)
+        const bool one_pass = sort_q && packed && drop < 0 && idx->method == DTS_METHOD_GRID &&
+                              nq > 1 && idx->key_bits > 0;
         const int dr = drop >= 0 ? drop : std::max(0, idx->key_bits - 16);
-        const int lo = row_bits + std::min(dr, std::max(0, idx->key_bits - 8));
-        const bool fused = sort_q && packed && radix_onesweep(nq) && nq > 1 &&
+        const int lo = one_pass ? row_bits + std::max(0, idx->key_bits - 9)
+                                : row_bits + std::min(dr, std::max(0, idx->key_bits - 8));
+        const bool fused = !one_pass && sort_q && packed && radix_onesweep(nq) && nq > 1 &&
                            row_bits + idx->key_bits > lo;
-        const PassPlan plan = fused ? plan_passes(lo, row_bits + idx->key_bits, true) : PassPlan{};
-        DevBuf<uint32_t> hist(fused ? (size_t)plan.npass * OS_HSTRIDE : 0, s);
-        if (fused)
-            DTS_CUDA(cudaMemsetAsync(hist.p, 0, (size_t)plan.npass * OS_HSTRIDE * 4, s));
+        const PassPlan plan = fused ? plan_passes(lo, row_bits + idx->key_bits, true)
+                                    : (one_pass ? PassPlan{1, {lo}, {row_bits + idx->key_bits - lo}}
+                                                : PassPlan{});
+        DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q && !one_pass ? nq : 0, s);
+        // (one_pass: the digit counts, then the per-digit cursors)
+        DevBuf<uint32_t> hist(fused ? (size_t)plan.npass * OS_HSTRIDE : (one_pass ? 2 * OS_HSTRIDE : 0), s);
+        if (fused || one_pass)
+            DTS_CUDA(cudaMemsetAsync(hist.p, 0, hist.n * 4, s));
         k_qkeys<<<(unsigned)std::min<size_t>(blocks(nq, PT), (size_t)nsm_prep * 8), PT, 0, s>>>(
             Q, (uint32_t)nq, idx->gp, qk.p, (packed && sort_q) ? nullptr : order.p, row_bits,
-            ctr.p, plan, fused ? hist.p : nullptr);
+            ctr.p, plan, (fused || one_pass) ? hist.p : nullptr);
         DTS_LAUNCH_CHECK();
-        if (!sort_q) {
+        if (one_pass) {
+            k_qscatter<<<blocks(nq, PT * QS_ITEMS), PT, 0, s>>>(
+                qk.p, (uint32_t)nq, plan.shift[0], plan.bits[0], hist.p, hist.p + OS_HSTRIDE,
+                (1ull << row_bits) - 1ull, order.p);
+            DTS_LAUNCH_CHECK();
+        } else if (!sort_q) {
             // order = identity (written by k_qkeys)
         } else if (fused) {
             radix_sort_keys_hist(qk.p, qk_tmp.p, nq, plan, hist.p, s, order.p,
@@ -616,6 +728,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // so ms_count times pass 1 alone)
     if (idx->ready) DTS_CUDA(cudaStreamWaitEvent(s, idx->ready, 0));
     tm.mark();
+    tr.mark("prep");
 
     // ---- pass 1: warp tiles, count + staging (spilling output-heavy tiles)
     const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
@@ -639,9 +752,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         : std::max<unsigned long long>(8ull * nq + (1ull << 20),
                                        idx->spill_hint.load(std::memory_order_relaxed));
     DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s), spill_tiles(ntiles, s);
-    DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s);
+    DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s),
+        qstage(count_only ? 0 : nq, s);
     DevBuf<dts_result> stage(stage_cap, s), spill(std::max<unsigned long long>(spill_cap, 1), s);
     DTS_CUDA(cudaMemsetAsync(&ctr.p->spill_valid, 0xFF, sizeof(unsigned long long), s));
+    tr.mark("bufs");
     TileArgs ta{};
     ta.Q = Q;
     ta.order = order.p;
@@ -677,6 +792,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.method = idx->method;
     ta.sb = idx->sb;
     ta.out = idx->out;
+    ta.qstage = count_only ? nullptr : qstage.p;
     int nsm = 148;
     {
         int dev = 0;
@@ -723,6 +839,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         DTS_LAUNCH_CHECK();
     };
     launch_pass1(ta, ntiles);
+    tr.mark("pass1");
     if (ta.out.okeys && !count_only) {
         // ---- long-segment copies: spilled records carry sorted positions
         //      and their tiles' counts include hits on non-canonical copies;
@@ -775,7 +892,23 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     tm.mark();
     scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
     tm.mark();
+    tr.mark("scan");
 
+    // pass 2: staged hits gathered into the output (DTS_EMIT=tile: the
+    // per-tile scatter kernel)
+    static const bool emit_tile = [] {
+        const char* e = getenv("DTS_EMIT");
+        return e && e[0] == 't';
+    }();
+    auto launch_emit = [&](dts_result* dst, unsigned long long cap) {
+        if (emit_tile)
+            k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
+                                                             offsets.p, tile_base.p, stage.p, dst,
+                                                             cap);
+        else
+            k_emit_gather<<<(unsigned)blocks(nq, 256), 256, 0, s>>>(
+                (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, dst, cap);
+    };
     // pass 2 launched before the host learns the total, into a buffer sized
     // by this index's previous result count: a repeated search of one index
     // then has no host round trip between the scan and the copy (a buffer
@@ -798,9 +931,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     }();
     if (spec_on && hint > 0) {
         spec.p = static_cast<dts_result*>(cache_alloc(hint * sizeof(dts_result)));
-        k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
-                                                         offsets.p, tile_base.p, stage.p, spec.p,
-                                                         hint);
+        launch_emit(spec.p, hint);
         DTS_LAUNCH_CHECK();
     }
     struct {
@@ -810,7 +941,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     DTS_CUDA(cudaMemcpyAsync(&h.c, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaMemcpyAsync(&h.total, offsets.p + nq, sizeof(unsigned long long),
                              cudaMemcpyDeviceToHost, s));
+    tr.mark("emit");
     DTS_CUDA(cudaStreamSynchronize(s));
+    tr.mark("sync");
     if (!count_only) idx->result_hint.store(h.total + h.total / 8 + 4096);
     if (h.c.bad & 1) throw Error(DTS_EINVAL, "query segment with a non-finite coordinate or time");
     if (h.c.bad & 2) throw Error(DTS_EINVAL, "query segment with t_end < t_start");
@@ -827,7 +960,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         out->count = (size_t)h.total;
         tm.mark();
         tm.mark();
-        if (local.time_kernels) {
+        if (local.time_kernels == 2) {
+            local.timer_slot = tm.handle;
+        } else if (local.time_kernels) {
             local.ms_prep = tm.ms(0);
             local.ms_count = tm.ms(1);
             local.ms_scan = tm.ms(2);
@@ -884,10 +1019,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         try {
             // ---- pass 2: staged tiles are copied to their exact offsets
             if (!emitted) {
-                k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq,
-                                                                 counts.p, offsets.p,
-                                                                 tile_base.p, stage.p, fin,
-                                                                 h.total);
+                launch_emit(fin, h.total);
                 DTS_LAUNCH_CHECK();
             }
             tm.mark();
@@ -1053,7 +1185,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         tm.mark();
         tm.mark();
     }
-    if (local.time_kernels) {
+    tr.mark("done");
+    if (local.time_kernels == 2) {
+        local.timer_slot = tm.handle;
+    } else if (local.time_kernels) {
         DTS_CUDA(cudaStreamSynchronize(s));
         local.ms_prep = tm.ms(0);
         local.ms_count = tm.ms(1);
@@ -1062,6 +1197,23 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         local.ms_canon = tm.ms(4);
     }
     if (stats) *stats = local;
+}
+
+void search_read_times(dts_search_stats* st) {
+    int dev = 0;
+    DTS_CUDA(cudaGetDevice(&dev));
+    TimerRing& r = timer_ring(dev);
+    const uint32_t h = st->timer_slot, i = h % TIMER_SETS;
+    if (h >= r.next || r.next - h > TIMER_SETS || !r.made[i])
+        throw Error(DTS_EINVAL, "timer slot recycled or not from this thread and device");
+    const int k = r.k[i];
+    if (k > 0) DTS_CUDA(cudaEventSynchronize(r.ev[i][k - 1]));
+    float* out[5] = {&st->ms_prep, &st->ms_count, &st->ms_scan, &st->ms_scatter, &st->ms_canon};
+    for (int j = 0; j < 5; ++j) {
+        float t = 0.f;
+        if (j + 1 < k) DTS_CUDA(cudaEventElapsedTime(&t, r.ev[i][j], r.ev[i][j + 1]));
+        *out[j] = t;
+    }
 }
 
 void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,

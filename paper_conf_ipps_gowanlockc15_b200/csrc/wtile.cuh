@@ -90,6 +90,7 @@ struct TileArgs {
     uint32_t method;
     SubbinIndex sb;
     OutlierIndex out;                  // long-segment copies (okeys NULL: none)
+    unsigned long long* qstage;        // per query id: first staged slot (pass 2), or NULL
 };
 
 __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
@@ -383,6 +384,7 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
     __syncwarp();
     const uint32_t nh = S.nhit;
     bool over = S.over != 0u;
+    unsigned long long sbase = NONE;          // the tile's staged range, when staged
     if (a.spill_all) {
         // re-run: every hit is in the spill buffer (exactly sized)
     } else if (!over && S.spilled) {
@@ -436,6 +438,7 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
                 a.stage[b + S.qoff[q] + rank] = r;
             }
             if (lane == 0) a.tile_base[wt] = b;
+            sbase = b;
         }
     } else if (!over && lane == 0) {
         a.tile_base[wt] = NONE - 1;          // no hits: nothing to emit
@@ -444,6 +447,10 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
         a.tile_base[wt] = NONE;
         a.over_tiles[atomicAdd(&a.ctr->n_over, 1u)] = wt;
     }
+    // per query id: where its staged hits start (NONE: spilled or re-run,
+    // placed by the spill path), for pass 2's gather
+    if (a.qstage && !a.spill_all && lane < WQ && sp < a.nq && cnt)
+        a.qstage[S.qid[lane]] = sbase == NONE ? NONE : sbase + S.qoff[lane];
 }
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
@@ -656,6 +663,56 @@ __global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ 
         const unsigned long long o = __shfl_sync(0xffffffffu, off, q);
         const uint32_t e = __shfl_sync(0xffffffffu, excl, q);
         if (i < nh && o + (i - e) < cap) out[o + (i - e)] = stage[tb + i];
+    }
+}
+
+// Pass 2 as a gather: a warp per 32 consecutive query ids.  The warp's
+// staged queries (at most WH hits each: a staged tile holds at most WH) are
+// numbered by a shuffle scan of their counts; lane j of each 32-record step
+// finds its query by a shuffle search of that scan and copies the query's
+// staged record to its exact offset (queries ascend, so the writes of a
+// step are contiguous unless a spilled query sits in between).  Queries of
+// spilled or re-run tiles (qstage NONE) are left to the spill path; slots
+// from cap on are not written (speculative launch).
+__global__ void __launch_bounds__(256) k_emit_gather(uint32_t nq,
+                                                    const uint32_t* __restrict__ counts,
+                                                    const unsigned long long* __restrict__ offsets,
+                                                    const unsigned long long* __restrict__ qstage,
+                                                    const dts_result* __restrict__ stage,
+                                                    dts_result* __restrict__ out,
+                                                    unsigned long long cap) {
+    const uint32_t lane = threadIdx.x & 31;
+    const uint32_t q0 = (blockIdx.x * 256 + threadIdx.x) & ~31u;
+    if (q0 >= nq) return;
+    const uint32_t q = q0 + lane;
+    uint32_t c = 0;
+    unsigned long long o = 0, sp = NONE;
+    if (q < nq) {
+        c = counts[q];
+        if (c) sp = qstage[q];
+        if (sp != NONE) o = offsets[q];
+        else c = 0;
+    }
+    uint32_t inc = c;                         // staged records of lanes <= this one
+#pragma unroll
+    for (int k = 1; k < 32; k <<= 1) {
+        const uint32_t u = __shfl_up_sync(0xffffffffu, inc, k);
+        if (lane >= (uint32_t)k) inc += u;
+    }
+    const uint32_t total = __shfl_sync(0xffffffffu, inc, 31);
+    for (uint32_t k0 = 0; k0 < total; k0 += 32) {
+        const uint32_t k = k0 + lane;
+        int src = 0;                          // the first lane whose records reach past k
+#pragma unroll
+        for (int step = 16; step; step >>= 1) {
+            const uint32_t e = __shfl_sync(0xffffffffu, inc, src + step - 1);
+            src += e <= k ? step : 0;
+        }
+        const uint32_t ex = __shfl_sync(0xffffffffu, inc - c, src);
+        const unsigned long long os = __shfl_sync(0xffffffffu, o, src);
+        const unsigned long long ss = __shfl_sync(0xffffffffu, sp, src);
+        const unsigned long long j = os + (k - ex);
+        if (k < total && j < cap) out[j] = stage[ss + (k - ex)];
     }
 }
 

@@ -112,6 +112,37 @@ def test_concurrent_searches_two_streams(dts):
     idx.free()
 
 
+def test_deferred_phase_times(dts):
+    """time_kernels="defer": the call returns without reading its phase
+    events; dts_search_read_times reads them afterwards (the same numbers a
+    time_kernels=1 call reports, to within event resolution), and rejects a
+    slot that was never recorded."""
+    import torch
+    c = synth.make_config("C2", scale=0.05)
+    idx = dts.build_index(c.D)
+    Qd = torch.from_numpy(c.Q).cuda()
+    res0, st0 = dts.search_device(idx, Qd, c.d, time_kernels=True)
+    ref = res0.numpy().tobytes()
+    res0.free()
+    slots = []
+    for _ in range(3):
+        res, st = dts.search_device(idx, Qd, c.d, time_kernels="defer")
+        assert res.numpy().tobytes() == ref
+        assert st["ms_count"] == 0.0 and st["timer_slot"] != 0xFFFFFFFF
+        slots.append(st)
+        res.free()
+    assert len({s["timer_slot"] for s in slots}) == 3
+    for st in slots:
+        t = dts.read_times(st)
+        assert t["ms_count"] > 0.0 and t["ms_prep"] > 0.0 and t["ms_scan"] > 0.0
+        assert t["candidates"] == st0["candidates"]
+    _, st_off = dts.search_device(idx, Qd, c.d)
+    assert st_off["timer_slot"] == 0xFFFFFFFF
+    with pytest.raises(dts.DTSError):
+        dts.read_times(st_off)
+    idx.free()
+
+
 def test_query_costs_match_candidates(dts):
     """dts_query_costs_device sums, per block of queries, exactly the
     candidate pairs the search refines (its `candidates` statistic)."""

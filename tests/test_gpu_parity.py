@@ -114,7 +114,7 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_SLOTS": "1.2"},
                 {"DTS_FUSED_KEYS": "0"}, {"DTS_OS_SHAPE": "0"}, {"DTS_GATHER": "4"},
                 {"DTS_GATHER": "1"}, {"DTS_TILE_OCC": "6"}, {"DTS_TILE_OCC": "8"},
-                {"DTS_QSORT_MIN": "0"}):
+                {"DTS_QSORT_MIN": "0"}, {"DTS_QSORT_MIN": "0", "DTS_QSORT_DROP": "0"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
         import sys

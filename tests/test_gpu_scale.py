@@ -121,8 +121,8 @@ def _run_sub(code, env):
 
 
 def test_sorted_query_path_forced(dts, oracle_mod):
-    """The grid method sorts queries by index key only from 2^18 queries
-    (DTS_QSORT_MIN); forcing the sorted path on small sets (adversarial sets,
+    """The grid method sorts queries (by the key's top 9 bits, one counting
+    pass) only from 2^18 queries (DTS_QSORT_MIN); forcing the sorted path on small sets (adversarial sets,
     C2 at several d) gives the same bytes as the unsorted path and matches
     the oracle."""
     code = ("import sys; sys.path[:0] = [%r, %r]; import numpy as np, synth, "
@@ -146,8 +146,12 @@ def test_sorted_query_path_forced(dts, oracle_mod):
         return parts
     sorted_out = split(_run_sub(code, {"DTS_QSORT_MIN": "0"}))
     plain_out = split(_run_sub(code, {"DTS_QSORT_MIN": "1000000000"}))
+    # the multi-pass radix sort of the key's top bits (DTS_QSORT_DROP) instead
+    # of the one-pass counting sort of the bin bits
+    multi_out = split(_run_sub(code, {"DTS_QSORT_MIN": "0", "DTS_QSORT_DROP": "4"}))
     assert len(sorted_out) == 43
     assert sorted_out == plain_out
+    assert multi_out == plain_out
     for seed in range(40):
         D, Q = synth.adversarial(7000 + seed, 60, 60)
         d = [0.0, 0.03, 0.1, 0.3][seed % 4]
