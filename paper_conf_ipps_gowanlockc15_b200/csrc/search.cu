@@ -349,7 +349,7 @@ __device__ __forceinline__ void resolve(const GridParams& g, const HashTable& ht
 // Query keys (grid-stride), validation, and -- for the packed keys-only sort
 // -- the digit counts of every pass of its plan (hist != NULL; one pass over
 // the keys fewer than a separate histogram kernel).
-__global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uint32_t nq,
+__global__ void __launch_bounds__(PT, 4) k_qkeys(const double4* __restrict__ Q, uint32_t nq,
                                              GridParams g, unsigned long long* __restrict__ keys,
                                              uint32_t* __restrict__ ids, int shift,
                                              Counters* __restrict__ ctr, const PassPlan plan,
@@ -360,8 +360,7 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
         __syncthreads();
     }
     unsigned bad_all = 0;
-    for (uint32_t i = blockIdx.x * PT + threadIdx.x; i < nq; i += gridDim.x * PT) {
-        const double4 s0 = Q[2 * (size_t)i], s1 = Q[2 * (size_t)i + 1];
+    auto one = [&](uint32_t i, const double4 s0, const double4 s1) {
         const double c[8] = {s0.x, s0.y, s0.z, s0.w, s1.x, s1.y, s1.z, s1.w};
         unsigned bad = 0;
 #pragma unroll
@@ -393,7 +392,17 @@ __global__ void __launch_bounds__(PT) k_qkeys(const double4* __restrict__ Q, uin
                         atomicAdd(&h[p * OS_HSTRIDE + ((v >> plan.shift[p]) & ((1u << plan.bits[p]) - 1u))], 1u);
             }
         }
+    };
+    // grid-stride, two queries per step with both records' loads issued first
+    const uint32_t st = gridDim.x * PT;
+    uint32_t i = blockIdx.x * PT + threadIdx.x;
+    for (; i < nq && st <= nq - 1 - i; i += 2 * st) {
+        const double4 a0 = Q[2 * (size_t)i], a1 = Q[2 * (size_t)i + 1];
+        const double4 b0 = Q[2 * (size_t)(i + st)], b1 = Q[2 * (size_t)(i + st) + 1];
+        one(i, a0, a1);
+        one(i + st, b0, b1);
     }
+    if (i < nq) one(i, Q[2 * (size_t)i], Q[2 * (size_t)i + 1]);
     if (bad_all) atomicOr(&ctr->bad, bad_all);
     if (hist) {
         __syncthreads();
@@ -419,6 +428,15 @@ __global__ void __launch_bounds__(PT) k_qscatter(const unsigned long long* __res
                                                 uint32_t* __restrict__ order) {
     __shared__ uint32_t base[OS_HSTRIDE], lcnt[OS_HSTRIDE], wsum[PT / 32];
     const uint32_t nd = 1u << bits, t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    // the tile's keys and the digit counts are loaded together (one round trip)
+    const uint32_t i0 = blockIdx.x * (PT * QS_ITEMS) + t;
+    unsigned long long k[QS_ITEMS];
+    uint32_t r[QS_ITEMS];
+#pragma unroll
+    for (int j = 0; j < QS_ITEMS; ++j) {
+        const uint32_t i = i0 + (uint32_t)j * PT;
+        k[j] = i < nq ? keys[i] : 0ull;
+    }
     // exclusive bases of the digits (nd <= 512: two per thread)
     const uint32_t h0 = 2 * t < nd ? hist[2 * t] : 0u, h1 = 2 * t + 1 < nd ? hist[2 * t + 1] : 0u;
     uint32_t inc = h0 + h1;
@@ -435,14 +453,6 @@ __global__ void __launch_bounds__(PT) k_qscatter(const unsigned long long* __res
     for (uint32_t w = 0; w < warp; ++w) pre += wsum[w];
     base[2 * t] = pre;
     base[2 * t + 1] = pre + h0;
-    const uint32_t i0 = blockIdx.x * (PT * QS_ITEMS) + t;
-    unsigned long long k[QS_ITEMS];
-    uint32_t r[QS_ITEMS];
-#pragma unroll
-    for (int j = 0; j < QS_ITEMS; ++j) {
-        const uint32_t i = i0 + (uint32_t)j * PT;
-        k[j] = i < nq ? keys[i] : 0ull;
-    }
     __syncthreads();
 #pragma unroll
     for (int j = 0; j < QS_ITEMS; ++j) {
@@ -696,7 +706,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         DevBuf<uint32_t> hist(fused ? (size_t)plan.npass * OS_HSTRIDE : (one_pass ? 2 * OS_HSTRIDE : 0), s);
         if (fused || one_pass)
             DTS_CUDA(cudaMemsetAsync(hist.p, 0, hist.n * 4, s));
-        k_qkeys<<<(unsigned)std::min<size_t>(blocks(nq, PT), (size_t)nsm_prep * 8), PT, 0, s>>>(
+        k_qkeys<<<(unsigned)std::min<size_t>(blocks(nq, PT), (size_t)nsm_prep * 4), PT, 0, s>>>(
             Q, (uint32_t)nq, idx->gp, qk.p, (packed && sort_q) ? nullptr : order.p, row_bits,
             ctr.p, plan, (fused || one_pass) ? hist.p : nullptr);
         DTS_LAUNCH_CHECK();

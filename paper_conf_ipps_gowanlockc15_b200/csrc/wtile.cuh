@@ -687,11 +687,11 @@ __global__ void __launch_bounds__(256) k_emit_gather(uint32_t nq,
     const uint32_t q = q0 + lane;
     uint32_t c = 0;
     unsigned long long o = 0, sp = NONE;
-    if (q < nq) {
+    if (q < nq) {                             // three independent coalesced loads
         c = counts[q];
-        if (c) sp = qstage[q];
-        if (sp != NONE) o = offsets[q];
-        else c = 0;
+        sp = qstage[q];                       // (stale for c == 0: not used)
+        o = offsets[q];
+        if (c == 0 || sp == NONE) c = 0;
     }
     uint32_t inc = c;                         // staged records of lanes <= this one
 #pragma unroll
