@@ -144,6 +144,8 @@ typedef struct {
     float    ms_scatter;        /* pass 2 (fused streaming + refine, scatter)           */
     float    ms_canon;          /* per-query sort by entry id                           */
     uint32_t timer_slot;        /* out (time_kernels == 2): the call's event set        */
+    uint32_t tile_queries;      /* out: queries per warp tile of pass 1                 */
+    float    work_estimate;     /* out: expected candidates per query (grid method)     */
 } dts_search_stats;
 
 /* The phase times of a search made with time_kernels == 2: fills ms_* of

@@ -75,7 +75,8 @@ class SearchStats(ctypes.Structure):
                 ("time_kernels", ctypes.c_uint32), ("ms_prep", ctypes.c_float),
                 ("ms_count", ctypes.c_float), ("ms_scan", ctypes.c_float),
                 ("ms_scatter", ctypes.c_float), ("ms_canon", ctypes.c_float),
-                ("timer_slot", ctypes.c_uint32)]
+                ("timer_slot", ctypes.c_uint32), ("tile_queries", ctypes.c_uint32),
+                ("work_estimate", ctypes.c_float)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

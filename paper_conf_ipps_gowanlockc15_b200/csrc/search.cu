@@ -39,7 +39,6 @@
 namespace dts {
 namespace {
 
-constexpr int TQ = 16;                  // queries per warp tile (WQ of wtile.cuh)
 constexpr int PT = 256;                 // threads per CTA in warp-per-query kernels
 constexpr int PW = PT / 32;
 constexpr unsigned long long NONE = ~0ull;
@@ -485,12 +484,13 @@ __global__ void __launch_bounds__(PT) k_unpack_order(const unsigned long long* _
 // queries (their records in the first spill buffer are stale; the scan of
 // cover sizes the re-run's exact spill buffer).
 __global__ void __launch_bounds__(PT) k_mark_over(const uint32_t* __restrict__ tiles,
+                                                 uint32_t tq,
                                                  const uint32_t* __restrict__ order, uint32_t nq,
                                                  const uint32_t* __restrict__ counts,
                                                  uint32_t* __restrict__ cover) {
     const uint32_t tile = tiles[blockIdx.x];
-    const uint32_t sp = tile * TQ + threadIdx.x;
-    if (threadIdx.x < (unsigned)TQ && sp < nq) {
+    const uint32_t sp = tile * tq + threadIdx.x;
+    if (threadIdx.x < tq && sp < nq) {
         const uint32_t q = order[sp];
         cover[q] = counts[q];
     }
@@ -642,6 +642,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
         return v;
     }();
+    // expected candidates per query: entries per non-empty cell x stencil
+    // cells x bins a query spans (sizes the query sort and the warp tiles)
+    double work = idx->n_cells ? (double)idx->n / (double)idx->n_cells : 0.0;
+    for (int a = 0; a < 3; ++a)
+        work *= std::floor(2.0 * (d + idx->gp.half_ext[a]) / idx->gp.w[a]) + 2.0;
+    work *= std::floor(idx->gp.maxdur / idx->gp.b) + 2.0;
     // ---- query prep: key + sort
     DevBuf<uint32_t> order(nq, s);
     {
@@ -670,10 +676,6 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             const char* e = getenv("DTS_QSORT_WORK");
             return e ? atof(e) : 1024.0;
         }();
-        double work = idx->n_cells ? (double)idx->n / (double)idx->n_cells : 0.0;
-        for (int a = 0; a < 3; ++a)
-            work *= std::floor(2.0 * (d + idx->gp.half_ext[a]) / idx->gp.w[a]) + 2.0;
-        work *= std::floor(idx->gp.maxdur / idx->gp.b) + 2.0;          // bins a query spans
         const bool sort_q = nq >= qsort_min || idx->method != DTS_METHOD_GRID ||
                             (idx->method == DTS_METHOD_GRID && work >= qsort_work);
         static const int drop = [] {           // DTS_QSORT_DROP: low key bits left unsorted
@@ -741,7 +743,37 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     tr.mark("prep");
 
     // ---- pass 1: warp tiles, count + staging (spilling output-heavy tiles)
-    const uint32_t ntiles = (uint32_t)((nq + WQ - 1) / WQ);
+    // queries per warp tile: WQ, or fewer when the query set would not give
+    // every resident warp of pass 1 DTS_TILE_FILL (default 4) tiles -- a
+    // small set then runs on more warps, each with a shorter latency chain --
+    // but not below 7 / 4 / 2 queries for light (< 64 expected candidates per
+    // query) / medium / heavy (>= 400) queries.  Measured (device search, ms,
+    // tiles of 2 / 4 / 7 / 16 queries): C1 0.146 / 0.131 / 0.131 / 0.143; C2
+    // d = 2 0.377 / 0.382 / 0.389 / 0.466; C2 d = 8 3.42 / 3.45 / 3.61 / 4.15;
+    // S1 d = 50 0.201 / 0.189 / 0.229 / 0.250; S2 d = 0.1 0.643 / 0.744 /
+    // 0.899 / 1.329; S3 d = 0.01 0.215 / 0.181 / 0.169 / 0.166
+    static const int nsm_tiles = [] {
+        int dev = 0, v = 148;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+        return v;
+    }();
+    static const double tile_fill = [] {
+        const char* e = getenv("DTS_TILE_FILL");
+        return e ? atof(e) : 4.0;
+    }();
+    const double slots = (double)nsm_tiles * 7.0 * WW;            // resident warps of pass 1
+    const double tmin = work < 64.0 ? 7.0 : (work >= 400.0 ? 2.0 : 4.0);
+    // (the temporal and subbin methods keep WQ: their tiles' queries share
+    //  runs, streamed once per group)
+    uint32_t tq = (tile_fill <= 0.0 || idx->method != DTS_METHOD_GRID) ? (uint32_t)WQ
+        : (uint32_t)std::max(tmin, std::min((double)WQ, std::ceil((double)nq / (tile_fill * slots))));
+    static const int tile_q_env = [] {          // DTS_TILE_Q: a fixed tile size (A/B)
+        const char* e = getenv("DTS_TILE_Q");
+        return e ? std::max(1, std::min(WQ, atoi(e))) : 0;
+    }();
+    if (tile_q_env && idx->method == DTS_METHOD_GRID) tq = (uint32_t)tile_q_env;
+    const uint32_t ntiles = (uint32_t)((nq + tq - 1) / tq);
     // (DTS_STAGE_CAP: a fixed staging capacity, testing knob for the re-run
     //  of tiles that find the stage full)
     static const long long stage_env = [] {
@@ -803,6 +835,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.sb = idx->sb;
     ta.out = idx->out;
     ta.qstage = count_only ? nullptr : qstage.p;
+    ta.tq = tq;
+    local.tile_queries = tq;
+    local.work_estimate = (float)work;
     int nsm = 148;
     {
         int dev = 0;
@@ -894,8 +929,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             DTS_LAUNCH_CHECK();
         }
         if (c1.n_spill) {
-            k_spill_max<<<blocks((size_t)c1.n_spill * WQ, 128), 128, 0, s>>>(
-                spill_tiles.p, c1.n_spill, order.p, (uint32_t)nq, counts.p, ctr.p);
+            k_spill_max<<<blocks((size_t)c1.n_spill * tq, 128), 128, 0, s>>>(
+                spill_tiles.p, c1.n_spill, tq, order.p, (uint32_t)nq, counts.p, ctr.p);
             DTS_LAUNCH_CHECK();
         }
     }
@@ -904,20 +939,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     tm.mark();
     tr.mark("scan");
 
-    // pass 2: staged hits gathered into the output (DTS_EMIT=tile: the
-    // per-tile scatter kernel)
-    static const bool emit_tile = [] {
-        const char* e = getenv("DTS_EMIT");
-        return e && e[0] == 't';
-    }();
+    // pass 2: staged hits gathered into the output
     auto launch_emit = [&](dts_result* dst, unsigned long long cap) {
-        if (emit_tile)
-            k_wtile_emit<<<(ntiles + WW - 1) / WW, WT, 0, s>>>(order.p, (uint32_t)nq, counts.p,
-                                                             offsets.p, tile_base.p, stage.p, dst,
-                                                             cap);
-        else
-            k_emit_gather<<<(unsigned)blocks(nq, 256), 256, 0, s>>>(
-                (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, dst, cap);
+        k_emit_gather<<<(unsigned)blocks(nq, 256), 256, 0, s>>>(
+            (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, dst, cap);
     };
     // pass 2 launched before the host learns the total, into a buffer sized
     // by this index's previous result count: a repeated search of one index
@@ -1044,7 +1069,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     //      into a buffer of exactly their result count
                     DevBuf<unsigned long long> cover_off(nq + 1, s);
                     DTS_CUDA(cudaMemsetAsync(cover.p, 0, nq * sizeof(uint32_t), s));
-                    k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, order.p, (uint32_t)nq,
+                    k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, tq, order.p, (uint32_t)nq,
                                                           counts.p, cover.p);
                     DTS_LAUNCH_CHECK();
                     scan_exclusive_u32_to_u64(cover.p, cover_off.p, nq, s);
@@ -1089,19 +1114,19 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
                 DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 5 * sizeof(unsigned int), s));
-                const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * WQ;
+                const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * tq;
                 DevBuf<uint32_t> lists(3 * nslots, s);
                 const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
-                    k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * WQ, 4), 128, 0, s>>>(
-                        spill_tiles.p, h.c.n_spill * WQ, order.p, (uint32_t)nq, counts.p,
+                    k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * tq, 4), 128, 0, s>>>(
+                        spill_tiles.p, h.c.n_spill * tq, tq, order.p, (uint32_t)nq, counts.p,
                         offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
                         ctr.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
-                    k_seg_sort_warp<<<blocks((size_t)h.c.n_over * WQ, 4), 128, 0, s>>>(
-                        over_tiles.p, h.c.n_over * WQ, order.p, (uint32_t)nq, counts.p,
+                    k_seg_sort_warp<<<blocks((size_t)h.c.n_over * tq, 4), 128, 0, s>>>(
+                        over_tiles.p, h.c.n_over * tq, tq, order.p, (uint32_t)nq, counts.p,
                         offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
                         ctr.p);
                     DTS_LAUNCH_CHECK();

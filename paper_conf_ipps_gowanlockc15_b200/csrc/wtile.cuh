@@ -91,6 +91,7 @@ struct TileArgs {
     SubbinIndex sb;
     OutlierIndex out;                  // long-segment copies (okeys NULL: none)
     unsigned long long* qstage;        // per query id: first staged slot (pass 2), or NULL
+    uint32_t tq;                       // queries per tile (1..WQ; fewer on small query sets)
 };
 
 __device__ __forceinline__ QState smem_query(const WarpSmem& S, int qi) {
@@ -375,8 +376,9 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
         if (!S.over && !a.count_only && !S.spilled && !a.spill_all)
             filter_resolve_ids(S, s_oa, s_g, lane);
     }
-    const uint32_t cnt = lane < WQ ? S.qcount[lane] : 0u;
-    if (lane < WQ && sp < a.nq) {
+    const bool mine = lane < a.tq && sp < a.nq;
+    const uint32_t cnt = mine ? S.qcount[lane] : 0u;
+    if (mine) {
         a.counts[S.qid[lane]] = cnt;
         if (cnt && !(OUT && S.spilled)) atomicMax(&a.ctr->max_count, cnt);
     }
@@ -449,7 +451,7 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
     }
     // per query id: where its staged hits start (NONE: spilled or re-run,
     // placed by the spill path), for pass 2's gather
-    if (a.qstage && !a.spill_all && lane < WQ && sp < a.nq && cnt)
+    if (a.qstage && !a.spill_all && mine && cnt)
         a.qstage[S.qid[lane]] = sbase == NONE ? NONE : sbase + S.qoff[lane];
 }
 
@@ -481,7 +483,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
     WarpSmem& S = SW[warp];
     const GridParams& g = a.g;
     const double d = a.d, d2 = d * d;
-    const uint32_t ntiles = a.tile_list ? a.n_list : (a.nq + WQ - 1) / WQ;
+    const uint32_t ntiles = a.tile_list ? a.n_list : (a.nq + a.tq - 1) / a.tq;
     unsigned long long n_cand = 0;
     uint32_t n_probe = 0;
 
@@ -496,13 +498,13 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
         unsigned long long nlook = 0;
         bool single = false;                 // one-run query (temporal / subbin / fallback)
         uint32_t rs = 0, rc = 0, ri = 0;
-        const uint32_t sp = wt * WQ + lane;
+        const uint32_t sp = wt * a.tq + lane;
         if (lane < WQ) {
             QState q{};
             double qlo[3] = {0, 0, 0}, qhi[3] = {0, 0, 0};
             bool live = false;
             uint32_t qid = 0;
-            if (sp < a.nq) {
+            if (lane < a.tq && sp < a.nq) {
                 qid = a.order[sp];
                 live = load_query(a.Q, qid, q, qlo, qhi);
             }
@@ -521,7 +523,7 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
             qs.rstart = st.rstart; qs.rcnt = st.rcnt;
             S.qs[lane] = qs;
             S.qid[lane] = qid;
-            S.qtraj[lane] = (EXCL && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
+            S.qtraj[lane] = (EXCL && lane < a.tq && sp < a.nq) ? __ldg(a.qtraj + qid) : 0u;
             S.qcount[lane] = 0;
             nlook = st.nlook;
             if (GROUP && st.mode == MODE_TEMPORAL && st.rcnt > 0) {   // streamed in 1a
@@ -621,51 +623,6 @@ __global__ void __launch_bounds__(WT, MINB) k_wtile_count(const TileArgs a) {
 }
 
 // ------------------------------------------------------ pass 2: emission
-// One warp per warp tile: the tile's staged hits are contiguous and grouped
-// by query in canonical order; copy each query's group to its exact offset
-// (positions from cap on are not written: a speculative launch into a
-// buffer that turned out too small is discarded).
-__global__ void __launch_bounds__(WT) k_wtile_emit(const uint32_t* __restrict__ order, uint32_t nq,
-                                                  const uint32_t* __restrict__ counts,
-                                                  const unsigned long long* __restrict__ offsets,
-                                                  const unsigned long long* __restrict__ tile_base,
-                                                  const dts_result* __restrict__ stage,
-                                                  dts_result* __restrict__ out,
-                                                  unsigned long long cap) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const uint32_t ntiles = (nq + WQ - 1) / WQ;
-    const uint32_t wt = blockIdx.x * WW + warp;
-    if (wt >= ntiles) return;
-    const unsigned long long tb = tile_base[wt];
-    if (tb >= SPILLED) return;                       // spilled, re-run or empty tile
-    const uint32_t sp = wt * WQ + lane;
-    uint32_t cnt = 0;
-    unsigned long long off = 0;
-    if (lane < WQ && sp < nq) {
-        const uint32_t qid = order[sp];
-        cnt = counts[qid];
-        off = offsets[qid];
-    }
-    uint32_t incl = cnt;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t u = __shfl_up_sync(0xffffffffu, incl, o);
-        if (lane >= o) incl += u;
-    }
-    const uint32_t excl = incl - cnt;
-    const uint32_t nh = __shfl_sync(0xffffffffu, incl, 31);
-    for (uint32_t base = 0; base < nh; base += 32) {
-        const uint32_t i = base + lane;
-        int q = 0;
-#pragma unroll
-        for (int step = 16; step; step >>= 1)
-            if (__shfl_sync(0xffffffffu, incl, q + step - 1) <= i) q += step;
-        const unsigned long long o = __shfl_sync(0xffffffffu, off, q);
-        const uint32_t e = __shfl_sync(0xffffffffu, excl, q);
-        if (i < nh && o + (i - e) < cap) out[o + (i - e)] = stage[tb + i];
-    }
-}
-
 // Pass 2 as a gather: a warp per 32 consecutive query ids.  The warp's
 // staged queries (at most WH hits each: a staged tile holds at most WH) are
 // numbered by a shuffle scan of their counts; lane j of each 32-record step
@@ -753,12 +710,13 @@ __global__ void __launch_bounds__(128) k_spill_filter(const TileArgs a, unsigned
 
 // The largest count among the spilled tiles' queries (after k_spill_filter).
 __global__ void __launch_bounds__(128) k_spill_max(const uint32_t* __restrict__ tiles,
-                                                  uint32_t ntl, const uint32_t* __restrict__ order,
+                                                  uint32_t ntl, uint32_t tq,
+                                                  const uint32_t* __restrict__ order,
                                                   uint32_t nq, const uint32_t* __restrict__ counts,
                                                   Counters* __restrict__ ctr) {
     const uint32_t i = blockIdx.x * 128 + threadIdx.x;
-    if (i >= ntl * WQ) return;
-    const uint32_t sp = tiles[i / WQ] * WQ + i % WQ;
+    if (i >= ntl * tq) return;
+    const uint32_t sp = tiles[i / tq] * tq + i % tq;
     if (sp >= nq) return;
     const uint32_t c = counts[order[sp]];
     if (c) atomicMax(&ctr->max_count, c);
@@ -875,7 +833,7 @@ struct SegWarpSmem {
 };
 
 __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restrict__ tiles,
-                                                      uint32_t nslots,
+                                                      uint32_t nslots, uint32_t tq,
                                                       const uint32_t* __restrict__ order,
                                                       uint32_t nq,
                                                       const uint32_t* __restrict__ counts,
@@ -893,7 +851,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const uint32_t w = blockIdx.x * 4 + warp;
     if (w >= nslots) return;
-    const uint32_t sp = tiles[w / WQ] * WQ + w % WQ;
+    const uint32_t sp = tiles[w / tq] * tq + w % tq;
     if (sp >= nq) return;
     const uint32_t q = order[sp];
     const uint32_t c = counts[q];

@@ -65,7 +65,7 @@ for pt in a.points:
                       "count_ms": statistics.median(x["ms_count"] for x in sts),
                       "prep_ms": statistics.median(x["ms_prep"] for x in sts),
                       "emit_ms": statistics.median(x["ms_scatter"] for x in sts),
-                      "canon_ms": statistics.median(x["ms_canon"] for x in sts),
+                      "canon_ms": statistics.median(x["ms_canon"] for x in sts), "tq": sts[-1].get("tile_queries"), "work": sts[-1].get("work_estimate"),
                       "results": n, "candidates": sts[-1]["candidates"],
                       "build_ms": binf["ms_build"], "build_phases": binf["ms_phase"],
                       "hash_bytes": binf["hash_bytes"]}), flush=True)
