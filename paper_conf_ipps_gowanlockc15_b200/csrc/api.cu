@@ -292,8 +292,12 @@ dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_
                              uint32_t qid_base, cudaStream_t s, size_t chunk,
                              const uint32_t* dmap, const uint32_t* dtraj, bool excl,
                              dts_search_stats* stats, size_t* out_count) {
-    cudaStream_t cs = nullptr;
+    // H2D of chunk i+1 on cs and D2H of chunk i-1's results on ds run while
+    // chunk i is searched on s: the two copy directions overlap (PCIe is
+    // full duplex) and both overlap the search
+    cudaStream_t cs = nullptr, ds = nullptr;
     DTS_CUDA(cudaStreamCreateWithFlags(&cs, cudaStreamNonBlocking));
+    DTS_CUDA(cudaStreamCreateWithFlags(&ds, cudaStreamNonBlocking));
     cudaEvent_t h2d[2] = {nullptr, nullptr};
     struct Pending {
         dts_result* dev;
@@ -306,11 +310,13 @@ dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_
     if (stats) agg.time_kernels = stats->time_kernels;
     auto cleanup = [&]() {
         if (cs) cudaStreamSynchronize(cs);
+        if (ds) cudaStreamSynchronize(ds);
         for (auto& p : pending) cache_free(p.dev);
         pending.clear();
         for (auto& e : h2d) if (e) cudaEventDestroy(e);
         if (cs) cudaStreamDestroy(cs);
-        cs = nullptr;
+        if (ds) cudaStreamDestroy(ds);
+        cs = ds = nullptr;
     };
     try {
         for (auto& e : h2d) DTS_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
@@ -336,7 +342,7 @@ dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_
                           ~0ull, dmap ? dmap + a : nullptr, dtraj ? dtraj + a : nullptr, excl);
             if (so.count) {
                 if (used + so.count > cap) {          // grow the pinned output
-                    DTS_CUDA(cudaStreamSynchronize(cs));
+                    DTS_CUDA(cudaStreamSynchronize(ds));
                     const size_t want = std::max(used + so.count,
                                                  (size_t)((double)(used + so.count) *
                                                           (double)nchunks / (double)(i + 1) * 1.2));
@@ -348,7 +354,7 @@ dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_
                     cap = want;
                 }
                 DTS_CUDA(cudaMemcpyAsync(out + used, so.results, so.count * sizeof(dts_result),
-                                         cudaMemcpyDeviceToHost, cs));
+                                         cudaMemcpyDeviceToHost, ds));
                 pending.push_back({so.results, so.count});
                 used += so.count;
             }
@@ -363,6 +369,7 @@ dts_result* search_pipelined(const dts_index* index, const dts_segment* Q, size_
             agg.ms_canon += cs_stats.ms_canon;
         }
         DTS_CUDA(cudaStreamSynchronize(cs));
+        DTS_CUDA(cudaStreamSynchronize(ds));
     } catch (...) {
         cleanup();
         pinned_free(out);

@@ -79,6 +79,21 @@ extern std::atomic<unsigned long long> g_launches;
         DTS_CUDA(cudaGetLastError());                                               \
     } while (0)
 
+// Device-side invariant checks, compiled in only for the checked build
+// (DTS_NVCC_EXTRA=-DDTS_CHECKED, scripts/gpu_checked.sh): a failed check
+// prints its condition and traps, which fails the calling test.
+#ifdef DTS_CHECKED
+#define DTS_DCHECK(c)                                                               \
+    do {                                                                            \
+        if (!(c)) {                                                                 \
+            printf("DTS_DCHECK failed %s:%d: %s\n", __FILE__, __LINE__, #c);       \
+            __trap();                                                               \
+        }                                                                           \
+    } while (0)
+#else
+#define DTS_DCHECK(c) do {} while (0)
+#endif
+
 // Stream-ordered device buffer (pool allocator; freed on scope exit).
 template <typename T>
 struct DevBuf {

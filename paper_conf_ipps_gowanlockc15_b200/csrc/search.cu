@@ -465,7 +465,10 @@ __global__ void __launch_bounds__(PT) k_qscatter(const unsigned long long* __res
 #pragma unroll
     for (int j = 0; j < QS_ITEMS; ++j) {
         const uint32_t i = i0 + (uint32_t)j * PT;
-        if (i < nq) order[base[(uint32_t)(k[j] >> shift) & (nd - 1u)] + r[j]] = (uint32_t)(k[j] & row_mask);
+        if (i < nq) {
+            DTS_DCHECK(base[(uint32_t)(k[j] >> shift) & (nd - 1u)] + r[j] < nq);
+            order[base[(uint32_t)(k[j] >> shift) & (nd - 1u)] + r[j]] = (uint32_t)(k[j] & row_mask);
+        }
     }
 }
 
@@ -942,7 +945,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // pass 2: staged hits gathered into the output
     auto launch_emit = [&](dts_result* dst, unsigned long long cap) {
         k_emit_gather<<<(unsigned)blocks(nq, 256), 256, 0, s>>>(
-            (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, dst, cap);
+            (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, stage_cap, dst, cap);
     };
     // pass 2 launched before the host learns the total, into a buffer sized
     // by this index's previous result count: a repeated search of one index

@@ -432,6 +432,8 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
                     }
                 }
                 const uint32_t slot = (uint32_t)(k & 1023ull);
+                DTS_DCHECK(slot < (uint32_t)WH && rank < S.qcount[q] &&
+                           b + S.qoff[q] + rank < a.stage_cap && b + S.qoff[q] + rank < b + nh);
                 dts_result r;
                 r.query_id = a.qmap ? __ldg(a.qmap + S.qid[q]) : S.qid[q] + a.qid_base;
                 r.entry_id = e;
@@ -451,8 +453,10 @@ __device__ __forceinline__ void tile_finish(WarpSmem& S, const TileArgs& a, int 
     }
     // per query id: where its staged hits start (NONE: spilled or re-run,
     // placed by the spill path), for pass 2's gather
-    if (a.qstage && !a.spill_all && mine && cnt)
+    if (a.qstage && !a.spill_all && mine && cnt) {
+        DTS_DCHECK(S.qid[lane] < a.nq && (sbase == NONE || cnt <= (uint32_t)WH));
         a.qstage[S.qid[lane]] = sbase == NONE ? NONE : sbase + S.qoff[lane];
+    }
 }
 
 // SB: the subbin method (candidates through the X/Y/Z arrays); the grid and
@@ -636,8 +640,10 @@ __global__ void __launch_bounds__(256) k_emit_gather(uint32_t nq,
                                                     const unsigned long long* __restrict__ offsets,
                                                     const unsigned long long* __restrict__ qstage,
                                                     const dts_result* __restrict__ stage,
+                                                    unsigned long long stage_n,
                                                     dts_result* __restrict__ out,
                                                     unsigned long long cap) {
+    (void)stage_n;
     const uint32_t lane = threadIdx.x & 31;
     const uint32_t q0 = (blockIdx.x * 256 + threadIdx.x) & ~31u;
     if (q0 >= nq) return;
@@ -669,6 +675,7 @@ __global__ void __launch_bounds__(256) k_emit_gather(uint32_t nq,
         const unsigned long long os = __shfl_sync(0xffffffffu, o, src);
         const unsigned long long ss = __shfl_sync(0xffffffffu, sp, src);
         const unsigned long long j = os + (k - ex);
+        DTS_DCHECK(k >= total || (k >= ex && ss != NONE && ss + (k - ex) < stage_n));
         if (k < total && j < cap) out[j] = stage[ss + (k - ex)];
     }
 }
@@ -762,6 +769,7 @@ __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restric
     uint32_t base = 0;
     if (lane == leader) base = atomicAdd(&cursor[q], (uint32_t)__popc(grp));
     base = __shfl_sync(grp, base, leader);
+    DTS_DCHECK(offsets[q] + base + (uint32_t)__popc(grp) <= offsets[q + 1]);
     rkeys[offsets[q] + base + __popc(grp & ((1u << lane) - 1u))] =
         ((unsigned long long)e << 32) | (uint32_t)(base_idx + k);
 }

@@ -107,14 +107,15 @@ def test_index_layout_variants_invariant(dts, oracle_mod, monkeypatch):
     """Same result bytes whatever digit plan the build's radix sort takes
     (8-bit only, or 9-bit digits where they save a pass), whichever grid
     source (sampled + fused keys pass, or exact bounds first), hash load,
-    gather shape and pass-1 occupancy the index and search use: they only
-    change the layout and the schedule."""
+    gather shape, pass-1 occupancy, query order and queries per warp tile the
+    index and search use: they only change the layout and the schedule."""
     c = synth.make_config("C1", scale=0.1)
     ref = None
     for env in ({"DTS_RADIX9": "0"}, {"DTS_RADIX9": "1"}, {"DTS_HASH_SLOTS": "1.2"},
                 {"DTS_FUSED_KEYS": "0"}, {"DTS_OS_SHAPE": "0"}, {"DTS_GATHER": "4"},
                 {"DTS_GATHER": "1"}, {"DTS_TILE_OCC": "6"}, {"DTS_TILE_OCC": "8"},
-                {"DTS_QSORT_MIN": "0"}, {"DTS_QSORT_MIN": "0", "DTS_QSORT_DROP": "0"}):
+                {"DTS_QSORT_MIN": "0"}, {"DTS_QSORT_MIN": "0", "DTS_QSORT_DROP": "0"},
+                {"DTS_TILE_FILL": "0"}, {"DTS_TILE_Q": "1"}, {"DTS_TILE_Q": "3"}):
         # the toggles are read once per process: run each in a subprocess
         import subprocess
         import sys
@@ -506,12 +507,16 @@ def test_spill_paths_same_bytes(dts, oracle_mod):
             k += 8 + n
         return parts
     runs = []
-    for env in ({}, {"DTS_SPILL_CAP": "1000"}, {"DTS_SPILL_CAP": "0"}):
+    # (and with 16- and 2-query warp tiles: the tile size sets which hits
+    #  share a stage, so which tiles spill)
+    for env in ({}, {"DTS_SPILL_CAP": "1000"}, {"DTS_SPILL_CAP": "0"},
+                {"DTS_TILE_FILL": "0", "DTS_SPILL_CAP": "1000"},
+                {"DTS_TILE_Q": "2", "DTS_SPILL_CAP": "0"}):
         out = subprocess.run([sys.executable, "-c", code], env={**os.environ, **env},
                              capture_output=True, timeout=900)
         assert out.returncode == 0, out.stderr.decode()[-3000:]
         runs.append(split(out.stdout))
-    assert runs[0] == runs[1] == runs[2]
+    assert all(r == runs[0] for r in runs[1:])
     c = synth.make_config("C2", scale=0.004)
     for k, d in enumerate((2.0, 8.0)):
         got = np.frombuffer(runs[0][k], dtype=dts.RESULT_DTYPE)
