@@ -310,7 +310,7 @@ def run_own(args):
     idx = dts.build_index_device(D_dev, device=local, stream=stream)
     build_info = idx.info()
 
-    def search_step(dd, timed_kernels="defer"):
+    def search_step(dd, timed_kernels="pass1"):
         """One search of the whole query set (this rank's balanced share of
         it at N > 1).  Returns (results, stats, (lo, hi))."""
         if world == 1:
@@ -365,7 +365,14 @@ def run_own(args):
     nq_rank = hi - lo
     st0 = stats[-1]
     mean = lambda k: statistics.mean(s[k] for s in stats)   # noqa: E731
-    ph = {k: mean(k) for k in ("ms_prep", "ms_count", "ms_scan", "ms_scatter", "ms_canon")}
+    # pass 1's duration from its two events in every timed step; the other
+    # phases from a few fully instrumented steps after the timed region (six
+    # timing events per call add ~25 us to a C4 step, two ~8)
+    ph_steps = [o[0] for o in timed(lambda: search_step(d, "defer"), 5, 1)[2]]
+    ph_steps = [dts.read_times(x) for x in ph_steps]
+    ph = {k: statistics.mean(x[k] for x in ph_steps)
+          for k in ("ms_prep", "ms_scan", "ms_scatter", "ms_canon")}
+    ph["ms_count"] = mean("ms_count")
 
     # ---- roofline of the dominant kernel: pass 1 (k_wtile_count)
     peak, peak_src = load_peaks()
@@ -396,7 +403,7 @@ def run_own(args):
     # ---- extra d points of the same workload (fewer steps)
     points = []
     for dp in ([] if args.no_points else POINTS.get(args.config, [])):
-        pms, _, pouts, pres, _ = timed(lambda: search_step(dp), max(3, args.steps // 5), 2)
+        pms, _, pouts, pres, _ = timed(lambda: search_step(dp, "defer"), max(3, args.steps // 5), 2)
         pouts = [(dts.read_times(o[0]), o[1]) for o in pouts]
         pst = pouts[-1][0]
         plo, phi = pouts[-1][1]
@@ -491,7 +498,9 @@ def run_own(args):
                            "replicated" if world > 1 else "one GPU",
             "phases_ms": {"prep": ph["ms_prep"], "count_pass": ph["ms_count"],
                           "scan": ph["ms_scan"], "emit_pass": ph["ms_scatter"],
-                          "overflow_sort": ph["ms_canon"]},
+                          "overflow_sort": ph["ms_canon"],
+                          "note": "count_pass: pass-1 events of every timed step; the rest: "
+                                  "5 fully instrumented steps after the timed region"},
             "step_ms_min_median_max": [min(step_ms), statistics.median(step_ms), max(step_ms)],
             "work": {"candidates": st0["candidates"], "offset_lookups": st0["cell_lookups"],
                      "results": results, "queries_rank0": nq_rank},

@@ -137,7 +137,8 @@ typedef struct {
     uint32_t time_kernels;      /* in: 1 = record CUDA-event phase times below and read
                                    them before returning; 2 = record them only (read
                                    later by dts_search_read_times, so that the call
-                                   returns as soon as its results are ready)          */
+                                   returns as soon as its results are ready); 3 = as 2,
+                                   pass 1 (ms_count) only: two events instead of six */
     float    ms_prep;           /* query keys + sort                                    */
     float    ms_count;          /* pass 1 (fused candidate streaming + refine, count)   */
     float    ms_scan;           /* exclusive scan of per-query counts                   */

@@ -375,10 +375,13 @@ def search(index: Index, Q, d: float, query_id_base: int = 0, stream=None) -> np
 
 def _timing_mode(time_kernels) -> int:
     """time_kernels: False/0 off, True/1 phase times read before the call
-    returns, "defer"/2 recorded only (read later by read_times)."""
+    returns, "defer"/2 recorded only (read later by read_times), "pass1"/3
+    as "defer" for pass 1's two events only."""
     if time_kernels == "defer":
         return 2
-    return int(time_kernels) if time_kernels in (0, 1, 2) else (1 if time_kernels else 0)
+    if time_kernels == "pass1":
+        return 3
+    return int(time_kernels) if time_kernels in (0, 1, 2, 3) else (1 if time_kernels else 0)
 
 
 def read_times(stats: dict) -> dict:

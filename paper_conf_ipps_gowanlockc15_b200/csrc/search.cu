@@ -553,7 +553,7 @@ struct TimerRing {
     cudaEvent_t ev[TIMER_SETS][6];
     bool made[TIMER_SETS] = {false};
     uint32_t next = 0;            // calls so far (slot = next % TIMER_SETS)
-    int k[TIMER_SETS] = {0};      // events recorded per set
+    uint32_t rec[TIMER_SETS] = {0};   // bit j: event j (phase boundary j) recorded
 };
 TimerRing& timer_ring(int dev) {
     static thread_local TimerRing* rings[64] = {nullptr};
@@ -562,18 +562,21 @@ TimerRing& timer_ring(int dev) {
     return *rings[dev];
 }
 
+// mode 1, 2: all six phase boundaries; mode 3: only pass 1's two (a timing
+// event between two kernels costs the stream a few microseconds: six of them
+// add ~25 us to a C4 search, two ~8)
 struct EventTimer {
     bool on;
     cudaStream_t s;
     cudaEvent_t* ev = nullptr;
-    int* k = nullptr;
+    uint32_t* rec = nullptr;
+    uint32_t want = 0x3f, rec0 = 0;
+    int calls = 0;
     uint32_t handle = 0;
-    int k0 = 0;
-    EventTimer(bool enable, cudaStream_t st) : on(enable), s(st) {
-        if (!on) {
-            k = &k0;
-            return;
-        }
+    EventTimer(uint32_t mode, cudaStream_t st) : on(mode != 0), s(st) {
+        rec = &rec0;
+        if (!on) return;
+        if (mode == 3) want = (1u << 1) | (1u << 2);
         int dev = 0;
         DTS_CUDA(cudaGetDevice(&dev));
         TimerRing& r = timer_ring(dev);
@@ -584,13 +587,19 @@ struct EventTimer {
             r.made[i] = true;
         }
         ev = r.ev[i];
-        k = &r.k[i];
-        *k = 0;
+        rec = &r.rec[i];
+        *rec = 0;
     }
-    void mark() { if (on && *k < 6) DTS_CUDA(cudaEventRecord(ev[(*k)++], s)); }
+    void mark() {
+        if (on && calls < 6 && ((want >> calls) & 1u)) {
+            DTS_CUDA(cudaEventRecord(ev[calls], s));
+            *rec |= 1u << calls;
+        }
+        ++calls;
+    }
     float ms(int i) {
         float t = 0.f;
-        if (on && i + 1 < *k) cudaEventElapsedTime(&t, ev[i], ev[i + 1]);
+        if (on && ((*rec >> i) & 3u) == 3u) cudaEventElapsedTime(&t, ev[i], ev[i + 1]);
         return t;
     }
 };
@@ -637,7 +646,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         return;
     }
 
-    EventTimer tm(local.time_kernels != 0, s);
+    EventTimer tm(local.time_kernels, s);
     tm.mark();
     static const int nsm_prep = [] {
         int dev = 0, v = 148;
@@ -972,16 +981,21 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         launch_emit(spec.p, hint);
         DTS_LAUNCH_CHECK();
     }
-    struct {
+    // counters and total read back through a pinned buffer of the calling
+    // thread (a pageable destination adds a staging copy to the call)
+    struct Readback {
         Counters c;
         unsigned long long total;
-    } h;
-    DTS_CUDA(cudaMemcpyAsync(&h.c, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
-    DTS_CUDA(cudaMemcpyAsync(&h.total, offsets.p + nq, sizeof(unsigned long long),
+    };
+    static thread_local Readback* rb = nullptr;
+    if (!rb) DTS_CUDA(cudaMallocHost((void**)&rb, sizeof(Readback)));
+    DTS_CUDA(cudaMemcpyAsync(&rb->c, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
+    DTS_CUDA(cudaMemcpyAsync(&rb->total, offsets.p + nq, sizeof(unsigned long long),
                              cudaMemcpyDeviceToHost, s));
     tr.mark("emit");
     DTS_CUDA(cudaStreamSynchronize(s));
     tr.mark("sync");
+    const Readback h = *rb;
     if (!count_only) idx->result_hint.store(h.total + h.total / 8 + 4096);
     if (h.c.bad & 1) throw Error(DTS_EINVAL, "query segment with a non-finite coordinate or time");
     if (h.c.bad & 2) throw Error(DTS_EINVAL, "query segment with t_end < t_start");
@@ -998,7 +1012,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         out->count = (size_t)h.total;
         tm.mark();
         tm.mark();
-        if (local.time_kernels == 2) {
+        if (local.time_kernels >= 2) {
             local.timer_slot = tm.handle;
         } else if (local.time_kernels) {
             local.ms_prep = tm.ms(0);
@@ -1224,7 +1238,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         tm.mark();
     }
     tr.mark("done");
-    if (local.time_kernels == 2) {
+    if (local.time_kernels >= 2) {
         local.timer_slot = tm.handle;
     } else if (local.time_kernels) {
         DTS_CUDA(cudaStreamSynchronize(s));
@@ -1244,12 +1258,12 @@ void search_read_times(dts_search_stats* st) {
     const uint32_t h = st->timer_slot, i = h % TIMER_SETS;
     if (h >= r.next || r.next - h > TIMER_SETS || !r.made[i])
         throw Error(DTS_EINVAL, "timer slot recycled or not from this thread and device");
-    const int k = r.k[i];
-    if (k > 0) DTS_CUDA(cudaEventSynchronize(r.ev[i][k - 1]));
+    const uint32_t rec = r.rec[i];
+    if (rec) DTS_CUDA(cudaEventSynchronize(r.ev[i][31 - __builtin_clz(rec)]));
     float* out[5] = {&st->ms_prep, &st->ms_count, &st->ms_scan, &st->ms_scatter, &st->ms_canon};
     for (int j = 0; j < 5; ++j) {
         float t = 0.f;
-        if (j + 1 < k) DTS_CUDA(cudaEventElapsedTime(&t, r.ev[i][j], r.ev[i][j + 1]));
+        if (((rec >> j) & 3u) == 3u) DTS_CUDA(cudaEventElapsedTime(&t, r.ev[i][j], r.ev[i][j + 1]));
         *out[j] = t;
     }
 }

@@ -21,7 +21,7 @@ Qd = torch.from_numpy(c.Q).cuda()
 idx = dts.build_index_device(Dd)
 flush = torch.empty(256 << 20, dtype=torch.uint8, device="cuda")
 s = torch.cuda.current_stream()
-for nq, tk in ((len(c.Q), False), (len(c.Q), True), (16, False), (16, True), (1024, False), (65536, False))[: int(os.environ.get("NPTS", "6"))]:
+for nq, tk in ((len(c.Q), False), (len(c.Q), True), (len(c.Q), "defer"), (16, False), (16, True), (16, "defer"), (1024, False), (65536, False))[: int(os.environ.get("NPTS", "8"))]:
     Q = Qd[:nq].contiguous()
     for _ in range(3):
         r, _st = dts.search_device(idx, Q, c.d, stream=s, time_kernels=tk)

@@ -136,6 +136,11 @@ def test_deferred_phase_times(dts):
         t = dts.read_times(st)
         assert t["ms_count"] > 0.0 and t["ms_prep"] > 0.0 and t["ms_scan"] > 0.0
         assert t["candidates"] == st0["candidates"]
+    # pass 1's two events only
+    res, st = dts.search_device(idx, Qd, c.d, time_kernels="pass1")
+    res.free()
+    t = dts.read_times(st)
+    assert t["ms_count"] > 0.0 and t["ms_prep"] == 0.0 and t["ms_scan"] == 0.0
     _, st_off = dts.search_device(idx, Qd, c.d)
     assert st_off["timer_slot"] == 0xFFFFFFFF
     with pytest.raises(dts.DTSError):
