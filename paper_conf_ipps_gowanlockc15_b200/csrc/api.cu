@@ -3,13 +3,18 @@
 // search itself runs in the kernels of build.cu / search.cu / prims.cu.
 #include <cuda_runtime.h>
 
+#include <sys/mman.h>
+
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <cstring>
 #include <map>
 #include <mutex>
 #include <new>
 #include <string>
+#include <thread>
+#include <vector>
 
 #include "internal.cuh"
 
@@ -101,13 +106,76 @@ void* pinned_alloc(size_t bytes) {
     size_t kind = 0;
     if (e != cudaSuccess) {
         cudaGetLastError();
-        b = std::malloc(bytes + HDR);
+        // 2 MiB aligned and backed by transparent huge pages where the
+        // kernel allows: first-touch faults of a 10 GB result array at 4 KiB
+        // granularity cost more than its PCIe transfer
+        if (posix_memalign(&b, size_t(2) << 20, bytes + HDR) != 0) b = nullptr;
         if (!b) throw Error(DTS_ENOMEM, "host allocation failed for the result buffer");
+        madvise(b, bytes + HDR, MADV_HUGEPAGE);
         kind = 1;
     }
     static_cast<size_t*>(b)[0] = bytes;
     static_cast<size_t*>(b)[1] = kind;
     return static_cast<char*>(b) + HDR;
+}
+
+bool is_pageable_block(const void* p) {
+    const void* b = static_cast<const char*>(p) - HDR;
+    return static_cast<const size_t*>(b)[1] == 1;
+}
+
+// Device -> host copy of `bytes` into (part of) a result block of
+// pinned_alloc (`pageable`: is_pageable_block of that block).  A pinned
+// block takes one cudaMemcpyAsync; a pageable one (outputs over
+// 1 GB) is staged through two pinned 64 MiB buffers of the calling thread:
+// the DMA of chunk i runs while host threads copy chunk i-1 out (and take
+// the destination's first-touch page faults in parallel) -- a single
+// driver-staged copy into pageable memory runs at the speed of one core.
+void copy_results_d2h(void* dst, const void* src, size_t bytes, cudaStream_t s, bool pageable) {
+    if (!bytes) return;
+    if (!pageable || bytes < (size_t(256) << 20)) {
+        DTS_CUDA(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaStreamSynchronize(s));
+        return;
+    }
+    constexpr size_t CH = size_t(64) << 20;
+    struct Stage {
+        void* buf[2] = {nullptr, nullptr};
+        cudaEvent_t ev[2] = {nullptr, nullptr};
+    };
+    static thread_local Stage st;
+    if (!st.buf[0]) {
+        for (int i = 0; i < 2; ++i) {
+            DTS_CUDA(cudaMallocHost(&st.buf[i], CH));
+            DTS_CUDA(cudaEventCreateWithFlags(&st.ev[i], cudaEventDisableTiming));
+        }
+    }
+    const unsigned hw = std::max(1u, std::thread::hardware_concurrency());
+    const unsigned nt = std::min(8u, hw);
+    auto host_copy = [&](char* d, const char* p, size_t n) {
+        std::vector<std::thread> th;
+        const size_t per = (n + nt - 1) / nt;
+        for (unsigned t = 1; t < nt; ++t) {
+            const size_t a = std::min(n, t * per), b = std::min(n, a + per);
+            if (a < b) th.emplace_back([=] { std::memcpy(d + a, p + a, b - a); });
+        }
+        std::memcpy(d, p, std::min(n, per));
+        for (auto& x : th) x.join();
+    };
+    const size_t nch = (bytes + CH - 1) / CH;
+    for (size_t i = 0; i <= nch; ++i) {
+        if (i < nch) {
+            const size_t off = i * CH, n = std::min(CH, bytes - off);
+            DTS_CUDA(cudaMemcpyAsync(st.buf[i & 1], static_cast<const char*>(src) + off, n,
+                                     cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaEventRecord(st.ev[i & 1], s));
+        }
+        if (i > 0) {
+            const size_t j = i - 1, off = j * CH, n = std::min(CH, bytes - off);
+            DTS_CUDA(cudaEventSynchronize(st.ev[j & 1]));
+            host_copy(static_cast<char*>(dst) + off, static_cast<const char*>(st.buf[j & 1]), n);
+        }
+    }
 }
 
 void pinned_free(void* p) {
@@ -261,9 +329,8 @@ dts_result* search_streamed(const dts_index* index, const dts_segment* dQ, size_
                 throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
             }
             if (so.count) {
-                DTS_CUDA(cudaMemcpyAsync(h + off, so.results, so.count * sizeof(dts_result),
-                                         cudaMemcpyDeviceToHost, s));
-                DTS_CUDA(cudaStreamSynchronize(s));
+                copy_results_d2h(h + off, so.results, so.count * sizeof(dts_result), s,
+                                 is_pageable_block(h));
                 cache_free(so.results);
             }
             off += so.count;
@@ -464,9 +531,8 @@ dts_status search_common(const dts_index* index, const dts_segment* Q, size_t nq
                 dts_result* h = nullptr;
                 try {
                     h = static_cast<dts_result*>(pinned_alloc(so.count * sizeof(dts_result)));
-                    DTS_CUDA(cudaMemcpyAsync(h, so.results, so.count * sizeof(dts_result),
-                                             cudaMemcpyDeviceToHost, s));
-                    DTS_CUDA(cudaStreamSynchronize(s));
+                    copy_results_d2h(h, so.results, so.count * sizeof(dts_result), s,
+                                     is_pageable_block(h));
                 } catch (...) {
                     pinned_free(h);
                     cudaStreamSynchronize(s);

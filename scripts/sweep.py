@@ -27,6 +27,8 @@ PAPER_V = {"S1": 4, "S2": 16, "S3": 4, "C1": 16, "C4": 16, "C2": 4, "C3": 4}
 
 
 def timed_search(idx, Qd, d, reps):
+    """Median device time of uninstrumented searches; the phase times come
+    from one more, instrumented, search."""
     s = torch.cuda.current_stream()
     res, st = dts.search_device(idx, Qd, d, stream=s, time_kernels=True)
     res.free()
@@ -35,7 +37,7 @@ def timed_search(idx, Qd, d, reps):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(s)
-        res, st = dts.search_device(idx, Qd, d, stream=s, time_kernels=True)
+        res, _ = dts.search_device(idx, Qd, d, stream=s)
         e1.record(s)
         torch.cuda.synchronize()
         ts.append(e0.elapsed_time(e1))
