@@ -13,6 +13,8 @@
 #include <mutex>
 #include <new>
 #include <string>
+#include <condition_variable>
+#include <exception>
 #include <thread>
 #include <vector>
 
@@ -142,6 +144,12 @@ void copy_results_d2h(void* dst, const void* src, size_t bytes, cudaStream_t s, 
     struct Stage {
         void* buf[2] = {nullptr, nullptr};
         cudaEvent_t ev[2] = {nullptr, nullptr};
+        ~Stage() {                                // thread exit (stream workers)
+            for (int i = 0; i < 2; ++i) {
+                if (buf[i]) cudaFreeHost(buf[i]);
+                if (ev[i]) cudaEventDestroy(ev[i]);
+            }
+        }
     };
     static thread_local Stage st;
     if (!st.buf[0]) {
@@ -636,39 +644,104 @@ void stream_common(const dts_index* index, const dts_segment* Q, size_t nq, doub
             a = b;
         }
     }
-    dts_result* hbuf = nullptr;
-    if (biggest) hbuf = static_cast<dts_result*>(pinned_alloc(biggest * sizeof(dts_result)));
-    dts_search_stats agg = cst;
-    agg.results = 0;
-    try {
+    // chunks of contiguous query ids (canonical order = chunk order)
+    struct Chunk {
+        size_t a, b;
+        uint64_t n;
+    };
+    std::vector<Chunk> chunks;
+    {
         size_t a = 0;
         while (a < nq) {
             size_t b = a;
             uint64_t acc = 0;
             while (b < nq && (b == a || acc + counts[b] <= chunk_results)) acc += counts[b++];
-            if (acc) {
-                SearchOut co;
-                search_device(index, dQ.p + a, b - a, d, qid_base + (uint32_t)a, s, &co, nullptr,
-                              ~0ull, dmap.p ? dmap.p + a : nullptr, dtraj.p ? dtraj.p + a : nullptr,
-                              excl);
-                if (co.count != acc) {
-                    cache_free(co.results);
-                    throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
-                }
-                DTS_CUDA(cudaMemcpyAsync(hbuf, co.results, acc * sizeof(dts_result),
-                                         cudaMemcpyDeviceToHost, s));
-                DTS_CUDA(cudaStreamSynchronize(s));
-                cache_free(co.results);
-                agg.results += acc;
-                if (cb(hbuf, (size_t)acc, user) != 0) break;      // the caller stops early
-            }
+            if (acc) chunks.push_back({a, b, acc});
             a = b;
         }
+    }
+    // two landing buffers: a worker thread searches chunk k + 1 and copies it
+    // out while the caller's callback consumes chunk k
+    dts_result* hbuf[2] = {nullptr, nullptr};
+    dts_search_stats agg = cst;
+    agg.results = 0;
+    int dev = 0;
+    DTS_CUDA(cudaGetDevice(&dev));
+    std::mutex mu;
+    std::condition_variable cv;
+    size_t produced = 0, consumed = 0;
+    bool stop = false;
+    std::exception_ptr err;
+    std::thread worker;
+    try {
+        for (int i = 0; i < 2 && (size_t)i < chunks.size(); ++i)
+            hbuf[i] = static_cast<dts_result*>(pinned_alloc(biggest * sizeof(dts_result)));
+        worker = std::thread([&] {
+            try {
+                DTS_CUDA(cudaSetDevice(dev));
+                for (size_t k = 0; k < chunks.size(); ++k) {
+                    {
+                        std::unique_lock<std::mutex> lk(mu);
+                        cv.wait(lk, [&] { return stop || k < consumed + 2; });
+                        if (stop) return;
+                    }
+                    const Chunk& c = chunks[k];
+                    SearchOut co;
+                    search_device(index, dQ.p + c.a, c.b - c.a, d, qid_base + (uint32_t)c.a, s,
+                                  &co, nullptr, ~0ull, dmap.p ? dmap.p + c.a : nullptr,
+                                  dtraj.p ? dtraj.p + c.a : nullptr, excl);
+                    if (co.count != c.n) {
+                        cache_free(co.results);
+                        throw Error(DTS_EINTERNAL, "streamed chunk count mismatch");
+                    }
+                    copy_results_d2h(hbuf[k & 1], co.results, c.n * sizeof(dts_result), s,
+                                     is_pageable_block(hbuf[k & 1]));
+                    cache_free(co.results);
+                    std::lock_guard<std::mutex> lk(mu);
+                    produced = k + 1;
+                    cv.notify_all();
+                }
+            } catch (...) {
+                std::lock_guard<std::mutex> lk(mu);
+                err = std::current_exception();
+                stop = true;
+                cv.notify_all();
+            }
+        });
+        for (size_t k = 0; k < chunks.size(); ++k) {
+            {
+                std::unique_lock<std::mutex> lk(mu);
+                cv.wait(lk, [&] { return stop || produced > k; });
+                if (produced <= k) break;                // the worker failed
+            }
+            agg.results += chunks[k].n;
+            const bool more = cb(hbuf[k & 1], (size_t)chunks[k].n, user) == 0;
+            std::lock_guard<std::mutex> lk(mu);
+            consumed = k + 1;
+            if (!more) stop = true;                      // the caller stops early
+            cv.notify_all();
+            if (!more) break;
+        }
+        {
+            std::lock_guard<std::mutex> lk(mu);
+            stop = true;
+            cv.notify_all();
+        }
+        worker.join();
     } catch (...) {
-        pinned_free(hbuf);
+        {
+            std::lock_guard<std::mutex> lk(mu);
+            stop = true;
+            cv.notify_all();
+        }
+        if (worker.joinable()) worker.join();
+        pinned_free(hbuf[0]);
+        pinned_free(hbuf[1]);
         throw;
     }
-    pinned_free(hbuf);
+    pinned_free(hbuf[0]);
+    pinned_free(hbuf[1]);
+    if (err) std::rethrow_exception(err);
     if (stats) *stats = agg;
 }
 

@@ -987,8 +987,13 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         Counters c;
         unsigned long long total;
     };
-    static thread_local Readback* rb = nullptr;
-    if (!rb) DTS_CUDA(cudaMallocHost((void**)&rb, sizeof(Readback)));
+    struct RbHolder {
+        Readback* p = nullptr;
+        ~RbHolder() { if (p) cudaFreeHost(p); }   // thread exit (stream workers)
+    };
+    static thread_local RbHolder rbh;
+    if (!rbh.p) DTS_CUDA(cudaMallocHost((void**)&rbh.p, sizeof(Readback)));
+    Readback* rb = rbh.p;
     DTS_CUDA(cudaMemcpyAsync(&rb->c, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
     DTS_CUDA(cudaMemcpyAsync(&rb->total, offsets.p + nq, sizeof(unsigned long long),
                              cudaMemcpyDeviceToHost, s));
