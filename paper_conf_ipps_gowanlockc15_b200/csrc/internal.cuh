@@ -364,7 +364,7 @@ __host__ __device__ inline double from_ordered_bits(unsigned long long u) {
 // Exclusive scan of n values; out has n + 1 entries, out[n] = total.
 void scan_exclusive_u32_to_u32(const uint32_t* in, uint32_t* out, size_t n, cudaStream_t s);
 void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size_t n,
-                               cudaStream_t s);
+                               cudaStream_t s, unsigned long long* total_out = nullptr);
 
 // Stable LSD radix sort of (key, value) pairs on key bits [0, nbits).
 // Sorts in place from the caller's view: on return keys/vals hold the result.

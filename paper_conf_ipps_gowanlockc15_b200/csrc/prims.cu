@@ -76,7 +76,8 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_reduce(const Tin* __restr
 template <typename Tin, typename Tout>
 __global__ void __launch_bounds__(SCAN_THREADS) k_scan_down(const Tin* __restrict__ in, size_t n,
                                                             const Tout* __restrict__ prefix,
-                                                            Tout* __restrict__ out) {
+                                                            Tout* __restrict__ out,
+                                                            Tout* __restrict__ total_out) {
     size_t base = (size_t)blockIdx.x * SCAN_TILE + (size_t)threadIdx.x * SCAN_ITEMS;
     Tout v[SCAN_ITEMS];
     Tout s = 0;
@@ -96,24 +97,31 @@ __global__ void __launch_bounds__(SCAN_THREADS) k_scan_down(const Tin* __restric
         if (idx < n) out[idx] = run;
         run += v[i];
     }
-    if (prefix == nullptr && threadIdx.x == 0) out[n] = total;
-    if (prefix != nullptr && blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+    if (prefix == nullptr && threadIdx.x == 0) {
+        out[n] = total;
+        if (total_out) *total_out = total;
+    }
+    if (prefix != nullptr && blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
         out[n] = prefix[gridDim.x];
+        if (total_out) *total_out = prefix[gridDim.x];
+    }
 }
 
 template <typename Tin, typename Tout>
-void scan_exclusive(const Tin* in, Tout* out, size_t n, cudaStream_t s) {
+void scan_exclusive(const Tin* in, Tout* out, size_t n, cudaStream_t s, Tout* total_out = nullptr) {
     if (n <= (size_t)SCAN_TILE) {
-        k_scan_down<Tin, Tout><<<1, SCAN_THREADS, 0, s>>>(in, n, nullptr, out);
+        k_scan_down<Tin, Tout><<<1, SCAN_THREADS, 0, s>>>(in, n, nullptr, out, total_out);
         DTS_LAUNCH_CHECK();
         return;
     }
     size_t nb = (n + SCAN_TILE - 1) / SCAN_TILE;
-    DevBuf<Tout> sums(nb, s), pre(nb + 1, s);
-    k_scan_reduce<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, sums.p);
+    DevBuf<Tout> sp(2 * nb + 1, s);                  // block sums, then their scan
+    Tout* const sums = sp.p;
+    Tout* const pre = sp.p + nb;
+    k_scan_reduce<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, sums);
     DTS_LAUNCH_CHECK();
-    scan_exclusive<Tout, Tout>(sums.p, pre.p, nb, s);
-    k_scan_down<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, pre.p, out);
+    scan_exclusive<Tout, Tout>(sums, pre, nb, s);
+    k_scan_down<Tin, Tout><<<(unsigned)nb, SCAN_THREADS, 0, s>>>(in, n, pre, out, total_out);
     DTS_LAUNCH_CHECK();
 }
 }  // namespace
@@ -122,8 +130,8 @@ void scan_exclusive_u32_to_u32(const uint32_t* in, uint32_t* out, size_t n, cuda
     scan_exclusive<uint32_t, uint32_t>(in, out, n, s);
 }
 void scan_exclusive_u32_to_u64(const uint32_t* in, unsigned long long* out, size_t n,
-                               cudaStream_t s) {
-    scan_exclusive<uint32_t, unsigned long long>(in, out, n, s);
+                               cudaStream_t s, unsigned long long* total_out) {
+    scan_exclusive<uint32_t, unsigned long long>(in, out, n, s, total_out);
 }
 // ============================================================== radix sort
 namespace {

@@ -59,6 +59,7 @@ struct Counters {                       // device-side statistics / flags
     unsigned int n_skew;                // ... whose ids cluster (radix sort)
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
+    unsigned long long total;           // results (the scan's total, read back with the rest)
 };
 
 // Query in the velocity form used by the refinement.
@@ -354,6 +355,7 @@ __global__ void __launch_bounds__(PT, 4) k_qkeys(const double4* __restrict__ Q, 
                                              Counters* __restrict__ ctr, const PassPlan plan,
                                              uint32_t* __restrict__ hist) {
     __shared__ uint32_t h[OS_MAXPASS * OS_HSTRIDE];
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctr->spill_valid = ~0ull;   // counters zeroed before
     if (hist) {
         for (int j = threadIdx.x; j < plan.npass * OS_HSTRIDE; j += PT) h[j] = 0;
         __syncthreads();
@@ -627,15 +629,21 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         return;
     }
     const double4* Q = reinterpret_cast<const double4*>(Q_dev);
-    DevBuf<Counters> ctr(1, s);
-    DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
+    // the counters and the query sort's digit counts in one buffer, zeroed by
+    // one memset (spill_valid is set to ~0 by k_qkeys)
+    constexpr size_t CTR_BYTES = (sizeof(Counters) + 255) / 256 * 256;
+    constexpr size_t HIST_N = (size_t)OS_MAXPASS * OS_HSTRIDE;
+    DevBuf<unsigned char> small(CTR_BYTES + HIST_N * sizeof(uint32_t), s);
+    Counters* const ctr_p = reinterpret_cast<Counters*>(small.p);
+    uint32_t* const hist_p = reinterpret_cast<uint32_t*>(small.p + CTR_BYTES);
+    DTS_CUDA(cudaMemsetAsync(small.p, 0, small.n, s));
     tr.mark("ctr");
 
     if (idx->n == 0) {   // empty index: validate only
-        k_validate_only<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, ctr.p);
+        k_validate_only<<<blocks(nq, PT), PT, 0, s>>>(Q, (uint32_t)nq, ctr_p);
         DTS_LAUNCH_CHECK();
         Counters hc;
-        DTS_CUDA(cudaMemcpyAsync(&hc, ctr.p, sizeof(hc), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaMemcpyAsync(&hc, ctr_p, sizeof(hc), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         if (hc.bad) throw Error(DTS_EINVAL, "invalid query segment (non-finite or t_end < t_start)");
         if (count_only && counts_out) {
@@ -661,7 +669,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         work *= std::floor(2.0 * (d + idx->gp.half_ext[a]) / idx->gp.w[a]) + 2.0;
     work *= std::floor(idx->gp.maxdur / idx->gp.b) + 2.0;
     // ---- query prep: key + sort
-    DevBuf<uint32_t> order(nq, s);
+    // query keys (and the multi-pass sort's second key buffer) and the order
+    // in one allocation
+    DevBuf<unsigned char> prepbuf(nq * (2 * sizeof(unsigned long long) + sizeof(uint32_t)), s);
+    uint32_t* const order_p =
+        reinterpret_cast<uint32_t*>(prepbuf.p + nq * 2 * sizeof(unsigned long long));
     {
         // packed (key << row bits | row) keys-only sort when it fits 64 bits
         const int row_bits = std::max(1, bits_for(nq - 1));
@@ -715,34 +727,33 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         const PassPlan plan = fused ? plan_passes(lo, row_bits + idx->key_bits, true)
                                     : (one_pass ? PassPlan{1, {lo}, {row_bits + idx->key_bits - lo}}
                                                 : PassPlan{});
-        DevBuf<unsigned long long> qk(nq, s), qk_tmp(sort_q && !one_pass ? nq : 0, s);
-        // (one_pass: the digit counts, then the per-digit cursors)
-        DevBuf<uint32_t> hist(fused ? (size_t)plan.npass * OS_HSTRIDE : (one_pass ? 2 * OS_HSTRIDE : 0), s);
-        if (fused || one_pass)
-            DTS_CUDA(cudaMemsetAsync(hist.p, 0, hist.n * 4, s));
+        unsigned long long* const qk_p = reinterpret_cast<unsigned long long*>(prepbuf.p);
+        unsigned long long* const qk_tmp_p = qk_p + nq;
+        // (hist_p: the digit counts, zeroed with the counters; one_pass: the
+        //  digit counts, then the per-digit cursors)
         k_qkeys<<<(unsigned)std::min<size_t>(blocks(nq, PT), (size_t)nsm_prep * 4), PT, 0, s>>>(
-            Q, (uint32_t)nq, idx->gp, qk.p, (packed && sort_q) ? nullptr : order.p, row_bits,
-            ctr.p, plan, (fused || one_pass) ? hist.p : nullptr);
+            Q, (uint32_t)nq, idx->gp, qk_p, (packed && sort_q) ? nullptr : order_p, row_bits,
+            ctr_p, plan, (fused || one_pass) ? hist_p : nullptr);
         DTS_LAUNCH_CHECK();
         if (one_pass) {
             k_qscatter<<<blocks(nq, PT * QS_ITEMS), PT, 0, s>>>(
-                qk.p, (uint32_t)nq, plan.shift[0], plan.bits[0], hist.p, hist.p + OS_HSTRIDE,
-                (1ull << row_bits) - 1ull, order.p);
+                qk_p, (uint32_t)nq, plan.shift[0], plan.bits[0], hist_p, hist_p + OS_HSTRIDE,
+                (1ull << row_bits) - 1ull, order_p);
             DTS_LAUNCH_CHECK();
         } else if (!sort_q) {
             // order = identity (written by k_qkeys)
         } else if (fused) {
-            radix_sort_keys_hist(qk.p, qk_tmp.p, nq, plan, hist.p, s, order.p,
+            radix_sort_keys_hist(qk_p, qk_tmp_p, nq, plan, hist_p, s, order_p,
                                  (1ull << row_bits) - 1ull);
         } else if (packed) {
             const unsigned long long* sorted =
-                radix_sort_keys(qk.p, qk_tmp.p, nq, lo, row_bits + idx->key_bits, s);
+                radix_sort_keys(qk_p, qk_tmp_p, nq, lo, row_bits + idx->key_bits, s);
             k_unpack_order<<<blocks(nq, PT), PT, 0, s>>>(sorted, (uint32_t)nq,
-                                                        (1ull << row_bits) - 1ull, order.p);
+                                                        (1ull << row_bits) - 1ull, order_p);
             DTS_LAUNCH_CHECK();
         } else {
             DevBuf<uint32_t> order_tmp(nq, s);
-            radix_sort_pairs(qk.p, order.p, qk_tmp.p, order_tmp.p, nq, idx->key_bits, s);
+            radix_sort_pairs(qk_p, order_p, qk_tmp_p, order_tmp.p, nq, idx->key_bits, s);
         }
     }
     // the build may still run (dts_build_index_device returns once its last
@@ -805,15 +816,29 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     unsigned long long spill_cap = spill_env >= 0 ? (unsigned long long)spill_env
         : std::max<unsigned long long>(8ull * nq + (1ull << 20),
                                        idx->spill_hint.load(std::memory_order_relaxed));
-    DevBuf<uint32_t> counts(nq, s), over_tiles(ntiles, s), spill_tiles(ntiles, s);
-    DevBuf<unsigned long long> offsets(nq + 1, s), tile_base(ntiles, s),
-        qstage(count_only ? 0 : nq, s);
+    // pass-1 bookkeeping in one allocation (256-byte aligned pieces)
+    size_t p1_bytes = 0;
+    auto piece = [&](size_t bytes) {
+        const size_t o = p1_bytes;
+        p1_bytes += (bytes + 255) / 256 * 256;
+        return o;
+    };
+    const size_t o_counts = piece(nq * 4), o_over = piece((size_t)ntiles * 4),
+                 o_stiles = piece((size_t)ntiles * 4), o_off = piece((nq + 1) * 8),
+                 o_tbase = piece((size_t)ntiles * 8), o_qstage = piece(count_only ? 0 : nq * 8);
+    DevBuf<unsigned char> p1buf(p1_bytes, s);
+    uint32_t* const counts_p = reinterpret_cast<uint32_t*>(p1buf.p + o_counts);
+    uint32_t* const over_tiles_p = reinterpret_cast<uint32_t*>(p1buf.p + o_over);
+    uint32_t* const spill_tiles_p = reinterpret_cast<uint32_t*>(p1buf.p + o_stiles);
+    unsigned long long* const offsets_p = reinterpret_cast<unsigned long long*>(p1buf.p + o_off);
+    unsigned long long* const tile_base_p = reinterpret_cast<unsigned long long*>(p1buf.p + o_tbase);
+    unsigned long long* const qstage_p =
+        count_only ? nullptr : reinterpret_cast<unsigned long long*>(p1buf.p + o_qstage);
     DevBuf<dts_result> stage(stage_cap, s), spill(std::max<unsigned long long>(spill_cap, 1), s);
-    DTS_CUDA(cudaMemsetAsync(&ctr.p->spill_valid, 0xFF, sizeof(unsigned long long), s));
     tr.mark("bufs");
     TileArgs ta{};
     ta.Q = Q;
-    ta.order = order.p;
+    ta.order = order_p;
     ta.nq = (uint32_t)nq;
     ta.d = d;
     ta.g = idx->gp;
@@ -822,12 +847,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.bin_t0min = idx->bin_t0min;
     ta.bin_t1max = idx->bin_t1max;
     ta.bin_start = idx->bin_start;
-    ta.counts = counts.p;
+    ta.counts = counts_p;
     ta.stage = stage.p;
     ta.stage_cap = stage_cap;
-    ta.tile_base = tile_base.p;
-    ta.over_tiles = over_tiles.p;
-    ta.spill_tiles = spill_tiles.p;
+    ta.tile_base = tile_base_p;
+    ta.over_tiles = over_tiles_p;
+    ta.spill_tiles = spill_tiles_p;
     ta.spill = spill.p;
     ta.spill_cap = spill_cap;
     ta.tile_list = nullptr;
@@ -842,11 +867,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     if (exclude_same_traj && !(qtraj && idx->etraj))
         throw Error(DTS_EINVAL, "exclude_same_trajectory needs query_traj and an index built "
                                 "with entry_traj");
-    ta.ctr = ctr.p;
+    ta.ctr = ctr_p;
     ta.method = idx->method;
     ta.sb = idx->sb;
     ta.out = idx->out;
-    ta.qstage = count_only ? nullptr : qstage.p;
+    ta.qstage = count_only ? nullptr : qstage_p;
     ta.tq = tq;
     local.tile_queries = tq;
     local.work_estimate = (float)work;
@@ -905,12 +930,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         //      sends pass 1 round again, the overflowed buffer sized by the
         //      sum of the counts (an upper bound of what it must hold).
         Counters c1;
-        DTS_CUDA(cudaMemcpyAsync(&c1, ctr.p, sizeof(c1), cudaMemcpyDeviceToHost, s));
+        DTS_CUDA(cudaMemcpyAsync(&c1, ctr_p, sizeof(c1), cudaMemcpyDeviceToHost, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         if (c1.n_over) {
-            scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
+            scan_exclusive_u32_to_u64(counts_p, offsets_p, nq, s);
             unsigned long long bound = 0;
-            DTS_CUDA(cudaMemcpyAsync(&bound, offsets.p + nq, sizeof(bound),
+            DTS_CUDA(cudaMemcpyAsync(&bound, offsets_p + nq, sizeof(bound),
                                      cudaMemcpyDeviceToHost, s));
             DTS_CUDA(cudaStreamSynchronize(s));
             if (c1.staged > stage_cap) {
@@ -927,10 +952,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 unsigned long long want = bound + (1ull << 20), cur = idx->spill_hint.load();
                 while (cur < want && !idx->spill_hint.compare_exchange_weak(cur, want)) {}
             }
-            DTS_CUDA(cudaMemsetAsync(ctr.p, 0, sizeof(Counters), s));
-            DTS_CUDA(cudaMemsetAsync(&ctr.p->spill_valid, 0xFF, sizeof(unsigned long long), s));
+            DTS_CUDA(cudaMemsetAsync(ctr_p, 0, sizeof(Counters), s));
+            DTS_CUDA(cudaMemsetAsync(&ctr_p->spill_valid, 0xFF, sizeof(unsigned long long), s));
             launch_pass1(ta, ntiles);
-            DTS_CUDA(cudaMemcpyAsync(&c1, ctr.p, sizeof(c1), cudaMemcpyDeviceToHost, s));
+            DTS_CUDA(cudaMemcpyAsync(&c1, ctr_p, sizeof(c1), cudaMemcpyDeviceToHost, s));
             DTS_CUDA(cudaStreamSynchronize(s));
             if (c1.n_over) throw Error(DTS_EINTERNAL, "pass 1 overflowed buffers sized by its counts");
         }
@@ -942,19 +967,19 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         }
         if (c1.n_spill) {
             k_spill_max<<<blocks((size_t)c1.n_spill * tq, 128), 128, 0, s>>>(
-                spill_tiles.p, c1.n_spill, tq, order.p, (uint32_t)nq, counts.p, ctr.p);
+                spill_tiles_p, c1.n_spill, tq, order_p, (uint32_t)nq, counts_p, ctr_p);
             DTS_LAUNCH_CHECK();
         }
     }
     tm.mark();
-    scan_exclusive_u32_to_u64(counts.p, offsets.p, nq, s);
+    scan_exclusive_u32_to_u64(counts_p, offsets_p, nq, s, &ctr_p->total);
     tm.mark();
     tr.mark("scan");
 
     // pass 2: staged hits gathered into the output
     auto launch_emit = [&](dts_result* dst, unsigned long long cap) {
         k_emit_gather<<<(unsigned)blocks(nq, 256), 256, 0, s>>>(
-            (uint32_t)nq, counts.p, offsets.p, qstage.p, stage.p, stage_cap, dst, cap);
+            (uint32_t)nq, counts_p, offsets_p, qstage_p, stage.p, stage_cap, dst, cap);
     };
     // pass 2 launched before the host learns the total, into a buffer sized
     // by this index's previous result count: a repeated search of one index
@@ -994,13 +1019,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     static thread_local RbHolder rbh;
     if (!rbh.p) DTS_CUDA(cudaMallocHost((void**)&rbh.p, sizeof(Readback)));
     Readback* rb = rbh.p;
-    DTS_CUDA(cudaMemcpyAsync(&rb->c, ctr.p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
-    DTS_CUDA(cudaMemcpyAsync(&rb->total, offsets.p + nq, sizeof(unsigned long long),
-                             cudaMemcpyDeviceToHost, s));
+    DTS_CUDA(cudaMemcpyAsync(&rb->c, ctr_p, sizeof(Counters), cudaMemcpyDeviceToHost, s));
     tr.mark("emit");
     DTS_CUDA(cudaStreamSynchronize(s));
     tr.mark("sync");
-    const Readback h = *rb;
+    Readback h = *rb;
+    h.total = h.c.total;
     if (!count_only) idx->result_hint.store(h.total + h.total / 8 + 4096);
     if (h.c.bad & 1) throw Error(DTS_EINVAL, "query segment with a non-finite coordinate or time");
     if (h.c.bad & 2) throw Error(DTS_EINVAL, "query segment with t_end < t_start");
@@ -1011,7 +1035,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     local.max_results_per_query = h.c.max_count;
     if (count_only) {                   // counts and total only (dts_search_count)
         if (counts_out && nq)
-            DTS_CUDA(cudaMemcpyAsync(counts_out, counts.p, nq * sizeof(uint32_t),
+            DTS_CUDA(cudaMemcpyAsync(counts_out, counts_p, nq * sizeof(uint32_t),
                                      cudaMemcpyDefault, s));
         DTS_CUDA(cudaStreamSynchronize(s));
         out->count = (size_t)h.total;
@@ -1051,7 +1075,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         if ((double)h.total * per > 0.8 * (double)free_b || h.total > max_results) {
             ResultsTooLarge e(h.total);
             e.counts.resize(nq);
-            DTS_CUDA(cudaMemcpyAsync(e.counts.data(), counts.p, nq * sizeof(uint32_t),
+            DTS_CUDA(cudaMemcpyAsync(e.counts.data(), counts_p, nq * sizeof(uint32_t),
                                      cudaMemcpyDeviceToHost, s));
             DTS_CUDA(cudaStreamSynchronize(s));
             throw e;
@@ -1091,8 +1115,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     //      into a buffer of exactly their result count
                     DevBuf<unsigned long long> cover_off(nq + 1, s);
                     DTS_CUDA(cudaMemsetAsync(cover.p, 0, nq * sizeof(uint32_t), s));
-                    k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles.p, tq, order.p, (uint32_t)nq,
-                                                          counts.p, cover.p);
+                    k_mark_over<<<h.c.n_over, PT, 0, s>>>(over_tiles_p, tq, order_p, (uint32_t)nq,
+                                                          counts_p, cover.p);
                     DTS_LAUNCH_CHECK();
                     scan_exclusive_u32_to_u64(cover.p, cover_off.p, nq, s);
                     DTS_CUDA(cudaMemcpyAsync(&n_raw, cover_off.p + nq, sizeof(n_raw),
@@ -1106,7 +1130,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                     tb.ctr = ctr2.p;
                     tb.spill = spill2.p;
                     tb.spill_cap = n_raw;
-                    tb.tile_list = over_tiles.p;
+                    tb.tile_list = over_tiles_p;
                     tb.n_list = h.c.n_over;
                     tb.spill_all = 1;
                     launch_pass1(tb, h.c.n_over);
@@ -1124,37 +1148,37 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 const SpillSrc src{spill.p, n1, spill2.p};
                 if (n1) {
                     k_spill_place<<<blocks(n1, 256), 256, 0, s>>>(
-                        spill.p, n1, 0u, h.c.n_over ? cover.p : nullptr, offsets.p, cursor.p,
+                        spill.p, n1, 0u, h.c.n_over ? cover.p : nullptr, offsets_p, cursor.p,
                         rkeys.p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (n_raw) {
                     k_spill_place<<<blocks(n_raw, 256), 256, 0, s>>>(
-                        spill2.p, n_raw, (uint32_t)n1, nullptr, offsets.p, cursor.p, rkeys.p);
+                        spill2.p, n_raw, (uint32_t)n1, nullptr, offsets_p, cursor.p, rkeys.p);
                     DTS_LAUNCH_CHECK();
                 }
                 DevBuf<uint32_t> bigc(nq, s);
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
-                DTS_CUDA(cudaMemsetAsync(&ctr.p->n_big, 0, 5 * sizeof(unsigned int), s));
+                DTS_CUDA(cudaMemsetAsync(&ctr_p->n_big, 0, 5 * sizeof(unsigned int), s));
                 const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * tq;
                 DevBuf<uint32_t> lists(3 * nslots, s);
                 const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * tq, 4), 128, 0, s>>>(
-                        spill_tiles.p, h.c.n_spill * tq, tq, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
-                        ctr.p);
+                        spill_tiles_p, h.c.n_spill * tq, tq, order_p, (uint32_t)nq, counts_p,
+                        offsets_p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
+                        ctr_p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (h.c.n_over) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_over * tq, 4), 128, 0, s>>>(
-                        over_tiles.p, h.c.n_over * tq, tq, order.p, (uint32_t)nq, counts.p,
-                        offsets.p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
-                        ctr.p);
+                        over_tiles_p, h.c.n_over * tq, tq, order_p, (uint32_t)nq, counts_p,
+                        offsets_p, rkeys.p, src, qmap, qid_base, eb, fin, lists.p, nslots, bigc.p,
+                        ctr_p);
                     DTS_LAUNCH_CHECK();
                 }
                 unsigned int nbm[5] = {0, 0, 0, 0, 0};   // n_big, n_cls[3], n_skew
-                DTS_CUDA(cudaMemcpyAsync(nbm, &ctr.p->n_big, sizeof(nbm),
+                DTS_CUDA(cudaMemcpyAsync(nbm, &ctr_p->n_big, sizeof(nbm),
                                          cudaMemcpyDeviceToHost, s));
                 DTS_CUDA(cudaStreamSynchronize(s));
                 static const bool smem_ok = [] {
@@ -1175,31 +1199,31 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 DevBuf<uint32_t> skew_list(nbm[1] + nbm[2] + nbm[3], s);
                 if (nbm[1]) {
                     k_seg_bucket<512, 8, 2><<<nbm[1], 512, SEG_MID * 12, s>>>(
-                        lists.p, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, fin,
-                        skew_list.p, ctr.p);
+                        lists.p, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, fin,
+                        skew_list.p, ctr_p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (nbm[2]) {
                     k_seg_bucket<512, 16, 2><<<nbm[2], 512, SEG_MID2 * 12, s>>>(
-                        lists.p + nslots, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, fin,
-                        skew_list.p, ctr.p);
+                        lists.p + nslots, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, fin,
+                        skew_list.p, ctr_p);
                     DTS_LAUNCH_CHECK();
                 }
                 if (nbm[3]) {
                     k_seg_bucket<1024, 16, 1><<<nbm[3], 1024, SEG_CAP * 12, s>>>(
-                        lists.p + 2 * nslots, counts.p, offsets.p, rkeys.p, src, qmap, qid_base,
-                        fin, skew_list.p, ctr.p);
+                        lists.p + 2 * nslots, counts_p, offsets_p, rkeys.p, src, qmap, qid_base,
+                        fin, skew_list.p, ctr_p);
                     DTS_LAUNCH_CHECK();
                 }
                 unsigned int n_skew = 0;
                 if (nbm[1] + nbm[2] + nbm[3]) {
-                    DTS_CUDA(cudaMemcpyAsync(&n_skew, &ctr.p->n_skew, sizeof(n_skew),
+                    DTS_CUDA(cudaMemcpyAsync(&n_skew, &ctr_p->n_skew, sizeof(n_skew),
                                              cudaMemcpyDeviceToHost, s));
                     DTS_CUDA(cudaStreamSynchronize(s));
                 }
                 if (n_skew) {
                     k_seg_radix<1024, 16, 1><<<n_skew, 1024, SEG_CAP * 8, s>>>(
-                        skew_list.p, counts.p, offsets.p, rkeys.p, src, qmap, qid_base, eb, fin);
+                        skew_list.p, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, eb, fin);
                     DTS_LAUNCH_CHECK();
                 }
                 const unsigned int n_big = nbm[0];
@@ -1219,12 +1243,12 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                         throw Error(DTS_ENOTSUP, "long result segments: sort key exceeds 64 bits");
                     DevBuf<unsigned long long> k1(nb, s), k2(nb, s);
                     k_big_keys<<<blocks((size_t)nq * 32, 256), 256, 0, s>>>(
-                        (uint32_t)nq, bigc.p, bigoff.p, offsets.p, rkeys.p, eb, sb, k1.p);
+                        (uint32_t)nq, bigc.p, bigoff.p, offsets_p, rkeys.p, eb, sb, k1.p);
                     DTS_LAUNCH_CHECK();
                     const unsigned long long* sk =
                         radix_sort_keys(k1.p, k2.p, nb, sb, sb + eb + qb, s);
                     k_big_place<<<blocks(nb, 256), 256, 0, s>>>(sk, nb, eb, sb, bigoff.p,
-                                                               offsets.p, rkeys.p, src, qmap, qid_base,
+                                                               offsets_p, rkeys.p, src, qmap, qid_base,
                                                                fin);
                     DTS_LAUNCH_CHECK();
                 }
