@@ -33,7 +33,7 @@ EXPORTED_SYMBOLS = (
     "dts_index_get_info", "dts_last_error", "dts_version", "dts_kernel_launches",
     "dts_search_device_ex", "dts_canonicalize_device", "dts_merge_trajectories_device",
     "dts_query_costs_device", "dts_search_count", "dts_search_count_device",
-    "dts_search_stream", "dts_search_read_times",
+    "dts_search_stream", "dts_search_read_times", "dts_query_costs_sampled_device",
 )
 
 _STATUS = {0: "DTS_OK", -1: "DTS_EINVAL", -2: "DTS_ENOMEM", -3: "DTS_ECUDA",
@@ -147,6 +147,9 @@ def load():
                                       ctypes.POINTER(SearchStats)]
     lib.dts_search_stream.restype = ctypes.c_int
     lib.dts_query_costs_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32, P, P]
+    lib.dts_query_costs_sampled_device.argtypes = [P, P, S, ctypes.c_double, ctypes.c_uint32,
+                                                   ctypes.c_uint32, P, P]
+    lib.dts_query_costs_sampled_device.restype = ctypes.c_int
     lib.dts_query_costs_device.restype = ctypes.c_int
     lib.dts_search_read_times.argtypes = [ctypes.POINTER(SearchStats)]
     lib.dts_search_read_times.restype = ctypes.c_int
@@ -500,20 +503,27 @@ def search_stream(index: Index, Q, d: float, callback, chunk_results: int = 0,
     return st.as_dict()
 
 
-def query_costs_device(index: Index, Q_dev, d: float, block: int = 1, stream=None, out=None):
-    """dts_query_costs_device: Q_dev CUDA tensor (nq, 8) float64 -> CUDA int64
-    tensor of ceil(nq / block) candidate counts (sum over each block of
-    `block` consecutive queries of the pairs the search would refine)."""
+def query_costs_device(index: Index, Q_dev, d: float, block: int = 1, stream=None, out=None,
+                       stride: int = 1):
+    """dts_query_costs_device (dts_query_costs_sampled_device when stride >
+    1): Q_dev CUDA tensor (nq, 8) float64 -> CUDA int64 tensor of
+    ceil(nq / block) candidate counts (sum over each block of `block`
+    consecutive queries of the pairs the search would refine; estimated from
+    every stride-th query)."""
     import torch
     lib = load()
     nq = int(Q_dev.shape[0])
     nb = (nq + int(block) - 1) // int(block)
     if out is None:
         out = torch.empty(nb, dtype=torch.int64, device=Q_dev.device)
-    _check(lib.dts_query_costs_device(index.handle, ctypes.c_void_p(Q_dev.data_ptr() if nq else 0),
-                                      nq, float(d), int(block),
-                                      ctypes.c_void_p(_stream_ptr(stream)),
-                                      ctypes.c_void_p(out.data_ptr() if nb else 0)))
+    qp = ctypes.c_void_p(Q_dev.data_ptr() if nq else 0)
+    op = ctypes.c_void_p(out.data_ptr() if nb else 0)
+    sp = ctypes.c_void_p(_stream_ptr(stream))
+    if int(stride) == 1:
+        _check(lib.dts_query_costs_device(index.handle, qp, nq, float(d), int(block), sp, op))
+    else:
+        _check(lib.dts_query_costs_sampled_device(index.handle, qp, nq, float(d), int(block),
+                                                  int(stride), sp, op))
     return out
 
 

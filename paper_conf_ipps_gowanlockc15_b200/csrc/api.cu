@@ -866,23 +866,30 @@ dts_status dts_search_stream(const dts_index* index, const dts_segment* Q, size_
     });
 }
 
-dts_status dts_query_costs_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
-                                  double d, uint32_t block, void* cuda_stream,
-                                  uint64_t* costs_dev) {
+dts_status dts_query_costs_sampled_device(const dts_index* index, const dts_segment* Q_dev,
+                                          size_t nq, double d, uint32_t block, uint32_t stride,
+                                          void* cuda_stream, uint64_t* costs_dev) {
     DeviceGuard dg;
     return guarded([&] {
         if (!index) throw Error(DTS_EINVAL, "index is NULL");
         if (nq > 0 && (!Q_dev || !costs_dev)) throw Error(DTS_EINVAL, "NULL pointer with nq > 0");
         if (nq >= (size_t(1) << 32)) throw Error(DTS_EINVAL, "nq must be < 2^32");
         if (block == 0) throw Error(DTS_EINVAL, "block must be >= 1");
+        if (stride == 0) throw Error(DTS_EINVAL, "stride must be >= 1");
         if (!(d >= 0.0) || !std::isfinite(d)) throw Error(DTS_EINVAL, "d must be finite and >= 0");
         prepare_device(index->device);
         if (nq) check_aligned(Q_dev, "Q_dev");
         const cudaStream_t s = static_cast<cudaStream_t>(cuda_stream);
         query_costs_device(index, Q_dev, nq, d, block,
-                           reinterpret_cast<unsigned long long*>(costs_dev), s);
+                           reinterpret_cast<unsigned long long*>(costs_dev), s, stride);
         DTS_CUDA(cudaStreamSynchronize(s));
     });
+}
+
+dts_status dts_query_costs_device(const dts_index* index, const dts_segment* Q_dev, size_t nq,
+                                  double d, uint32_t block, void* cuda_stream,
+                                  uint64_t* costs_dev) {
+    return dts_query_costs_sampled_device(index, Q_dev, nq, d, block, 1, cuda_stream, costs_dev);
 }
 
 dts_status dts_canonicalize_device(dts_result* results_dev, size_t n, void* cuda_stream) {

@@ -508,7 +508,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
 // Per-query candidate counts summed per block of `block` queries (search.cu).
 void search_read_times(dts_search_stats* stats);
 void query_costs_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, double d,
-                        uint32_t block, unsigned long long* out, cudaStream_t s);
+                        uint32_t block, unsigned long long* out, cudaStream_t s,
+                        uint32_t stride = 1);
 // Trajectory-level merge (traj.cu); output in cache_alloc'd device memory.
 void merge_trajectories_device(const dts_result* r, size_t n, const uint32_t* qtraj,
                                size_t nqid, const uint32_t* etraj, size_t neid,

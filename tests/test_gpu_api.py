@@ -167,6 +167,14 @@ def test_query_costs_match_candidates(dts):
             # sub-ranges: the costs of rows [a, b) alone
             a, b = c.Q.shape[0] // 3, c.Q.shape[0] // 2
             assert torch.equal(dts.query_costs_device(idx, Qd[a:b], d), per[a:b])
+            # sampled estimate (every 4th query counted 4 times): per block it
+            # is exactly 4 x the sum of the sampled queries' exact costs
+            smp = dts.query_costs_device(idx, Qd, d, block=100, stride=4)
+            keep = torch.zeros_like(per)
+            keep[::4] = per[::4] * 4
+            ref4 = torch.nn.functional.pad(keep, (0, blk.numel() * 100 - keep.numel()))
+            assert torch.equal(ref4.view(-1, 100).sum(1), smp)
+            assert torch.equal(dts.query_costs_device(idx, Qd, d, block=100, stride=1), blk)
             res.free()
             idx.free()
 
