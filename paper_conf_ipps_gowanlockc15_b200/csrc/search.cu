@@ -791,9 +791,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // ---- pass 1: warp tiles, count + staging (spilling output-heavy tiles)
     // queries per warp tile: WQ, or fewer when the query set would not give
     // every resident warp of pass 1 F tiles -- a small set then runs on more
-    // warps, each with a shorter latency chain -- with F = 2.5, or 5 for heavy
-    // queries (work >= 160 expected candidates, about 40 actual: the estimate
-    // runs ~4x high), and at least 4 queries (2 from work >= 1600).  Measured
+    // warps, each with a shorter latency chain -- with F = 2.5 and at least 4
+    // queries; heavy queries (work >= 160 expected candidates, about 40
+    // actual: the estimate runs ~4x high) F = 12 and at least 2; work >=
+    // 4000: F = 24, tiles down to one query.  Measured
     // (device search, ms, tiles of 2 / 4 / 7 / 10 / 16 queries): C1 0.146 /
     // 0.131 / 0.131 / 0.134 / 0.143; C2 d = 2 0.377 / 0.382 / 0.389 / 0.432 /
     // 0.466; C2 d = 8 3.42 / 3.45 / 3.61 / 3.76 / 4.15; S1 d = 50 0.201 /
@@ -801,7 +802,10 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     // 0.979 / 1.329; S3 d = 0.01 0.215 / 0.181 / 0.169 / 0.174 / 0.166; the
     // C4 query set's 1/8 (125 k, a rank's share at N = 8): 8 0.209, 13 0.184,
     // 16 0.187.  F: 2 / 2.5 / 4 -- S1 d = 50 0.204 / 0.168 / 0.168, S3 d =
-    // 0.05 0.157 / 0.167 / 0.167, the C4 1/8 share 0.185 / 0.184 / 0.209
+    // 0.05 0.157 / 0.167 / 0.167, the C4 1/8 share 0.185 / 0.184 / 0.209.
+    // Heavy (tiles of 1 / 2 / 3 / 4): S2 d = 1 29.3 / 31.0 / 32.6 / 34.0;
+    // S2 d = 0.1 0.632 / 0.625 / 0.678 / 0.720; C2 d = 8 3.42 / 3.40 / 3.40 /
+    // 3.43; C2 d = 2 0.597 / 0.360 / - / 0.382
     static const int nsm_tiles = [] {
         int dev = 0, v = 148;
         cudaGetDevice(&dev);
@@ -813,8 +817,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         return e ? atof(e) : 2.5;
     }();
     const double slots = (double)nsm_tiles * 7.0 * WW;            // resident warps of pass 1
-    const double fill = work >= 160.0 ? 2.0 * tile_fill : tile_fill;
-    const double tmin = work >= 1600.0 ? 2.0 : 4.0;
+    const double fill = work >= 4000.0 ? 9.6 * tile_fill : (work >= 160.0 ? 4.8 * tile_fill : tile_fill);
+    const double tmin = work >= 4000.0 ? 1.0 : (work >= 160.0 ? 2.0 : 4.0);
     // (the temporal and subbin methods keep WQ: their tiles' queries share
     //  runs, streamed once per group)
     uint32_t tq = (tile_fill <= 0.0 || idx->method != DTS_METHOD_GRID) ? (uint32_t)WQ
