@@ -310,3 +310,35 @@ def test_mem_budget_temporal_shards(dts, oracle_mod, budget_mb):
                    oracle_mod.search_queries(c.D, c.Q, qs, 2.0), c.D, c.Q, 2.0, oracle_mod)
     idx.free()
     ref_idx.free()
+
+
+def test_host_results_over_1gb(dts, oracle_mod):
+    """A host search whose results exceed 1 GB lands in huge-page backed
+    pageable memory through the staged, multi-threaded copy: the bytes equal
+    the device search's, and sampled queries match the oracle."""
+    import torch
+    g = np.random.default_rng(11)
+    n, nq = 20000, 2400                       # 4.8e7 results, 1.15 GB
+    D = np.zeros((n, 8))
+    D[:, 4] = 1.0
+    D[:, 1:4] = g.uniform(0, 0.01, (n, 3))
+    D[:, 5:8] = D[:, 1:4] + g.uniform(-1e-3, 1e-3, (n, 3))
+    Q = np.zeros((nq, 8))
+    Q[:, 4] = 1.0
+    Q[:, 1:4] = g.uniform(0, 0.01, (nq, 3))
+    Q[:, 5:8] = Q[:, 1:4]
+    d = 0.1                                   # every pair, the whole time
+    idx = dts.build_index(D)
+    host = dts.search(idx, Q, d)
+    assert host.shape[0] == n * nq and host.nbytes > (1 << 30)
+    dev, _ = dts.search_device(idx, torch.from_numpy(Q).cuda(), d)
+    assert dev.count == host.shape[0]
+    assert np.array_equal(dev.numpy().view(np.uint8), host.view(np.uint8))
+    dev.free()
+    for q in (0, 777, nq - 1):
+        got = host[host["query_id"] == q].copy()
+        got["query_id"] = 0
+        info = parity.compare(got, oracle_mod.search(D, Q[q:q + 1], d), D, Q[q:q + 1], d,
+                              oracle_mod)
+        assert info["common"] == n
+    idx.free()
