@@ -60,6 +60,9 @@ struct Counters {                       // device-side statistics / flags
     unsigned int bad;
     unsigned int work;                  // dynamic warp-tile counter
     unsigned long long total;           // results (the scan's total, read back with the rest)
+    unsigned int n_desc;                // sub-segments of split long segments
+    unsigned int n_dskew;               // ... whose ids cluster (radix sort)
+    unsigned int n_bigfb;               // long segments left to the device-wide sort
 };
 
 // Query in the velocity form used by the refinement.
@@ -1193,7 +1196,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 DTS_CUDA(cudaMemsetAsync(bigc.p, 0, nq * sizeof(uint32_t), s));
                 DTS_CUDA(cudaMemsetAsync(&ctr_p->n_big, 0, 5 * sizeof(unsigned int), s));
                 const size_t nslots = ((size_t)h.c.n_spill + h.c.n_over) * tq;
-                DevBuf<uint32_t> lists(3 * nslots, s);
+                DevBuf<uint32_t> lists(4 * nslots, s);       // 3 size classes + long segments
                 const int eb = idx->eid_bits;
                 if (h.c.n_spill) {
                     k_seg_sort_warp<<<blocks((size_t)h.c.n_spill * tq, 4), 128, 0, s>>>(
@@ -1225,26 +1228,32 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                                                 SEG_MID2 * 12) == cudaSuccess &&
                            cudaFuncSetAttribute(k_seg_bucket<512, 8, 2>,
                                                 cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                                SEG_MID * 12) == cudaSuccess;
+                                                SEG_MID * 12) == cudaSuccess &&
+                           cudaFuncSetAttribute(k_seg_bucket<1024, 16, 1, true>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_CAP * 12) == cudaSuccess &&
+                           cudaFuncSetAttribute(k_seg_radix<1024, 16, 1, true>,
+                                                cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                                SEG_CAP * 8) == cudaSuccess;
                 }();
                 if (!smem_ok) throw Error(DTS_ECUDA, "segment sort: shared memory size refused");
                 DevBuf<uint32_t> skew_list(nbm[1] + nbm[2] + nbm[3], s);
                 if (nbm[1]) {
                     k_seg_bucket<512, 8, 2><<<nbm[1], 512, SEG_MID * 12, s>>>(
                         lists.p, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, fin,
-                        skew_list.p, ctr_p);
+                        skew_list.p, ctr_p, SegDesc{});
                     DTS_LAUNCH_CHECK();
                 }
                 if (nbm[2]) {
                     k_seg_bucket<512, 16, 2><<<nbm[2], 512, SEG_MID2 * 12, s>>>(
                         lists.p + nslots, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, fin,
-                        skew_list.p, ctr_p);
+                        skew_list.p, ctr_p, SegDesc{});
                     DTS_LAUNCH_CHECK();
                 }
                 if (nbm[3]) {
                     k_seg_bucket<1024, 16, 1><<<nbm[3], 1024, SEG_CAP * 12, s>>>(
                         lists.p + 2 * nslots, counts_p, offsets_p, rkeys.p, src, qmap, qid_base,
-                        fin, skew_list.p, ctr_p);
+                        fin, skew_list.p, ctr_p, SegDesc{});
                     DTS_LAUNCH_CHECK();
                 }
                 unsigned int n_skew = 0;
@@ -1255,10 +1264,49 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                 }
                 if (n_skew) {
                     k_seg_radix<1024, 16, 1><<<n_skew, 1024, SEG_CAP * 8, s>>>(
-                        skew_list.p, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, eb, fin);
+                        skew_list.p, counts_p, offsets_p, rkeys.p, src, qmap, qid_base, eb, fin,
+                        SegDesc{});
                     DTS_LAUNCH_CHECK();
                 }
-                const unsigned int n_big = nbm[0];
+                // ---- segments longer than a CTA sort: split into ordered
+                //      id ranges that each fit one (k_big_split), sorted as
+                //      sub-segments; those that do not split go to one
+                //      device-wide keys-only radix sort
+                unsigned int n_big = 0;
+                if (nbm[0]) {
+                    const unsigned int nlong = nbm[0];
+                    DevBuf<unsigned long long> rk2(h.total, s), d_off((size_t)nlong * SPLIT_MAXB, s);
+                    DevBuf<uint32_t> d_cnt((size_t)nlong * SPLIT_MAXB, s),
+                        d_q((size_t)nlong * SPLIT_MAXB, s);
+                    k_big_split<<<nlong, 256, 0, s>>>(lists.p + 3 * nslots, counts_p, offsets_p,
+                                                     rkeys.p, rk2.p, bigc.p, d_off.p, d_cnt.p,
+                                                     d_q.p, ctr_p);
+                    DTS_LAUNCH_CHECK();
+                    unsigned int nd[3] = {0, 0, 0};            // n_desc, n_dskew, n_bigfb
+                    DTS_CUDA(cudaMemcpyAsync(nd, &ctr_p->n_desc, sizeof(nd),
+                                             cudaMemcpyDeviceToHost, s));
+                    DTS_CUDA(cudaStreamSynchronize(s));
+                    const SegDesc ds{d_off.p, d_cnt.p, d_q.p};
+                    if (nd[0]) {
+                        DevBuf<uint32_t> dskew(nd[0], s);
+                        k_seg_bucket<1024, 16, 1, true><<<nd[0], 1024, SEG_CAP * 12, s>>>(
+                            nullptr, counts_p, offsets_p, rk2.p, src, qmap, qid_base, fin, dskew.p,
+                            ctr_p, ds);
+                        DTS_LAUNCH_CHECK();
+                        unsigned int nsk = 0;
+                        DTS_CUDA(cudaMemcpyAsync(&nsk, &ctr_p->n_dskew, sizeof(nsk),
+                                                 cudaMemcpyDeviceToHost, s));
+                        DTS_CUDA(cudaStreamSynchronize(s));
+                        if (nsk) {
+                            k_seg_radix<1024, 16, 1, true><<<nsk, 1024, SEG_CAP * 8, s>>>(
+                                dskew.p, counts_p, offsets_p, rk2.p, src, qmap, qid_base, eb, fin,
+                                ds);
+                            DTS_LAUNCH_CHECK();
+                        }
+                        DTS_CUDA(cudaStreamSynchronize(s));    // before the scratch goes
+                    }
+                    n_big = nd[2];
+                }
                 if (n_big) {
                     // ---- segments longer than a CTA sort: one device-wide
                     //      keys-only radix sort over those only

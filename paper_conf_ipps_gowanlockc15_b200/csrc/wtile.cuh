@@ -851,7 +851,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
                                                       const uint32_t* __restrict__ qmap,
                                                       uint32_t qid_base, int eb,
                                                       dts_result* __restrict__ out,
-                                                      uint32_t* __restrict__ lists,   // 3 x lstride
+                                                      uint32_t* __restrict__ lists,   // 4 x lstride
                                                       size_t lstride,
                                                       uint32_t* __restrict__ bigc,
                                                       Counters* __restrict__ ctr) {
@@ -869,9 +869,8 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
             if (c <= (uint32_t)SEG_CAP) {
                 const int k = c <= (uint32_t)SEG_MID ? 0 : (c <= (uint32_t)SEG_MID2 ? 1 : 2);
                 lists[(size_t)k * lstride + atomicAdd(&ctr->n_cls[k], 1u)] = q;
-            } else {
-                bigc[q] = c;
-                atomicAdd(&ctr->n_big, 1u);
+            } else {                              // listed in region 3 (k_big_split)
+                lists[(size_t)3 * lstride + atomicAdd(&ctr->n_big, 1u)] = q;
             }
         }
         return;
@@ -932,6 +931,31 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
     seg_gather<4>(S.buf[cur], src, c, qrep, out + off, lane, 32);
 }
 
+// A segment to sort: `c` keys at key_base + off, sorted into out + off with
+// the reported id of query q.  DESC: the i-th entry of a descriptor list
+// (sub-segments of split long segments, k_big_split); else the listed
+// query's whole segment.
+struct SegDesc {
+    const unsigned long long* off;
+    const uint32_t* cnt;
+    const uint32_t* q;
+};
+template <bool DESC>
+__device__ __forceinline__ void seg_of(const uint32_t* list, const SegDesc& ds, uint32_t i,
+                                       const uint32_t* counts,
+                                       const unsigned long long* offsets, uint32_t& q, uint32_t& c,
+                                       unsigned long long& off) {
+    if (DESC) {
+        q = ds.q[i];
+        c = ds.cnt[i];
+        off = ds.off[i];
+    } else {
+        q = list[i];
+        c = counts[q];
+        off = offsets[q];
+    }
+}
+
 // One CTA of SEGC_T threads per listed query (SEGW_CAP < count <= SEGC_T *
 // ITEMS): an LSD radix sort of the (entry id << 32 | slot) keys over the
 // entry id bits, 8 bits per pass, the keys in one shared-memory buffer
@@ -940,7 +964,7 @@ __global__ void __launch_bounds__(128) k_seg_sort_warp(const uint32_t* __restric
 // ranks), the per-warp digit counts are scanned across warps and digits,
 // and every key is stored at its stable position (all keys are in
 // registers by then, so the buffer is overwritten in place).
-template <int SEGC_T, int ITEMS, int MINB>
+template <int SEGC_T, int ITEMS, int MINB, bool DESC = false>
 __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __restrict__ list,
                                                         const uint32_t* __restrict__ counts,
                                                         const unsigned long long* __restrict__ offsets,
@@ -948,14 +972,16 @@ __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __re
                                                       const SpillSrc src,
                                                         const uint32_t* __restrict__ qmap,
                                                         uint32_t qid_base, int eb,
-                                                        dts_result* __restrict__ out) {
+                                                        dts_result* __restrict__ out,
+                                                        const SegDesc ds) {
     constexpr int SEGC_W = SEGC_T / 32;
     extern __shared__ unsigned long long sbuf[];        // SEGC_T * ITEMS keys
     __shared__ uint32_t wcnt[SEGC_W][257];
     __shared__ uint32_t wtot[8];
-    const uint32_t q = list[blockIdx.x];
-    const uint32_t c = counts[q];
-    const unsigned long long off = offsets[q];
+    uint32_t q, c;
+    unsigned long long off;
+    seg_of<DESC>(list, ds, DESC ? list[blockIdx.x] : blockIdx.x, counts, offsets, q, c, off);
+    // (non-DESC: seg_of reads list[blockIdx.x] as the query)
     const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
     seg_keys_load<8>(sbuf, rkeys + off, c, t, SEGC_T);
     const uint32_t lt = (1u << lane) - 1u;
@@ -1033,7 +1059,7 @@ __global__ void __launch_bounds__(SEGC_T, MINB) k_seg_radix(const uint32_t* __re
 // ballot multisplit (9 ballots per key per 8-bit pass) took 13.0 ms.
 constexpr int SEGB_MAX = 32;
 
-template <int T, int ITEMS, int MINB>
+template <int T, int ITEMS, int MINB, bool DESC = false>
 __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restrict__ list,
                                                        const uint32_t* __restrict__ counts,
                                                        const unsigned long long* __restrict__ offsets,
@@ -1043,14 +1069,16 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
                                                        uint32_t qid_base,
                                                        dts_result* __restrict__ out,
                                                        uint32_t* __restrict__ skew_list,
-                                                       Counters* __restrict__ ctr) {
+                                                       Counters* __restrict__ ctr,
+                                                       const SegDesc ds) {
     constexpr uint32_t CAP = (uint32_t)T * ITEMS;
     extern __shared__ unsigned long long bbuf[];        // CAP keys, then CAP bucket counters
     uint32_t* cnt = reinterpret_cast<uint32_t*>(bbuf + CAP);
     __shared__ uint32_t s_min, s_max, s_bmax, s_wsum[T / 32];
-    const uint32_t q = list[blockIdx.x];
-    const uint32_t c = counts[q];
-    const unsigned long long off = offsets[q];
+    // (DESC: blockIdx.x is the descriptor; skewed ones are listed by index)
+    uint32_t q, c;
+    unsigned long long off;
+    seg_of<DESC>(list, ds, blockIdx.x, counts, offsets, q, c, off);
     const unsigned long long* rk = rkeys + off;
     const uint32_t t = threadIdx.x, lane = t & 31, warp = t >> 5;
     if (t == 0) { s_min = ~0u; s_max = 0u; s_bmax = 0u; }
@@ -1103,7 +1131,10 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
     if (lane == 0) atomicMax(&s_bmax, bmax);
     __syncthreads();
     if (s_bmax > (uint32_t)SEGB_MAX) {              // clustered ids: the radix sort
-        if (t == 0) skew_list[atomicAdd(&ctr->n_skew, 1u)] = q;
+        if (t == 0) {
+            if (DESC) skew_list[atomicAdd(&ctr->n_dskew, 1u)] = blockIdx.x;
+            else skew_list[atomicAdd(&ctr->n_skew, 1u)] = q;
+        }
         return;
     }
     uint32_t run = inc - sum;
@@ -1132,6 +1163,90 @@ __global__ void __launch_bounds__(T, MINB) k_seg_bucket(const uint32_t* __restri
     __syncthreads();
     const uint32_t qrep = qmap ? __ldg(qmap + q) : q + qid_base;
     seg_gather<4>(bbuf, src, c, qrep, out + off, t, T);
+}
+
+// Segments longer than SEG_CAP, one CTA each: the keys are split into
+// B = ceil(c / SEG_SPLIT) equal-width ranges of (entry id - the segment's
+// least id) -- ordered ranges, so sorting each range in place sorts the
+// segment -- written to `rk2` at the segment's offsets, and one descriptor
+// per non-empty range is listed for k_seg_bucket<DESC>.  A segment whose
+// ranges do not all fit a CTA sort (ids clustered) is left to the
+// device-wide sort (bigc[q] = c).
+constexpr int SEG_SPLIT = 8192;
+constexpr int SPLIT_MAXB = 256;
+__global__ void __launch_bounds__(256) k_big_split(const uint32_t* __restrict__ list,
+                                                  const uint32_t* __restrict__ counts,
+                                                  const unsigned long long* __restrict__ offsets,
+                                                  const unsigned long long* __restrict__ rkeys,
+                                                  unsigned long long* __restrict__ rk2,
+                                                  uint32_t* __restrict__ bigc,
+                                                  unsigned long long* __restrict__ d_off,
+                                                  uint32_t* __restrict__ d_cnt,
+                                                  uint32_t* __restrict__ d_q,
+                                                  Counters* __restrict__ ctr) {
+    __shared__ uint32_t s_min, s_max, s_ok, cnt[SPLIT_MAXB], base[SPLIT_MAXB];
+    const uint32_t q = list[blockIdx.x];
+    const uint32_t c = counts[q];
+    const unsigned long long off = offsets[q];
+    const unsigned long long* rk = rkeys + off;
+    const uint32_t t = threadIdx.x;
+    uint32_t B = (c + SEG_SPLIT - 1) / SEG_SPLIT;
+    if (t == 0) { s_min = ~0u; s_max = 0u; s_ok = 1u; }
+    for (uint32_t j = t; j < SPLIT_MAXB; j += 256) cnt[j] = 0;
+    __syncthreads();
+    if (B > (uint32_t)SPLIT_MAXB) {                  // beyond the split: device sort
+        if (t == 0) {
+            bigc[q] = c;
+            atomicAdd(&ctr->n_bigfb, 1u);
+        }
+        return;
+    }
+    uint32_t mn = ~0u, mx = 0u;
+    for (uint32_t i = t; i < c; i += 256) {
+        const uint32_t e = (uint32_t)(rk[i] >> 32);
+        mn = min(mn, e);
+        mx = max(mx, e);
+    }
+    mn = __reduce_min_sync(0xffffffffu, mn);
+    mx = __reduce_max_sync(0xffffffffu, mx);
+    if ((t & 31) == 0) { atomicMin(&s_min, mn); atomicMax(&s_max, mx); }
+    __syncthreads();
+    mn = s_min;
+    const unsigned long long span = (unsigned long long)(s_max - mn) + 1ull;
+    auto bucket = [&](unsigned long long k) {
+        return (uint32_t)(((unsigned long long)((uint32_t)(k >> 32) - mn) * B) / span);
+    };
+    for (uint32_t i = t; i < c; i += 256) atomicAdd(&cnt[bucket(rk[i])], 1u);
+    __syncthreads();
+    if (t == 0) {
+        uint32_t run = 0;
+        for (uint32_t b = 0; b < B; ++b) {
+            if (cnt[b] > (uint32_t)SEG_CAP) s_ok = 0u;
+            base[b] = run;
+            run += cnt[b];
+        }
+    }
+    __syncthreads();
+    if (!s_ok) {                                     // clustered ids: device sort
+        if (t == 0) {
+            bigc[q] = c;
+            atomicAdd(&ctr->n_bigfb, 1u);
+        }
+        return;
+    }
+    if (t < B && cnt[t]) {
+        const uint32_t k = atomicAdd(&ctr->n_desc, 1u);
+        d_off[k] = off + base[t];
+        d_cnt[k] = cnt[t];
+        d_q[k] = q;
+    }
+    __syncthreads();
+    for (uint32_t i = t; i < c; i += 256) {
+        const unsigned long long k = rk[i];
+        const uint32_t pos = atomicAdd(&base[bucket(k)], 1u);
+        DTS_DCHECK(bucket(k) < B && pos < c);
+        rk2[off + pos] = k;
+    }
 }
 
 // Segments longer than SEG_CAP: one device-wide keys-only radix sort of

@@ -768,3 +768,31 @@ def test_repeated_searches_speculative_pass2(dts, oracle_mod):
     qs = np.arange(0, c.Q.shape[0], 7)
     parity.compare(parity.restrict(r, qs), oracle_mod.search_queries(c.D, c.Q, qs, 0.05),
                    c.D, c.Q, 0.05, oracle_mod)
+
+
+def test_long_segment_split_and_fallback(dts, oracle_mod):
+    """Result segments over one CTA sort are split into ordered id ranges
+    sorted separately (k_big_split); a segment whose ids cluster so that one
+    range exceeds a CTA sort goes to the device-wide sort instead.  Both
+    give the canonical order and match the oracle."""
+    g = synth.rng(91)
+    m = 20000
+    P = np.zeros((m, 8))
+    P[:, 4] = 1.0
+    P[:, 1:4] = g.uniform(0, 0.01, size=(m, 3))
+    P[:, 5:8] = P[:, 1:4]
+    D = P[g.permutation(m)]
+    Q = np.array([[0.0, 0.005, 0.005, 0.005, 1.0, 0.005, 0.005, 0.005]] * 2)
+    got, info = run_and_compare(dts, oracle_mod, D, Q, 0.05)     # uniform ids: split
+    assert np.array_equal(np.bincount(got["query_id"], minlength=2), [m, m])
+    # clustered caller ids: 19,990 consecutive ids and 10 far away
+    ids = np.arange(m, dtype=np.uint32)
+    ids[-10:] = (1 << 31) + np.arange(10, dtype=np.uint32)
+    ids = ids[g.permutation(m)]
+    idx = dts.build_index(D, entry_ids=ids)
+    got2 = dts.search(idx, Q, 0.05)
+    idx.free()
+    for qi in range(2):
+        e = got2["entry_id"][got2["query_id"] == qi]
+        assert e.shape[0] == m and np.all(np.diff(e.astype(np.int64)) > 0)
+        assert np.array_equal(np.sort(e), np.sort(ids))
