@@ -469,9 +469,10 @@ struct dts_index {
     // spill-buffer size hint (records): the largest output a search of this
     // index has produced after its spill buffer filled (search.cu)
     mutable std::atomic<unsigned long long> spill_hint{0};
-    // capacity for the next search's speculative pass 2 (the last result
-    // count of this index plus an eighth; 0: none yet)
-    mutable std::atomic<unsigned long long> result_hint{0};
+    // results per query of the last search of this index: the next search's
+    // speculative pass 2 gets that rate x its queries plus an eighth (0: none
+    // yet)
+    mutable std::atomic<double> result_hint{0.0};
     int eid_bits = 32;             // bits of the largest reported entry id
     dts::OutlierIndex out{};       // long-segment copies (build.cu), okeys NULL if none
     void* out_block = nullptr;     // backing memory of out (cache)

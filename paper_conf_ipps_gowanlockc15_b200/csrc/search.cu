@@ -1031,7 +1031,11 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
         }
     } spec;
     spec.s = s;
-    const unsigned long long hint = count_only ? 0ull : idx->result_hint.load();
+    // (the hint scales the last search's results per query to this query
+    //  set: chunks of one host search differ in size)
+    const double rate = count_only ? 0.0 : idx->result_hint.load();
+    const unsigned long long hint =
+        rate > 0.0 ? (unsigned long long)(rate * (double)nq * 1.125) + 4096ull : 0ull;
     static const bool spec_on = [] {          // DTS_SPEC_EMIT=0: off
         const char* e = getenv("DTS_SPEC_EMIT");
         return !(e && e[0] == '0');
@@ -1060,7 +1064,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     tr.mark("sync");
     Readback h = *rb;
     h.total = h.c.total;
-    if (!count_only) idx->result_hint.store(h.total + h.total / 8 + 4096);
+    if (!count_only) idx->result_hint.store((double)h.total / (double)nq);
     if (h.c.bad & 1) throw Error(DTS_EINVAL, "query segment with a non-finite coordinate or time");
     if (h.c.bad & 2) throw Error(DTS_EINVAL, "query segment with t_end < t_start");
     if (h.c.bad & 4) throw Error(DTS_EINVAL, "query segment whose speed overflows fp64");
