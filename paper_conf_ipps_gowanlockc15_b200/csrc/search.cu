@@ -869,7 +869,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     unsigned long long* const tile_base_p = reinterpret_cast<unsigned long long*>(p1buf.p + o_tbase);
     unsigned long long* const qstage_p =
         count_only ? nullptr : reinterpret_cast<unsigned long long*>(p1buf.p + o_qstage);
-    DevBuf<dts_result> stage(stage_cap, s), spill(std::max<unsigned long long>(spill_cap, 1), s);
+    DevBuf<dts_result> stage(stage_cap, s);
+    DevBuf<uint2> spill(std::max<unsigned long long>(spill_cap, 1), s);        // (query, entry)
+    DevBuf<double2> spill_t(std::max<unsigned long long>(spill_cap, 1), s);    // intervals
     tr.mark("bufs");
     TileArgs ta{};
     ta.Q = Q;
@@ -888,7 +890,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
     ta.tile_base = tile_base_p;
     ta.over_tiles = over_tiles_p;
     ta.spill_tiles = spill_tiles_p;
-    ta.spill = spill.p;
+    ta.spill_qe = spill.p;
+    ta.spill_t = spill_t.p;
     ta.spill_cap = spill_cap;
     ta.tile_list = nullptr;
     ta.n_list = 0;
@@ -982,7 +985,9 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             if (c1.spill_valid != ~0ull) {
                 spill_cap = std::max(spill_cap, bound);
                 spill.alloc(std::max<unsigned long long>(spill_cap, 1), s);
-                ta.spill = spill.p;
+                spill_t.alloc(std::max<unsigned long long>(spill_cap, 1), s);
+                ta.spill_qe = spill.p;
+                ta.spill_t = spill_t.p;
                 ta.spill_cap = spill_cap;
                 unsigned long long want = bound + (1ull << 20), cur = idx->spill_hint.load();
                 while (cur < want && !idx->spill_hint.compare_exchange_weak(cur, want)) {}
@@ -1146,7 +1151,8 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
             if (h.c.n_spill || h.c.n_over) {
                 DevBuf<uint32_t> cursor(nq, s), cover(h.c.n_over ? nq : 0, s);
                 DTS_CUDA(cudaMemsetAsync(cursor.p, 0, nq * sizeof(uint32_t), s));
-                DevBuf<dts_result> spill2(0, s);
+                DevBuf<uint2> spill2(0, s);
+                DevBuf<double2> spill2_t(0, s);
                 unsigned long long n_raw = 0;
                 if (h.c.n_over) {
                     // ---- tiles that found the spill buffer full: pass 1
@@ -1162,12 +1168,14 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                                              cudaMemcpyDeviceToHost, s));
                     DTS_CUDA(cudaStreamSynchronize(s));
                     spill2.alloc(std::max<unsigned long long>(n_raw, 1), s);
+                    spill2_t.alloc(std::max<unsigned long long>(n_raw, 1), s);
                     DevBuf<Counters> ctr2(1, s);
                     DTS_CUDA(cudaMemsetAsync(ctr2.p, 0, sizeof(Counters), s));
                     DTS_CUDA(cudaMemsetAsync(&ctr2.p->spill_valid, 0xFF, 8, s));
                     TileArgs tb = ta;
                     tb.ctr = ctr2.p;
-                    tb.spill = spill2.p;
+                    tb.spill_qe = spill2.p;
+                    tb.spill_t = spill2_t.p;
                     tb.spill_cap = n_raw;
                     tb.tile_list = over_tiles_p;
                     tb.n_list = h.c.n_over;
@@ -1184,7 +1192,7 @@ void search_device(const dts_index* idx, const dts_segment* Q_dev, size_t nq, do
                                                        h.c.spill_valid);
                 if (n1 + n_raw >= (1ull << 32))
                     throw Error(DTS_ENOTSUP, "more than 2^32 spilled results in one search call");
-                const SpillSrc src{spill.p, n1, spill2.p};
+                const SpillSrc src{spill_t.p, n1, spill2_t.p};
                 if (n1) {
                     k_spill_place<<<blocks(n1, 256), 256, 0, s>>>(
                         spill.p, n1, 0u, h.c.n_over ? cover.p : nullptr, offsets_p, cursor.p,

@@ -75,7 +75,9 @@ struct TileArgs {
                                        // SPILLED spilled, NONE re-run
     uint32_t* over_tiles;              // tiles to re-run (spill buffer full)
     uint32_t* spill_tiles;             // tiles whose hits went to the spill buffer
-    dts_result* spill;                 // spilled hits (query_id = LOCAL query id)
+    uint2* spill_qe;                   // spilled hits: (LOCAL query id, entry id) ...
+    double2* spill_t;                  // ... and their interval (two arrays: the
+                                       // placement reads only the ids)
     unsigned long long spill_cap;
     const uint32_t* tile_list;         // re-run: the tiles to process (else 0..ntiles-1)
     uint32_t n_list;
@@ -253,12 +255,9 @@ __device__ __forceinline__ void flush_spill(WarpSmem& S, const TileArgs& a, int 
     }
     for (uint32_t i = lane; i < nh; i += 32) {
         const unsigned long long k = S.hkey[i];
-        dts_result r;
-        r.query_id = S.qid[(uint32_t)(k >> 42)];
-        r.entry_id = OUT ? (uint32_t)(k >> 10) : __ldg(a.soa.eid + (uint32_t)(k >> 10));
-        r.t_start = S.h0[i];
-        r.t_end = S.h1[i];
-        a.spill[b + i] = r;
+        a.spill_qe[b + i] = make_uint2(S.qid[(uint32_t)(k >> 42)],
+                                       OUT ? (uint32_t)(k >> 10) : __ldg(a.soa.eid + (uint32_t)(k >> 10)));
+        a.spill_t[b + i] = make_double2(S.h0[i], S.h1[i]);
     }
     __syncwarp();
     if (lane == 0) {
@@ -688,16 +687,16 @@ __global__ void __launch_bounds__(256) k_emit_gather(uint32_t nq,
 // the query and the index, so it is the one pass 1 used).  Before the scan.
 constexpr uint32_t DROPPED = 0xffffffffu;
 __global__ void __launch_bounds__(128) k_spill_filter(const TileArgs a, unsigned long long n,
-                                                     dts_result* __restrict__ sp) {
+                                                     uint2* __restrict__ sp) {
     const OutlierArgs oa{a.out, a.soa, a.bin_t0min, a.bin_t1max};
     for (unsigned long long k = (unsigned long long)blockIdx.x * 128 + threadIdx.x; k < n;
          k += (unsigned long long)gridDim.x * 128) {
-        dts_result r = sp[k];
-        const uint32_t p = r.entry_id;
+        const uint2 r = sp[k];                        // (query id, sorted position)
+        const uint32_t p = r.y;
         if (is_copy(a.out, p)) {
             QState q{};
             double qlo[3], qhi[3];
-            const bool live = load_query(a.Q, r.query_id, q, qlo, qhi);
+            const bool live = load_query(a.Q, r.x, q, qlo, qhi);
             const Stencil st = make_stencil(a.g, q, qlo, qhi, a.d, live, a.bin_start,
                                             a.bin_t0min, a.bin_t1max, a.method, a.sb);
             QStencil qs;
@@ -706,12 +705,12 @@ __global__ void __launch_bounds__(128) k_spill_filter(const TileArgs a, unsigned
             for (int ax = 0; ax < 3; ++ax) { qs.clo[ax] = st.clo[ax]; qs.cn[ax] = st.cn[ax]; }
             qs.rstart = st.rstart; qs.rcnt = st.rcnt;
             if (!outlier_canonical(&oa, &a.g, &qs, q.t0, q.t1, p)) {
-                atomicSub(&a.counts[r.query_id], 1u);
-                sp[k].query_id = DROPPED;
+                atomicSub(&a.counts[r.x], 1u);
+                sp[k].x = DROPPED;
                 continue;
             }
         }
-        sp[k].entry_id = __ldg(a.soa.eid + p);
+        sp[k].y = __ldg(a.soa.eid + p);
     }
 }
 
@@ -732,11 +731,20 @@ __global__ void __launch_bounds__(128) k_spill_max(const uint32_t* __restrict__ 
 // ------------------------------------------- spilled tiles: place + sort
 // The spilled records: the first spill buffer, then the re-run's (index
 // space [0, na) then [na, na + nb)).
-struct SpillSrc {
-    const dts_result* a;
+struct SpillSrc {                       // the spilled intervals; the ids come with the keys
+    const double2* a;
     unsigned long long na;
-    const dts_result* b;
-    __device__ __forceinline__ dts_result at(uint32_t i) const { return i < na ? a[i] : b[i - na]; }
+    const double2* b;
+    // the record of spill index i with entry id e
+    __device__ __forceinline__ dts_result at(uint32_t i, uint32_t e) const {
+        const double2 t = i < na ? a[i] : b[i - na];
+        dts_result r;
+        r.query_id = 0;
+        r.entry_id = e;
+        r.t_start = t.x;
+        r.t_end = t.y;
+        return r;
+    }
 };
 
 // Each live spilled record's key (entry id << 32 | its spill index) goes to
@@ -746,7 +754,7 @@ struct SpillSrc {
 // stale and skipped, and so are records the outlier filter dropped.  (Keys,
 // 8 bytes, instead of the 24-byte records: the sorts read them contiguously
 // and gather each record once, from the spill buffer.)
-__global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restrict__ sp,
+__global__ void __launch_bounds__(256) k_spill_place(const uint2* __restrict__ sp,
                                                     unsigned long long n, uint32_t base_idx,
                                                     const uint32_t* __restrict__ cover,
                                                     const unsigned long long* __restrict__ offsets,
@@ -757,7 +765,7 @@ __global__ void __launch_bounds__(256) k_spill_place(const dts_result* __restric
     uint32_t q = 0xffffffffu, e = 0;
     bool live = k < n;
     if (live) {
-        const uint2 qe = *reinterpret_cast<const uint2*>(sp + k);   // (query_id, entry_id)
+        const uint2 qe = sp[k];                                    // (query_id, entry_id)
         q = qe.x;
         e = qe.y;
         if (q == DROPPED || (cover && cover[q])) live = false;
@@ -822,7 +830,7 @@ __device__ __forceinline__ void seg_gather(const unsigned long long* key, const 
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
             const uint32_t i = b + (uint32_t)j * nt;
-            if (i < c) r[j] = src.at((uint32_t)(key[i] & 0xffffffffull));
+            if (i < c) r[j] = src.at((uint32_t)(key[i] & 0xffffffffull), (uint32_t)(key[i] >> 32));
         }
 #pragma unroll
         for (int j = 0; j < UNR; ++j) {
@@ -1284,7 +1292,8 @@ __global__ void __launch_bounds__(256) k_big_place(const unsigned long long* __r
     const unsigned long long key = keys[k];
     const uint32_t q = (uint32_t)(key >> (eb + sb));
     const unsigned long long slot = key & ((1ull << sb) - 1ull);
-    dts_result r = src.at((uint32_t)(rkeys[offsets[q] + slot] & 0xffffffffull));
+    const unsigned long long rkey = rkeys[offsets[q] + slot];
+    dts_result r = src.at((uint32_t)(rkey & 0xffffffffull), (uint32_t)(rkey >> 32));
     r.query_id = qmap ? __ldg(qmap + q) : q + qid_base;
     out[offsets[q] + (k - bigoff[q])] = r;
 }
